@@ -1,0 +1,84 @@
+/*
+ * hqgen.h -- deterministic TPC-H / SSB shaped data generator (C ABI).
+ *
+ * This module is the ONLY thing the oracle (oracle/) and the CUDA path
+ * (paper_conf_sigmod_funkebnmt18_b200/) share: it produces the input columns
+ * both consume and holds none of the query arithmetic.  Recipe: SURVEY.md
+ * §8(d.1); DESIGN.md "Input recipe".
+ *
+ * Every value is a pure function of (seed, scale factor, table, column, row):
+ * a counter-based splitmix64 stream, so any row range can be generated
+ * independently (partition invariance) and by any number of threads.
+ *
+ * Types: keys, dates (yyyymmdd) and SSB measures are int32; TPC-H DECIMAL
+ * columns are int64 fixed point with scale 2; strings are order-preserving
+ * int8 dictionary codes (dictionaries in hqgen/__init__.py).
+ *
+ * Errors: functions return 0 on success, a negative value on a bad argument.
+ * Ownership: output buffers belong to the caller; the library keeps a small
+ * per-(table, sf, seed) cache of order->row offsets, guarded by a mutex.
+ */
+#ifndef HQGEN_H
+#define HQGEN_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define HQG_DEFAULT_SEED 20180610ULL
+
+/* tables */
+enum {
+  HQG_SSB_LINEORDER = 1,
+  HQG_SSB_DATE = 2,
+  HQG_SSB_CUSTOMER = 3,
+  HQG_SSB_SUPPLIER = 4,
+  HQG_SSB_PART = 5,
+  HQG_TPCH_LINEITEM = 11,
+  HQG_TPCH_ORDERS = 12,
+  HQG_TPCH_CUSTOMER = 13
+};
+
+/* SSB lineorder columns (all int32) */
+enum {
+  LO_ORDERKEY = 0, LO_LINENUMBER, LO_CUSTKEY, LO_PARTKEY, LO_SUPPKEY, LO_ORDERDATE,
+  LO_QUANTITY, LO_EXTENDEDPRICE, LO_DISCOUNT, LO_REVENUE, LO_SUPPLYCOST, LO_TAX,
+  LO_NCOLS
+};
+/* SSB date (int32) */
+enum { D_DATEKEY = 0, D_YEAR, D_YEARMONTHNUM, D_WEEKNUMINYEAR, D_NCOLS };
+/* SSB customer: custkey i32, nation i8, region i8, city i32 */
+enum { C_CUSTKEY = 0, C_NATION, C_REGION, C_CITY, C_NCOLS };
+/* SSB supplier: suppkey i32, nation i8, region i8, city i32 */
+enum { S_SUPPKEY = 0, S_NATION, S_REGION, S_CITY, S_NCOLS };
+/* SSB part: partkey i32, mfgr i8, category i8, brand1 i32 */
+enum { P_PARTKEY = 0, P_MFGR, P_CATEGORY, P_BRAND1, P_NCOLS };
+/* TPC-H lineitem */
+enum {
+  L_ORDERKEY = 0, L_PARTKEY, L_QUANTITY, L_EXTENDEDPRICE, L_DISCOUNT, L_TAX,
+  L_RETURNFLAG, L_LINESTATUS, L_SHIPDATE, L_RECEIPTDATE, L_LINENUMBER, L_NCOLS
+};
+/* TPC-H orders */
+enum { O_ORDERKEY = 0, O_CUSTKEY, O_ORDERDATE, O_SHIPPRIORITY, O_NCOLS };
+/* TPC-H customer */
+enum { TC_CUSTKEY = 0, TC_MKTSEGMENT, TC_NATIONKEY, TC_NCOLS };
+
+/* Number of rows of a table at scale factor sf (lineorder/lineitem count
+ * the 1..7 lines of every order, computed once and cached). <0 on error. */
+int64_t hqg_table_rows(int table, double sf, uint64_t seed, int nthreads);
+/* Byte width of a column (1, 4 or 8); <0 on error. */
+int hqg_column_width(int table, int col);
+/* Number of columns of a table; <0 on error. */
+int hqg_table_ncols(int table);
+/* Generate rows [row_begin, row_end) of the given columns into outs[i]
+ * (outs[i] must hold (row_end-row_begin)*width bytes).  nthreads<=0 means
+ * hardware concurrency. */
+int hqg_generate(int table, double sf, uint64_t seed, int64_t row_begin, int64_t row_end,
+                 int ncols, const int32_t* cols, void* const* outs, int nthreads);
+/* yyyymmdd of day d counted from 1992-01-01 (d=0). */
+int32_t hqg_date_from_day(int32_t d);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,297 @@
+"""oracle -- TEST INFRASTRUCTURE ONLY.
+
+A plain tuple-at-a-time CPU oracle (C++17, ``oracle.cpp``) for the queries of
+SURVEY.md §8(c.1).  Only ``tests/``, ``__graft_entry__.smoke()`` and
+``bench.py`` (its ``cpu_baseline`` leg and ``--impl reference``) may import
+this package.  It shares no code with the CUDA path
+(``paper_conf_sigmod_funkebnmt18_b200``); the only common module is the input
+generator ``hqgen``.
+
+Pins (tests/test_oracle.py): hand-computed fixtures F1-F6 (tests/golden/),
+brute-force nested-loop joins, numpy library cross-checks, invariants
+(COUNT(*) = qualifying rows, sum of group counts = total, sum of group sums =
+scalar sum) and the generator's closed-form selectivities.  No function is
+"parity unpinned".
+
+Each function takes dicts of numpy columns named as in ``hqgen.SCHEMAS`` and
+returns an :class:`OracleResult` with named int64 / float64 columns.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from dataclasses import dataclass, field
+from typing import Dict, List
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = os.path.join(_HERE, "oracle.cpp")
+
+P_I32 = ctypes.POINTER(ctypes.c_int32)
+P_I64 = ctypes.POINTER(ctypes.c_int64)
+P_I8 = ctypes.POINTER(ctypes.c_int8)
+
+
+class _Result(ctypes.Structure):
+    _fields_ = [("nrows", ctypes.c_int64), ("ni", ctypes.c_int32), ("nf", ctypes.c_int32),
+                ("icol", P_I64), ("fcol", ctypes.POINTER(ctypes.c_double)),
+                ("qualifying", ctypes.c_int64)]
+
+
+class _Lineorder(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64)] + [(c, P_I32) for c in (
+        "orderkey", "custkey", "partkey", "suppkey", "orderdate", "quantity", "extendedprice",
+        "discount", "revenue", "supplycost", "tax")]
+
+
+class _Date(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("datekey", P_I32), ("year", P_I32),
+                ("yearmonthnum", P_I32), ("weeknuminyear", P_I32)]
+
+
+class _SsbDim(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("key", P_I32), ("nation", P_I8), ("region", P_I8)]
+
+
+class _Part(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("partkey", P_I32), ("mfgr", P_I8)]
+
+
+class _Lineitem(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("orderkey", P_I32), ("quantity", P_I64),
+                ("extendedprice", P_I64), ("discount", P_I64), ("tax", P_I64),
+                ("returnflag", P_I8), ("linestatus", P_I8), ("shipdate", P_I32)]
+
+
+class _Orders(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("orderkey", P_I32), ("custkey", P_I32),
+                ("orderdate", P_I32), ("shippriority", P_I32)]
+
+
+class _TCustomer(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("custkey", P_I32), ("mktsegment", P_I8)]
+
+
+class OracleError(RuntimeError):
+    def __init__(self, rc: int):
+        super().__init__({-4: "duplicate build key", -6: "int64 overflow", -1: "bad argument"}.get(rc, str(rc)))
+        self.rc = rc
+
+
+@dataclass
+class OracleResult:
+    columns: Dict[str, np.ndarray] = field(default_factory=dict)
+    qualifying: int = 0
+
+    @property
+    def nrows(self) -> int:
+        return len(next(iter(self.columns.values()))) if self.columns else 0
+
+    def rows(self, names: List[str] = None) -> List[tuple]:
+        names = names or list(self.columns)
+        return list(zip(*[self.columns[n].tolist() for n in names]))
+
+
+_lib = None
+
+
+def build() -> str:
+    subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-pthread", "-o", _SO, _SRC])
+    return _SO
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+            build()
+        L = ctypes.CDLL(_SO)
+        P = ctypes.POINTER
+        sig = {
+            "orc_tpch_q6": [P(_Lineitem), ctypes.c_int],
+            "orc_tpch_q1": [P(_Lineitem), ctypes.c_int],
+            "orc_ssb_q1": [ctypes.c_int, P(_Lineorder), P(_Date), ctypes.c_int, ctypes.c_int],
+            "orc_ssb_q31": [P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
+            "orc_ssb_q31_mat": [P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
+            "orc_ssb_q41": [P(_Lineorder), P(_Date), P(_SsbDim), P(_SsbDim), P(_Part), ctypes.c_int, ctypes.c_int],
+            "orc_tpch_q3": [P(_TCustomer), P(_Orders), P(_Lineitem), ctypes.c_int, ctypes.c_int],
+            "orc_micro_select": [P(_Lineorder), ctypes.c_int32, ctypes.c_int],
+            "orc_micro_sum": [P(_Lineorder), ctypes.c_int32, ctypes.c_int],
+            "orc_micro_groupby": [P(_Lineorder), ctypes.c_int32, ctypes.c_int],
+        }
+        for name, args in sig.items():
+            f = getattr(L, name)
+            f.restype = ctypes.c_int
+            f.argtypes = args + [P(_Result)]
+        L.orc_free.restype = None
+        L.orc_free.argtypes = [P(_Result)]
+        _lib = L
+    return _lib
+
+
+def _ptr(arr, ctype, keep):
+    if arr is None:
+        return None
+    a = np.ascontiguousarray(arr, dtype={P_I32: np.int32, P_I64: np.int64, P_I8: np.int8}[ctype])
+    keep.append(a)
+    return a.ctypes.data_as(ctype)
+
+
+def _n(cols) -> int:
+    return len(next(iter(cols.values())))
+
+
+def _lineorder(t, keep):
+    s = _Lineorder()
+    s.n = _n(t)
+    for f in ("orderkey", "custkey", "partkey", "suppkey", "orderdate", "quantity", "extendedprice",
+              "discount", "revenue", "supplycost", "tax"):
+        setattr(s, f, _ptr(t.get("lo_" + f), P_I32, keep))
+    return s
+
+
+def _date(t, keep):
+    s = _Date()
+    s.n = _n(t)
+    for f in ("datekey", "year", "yearmonthnum", "weeknuminyear"):
+        setattr(s, f, _ptr(t.get("d_" + f), P_I32, keep))
+    return s
+
+
+def _dim(t, prefix, keep):
+    s = _SsbDim()
+    s.n = _n(t)
+    s.key = _ptr(t[prefix + ("custkey" if prefix == "c_" else "suppkey")], P_I32, keep)
+    s.nation = _ptr(t.get(prefix + "nation"), P_I8, keep)
+    s.region = _ptr(t.get(prefix + "region"), P_I8, keep)
+    return s
+
+
+def _part(t, keep):
+    s = _Part()
+    s.n = _n(t)
+    s.partkey = _ptr(t["p_partkey"], P_I32, keep)
+    s.mfgr = _ptr(t.get("p_mfgr"), P_I8, keep)
+    return s
+
+
+def _lineitem(t, keep):
+    s = _Lineitem()
+    s.n = _n(t)
+    s.orderkey = _ptr(t.get("l_orderkey"), P_I32, keep)
+    for f in ("quantity", "extendedprice", "discount", "tax"):
+        setattr(s, f, _ptr(t.get("l_" + f), P_I64, keep))
+    s.returnflag = _ptr(t.get("l_returnflag"), P_I8, keep)
+    s.linestatus = _ptr(t.get("l_linestatus"), P_I8, keep)
+    s.shipdate = _ptr(t.get("l_shipdate"), P_I32, keep)
+    return s
+
+
+def _orders(t, keep):
+    s = _Orders()
+    s.n = _n(t)
+    for f in ("orderkey", "custkey", "orderdate", "shippriority"):
+        setattr(s, f, _ptr(t.get("o_" + f), P_I32, keep))
+    return s
+
+
+def _tcust(t, keep):
+    s = _TCustomer()
+    s.n = _n(t)
+    s.custkey = _ptr(t["c_custkey"], P_I32, keep)
+    s.mktsegment = _ptr(t.get("c_mktsegment"), P_I8, keep)
+    return s
+
+
+def _call(fname, args, icols, fcols=()):
+    r = _Result()
+    rc = getattr(lib(), fname)(*args, ctypes.byref(r))
+    if rc != 0:
+        raise OracleError(rc)
+    try:
+        n = r.nrows
+        out = OracleResult(qualifying=int(r.qualifying))
+        if n > 0:
+            ia = np.ctypeslib.as_array(r.icol, shape=(r.ni * n,)).reshape(r.ni, n).copy() if r.ni else None
+            fa = np.ctypeslib.as_array(r.fcol, shape=(r.nf * n,)).reshape(r.nf, n).copy() if r.nf else None
+        for k, name in enumerate(icols):
+            out.columns[name] = ia[k] if n > 0 else np.zeros(0, np.int64)
+        for k, name in enumerate(fcols):
+            out.columns[name] = fa[k] if n > 0 else np.zeros(0, np.float64)
+        return out
+    finally:
+        lib().orc_free(ctypes.byref(r))
+
+
+def tpch_q6(lineitem, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_tpch_q6", [ctypes.byref(_lineitem(lineitem, keep)), nthreads], ["revenue", "count"])
+
+
+def tpch_q1(lineitem, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_tpch_q1", [ctypes.byref(_lineitem(lineitem, keep)), nthreads],
+                 ["l_returnflag", "l_linestatus", "sum_qty", "sum_base_price", "sum_disc_price",
+                  "sum_charge", "count_order"], ["avg_qty", "avg_price", "avg_disc"])
+
+
+def ssb_q1(variant, lineorder, date, brute=False, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_ssb_q1", [variant, ctypes.byref(_lineorder(lineorder, keep)),
+                                ctypes.byref(_date(date, keep)), int(brute), nthreads],
+                 ["revenue", "count"])
+
+
+def ssb_q31(lineorder, customer, supplier, date, brute=False, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_ssb_q31", [ctypes.byref(_lineorder(lineorder, keep)),
+                                 ctypes.byref(_dim(customer, "c_", keep)),
+                                 ctypes.byref(_dim(supplier, "s_", keep)),
+                                 ctypes.byref(_date(date, keep)), int(brute), nthreads],
+                 ["c_nation", "s_nation", "d_year", "revenue", "count"])
+
+
+def ssb_q31_mat(lineorder, customer, supplier, date, brute=False, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_ssb_q31_mat", [ctypes.byref(_lineorder(lineorder, keep)),
+                                     ctypes.byref(_dim(customer, "c_", keep)),
+                                     ctypes.byref(_dim(supplier, "s_", keep)),
+                                     ctypes.byref(_date(date, keep)), int(brute), nthreads],
+                 ["c_nation", "s_nation", "d_year", "lo_revenue"])
+
+
+def ssb_q41(lineorder, date, customer, supplier, part, brute=False, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_ssb_q41", [ctypes.byref(_lineorder(lineorder, keep)),
+                                 ctypes.byref(_date(date, keep)),
+                                 ctypes.byref(_dim(customer, "c_", keep)),
+                                 ctypes.byref(_dim(supplier, "s_", keep)),
+                                 ctypes.byref(_part(part, keep)), int(brute), nthreads],
+                 ["d_year", "c_nation", "profit", "count"])
+
+
+def tpch_q3(customer, orders, lineitem, brute=False, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_tpch_q3", [ctypes.byref(_tcust(customer, keep)),
+                                 ctypes.byref(_orders(orders, keep)),
+                                 ctypes.byref(_lineitem(lineitem, keep)), int(brute), nthreads],
+                 ["l_orderkey", "revenue", "o_orderdate", "o_shippriority", "count"])
+
+
+def micro_select(lineorder, x, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_micro_select", [ctypes.byref(_lineorder(lineorder, keep)), int(x), nthreads], ["revenue"])
+
+
+def micro_sum(lineorder, x, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_micro_sum", [ctypes.byref(_lineorder(lineorder, keep)), int(x), nthreads], ["revenue", "count"])
+
+
+def micro_groupby(lineorder, x, nthreads=1) -> OracleResult:
+    keep = []
+    return _call("orc_micro_groupby", [ctypes.byref(_lineorder(lineorder, keep)), int(x), nthreads],
+                 ["key", "sum", "count"])

@@ -1,0 +1,99 @@
+/*
+ * oracle.h -- TEST INFRASTRUCTURE ONLY.  A plain, slow, tuple-at-a-time CPU
+ * implementation of the SQL results the fused pipeline computes.
+ *
+ * Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+ * --impl reference legs may load or call this library.  It shares no code,
+ * header, helper or constant with the CUDA path (paper_conf_sigmod_funkebnmt18_b200);
+ * the only shared module is the input generator hqgen/.
+ *
+ * What it computes: HorseQC computes exactly the
+ * relational result (§5-§6); the only relaxation is the
+ * order of materialised rows.  So every function here
+ * is the plain SQL definition of one query written out: dimension predicates
+ * + std::unordered_map (or nested loops in brute-force mode) for joins, the
+ * fact predicates in SQL order, exact integer arithmetic in __int128 with an
+ * int64 range check, std::map for GROUP BY, std::sort for ORDER BY.
+ *
+ * Conventions: every function returns 0 on success; on a duplicate build key
+ * -4, on int64 overflow of a result -6, on bad arguments -1.  Results are
+ * column-major int64 (icol) and double (fcol) arrays allocated with malloc
+ * and released with orc_free.  `nthreads` > 1 splits the fact table into
+ * contiguous ranges whose integer partial aggregates are merged exactly
+ * (SURVEY.md §8(c.2) step 6).  `brute` != 0 replaces the hash joins with
+ * nested loops over the dimension arrays (step 5).
+ */
+#ifndef HQ_ORACLE_H
+#define HQ_ORACLE_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct {
+  int64_t nrows;      /* rows of the full (pre-LIMIT) result */
+  int32_t ni, nf;     /* number of int64 / double columns */
+  int64_t* icol;      /* ni * nrows, column-major */
+  double* fcol;       /* nf * nrows, column-major */
+  int64_t qualifying; /* rows that reached the sink (COUNT(*)) */
+} orc_result;
+
+/* SSB lineorder (int32 columns; NULL for columns a query does not read) */
+typedef struct {
+  int64_t n;
+  const int32_t *orderkey, *custkey, *partkey, *suppkey, *orderdate, *quantity,
+      *extendedprice, *discount, *revenue, *supplycost, *tax;
+} orc_lineorder;
+typedef struct { int64_t n; const int32_t *datekey, *year, *yearmonthnum, *weeknuminyear; } orc_date;
+/* SSB customer or supplier */
+typedef struct { int64_t n; const int32_t* key; const int8_t *nation, *region; } orc_ssb_dim;
+typedef struct { int64_t n; const int32_t* partkey; const int8_t* mfgr; } orc_part;
+/* TPC-H lineitem: DECIMALs are int64 fixed point, scale 2 */
+typedef struct {
+  int64_t n;
+  const int32_t* orderkey;
+  const int64_t *quantity, *extendedprice, *discount, *tax;
+  const int8_t *returnflag, *linestatus;
+  const int32_t* shipdate;
+} orc_lineitem;
+typedef struct { int64_t n; const int32_t *orderkey, *custkey, *orderdate, *shippriority; } orc_orders;
+typedef struct { int64_t n; const int32_t* custkey; const int8_t* mktsegment; } orc_tpch_customer;
+
+/* TPC-H Q6 -> 1 row: [revenue (scale 4), count] */
+int orc_tpch_q6(const orc_lineitem* li, int nthreads, orc_result* out);
+/* TPC-H Q1 -> rows [rf, ls, sum_qty, sum_base_price, sum_disc_price(s4), sum_charge(s6), count]
+ *            + f [avg_qty, avg_price, avg_disc], ORDER BY rf, ls */
+int orc_tpch_q1(const orc_lineitem* li, int nthreads, orc_result* out);
+/* SSB Q1.1 / Q1.2 / Q1.3 (variant 1..3) -> 1 row: [revenue, count] */
+int orc_ssb_q1(int variant, const orc_lineorder* lo, const orc_date* d, int brute, int nthreads,
+               orc_result* out);
+/* SSB Q3.1 (Fig 23) -> rows [c_nation, s_nation, d_year, revenue, count]
+ * ORDER BY d_year asc, revenue desc, c_nation, s_nation */
+int orc_ssb_q31(const orc_lineorder* lo, const orc_ssb_dim* c, const orc_ssb_dim* s,
+                const orc_date* d, int brute, int nthreads, orc_result* out);
+/* SSB Q3.1 materialised join result -> rows [c_nation, s_nation, d_year, lo_revenue],
+ * sorted lexicographically (a multiset: P:1203-1210) */
+int orc_ssb_q31_mat(const orc_lineorder* lo, const orc_ssb_dim* c, const orc_ssb_dim* s,
+                    const orc_date* d, int brute, int nthreads, orc_result* out);
+/* SSB Q4.1 -> rows [d_year, c_nation, profit, count], ORDER BY d_year, c_nation */
+int orc_ssb_q41(const orc_lineorder* lo, const orc_date* d, const orc_ssb_dim* c,
+                const orc_ssb_dim* s, const orc_part* p, int brute, int nthreads, orc_result* out);
+/* TPC-H Q3 -> rows [l_orderkey, revenue(s4), o_orderdate, o_shippriority, count],
+ * ORDER BY revenue desc, o_orderdate asc, l_orderkey asc (full result; caller applies LIMIT 10) */
+int orc_tpch_q3(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li, int brute,
+                int nthreads, orc_result* out);
+/* PAPER.md Fig 16 "Query 1": revenue = lo_extendedprice*lo_discount+lo_tax
+ * where lo_quantity between 25-x and 25+x -> rows [revenue] sorted (a multiset) */
+int orc_micro_select(const orc_lineorder* lo, int32_t x, int nthreads, orc_result* out);
+/* App G.1: sum(revenue) of the same selection -> 1 row [sum, count] */
+int orc_micro_sum(const orc_lineorder* lo, int32_t x, int nthreads, orc_result* out);
+/* Fig 26: select sum(lo_extendedprice), lo_orderkey % x group by lo_orderkey % x
+ * -> rows [lo_orderkey % x, sum, count] ORDER BY key */
+int orc_micro_groupby(const orc_lineorder* lo, int32_t x, int nthreads, orc_result* out);
+
+void orc_free(orc_result* r);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
