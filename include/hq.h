@@ -1,0 +1,291 @@
+/*
+ * hq.h -- C ABI of libhq, the B200-native (sm_100a) fused query-pipeline engine.
+ *
+ * Implements the data-parallel hot path of HorseQC (Funke, Bress, Noll, Markl,
+ * Teubner, "Pipelined Query Processing in Coprocessor Environments", SIGMOD'18;
+ * /root/reference/PAPER.md, cited as P:<line>):
+ *
+ *   hq_load_columns   columnar input, resident in device memory before the
+ *                     query runs.
+ *   hq_build_hash     the pipeline breaker of a join: dimension rows filtered by
+ *                     their predicates and inserted into an open-addressing hash
+ *                     table in global memory with atomics (P:186-195,
+ *                     P:1033-1036; Table 4 "Pipeline Breaker").
+ *   hq_run_pipeline   one *fusion operator* (P:495-500): a plan descriptor
+ *                     scan -> filter -> probe* -> compute -> aggregate |
+ *                     materialise, executed as ONE compound kernel (§5.2,
+ *                     Fig 12) whose write offsets / aggregates use
+ *                     local resolution + global propagation (§6.1, P:1056-1210;
+ *                     Fig 25).  The same descriptor can also be run
+ *                     operator-at-a-time (Fig 6) as the bytes-moved
+ *                     baseline (HQ_EXEC_OAAT).
+ *   hq_fetch_result   post-processing outside the pipeline (ORDER BY, LIMIT,
+ *                     AVG) and the device->host copy.
+ *
+ * ---------------------------------------------------------------------------
+ * Conventions
+ *  - Every call returns hq_status (0 = HQ_OK, negative = error).  Out-params are
+ *    written only on HQ_OK.  No exception, abort or exit crosses the ABI.  The
+ *    message of the last failing call of the calling thread: hq_last_error().
+ *  - Device work is enqueued asynchronously on the context stream (the caller's
+ *    cudaStream_t, typically torch's current stream).  Device-side faults
+ *    detected inside kernels (duplicate build key, int64 overflow guard, group
+ *    key out of its declared domain, hash-table or capacity overflow) are raised
+ *    at the next *syncing* call on that object: hq_hash_info, hq_result_info_get,
+ *    hq_fetch_result, hq_finalize (when it has to size a sort).
+ *  - Ownership: the library owns device memory of tables loaded with
+ *    HQ_HOST_COPY, of hash tables and of results; it is allocated through the
+ *    caller-supplied hq_allocator (NULL: cudaMallocAsync on the ctx stream).
+ *    The caller owns host buffers, device buffers passed with
+ *    HQ_DEVICE_BORROW / hq_hash_import (they must outlive the handle) and the
+ *    stream.  Handles are reference counted internally: hq_free_* releases the
+ *    caller's reference; memory goes away once no hash/result uses it.
+ *  - Layout: columns are dense arrays (SoA), one value per row, little endian,
+ *    int8 / int32 / int64.  Device column pointers must be 16-byte aligned
+ *    (HQ_ERR_ARG otherwise) -- required by the TMA bulk copies of the pipeline.
+ *  - Limits: <=16 columns per table, <=16 ops, <=4 probes payload words,
+ *    <=4 group keys, <=8 aggregates, <=8 output columns, <=8 temporaries,
+ *    <=64 expression instructions per plan.  Larger plans: HQ_ERR_UNSUPPORTED.
+ *    There is no CPU fallback: without a CUDA device every call fails with
+ *    HQ_ERR_NO_DEVICE.
+ *  - Threading: a context may be used by one host thread at a time.
+ */
+#ifndef HQ_H
+#define HQ_H
+#include <stddef.h>
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define HQ_ABI_VERSION 1
+
+typedef int32_t hq_status;
+enum {
+  HQ_OK = 0,
+  HQ_ERR_ARG = -1,         /* invalid argument / plan */
+  HQ_ERR_CUDA = -2,        /* CUDA runtime error */
+  HQ_ERR_OOM = -3,         /* allocation failed */
+  HQ_ERR_DUP_KEY = -4,     /* duplicate key inserted into a join hash table */
+  HQ_ERR_UNSUPPORTED = -5, /* plan exceeds the limits above */
+  HQ_ERR_OVERFLOW = -6,    /* int64 guard, group table or output capacity exceeded */
+  HQ_ERR_STATE = -7,       /* object in the wrong state for the call */
+  HQ_ERR_NO_DEVICE = -8    /* no CUDA device */
+};
+
+typedef enum { HQ_I8 = 1, HQ_I32 = 3, HQ_I64 = 4, HQ_F64 = 5 } hq_type;
+
+#define HQ_MAX_COLS 16
+#define HQ_MAX_OPS 16
+#define HQ_MAX_PAYLOAD 3
+#define HQ_MAX_KEYS 4
+#define HQ_MAX_AGGS 8
+#define HQ_MAX_OUT 8
+#define HQ_MAX_TMP 8
+#define HQ_MAX_INSN 16
+#define HQ_MAX_PREDS 8
+#define HQ_MAX_ORDER 4
+/* Register numbering inside a plan: 0..ncols-1 are the fact table's columns,
+ * HQ_TMP(k) (k < HQ_MAX_TMP) are temporaries written by PROBE payloads (int32)
+ * and COMPUTE ops (int64). */
+#define HQ_TMP(k) (0x100 + (k))
+
+typedef struct hq_ctx hq_ctx;
+typedef struct hq_table hq_table;
+typedef struct hq_hash hq_hash;
+typedef struct hq_result hq_result;
+
+/* Device memory hooks.  alloc returns a device pointer (>= 256-B aligned) or
+ * NULL; both are called with the ctx stream. */
+typedef struct {
+  void* (*alloc)(size_t bytes, void* stream, void* user);
+  void (*free)(void* ptr, size_t bytes, void* stream, void* user);
+  void* user;
+} hq_allocator;
+
+/* ---------------------------------------------------------------- context */
+/* device: CUDA ordinal; stream: cudaStream_t (NULL = legacy default stream);
+ * alloc: NULL = cudaMallocAsync/cudaFreeAsync on the stream. */
+hq_status hq_ctx_create(int32_t device, void* stream, const hq_allocator* alloc, hq_ctx** out);
+hq_status hq_ctx_destroy(hq_ctx* ctx);
+hq_status hq_ctx_set_stream(hq_ctx* ctx, void* stream);
+hq_status hq_ctx_sync(hq_ctx* ctx);
+/* Thread-local message of the last non-OK status (never NULL). */
+const char* hq_last_error(void);
+int32_t hq_abi_version(void);
+/* sizeof of the public structs, so bindings can check their mirrors. */
+size_t hq_sizeof(const char* struct_name);
+
+/* Kernel timing: when enabled, CUDA events are recorded on the ctx stream
+ * around every fused-pipeline kernel launch.  hq_ctx_kernel_times syncs and
+ * returns (and clears) the durations in ms, oldest first; *n = count. */
+hq_status hq_ctx_enable_timing(hq_ctx* ctx, int32_t on);
+hq_status hq_ctx_kernel_times(hq_ctx* ctx, float* ms, int32_t max, int32_t* n);
+
+/* ----------------------------------------------------------------- tables */
+typedef struct {
+  const char* name; /* informational, may be NULL */
+  int32_t type;     /* hq_type: HQ_I8, HQ_I32 or HQ_I64 */
+  int32_t reserved;
+  const void* data; /* host pointer (HQ_HOST_COPY) or device pointer (HQ_DEVICE_BORROW) */
+} hq_column;
+#define HQ_HOST_COPY 1     /* library allocates device memory and copies (async; host buffer must stay valid until the next ctx sync) */
+#define HQ_DEVICE_BORROW 2 /* data are device pointers kept alive by the caller */
+hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int64_t nrows,
+                          int32_t flags, hq_table** out);
+hq_status hq_table_info(const hq_table* t, int64_t* nrows, int32_t* ncols);
+hq_status hq_table_column(const hq_table* t, int32_t col, const void** dev_ptr, int32_t* type);
+hq_status hq_free_table(hq_table* t);
+
+/* ------------------------------------------------------------- predicates */
+typedef enum {
+  HQ_EQ = 1, HQ_NE, HQ_LT, HQ_LE, HQ_GT, HQ_GE,
+  HQ_BETWEEN,   /* lo <= v <= hi (SQL BETWEEN, inclusive) */
+  HQ_IN_BITMAP  /* 0 <= v < 256 and bit v of bitmap set (IN-lists over dictionary codes) */
+} hq_cmp;
+typedef struct {
+  int32_t reg;   /* column (build side: column of the source table) or HQ_TMP(k) */
+  int32_t cmp;   /* hq_cmp */
+  int64_t lo;    /* comparison constant (EQ..GE) / lower bound (BETWEEN) */
+  int64_t hi;    /* upper bound (BETWEEN) */
+  uint64_t bitmap[4];
+} hq_pred;
+
+/* ------------------------------------------------------------ hash build */
+typedef struct {
+  const hq_table* src;   /* dimension table, or hq_result_as_table of a materialised result */
+  int32_t npreds;
+  hq_pred preds[HQ_MAX_PREDS]; /* conjunction over src columns */
+  int32_t key_col;       /* int32 (or int8/int64 whose values fit int32, != INT32_MIN) */
+  int32_t npayload;      /* 0 = semi-join table (keys only), 1..3 payload columns (values must fit int32) */
+  int32_t payload_cols[HQ_MAX_PAYLOAD];
+  int64_t expected_rows; /* >0: capacity sized for this many keys (no count pass, no host sync);
+                            <=0: a count pass sizes the table exactly (one ctx sync) */
+} hq_build_desc;
+/* Open addressing, linear probing, power-of-two capacity >= keys/0.6, slot =
+ * {int32 key, payload...} of 4, 8 or 16 bytes, empty key INT32_MIN, inserted
+ * with one atomicCAS on the key.  Duplicate keys: HQ_ERR_DUP_KEY at hq_hash_info. */
+hq_status hq_build_hash(hq_ctx* ctx, const hq_build_desc* desc, hq_hash** out);
+typedef struct {
+  int64_t capacity;     /* slots (power of two) */
+  int32_t slot_words;   /* 1, 2 or 4 int32 words per slot */
+  int32_t npayload;
+  int64_t nkeys;        /* keys inserted (valid after hq_hash_info) */
+  int64_t bytes;        /* capacity * slot_words * 4 */
+} hq_hash_meta;
+hq_status hq_hash_info(hq_ctx* ctx, const hq_hash* h, hq_hash_meta* meta);  /* syncs, reports build faults */
+/* Multi-GPU glue: raw device view of the slot array (to broadcast it with NCCL)
+ * and import of such a buffer on another device (borrowed, caller keeps it). */
+hq_status hq_hash_device_view(const hq_hash* h, void** dev_ptr, hq_hash_meta* meta);
+hq_status hq_hash_import(hq_ctx* ctx, const hq_hash_meta* meta, void* dev_ptr, hq_hash** out);
+hq_status hq_free_hash(hq_hash* h);
+
+/* ------------------------------------------------------------------ plans */
+typedef enum { HQ_OP_FILTER = 1, HQ_OP_PROBE = 2, HQ_OP_COMPUTE = 3 } hq_op_kind;
+typedef enum { HQ_PROBE_INNER = 0, HQ_PROBE_SEMI = 1, HQ_PROBE_ANTI = 2 } hq_probe_mode;
+/* Expression code: an accumulator machine evaluated per row in int64.
+ * operand = register `reg`, or the immediate `imm` when reg < 0. */
+typedef enum {
+  HQ_I_LOAD = 1, /* acc = operand            */
+  HQ_I_ADD,      /* acc = acc + operand      */
+  HQ_I_SUB,      /* acc = acc - operand      */
+  HQ_I_RSUB,     /* acc = operand - acc      */
+  HQ_I_MUL,      /* acc = acc * operand      */
+  HQ_I_DIV,      /* acc = acc / operand (C truncation; /0 -> HQ_ERR_ARG) */
+  HQ_I_MOD       /* acc = acc % operand (C semantics; %0 -> HQ_ERR_ARG) */
+} hq_opcode;
+typedef struct {
+  int32_t opc;
+  int32_t reg;
+  int64_t imm;
+} hq_insn;
+typedef struct {
+  int32_t kind;           /* hq_op_kind */
+  /* FILTER */
+  hq_pred filter;
+  /* PROBE: row survives if key found (INNER/SEMI) or not found (ANTI);
+   * INNER copies the matching slot's payload words to payload_dst temps. */
+  const hq_hash* ht;
+  int32_t key_reg;
+  int32_t mode;           /* hq_probe_mode */
+  int32_t npayload;
+  int32_t payload_dst[HQ_MAX_PAYLOAD];
+  /* COMPUTE: dst temp = value of code[0..ninsn) */
+  int32_t dst;
+  int32_t ninsn;
+  hq_insn code[HQ_MAX_INSN];
+} hq_op;
+
+typedef enum { HQ_AGG_SUM = 1, HQ_AGG_COUNT, HQ_AGG_MIN, HQ_AGG_MAX, HQ_AGG_AVG } hq_agg_fn;
+typedef enum { HQ_SINK_AGG = 1, HQ_SINK_MATERIALISE = 2 } hq_sink_kind;
+/* Reduction technique of the sink (Table 4):
+ * LRGP = local resolution in registers/shared memory + global propagation with
+ *        one atomic per block and tile (A3, B3, C3) -- the default;
+ * ATOMIC = per-row global atomics (A2, B2, C2), kept as an ablation. */
+typedef enum { HQ_RES_LRGP = 0, HQ_RES_ATOMIC = 1 } hq_resolution;
+typedef enum { HQ_EXEC_FUSED = 0, HQ_EXEC_OAAT = 1 } hq_exec;
+
+typedef struct {
+  const hq_table* fact;
+  int64_t row_begin, row_end; /* range partition of the fact table; row_end < 0 = all rows */
+  int32_t nops;
+  hq_op ops[HQ_MAX_OPS];
+  int32_t sink;               /* hq_sink_kind */
+  int32_t resolution;         /* hq_resolution */
+  int32_t exec;               /* hq_exec */
+  int32_t ntmp_types;         /* unused, must be 0 */
+  /* AGG sink: GROUP BY key_reg[] (each value v must satisfy key_min <= v <
+   * key_min + key_card; the packed index sum((v-min)*stride) selects a dense
+   * table when prod(card) <= 65536, else a global hash table); aggregates. */
+  int32_t nkeys;
+  int32_t key_reg[HQ_MAX_KEYS];
+  int64_t key_min[HQ_MAX_KEYS];
+  int64_t key_card[HQ_MAX_KEYS];
+  int32_t naggs;
+  int32_t agg_fn[HQ_MAX_AGGS];    /* hq_agg_fn */
+  int32_t agg_reg[HQ_MAX_AGGS];   /* ignored for COUNT */
+  int32_t agg_scale[HQ_MAX_AGGS]; /* AVG: result = sum / count / 10^scale (fp64) */
+  int64_t group_capacity;         /* hash group-by: expected #groups (0 = auto) */
+  /* MATERIALISE sink: output columns out_reg[] cast to out_type[] */
+  int32_t nout;
+  int32_t out_reg[HQ_MAX_OUT];
+  int32_t out_type[HQ_MAX_OUT];
+  int64_t capacity;               /* output rows (0 = rows of the range) */
+  /* post-processing of AGG results: ORDER BY result columns
+   * (keys first, then aggregates), remaining ties by the group keys; LIMIT. */
+  int32_t norder;
+  int32_t order_col[HQ_MAX_ORDER];
+  int32_t order_desc[HQ_MAX_ORDER];
+  int64_t limit;                  /* <= 0: no limit */
+} hq_plan;
+
+/* Enqueue the pipeline (async).  The plan is copied; hash tables and the fact
+ * table it references are retained by the result. */
+hq_status hq_run_pipeline(hq_ctx* ctx, const hq_plan* plan, hq_result** out);
+/* Post-process an AGG result in place (compaction, AVG, ORDER BY, LIMIT);
+ * idempotent; implied by hq_result_info_get / hq_fetch_result. */
+hq_status hq_finalize(hq_ctx* ctx, hq_result* r);
+
+typedef struct {
+  int64_t nrows;            /* rows of the (finalized, limited) result */
+  int64_t qualifying_rows;  /* rows that reached the sink (COUNT(*)) */
+  int32_t ncols;
+  int32_t types[HQ_MAX_KEYS + HQ_MAX_AGGS]; /* hq_type of each result column */
+} hq_result_info;
+hq_status hq_result_info_get(hq_ctx* ctx, hq_result* r, hq_result_info* out); /* syncs */
+/* Copy the result into caller host buffers host_cols[c] (capacity_rows rows
+ * each, typed as hq_result_info.types).  Syncs. */
+hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int64_t capacity_rows,
+                          int64_t* nrows_out);
+/* Materialised result viewed as a table (borrows the result's buffers). */
+hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out);
+/* Multi-GPU glue for dense AGG results: the raw partial-aggregate array
+ * (int64, ngroups x (1+naggs): [count, agg...]) before finalization, so ranks
+ * can sum it with NCCL; only SUM/COUNT/AVG plans (HQ_ERR_UNSUPPORTED else). */
+hq_status hq_result_partials_view(hq_result* r, void** dev_ptr, size_t* bytes);
+hq_status hq_free_result(hq_result* r);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

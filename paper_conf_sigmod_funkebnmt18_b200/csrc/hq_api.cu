@@ -1,0 +1,395 @@
+// hq_api.cu -- the extern "C" boundary of libhq (include/hq.h): contexts,
+// column loading, hash build/import, pipeline runs, result fetch, errors.
+#include <cstring>
+#include <string>
+
+#include "hq_internal.h"
+
+void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h);
+void hq_hash_check(hq_ctx* ctx, hq_hash* h);
+
+namespace {
+thread_local std::string g_last_error = "";
+
+template <class F>
+hq_status guarded(F f) {
+  try {
+    f();
+    return HQ_OK;
+  } catch (const HqError& e) {
+    g_last_error = e.msg;
+    return e.code;
+  } catch (const std::bad_alloc&) {
+    g_last_error = "host allocation failed";
+    return HQ_ERR_OOM;
+  } catch (const std::exception& e) {
+    g_last_error = e.what();
+    return HQ_ERR_ARG;
+  }
+}
+
+void require_device() {
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
+    cudaGetLastError();
+    HQ_THROW(HQ_ERR_NO_DEVICE, "no CUDA device: libhq has no CPU fallback");
+  }
+}
+}  // namespace
+
+void hq_set_error(const std::string& msg) { g_last_error = msg; }
+
+void* hq_ctx::alloc_bytes(size_t bytes) {
+  if (bytes == 0) bytes = 16;
+  void* p = nullptr;
+  if (has_alloc) {
+    p = alloc.alloc(bytes, (void*)stream, alloc.user);
+  } else {
+    cudaError_t e = cudaMallocAsync(&p, bytes, stream);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+    }
+  }
+  if (!p) HQ_THROW(HQ_ERR_OOM, "device allocation of " + std::to_string(bytes) + " bytes failed");
+  return p;
+}
+void hq_ctx::free_bytes(void* p, size_t bytes) {
+  if (!p) return;
+  if (has_alloc) alloc.free(p, bytes, (void*)stream, alloc.user);
+  else cudaFreeAsync(p, stream);
+}
+
+hq_table::~hq_table() {
+  owned.clear();
+  if (backing) backing->release();
+}
+hq_result::~hq_result() {
+  if (fact) fact->release();
+  for (auto* h : hashes) h->release();
+}
+
+extern "C" {
+
+int32_t hq_abi_version(void) { return HQ_ABI_VERSION; }
+const char* hq_last_error(void) { return g_last_error.c_str(); }
+
+size_t hq_sizeof(const char* name) {
+  if (!name) return 0;
+  const std::string n(name);
+  if (n == "hq_column") return sizeof(hq_column);
+  if (n == "hq_pred") return sizeof(hq_pred);
+  if (n == "hq_build_desc") return sizeof(hq_build_desc);
+  if (n == "hq_hash_meta") return sizeof(hq_hash_meta);
+  if (n == "hq_insn") return sizeof(hq_insn);
+  if (n == "hq_op") return sizeof(hq_op);
+  if (n == "hq_plan") return sizeof(hq_plan);
+  if (n == "hq_result_info") return sizeof(hq_result_info);
+  if (n == "hq_allocator") return sizeof(hq_allocator);
+  return 0;
+}
+
+hq_status hq_ctx_create(int32_t device, void* stream, const hq_allocator* alloc, hq_ctx** out) {
+  return guarded([&] {
+    if (!out) HQ_THROW(HQ_ERR_ARG, "out is NULL");
+    require_device();
+    HQ_CUDA(cudaSetDevice(device));
+    hq_ctx* c = new hq_ctx();
+    c->device = device;
+    c->stream = (cudaStream_t)stream;
+    if (alloc && alloc->alloc && alloc->free) {
+      c->alloc = *alloc;
+      c->has_alloc = true;
+    }
+    int v = 0;
+    HQ_CUDA(cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device));
+    c->num_sms = v;
+    HQ_CUDA(cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, device));
+    c->max_smem = (size_t)v;
+    if (!c->has_alloc) {  // keep freed blocks cached in the stream-ordered pool
+      cudaMemPool_t pool;
+      if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+      }
+      cudaGetLastError();
+    }
+    *out = c;
+  });
+}
+
+hq_status hq_ctx_destroy(hq_ctx* ctx) {
+  return guarded([&] {
+    if (!ctx) return;
+    cudaStreamSynchronize(ctx->stream);
+    for (auto& e : ctx->events) {
+      cudaEventDestroy(e.first);
+      cudaEventDestroy(e.second);
+    }
+    for (auto e : ctx->event_pool) cudaEventDestroy(e);
+    delete ctx;
+  });
+}
+
+hq_status hq_ctx_set_stream(hq_ctx* ctx, void* stream) {
+  return guarded([&] {
+    if (!ctx) HQ_THROW(HQ_ERR_ARG, "ctx is NULL");
+    ctx->stream = (cudaStream_t)stream;
+  });
+}
+
+hq_status hq_ctx_sync(hq_ctx* ctx) {
+  return guarded([&] {
+    if (!ctx) HQ_THROW(HQ_ERR_ARG, "ctx is NULL");
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  });
+}
+
+hq_status hq_ctx_enable_timing(hq_ctx* ctx, int32_t on) {
+  return guarded([&] {
+    if (!ctx) HQ_THROW(HQ_ERR_ARG, "ctx is NULL");
+    ctx->timing = on != 0;
+  });
+}
+
+hq_status hq_ctx_kernel_times(hq_ctx* ctx, float* ms, int32_t max, int32_t* n) {
+  return guarded([&] {
+    if (!ctx || !n) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    int32_t k = 0;
+    for (auto& e : ctx->events) {
+      HQ_CUDA(cudaEventSynchronize(e.second));
+      float t = 0;
+      HQ_CUDA(cudaEventElapsedTime(&t, e.first, e.second));
+      if (ms && k < max) ms[k] = t;
+      ++k;
+      ctx->event_pool.push_back(e.first);
+      ctx->event_pool.push_back(e.second);
+    }
+    ctx->events.clear();
+    *n = k;
+  });
+}
+
+// ------------------------------------------------------------------ tables
+hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int64_t nrows, int32_t flags,
+                          hq_table** out) {
+  return guarded([&] {
+    if (!ctx || !out || (!cols && ncols > 0)) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    if (ncols < 0 || ncols > HQ_MAX_COLS) HQ_THROW(HQ_ERR_UNSUPPORTED, "tables have 0..16 columns");
+    if (nrows < 0) HQ_THROW(HQ_ERR_ARG, "nrows < 0");
+    if (flags != HQ_HOST_COPY && flags != HQ_DEVICE_BORROW) HQ_THROW(HQ_ERR_ARG, "flags must be HQ_HOST_COPY or HQ_DEVICE_BORROW");
+    hq_table* t = new hq_table();
+    t->ctx = ctx;
+    t->nrows = nrows;
+    t->ncols = ncols;
+    try {
+      for (int c = 0; c < ncols; ++c) {
+        const int w = hq_type_width(cols[c].type);
+        if (w == 0 || cols[c].type == HQ_F64) HQ_THROW(HQ_ERR_ARG, "column type must be HQ_I8/I32/I64");
+        if (!cols[c].data && nrows > 0) HQ_THROW(HQ_ERR_ARG, "column data is NULL");
+        t->cols[c].type = cols[c].type;
+        t->cols[c].width = w;
+        if (flags == HQ_HOST_COPY) {
+          const size_t bytes = (size_t)nrows * w;
+          // padded to a 16-B multiple so every TMA tile of the column is in bounds
+          t->owned.emplace_back(ctx, (bytes + 255) / 256 * 256 + 256);
+          if (bytes) HQ_CUDA(cudaMemcpyAsync(t->owned.back().p, cols[c].data, bytes, cudaMemcpyHostToDevice, ctx->stream));
+          t->cols[c].ptr = t->owned.back().p;
+        } else {
+          if (((uintptr_t)cols[c].data & 15) != 0) HQ_THROW(HQ_ERR_ARG, "device column pointer must be 16-byte aligned");
+          t->cols[c].ptr = cols[c].data;
+        }
+      }
+    } catch (...) {
+      t->release();
+      throw;
+    }
+    *out = t;
+  });
+}
+
+hq_status hq_table_info(const hq_table* t, int64_t* nrows, int32_t* ncols) {
+  return guarded([&] {
+    if (!t) HQ_THROW(HQ_ERR_ARG, "table is NULL");
+    if (nrows) *nrows = t->nrows;
+    if (ncols) *ncols = t->ncols;
+  });
+}
+
+hq_status hq_table_column(const hq_table* t, int32_t col, const void** dev_ptr, int32_t* type) {
+  return guarded([&] {
+    if (!t || col < 0 || col >= t->ncols) HQ_THROW(HQ_ERR_ARG, "bad table/column");
+    if (dev_ptr) *dev_ptr = t->cols[col].ptr;
+    if (type) *type = t->cols[col].type;
+  });
+}
+
+hq_status hq_free_table(hq_table* t) {
+  return guarded([&] {
+    if (t) t->release();
+  });
+}
+
+// -------------------------------------------------------------- hash tables
+hq_status hq_build_hash(hq_ctx* ctx, const hq_build_desc* desc, hq_hash** out) {
+  return guarded([&] {
+    if (!ctx || !desc || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    hq_hash* h = new hq_hash();
+    h->ctx = ctx;
+    try {
+      hq_build_hash_impl(ctx, desc, h);
+    } catch (...) {
+      h->release();
+      throw;
+    }
+    *out = h;
+  });
+}
+
+hq_status hq_hash_info(hq_ctx* ctx, const hq_hash* h, hq_hash_meta* meta) {
+  return guarded([&] {
+    if (!ctx || !h) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    hq_hash_check(ctx, const_cast<hq_hash*>(h));
+    if (meta) *meta = h->meta;
+  });
+}
+
+hq_status hq_hash_device_view(const hq_hash* h, void** dev_ptr, hq_hash_meta* meta) {
+  return guarded([&] {
+    if (!h) HQ_THROW(HQ_ERR_ARG, "hash is NULL");
+    if (dev_ptr) *dev_ptr = h->slots;
+    if (meta) *meta = h->meta;
+  });
+}
+
+hq_status hq_hash_import(hq_ctx* ctx, const hq_hash_meta* meta, void* dev_ptr, hq_hash** out) {
+  return guarded([&] {
+    if (!ctx || !meta || !dev_ptr || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    const int64_t cap = meta->capacity;
+    if (cap < 16 || (cap & (cap - 1)) != 0) HQ_THROW(HQ_ERR_ARG, "import: capacity must be a power of two >= 16");
+    if (meta->slot_words != 1 && meta->slot_words != 2 && meta->slot_words != 4) HQ_THROW(HQ_ERR_ARG, "import: slot_words");
+    if (meta->npayload < 0 || meta->npayload > meta->slot_words - 1 + (meta->slot_words == 1 ? 0 : 0) ||
+        (meta->slot_words == 1 && meta->npayload != 0))
+      HQ_THROW(HQ_ERR_ARG, "import: npayload");
+    if (((uintptr_t)dev_ptr & 15) != 0) HQ_THROW(HQ_ERR_ARG, "import: pointer must be 16-byte aligned");
+    hq_hash* h = new hq_hash();
+    h->ctx = ctx;
+    h->meta = *meta;
+    h->meta.bytes = cap * meta->slot_words * 4;
+    h->slots = (uint32_t*)dev_ptr;
+    int l = 0;
+    while ((1LL << l) < cap) ++l;
+    h->log2cap = l;
+    h->checked = true;
+    *out = h;
+  });
+}
+
+hq_status hq_free_hash(hq_hash* h) {
+  return guarded([&] {
+    if (h) h->release();
+  });
+}
+
+// ---------------------------------------------------------------- pipelines
+hq_status hq_run_pipeline(hq_ctx* ctx, const hq_plan* plan, hq_result** out) {
+  return guarded([&] {
+    if (!ctx || !plan || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    if (!plan->fact) HQ_THROW(HQ_ERR_ARG, "plan: fact table is NULL");
+    hq_result* r = new hq_result();
+    r->fact = const_cast<hq_table*>(plan->fact);
+    r->fact->retain();
+    for (int o = 0; o < plan->nops && o < HQ_MAX_OPS; ++o)
+      if (plan->ops[o].kind == HQ_OP_PROBE && plan->ops[o].ht) {
+        hq_hash* h = const_cast<hq_hash*>(plan->ops[o].ht);
+        h->retain();
+        r->hashes.push_back(h);
+      }
+    try {
+      hq_prepare_result(ctx, plan, r);
+    } catch (...) {
+      r->release();
+      throw;
+    }
+    *out = r;
+  });
+}
+
+hq_status hq_finalize(hq_ctx* ctx, hq_result* r) {
+  return guarded([&] {
+    if (!ctx || !r) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    hq_finalize_impl(ctx, r);
+  });
+}
+
+hq_status hq_result_info_get(hq_ctx* ctx, hq_result* r, hq_result_info* out) {
+  return guarded([&] {
+    if (!ctx || !r || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    hq_finalize_impl(ctx, r);
+    std::memset(out, 0, sizeof(*out));
+    out->nrows = r->nrows;
+    out->qualifying_rows = r->qualifying;
+    out->ncols = r->ncols;
+    for (int c = 0; c < r->ncols; ++c) out->types[c] = r->types[c];
+  });
+}
+
+hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int64_t capacity_rows,
+                          int64_t* nrows_out) {
+  return guarded([&] {
+    if (!ctx || !r) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    hq_finalize_impl(ctx, r);
+    const int64_t n = std::min<int64_t>(r->nrows, capacity_rows);
+    if (n > 0 && !host_cols) HQ_THROW(HQ_ERR_ARG, "host_cols is NULL");
+    for (int c = 0; c < r->ncols && n > 0; ++c) {
+      if (!host_cols[c]) continue;
+      const void* src = r->sink == HQ_SINK_MATERIALISE ? r->outcols[c].p : r->rescols[c].p;
+      const size_t w = (size_t)hq_type_width(r->types[c]);
+      HQ_CUDA(cudaMemcpyAsync(host_cols[c], src, (size_t)n * w, cudaMemcpyDeviceToHost, ctx->stream));
+    }
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    if (nrows_out) *nrows_out = r->nrows;
+  });
+}
+
+hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out) {
+  return guarded([&] {
+    if (!ctx || !r || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    if (r->sink != HQ_SINK_MATERIALISE) HQ_THROW(HQ_ERR_STATE, "only materialised results can be viewed as tables");
+    hq_finalize_impl(ctx, r);
+    hq_table* t = new hq_table();
+    t->ctx = ctx;
+    t->nrows = r->nrows;
+    t->ncols = r->ncols;
+    for (int c = 0; c < r->ncols; ++c) {
+      t->cols[c].ptr = r->outcols[c].p;
+      t->cols[c].type = r->types[c];
+      t->cols[c].width = hq_type_width(r->types[c]);
+    }
+    r->retain();
+    t->backing = r;
+    *out = t;
+  });
+}
+
+hq_status hq_result_partials_view(hq_result* r, void** dev_ptr, size_t* bytes) {
+  return guarded([&] {
+    if (!r) HQ_THROW(HQ_ERR_ARG, "result is NULL");
+    if (r->sink != HQ_SINK_AGG || r->gmode == hqk::GM_HASH)
+      HQ_THROW(HQ_ERR_UNSUPPORTED, "partials view needs a dense (or scalar) aggregation result");
+    for (int a = 0; a < r->plan.naggs; ++a)
+      if (r->plan.agg_fn[a] == HQ_AGG_MIN || r->plan.agg_fn[a] == HQ_AGG_MAX)
+        HQ_THROW(HQ_ERR_UNSUPPORTED, "partials view: MIN/MAX do not combine with a SUM reduce");
+    if (r->finalized) HQ_THROW(HQ_ERR_STATE, "result already finalized");
+    if (dev_ptr) *dev_ptr = r->gtab.p;
+    if (bytes) *bytes = (size_t)r->ngroups * r->vwords * 8;
+  });
+}
+
+hq_status hq_free_result(hq_result* r) {
+  return guarded([&] {
+    if (r) r->release();
+  });
+}
+
+}  // extern "C"

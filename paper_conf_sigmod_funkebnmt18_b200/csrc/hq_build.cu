@@ -1,0 +1,224 @@
+// hq_build.cu -- hash-join build, the pipeline breaker of a join (PAPER.md
+// P:186-195 "build hash table", P:1033-1036 inserts isolated with atomics,
+// P:1719-1720 dimension hash tables in GPU global memory).
+//
+// Open addressing with linear probing in a power-of-two slot array; a slot is
+// {int32 key, int32 payload[0..3]} of 1, 2 or 4 words (16-B slots load as one
+// int4 sector-aligned vector in the probe); the empty key is INT32_MIN.  A key
+// is claimed with ONE atomicCAS on the key word; payload words are then written
+// by the claiming thread (readers only run in later kernels, stream-ordered).
+// Capacity: next_pow2(ceil(keys / 0.6)) >= 16, keys counted exactly by a
+// predicate-only count pass unless the caller supplies expected_rows.
+#include <climits>
+
+#include "hq_internal.h"
+
+namespace {
+
+struct KBuildPred {
+  int16_t col;
+  uint8_t kind, neg;
+  int64_t lo, hi;
+  uint64_t bm[4];
+};
+struct KBuild {
+  int64_t n;
+  const char* col[HQ_MAX_COLS];
+  int32_t colw[HQ_MAX_COLS];
+  int32_t npreds;
+  KBuildPred preds[HQ_MAX_PREDS];
+  int32_t key_col, npay;
+  int32_t pay_col[HQ_MAX_PAYLOAD];
+  uint32_t* slots;
+  uint32_t mask;
+  int32_t log2cap, words;
+  int* err;
+  unsigned long long* nkeys;
+};
+
+__device__ __forceinline__ long long ld_col(const KBuild& b, int c, long long row) {
+  const int w = b.colw[c];
+  if (w == 4) return ((const int*)b.col[c])[row];
+  if (w == 8) return ((const long long*)b.col[c])[row];
+  return ((const signed char*)b.col[c])[row];
+}
+__device__ __forceinline__ bool row_passes(const KBuild& b, long long row) {
+  for (int i = 0; i < b.npreds; ++i) {
+    const KBuildPred& f = b.preds[i];
+    const long long v = ld_col(b, f.col, row);
+    bool ok;
+    if (f.kind == 0) ok = (v >= f.lo && v <= f.hi) != (bool)f.neg;
+    else ok = (unsigned long long)v < 256 && ((f.bm[v >> 6] >> (v & 63)) & 1ull);
+    if (!ok) return false;
+  }
+  return true;
+}
+
+__global__ void hq_build_count_kernel(const __grid_constant__ KBuild b) {
+  unsigned long long c = 0;
+  for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < b.n; r += (long long)gridDim.x * blockDim.x)
+    c += row_passes(b, r);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  __shared__ unsigned long long red[32];
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t = 0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
+    if (t) atomicAdd(b.nkeys, t);
+  }
+}
+
+__global__ void hq_fill_kernel(uint32_t* p, long long n, uint32_t v) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+    p[i] = v;
+}
+
+__global__ void hq_build_hash_kernel(const __grid_constant__ KBuild b) {
+  unsigned long long inserted = 0;
+  int fault = 0;
+  const uint32_t shift = 32u - b.log2cap;
+  for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < b.n; r += (long long)gridDim.x * blockDim.x) {
+    if (!row_passes(b, r)) continue;
+    const long long kv = ld_col(b, b.key_col, r);
+    if (kv <= (long long)INT_MIN || kv > (long long)INT_MAX) {
+      fault |= HQF_BAD_KEY;
+      continue;
+    }
+    const int key = (int)kv;
+    int pay[HQ_MAX_PAYLOAD] = {0, 0, 0};
+    for (int k = 0; k < b.npay; ++k) {
+      const long long v = ld_col(b, b.pay_col[k], r);
+      if (v < (long long)INT_MIN || v > (long long)INT_MAX) fault |= HQF_BAD_PAYLOAD;
+      pay[k] = (int)v;
+    }
+    uint32_t pos = ((uint32_t)key * 0x9E3779B1u) >> shift;
+    uint32_t i = 0;
+    for (; i <= b.mask; ++i) {
+      uint32_t* slot = b.slots + (size_t)pos * b.words;
+      const int old = atomicCAS((int*)slot, INT_MIN, key);
+      if (old == INT_MIN) {
+        for (int k = 0; k < b.npay; ++k) slot[1 + k] = (uint32_t)pay[k];
+        ++inserted;
+        break;
+      }
+      if (old == key) {
+        fault |= HQF_DUP_KEY;  // join keys must be unique (R6)
+        break;
+      }
+      pos = (pos + 1) & b.mask;
+    }
+    if (i > b.mask) fault |= HQF_HT_FULL;
+  }
+  if (fault) atomicOr(b.err, fault);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) inserted += __shfl_xor_sync(0xffffffffu, inserted, o);
+  if ((threadIdx.x & 31) == 0 && inserted) atomicAdd(b.nkeys, inserted);
+}
+
+int64_t next_pow2(int64_t x) {
+  int64_t c = 1;
+  while (c < x) c <<= 1;
+  return c;
+}
+
+void to_kpred(const hq_pred& in, KBuildPred& out, int ncols) {
+  if (in.reg < 0 || in.reg >= ncols) HQ_THROW(HQ_ERR_ARG, "build predicate column out of range");
+  out.col = (int16_t)in.reg;
+  out.kind = 0;
+  out.neg = 0;
+  std::memset(out.bm, 0, sizeof(out.bm));
+  switch (in.cmp) {
+    case HQ_EQ: out.lo = out.hi = in.lo; break;
+    case HQ_NE: out.lo = out.hi = in.lo; out.neg = 1; break;
+    case HQ_LT:
+      if (in.lo == LLONG_MIN) { out.lo = 1; out.hi = 0; } else { out.lo = LLONG_MIN; out.hi = in.lo - 1; }
+      break;
+    case HQ_LE: out.lo = LLONG_MIN; out.hi = in.lo; break;
+    case HQ_GT:
+      if (in.lo == LLONG_MAX) { out.lo = 1; out.hi = 0; } else { out.lo = in.lo + 1; out.hi = LLONG_MAX; }
+      break;
+    case HQ_GE: out.lo = in.lo; out.hi = LLONG_MAX; break;
+    case HQ_BETWEEN: out.lo = in.lo; out.hi = in.hi; break;
+    case HQ_IN_BITMAP: out.kind = 1; std::memcpy(out.bm, in.bitmap, sizeof(out.bm)); break;
+    default: HQ_THROW(HQ_ERR_ARG, "unknown comparison");
+  }
+}
+
+}  // namespace
+
+// Host side of hq_build_hash (called from hq_api.cu).
+void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
+  const hq_table* t = d->src;
+  if (!t) HQ_THROW(HQ_ERR_ARG, "build: NULL source table");
+  if (d->npreds < 0 || d->npreds > HQ_MAX_PREDS) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: too many predicates");
+  if (d->npayload < 0 || d->npayload > HQ_MAX_PAYLOAD) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: 0..3 payload columns");
+  if (d->key_col < 0 || d->key_col >= t->ncols) HQ_THROW(HQ_ERR_ARG, "build: key column out of range");
+  KBuild b{};
+  b.n = t->nrows;
+  for (int c = 0; c < t->ncols; ++c) {
+    b.col[c] = (const char*)t->cols[c].ptr;
+    b.colw[c] = t->cols[c].width;
+  }
+  b.npreds = d->npreds;
+  for (int i = 0; i < d->npreds; ++i) to_kpred(d->preds[i], b.preds[i], t->ncols);
+  b.key_col = d->key_col;
+  b.npay = d->npayload;
+  for (int k = 0; k < d->npayload; ++k) {
+    if (d->payload_cols[k] < 0 || d->payload_cols[k] >= t->ncols) HQ_THROW(HQ_ERR_ARG, "build: payload column out of range");
+    b.pay_col[k] = d->payload_cols[k];
+  }
+  h->dstate = DevBuf(ctx, 64);
+  HQ_CUDA(cudaMemsetAsync(h->dstate.p, 0, 64, ctx->stream));
+  b.err = h->dstate.as<int>();
+  b.nkeys = (unsigned long long*)(h->dstate.as<char>() + 8);
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((b.n + 255) / 256, (int64_t)ctx->num_sms * 8));
+  int64_t keys = d->expected_rows;
+  if (keys <= 0) {  // exact count pass (one sync)
+    if (b.n > 0) hq_build_count_kernel<<<grid, 256, 0, ctx->stream>>>(b);
+    HQ_CUDA(cudaGetLastError());
+    unsigned long long cnt = 0;
+    HQ_CUDA(cudaMemcpyAsync(&cnt, b.nkeys, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    HQ_CUDA(cudaMemsetAsync(b.nkeys, 0, 8, ctx->stream));
+    keys = (int64_t)cnt;
+  }
+  const int64_t cap = std::max<int64_t>(16, next_pow2((keys * 5 + 2) / 3));  // load factor <= 0.6
+  if (cap > (1LL << 31)) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: hash table too large");
+  const int words = d->npayload == 0 ? 1 : (d->npayload == 1 ? 2 : 4);
+  int log2 = 0;
+  while ((1LL << log2) < cap) ++log2;
+  h->owned = DevBuf(ctx, (size_t)cap * words * 4);
+  h->slots = h->owned.as<uint32_t>();
+  h->log2cap = log2;
+  h->meta.capacity = cap;
+  h->meta.slot_words = words;
+  h->meta.npayload = d->npayload;
+  h->meta.nkeys = -1;
+  h->meta.bytes = cap * words * 4;
+  const int64_t nw = cap * words;
+  const int fgrid = (int)std::max<int64_t>(1, std::min<int64_t>((nw + 255) / 256, (int64_t)ctx->num_sms * 8));
+  hq_fill_kernel<<<fgrid, 256, 0, ctx->stream>>>(h->slots, nw, 0x80000000u);
+  HQ_CUDA(cudaGetLastError());
+  b.slots = h->slots;
+  b.mask = (uint32_t)(cap - 1);
+  b.log2cap = log2;
+  b.words = words;
+  if (b.n > 0) hq_build_hash_kernel<<<grid, 256, 0, ctx->stream>>>(b);
+  HQ_CUDA(cudaGetLastError());
+}
+
+// Sync and report build faults (HQ_ERR_DUP_KEY etc.).
+void hq_hash_check(hq_ctx* ctx, hq_hash* h) {
+  if (h->checked || !h->dstate.p) return;
+  int st[4];
+  HQ_CUDA(cudaMemcpyAsync(st, h->dstate.p, 16, cudaMemcpyDeviceToHost, ctx->stream));
+  HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  h->meta.nkeys = (int64_t)(*(unsigned long long*)(st + 2));
+  h->checked = true;
+  if (st[0] & HQF_DUP_KEY) HQ_THROW(HQ_ERR_DUP_KEY, "hash build: duplicate key (join keys must be unique)");
+  if (st[0] & HQF_BAD_KEY) HQ_THROW(HQ_ERR_ARG, "hash build: key INT32_MIN or outside int32");
+  if (st[0] & HQF_BAD_PAYLOAD) HQ_THROW(HQ_ERR_ARG, "hash build: payload outside int32");
+  if (st[0] & HQF_HT_FULL) HQ_THROW(HQ_ERR_OVERFLOW, "hash build: table full (expected_rows too small)");
+}

@@ -1,0 +1,281 @@
+// hq_finalize.cu -- post-processing of aggregation results outside the
+// pipeline (sorting and decompression run after the
+// compiled kernels): compaction of the global group table into rows, AVG,
+// ORDER BY with a total tie-break, LIMIT.  Runs on the device of the context
+// (GPU 0 in the multi-GPU flow).
+#include <algorithm>
+#include <climits>
+#include <cstring>
+
+#include "hq_internal.h"
+
+using namespace hqk;
+
+namespace {
+
+constexpr int SORT_CHUNK = 2048;  // rows sorted per block in shared memory
+constexpr int MAXRC = HQ_MAX_KEYS + HQ_MAX_AGGS;
+
+struct KCompact {
+  const long long* gtab;
+  long long ngroups;  // dense groups or hash capacity
+  uint32_t vwords;
+  int hash;
+  int nkeys, naggs;
+  long long key_min[HQ_MAX_KEYS], key_card[HQ_MAX_KEYS], key_stride[HQ_MAX_KEYS];
+  uint8_t agg_fn[HQ_MAX_AGGS];
+  double agg_div[HQ_MAX_AGGS];  // 10^scale for AVG
+  long long* out[MAXRC];
+  unsigned long long* nout;     // [0] rows, [1] qualifying
+  int* err;
+  int scalar;
+};
+
+__global__ void hq_compact_kernel(const __grid_constant__ KCompact k) {
+  const uint32_t stride = k.vwords + (k.hash ? 1 : 0);
+  for (long long g = blockIdx.x * (long long)blockDim.x + threadIdx.x; g < k.ngroups;
+       g += (long long)gridDim.x * blockDim.x) {
+    const long long* e = k.gtab + g * stride;
+    unsigned long long key = (unsigned long long)g;
+    if (k.hash) {
+      key = (unsigned long long)e[0];
+      ++e;
+      if (key == EMPTY_KEY) continue;
+    }
+    const long long cnt = e[0];
+    if (cnt == 0 && !k.scalar) continue;
+    const unsigned long long row = atomicAdd(k.nout, 1ull);
+    atomicAdd(k.nout + 1, (unsigned long long)cnt);
+    for (int i = 0; i < k.nkeys; ++i)
+      k.out[i][row] = k.key_min[i] + (long long)((key / (unsigned long long)k.key_stride[i]) % (unsigned long long)k.key_card[i]);
+    bool big = false;
+    for (int a = 0; a < k.naggs; ++a) {
+      const long long v = e[1 + a];
+      long long* o = k.out[k.nkeys + a];
+      if (k.agg_fn[a] == HQ_AGG_AVG) {
+        const double d = cnt ? (double)v / (double)cnt / k.agg_div[a] : __longlong_as_double(0x7ff8000000000000LL);
+        o[row] = __double_as_longlong(d);
+      } else {
+        o[row] = v;
+      }
+      if ((k.agg_fn[a] == HQ_AGG_SUM || k.agg_fn[a] == HQ_AGG_AVG) && (v >= (1LL << 62) || v <= -(1LL << 62))) big = true;
+    }
+    if (big) atomicOr(k.err, HQF_OVERFLOW);
+  }
+}
+
+struct KSort {
+  const long long* col[MAXRC];
+  uint8_t isf[MAXRC];
+  int norder;
+  int ocol[HQ_MAX_ORDER];
+  int odesc[HQ_MAX_ORDER];
+  int nkeys;
+};
+
+__device__ __forceinline__ int cmp_val(const KSort& s, int c, int a, int b) {
+  const long long x = s.col[c][a], y = s.col[c][b];
+  if (s.isf[c]) {
+    const double dx = __longlong_as_double(x), dy = __longlong_as_double(y);
+    return dx < dy ? -1 : (dx > dy ? 1 : 0);
+  }
+  return x < y ? -1 : (x > y ? 1 : 0);
+}
+// total order: ORDER BY columns, then the group keys ascending, then row id
+__device__ __forceinline__ bool row_less(const KSort& s, int a, int b) {
+  if (a < 0) return false;  // padding sorts last
+  if (b < 0) return true;
+  for (int i = 0; i < s.norder; ++i) {
+    int c = cmp_val(s, s.ocol[i], a, b);
+    if (s.odesc[i]) c = -c;
+    if (c) return c < 0;
+  }
+  for (int i = 0; i < s.nkeys; ++i) {
+    const int c = cmp_val(s, i, a, b);
+    if (c) return c < 0;
+  }
+  return a < b;
+}
+
+// Each block sorts one chunk of <= SORT_CHUNK indices (bitonic network in
+// shared memory) and keeps its first `keep` rows.
+__global__ void __launch_bounds__(1024) hq_chunk_sort_kernel(const __grid_constant__ KSort s, const int* in, long long n,
+                                                             int* out, int keep) {
+  __shared__ int idx[SORT_CHUNK];
+  const long long base = (long long)blockIdx.x * SORT_CHUNK;
+  const int cnt = (int)(n - base < SORT_CHUNK ? n - base : SORT_CHUNK);
+  for (int i = threadIdx.x; i < SORT_CHUNK; i += blockDim.x) idx[i] = i < cnt ? (in ? in[base + i] : (int)(base + i)) : -1;
+  __syncthreads();
+  for (int k = 2; k <= SORT_CHUNK; k <<= 1) {
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < SORT_CHUNK; i += blockDim.x) {
+        const int l = i ^ j;
+        if (l > i) {
+          const int a = idx[i], b = idx[l];
+          const bool up = (i & k) == 0;
+          const bool sw = up ? row_less(s, b, a) : row_less(s, a, b);
+          if (sw) { idx[i] = b; idx[l] = a; }
+        }
+      }
+      __syncthreads();
+    }
+  }
+  const int m = keep < cnt ? keep : cnt;
+  for (int i = threadIdx.x; i < m; i += blockDim.x) out[(long long)blockIdx.x * keep + i] = idx[i];
+  for (int i = m + threadIdx.x; i < keep; i += blockDim.x) out[(long long)blockIdx.x * keep + i] = -1;
+}
+
+// one step of a global bitonic sort over a power-of-two index array
+__global__ void hq_bitonic_step_kernel(const __grid_constant__ KSort s, int* idx, long long n, long long j, long long k) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    const long long l = i ^ j;
+    if (l > i) {
+      const int a = idx[i], b = idx[l];
+      const bool up = (i & k) == 0;
+      const bool sw = up ? row_less(s, b, a) : row_less(s, a, b);
+      if (sw) { idx[i] = b; idx[l] = a; }
+    }
+  }
+}
+__global__ void hq_iota_kernel(int* idx, long long n, long long valid) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+    idx[i] = i < valid ? (int)i : -1;
+}
+__global__ void hq_gather_kernel(const long long* src, const int* idx, long long n, long long* dst) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+    dst[i] = src[idx[i]];
+}
+
+int grid_for(hq_ctx* ctx, long long n) {
+  return (int)std::max<long long>(1, std::min<long long>((n + 255) / 256, (long long)ctx->num_sms * 8));
+}
+
+}  // namespace
+
+void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
+  if (r->finalized) return;
+  hq_check_result_faults(ctx, r);
+  const hq_plan& P = r->plan;
+  if (r->sink == HQ_SINK_MATERIALISE) {
+    unsigned long long cnt = 0;
+    HQ_CUDA(cudaMemcpyAsync(&cnt, r->dstate.p, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    r->qualifying = (int64_t)cnt;
+    r->nrows = std::min<int64_t>((int64_t)cnt, r->capacity);
+    r->ncols = P.nout;
+    for (int j = 0; j < P.nout; ++j) r->types[j] = P.out_type[j];
+    r->finalized = true;
+    return;
+  }
+  // ---- AGG: compact
+  const int nk = P.nkeys, na = P.naggs, nc = nk + na;
+  r->ncols = nc;
+  const int64_t cap = std::max<int64_t>(r->ngroups, 1);
+  std::vector<DevBuf> cols;
+  for (int c = 0; c < nc; ++c) cols.emplace_back(ctx, (size_t)cap * 8);
+  DevBuf scratch(ctx, 64);
+  HQ_CUDA(cudaMemsetAsync(scratch.p, 0, 64, ctx->stream));
+  KCompact k{};
+  k.gtab = r->gtab.as<long long>();
+  k.ngroups = r->ngroups;
+  k.vwords = r->vwords;
+  k.hash = r->gmode == GM_HASH;
+  k.nkeys = nk;
+  k.naggs = na;
+  int64_t st = 1;
+  for (int i = nk - 1; i >= 0; --i) {
+    k.key_stride[i] = st;
+    st *= P.key_card[i];
+  }
+  for (int i = 0; i < nk; ++i) {
+    k.key_min[i] = P.key_min[i];
+    k.key_card[i] = P.key_card[i];
+    r->types[i] = HQ_I64;
+  }
+  for (int a = 0; a < na; ++a) {
+    k.agg_fn[a] = (uint8_t)P.agg_fn[a];
+    double d = 1.0;
+    for (int s = 0; s < P.agg_scale[a]; ++s) d *= 10.0;
+    k.agg_div[a] = d;
+    r->types[nk + a] = P.agg_fn[a] == HQ_AGG_AVG ? HQ_F64 : HQ_I64;
+  }
+  for (int c = 0; c < nc; ++c) k.out[c] = cols[c].as<long long>();
+  k.nout = scratch.as<unsigned long long>();
+  k.err = (int*)(scratch.as<char>() + 16);
+  k.scalar = nk == 0;
+  hq_compact_kernel<<<grid_for(ctx, r->ngroups), 256, 0, ctx->stream>>>(k);
+  HQ_CUDA(cudaGetLastError());
+  struct { unsigned long long rows, qual; int err; int pad; } st2{};
+  HQ_CUDA(cudaMemcpyAsync(&st2, scratch.p, sizeof(st2), cudaMemcpyDeviceToHost, ctx->stream));
+  HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  if (st2.err & HQF_OVERFLOW) HQ_THROW(HQ_ERR_OVERFLOW, "aggregate exceeds the int64 guard (|v| >= 2^62)");
+  const int64_t n = (int64_t)st2.rows;
+  r->qualifying = (int64_t)st2.qual;
+  int64_t nfinal = n;
+  if (P.limit > 0) nfinal = std::min<int64_t>(nfinal, P.limit);
+  // ---- ORDER BY (+ LIMIT)
+  if ((P.norder > 0 || nk > 0) && n > 1) {
+    KSort s{};
+    for (int c = 0; c < nc; ++c) {
+      s.col[c] = cols[c].as<long long>();
+      s.isf[c] = r->types[c] == HQ_F64;
+    }
+    if (P.norder < 0 || P.norder > HQ_MAX_ORDER) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: 0..4 ORDER BY columns");
+    s.norder = P.norder;
+    for (int i = 0; i < P.norder; ++i) {
+      if (P.order_col[i] < 0 || P.order_col[i] >= nc) HQ_THROW(HQ_ERR_ARG, "plan: ORDER BY column out of range");
+      s.ocol[i] = P.order_col[i];
+      s.odesc[i] = P.order_desc[i];
+    }
+    s.nkeys = nk;
+    DevBuf ia(ctx, (size_t)std::max<int64_t>(n, SORT_CHUNK) * 4 + 16), ib;
+    const int* cur = nullptr;  // NULL = identity
+    int64_t cur_n = n;
+    int* sorted = nullptr;
+    if (P.limit > 0 && P.limit <= SORT_CHUNK / 2) {
+      // top-k: chunk sorts keep `limit` rows each until one chunk remains
+      const int keep = (int)P.limit;
+      ib = DevBuf(ctx, (size_t)((n + SORT_CHUNK - 1) / SORT_CHUNK) * keep * 4 + 16);
+      int* bufs[2] = {ia.as<int>(), ib.as<int>()};
+      int which = 1;
+      while (true) {
+        const int64_t chunks = (cur_n + SORT_CHUNK - 1) / SORT_CHUNK;
+        const int kp = chunks == 1 ? (int)std::min<int64_t>(cur_n, SORT_CHUNK) : keep;
+        int* dst = bufs[which];
+        hq_chunk_sort_kernel<<<(unsigned)chunks, 1024, 0, ctx->stream>>>(s, cur, cur_n, dst, kp);
+        HQ_CUDA(cudaGetLastError());
+        cur = dst;
+        cur_n = chunks * kp;
+        which ^= 1;
+        if (chunks == 1) break;
+      }
+      sorted = (int*)cur;
+    } else if (n <= SORT_CHUNK) {
+      hq_chunk_sort_kernel<<<1, 1024, 0, ctx->stream>>>(s, nullptr, n, ia.as<int>(), SORT_CHUNK);
+      HQ_CUDA(cudaGetLastError());
+      sorted = ia.as<int>();
+    } else {
+      int64_t N = 1;
+      while (N < n) N <<= 1;
+      ia = DevBuf(ctx, (size_t)N * 4);
+      hq_iota_kernel<<<grid_for(ctx, N), 256, 0, ctx->stream>>>(ia.as<int>(), N, n);
+      for (int64_t kk = 2; kk <= N; kk <<= 1)
+        for (int64_t j = kk >> 1; j > 0; j >>= 1)
+          hq_bitonic_step_kernel<<<grid_for(ctx, N), 256, 0, ctx->stream>>>(s, ia.as<int>(), N, j, kk);
+      HQ_CUDA(cudaGetLastError());
+      sorted = ia.as<int>();
+    }
+    std::vector<DevBuf> out;
+    for (int c = 0; c < nc; ++c) {
+      out.emplace_back(ctx, (size_t)std::max<int64_t>(nfinal, 1) * 8);
+      hq_gather_kernel<<<grid_for(ctx, nfinal), 256, 0, ctx->stream>>>(cols[c].as<long long>(), sorted, nfinal,
+                                                                      out.back().as<long long>());
+    }
+    HQ_CUDA(cudaGetLastError());
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));  // scratch index buffers are released below
+    cols = std::move(out);
+  }
+  r->rescols = std::move(cols);
+  r->nrows = nfinal;
+  r->finalized = true;
+}

@@ -1,0 +1,269 @@
+// hq_internal.h -- internal objects and the device plan of libhq (not part of
+// the ABI).  See include/hq.h for the public contract and DESIGN.md for the
+// kernel design.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "hq.h"
+
+// ---------------------------------------------------------------- errors
+struct HqError {
+  hq_status code;
+  std::string msg;
+};
+void hq_set_error(const std::string& msg);
+#define HQ_THROW(code, msg)               \
+  do {                                    \
+    throw HqError{(code), (msg)};         \
+  } while (0)
+#define HQ_CUDA(call)                                                                    \
+  do {                                                                                   \
+    cudaError_t e_ = (call);                                                             \
+    if (e_ != cudaSuccess)                                                               \
+      throw HqError{HQ_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_)};    \
+  } while (0)
+
+// Device-side fault bits (KPlan::err), reported at the next syncing call.
+enum : int {
+  HQF_CAPACITY = 1,     // materialise output capacity exceeded
+  HQF_KEY_DOMAIN = 2,   // group key outside [key_min, key_min+key_card)
+  HQF_GROUP_FULL = 4,   // global group hash table full
+  HQF_DIV_ZERO = 8,     // division / modulo by zero
+  HQF_DUP_KEY = 16,     // duplicate build key
+  HQF_BAD_KEY = 32,     // build key INT32_MIN or outside int32
+  HQF_BAD_PAYLOAD = 64, // build payload outside int32
+  HQF_HT_FULL = 128,    // join hash table full (cannot happen when sized by the count pass)
+  HQF_OVERFLOW = 256    // int64 guard tripped (|aggregate| >= 2^62)
+};
+
+// ---------------------------------------------------------------- objects
+struct hq_ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  hq_allocator alloc{};
+  bool has_alloc = false;
+  int num_sms = 148;
+  size_t max_smem = 232448;
+  bool timing = false;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> events;  // recorded, not yet read
+  std::vector<cudaEvent_t> event_pool;
+  void* alloc_bytes(size_t bytes);
+  void free_bytes(void* p, size_t bytes);
+};
+
+// A device allocation owned through the context allocator.
+struct DevBuf {
+  hq_ctx* ctx = nullptr;
+  void* p = nullptr;
+  size_t bytes = 0;
+  DevBuf() = default;
+  DevBuf(hq_ctx* c, size_t n) : ctx(c), bytes(n) { p = c->alloc_bytes(n); }
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+  DevBuf(DevBuf&& o) noexcept : ctx(o.ctx), p(o.p), bytes(o.bytes) { o.p = nullptr; }
+  DevBuf& operator=(DevBuf&& o) noexcept {
+    release();
+    ctx = o.ctx; p = o.p; bytes = o.bytes; o.p = nullptr;
+    return *this;
+  }
+  ~DevBuf() { release(); }
+  void release() {
+    if (p && ctx) ctx->free_bytes(p, bytes);
+    p = nullptr;
+  }
+  template <class T> T* as() const { return (T*)p; }
+};
+
+struct RefObj {
+  std::atomic<int> refs{1};
+  virtual ~RefObj() {}
+  void retain() { refs.fetch_add(1); }
+  void release() {
+    if (refs.fetch_sub(1) == 1) delete this;
+  }
+};
+
+struct hq_result;
+
+struct TableCol {
+  const void* ptr = nullptr;
+  int type = 0;
+  int width = 0;
+};
+
+struct hq_table : RefObj {
+  hq_ctx* ctx = nullptr;
+  int64_t nrows = 0;
+  int ncols = 0;
+  TableCol cols[HQ_MAX_COLS];
+  std::vector<DevBuf> owned;
+  hq_result* backing = nullptr;  // retained when the table views a result
+  ~hq_table() override;
+};
+
+struct hq_hash : RefObj {
+  hq_ctx* ctx = nullptr;
+  hq_hash_meta meta{};
+  int log2cap = 0;
+  uint32_t* slots = nullptr;
+  DevBuf owned;      // slot array (empty when imported)
+  DevBuf dstate;     // [0] fault bits (int), [1..2] nkeys (u64) -- see hq_build.cu
+  bool checked = false;
+};
+
+// ------------------------------------------------- device plan (kernel param)
+namespace hqk {
+constexpr int NW = 16;                   // consumer warps per CTA
+constexpr int NTHREADS = (NW + 1) * 32;  // + 1 TMA producer warp
+constexpr int MAX_STAGES = 10;
+constexpr int MAX_PREDS = 16;
+constexpr int MAX_PROBES = 8;
+constexpr int MAX_COMPUTES = 8;
+constexpr int MAX_INSNS = 64;
+constexpr int NREGS = HQ_MAX_COLS + HQ_MAX_TMP;
+constexpr int SMEM_AGG_BYTES = 32 * 1024;
+constexpr int64_t DENSE_LIMIT = 65536;
+constexpr unsigned long long EMPTY_KEY = ~0ULL;
+
+enum : uint8_t { OP_FILTER = 1, OP_PROBE = 2, OP_COMPUTE = 3 };
+enum : uint8_t { GM_SCALAR = 0, GM_DENSE = 1, GM_HASH = 2 };   // global group table
+enum : uint8_t { SM_NONE = 0, SM_DENSE = 1, SM_HASH = 2 };     // smem pre-aggregation table
+
+struct KReg {
+  uint32_t off;      // byte offset of row 0 in the stage (column) or tmp region (temporary)
+  uint8_t width;     // 1, 4, 8
+  uint8_t in_stage;  // 1 = fact column staged by TMA, 0 = temporary
+  uint8_t pad[2];
+};
+struct KCol {
+  const char* ptr;
+  uint32_t width;
+  uint32_t soff;     // byte offset inside a stage
+};
+struct KPred {
+  int16_t reg;
+  uint8_t kind;      // 0 = range [lo, hi], 1 = bitmap
+  uint8_t neg;       // result negated (NE)
+  int32_t lo32, hi32;
+  int64_t lo, hi;
+  uint64_t bm[4];
+};
+struct KProbe {
+  const uint32_t* slots;
+  uint32_t mask;     // capacity - 1
+  uint8_t log2cap;
+  uint8_t words;     // 1, 2, 4
+  uint8_t mode;      // hq_probe_mode
+  uint8_t npay;
+  int16_t key_reg;
+  int16_t dst[HQ_MAX_PAYLOAD];
+};
+struct KCompute {
+  int16_t dst;
+  uint8_t first;
+  uint8_t n;
+};
+struct KInsn {
+  uint8_t opc;
+  uint8_t pad;
+  int16_t reg;       // < 0: immediate
+  int32_t pad2;
+  int64_t imm;
+};
+struct KOp {
+  uint8_t kind;
+  uint8_t idx;
+};
+
+struct KPlan {
+  int64_t row_begin, row_end;
+  int32_t R, tile_rows, nstages;
+  uint32_t stage_bytes;      // bytes of one stage's columns (= tile_rows * row width)
+  uint32_t stage_stride;     // stage spacing in smem (>= stage_bytes, 128-B multiple)
+  uint32_t off_tmp, off_agg, off_stage;  // dynamic smem layout
+  int32_t ncols;
+  KCol cols[HQ_MAX_COLS];
+  KReg regs[NREGS];
+  int32_t nops;
+  KOp ops[HQ_MAX_OPS];
+  KPred preds[MAX_PREDS];
+  KProbe probes[MAX_PROBES];
+  KCompute comps[MAX_COMPUTES];
+  KInsn insns[MAX_INSNS];
+  // sink
+  int32_t sink, resolution;
+  int32_t nkeys;
+  int16_t key_reg[HQ_MAX_KEYS];
+  int64_t key_min[HQ_MAX_KEYS];
+  int64_t key_card[HQ_MAX_KEYS];
+  int64_t key_stride[HQ_MAX_KEYS];
+  int32_t naggs;
+  uint8_t agg_fn[HQ_MAX_AGGS];
+  int16_t agg_reg[HQ_MAX_AGGS];
+  uint8_t gmode, smode;
+  uint32_t vwords;           // 1 + naggs: [count, agg...] per group
+  long long* gtab;           // global dense table or hash entries [key, count, agg...]
+  uint64_t gmask;            // hash capacity - 1
+  int32_t glog2;
+  uint32_t smem_cap;         // smem dense groups or smem hash slots
+  int32_t slog2;
+  // materialise
+  int32_t nout;
+  int16_t out_reg[HQ_MAX_OUT];
+  uint8_t out_width[HQ_MAX_OUT];
+  void* out_ptr[HQ_MAX_OUT];
+  int64_t capacity;
+  // status
+  unsigned long long* counter;  // qualifying rows / write counter
+  int* err;
+};
+}  // namespace hqk
+
+struct hq_result : RefObj {
+  hq_ctx* ctx = nullptr;
+  hq_plan plan{};
+  hq_table* fact = nullptr;
+  std::vector<hq_hash*> hashes;
+  int sink = 0;
+  uint8_t gmode = 0;
+  int64_t ngroups = 0;        // dense groups or hash capacity
+  uint32_t vwords = 0;
+  DevBuf gtab;                // group table
+  DevBuf dstate;              // [0..1] counter (u64), [2] fault bits (int), [3] spare
+  // materialise
+  std::vector<DevBuf> outcols;
+  int64_t capacity = 0;
+  // finalized AGG rows
+  bool finalized = false;
+  bool checked = false;
+  int64_t nrows = 0;
+  int64_t qualifying = 0;
+  int ncols = 0;
+  int types[HQ_MAX_KEYS + HQ_MAX_AGGS] = {0};
+  std::vector<DevBuf> rescols;  // finalized result columns (int64 / f64)
+  ~hq_result() override;
+};
+
+// ---------------------------------------------------------------- launchers
+namespace hqk {
+void launch_fused(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem);
+void launch_init_groups(hq_ctx* ctx, long long* tab, int64_t ngroups, uint32_t vwords, bool hash,
+                        const uint8_t* agg_fn, int naggs);
+int64_t fused_smem_bytes(const KPlan& kp);
+}  // namespace hqk
+
+// finalize: compaction + AVG + ORDER BY + LIMIT (hq_finalize.cu)
+void hq_finalize_impl(hq_ctx* ctx, hq_result* r);
+// op-at-a-time execution of a plan (hq_oaat.cu)
+void hq_run_oaat(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
+// shared plan preparation (hq_pipeline.cu)
+void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
+void hq_check_result_faults(hq_ctx* ctx, hq_result* r);
+int hq_type_width(int type);

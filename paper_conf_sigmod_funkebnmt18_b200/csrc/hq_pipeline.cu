@@ -1,0 +1,759 @@
+// hq_pipeline.cu -- the fused pipeline ("compound") kernel of HorseQC on sm_100a.
+//
+// PAPER.md §5.2 / Fig 12: all phases of a fusion operator -- select,
+// join probe, (prefix sum | reduction), project/write -- run in ONE kernel; flags,
+// probe payloads and write offsets stay on chip (registers / shared memory).
+// §6.1: write offsets and aggregates use *local resolution, global
+// propagation* (LRGP): resolve inside the thread group first (warp ballots /
+// shuffles, block scan, shared-memory tables), then one global atomic per group.
+//
+// B200 design:
+//  * persistent grid, one CTA per SM, 16 consumer warps + 1 TMA producer warp;
+//  * the producer streams the referenced fact columns tile by tile with 1-D TMA
+//    bulk copies (cp.async.bulk, L2 evict_first) into an S-stage shared-memory
+//    ring guarded by mbarriers (full: tx bytes, empty: one arrive per consumer
+//    warp), so HBM reads run ahead of the processing;
+//  * each consumer warp owns 32*R consecutive rows of a tile (lane + 32 r) and
+//    walks the plan's ops over them: predicates -> per-thread live bit masks,
+//    probes -> open-addressing lookups with R independent loads in flight,
+//    expressions -> int64 accumulator machine; temporaries live in a per-lane
+//    shared-memory region;
+//  * sinks: scalar aggregates in registers (B3), grouped aggregates combined per
+//    warp (match_any + shuffle reduction) into a shared-memory dense or hash
+//    table and merged with global atomics at the end (C3, overflow -> C2),
+//    materialisation with a ballot/popc warp scan, a block scan and ONE atomicAdd
+//    per block and tile (A3, Fig 25 P:2064-2092 / P:1069-1072).
+#include <climits>
+#include <cstring>
+
+#include "hq_internal.h"
+
+namespace hqk {
+
+#define FULLMASK 0xffffffffu
+
+// ----------------------------------------------------------- PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t tx) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(tx) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "HQ_WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra HQ_WAIT_%=;\n}\n" ::"r"(smem_u32(b)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
+                                            uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void consumer_bar() {  // all consumer warps (not the producer)
+  asm volatile("bar.sync 1, %0;" ::"n"(NW * 32) : "memory");
+}
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+// ------------------------------------------------------------ reg access
+template <int R>
+__device__ __forceinline__ void load_rows(const KPlan& p, int reg, const char* stage, const char* tmp,
+                                          int row0, long long (&v)[R]) {
+  const KReg d = p.regs[reg];
+  const char* base = (d.in_stage ? stage : tmp) + d.off;
+  if (d.width == 4) {
+    const int* b = (const int*)base + row0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) v[r] = b[r * 32];
+  } else if (d.width == 8) {
+    const long long* b = (const long long*)base + row0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) v[r] = b[r * 32];
+  } else {
+    const signed char* b = (const signed char*)base + row0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) v[r] = b[r * 32];
+  }
+}
+__device__ __forceinline__ long long load_one(const KPlan& p, int reg, const char* stage, const char* tmp,
+                                              int row) {
+  const KReg d = p.regs[reg];
+  const char* base = (d.in_stage ? stage : tmp) + d.off;
+  if (d.width == 4) return ((const int*)base)[row];
+  if (d.width == 8) return ((const long long*)base)[row];
+  return ((const signed char*)base)[row];
+}
+template <int R>
+__device__ __forceinline__ void store_tmp(const KPlan& p, int reg, char* tmp, int row0, const long long (&v)[R]) {
+  const KReg d = p.regs[reg];
+  if (d.width == 8) {
+    long long* b = (long long*)(tmp + d.off) + row0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) b[r * 32] = v[r];
+  } else {
+    int* b = (int*)(tmp + d.off) + row0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) b[r * 32] = (int)v[r];
+  }
+}
+
+// ------------------------------------------------------------------ ops
+// Selection (Fig 8 count kernel "select"): conjunction of
+// range / bitmap predicates folded into the per-thread live mask.
+template <int R>
+__device__ __forceinline__ uint32_t op_filter(const KPlan& p, int idx, const char* stage, const char* tmp,
+                                              int row0, uint32_t mask) {
+  const KPred& f = p.preds[idx];
+  const KReg d = p.regs[f.reg];
+  const char* base = (d.in_stage ? stage : tmp) + d.off;
+  if (f.kind == 0 && d.width == 4) {
+    const int* b = (const int*)base + row0;
+    const int lo = f.lo32, hi = f.hi32;
+    const bool neg = f.neg;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int v = b[r * 32];
+      const bool ok = (v >= lo && v <= hi) != neg;
+      if (!ok) mask &= ~(1u << r);
+    }
+    return mask;
+  }
+  long long v[R];
+  load_rows<R>(p, f.reg, stage, tmp, row0, v);
+  if (f.kind == 0) {
+    const long long lo = f.lo, hi = f.hi;
+    const bool neg = f.neg;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const bool ok = (v[r] >= lo && v[r] <= hi) != neg;
+      if (!ok) mask &= ~(1u << r);
+    }
+  } else {
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const unsigned long long x = (unsigned long long)v[r];
+      const bool ok = x < 256 && ((f.bm[x >> 6] >> (x & 63)) & 1ull);
+      if (!ok) mask &= ~(1u << r);
+    }
+  }
+  return mask;
+}
+
+// Join probe (Fig 8 "check match" + "build tuple"): in the
+// compound kernel the probe runs once and the payload stays on chip
+// (P:947-953).  Linear probing over {key, payload...} slots of W words.
+template <int R, int W>
+__device__ __forceinline__ uint32_t probe_rows(const KPlan& p, const KProbe& pr, const long long (&kv)[R],
+                                               char* tmp, int row0, uint32_t mask) {
+  uint32_t pending = mask, found = 0;
+  uint32_t pos[R];
+  const uint32_t shift = 32u - pr.log2cap;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const bool ok = kv[r] > (long long)INT_MIN && kv[r] <= (long long)INT_MAX;
+    if (!ok) pending &= ~(1u << r);
+    pos[r] = ((uint32_t)(int)kv[r] * 0x9E3779B1u) >> shift;
+  }
+  const bool inner = pr.mode == HQ_PROBE_INNER;
+  int* dst0 = (int*)(tmp + p.regs[pr.dst[0]].off) + row0;
+  int* dst1 = (int*)(tmp + p.regs[pr.dst[W > 2 ? 1 : 0]].off) + row0;
+  int* dst2 = (int*)(tmp + p.regs[pr.dst[W > 2 ? 2 : 0]].off) + row0;
+  while (pending) {
+    int4 sl[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {  // R independent slot loads in flight
+      if (pending & (1u << r)) {
+        if (W == 1) sl[r].x = __ldg((const int*)pr.slots + pos[r]);
+        else if (W == 2) { const int2 t = __ldg((const int2*)pr.slots + pos[r]); sl[r].x = t.x; sl[r].y = t.y; }
+        else sl[r] = __ldg((const int4*)pr.slots + pos[r]);
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (pending & (1u << r)) {
+        if (sl[r].x == (int)kv[r]) {
+          found |= 1u << r;
+          pending &= ~(1u << r);
+          if (W > 1 && inner) {  // payload stays on chip
+            if (pr.npay > 0) dst0[r * 32] = sl[r].y;
+            if (W > 2 && pr.npay > 1) dst1[r * 32] = sl[r].z;
+            if (W > 2 && pr.npay > 2) dst2[r * 32] = sl[r].w;
+          }
+        } else if (sl[r].x == INT_MIN) {
+          pending &= ~(1u << r);
+        } else {
+          pos[r] = (pos[r] + 1) & pr.mask;
+        }
+      }
+    }
+  }
+  if (pr.mode == HQ_PROBE_ANTI) return mask & ~found;
+  return mask & found;
+}
+
+template <int R>
+__device__ __forceinline__ uint32_t op_probe(const KPlan& p, int idx, const char* stage, char* tmp, int row0,
+                                             uint32_t mask) {
+  const KProbe& pr = p.probes[idx];
+  long long kv[R];
+  load_rows<R>(p, pr.key_reg, stage, tmp, row0, kv);
+  if (pr.words == 1) return probe_rows<R, 1>(p, pr, kv, tmp, row0, mask);
+  if (pr.words == 2) return probe_rows<R, 2>(p, pr, kv, tmp, row0, mask);
+  return probe_rows<R, 4>(p, pr, kv, tmp, row0, mask);
+}
+
+// Projection / arithmetic (revenue[wp] = price[tid]*discount[tid]):
+// an int64 accumulator machine, one instruction stream per plan, evaluated for
+// the lane's R rows at once.
+template <int R>
+__device__ __forceinline__ void op_compute(const KPlan& p, int idx, const char* stage, char* tmp, int row0,
+                                           uint32_t mask) {
+  const KCompute c = p.comps[idx];
+  long long acc[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) acc[r] = 0;
+  for (int i = c.first; i < c.first + c.n; ++i) {
+    const KInsn in = p.insns[i];
+    long long o[R];
+    if (in.reg < 0) {
+#pragma unroll
+      for (int r = 0; r < R; ++r) o[r] = in.imm;
+    } else {
+      load_rows<R>(p, in.reg, stage, tmp, row0, o);
+    }
+    switch (in.opc) {
+      case HQ_I_LOAD:
+#pragma unroll
+        for (int r = 0; r < R; ++r) acc[r] = o[r];
+        break;
+      case HQ_I_ADD:
+#pragma unroll
+        for (int r = 0; r < R; ++r) acc[r] += o[r];
+        break;
+      case HQ_I_SUB:
+#pragma unroll
+        for (int r = 0; r < R; ++r) acc[r] -= o[r];
+        break;
+      case HQ_I_RSUB:
+#pragma unroll
+        for (int r = 0; r < R; ++r) acc[r] = o[r] - acc[r];
+        break;
+      case HQ_I_MUL:
+#pragma unroll
+        for (int r = 0; r < R; ++r) acc[r] *= o[r];
+        break;
+      default: {  // DIV / MOD
+        bool bad = false;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (o[r] == 0) {
+            bad |= (mask >> r) & 1u;
+            acc[r] = 0;
+          } else {
+            acc[r] = in.opc == HQ_I_DIV ? acc[r] / o[r] : acc[r] % o[r];
+          }
+        }
+        if (bad) atomicOr(p.err, HQF_DIV_ZERO);
+      }
+    }
+  }
+  store_tmp<R>(p, c.dst, tmp, row0, acc);
+}
+
+// --------------------------------------------------------------- agg tables
+__device__ __forceinline__ long long agg_identity(uint8_t fn) {
+  return fn == HQ_AGG_MIN ? LLONG_MAX : (fn == HQ_AGG_MAX ? LLONG_MIN : 0);
+}
+__device__ __forceinline__ long long agg_combine(uint8_t fn, long long a, long long b) {
+  return fn == HQ_AGG_MIN ? (a < b ? a : b) : (fn == HQ_AGG_MAX ? (a > b ? a : b) : a + b);
+}
+__device__ __forceinline__ long long warp_reduce(uint8_t fn, long long v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = agg_combine(fn, v, __shfl_xor_sync(FULLMASK, v, o));
+  return v;
+}
+// one aggregate update with a shared- or global-memory atomic
+__device__ __forceinline__ void agg_atomic(uint8_t fn, long long* t, long long v, unsigned long long cnt) {
+  if (fn == HQ_AGG_MIN) atomicMin(t, v);
+  else if (fn == HQ_AGG_MAX) atomicMax(t, v);
+  else if (fn == HQ_AGG_COUNT) atomicAdd((unsigned long long*)t, cnt);
+  else atomicAdd((unsigned long long*)t, (unsigned long long)v);
+}
+// accumulate (count, vals) into one table entry [count, agg...] with atomics
+__device__ __forceinline__ void entry_update(const KPlan& p, long long* e, unsigned long long cnt,
+                                             const long long* vals) {
+  atomicAdd((unsigned long long*)e, cnt);
+  for (int a = 0; a < p.naggs; ++a) agg_atomic(p.agg_fn[a], e + 1 + a, vals[a], cnt);
+}
+__device__ __forceinline__ uint32_t hash64(unsigned long long k, int log2) {
+  return (uint32_t)((k * 0x9E3779B97F4A7C15ull) >> (64 - log2));
+}
+// Global propagation target: dense array slot, or the entry of `key` in the
+// global hash table, claimed with atomicCAS ("atomic_hash_reduce", App C
+// P:2049-2052).  NULL (fault raised) when the hash table is full.
+__device__ long long* global_locate(const KPlan& p, unsigned long long key) {
+  if (p.gmode != GM_HASH) return p.gtab + key * p.vwords;
+  const uint32_t vw1 = p.vwords + 1;
+  uint64_t h = hash64(key, p.glog2);
+  for (uint64_t i = 0; i <= p.gmask; ++i) {
+    unsigned long long* kp = (unsigned long long*)(p.gtab + h * vw1);
+    const unsigned long long k = *(volatile unsigned long long*)kp;
+    if (k == key) return p.gtab + h * vw1 + 1;
+    if (k == EMPTY_KEY) {
+      const unsigned long long old = atomicCAS(kp, EMPTY_KEY, key);
+      if (old == EMPTY_KEY || old == key) return p.gtab + h * vw1 + 1;
+    }
+    h = (h + 1) & p.gmask;
+  }
+  atomicOr(p.err, HQF_GROUP_FULL);
+  return nullptr;
+}
+__device__ __forceinline__ void global_update(const KPlan& p, unsigned long long key, unsigned long long cnt,
+                                              const long long* vals) {
+  long long* e = global_locate(p, key);
+  if (e) entry_update(p, e, cnt, vals);
+}
+// Local resolution target: the shared-memory dense table or hash table entry;
+// falls back to the global table when the smem hash table is full (C3 -> C2).
+__device__ __forceinline__ long long* local_locate(const KPlan& p, char* sagg, unsigned long long key) {
+  if (p.smode == SM_DENSE) return (long long*)sagg + key * p.vwords;
+  if (p.smode == SM_HASH) {
+    unsigned long long* keys = (unsigned long long*)sagg;
+    long long* ent = (long long*)sagg + p.smem_cap;
+    const uint32_t m = p.smem_cap - 1;
+    uint32_t h = hash64(key, p.slog2);
+#pragma unroll 1
+    for (int i = 0; i < 32; ++i) {
+      const unsigned long long k = keys[h];
+      bool hit = k == key;
+      if (!hit && k == EMPTY_KEY) {
+        const unsigned long long old = atomicCAS(keys + h, EMPTY_KEY, key);
+        hit = old == EMPTY_KEY || old == key;
+      }
+      if (hit) return ent + (size_t)h * p.vwords;
+      h = (h + 1) & m;
+    }
+  }
+  return global_locate(p, key);
+}
+
+// ------------------------------------------------------------------- sinks
+// Grouped aggregation with local resolution (C3-style, P:1211-1220,
+// P:2040-2057): per row slot, lanes with equal keys are combined with
+// match_any + shuffle reductions so each distinct key of a warp costs one
+// shared-memory update; singletons update directly.
+template <int R>
+__device__ __forceinline__ void sink_group(const KPlan& p, const char* stage, const char* tmp, char* sagg,
+                                           int row0, uint32_t mask, int lane) {
+  unsigned long long gk[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) gk[r] = 0;
+  for (int i = 0; i < p.nkeys; ++i) {
+    long long v[R];
+    load_rows<R>(p, p.key_reg[i], stage, tmp, row0, v);
+    const long long mn = p.key_min[i], card = p.key_card[i], st = p.key_stride[i];
+    bool bad = false;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const long long d = v[r] - mn;
+      if (d < 0 || d >= card) {
+        bad |= (mask >> r) & 1u;
+        mask &= ~(1u << r);
+      }
+      gk[r] += (unsigned long long)d * (unsigned long long)st;
+    }
+    if (bad) atomicOr(p.err, HQF_KEY_DOMAIN);
+  }
+  const bool c2 = p.resolution == HQ_RES_ATOMIC;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const bool live = (mask >> r) & 1u;
+    const uint32_t act = __ballot_sync(FULLMASK, live);
+    if (!act) continue;
+    const int row = row0 + r * 32;
+    const unsigned long long mk = live ? gk[r] : EMPTY_KEY;
+    const uint32_t peers = c2 ? (1u << lane) & act : __match_any_sync(FULLMASK, mk) & act;
+    const bool single = live && __popc(peers) == 1;
+    if (single) {  // C2 rows, and keys unique within the warp: direct update
+      long long* e = c2 ? global_locate(p, gk[r]) : local_locate(p, sagg, gk[r]);
+      if (e) {
+        atomicAdd((unsigned long long*)e, 1ull);
+        for (int a = 0; a < p.naggs; ++a) {
+          const uint8_t fn = p.agg_fn[a];
+          agg_atomic(fn, e + 1 + a, fn == HQ_AGG_COUNT ? 1 : load_one(p, p.agg_reg[a], stage, tmp, row), 1);
+        }
+      }
+    }
+    uint32_t multi = act & ~__ballot_sync(FULLMASK, single);
+    while (multi) {  // one warp-wide reduction per distinct key, leader updates
+      const int leader = __ffs(multi) - 1;
+      const uint32_t grp = __shfl_sync(FULLMASK, peers, leader);
+      const bool mine = (grp >> lane) & 1u;
+      long long* e = nullptr;
+      if (lane == leader) {
+        e = local_locate(p, sagg, gk[r]);
+        if (e) atomicAdd((unsigned long long*)e, (unsigned long long)__popc(grp));
+      }
+      for (int a = 0; a < p.naggs; ++a) {
+        const uint8_t fn = p.agg_fn[a];
+        long long v = agg_identity(fn);
+        if (mine) v = fn == HQ_AGG_COUNT ? 1 : load_one(p, p.agg_reg[a], stage, tmp, row);
+        v = warp_reduce(fn, v);
+        if (lane == leader && e) agg_atomic(fn, e + 1 + a, v, (unsigned long long)__popc(grp));
+      }
+      multi &= ~grp;
+    }
+  }
+}
+
+// Materialisation with LRGP (A3; Fig 25): warp
+// ballot/popc prefix, block scan over the warps, one atomicAdd per block and
+// tile, write at local offset + global offset.  Rows stay in order inside the
+// block's segment; segments are permuted.
+template <int R>
+__device__ __forceinline__ void sink_materialise(const KPlan& p, const char* stage, const char* tmp, int row0,
+                                                 uint32_t mask, int warp, int lane, int* s_wtot,
+                                                 unsigned long long* s_base) {
+  uint32_t b[R];
+  int wtot = 0;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    b[r] = __ballot_sync(FULLMASK, (mask >> r) & 1u);
+    wtot += __popc(b[r]);
+  }
+  unsigned long long base;
+  if (p.resolution == HQ_RES_ATOMIC) {
+    base = 0;  // per-row atomics below (A2)
+  } else {
+    if (lane == 0) s_wtot[warp] = wtot;
+    consumer_bar();
+    if (warp == 0) {
+      int v = lane < NW ? s_wtot[lane] : 0;
+      int incl = v;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(FULLMASK, incl, o);
+        if (lane >= o) incl += t;
+      }
+      const int total = __shfl_sync(FULLMASK, incl, 31);
+      unsigned long long g = 0;
+      if (lane == 0 && total > 0) g = atomicAdd(p.counter, (unsigned long long)total);  // global propagation
+      g = __shfl_sync(FULLMASK, g, 0);
+      if (lane < NW) s_base[lane] = g + (unsigned long long)(incl - v);
+    }
+    consumer_bar();
+    base = s_base[warp];
+  }
+  const uint32_t lt = lanemask_lt();
+  unsigned long long run = 0;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    if ((mask >> r) & 1u) {
+      unsigned long long pos;
+      if (p.resolution == HQ_RES_ATOMIC) pos = atomicAdd(p.counter, 1ull);
+      else pos = base + run + __popc(b[r] & lt);
+      if ((long long)pos < p.capacity) {
+        const int row = row0 + r * 32;
+        for (int j = 0; j < p.nout; ++j) {
+          const long long v = load_one(p, p.out_reg[j], stage, tmp, row);
+          const uint8_t w = p.out_width[j];
+          if (w == 8) ((long long*)p.out_ptr[j])[pos] = v;
+          else if (w == 4) ((int*)p.out_ptr[j])[pos] = (int)v;
+          else ((signed char*)p.out_ptr[j])[pos] = (signed char)v;
+        }
+      } else {
+        atomicOr(p.err, HQF_CAPACITY);
+      }
+    }
+    run += __popc(b[r]);
+  }
+}
+
+// ------------------------------------------------------------------ kernel
+// SK: sink kind, a template parameter so each instantiation only carries the
+// registers of its own sink (0 = scalar aggregate, 1 = grouped, 2 = materialise).
+enum { SK_SCALAR = 0, SK_GROUP = 1, SK_MAT = 2 };
+template <int R, int SK>
+__global__ void __launch_bounds__(NTHREADS, 1) hq_fused_pipeline_kernel(const __grid_constant__ KPlan p) {
+  extern __shared__ __align__(128) char smem[];
+  uint64_t* full = (uint64_t*)smem;
+  uint64_t* empty = full + MAX_STAGES;
+  unsigned long long* s_base = (unsigned long long*)(empty + MAX_STAGES);  // [NW]
+  int* s_wtot = (int*)(s_base + NW);                                         // [NW]
+  long long* s_red = (long long*)(s_wtot + NW);                              // [NW][1+MAX_AGGS]
+  char* tmp = smem + p.off_tmp;
+  char* sagg = smem + p.off_agg;
+  char* stages = smem + p.off_stage;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int T = p.tile_rows, S = p.nstages;
+  const long long first_tile = p.row_begin / T;
+  const long long ntiles = p.row_end > p.row_begin ? (p.row_end + T - 1) / T - first_tile : 0;
+  const long long nj = ntiles > blockIdx.x ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NW);
+    }
+    fence_mbar_init();
+  }
+  // smem pre-aggregation table: identities
+  if (SK == SK_GROUP && warp < NW && p.smode != SM_NONE) {
+    if (p.smode == SM_DENSE) {
+      long long* t = (long long*)sagg;
+      for (uint32_t i = threadIdx.x; i < p.smem_cap * p.vwords; i += NW * 32) {
+        const uint32_t c = i % p.vwords;
+        t[i] = c == 0 ? 0 : agg_identity(p.agg_fn[c - 1]);
+      }
+    } else {
+      unsigned long long* keys = (unsigned long long*)sagg;
+      long long* ent = (long long*)sagg + p.smem_cap;
+      for (uint32_t i = threadIdx.x; i < p.smem_cap; i += NW * 32) keys[i] = EMPTY_KEY;
+      for (uint32_t i = threadIdx.x; i < p.smem_cap * p.vwords; i += NW * 32) {
+        const uint32_t c = i % p.vwords;
+        ent[i] = c == 0 ? 0 : agg_identity(p.agg_fn[c - 1]);
+      }
+    }
+  }
+  __syncthreads();
+
+  if (warp == NW) {
+    // ------------------------------------------------ TMA producer warp
+    if (lane == 0) {
+      const uint64_t pol = policy_evict_first();
+      for (long long j = 0; j < nj; ++j) {
+        const int s = (int)(j % S);
+        if (j >= S) mbar_wait(&empty[s], (uint32_t)(((j / S) - 1) & 1));
+        const long long t0 = (first_tile + blockIdx.x + j * gridDim.x) * (long long)T;
+        char* st = stages + (size_t)s * p.stage_stride;
+        if (t0 >= p.row_begin && t0 + T <= p.row_end) {
+          mbar_expect_tx(&full[s], p.stage_bytes);
+          for (int c = 0; c < p.ncols; ++c) {
+            const KCol col = p.cols[c];
+            tma_load_1d(st + col.soff, col.ptr + t0 * col.width, (uint32_t)T * col.width, &full[s], pol);
+          }
+        } else {
+          mbar_arrive(&full[s]);  // ragged head/tail tile: consumers load it themselves
+        }
+      }
+    }
+    return;
+  }
+
+  // ------------------------------------------------------ consumer warps
+  const int row0 = warp * 32 * R + lane;
+  long long sacc[SK == SK_SCALAR ? HQ_MAX_AGGS : 1];
+  unsigned long long scount = 0;
+  if constexpr (SK == SK_SCALAR) {
+#pragma unroll
+    for (int a = 0; a < HQ_MAX_AGGS; ++a) sacc[a] = a < p.naggs ? agg_identity(p.agg_fn[a]) : 0;
+  }
+
+  for (long long j = 0; j < nj; ++j) {
+    const int s = (int)(j % S);
+    mbar_wait(&full[s], (uint32_t)((j / S) & 1));
+    const long long t0 = (first_tile + blockIdx.x + j * gridDim.x) * (long long)T;
+    const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);
+    const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);
+    char* stage = stages + (size_t)s * p.stage_stride;
+    uint32_t mask = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const int row = row0 + r * 32;
+      if (row >= lo && row < hi) mask |= 1u << r;
+    }
+    if (lo > 0 || hi < T) {  // ragged tile: each lane copies its own rows
+      for (int c = 0; c < p.ncols; ++c) {
+        const KCol col = p.cols[c];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (mask & (1u << r)) {
+            const int row = row0 + r * 32;
+            const long long g = t0 + row;
+            char* dst = stage + col.soff;
+            if (col.width == 4) ((int*)dst)[row] = ((const int*)col.ptr)[g];
+            else if (col.width == 8) ((long long*)dst)[row] = ((const long long*)col.ptr)[g];
+            else ((signed char*)dst)[row] = ((const signed char*)col.ptr)[g];
+          }
+        }
+      }
+      fence_proxy_async();
+      __syncwarp();
+    }
+    // ---- the plan's operators, in order
+    for (int o = 0; o < p.nops; ++o) {
+      if (!__any_sync(FULLMASK, mask)) break;
+      const KOp op = p.ops[o];
+      if (op.kind == OP_FILTER) mask = op_filter<R>(p, op.idx, stage, tmp, row0, mask);
+      else if (op.kind == OP_PROBE) mask = op_probe<R>(p, op.idx, stage, tmp, row0, mask);
+      else op_compute<R>(p, op.idx, stage, tmp, row0, mask);
+    }
+    // ---- sink
+    if constexpr (SK == SK_MAT) {
+      sink_materialise<R>(p, stage, tmp, row0, mask, warp, lane, s_wtot, s_base);
+    } else if constexpr (SK == SK_SCALAR) {
+      if (p.resolution == HQ_RES_ATOMIC) {  // B2: per-row atomic reduce
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (mask & (1u << r)) {
+            long long vals[HQ_MAX_AGGS];
+#pragma unroll
+            for (int a = 0; a < HQ_MAX_AGGS; ++a)
+              if (a < p.naggs)
+                vals[a] = p.agg_fn[a] == HQ_AGG_COUNT ? 1 : load_one(p, p.agg_reg[a], stage, tmp, row0 + r * 32);
+            entry_update(p, p.gtab, 1, vals);
+          }
+        }
+      } else {  // B3: register partials, reduced once at the end
+        scount += __popc(mask);
+#pragma unroll
+        for (int a = 0; a < HQ_MAX_AGGS; ++a) {
+          if (a < p.naggs && p.agg_fn[a] != HQ_AGG_COUNT) {
+            long long v[R];
+            load_rows<R>(p, p.agg_reg[a], stage, tmp, row0, v);
+            const uint8_t fn = p.agg_fn[a];
+#pragma unroll
+            for (int r = 0; r < R; ++r)
+              if (mask & (1u << r)) sacc[SK == SK_SCALAR ? a : 0] = agg_combine(fn, sacc[SK == SK_SCALAR ? a : 0], v[r]);
+          }
+        }
+      }
+    } else {
+      sink_group<R>(p, stage, tmp, sagg, row0, mask, lane);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[s]);
+  }
+
+  // ---------------------------------------------- global propagation (end)
+  {
+    if (SK == SK_SCALAR && p.resolution != HQ_RES_ATOMIC) {
+      // B3: warp reduction -> block reduction in smem -> one atomic per aggregate
+      unsigned long long c = scount;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(FULLMASK, c, o);
+      long long red[HQ_MAX_AGGS];
+#pragma unroll
+      for (int a = 0; a < HQ_MAX_AGGS; ++a) red[a] = a < p.naggs ? warp_reduce(p.agg_fn[a], sacc[SK == SK_SCALAR ? a : 0]) : 0;
+      if (lane == 0) {
+        s_red[warp * (1 + HQ_MAX_AGGS)] = (long long)c;
+#pragma unroll
+        for (int a = 0; a < HQ_MAX_AGGS; ++a) s_red[warp * (1 + HQ_MAX_AGGS) + 1 + a] = red[a];
+      }
+      consumer_bar();
+      if (threadIdx.x == 0) {
+        unsigned long long cnt = 0;
+        long long vals[HQ_MAX_AGGS];
+#pragma unroll
+        for (int a = 0; a < HQ_MAX_AGGS; ++a) vals[a] = a < p.naggs ? agg_identity(p.agg_fn[a]) : 0;
+        for (int w = 0; w < NW; ++w) {
+          cnt += (unsigned long long)s_red[w * (1 + HQ_MAX_AGGS)];
+#pragma unroll
+          for (int a = 0; a < HQ_MAX_AGGS; ++a)
+            if (a < p.naggs) vals[a] = agg_combine(p.agg_fn[a], vals[a], s_red[w * (1 + HQ_MAX_AGGS) + 1 + a]);
+        }
+        if (cnt) entry_update(p, p.gtab, cnt, vals);
+      }
+    } else if (SK == SK_GROUP && p.smode != SM_NONE) {
+      // C3: merge the block's pre-aggregates into the global table
+      consumer_bar();
+      if (p.smode == SM_DENSE) {
+        const long long* t = (const long long*)sagg;
+        for (uint32_t g = threadIdx.x; g < p.smem_cap; g += NW * 32) {
+          const long long* e = t + (size_t)g * p.vwords;
+          if (e[0] != 0) global_update(p, g, (unsigned long long)e[0], e + 1);
+        }
+      } else {
+        const unsigned long long* keys = (const unsigned long long*)sagg;
+        const long long* ent = (const long long*)sagg + p.smem_cap;
+        for (uint32_t h = threadIdx.x; h < p.smem_cap; h += NW * 32) {
+          if (keys[h] != EMPTY_KEY) {
+            const long long* e = ent + (size_t)h * p.vwords;
+            global_update(p, keys[h], (unsigned long long)e[0], e + 1);
+          }
+        }
+      }
+    }
+  }
+}
+
+// group table initialisation (identities; hash keys EMPTY)
+__global__ void hq_init_groups_kernel(long long* tab, long long n, uint32_t vwords, int hash, uint64_t fns_lo) {
+  const uint32_t stride = vwords + (hash ? 1 : 0);
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n * stride;
+       i += (long long)gridDim.x * blockDim.x) {
+    const uint32_t c = (uint32_t)(i % stride);
+    long long v;
+    if (hash && c == 0) v = (long long)EMPTY_KEY;
+    else {
+      const uint32_t k = c - (hash ? 1 : 0);
+      v = k == 0 ? 0 : agg_identity((uint8_t)((fns_lo >> (8 * (k - 1))) & 0xff));
+    }
+    tab[i] = v;
+  }
+}
+
+int64_t fused_smem_bytes(const KPlan& kp) {
+  return (int64_t)kp.off_stage + (int64_t)kp.nstages * kp.stage_stride;
+}
+
+template <int R, int SK>
+static void launch_one(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
+  HQ_CUDA(cudaFuncSetAttribute(hq_fused_pipeline_kernel<R, SK>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  hq_fused_pipeline_kernel<R, SK><<<grid, NTHREADS, smem, ctx->stream>>>(kp);
+}
+
+void launch_fused(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
+  const int sk = kp.sink == HQ_SINK_MATERIALISE ? SK_MAT : (kp.nkeys == 0 ? SK_SCALAR : SK_GROUP);
+  if (kp.R == 4) {
+    if (sk == SK_SCALAR) launch_one<4, SK_SCALAR>(ctx, kp, grid, smem);
+    else if (sk == SK_GROUP) launch_one<4, SK_GROUP>(ctx, kp, grid, smem);
+    else launch_one<4, SK_MAT>(ctx, kp, grid, smem);
+  } else {
+    if (sk == SK_SCALAR) launch_one<2, SK_SCALAR>(ctx, kp, grid, smem);
+    else if (sk == SK_GROUP) launch_one<2, SK_GROUP>(ctx, kp, grid, smem);
+    else launch_one<2, SK_MAT>(ctx, kp, grid, smem);
+  }
+  HQ_CUDA(cudaGetLastError());
+}
+
+void launch_init_groups(hq_ctx* ctx, long long* tab, int64_t ngroups, uint32_t vwords, bool hash,
+                        const uint8_t* agg_fn, int naggs) {
+  uint64_t fns = 0;
+  for (int a = 0; a < naggs; ++a) fns |= (uint64_t)agg_fn[a] << (8 * a);
+  const long long total = ngroups * (long long)(vwords + (hash ? 1 : 0));
+  int grid = (int)std::min<long long>((total + 255) / 256, (long long)ctx->num_sms * 8);
+  if (grid < 1) grid = 1;
+  hq_init_groups_kernel<<<grid, 256, 0, ctx->stream>>>(tab, ngroups, vwords, hash ? 1 : 0, fns);
+  HQ_CUDA(cudaGetLastError());
+}
+
+}  // namespace hqk

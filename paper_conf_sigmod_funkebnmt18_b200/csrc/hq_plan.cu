@@ -1,0 +1,360 @@
+// hq_plan.cu -- validation of an hq_plan and its translation into the fused
+// kernel's device plan (KPlan): register map, TMA stage layout, shared-memory
+// budget, sink tables.  One plan = one fusion operator (§4.1).
+#include <algorithm>
+#include <climits>
+#include <cstring>
+
+#include "hq_internal.h"
+
+using namespace hqk;
+
+namespace {
+
+int64_t next_pow2(int64_t x) {
+  int64_t c = 1;
+  while (c < x) c <<= 1;
+  return c;
+}
+uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
+
+constexpr uint32_t MISC_BYTES = 2048;  // barriers, block-scan and reduction scratch
+
+struct RegInfo {
+  int width = 0;       // 0 = undefined
+  bool is_col = false;
+};
+
+// external register id -> internal index (columns 0..15, temporaries 16..23)
+int reg_index(int32_t reg, int ncols) {
+  if (reg >= 0 && reg < ncols) return reg;
+  if (reg >= HQ_TMP(0) && reg < HQ_TMP(HQ_MAX_TMP)) return HQ_MAX_COLS + (reg - HQ_TMP(0));
+  return -1;
+}
+
+void fold_pred(const hq_pred& in, KPred& out, int16_t reg) {
+  out.reg = reg;
+  out.kind = 0;
+  out.neg = 0;
+  std::memset(out.bm, 0, sizeof(out.bm));
+  switch (in.cmp) {
+    case HQ_EQ: out.lo = out.hi = in.lo; break;
+    case HQ_NE: out.lo = out.hi = in.lo; out.neg = 1; break;
+    case HQ_LT:
+      if (in.lo == LLONG_MIN) { out.lo = 1; out.hi = 0; } else { out.lo = LLONG_MIN; out.hi = in.lo - 1; }
+      break;
+    case HQ_LE: out.lo = LLONG_MIN; out.hi = in.lo; break;
+    case HQ_GT:
+      if (in.lo == LLONG_MAX) { out.lo = 1; out.hi = 0; } else { out.lo = in.lo + 1; out.hi = LLONG_MAX; }
+      break;
+    case HQ_GE: out.lo = in.lo; out.hi = LLONG_MAX; break;
+    case HQ_BETWEEN: out.lo = in.lo; out.hi = in.hi; break;
+    case HQ_IN_BITMAP: out.kind = 1; std::memcpy(out.bm, in.bitmap, sizeof(out.bm)); break;
+    default: HQ_THROW(HQ_ERR_ARG, "unknown comparison in filter");
+  }
+  // int32 fast path bounds (an empty range stays empty after clamping)
+  if (out.lo > out.hi || out.lo > INT_MAX || out.hi < INT_MIN) {
+    out.lo32 = 1;
+    out.hi32 = 0;
+  } else {
+    out.lo32 = (int32_t)std::max<int64_t>(out.lo, INT_MIN);
+    out.hi32 = (int32_t)std::min<int64_t>(out.hi, INT_MAX);
+  }
+}
+
+}  // namespace
+
+int hq_type_width(int type) {
+  switch (type) {
+    case HQ_I8: return 1;
+    case HQ_I32: return 4;
+    case HQ_I64: return 8;
+    case HQ_F64: return 8;
+  }
+  return 0;
+}
+
+// Build the device plan; allocates the result's sink buffers on first use.
+static void build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int64_t mat_cap) {
+  const hq_plan& P = r->plan;
+  const hq_table* F = r->fact;
+  std::memset(&kp, 0, sizeof(kp));
+  const int64_t rb = P.row_begin, re = P.row_end < 0 ? F->nrows : P.row_end;
+  if (rb < 0 || re < rb || re > F->nrows) HQ_THROW(HQ_ERR_ARG, "plan: row range outside the fact table");
+  kp.row_begin = rb;
+  kp.row_end = re;
+  if (P.nops < 0 || P.nops > HQ_MAX_OPS) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: too many ops");
+
+  RegInfo regs[NREGS];
+  bool col_used[HQ_MAX_COLS] = {false};
+  for (int c = 0; c < F->ncols; ++c) {
+    regs[c].width = F->cols[c].width;
+    regs[c].is_col = true;
+  }
+  auto use = [&](int32_t reg, const char* what) -> int {
+    const int i = reg_index(reg, F->ncols);
+    if (i < 0 || regs[i].width == 0)
+      HQ_THROW(HQ_ERR_ARG, std::string("plan: ") + what + " reads an undefined register " + std::to_string(reg));
+    if (i < HQ_MAX_COLS) col_used[i] = true;
+    return i;
+  };
+  auto def = [&](int32_t reg, int width, const char* what) -> int {
+    const int i = reg_index(reg, F->ncols);
+    if (i < HQ_MAX_COLS) HQ_THROW(HQ_ERR_ARG, std::string("plan: ") + what + " must write a temporary HQ_TMP(k)");
+    if (regs[i].width != 0 && regs[i].width != width)
+      HQ_THROW(HQ_ERR_ARG, std::string("plan: temporary redefined with another type by ") + what);
+    regs[i].width = width;
+    return i;
+  };
+
+  int npred = 0, nprobe = 0, ncomp = 0, ninsn = 0;
+  kp.nops = P.nops;
+  for (int o = 0; o < P.nops; ++o) {
+    const hq_op& op = P.ops[o];
+    if (op.kind == HQ_OP_FILTER) {
+      if (npred >= MAX_PREDS) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: too many filters");
+      const int i = use(op.filter.reg, "filter");
+      fold_pred(op.filter, kp.preds[npred], (int16_t)i);
+      kp.ops[o] = {OP_FILTER, (uint8_t)npred++};
+    } else if (op.kind == HQ_OP_PROBE) {
+      if (nprobe >= MAX_PROBES) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: too many probes");
+      if (!op.ht) HQ_THROW(HQ_ERR_ARG, "plan: probe without hash table");
+      if (op.mode < HQ_PROBE_INNER || op.mode > HQ_PROBE_ANTI) HQ_THROW(HQ_ERR_ARG, "plan: bad probe mode");
+      KProbe& pr = kp.probes[nprobe];
+      pr.key_reg = (int16_t)use(op.key_reg, "probe key");
+      pr.slots = op.ht->slots;
+      pr.mask = (uint32_t)(op.ht->meta.capacity - 1);
+      pr.log2cap = (uint8_t)op.ht->log2cap;
+      pr.words = (uint8_t)op.ht->meta.slot_words;
+      pr.mode = (uint8_t)op.mode;
+      const int npay = op.mode == HQ_PROBE_INNER ? op.npayload : 0;
+      if (npay < 0 || npay > op.ht->meta.npayload) HQ_THROW(HQ_ERR_ARG, "plan: probe asks for more payload words than the table holds");
+      pr.npay = (uint8_t)npay;
+      for (int k = 0; k < npay; ++k) pr.dst[k] = (int16_t)def(op.payload_dst[k], 4, "probe payload");
+      kp.ops[o] = {OP_PROBE, (uint8_t)nprobe++};
+    } else if (op.kind == HQ_OP_COMPUTE) {
+      if (ncomp >= MAX_COMPUTES) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: too many compute ops");
+      if (op.ninsn < 1 || op.ninsn > HQ_MAX_INSN || ninsn + op.ninsn > MAX_INSNS)
+        HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: expression length");
+      if (op.code[0].opc != HQ_I_LOAD) HQ_THROW(HQ_ERR_ARG, "plan: expression must start with HQ_I_LOAD");
+      KCompute& c = kp.comps[ncomp];
+      c.first = (uint8_t)ninsn;
+      c.n = (uint8_t)op.ninsn;
+      for (int k = 0; k < op.ninsn; ++k) {
+        const hq_insn& in = op.code[k];
+        if (in.opc < HQ_I_LOAD || in.opc > HQ_I_MOD) HQ_THROW(HQ_ERR_ARG, "plan: bad opcode");
+        KInsn& ki = kp.insns[ninsn++];
+        ki.opc = (uint8_t)in.opc;
+        ki.reg = in.reg < 0 ? (int16_t)-1 : (int16_t)use(in.reg, "expression");
+        ki.imm = in.imm;
+      }
+      c.dst = (int16_t)def(op.dst, 8, "compute");
+      kp.ops[o] = {OP_COMPUTE, (uint8_t)ncomp++};
+    } else {
+      HQ_THROW(HQ_ERR_ARG, "plan: unknown op kind");
+    }
+  }
+
+  // ---- sink
+  kp.sink = P.sink;
+  kp.resolution = P.resolution;
+  if (P.resolution != HQ_RES_LRGP && P.resolution != HQ_RES_ATOMIC) HQ_THROW(HQ_ERR_ARG, "plan: bad resolution");
+  uint32_t agg_smem = 0;
+  if (P.sink == HQ_SINK_AGG) {
+    if (P.nkeys < 0 || P.nkeys > HQ_MAX_KEYS) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: 0..4 group keys");
+    if (P.naggs < 0 || P.naggs > HQ_MAX_AGGS) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: 0..8 aggregates");
+    kp.nkeys = P.nkeys;
+    __int128 prod = 1;
+    for (int i = 0; i < P.nkeys; ++i) {
+      if (P.key_card[i] <= 0) HQ_THROW(HQ_ERR_ARG, "plan: key cardinality must be > 0");
+      kp.key_reg[i] = (int16_t)use(P.key_reg[i], "group key");
+      kp.key_min[i] = P.key_min[i];
+      kp.key_card[i] = P.key_card[i];
+      prod *= P.key_card[i];
+      if (prod >= ((__int128)1 << 62)) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: packed group key exceeds 62 bits");
+    }
+    int64_t st = 1;
+    for (int i = P.nkeys - 1; i >= 0; --i) {
+      kp.key_stride[i] = st;
+      st *= P.key_card[i];
+    }
+    const int64_t ngroups = (int64_t)prod;
+    kp.naggs = P.naggs;
+    for (int a = 0; a < P.naggs; ++a) {
+      if (P.agg_fn[a] < HQ_AGG_SUM || P.agg_fn[a] > HQ_AGG_AVG) HQ_THROW(HQ_ERR_ARG, "plan: bad aggregate");
+      kp.agg_fn[a] = (uint8_t)P.agg_fn[a];
+      kp.agg_reg[a] = P.agg_fn[a] == HQ_AGG_COUNT ? (int16_t)0 : (int16_t)use(P.agg_reg[a], "aggregate");
+    }
+    kp.vwords = 1 + P.naggs;
+    if (P.nkeys == 0) {
+      kp.gmode = GM_SCALAR;
+      r->ngroups = 1;
+    } else if (ngroups <= DENSE_LIMIT) {
+      kp.gmode = GM_DENSE;
+      r->ngroups = ngroups;
+    } else {
+      kp.gmode = GM_HASH;
+      int64_t cap = group_cap > 0 ? group_cap : (P.group_capacity > 0 ? P.group_capacity : std::min<int64_t>(ngroups, 1 << 20));
+      cap = std::max<int64_t>(1024, next_pow2(cap * 2));
+      r->ngroups = cap;
+      kp.gmask = (uint64_t)(cap - 1);
+      int l = 0;
+      while ((1LL << l) < cap) ++l;
+      kp.glog2 = l;
+    }
+    r->gmode = kp.gmode;
+    r->vwords = kp.vwords;
+    const size_t gbytes = (size_t)r->ngroups * (kp.vwords + (kp.gmode == GM_HASH ? 1 : 0)) * 8;
+    if (!r->gtab.p || r->gtab.bytes < gbytes) r->gtab = DevBuf(ctx, gbytes);
+    kp.gtab = r->gtab.as<long long>();
+    // local-resolution table in shared memory
+    kp.smode = SM_NONE;
+    if (P.nkeys > 0 && P.resolution == HQ_RES_LRGP) {
+      if (kp.gmode == GM_DENSE && (uint64_t)ngroups * kp.vwords * 8 <= (uint64_t)SMEM_AGG_BYTES) {
+        kp.smode = SM_DENSE;
+        kp.smem_cap = (uint32_t)ngroups;
+        agg_smem = (uint32_t)(ngroups * kp.vwords * 8);
+      } else {
+        uint32_t cap = 4096;
+        while (cap > 64 && (uint64_t)cap * (kp.vwords + 1) * 8 > (uint64_t)SMEM_AGG_BYTES) cap >>= 1;
+        kp.smode = SM_HASH;
+        kp.smem_cap = cap;
+        int l = 0;
+        while ((1u << l) < cap) ++l;
+        kp.slog2 = l;
+        agg_smem = cap * (kp.vwords + 1) * 8;
+      }
+    }
+  } else if (P.sink == HQ_SINK_MATERIALISE) {
+    if (P.nout < 1 || P.nout > HQ_MAX_OUT) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: 1..8 output columns");
+    const int64_t cap = mat_cap > 0 ? mat_cap : (P.capacity > 0 ? P.capacity : std::max<int64_t>(re - rb, 0));
+    const bool realloc = (int)r->outcols.size() != P.nout || r->capacity < cap;
+    if (realloc) r->outcols.clear();
+    kp.nout = P.nout;
+    for (int j = 0; j < P.nout; ++j) {
+      kp.out_reg[j] = (int16_t)use(P.out_reg[j], "output column");
+      const int w = hq_type_width(P.out_type[j]);
+      if (w == 0 || P.out_type[j] == HQ_F64) HQ_THROW(HQ_ERR_ARG, "plan: output type must be HQ_I8/I32/I64");
+      kp.out_width[j] = (uint8_t)w;
+      if (realloc) r->outcols.emplace_back(ctx, (size_t)std::max<int64_t>(cap, 1) * w + 16);
+      kp.out_ptr[j] = r->outcols[j].p;
+    }
+    r->capacity = std::max(r->capacity, cap);
+    kp.capacity = r->capacity;
+  } else {
+    HQ_THROW(HQ_ERR_ARG, "plan: bad sink");
+  }
+
+  // ---- stage layout: only referenced columns are streamed
+  kp.ncols = 0;
+  uint32_t rowbytes = 0;
+  for (int c = 0; c < F->ncols; ++c) {
+    if (!col_used[c]) continue;
+    if (((uintptr_t)F->cols[c].ptr & 15) != 0) HQ_THROW(HQ_ERR_ARG, "column pointer not 16-byte aligned");
+    rowbytes += (uint32_t)F->cols[c].width;
+  }
+  uint32_t tmp_row = 0;
+  for (int k = 0; k < HQ_MAX_TMP; ++k) tmp_row += (uint32_t)regs[HQ_MAX_COLS + k].width;
+
+  int chosen_R = 0;
+  for (int R : {4, 2}) {
+    const uint32_t T = (uint32_t)(NW * 32 * R);
+    const uint32_t off_tmp = MISC_BYTES;
+    const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
+    const uint32_t off_stage = align_up(off_agg + agg_smem, 128);
+    const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
+    if (off_stage >= ctx->max_smem) continue;
+    const int S = (int)std::min<int64_t>(MAX_STAGES, (ctx->max_smem - off_stage) / stride);
+    if (S >= 3 || (R == 2 && S >= 2)) {
+      chosen_R = R;
+      kp.R = R;
+      kp.tile_rows = (int32_t)T;
+      kp.nstages = S;
+      kp.stage_bytes = T * rowbytes;
+      kp.stage_stride = stride;
+      kp.off_tmp = off_tmp;
+      kp.off_agg = off_agg;
+      kp.off_stage = off_stage;
+      break;
+    }
+  }
+  if (!chosen_R) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: rows too wide for the shared-memory stage ring");
+  const uint32_t T = (uint32_t)kp.tile_rows;
+  uint32_t soff = 0;
+  for (int c = 0; c < F->ncols; ++c) {
+    if (!col_used[c]) continue;
+    KCol& kc = kp.cols[kp.ncols++];
+    kc.ptr = (const char*)F->cols[c].ptr;
+    kc.width = (uint32_t)F->cols[c].width;
+    kc.soff = soff;
+    kp.regs[c] = {soff, (uint8_t)kc.width, 1, {0, 0}};
+    soff += T * kc.width;
+  }
+  uint32_t toff = 0;
+  for (int k = 0; k < HQ_MAX_TMP; ++k) {
+    const int w = regs[HQ_MAX_COLS + k].width;
+    if (!w) continue;
+    kp.regs[HQ_MAX_COLS + k] = {toff, (uint8_t)w, 0, {0, 0}};
+    toff += T * (uint32_t)w;
+  }
+  kp.counter = (unsigned long long*)r->dstate.p;
+  kp.err = (int*)(r->dstate.as<char>() + 8);
+}
+
+static void launch_pipeline(hq_ctx* ctx, hq_result* r, int64_t group_cap, int64_t mat_cap) {
+  KPlan kp;
+  build_kplan(ctx, r, kp, group_cap, mat_cap);
+  HQ_CUDA(cudaMemsetAsync(r->dstate.p, 0, r->dstate.bytes, ctx->stream));
+  if (r->plan.sink == HQ_SINK_AGG)
+    launch_init_groups(ctx, kp.gtab, r->ngroups, kp.vwords, kp.gmode == GM_HASH, kp.agg_fn, kp.naggs);
+  const long long T = kp.tile_rows;
+  const long long ntiles = kp.row_end > kp.row_begin ? (kp.row_end + T - 1) / T - kp.row_begin / T : 0;
+  const int grid = (int)std::max<long long>(1, std::min<long long>(ntiles, ctx->num_sms));
+  const size_t smem = (size_t)fused_smem_bytes(kp);
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  if (ctx->timing) {
+    for (cudaEvent_t* e : {&e0, &e1}) {
+      if (!ctx->event_pool.empty()) { *e = ctx->event_pool.back(); ctx->event_pool.pop_back(); }
+      else HQ_CUDA(cudaEventCreate(e));
+    }
+    HQ_CUDA(cudaEventRecord(e0, ctx->stream));
+  }
+  launch_fused(ctx, kp, grid, smem);
+  if (ctx->timing) {
+    HQ_CUDA(cudaEventRecord(e1, ctx->stream));
+    ctx->events.emplace_back(e0, e1);
+  }
+}
+
+void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r) {
+  r->ctx = ctx;
+  r->plan = *plan;
+  r->sink = plan->sink;
+  r->dstate = DevBuf(ctx, 32);
+  if (plan->exec == HQ_EXEC_OAAT) {
+    hq_run_oaat(ctx, plan, r);
+    return;
+  }
+  if (plan->exec != HQ_EXEC_FUSED) HQ_THROW(HQ_ERR_ARG, "plan: bad exec mode");
+  launch_pipeline(ctx, r, 0, 0);
+}
+
+// Sync, read the device fault bits; re-run once with the exact size when an
+// output capacity or group table overflowed (SURVEY.md §5 failure handling).
+void hq_check_result_faults(hq_ctx* ctx, hq_result* r) {
+  if (r->checked) return;
+  for (int attempt = 0;; ++attempt) {
+    struct { unsigned long long counter; int err; int pad; } st{};
+    HQ_CUDA(cudaMemcpyAsync(&st, r->dstate.p, sizeof(st), cudaMemcpyDeviceToHost, ctx->stream));
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    const int err = st.err;
+    if (err & HQF_DIV_ZERO) HQ_THROW(HQ_ERR_ARG, "pipeline: division by zero");
+    if (err & HQF_KEY_DOMAIN) HQ_THROW(HQ_ERR_ARG, "pipeline: group key outside its declared [min, min+card)");
+    const bool fixable = (err & (HQF_CAPACITY | HQF_GROUP_FULL)) != 0;
+    if (!fixable) break;
+    if (attempt >= 3 || r->plan.exec == HQ_EXEC_OAAT) HQ_THROW(HQ_ERR_OVERFLOW, "pipeline: capacity exceeded");
+    if (err & HQF_CAPACITY) launch_pipeline(ctx, r, 0, (int64_t)st.counter);
+    else launch_pipeline(ctx, r, r->ngroups * 4, 0);
+  }
+  r->checked = true;
+}

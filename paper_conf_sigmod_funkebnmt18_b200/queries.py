@@ -1,0 +1,253 @@
+"""Plan builders for the benchmark queries.
+
+Each query is written as its fusion operators: hash builds (pipeline breakers,
+filtered dimension scans) followed by ONE probe pipeline over the fact table
+(the compound kernel), exactly as PAPER.md §4.1/§7 describes a plan with
+explicit fusion operators.  Constants are the SQL
+constants folded to the storage encoding (readings R2, R4, R5):
+decimals in hundredths, dates as yyyymmdd, strings as order-preserving
+dictionary codes from ``hqgen``.
+
+Predicate/probe order inside a pipeline is result-invariant (R14):
+cheap and selective first.
+"""
+from __future__ import annotations
+
+from typing import Callable, Dict, List, Optional
+
+import hqgen
+
+from . import hq
+from .engine import Engine, PlanBuilder, QueryResult, fetch
+
+ASIA = hqgen.code(hqgen.REGIONS, "ASIA")
+AMERICA = hqgen.code(hqgen.REGIONS, "AMERICA")
+BUILDING = hqgen.code(hqgen.MKTSEGMENTS, "BUILDING")
+MFGR1 = hqgen.code(hqgen.MFGRS, "MFGR#1")
+MFGR2 = hqgen.code(hqgen.MFGRS, "MFGR#2")
+
+
+class Query:
+    """A query: fact table, referenced columns per table, and run(E) which
+    builds the hash tables and returns (final Result, final PlanBuilder)."""
+
+    def __init__(self, name: str, bench: str, fact: str, columns: Dict[str, List[str]], run: Callable):
+        self.name, self.bench, self.fact, self.columns, self._run = name, bench, fact, columns, run
+
+    def run(self, E: Engine, **kw):
+        return self._run(E, **kw)
+
+    def execute(self, E: Engine, **kw) -> QueryResult:
+        res, pb = self._run(E, **kw)
+        return fetch(res, pb.result_names)
+
+    def fact_bytes_per_row(self) -> int:
+        """Algorithmic bytes per fact row: widths of the referenced fact columns."""
+        schema = dict(hqgen.SCHEMAS[hqgen.TABLE_NAMES[self.fact]])
+        return sum(int(schema[c][1]) for c in self.columns[self.fact])
+
+
+# ---------------------------------------------------------------- TPC-H Q6
+def _tpch_q6(E: Engine, **_):
+    pb = E.plan("lineitem")
+    pb.filter("l_shipdate", "between", 19940101, 19950101 - 1)  # >= 1994-01-01 and < 1995-01-01
+    pb.filter("l_discount", "between", 5, 7)                     # 0.06 +- 0.01 in hundredths
+    pb.filter("l_quantity", "<", 2400)                           # < 24 in hundredths
+    pb.compute("rev", [("load", "l_extendedprice"), ("mul", "l_discount")])  # scale 4
+    pb.aggregate(aggs=[("sum", "rev"), ("count", None)], agg_names=["revenue", "count"])
+    return E.run(pb), pb
+
+
+# ---------------------------------------------------------------- TPC-H Q1
+def _tpch_q1(E: Engine, **_):
+    pb = E.plan("lineitem")
+    pb.filter("l_shipdate", "<=", 19980902)  # 1998-12-01 - 90 days
+    pb.compute("disc_price", [("load", "l_discount"), ("rsub", 100), ("mul", "l_extendedprice")])  # scale 4
+    pb.compute("charge", [("load", "l_tax"), ("add", 100), ("mul", "disc_price")])                 # scale 6
+    pb.aggregate(keys=[("l_returnflag", 0, 3), ("l_linestatus", 0, 2)],
+                 aggs=[("sum", "l_quantity"), ("sum", "l_extendedprice"), ("sum", "disc_price"),
+                       ("sum", "charge"), ("avg", "l_quantity", 2), ("avg", "l_extendedprice", 2),
+                       ("avg", "l_discount", 2), ("count", None)],
+                 agg_names=["sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "avg_qty",
+                            "avg_price", "avg_disc", "count_order"])
+    return E.run(pb), pb
+
+
+# ---------------------------------------------------------------- SSB Q1.x
+_Q1X = {
+    1: ([("d_year", "=", 1993)], ("lo_quantity", "<", 25, 0), (1, 3)),
+    2: ([("d_yearmonthnum", "=", 199401)], ("lo_quantity", "between", 26, 35), (4, 6)),
+    3: ([("d_weeknuminyear", "=", 6), ("d_year", "=", 1994)], ("lo_quantity", "between", 26, 35), (5, 7)),
+}
+
+
+def _ssb_q1(v: int):
+    def run(E: Engine, **_):
+        dpreds, qf, (dlo, dhi) = _Q1X[v]
+        hd = E.hash("date", "d_datekey", preds=dpreds)  # semi-join table of qualifying dates
+        pb = E.plan("lineorder")
+        pb.filter(qf[0], qf[1], qf[2], qf[3])
+        pb.filter("lo_discount", "between", dlo, dhi)
+        pb.probe(hd, "lo_orderdate", "semi")
+        pb.compute("rev", [("load", "lo_extendedprice"), ("mul", "lo_discount")])
+        pb.aggregate(aggs=[("sum", "rev"), ("count", None)], agg_names=["revenue", "count"])
+        return E.run(pb), pb
+    return run
+
+
+# ---------------------------------------------------------------- SSB Q3.1
+def _ssb_q31_probes(E: Engine) -> PlanBuilder:
+    hc = E.hash("customer", "c_custkey", payload=["c_nation"], preds=[("c_region", "=", ASIA)])
+    hs = E.hash("supplier", "s_suppkey", payload=["s_nation"], preds=[("s_region", "=", ASIA)])
+    hd = E.hash("date", "d_datekey", payload=["d_year"], preds=[("d_year", "between", 1992, 1997)])
+    pb = E.plan("lineorder")
+    pb.probe(hs, "lo_suppkey", "inner", ["s_nation"])
+    pb.probe(hc, "lo_custkey", "inner", ["c_nation"])
+    pb.probe(hd, "lo_orderdate", "inner", ["d_year"])
+    return pb
+
+
+def _ssb_q31(E: Engine, **_):
+    pb = _ssb_q31_probes(E)
+    pb.aggregate(keys=[("c_nation", 0, 25), ("s_nation", 0, 25), ("d_year", 1992, 7)],
+                 aggs=[("sum", "lo_revenue"), ("count", None)],
+                 order=[("d_year", False), ("revenue", True)], agg_names=["revenue", "count"])
+    return E.run(pb), pb
+
+
+def _ssb_q31_mat(E: Engine, capacity: int = 0, **_):
+    pb = _ssb_q31_probes(E)
+    pb.materialise([("c_nation", "i32"), ("s_nation", "i32"), ("d_year", "i32"), ("lo_revenue", "i32")],
+                   capacity=capacity)
+    return E.run(pb), pb
+
+
+# ---------------------------------------------------------------- SSB Q4.1
+def _ssb_q41(E: Engine, **_):
+    hs = E.hash("supplier", "s_suppkey", preds=[("s_region", "=", AMERICA)])
+    hc = E.hash("customer", "c_custkey", payload=["c_nation"], preds=[("c_region", "=", AMERICA)])
+    hp = E.hash("part", "p_partkey", preds=[("p_mfgr", "in", [MFGR1, MFGR2])])
+    hd = E.hash("date", "d_datekey", payload=["d_year"])
+    pb = E.plan("lineorder")
+    pb.probe(hs, "lo_suppkey", "semi")
+    pb.probe(hc, "lo_custkey", "inner", ["c_nation"])
+    pb.probe(hp, "lo_partkey", "semi")
+    pb.probe(hd, "lo_orderdate", "inner", ["d_year"])
+    pb.compute("profit", [("load", "lo_revenue"), ("sub", "lo_supplycost")])
+    pb.aggregate(keys=[("d_year", 1992, 7), ("c_nation", 0, 25)],
+                 aggs=[("sum", "profit"), ("count", None)], agg_names=["profit", "count"])
+    return E.run(pb), pb
+
+
+# ---------------------------------------------------------------- TPC-H Q3
+def _tpch_q3(E: Engine, limit: int = 10, **_):
+    # pipeline 1: customer filter -> build (semi)
+    hc = E.hash("tpch_customer", "c_custkey", preds=[("c_mktsegment", "=", BUILDING)])
+    # pipeline 2: orders filter -> probe customer -> materialise -> build
+    po = E.plan("orders")
+    po.filter("o_orderdate", "<", 19950315)
+    po.probe(hc, "o_custkey", "semi")
+    po.materialise([("o_orderkey", "i32"), ("o_orderdate", "i32"), ("o_shippriority", "i32")])
+    ro = E.run(po, partitioned=False)
+    ho = E.hash_from(ro, ["o_orderkey", "o_orderdate", "o_shippriority"], "o_orderkey",
+                     ["o_orderdate", "o_shippriority"])
+    nk = max(int(ho.info().nkeys), 0)
+    # pipeline 3: lineitem filter -> probe orders -> group by orderkey
+    pl = E.plan("lineitem")
+    pl.filter("l_shipdate", ">", 19950315)
+    pl.probe(ho, "l_orderkey", "inner", ["o_orderdate", "o_shippriority"])
+    pl.compute("rev", [("load", "l_discount"), ("rsub", 100), ("mul", "l_extendedprice")])  # scale 4
+    pl.aggregate(keys=[("l_orderkey", 0, 1 << 31), ("o_orderdate", 19920101, 70000), ("o_shippriority", 0, 8)],
+                 aggs=[("sum", "rev"), ("count", None)],
+                 order=[("revenue", True), ("o_orderdate", False)], limit=limit,
+                 group_capacity=max(1024, nk // 8), agg_names=["revenue", "count"])
+    res = E.run(pl)
+    pl.keep += [ro, ho]
+    return res, pl
+
+
+# ------------------------------------------------ paper micro queries (f2)
+def _micro_select(E: Engine, x: int = 5, resolution=None, **_):
+    """PAPER.md Fig 16 'Query 1': selection + projection, materialised."""
+    pb = E.plan("lineorder")
+    pb.filter("lo_quantity", "between", 25 - x, 25 + x)
+    pb.compute("revenue", [("load", "lo_extendedprice"), ("mul", "lo_discount"), ("add", "lo_tax")])
+    pb.materialise([("revenue", "i64")])
+    return E.run(pb), pb
+
+
+def _micro_sum(E: Engine, x: int = 5, **_):
+    """App G.1: single-tuple aggregation of Query 1."""
+    pb = E.plan("lineorder")
+    pb.filter("lo_quantity", "between", 25 - x, 25 + x)
+    pb.compute("revenue", [("load", "lo_extendedprice"), ("mul", "lo_discount"), ("add", "lo_tax")])
+    pb.aggregate(aggs=[("sum", "revenue"), ("count", None)], agg_names=["revenue", "count"])
+    return E.run(pb), pb
+
+
+def _micro_groupby(E: Engine, x: int = 16, **_):
+    """Fig 26: sum(lo_extendedprice) group by lo_orderkey % x."""
+    pb = E.plan("lineorder")
+    pb.compute("k", [("load", "lo_orderkey"), ("mod", x)])
+    pb.aggregate(keys=[("k", 0, x)], aggs=[("sum", "lo_extendedprice"), ("count", None)],
+                 agg_names=["sum", "count"])
+    return E.run(pb), pb
+
+
+QUERIES: Dict[str, Query] = {q.name: q for q in [
+    Query("tpch_q6", "tpch", "lineitem",
+          {"lineitem": ["l_shipdate", "l_discount", "l_quantity", "l_extendedprice"]}, _tpch_q6),
+    Query("tpch_q1", "tpch", "lineitem",
+          {"lineitem": ["l_shipdate", "l_returnflag", "l_linestatus", "l_quantity", "l_extendedprice",
+                        "l_discount", "l_tax"]}, _tpch_q1),
+    Query("ssb_q11", "ssb", "lineorder",
+          {"lineorder": ["lo_orderdate", "lo_quantity", "lo_discount", "lo_extendedprice"],
+           "date": ["d_datekey", "d_year", "d_yearmonthnum", "d_weeknuminyear"]}, _ssb_q1(1)),
+    Query("ssb_q12", "ssb", "lineorder",
+          {"lineorder": ["lo_orderdate", "lo_quantity", "lo_discount", "lo_extendedprice"],
+           "date": ["d_datekey", "d_year", "d_yearmonthnum", "d_weeknuminyear"]}, _ssb_q1(2)),
+    Query("ssb_q13", "ssb", "lineorder",
+          {"lineorder": ["lo_orderdate", "lo_quantity", "lo_discount", "lo_extendedprice"],
+           "date": ["d_datekey", "d_year", "d_yearmonthnum", "d_weeknuminyear"]}, _ssb_q1(3)),
+    Query("ssb_q31", "ssb", "lineorder",
+          {"lineorder": ["lo_custkey", "lo_suppkey", "lo_orderdate", "lo_revenue"],
+           "customer": ["c_custkey", "c_nation", "c_region"], "supplier": ["s_suppkey", "s_nation", "s_region"],
+           "date": ["d_datekey", "d_year"]}, _ssb_q31),
+    Query("ssb_q31_mat", "ssb", "lineorder",
+          {"lineorder": ["lo_custkey", "lo_suppkey", "lo_orderdate", "lo_revenue"],
+           "customer": ["c_custkey", "c_nation", "c_region"], "supplier": ["s_suppkey", "s_nation", "s_region"],
+           "date": ["d_datekey", "d_year"]}, _ssb_q31_mat),
+    Query("ssb_q41", "ssb", "lineorder",
+          {"lineorder": ["lo_custkey", "lo_suppkey", "lo_partkey", "lo_orderdate", "lo_revenue", "lo_supplycost"],
+           "customer": ["c_custkey", "c_nation", "c_region"], "supplier": ["s_suppkey", "s_region"],
+           "part": ["p_partkey", "p_mfgr"], "date": ["d_datekey", "d_year"]}, _ssb_q41),
+    Query("tpch_q3", "tpch", "lineitem",
+          {"lineitem": ["l_orderkey", "l_shipdate", "l_extendedprice", "l_discount"],
+           "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority"],
+           "tpch_customer": ["c_custkey", "c_mktsegment"]}, _tpch_q3),
+    Query("micro_select", "ssb", "lineorder",
+          {"lineorder": ["lo_quantity", "lo_extendedprice", "lo_discount", "lo_tax"]}, _micro_select),
+    Query("micro_sum", "ssb", "lineorder",
+          {"lineorder": ["lo_quantity", "lo_extendedprice", "lo_discount", "lo_tax"]}, _micro_sum),
+    Query("micro_groupby", "ssb", "lineorder",
+          {"lineorder": ["lo_orderkey", "lo_extendedprice"]}, _micro_groupby),
+]}
+
+
+def load_tables(ctx: hq.Context, query: Query, sf: float, seed: int = hqgen.DEFAULT_SEED,
+                fact_range: Optional[tuple] = None, host: Optional[Dict[str, Dict]] = None,
+                skip_dims: bool = False) -> Dict[str, hq.Table]:
+    """Generate (or take from ``host``) the referenced columns and load them onto
+    the context's device.  fact_range: rows of the fact table to load (a range
+    partition).  skip_dims: load only the fact table (non-root ranks)."""
+    tables = {}
+    for t, cols in query.columns.items():
+        if skip_dims and t != query.fact:
+            continue
+        if host is not None and t in host:
+            data = {c: host[t][c] for c in cols}
+        else:
+            rr = fact_range if t == query.fact else None
+            data = hqgen.generate(t, sf, seed, columns=cols, row_range=rr)
+        tables[t] = ctx.load_columns(data)
+    return tables

@@ -1,0 +1,275 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by
+element, on the same seeded inputs.  Integer results bit-exact; AVG (fp64)
+within 1e-9 relative (north_star).  Materialised results compared as sorted
+multisets (several orders are correct)."""
+import numpy as np
+import pytest
+
+import hqgen
+import oracle
+from paper_conf_sigmod_funkebnmt18_b200 import hq
+from paper_conf_sigmod_funkebnmt18_b200.engine import Engine
+from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
+
+pytestmark = pytest.mark.gpu
+
+SF = 0.01
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    import torch
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    c = hq.Context(0)
+    yield c
+    c.close()
+
+
+@pytest.fixture(scope="module")
+def ssb():
+    return {t: hqgen.generate(t, SF) for t in hqgen.SSB_TABLES}
+
+
+@pytest.fixture(scope="module")
+def tpch():
+    return {t: hqgen.generate(t, SF) for t in hqgen.TPCH_TABLES}
+
+
+def gpu_run(ctx, qname, host, fact_range=None, exec_mode=hq.EXEC_FUSED, resolution=hq.RES_LRGP, **kw):
+    q = QUERIES[qname]
+    tables = {t: ctx.load_columns({c: host[t][c] for c in cols}) for t, cols in q.columns.items()}
+    E = Engine(ctx, tables, exec_mode=exec_mode, resolution=resolution, fact_range=fact_range)
+    return q.execute(E, **kw)
+
+
+def oracle_run(qname, t, **kw):
+    if qname == "tpch_q6":
+        return oracle.tpch_q6(t["lineitem"])
+    if qname == "tpch_q1":
+        return oracle.tpch_q1(t["lineitem"])
+    if qname in ("ssb_q11", "ssb_q12", "ssb_q13"):
+        return oracle.ssb_q1(int(qname[-1]), t["lineorder"], t["date"])
+    if qname == "ssb_q31":
+        return oracle.ssb_q31(t["lineorder"], t["customer"], t["supplier"], t["date"])
+    if qname == "ssb_q31_mat":
+        return oracle.ssb_q31_mat(t["lineorder"], t["customer"], t["supplier"], t["date"])
+    if qname == "ssb_q41":
+        return oracle.ssb_q41(t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"])
+    if qname == "tpch_q3":
+        return oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    raise KeyError(qname)
+
+
+INT_COLS = {
+    "tpch_q6": ["revenue", "count"],
+    "tpch_q1": ["l_returnflag", "l_linestatus", "sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "count_order"],
+    "ssb_q11": ["revenue", "count"], "ssb_q12": ["revenue", "count"], "ssb_q13": ["revenue", "count"],
+    "ssb_q31": ["c_nation", "s_nation", "d_year", "revenue", "count"],
+    "ssb_q41": ["d_year", "c_nation", "profit", "count"],
+    "tpch_q3": ["l_orderkey", "o_orderdate", "o_shippriority", "revenue", "count"],
+}
+
+
+def assert_same(qname, g, o):
+    cols = INT_COLS[qname]
+    assert g.nrows == o.nrows, (g.nrows, o.nrows)
+    for c in cols:
+        np.testing.assert_array_equal(np.asarray(g.columns[c], np.int64), np.asarray(o.columns[c], np.int64), err_msg=c)
+    for c in ("avg_qty", "avg_price", "avg_disc"):
+        if c in o.columns:
+            np.testing.assert_allclose(g.columns[c], o.columns[c], rtol=1e-9, atol=0)
+
+
+def host_for(qname, ssb, tpch):
+    return ssb if QUERIES[qname].bench == "ssb" else tpch
+
+
+@pytest.mark.parametrize("qname", ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q12", "ssb_q13", "ssb_q31", "ssb_q41"])
+def test_query_parity(ctx, ssb, tpch, qname):
+    host = host_for(qname, ssb, tpch)
+    g = gpu_run(ctx, qname, host)
+    o = oracle_run(qname, host)
+    assert_same(qname, g, o)
+    assert g.qualifying == o.qualifying
+
+
+def test_tpch_q3_parity(ctx, tpch):
+    o = oracle_run("tpch_q3", tpch)
+    full = gpu_run(ctx, "tpch_q3", tpch, limit=0)  # full pre-LIMIT set under the total order
+    assert_same("tpch_q3", full, o)
+    top = gpu_run(ctx, "tpch_q3", tpch, limit=10)
+    assert top.nrows == 10
+    for c in INT_COLS["tpch_q3"]:
+        np.testing.assert_array_equal(top.columns[c], o.columns[c][:10])
+
+
+def test_ssb_q31_materialise_parity(ctx, ssb):
+    g = gpu_run(ctx, "ssb_q31_mat", ssb)
+    o = oracle_run("ssb_q31_mat", ssb)
+    assert g.qualifying == o.nrows
+    assert sorted(g.rows(["c_nation", "s_nation", "d_year", "lo_revenue"])) == o.rows()
+    # invariant: sum of the materialised column == the aggregate sink's SUM
+    a = gpu_run(ctx, "ssb_q31", ssb)
+    assert int(g.columns["lo_revenue"].astype(np.int64).sum()) == int(a.columns["revenue"].sum())
+
+
+@pytest.mark.parametrize("qname", ["ssb_q41", "tpch_q1", "ssb_q11"])
+def test_resolution_ablation_identical(ctx, ssb, tpch, qname):
+    host = host_for(qname, ssb, tpch)
+    a = gpu_run(ctx, qname, host, resolution=hq.RES_LRGP)
+    b = gpu_run(ctx, qname, host, resolution=hq.RES_ATOMIC)
+    assert a.rows() == b.rows()
+
+
+@pytest.mark.parametrize("qname", ["ssb_q41", "tpch_q6", "tpch_q1"])
+def test_logical_partitions_sum_to_whole(ctx, ssb, tpch, qname):
+    """Range partitions (unaligned cut points) merged exactly == one run == oracle
+    (SURVEY.md §4.2 layer 5(i))."""
+    host = host_for(qname, ssb, tpch)
+    fact = QUERIES[qname].fact
+    n = len(next(iter(host[fact].values())))
+    cuts = [0, 777, n // 3, n // 3 + 1, n - 5, n]
+    whole = gpu_run(ctx, qname, host)
+    key_cols = {"ssb_q41": ["d_year", "c_nation"], "tpch_q6": [], "tpch_q1": ["l_returnflag", "l_linestatus"]}[qname]
+    sum_cols = {"ssb_q41": ["profit", "count"], "tpch_q6": ["revenue", "count"],
+                "tpch_q1": ["sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "count_order"]}[qname]
+    acc = {}
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        part = gpu_run(ctx, qname, host, fact_range=(a, b))
+        for row in part.rows(key_cols + sum_cols):
+            k = row[:len(key_cols)]
+            v = row[len(key_cols):]
+            acc[k] = tuple(x + y for x, y in zip(acc.get(k, (0,) * len(v)), v))
+    got = {k: v for k, v in acc.items() if v[-1] > 0}
+    exp = {r[:len(key_cols)]: r[len(key_cols):] for r in whole.rows(key_cols + sum_cols) if r[-1] > 0}
+    assert got == exp
+
+
+def test_golden_fixtures_on_gpu(ctx, golden):
+    """Hand-computed fixtures F1, F2, F4-F7 through the CUDA path (single ragged tile)."""
+    fx = golden("F1_ssb_q11_boundaries.json")
+    t = fx["tables"]
+    lo = dict(t["lineorder"])
+    g = gpu_run(ctx, "ssb_q11", {"lineorder": lo, "date": t["date"]})
+    assert g.rows(["revenue", "count"]) == [(3400, 3)]
+    fx = golden("F4_tpch_q6_fixedpoint.json")
+    g = gpu_run(ctx, "tpch_q6", fx["tables"])
+    assert g.rows(["revenue", "count"]) == [(514000, 2)]
+    fx = golden("F5_tpch_q1.json")
+    g = gpu_run(ctx, "tpch_q1", fx["tables"])
+    assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"]
+    np.testing.assert_allclose(np.stack([g.columns[c] for c in ("avg_qty", "avg_price", "avg_disc")], 1),
+                               fx["expected"]["avg"], rtol=1e-12)
+    fx = golden("F2_ssb_q31.json")
+    t = fx["tables"]
+    g = gpu_run(ctx, "ssb_q31", t)
+    assert [list(r) for r in g.rows(fx["expected"]["group_columns"])] == fx["expected"]["groups"]
+    m = gpu_run(ctx, "ssb_q31_mat", t)
+    assert sorted(map(list, m.rows())) == fx["expected"]["materialised"]
+    fx = golden("F6_ssb_q41.json")
+    g = gpu_run(ctx, "ssb_q41", fx["tables"])
+    assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"]
+    fx = golden("F7_tpch_q3.json")
+    g = gpu_run(ctx, "tpch_q3", fx["tables"])
+    assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"]
+
+
+def test_lrgp_positions_segment_ordered(ctx):
+    """F3 / PAPER.md P:1069-1072: materialised positions are dense,
+    rows are increasing inside each block segment, segments are permuted."""
+    n = 300_000
+    rng = np.random.default_rng(3)
+    rowid = np.arange(n, dtype=np.int32)
+    flag = (rng.random(n) < 0.3).astype(np.int32)
+    t = ctx.load_columns({"rowid": rowid, "flag": flag})
+    from paper_conf_sigmod_funkebnmt18_b200.engine import PlanBuilder
+    pb = PlanBuilder(t)
+    pb.filter("flag", "=", 1).materialise([("rowid", "i32")])
+    res = ctx.run(pb.plan, keep=pb.keep)
+    out = res.fetch()[0]
+    sel = rowid[flag == 1]
+    assert res.qualifying() == len(sel) == len(out)
+    assert np.array_equal(np.sort(out), sel)  # dense: every slot written exactly once
+    # each tile's selected rows occupy one contiguous segment, in row order
+    T = 2048
+    pos = np.empty(n, np.int64)
+    pos[out] = np.arange(len(out))
+    tile = sel // T
+    starts = np.r_[0, np.nonzero(np.diff(tile))[0] + 1]
+    ends = np.r_[starts[1:], len(sel)]
+    for s, e in zip(starts, ends):
+        p = pos[sel[s:e]]
+        assert p[-1] - p[0] == e - s - 1 and np.all(np.diff(p) == 1)
+
+
+def test_edge_cases(ctx):
+    from paper_conf_sigmod_funkebnmt18_b200.engine import PlanBuilder
+    # empty table, all-filtered, empty range
+    for n in (0, 1, 33, 2048, 2049):
+        a = np.arange(n, dtype=np.int32)
+        t = ctx.load_columns({"a": a, "b": (a * 7).astype(np.int64)})
+        pb = PlanBuilder(t)
+        pb.filter("a", ">=", 0).aggregate(aggs=[("sum", "b"), ("count", None), ("min", "b"), ("max", "b")],
+                                          agg_names=["s", "c", "mn", "mx"])
+        res = ctx.run(pb.plan, keep=pb.keep)
+        s, c, mn, mx = [x[0] for x in res.fetch()]
+        assert (s, c) == (int((a * 7).sum()), n)
+        if n:
+            assert (mn, mx) == (0, 7 * (n - 1))
+        pb = PlanBuilder(t)
+        pb.filter("a", "<", 0).materialise([("b", "i64")])
+        res = ctx.run(pb.plan, keep=pb.keep)
+        assert res.qualifying() == 0 and len(res.fetch()[0]) == 0
+
+
+def test_duplicate_build_key(ctx):
+    d = {"k": np.array([1, 2, 2, 3], np.int32), "v": np.array([1, 2, 3, 4], np.int32)}
+    t = ctx.load_columns(d)
+    h = ctx.build_hash(t, 0, [1])
+    with pytest.raises(hq.HQError) as e:
+        h.info()
+    assert e.value.code == hq.HQ_ERR_DUP_KEY
+
+
+def test_group_key_domain_fault(ctx):
+    from paper_conf_sigmod_funkebnmt18_b200.engine import PlanBuilder
+    t = ctx.load_columns({"g": np.array([0, 1, 5], np.int32)})
+    pb = PlanBuilder(t)
+    pb.aggregate(keys=[("g", 0, 3)], aggs=[("count", None)], agg_names=["c"])
+    res = ctx.run(pb.plan, keep=pb.keep)
+    with pytest.raises(hq.HQError) as e:
+        res.fetch()
+    assert e.value.code == hq.HQ_ERR_ARG
+
+
+def test_materialise_capacity_rerun(ctx, ssb):
+    """An undersized capacity triggers one exact re-run."""
+    g = gpu_run(ctx, "ssb_q31_mat", ssb, capacity=7)
+    o = oracle_run("ssb_q31_mat", ssb)
+    assert sorted(g.rows(["c_nation", "s_nation", "d_year", "lo_revenue"])) == o.rows()
+
+
+def test_micro_queries(ctx, ssb):
+    lo = ssb["lineorder"]
+    for x in (0, 5, 25):
+        g = gpu_run(ctx, "micro_select", ssb, x=x)
+        o = oracle.micro_select(lo, x)
+        np.testing.assert_array_equal(np.sort(g.columns["revenue"]), o.columns["revenue"])
+        s = gpu_run(ctx, "micro_sum", ssb, x=x)
+        os_ = oracle.micro_sum(lo, x)
+        assert s.rows(["revenue", "count"]) == os_.rows(["revenue", "count"])
+    for x in (2, 7, 1000, 16384):
+        g = gpu_run(ctx, "micro_groupby", ssb, x=x)
+        o = oracle.micro_groupby(lo, x)
+        assert g.rows(["k", "sum", "count"]) == o.rows(["key", "sum", "count"])
+
+
+def test_sf1_parity_multi_tile(ctx):
+    """Larger inputs: many tiles per CTA, every stage of the TMA ring reused."""
+    host = {t: hqgen.generate(t, 1.0) for t in hqgen.SSB_TABLES}
+    for qname in ("ssb_q41", "ssb_q31", "ssb_q11"):
+        g = gpu_run(ctx, qname, host)
+        o = {"ssb_q41": lambda: oracle.ssb_q41(host["lineorder"], host["date"], host["customer"], host["supplier"], host["part"], nthreads=8),
+             "ssb_q31": lambda: oracle.ssb_q31(host["lineorder"], host["customer"], host["supplier"], host["date"], nthreads=8),
+             "ssb_q11": lambda: oracle.ssb_q1(1, host["lineorder"], host["date"], nthreads=8)}[qname]()
+        assert_same(qname, g, o)
