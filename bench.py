@@ -1,0 +1,390 @@
+#!/usr/bin/env python
+"""bench.py -- fact rows/s of the fused query pipeline on B200 (driver contract).
+
+Default workload: SSB Q4.1 at SF 100 (600 M lineorder rows, 24 B/row = 14.4 GB of
+referenced fact columns), the BASELINE.json config quoted "partitioned across
+1/2/4/8 B200" (configs[4]).  One *step* = one full query: the four dimension
+hash builds (root builds + NCCL broadcast when N>1), the fused probe/aggregate
+pipeline over the (local) fact range, the partial-aggregate reduce (N>1) and
+finalisation + result fetch on rank 0.  Columns are HBM-resident when the timed
+region starts (14.4 GB >> 126 MB L2, so no flush is needed between steps).
+
+Also reported: the dominant kernel's roofline (algorithmic bytes / measured
+kernel time vs MEASURED_PEAKS.json's HBM copy bandwidth), e2e through the C ABI
+from pinned host buffers, the CPU oracle on a bounded sample (cpu_baseline),
+SM clocks during the timed region and the number of libhq kernel launches.
+At N=1 the other BASELINE.json configs are measured too ("per_query").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--query Q --sf S] [--impl reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import hqgen  # noqa: E402
+
+DEFAULT_QUERY, DEFAULT_SF = "ssb_q41", 100.0
+# other BASELINE.json configs, measured at N=1 into "per_query"
+EXTRA = [("tpch_q6", 10.0), ("tpch_q1", 10.0), ("ssb_q11", 10.0), ("ssb_q12", 10.0), ("ssb_q13", 10.0),
+         ("ssb_q31", 30.0), ("tpch_q3", 30.0)]
+METRIC = "fact rows/s per query"
+
+
+# ----------------------------------------------------------------- helpers
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+class ClockSampler:
+    """Samples SM clocks and clock-event reasons with NVML during the timed region."""
+
+    REASONS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks_setting"}
+
+    def __init__(self, device_index: int):
+        self.samples, self.reasons, self.ok = [], set(), False
+        try:
+            import pynvml
+            import torch
+            pynvml.nvmlInit()
+            pr = torch.cuda.get_device_properties(device_index)
+            bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+            self.h = pynvml.nvmlDeviceGetHandleByPciBusId(bus)
+            self.max = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.nv = pynvml
+            self.ok = True
+        except Exception as e:  # noqa: BLE001
+            self.err = str(e)
+
+    def _run(self):
+        while not self.stop:
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit:
+                        self.reasons.add(name)
+            except Exception:  # noqa: BLE001
+                pass
+            time.sleep(0.02)
+
+    def __enter__(self):
+        self.stop = False
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self.stop = True
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "error": getattr(self, "err", "")}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None, "sm_max_mhz": self.max,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def gen_host(q, sf, seed, fact_range, with_dims, pinned=True):
+    """Referenced columns as numpy arrays (pinned host memory for the fact table)."""
+    import torch
+    host = {}
+    for t, cols in q.columns.items():
+        if t != q.fact and not with_dims:
+            continue
+        rr = fact_range if t == q.fact else None
+        n = (rr[1] - rr[0]) if rr else hqgen.table_rows(t, sf, seed)
+        out = None
+        if pinned and t == q.fact:
+            schema = dict(hqgen.SCHEMAS[hqgen.TABLE_NAMES[t]])
+            tdt = {"i1": torch.int8, "i4": torch.int32, "i8": torch.int64}
+            out = {c: torch.empty(n, dtype=tdt[schema[c]], pin_memory=True).numpy() for c in cols}
+        host[t] = hqgen.generate(t, sf, seed, columns=cols, row_range=rr, out=out)
+    return host
+
+
+def oracle_call(qname, host, nthreads, fact_rows=None):
+    """The CPU oracle on the first `fact_rows` fact rows (bounded sample)."""
+    import oracle
+    from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
+    q = QUERIES[qname]
+    t = {k: dict(v) for k, v in host.items()}
+    if fact_rows is not None:
+        t[q.fact] = {c: a[:fact_rows] for c, a in t[q.fact].items()}
+    f = {
+        "tpch_q6": lambda: oracle.tpch_q6(t["lineitem"], nthreads),
+        "tpch_q1": lambda: oracle.tpch_q1(t["lineitem"], nthreads),
+        "ssb_q11": lambda: oracle.ssb_q1(1, t["lineorder"], t["date"], nthreads=nthreads),
+        "ssb_q12": lambda: oracle.ssb_q1(2, t["lineorder"], t["date"], nthreads=nthreads),
+        "ssb_q13": lambda: oracle.ssb_q1(3, t["lineorder"], t["date"], nthreads=nthreads),
+        "ssb_q31": lambda: oracle.ssb_q31(t["lineorder"], t["customer"], t["supplier"], t["date"], nthreads=nthreads),
+        "ssb_q41": lambda: oracle.ssb_q41(t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"],
+                                          nthreads=nthreads),
+        "tpch_q3": lambda: oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"], nthreads=nthreads),
+    }[qname]
+    t0 = time.perf_counter()
+    f()
+    return time.perf_counter() - t0
+
+
+def cpu_baseline(qname, host, n_fact, target_s=12.0):
+    """Time the oracle (as it stands) on a bounded prefix sample of the workload."""
+    cores = os.cpu_count() or 1
+    s0 = min(n_fact, 2_000_000)
+    dt = oracle_call(qname, host, cores, s0)
+    rate = s0 / max(dt, 1e-9)
+    s = int(min(n_fact, max(s0, rate * target_s)))
+    if s > s0:
+        dt = oracle_call(qname, host, cores, s)
+    else:
+        s = s0
+    return {"value": s / dt, "unit": "rows/s", "cores": cores, "kind": "oracle",
+            "sample": f"first {s} of {n_fact} fact rows (full dimension tables), tuple-at-a-time C++ oracle, "
+                      f"{cores} threads, {dt:.2f} s"}
+
+
+# --------------------------------------------------------- device measurement
+def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, host=None):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sigmod_funkebnmt18_b200 import hq
+    from paper_conf_sigmod_funkebnmt18_b200.dist import DistributedEngine, partition
+    from paper_conf_sigmod_funkebnmt18_b200.engine import Engine
+    from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
+
+    q = QUERIES[qname]
+    dev = torch.device("cuda", local)
+    n = hqgen.table_rows(q.fact, sf, seed)
+    a, b = partition(n, rank, world)
+    root = rank == 0
+    if host is None:
+        host = gen_host(q, sf, seed, (a, b), with_dims=root or world == 1)
+    ctx = hq.Context(local)
+    # HBM-resident copies (torch memory, borrowed by libhq)
+    dtab = {t: {c: torch.from_numpy(np.asarray(arr)).to(dev) for c, arr in cols.items()} for t, cols in host.items()}
+    torch.cuda.synchronize()
+    tables = {t: ctx.load_columns(cols) for t, cols in dtab.items()}
+
+    def make_engine(tbls):
+        if world > 1:
+            return DistributedEngine(ctx, tbls)
+        return Engine(ctx, tbls)
+
+    E = make_engine(tables)
+
+    def step(Eng):
+        res, pb = q.run(Eng)
+        return Eng.finish(res, pb)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    for _ in range(warmup):
+        out = step(E)
+    ctx.kernel_times()
+    ctx.enable_timing(True)
+    l0 = ctx.launches()
+    stream = torch.cuda.current_stream(dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        torch.cuda.synchronize()
+        e0.record(stream)
+        for _ in range(steps):
+            out = step(E)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+    ms = e0.elapsed_time(e1) / steps
+    launches = ctx.launches() - l0
+    kt = ctx.kernel_times()
+    ctx.enable_timing(False)
+    per_step = max(1, len(kt) // steps)
+    fact_kt = kt[per_step - 1::per_step]  # the fact-table pipeline is the last fused launch of a step
+    kms = statistics.mean(fact_kt) if fact_kt else float("nan")
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+
+    res = {"ms": ms, "kernel_ms": kms, "launches": launches, "clocks": clk.summary(), "rows": n,
+           "local_rows": b - a, "result": out}
+    # ---- e2e: host (pinned) buffers through the public API, H2D inside the timed region
+    if with_e2e:
+        e2e_steps = max(1, min(steps, 3))
+        h2d = sum(arr.nbytes for cols in host.values() for arr in cols.values())
+
+        def e2e_step():
+            tb = {t: ctx.load_columns(cols) for t, cols in host.items()}
+            Eng = make_engine(tb)
+            r, pb = q.run(Eng)
+            o = Eng.finish(r, pb)
+            d2h = sum(c.nbytes for c in o.columns.values()) if o is not None else 0
+            del r, Eng, tb
+            return d2h
+
+        e2e_step()
+        barrier()
+        torch.cuda.synchronize()
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        d2h = 0
+        for _ in range(e2e_steps):
+            d2h = e2e_step()
+        f1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ems = f0.elapsed_time(f1) / e2e_steps
+        if world > 1:
+            t = torch.tensor([ems], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        res["e2e"] = {"value": n / (ems / 1e3), "unit": "rows/s", "h2d_bytes_per_step": int(h2d),
+                      "d2h_bytes_per_step": int(d2h), "ms_per_step": ems, "steps": e2e_steps}
+    res["host"] = host
+    del tables, dtab, E
+    ctx.close()
+    torch.cuda.empty_cache()
+    return res
+
+
+def roofline(q, local_rows, kernel_ms, peak, peak_src):
+    bpr = q.fact_bytes_per_row()
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            tr = json.load(f)
+        e = tr.get(q.name)
+        if e and e.get("rows") == local_rows:
+            traffic = e.get("dram_bytes_per_launch")
+    achieved = local_rows * bpr / (kernel_ms / 1e3) / 1e9
+    return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": traffic, "algorithmic_bytes": local_rows * bpr, "bytes_per_row": bpr,
+            "kernel": "hq_fused_pipeline_kernel", "kernel_ms": kernel_ms, "peak_source": peak_src}
+
+
+# ----------------------------------------------------------------- arms
+def run_reference(args):
+    """--impl reference: the CPU oracle (the only reference this paper-only tier has),
+    on the bench config, each step a bounded prefix sample of the fact table."""
+    if int(os.environ.get("RANK", "0")) != 0:
+        return
+    from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
+    q = QUERIES[args.query]
+    n = hqgen.table_rows(q.fact, args.sf, args.seed)
+    cores = os.cpu_count() or 1
+    probe = min(n, 1_000_000)
+    host = gen_host(q, args.sf, args.seed, (0, probe), with_dims=True, pinned=False)
+    rate = probe / oracle_call(args.query, host, cores)
+    sample = int(min(n, max(probe, rate * 2.0)))  # ~2 s per step
+    host = gen_host(q, args.sf, args.seed, (0, sample), with_dims=True, pinned=False)
+    for _ in range(args.warmup):
+        oracle_call(args.query, host, cores)
+    ts = [oracle_call(args.query, host, cores) for _ in range(args.steps)]
+    dt = sum(ts) / len(ts)
+    v = sample / dt
+    line = {"metric": METRIC, "value": v, "unit": "rows/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic (hqgen)",
+            "impl": "reference",
+            "config": {"workload": f"{args.query}_sf{args.sf:g}", "query": args.query, "sf": args.sf,
+                       "fact_rows": n, "sample_rows_per_step": sample},
+            "cpu_baseline": {"value": v, "unit": "rows/s", "cores": cores, "kind": "oracle",
+                             "sample": f"first {sample} of {n} fact rows per step (full dimension tables)"},
+            "e2e": {"value": v, "unit": "rows/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_hq(args):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    peak, peak_src = peaks()
+    q = QUERIES[args.query]
+    r = measure(args.query, args.sf, args.steps, args.warmup, args.seed, rank, world, local)
+    value = r["rows"] / (r["ms"] / 1e3)
+    line = None
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "rows/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": r["ms"], "higher_is_better": True,
+                "scaling": "strong" if world > 1 else "strong", "vs_baseline": None, "dtype": "int64",
+                "data": "synthetic (hqgen TPC-H/SSB-shaped generator, seed %d)" % args.seed,
+                "config": {"workload": f"{args.query}_sf{args.sf:g}", "query": args.query, "sf": args.sf,
+                           "fact_rows": r["rows"], "fact_bytes": r["rows"] * q.fact_bytes_per_row(),
+                           "l2": "inputs larger than L2 (no flush needed)",
+                           "parallelism": f"fact range partition dp{world}, dimension HTs broadcast, 1 reduce",
+                           "step": "hash builds + fused pipeline + reduce + finalize/fetch"},
+                "roofline": roofline(q, r["local_rows"], r["kernel_ms"], peak, peak_src),
+                "e2e": r.get("e2e"), "gpu_launches": r["launches"], "clocks": r["clocks"]}
+        line["roofline"]["kernel_share_of_step"] = r["kernel_ms"] / r["ms"]
+        if world == 1:
+            line["cpu_baseline"] = cpu_baseline(args.query, r["host"], r["rows"])
+    del r
+    if world == 1 and not args.no_extra and args.query == DEFAULT_QUERY:
+        per = []
+        for qn, sf in EXTRA:
+            try:
+                x = measure(qn, sf, args.steps, args.warmup, args.seed, 0, 1, local, with_e2e=False)
+                qq = QUERIES[qn]
+                per.append({"query": qn, "sf": sf, "fact_rows": x["rows"], "value": x["rows"] / (x["ms"] / 1e3),
+                            "unit": "rows/s", "ms_per_step": x["ms"],
+                            "roofline": roofline(qq, x["local_rows"], x["kernel_ms"], peak, peak_src)})
+                del x
+            except Exception as e:  # noqa: BLE001
+                per.append({"query": qn, "sf": sf, "error": str(e)[:200]})
+        line["per_query"] = per
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="hq", choices=["hq", "reference"])
+    ap.add_argument("--query", default=DEFAULT_QUERY)
+    ap.add_argument("--sf", type=float, default=DEFAULT_SF)
+    ap.add_argument("--seed", type=int, default=hqgen.DEFAULT_SEED)
+    ap.add_argument("--no-extra", action="store_true", help="skip the per_query configs at N=1")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_hq(args)
+
+
+if __name__ == "__main__":
+    main()

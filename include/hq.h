@@ -121,6 +121,8 @@ size_t hq_sizeof(const char* struct_name);
  * returns (and clears) the durations in ms, oldest first; *n = count. */
 hq_status hq_ctx_enable_timing(hq_ctx* ctx, int32_t on);
 hq_status hq_ctx_kernel_times(hq_ctx* ctx, float* ms, int32_t max, int32_t* n);
+/* Cumulative number of CUDA kernels this context has launched. */
+hq_status hq_ctx_launches(hq_ctx* ctx, int64_t* n);
 
 /* ----------------------------------------------------------------- tables */
 typedef struct {
@@ -162,16 +164,25 @@ typedef struct {
   int64_t expected_rows; /* >0: capacity sized for this many keys (no count pass, no host sync);
                             <=0: a count pass sizes the table exactly (one ctx sync) */
 } hq_build_desc;
-/* Open addressing, linear probing, power-of-two capacity >= keys/0.6, slot =
- * {int32 key, payload...} of 4, 8 or 16 bytes, empty key INT32_MIN, inserted
- * with one atomicCAS on the key.  Duplicate keys: HQ_ERR_DUP_KEY at hq_hash_info. */
+/* Slot = {int32 key, payload...} of 4, 8 or 16 bytes, empty key INT32_MIN,
+ * claimed with one atomicCAS on the key.  Two layouts:
+ *  - HQ_HT_DIRECT (dense keys, chosen when the count pass finds the qualifying
+ *    keys' range <= 8 x their number or the array <= 2 MiB): slot = key - key_min,
+ *    one load per probe;
+ *  - HQ_HT_LINEAR: multiplicative hash, linear probing, power-of-two capacity
+ *    >= keys/0.6; probes scan whole aligned 16-B slot groups per load.
+ * Duplicate keys: HQ_ERR_DUP_KEY at hq_hash_info. */
 hq_status hq_build_hash(hq_ctx* ctx, const hq_build_desc* desc, hq_hash** out);
+enum { HQ_HT_LINEAR = 0, HQ_HT_DIRECT = 1 };
 typedef struct {
-  int64_t capacity;     /* slots (power of two) */
+  int64_t capacity;     /* slots (power of two for HQ_HT_LINEAR, key range for HQ_HT_DIRECT) */
   int32_t slot_words;   /* 1, 2 or 4 int32 words per slot */
   int32_t npayload;
   int64_t nkeys;        /* keys inserted (valid after hq_hash_info) */
   int64_t bytes;        /* capacity * slot_words * 4 */
+  int64_t key_min;      /* HQ_HT_DIRECT: key stored in slot 0 */
+  int32_t layout;       /* HQ_HT_LINEAR or HQ_HT_DIRECT */
+  int32_t reserved;
 } hq_hash_meta;
 hq_status hq_hash_info(hq_ctx* ctx, const hq_hash* h, hq_hash_meta* meta);  /* syncs, reports build faults */
 /* Multi-GPU glue: raw device view of the slot array (to broadcast it with NCCL)

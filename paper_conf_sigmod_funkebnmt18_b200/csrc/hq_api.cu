@@ -170,6 +170,13 @@ hq_status hq_ctx_kernel_times(hq_ctx* ctx, float* ms, int32_t max, int32_t* n) {
   });
 }
 
+hq_status hq_ctx_launches(hq_ctx* ctx, int64_t* n) {
+  return guarded([&] {
+    if (!ctx || !n) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    *n = ctx->launches;
+  });
+}
+
 // ------------------------------------------------------------------ tables
 hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int64_t nrows, int32_t flags,
                           hq_table** out) {
@@ -266,7 +273,13 @@ hq_status hq_hash_import(hq_ctx* ctx, const hq_hash_meta* meta, void* dev_ptr, h
   return guarded([&] {
     if (!ctx || !meta || !dev_ptr || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     const int64_t cap = meta->capacity;
-    if (cap < 16 || (cap & (cap - 1)) != 0) HQ_THROW(HQ_ERR_ARG, "import: capacity must be a power of two >= 16");
+    if (meta->layout == HQ_HT_DIRECT) {
+      if (cap < 1 || cap > (1LL << 30)) HQ_THROW(HQ_ERR_ARG, "import: direct capacity out of range");
+    } else if (meta->layout == HQ_HT_LINEAR) {
+      if (cap < 16 || (cap & (cap - 1)) != 0) HQ_THROW(HQ_ERR_ARG, "import: capacity must be a power of two >= 16");
+    } else {
+      HQ_THROW(HQ_ERR_ARG, "import: unknown layout");
+    }
     if (meta->slot_words != 1 && meta->slot_words != 2 && meta->slot_words != 4) HQ_THROW(HQ_ERR_ARG, "import: slot_words");
     if (meta->npayload < 0 || meta->npayload > meta->slot_words - 1 + (meta->slot_words == 1 ? 0 : 0) ||
         (meta->slot_words == 1 && meta->npayload != 0))

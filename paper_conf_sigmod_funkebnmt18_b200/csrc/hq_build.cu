@@ -30,10 +30,12 @@ struct KBuild {
   int32_t key_col, npay;
   int32_t pay_col[HQ_MAX_PAYLOAD];
   uint32_t* slots;
-  uint32_t mask;
+  uint32_t mask;     // LINEAR: capacity - 1; DIRECT: key range
   int32_t log2cap, words;
+  int32_t direct, dmin;
   int* err;
   unsigned long long* nkeys;
+  int* kminmax;      // count pass: [min, max] of the qualifying keys
 };
 
 __device__ __forceinline__ long long ld_col(const KBuild& b, int c, long long row) {
@@ -56,8 +58,22 @@ __device__ __forceinline__ bool row_passes(const KBuild& b, long long row) {
 
 __global__ void hq_build_count_kernel(const __grid_constant__ KBuild b) {
   unsigned long long c = 0;
-  for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < b.n; r += (long long)gridDim.x * blockDim.x)
-    c += row_passes(b, r);
+  int kmin = INT_MAX, kmax = INT_MIN;
+  for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < b.n; r += (long long)gridDim.x * blockDim.x) {
+    if (!row_passes(b, r)) continue;
+    ++c;
+    const long long kv = ld_col(b, b.key_col, r);
+    if (kv > (long long)INT_MIN && kv <= (long long)INT_MAX) {
+      kmin = min(kmin, (int)kv);
+      kmax = max(kmax, (int)kv);
+    }
+  }
+  kmin = __reduce_min_sync(0xffffffffu, kmin);
+  kmax = __reduce_max_sync(0xffffffffu, kmax);
+  if ((threadIdx.x & 31) == 0 && kmin <= kmax) {
+    atomicMin(b.kminmax, kmin);
+    atomicMax(b.kminmax + 1, kmax);
+  }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
   __shared__ unsigned long long red[32];
@@ -93,7 +109,11 @@ __global__ void hq_build_hash_kernel(const __grid_constant__ KBuild b) {
       if (v < (long long)INT_MIN || v > (long long)INT_MAX) fault |= HQF_BAD_PAYLOAD;
       pay[k] = (int)v;
     }
-    uint32_t pos = ((uint32_t)key * 0x9E3779B1u) >> shift;
+    uint32_t pos = b.direct ? (uint32_t)(key - b.dmin) : ((uint32_t)key * 0x9E3779B1u) >> shift;
+    if (b.direct && pos >= b.mask) {  // cannot happen: the range comes from the count pass
+      fault |= HQF_HT_FULL;
+      continue;
+    }
     uint32_t i = 0;
     for (; i <= b.mask; ++i) {
       uint32_t* slot = b.slots + (size_t)pos * b.words;
@@ -103,7 +123,7 @@ __global__ void hq_build_hash_kernel(const __grid_constant__ KBuild b) {
         ++inserted;
         break;
       }
-      if (old == key) {
+      if (old == key || b.direct) {
         fault |= HQF_DUP_KEY;  // join keys must be unique (R6)
         break;
       }
@@ -173,20 +193,31 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   HQ_CUDA(cudaMemsetAsync(h->dstate.p, 0, 64, ctx->stream));
   b.err = h->dstate.as<int>();
   b.nkeys = (unsigned long long*)(h->dstate.as<char>() + 8);
+  b.kminmax = (int*)(h->dstate.as<char>() + 16);
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((b.n + 255) / 256, (int64_t)ctx->num_sms * 8));
   int64_t keys = d->expected_rows;
-  if (keys <= 0) {  // exact count pass (one sync)
-    if (b.n > 0) hq_build_count_kernel<<<grid, 256, 0, ctx->stream>>>(b);
+  const int words = d->npayload == 0 ? 1 : (d->npayload == 1 ? 2 : 4);
+  bool direct = false;
+  int64_t kmin = 0, range = 0;
+  if (keys <= 0) {  // exact count pass (one sync): number and range of the qualifying keys
+    const int init[2] = {INT_MAX, INT_MIN};
+    HQ_CUDA(cudaMemcpyAsync(b.kminmax, init, 8, cudaMemcpyHostToDevice, ctx->stream));
+    if (b.n > 0) { ctx->launches++; hq_build_count_kernel<<<grid, 256, 0, ctx->stream>>>(b); }
     HQ_CUDA(cudaGetLastError());
-    unsigned long long cnt = 0;
-    HQ_CUDA(cudaMemcpyAsync(&cnt, b.nkeys, 8, cudaMemcpyDeviceToHost, ctx->stream));
+    struct { unsigned long long cnt; int kmin, kmax; } st{};
+    HQ_CUDA(cudaMemcpyAsync(&st, b.nkeys, 16, cudaMemcpyDeviceToHost, ctx->stream));
     HQ_CUDA(cudaStreamSynchronize(ctx->stream));
     HQ_CUDA(cudaMemsetAsync(b.nkeys, 0, 8, ctx->stream));
-    keys = (int64_t)cnt;
+    keys = (int64_t)st.cnt;
+    if (keys > 0 && st.kmin <= st.kmax) {
+      kmin = st.kmin;
+      range = (int64_t)st.kmax - st.kmin + 1;
+      // dense keys: direct-mapped slot array (one load per probe)
+      direct = range <= (1LL << 30) && (range <= 8 * keys || range * words * 4 <= (2LL << 20));
+    }
   }
-  const int64_t cap = std::max<int64_t>(16, next_pow2((keys * 5 + 2) / 3));  // load factor <= 0.6
+  const int64_t cap = direct ? range : std::max<int64_t>(16, next_pow2((keys * 5 + 2) / 3));  // load <= 0.6
   if (cap > (1LL << 31)) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: hash table too large");
-  const int words = d->npayload == 0 ? 1 : (d->npayload == 1 ? 2 : 4);
   int log2 = 0;
   while ((1LL << log2) < cap) ++log2;
   h->owned = DevBuf(ctx, (size_t)cap * words * 4);
@@ -197,15 +228,20 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   h->meta.npayload = d->npayload;
   h->meta.nkeys = -1;
   h->meta.bytes = cap * words * 4;
+  h->meta.layout = direct ? HQ_HT_DIRECT : HQ_HT_LINEAR;
+  h->meta.key_min = kmin;
   const int64_t nw = cap * words;
   const int fgrid = (int)std::max<int64_t>(1, std::min<int64_t>((nw + 255) / 256, (int64_t)ctx->num_sms * 8));
+  ctx->launches++;
   hq_fill_kernel<<<fgrid, 256, 0, ctx->stream>>>(h->slots, nw, 0x80000000u);
   HQ_CUDA(cudaGetLastError());
   b.slots = h->slots;
-  b.mask = (uint32_t)(cap - 1);
+  b.mask = direct ? (uint32_t)cap : (uint32_t)(cap - 1);
   b.log2cap = log2;
   b.words = words;
-  if (b.n > 0) hq_build_hash_kernel<<<grid, 256, 0, ctx->stream>>>(b);
+  b.direct = direct;
+  b.dmin = (int32_t)kmin;
+  if (b.n > 0) { ctx->launches++; hq_build_hash_kernel<<<grid, 256, 0, ctx->stream>>>(b); }
   HQ_CUDA(cudaGetLastError());
 }
 

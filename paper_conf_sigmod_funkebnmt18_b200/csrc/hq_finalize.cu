@@ -203,6 +203,7 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
   k.nout = scratch.as<unsigned long long>();
   k.err = (int*)(scratch.as<char>() + 16);
   k.scalar = nk == 0;
+  ctx->launches++;
   hq_compact_kernel<<<grid_for(ctx, r->ngroups), 256, 0, ctx->stream>>>(k);
   HQ_CUDA(cudaGetLastError());
   struct { unsigned long long rows, qual; int err; int pad; } st2{};
@@ -242,6 +243,7 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
         const int64_t chunks = (cur_n + SORT_CHUNK - 1) / SORT_CHUNK;
         const int kp = chunks == 1 ? (int)std::min<int64_t>(cur_n, SORT_CHUNK) : keep;
         int* dst = bufs[which];
+        ctx->launches++;
         hq_chunk_sort_kernel<<<(unsigned)chunks, 1024, 0, ctx->stream>>>(s, cur, cur_n, dst, kp);
         HQ_CUDA(cudaGetLastError());
         cur = dst;
@@ -251,6 +253,7 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
       }
       sorted = (int*)cur;
     } else if (n <= SORT_CHUNK) {
+      ctx->launches++;
       hq_chunk_sort_kernel<<<1, 1024, 0, ctx->stream>>>(s, nullptr, n, ia.as<int>(), SORT_CHUNK);
       HQ_CUDA(cudaGetLastError());
       sorted = ia.as<int>();
@@ -258,16 +261,20 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
       int64_t N = 1;
       while (N < n) N <<= 1;
       ia = DevBuf(ctx, (size_t)N * 4);
+      ctx->launches++;
       hq_iota_kernel<<<grid_for(ctx, N), 256, 0, ctx->stream>>>(ia.as<int>(), N, n);
       for (int64_t kk = 2; kk <= N; kk <<= 1)
-        for (int64_t j = kk >> 1; j > 0; j >>= 1)
+        for (int64_t j = kk >> 1; j > 0; j >>= 1) {
+          ctx->launches++;
           hq_bitonic_step_kernel<<<grid_for(ctx, N), 256, 0, ctx->stream>>>(s, ia.as<int>(), N, j, kk);
+        }
       HQ_CUDA(cudaGetLastError());
       sorted = ia.as<int>();
     }
     std::vector<DevBuf> out;
     for (int c = 0; c < nc; ++c) {
       out.emplace_back(ctx, (size_t)std::max<int64_t>(nfinal, 1) * 8);
+      ctx->launches++;
       hq_gather_kernel<<<grid_for(ctx, nfinal), 256, 0, ctx->stream>>>(cols[c].as<long long>(), sorted, nfinal,
                                                                       out.back().as<long long>());
     }

@@ -52,6 +52,7 @@ struct hq_ctx {
   int num_sms = 148;
   size_t max_smem = 232448;
   bool timing = false;
+  int64_t launches = 0;  // kernels this context has launched (hq_ctx_launches)
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> events;  // recorded, not yet read
   std::vector<cudaEvent_t> event_pool;
   void* alloc_bytes(size_t bytes);
@@ -134,7 +135,11 @@ constexpr unsigned long long EMPTY_KEY = ~0ULL;
 
 enum : uint8_t { OP_FILTER = 1, OP_PROBE = 2, OP_COMPUTE = 3 };
 enum : uint8_t { GM_SCALAR = 0, GM_DENSE = 1, GM_HASH = 2 };   // global group table
-enum : uint8_t { SM_NONE = 0, SM_DENSE = 1, SM_HASH = 2 };     // smem pre-aggregation table
+// smem pre-aggregation table: none, shared dense (atomics), shared hash (atomics),
+// lane-private dense accumulators (no atomics; tiny group domains, 8 warps)
+enum : uint8_t { SM_NONE = 0, SM_DENSE = 1, SM_HASH = 2, SM_LANE = 3 };
+constexpr int LANE_NW = 8;                 // consumer warps when SM_LANE
+constexpr int SMEM_LANE_BYTES = 96 * 1024; // lane-private table budget
 
 struct KReg {
   uint32_t off;      // byte offset of row 0 in the stage (column) or tmp region (temporary)
@@ -157,11 +162,14 @@ struct KPred {
 };
 struct KProbe {
   const uint32_t* slots;
-  uint32_t mask;     // capacity - 1
+  uint32_t mask;     // LINEAR: capacity - 1; DIRECT: key range (capacity)
+  int32_t dmin;      // DIRECT: key of slot 0
   uint8_t log2cap;
   uint8_t words;     // 1, 2, 4
   uint8_t mode;      // hq_probe_mode
   uint8_t npay;
+  uint8_t direct;    // 1 = direct-mapped (dense keys)
+  uint8_t pad;
   int16_t key_reg;
   int16_t dst[HQ_MAX_PAYLOAD];
 };
@@ -184,6 +192,7 @@ struct KOp {
 
 struct KPlan {
   int64_t row_begin, row_end;
+  int32_t nw;                // consumer warps (blockDim = (nw + 1) * 32)
   int32_t R, tile_rows, nstages;
   uint32_t stage_bytes;      // bytes of one stage's columns (= tile_rows * row width)
   uint32_t stage_stride;     // stage spacing in smem (>= stage_bytes, 128-B multiple)
@@ -214,6 +223,11 @@ struct KPlan {
   int32_t glog2;
   uint32_t smem_cap;         // smem dense groups or smem hash slots
   int32_t slog2;
+  // SM_LANE: deduplicated accumulators (0 = count; SUM and AVG of one register share)
+  int32_t nacc;
+  uint8_t acc_fn[HQ_MAX_AGGS + 1];
+  int16_t acc_reg[HQ_MAX_AGGS + 1];
+  uint8_t acc_of[HQ_MAX_AGGS];  // aggregate -> accumulator
   // materialise
   int32_t nout;
   int16_t out_reg[HQ_MAX_OUT];
@@ -263,7 +277,8 @@ int64_t fused_smem_bytes(const KPlan& kp);
 void hq_finalize_impl(hq_ctx* ctx, hq_result* r);
 // op-at-a-time execution of a plan (hq_oaat.cu)
 void hq_run_oaat(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
-// shared plan preparation (hq_pipeline.cu)
+// shared plan preparation (hq_plan.cu)
 void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
+void hq_build_kplan(hq_ctx* ctx, hq_result* r, hqk::KPlan& kp, int64_t group_cap, int64_t mat_cap);
 void hq_check_result_faults(hq_ctx* ctx, hq_result* r);
 int hq_type_width(int type);

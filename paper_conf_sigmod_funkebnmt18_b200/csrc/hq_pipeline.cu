@@ -27,6 +27,7 @@
 #include <cstring>
 
 #include "hq_internal.h"
+#include "hq_device.cuh"
 
 namespace hqk {
 
@@ -49,9 +50,9 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
   asm volatile(
       "{\n\t.reg .pred p;\n"
       "HQ_WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
       "@!p bra HQ_WAIT_%=;\n}\n" ::"r"(smem_u32(b)),
-      "r"(parity)
+      "r"(parity), "r"(1000000)  // suspend-time hint (ns): sleep in HW instead of spinning
       : "memory");
 }
 __device__ __forceinline__ uint64_t policy_evict_first() {
@@ -73,8 +74,8 @@ __device__ __forceinline__ void fence_proxy_async() {
 __device__ __forceinline__ void fence_mbar_init() {
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
 }
-__device__ __forceinline__ void consumer_bar() {  // all consumer warps (not the producer)
-  asm volatile("bar.sync 1, %0;" ::"n"(NW * 32) : "memory");
+__device__ __forceinline__ void consumer_bar(int nw) {  // all consumer warps (not the producer)
+  asm volatile("bar.sync 1, %0;" ::"r"(nw * 32) : "memory");
 }
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t m;
@@ -168,48 +169,80 @@ __device__ __forceinline__ uint32_t op_filter(const KPlan& p, int idx, const cha
 
 // Join probe (Fig 8 "check match" + "build tuple"): in the
 // compound kernel the probe runs once and the payload stays on chip
-// (P:947-953).  Linear probing over {key, payload...} slots of W words.
+// (P:947-953).  Slots are {key, payload...} of W words.  Direct-mapped tables
+// (dense keys) resolve every probe with one load; linear-probing tables load a
+// whole aligned 16-B group (4, 2 or 1 slots) per round and scan it in probe
+// order, so a warp's round count is rarely more than one.
 template <int R, int W>
 __device__ __forceinline__ uint32_t probe_rows(const KPlan& p, const KProbe& pr, const long long (&kv)[R],
                                                char* tmp, int row0, uint32_t mask) {
   uint32_t pending = mask, found = 0;
   uint32_t pos[R];
-  const uint32_t shift = 32u - pr.log2cap;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
     const bool ok = kv[r] > (long long)INT_MIN && kv[r] <= (long long)INT_MAX;
     if (!ok) pending &= ~(1u << r);
-    pos[r] = ((uint32_t)(int)kv[r] * 0x9E3779B1u) >> shift;
+    if (pr.direct) {
+      pos[r] = (uint32_t)((int)kv[r] - pr.dmin);
+      if (pos[r] >= pr.mask) pending &= ~(1u << r);  // outside the key range: miss
+    } else {
+      pos[r] = ((uint32_t)(int)kv[r] * 0x9E3779B1u) >> (32u - pr.log2cap);
+    }
   }
   const bool inner = pr.mode == HQ_PROBE_INNER;
   int* dst0 = (int*)(tmp + p.regs[pr.dst[0]].off) + row0;
   int* dst1 = (int*)(tmp + p.regs[pr.dst[W > 2 ? 1 : 0]].off) + row0;
   int* dst2 = (int*)(tmp + p.regs[pr.dst[W > 2 ? 2 : 0]].off) + row0;
+  constexpr int G = W == 1 ? 4 : (W == 2 ? 2 : 1);  // slots per 16-B group
   while (pending) {
     int4 sl[R];
 #pragma unroll
-    for (int r = 0; r < R; ++r) {  // R independent slot loads in flight
+    for (int r = 0; r < R; ++r) {  // R independent loads in flight
       if (pending & (1u << r)) {
-        if (W == 1) sl[r].x = __ldg((const int*)pr.slots + pos[r]);
-        else if (W == 2) { const int2 t = __ldg((const int2*)pr.slots + pos[r]); sl[r].x = t.x; sl[r].y = t.y; }
-        else sl[r] = __ldg((const int4*)pr.slots + pos[r]);
+        if (pr.direct) {
+          if (W == 1) sl[r].x = __ldg((const int*)pr.slots + pos[r]);
+          else if (W == 2) { const int2 t = __ldg((const int2*)pr.slots + pos[r]); sl[r].x = t.x; sl[r].y = t.y; }
+          else sl[r] = __ldg((const int4*)pr.slots + pos[r]);
+        } else {
+          sl[r] = __ldg((const int4*)pr.slots + pos[r] / G);
+        }
       }
     }
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       if (pending & (1u << r)) {
-        if (sl[r].x == (int)kv[r]) {
+        const int key = (int)kv[r];
+        int sk[G], sp0[G], sp1 = sl[r].z, sp2 = sl[r].w;
+        if (G == 4) { sk[0] = sl[r].x; sk[G > 1 ? 1 : 0] = sl[r].y; sk[G > 2 ? 2 : 0] = sl[r].z; sk[G > 3 ? 3 : 0] = sl[r].w; }
+        else if (G == 2) { sk[0] = sl[r].x; sp0[0] = sl[r].y; sk[G > 1 ? 1 : 0] = sl[r].z; sp0[G > 1 ? 1 : 0] = sl[r].w; }
+        else { sk[0] = sl[r].x; sp0[0] = sl[r].y; }
+        const int first = pr.direct ? 0 : (int)(pos[r] % G);
+        int hit = -1;
+        bool stop = pr.direct;
+#pragma unroll
+        for (int j = 0; j < G; ++j) {
+          if (!stop && j >= first) {
+            if (sk[j] == key) { hit = j; stop = true; }
+            else if (sk[j] == INT_MIN) stop = true;
+          }
+        }
+        if (pr.direct && sk[0] == key) hit = 0;
+        if (hit >= 0) {
           found |= 1u << r;
           pending &= ~(1u << r);
           if (W > 1 && inner) {  // payload stays on chip
-            if (pr.npay > 0) dst0[r * 32] = sl[r].y;
-            if (W > 2 && pr.npay > 1) dst1[r * 32] = sl[r].z;
-            if (W > 2 && pr.npay > 2) dst2[r * 32] = sl[r].w;
+            int v0 = sp0[0];
+#pragma unroll
+            for (int j = 1; j < G; ++j)
+              if (hit == j) v0 = sp0[j];
+            if (pr.npay > 0) dst0[r * 32] = v0;
+            if (W > 2 && pr.npay > 1) dst1[r * 32] = sp1;
+            if (W > 2 && pr.npay > 2) dst2[r * 32] = sp2;
           }
-        } else if (sl[r].x == INT_MIN) {
+        } else if (stop) {
           pending &= ~(1u << r);
         } else {
-          pos[r] = (pos[r] + 1) & pr.mask;
+          pos[r] = ((pos[r] / G + 1) * G) & pr.mask;  // next group
         }
       }
     }
@@ -287,63 +320,11 @@ __device__ __forceinline__ void op_compute(const KPlan& p, int idx, const char* 
   store_tmp<R>(p, c.dst, tmp, row0, acc);
 }
 
-// --------------------------------------------------------------- agg tables
-__device__ __forceinline__ long long agg_identity(uint8_t fn) {
-  return fn == HQ_AGG_MIN ? LLONG_MAX : (fn == HQ_AGG_MAX ? LLONG_MIN : 0);
-}
-__device__ __forceinline__ long long agg_combine(uint8_t fn, long long a, long long b) {
-  return fn == HQ_AGG_MIN ? (a < b ? a : b) : (fn == HQ_AGG_MAX ? (a > b ? a : b) : a + b);
-}
-__device__ __forceinline__ long long warp_reduce(uint8_t fn, long long v) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v = agg_combine(fn, v, __shfl_xor_sync(FULLMASK, v, o));
-  return v;
-}
-// one aggregate update with a shared- or global-memory atomic
-__device__ __forceinline__ void agg_atomic(uint8_t fn, long long* t, long long v, unsigned long long cnt) {
-  if (fn == HQ_AGG_MIN) atomicMin(t, v);
-  else if (fn == HQ_AGG_MAX) atomicMax(t, v);
-  else if (fn == HQ_AGG_COUNT) atomicAdd((unsigned long long*)t, cnt);
-  else atomicAdd((unsigned long long*)t, (unsigned long long)v);
-}
-// accumulate (count, vals) into one table entry [count, agg...] with atomics
-__device__ __forceinline__ void entry_update(const KPlan& p, long long* e, unsigned long long cnt,
-                                             const long long* vals) {
-  atomicAdd((unsigned long long*)e, cnt);
-  for (int a = 0; a < p.naggs; ++a) agg_atomic(p.agg_fn[a], e + 1 + a, vals[a], cnt);
-}
-__device__ __forceinline__ uint32_t hash64(unsigned long long k, int log2) {
-  return (uint32_t)((k * 0x9E3779B97F4A7C15ull) >> (64 - log2));
-}
-// Global propagation target: dense array slot, or the entry of `key` in the
-// global hash table, claimed with atomicCAS ("atomic_hash_reduce", App C
-// P:2049-2052).  NULL (fault raised) when the hash table is full.
-__device__ long long* global_locate(const KPlan& p, unsigned long long key) {
-  if (p.gmode != GM_HASH) return p.gtab + key * p.vwords;
-  const uint32_t vw1 = p.vwords + 1;
-  uint64_t h = hash64(key, p.glog2);
-  for (uint64_t i = 0; i <= p.gmask; ++i) {
-    unsigned long long* kp = (unsigned long long*)(p.gtab + h * vw1);
-    const unsigned long long k = *(volatile unsigned long long*)kp;
-    if (k == key) return p.gtab + h * vw1 + 1;
-    if (k == EMPTY_KEY) {
-      const unsigned long long old = atomicCAS(kp, EMPTY_KEY, key);
-      if (old == EMPTY_KEY || old == key) return p.gtab + h * vw1 + 1;
-    }
-    h = (h + 1) & p.gmask;
-  }
-  atomicOr(p.err, HQF_GROUP_FULL);
-  return nullptr;
-}
-__device__ __forceinline__ void global_update(const KPlan& p, unsigned long long key, unsigned long long cnt,
-                                              const long long* vals) {
-  long long* e = global_locate(p, key);
-  if (e) entry_update(p, e, cnt, vals);
-}
-// Local resolution target: the shared-memory dense table or hash table entry;
-// falls back to the global table when the smem hash table is full (C3 -> C2).
-__device__ __forceinline__ long long* local_locate(const KPlan& p, char* sagg, unsigned long long key) {
-  if (p.smode == SM_DENSE) return (long long*)sagg + key * p.vwords;
+// Local resolution target: the shared address of the shared-memory dense or
+// hash table entry, or 0 when the smem hash table is full -- the caller then
+// propagates to the global table directly (C3 -> C2).
+__device__ __forceinline__ uint32_t local_locate(const KPlan& p, char* sagg, unsigned long long key) {
+  if (p.smode == SM_DENSE) return smem_u32((long long*)sagg + key * p.vwords);
   if (p.smode == SM_HASH) {
     unsigned long long* keys = (unsigned long long*)sagg;
     long long* ent = (long long*)sagg + p.smem_cap;
@@ -357,11 +338,32 @@ __device__ __forceinline__ long long* local_locate(const KPlan& p, char* sagg, u
         const unsigned long long old = atomicCAS(keys + h, EMPTY_KEY, key);
         hit = old == EMPTY_KEY || old == key;
       }
-      if (hit) return ent + (size_t)h * p.vwords;
+      if (hit) return smem_u32(ent + (size_t)h * p.vwords);
       h = (h + 1) & m;
     }
   }
-  return global_locate(p, key);
+  return 0u;
+}
+// Update one group entry -- shared (split 32-bit atomics) when the local table
+// holds it, else global (red) -- with `cnt` rows whose aggregate values come
+// from val(a).
+template <class Val>
+__device__ __forceinline__ void group_update(const KPlan& p, char* sagg, unsigned long long key, bool local,
+                                             unsigned long long cnt, Val val) {
+  const uint32_t sa = local ? local_locate(p, sagg, key) : 0u;
+  if (sa) {
+    s_add64(sa, (long long)cnt);
+#pragma unroll
+    for (int a = 0; a < HQ_MAX_AGGS; ++a)
+      if (a < p.naggs) s_agg(p.agg_fn[a], sa + 8u * (1 + a), val(a), cnt);
+    return;
+  }
+  long long* e = global_locate(p, key);
+  if (!e) return;
+  g_add64(e, (long long)cnt);
+#pragma unroll
+  for (int a = 0; a < HQ_MAX_AGGS; ++a)
+    if (a < p.naggs) g_agg(p.agg_fn[a], e + 1 + a, val(a), cnt);
 }
 
 // ------------------------------------------------------------------- sinks
@@ -391,6 +393,25 @@ __device__ __forceinline__ void sink_group(const KPlan& p, const char* stage, co
     }
     if (bad) atomicOr(p.err, HQF_KEY_DOMAIN);
   }
+  if (p.smode == SM_LANE) {
+    // tiny dense group domain: every lane owns a private accumulator table in
+    // shared memory ([entry][lane] layout), updated with plain read-modify-write
+    long long* lt = (long long*)sagg + threadIdx.x;
+    const int nl = p.nw * 32;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if ((mask >> r) & 1u) {
+        const int row = row0 + r * 32;
+        long long* e = lt + (size_t)gk[r] * p.nacc * nl;
+        e[0] += 1;
+        for (int a = 1; a < p.nacc; ++a) {
+          const long long v = load_one(p, p.acc_reg[a], stage, tmp, row);
+          e[a * nl] = agg_combine(p.acc_fn[a], e[a * nl], v);
+        }
+      }
+    }
+    return;
+  }
   const bool c2 = p.resolution == HQ_RES_ATOMIC;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
@@ -402,32 +423,27 @@ __device__ __forceinline__ void sink_group(const KPlan& p, const char* stage, co
     const uint32_t peers = c2 ? (1u << lane) & act : __match_any_sync(FULLMASK, mk) & act;
     const bool single = live && __popc(peers) == 1;
     if (single) {  // C2 rows, and keys unique within the warp: direct update
-      long long* e = c2 ? global_locate(p, gk[r]) : local_locate(p, sagg, gk[r]);
-      if (e) {
-        atomicAdd((unsigned long long*)e, 1ull);
-        for (int a = 0; a < p.naggs; ++a) {
-          const uint8_t fn = p.agg_fn[a];
-          agg_atomic(fn, e + 1 + a, fn == HQ_AGG_COUNT ? 1 : load_one(p, p.agg_reg[a], stage, tmp, row), 1);
-        }
-      }
+      group_update(p, sagg, gk[r], !c2, 1ull, [&](int a) {
+        return p.agg_fn[a] == HQ_AGG_COUNT ? 1ll : load_one(p, p.agg_reg[a], stage, tmp, row);
+      });
     }
     uint32_t multi = act & ~__ballot_sync(FULLMASK, single);
     while (multi) {  // one warp-wide reduction per distinct key, leader updates
       const int leader = __ffs(multi) - 1;
       const uint32_t grp = __shfl_sync(FULLMASK, peers, leader);
       const bool mine = (grp >> lane) & 1u;
-      long long* e = nullptr;
-      if (lane == leader) {
-        e = local_locate(p, sagg, gk[r]);
-        if (e) atomicAdd((unsigned long long*)e, (unsigned long long)__popc(grp));
+      long long vals[HQ_MAX_AGGS];
+#pragma unroll
+      for (int a = 0; a < HQ_MAX_AGGS; ++a) {
+        if (a < p.naggs) {
+          const uint8_t fn = p.agg_fn[a];
+          long long v = agg_identity(fn);
+          if (mine) v = fn == HQ_AGG_COUNT ? 1 : load_one(p, p.agg_reg[a], stage, tmp, row);
+          vals[a] = warp_reduce(fn, v);
+        }
       }
-      for (int a = 0; a < p.naggs; ++a) {
-        const uint8_t fn = p.agg_fn[a];
-        long long v = agg_identity(fn);
-        if (mine) v = fn == HQ_AGG_COUNT ? 1 : load_one(p, p.agg_reg[a], stage, tmp, row);
-        v = warp_reduce(fn, v);
-        if (lane == leader && e) agg_atomic(fn, e + 1 + a, v, (unsigned long long)__popc(grp));
-      }
+      if (lane == leader)
+        group_update(p, sagg, gk[r], true, (unsigned long long)__popc(grp), [&](int a) { return vals[a]; });
       multi &= ~grp;
     }
   }
@@ -453,9 +469,9 @@ __device__ __forceinline__ void sink_materialise(const KPlan& p, const char* sta
     base = 0;  // per-row atomics below (A2)
   } else {
     if (lane == 0) s_wtot[warp] = wtot;
-    consumer_bar();
+    consumer_bar(p.nw);
     if (warp == 0) {
-      int v = lane < NW ? s_wtot[lane] : 0;
+      int v = lane < p.nw ? s_wtot[lane] : 0;
       int incl = v;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
@@ -466,9 +482,9 @@ __device__ __forceinline__ void sink_materialise(const KPlan& p, const char* sta
       unsigned long long g = 0;
       if (lane == 0 && total > 0) g = atomicAdd(p.counter, (unsigned long long)total);  // global propagation
       g = __shfl_sync(FULLMASK, g, 0);
-      if (lane < NW) s_base[lane] = g + (unsigned long long)(incl - v);
+      if (lane < p.nw) s_base[lane] = g + (unsigned long long)(incl - v);
     }
-    consumer_bar();
+    consumer_bar(p.nw);
     base = s_base[warp];
   }
   const uint32_t lt = lanemask_lt();
@@ -505,9 +521,10 @@ __global__ void __launch_bounds__(NTHREADS, 1) hq_fused_pipeline_kernel(const __
   extern __shared__ __align__(128) char smem[];
   uint64_t* full = (uint64_t*)smem;
   uint64_t* empty = full + MAX_STAGES;
-  unsigned long long* s_base = (unsigned long long*)(empty + MAX_STAGES);  // [NW]
-  int* s_wtot = (int*)(s_base + NW);                                         // [NW]
-  long long* s_red = (long long*)(s_wtot + NW);                              // [NW][1+MAX_AGGS]
+  unsigned long long* s_base = (unsigned long long*)(empty + MAX_STAGES);  // [NW max]
+  int* s_wtot = (int*)(s_base + NW);                                         // [NW max]
+  long long* s_red = (long long*)(s_wtot + NW);                              // [NW max][1+MAX_AGGS]
+  const int nw = p.nw;
   char* tmp = smem + p.off_tmp;
   char* sagg = smem + p.off_agg;
   char* stages = smem + p.off_stage;
@@ -521,23 +538,30 @@ __global__ void __launch_bounds__(NTHREADS, 1) hq_fused_pipeline_kernel(const __
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NW);
+      mbar_init(&empty[s], nw);
     }
     fence_mbar_init();
   }
   // smem pre-aggregation table: identities
-  if (SK == SK_GROUP && warp < NW && p.smode != SM_NONE) {
-    if (p.smode == SM_DENSE) {
+  if (SK == SK_GROUP && warp < nw && p.smode != SM_NONE) {
+    if (p.smode == SM_LANE) {
       long long* t = (long long*)sagg;
-      for (uint32_t i = threadIdx.x; i < p.smem_cap * p.vwords; i += NW * 32) {
+      const uint32_t nl = nw * 32, n = p.smem_cap * p.nacc * nl;
+      for (uint32_t i = threadIdx.x; i < n; i += nl) {
+        const uint32_t a = (i / nl) % p.nacc;
+        t[i] = a == 0 ? 0 : agg_identity(p.acc_fn[a]);
+      }
+    } else if (p.smode == SM_DENSE) {
+      long long* t = (long long*)sagg;
+      for (uint32_t i = threadIdx.x; i < p.smem_cap * p.vwords; i += nw * 32) {
         const uint32_t c = i % p.vwords;
         t[i] = c == 0 ? 0 : agg_identity(p.agg_fn[c - 1]);
       }
     } else {
       unsigned long long* keys = (unsigned long long*)sagg;
       long long* ent = (long long*)sagg + p.smem_cap;
-      for (uint32_t i = threadIdx.x; i < p.smem_cap; i += NW * 32) keys[i] = EMPTY_KEY;
-      for (uint32_t i = threadIdx.x; i < p.smem_cap * p.vwords; i += NW * 32) {
+      for (uint32_t i = threadIdx.x; i < p.smem_cap; i += nw * 32) keys[i] = EMPTY_KEY;
+      for (uint32_t i = threadIdx.x; i < p.smem_cap * p.vwords; i += nw * 32) {
         const uint32_t c = i % p.vwords;
         ent[i] = c == 0 ? 0 : agg_identity(p.agg_fn[c - 1]);
       }
@@ -545,7 +569,7 @@ __global__ void __launch_bounds__(NTHREADS, 1) hq_fused_pipeline_kernel(const __
   }
   __syncthreads();
 
-  if (warp == NW) {
+  if (warp == nw) {
     // ------------------------------------------------ TMA producer warp
     if (lane == 0) {
       const uint64_t pol = policy_evict_first();
@@ -668,13 +692,13 @@ __global__ void __launch_bounds__(NTHREADS, 1) hq_fused_pipeline_kernel(const __
 #pragma unroll
         for (int a = 0; a < HQ_MAX_AGGS; ++a) s_red[warp * (1 + HQ_MAX_AGGS) + 1 + a] = red[a];
       }
-      consumer_bar();
+      consumer_bar(nw);
       if (threadIdx.x == 0) {
         unsigned long long cnt = 0;
         long long vals[HQ_MAX_AGGS];
 #pragma unroll
         for (int a = 0; a < HQ_MAX_AGGS; ++a) vals[a] = a < p.naggs ? agg_identity(p.agg_fn[a]) : 0;
-        for (int w = 0; w < NW; ++w) {
+        for (int w = 0; w < nw; ++w) {
           cnt += (unsigned long long)s_red[w * (1 + HQ_MAX_AGGS)];
 #pragma unroll
           for (int a = 0; a < HQ_MAX_AGGS; ++a)
@@ -684,17 +708,35 @@ __global__ void __launch_bounds__(NTHREADS, 1) hq_fused_pipeline_kernel(const __
       }
     } else if (SK == SK_GROUP && p.smode != SM_NONE) {
       // C3: merge the block's pre-aggregates into the global table
-      consumer_bar();
-      if (p.smode == SM_DENSE) {
+      consumer_bar(nw);
+      if (p.smode == SM_LANE) {
+        const int nl = nw * 32;
         const long long* t = (const long long*)sagg;
-        for (uint32_t g = threadIdx.x; g < p.smem_cap; g += NW * 32) {
+        for (uint32_t g = threadIdx.x; g < p.smem_cap; g += nl) {
+          const long long* e = t + (size_t)g * p.nacc * nl;
+          unsigned long long cnt = 0;
+          for (int l = 0; l < nl; ++l) cnt += (unsigned long long)e[l];
+          if (!cnt) continue;
+          long long acc[HQ_MAX_AGGS + 1];
+          for (int a = 1; a < p.nacc; ++a) {
+            long long v = agg_identity(p.acc_fn[a]);
+            for (int l = 0; l < nl; ++l) v = agg_combine(p.acc_fn[a], v, e[a * nl + l]);
+            acc[a] = v;
+          }
+          long long vals[HQ_MAX_AGGS];
+          for (int k = 0; k < p.naggs; ++k) vals[k] = p.acc_of[k] ? acc[p.acc_of[k]] : (long long)cnt;
+          global_update(p, g, cnt, vals);
+        }
+      } else if (p.smode == SM_DENSE) {
+        const long long* t = (const long long*)sagg;
+        for (uint32_t g = threadIdx.x; g < p.smem_cap; g += nw * 32) {
           const long long* e = t + (size_t)g * p.vwords;
           if (e[0] != 0) global_update(p, g, (unsigned long long)e[0], e + 1);
         }
       } else {
         const unsigned long long* keys = (const unsigned long long*)sagg;
         const long long* ent = (const long long*)sagg + p.smem_cap;
-        for (uint32_t h = threadIdx.x; h < p.smem_cap; h += NW * 32) {
+        for (uint32_t h = threadIdx.x; h < p.smem_cap; h += nw * 32) {
           if (keys[h] != EMPTY_KEY) {
             const long long* e = ent + (size_t)h * p.vwords;
             global_update(p, keys[h], (unsigned long long)e[0], e + 1);
@@ -728,7 +770,8 @@ int64_t fused_smem_bytes(const KPlan& kp) {
 template <int R, int SK>
 static void launch_one(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
   HQ_CUDA(cudaFuncSetAttribute(hq_fused_pipeline_kernel<R, SK>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  hq_fused_pipeline_kernel<R, SK><<<grid, NTHREADS, smem, ctx->stream>>>(kp);
+  ctx->launches++;
+  hq_fused_pipeline_kernel<R, SK><<<grid, (kp.nw + 1) * 32, smem, ctx->stream>>>(kp);
 }
 
 void launch_fused(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
@@ -752,6 +795,7 @@ void launch_init_groups(hq_ctx* ctx, long long* tab, int64_t ngroups, uint32_t v
   const long long total = ngroups * (long long)(vwords + (hash ? 1 : 0));
   int grid = (int)std::min<long long>((total + 255) / 256, (long long)ctx->num_sms * 8);
   if (grid < 1) grid = 1;
+  ctx->launches++;
   hq_init_groups_kernel<<<grid, 256, 0, ctx->stream>>>(tab, ngroups, vwords, hash ? 1 : 0, fns);
   HQ_CUDA(cudaGetLastError());
 }

@@ -75,7 +75,7 @@ int hq_type_width(int type) {
 }
 
 // Build the device plan; allocates the result's sink buffers on first use.
-static void build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int64_t mat_cap) {
+void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int64_t mat_cap) {
   const hq_plan& P = r->plan;
   const hq_table* F = r->fact;
   std::memset(&kp, 0, sizeof(kp));
@@ -123,7 +123,9 @@ static void build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap,
       KProbe& pr = kp.probes[nprobe];
       pr.key_reg = (int16_t)use(op.key_reg, "probe key");
       pr.slots = op.ht->slots;
-      pr.mask = (uint32_t)(op.ht->meta.capacity - 1);
+      pr.direct = op.ht->meta.layout == HQ_HT_DIRECT;
+      pr.mask = pr.direct ? (uint32_t)op.ht->meta.capacity : (uint32_t)(op.ht->meta.capacity - 1);
+      pr.dmin = (int32_t)op.ht->meta.key_min;
       pr.log2cap = (uint8_t)op.ht->log2cap;
       pr.words = (uint8_t)op.ht->meta.slot_words;
       pr.mode = (uint8_t)op.mode;
@@ -207,10 +209,35 @@ static void build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap,
     const size_t gbytes = (size_t)r->ngroups * (kp.vwords + (kp.gmode == GM_HASH ? 1 : 0)) * 8;
     if (!r->gtab.p || r->gtab.bytes < gbytes) r->gtab = DevBuf(ctx, gbytes);
     kp.gtab = r->gtab.as<long long>();
+    // deduplicated accumulators for the lane-private mode: 0 = count,
+    // SUM/AVG of one register share one sum, MIN/MAX get their own
+    kp.nacc = 1;
+    kp.acc_fn[0] = HQ_AGG_COUNT;
+    kp.acc_reg[0] = 0;
+    for (int a = 0; a < P.naggs; ++a) {
+      const uint8_t cls = (P.agg_fn[a] == HQ_AGG_AVG) ? (uint8_t)HQ_AGG_SUM : (uint8_t)P.agg_fn[a];
+      if (cls == HQ_AGG_COUNT) { kp.acc_of[a] = 0; continue; }
+      int found = -1;
+      for (int k = 1; k < kp.nacc; ++k)
+        if (kp.acc_fn[k] == cls && kp.acc_reg[k] == kp.agg_reg[a]) found = k;
+      if (found < 0) {
+        found = kp.nacc++;
+        kp.acc_fn[found] = cls;
+        kp.acc_reg[found] = kp.agg_reg[a];
+      }
+      kp.acc_of[a] = (uint8_t)found;
+    }
     // local-resolution table in shared memory
     kp.smode = SM_NONE;
     if (P.nkeys > 0 && P.resolution == HQ_RES_LRGP) {
-      if (kp.gmode == GM_DENSE && (uint64_t)ngroups * kp.vwords * 8 <= (uint64_t)SMEM_AGG_BYTES) {
+      // lane-private tables halve the warps, so only for probe-free pipelines
+      // (no latency to hide) whose group domain is tiny
+      if (kp.gmode == GM_DENSE && nprobe == 0 && !getenv("HQ_DEBUG_NOLANE") &&
+          (uint64_t)ngroups * kp.nacc * LANE_NW * 32 * 8 <= (uint64_t)SMEM_LANE_BYTES) {
+        kp.smode = SM_LANE;  // tiny domain (e.g. TPC-H Q1): contention-free lane-private tables
+        kp.smem_cap = (uint32_t)ngroups;
+        agg_smem = (uint32_t)(ngroups * kp.nacc * LANE_NW * 32 * 8);
+      } else if (kp.gmode == GM_DENSE && (uint64_t)ngroups * kp.vwords * 8 <= (uint64_t)SMEM_AGG_BYTES) {
         kp.smode = SM_DENSE;
         kp.smem_cap = (uint32_t)ngroups;
         agg_smem = (uint32_t)(ngroups * kp.vwords * 8);
@@ -256,9 +283,11 @@ static void build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap,
   uint32_t tmp_row = 0;
   for (int k = 0; k < HQ_MAX_TMP; ++k) tmp_row += (uint32_t)regs[HQ_MAX_COLS + k].width;
 
+  kp.nw = kp.smode == SM_LANE ? LANE_NW : NW;
+  if (const char* e = getenv("HQ_DEBUG_NW")) kp.nw = atoi(e);  // debugging aid
   int chosen_R = 0;
   for (int R : {4, 2}) {
-    const uint32_t T = (uint32_t)(NW * 32 * R);
+    const uint32_t T = (uint32_t)(kp.nw * 32 * R);
     const uint32_t off_tmp = MISC_BYTES;
     const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
     const uint32_t off_stage = align_up(off_agg + agg_smem, 128);
@@ -303,7 +332,7 @@ static void build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap,
 
 static void launch_pipeline(hq_ctx* ctx, hq_result* r, int64_t group_cap, int64_t mat_cap) {
   KPlan kp;
-  build_kplan(ctx, r, kp, group_cap, mat_cap);
+  hq_build_kplan(ctx, r, kp, group_cap, mat_cap);
   HQ_CUDA(cudaMemsetAsync(r->dstate.p, 0, r->dstate.bytes, ctx->stream));
   if (r->plan.sink == HQ_SINK_AGG)
     launch_init_groups(ctx, kp.gtab, r->ngroups, kp.vwords, kp.gmode == GM_HASH, kp.agg_fn, kp.naggs);

@@ -1,0 +1,115 @@
+"""Multi-GPU orchestration: one process per GPU.
+
+* the fact table is range-partitioned: rank r owns rows [r*N/P, (r+1)*N/P);
+  the generator is partition-invariant, so the union equals the P=1 input;
+* dimension hash tables are built once on the root and broadcast as raw slot
+  arrays (``hq_hash_device_view`` -> ``dist.broadcast`` over NCCL/NVLink ->
+  ``hq_hash_import``); build-side pipelines (e.g. TPC-H Q3's orders side) run
+  on the root only;
+* each rank runs the fused pipeline over its range; dense partial aggregates
+  ([count, agg...] per group, int64) are combined with ONE ``dist.reduce``
+  (SUM) to the root, which finalizes (ORDER BY / LIMIT on GPU 0).
+
+The collectives here are backend-agnostic torch.distributed calls (NCCL on the
+GPUs; the CPU tests drive the same functions with gloo and a test-only
+stand-in for the device engine).  The paper itself is single-device; this is
+new (north_star).
+"""
+from __future__ import annotations
+
+from typing import List, Optional, Sequence, Tuple
+
+import torch
+import torch.distributed as dist
+
+from . import hq
+from .engine import Engine, PlanBuilder, QueryResult, fetch
+
+
+def partition(n: int, rank: int, world: int) -> Tuple[int, int]:
+    """Row range of `rank` in a range partition of n rows over `world` ranks."""
+    return n * rank // world, n * (rank + 1) // world
+
+
+def broadcast_blob(meta: Optional[Sequence[int]], buf: Optional[torch.Tensor], nbytes_index: int,
+                   root: int, device) -> Tuple[List[int], torch.Tensor]:
+    """Broadcast a small int64 meta vector, then a byte buffer whose size is
+    meta[nbytes_index].  Non-root ranks pass meta=None, buf=None."""
+    rank = dist.get_rank()
+    m = torch.zeros(8, dtype=torch.int64, device=device)
+    if rank == root:
+        m[: len(meta)] = torch.tensor(list(meta), dtype=torch.int64)
+    dist.broadcast(m, src=root)
+    meta_out = [int(x) for x in m.tolist()]
+    nbytes = meta_out[nbytes_index]
+    if rank != root:
+        buf = torch.empty(nbytes, dtype=torch.uint8, device=device)
+    dist.broadcast(buf, src=root)
+    return meta_out, buf
+
+
+def reduce_partials(t: torch.Tensor, root: int) -> None:
+    """Exact integer SUM of the ranks' partial aggregates onto the root."""
+    dist.reduce(t, dst=root, op=dist.ReduceOp.SUM)
+
+
+class _CudaView:
+    """Zero-copy torch view of a library-owned device buffer."""
+
+    def __init__(self, ptr: int, n: int, typestr: str):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3}
+
+
+def device_view(ptr: int, nbytes: int, dtype=torch.uint8) -> torch.Tensor:
+    typestr = {torch.uint8: "|u1", torch.int64: "<i8"}[dtype]
+    n = nbytes // (1 if dtype == torch.uint8 else 8)
+    return torch.as_tensor(_CudaView(ptr, n, typestr), device="cuda")
+
+
+class DistributedEngine(Engine):
+    """Engine whose builds happen on the root and are broadcast, and whose
+    partitioned pipelines end with one reduce of the dense partials."""
+
+    def __init__(self, ctx: hq.Context, tables, root: int = 0, **kw):
+        super().__init__(ctx, tables, **kw)
+        self.rank = dist.get_rank()
+        self.world = dist.get_world_size()
+        self.root = root
+        self.device = torch.device("cuda", ctx.device)
+
+    def _share(self, h: Optional[hq.Hash]) -> hq.Hash:
+        if self.rank == self.root:
+            m = h.info()  # syncs, reports build faults before anything is sent
+            ptr, _ = h.device_view()
+            buf = device_view(ptr, int(m.bytes))
+            meta = [m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout]
+        else:
+            meta, buf = None, None
+        meta, buf = broadcast_blob(meta, buf, 4, self.root, self.device)
+        if self.rank == self.root:
+            return h
+        hm = hq.HashMeta()
+        hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout = meta[:7]
+        return self.ctx.import_hash(hm, buf.data_ptr(), keep=buf)
+
+    def hash(self, table, key, payload=(), preds=(), expected_rows=0) -> hq.Hash:
+        h = super().hash(table, key, payload, preds, expected_rows) if self.rank == self.root else None
+        return self._share(h)
+
+    def hash_from(self, res, names, key, payload=()) -> hq.Hash:
+        h = super().hash_from(res, names, key, payload) if self.rank == self.root else None
+        return self._share(h)
+
+    def run(self, pb: PlanBuilder, partitioned: bool = True) -> Optional[hq.Result]:
+        if not partitioned and self.rank != self.root:
+            return None
+        return super().run(pb, partitioned)
+
+    def finish(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
+        """Reduce the dense partials onto the root and finalize there."""
+        ptr, nbytes = res.partials_view()
+        t = device_view(ptr, nbytes, torch.int64)
+        reduce_partials(t, self.root)
+        if self.rank != self.root:
+            return None
+        return fetch(res, pb.result_names)

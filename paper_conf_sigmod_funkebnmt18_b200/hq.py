@@ -62,7 +62,8 @@ class BuildDesc(ctypes.Structure):
 
 class HashMeta(ctypes.Structure):
     _fields_ = [("capacity", ctypes.c_int64), ("slot_words", ctypes.c_int32), ("npayload", ctypes.c_int32),
-                ("nkeys", ctypes.c_int64), ("bytes", ctypes.c_int64)]
+                ("nkeys", ctypes.c_int64), ("bytes", ctypes.c_int64), ("key_min", ctypes.c_int64),
+                ("layout", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 class Insn(ctypes.Structure):
@@ -110,7 +111,8 @@ STRUCTS = {"hq_column": Column, "hq_pred": Pred, "hq_build_desc": BuildDesc, "hq
 
 # every symbol include/hq.h declares
 EXPORTS = ["hq_ctx_create", "hq_ctx_destroy", "hq_ctx_set_stream", "hq_ctx_sync", "hq_last_error",
-           "hq_abi_version", "hq_sizeof", "hq_ctx_enable_timing", "hq_ctx_kernel_times", "hq_load_columns",
+           "hq_abi_version", "hq_sizeof", "hq_ctx_enable_timing", "hq_ctx_kernel_times", "hq_ctx_launches",
+           "hq_load_columns",
            "hq_table_info", "hq_table_column", "hq_free_table", "hq_build_hash", "hq_hash_info",
            "hq_hash_device_view", "hq_hash_import", "hq_free_hash", "hq_run_pipeline", "hq_finalize",
            "hq_result_info_get", "hq_fetch_result", "hq_result_as_table", "hq_result_partials_view",
@@ -139,6 +141,7 @@ def lib():
             "hq_ctx_destroy": [vp], "hq_ctx_set_stream": [vp, vp], "hq_ctx_sync": [vp],
             "hq_ctx_enable_timing": [vp, i32],
             "hq_ctx_kernel_times": [vp, P(ctypes.c_float), i32, P(i32)],
+            "hq_ctx_launches": [vp, P(i64)],
             "hq_load_columns": [vp, P(Column), i32, i64, i32, P(vp)],
             "hq_table_info": [vp, P(i64), P(i32)], "hq_table_column": [vp, i32, P(vp), P(i32)],
             "hq_free_table": [vp], "hq_build_hash": [vp, P(BuildDesc), P(vp)],
@@ -220,6 +223,12 @@ class Context:
         n = ctypes.c_int32()
         check(lib().hq_ctx_kernel_times(self.h, buf, max_n, ctypes.byref(n)))
         return list(buf[: min(n.value, max_n)])
+
+    def launches(self) -> int:
+        """Cumulative number of kernels launched by this context."""
+        n = ctypes.c_int64()
+        check(lib().hq_ctx_launches(self.h, ctypes.byref(n)))
+        return int(n.value)
 
     def close(self) -> None:
         if getattr(self, "h", None):

@@ -1,0 +1,100 @@
+"""Multi-process orchestration on CPU (gloo, world_size 2): the same
+range-partition / broadcast / reduce functions the NCCL path uses
+(paper_conf_sigmod_funkebnmt18_b200.dist), with a TEST-ONLY numpy stand-in for
+the device engine's partial aggregates.  Pins: the reduced partials of the two
+ranks equal the oracle on the whole table; broadcast blobs arrive intact."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import hqgen
+from paper_conf_sigmod_funkebnmt18_b200.dist import broadcast_blob, partition, reduce_partials
+
+SF = 0.01
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _q41_partials(lo, c, s, p, d):
+    """Test-only stand-in for the fused kernel's dense partial table: [count, profit]
+    per (d_year, c_nation) group, same layout as hq_result_partials_view."""
+    creg = c["c_region"][lo["lo_custkey"] - 1]
+    sreg = s["s_region"][lo["lo_suppkey"] - 1]
+    pm = p["p_mfgr"][lo["lo_partkey"] - 1]
+    m = (creg == 1) & (sreg == 1) & (pm <= 1)
+    year = lo["lo_orderdate"][m] // 10000
+    nat = c["c_nation"][lo["lo_custkey"][m] - 1].astype(np.int64)
+    g = (year - 1992) * 25 + nat
+    t = np.zeros((175, 2), np.int64)
+    np.add.at(t[:, 0], g, 1)
+    np.add.at(t[:, 1], g, lo["lo_revenue"][m].astype(np.int64) - lo["lo_supplycost"][m])
+    return t
+
+
+def _worker(rank, world, port, q):
+    try:
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        n = hqgen.table_rows("lineorder", SF)
+        a, b = partition(n, rank, world)
+        lo = hqgen.generate("lineorder", SF, row_range=(a, b))
+        dims = {t: hqgen.generate(t, SF) for t in ("customer", "supplier", "part", "date")}
+        # root "builds" and broadcasts a blob (the hash-table slot array on GPUs)
+        blob = np.ascontiguousarray(dims["customer"]["c_custkey"][dims["customer"]["c_region"] == 1]).view(np.uint8)
+        if rank == 0:
+            meta, buf = broadcast_blob([7, 2, 1, 0, blob.nbytes], torch.from_numpy(blob.copy()), 4, 0, "cpu")
+        else:
+            meta, buf = broadcast_blob(None, None, 4, 0, "cpu")
+        assert meta[:5] == [7, 2, 1, 0, blob.nbytes]
+        assert np.array_equal(buf.numpy(), blob)
+        part = torch.from_numpy(_q41_partials(lo, dims["customer"], dims["supplier"], dims["part"], dims["date"]).ravel().copy())
+        reduce_partials(part, 0)
+        if rank == 0:
+            q.put(("ok", part.numpy().reshape(175, 2), (a, b)))
+        else:
+            q.put(("ok", None, (a, b)))
+        dist.barrier()
+        dist.destroy_process_group()
+    except Exception as e:  # pragma: no cover
+        q.put(("err", repr(e), None))
+
+
+def test_partition_covers_range():
+    for n in (0, 1, 7, 1000, 600_037_902):
+        for w in (1, 2, 3, 8):
+            parts = [partition(n, r, w) for r in range(w)]
+            assert parts[0][0] == 0 and parts[-1][1] == n
+            assert all(parts[i][1] == parts[i + 1][0] for i in range(w - 1))
+
+
+def test_two_rank_reduce_matches_oracle():
+    import oracle
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    outs = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    assert all(o[0] == "ok" for o in outs), outs
+    table = next(o[1] for o in outs if o[1] is not None)
+    ranges = sorted(o[2] for o in outs)
+    assert ranges[0][0] == 0 and ranges[0][1] == ranges[1][0]
+    ssb = {t: hqgen.generate(t, SF) for t in hqgen.SSB_TABLES}
+    ref = oracle.ssb_q41(ssb["lineorder"], ssb["date"], ssb["customer"], ssb["supplier"], ssb["part"])
+    got = [(1992 + g // 25, g % 25, int(table[g, 1]), int(table[g, 0])) for g in range(175) if table[g, 0] > 0]
+    assert got == ref.rows()

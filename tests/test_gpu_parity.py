@@ -113,6 +113,21 @@ def test_ssb_q31_materialise_parity(ctx, ssb):
     assert int(g.columns["lo_revenue"].astype(np.int64).sum()) == int(a.columns["revenue"].sum())
 
 
+@pytest.mark.parametrize("qname", ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q31", "ssb_q41", "tpch_q3"])
+def test_operator_at_a_time_parity(ctx, ssb, tpch, qname):
+    """The op-at-a-time baseline (a11) of the same plan == oracle (two independent GPU paths)."""
+    host = host_for(qname, ssb, tpch)
+    kw = {"limit": 0} if qname == "tpch_q3" else {}
+    g = gpu_run(ctx, qname, host, exec_mode=hq.EXEC_OAAT, **kw)
+    assert_same(qname, g, oracle_run(qname, host))
+
+
+def test_operator_at_a_time_materialise(ctx, ssb):
+    g = gpu_run(ctx, "ssb_q31_mat", ssb, exec_mode=hq.EXEC_OAAT)
+    o = oracle_run("ssb_q31_mat", ssb)
+    assert sorted(g.rows(["c_nation", "s_nation", "d_year", "lo_revenue"])) == o.rows()
+
+
 @pytest.mark.parametrize("qname", ["ssb_q41", "tpch_q1", "ssb_q11"])
 def test_resolution_ablation_identical(ctx, ssb, tpch, qname):
     host = host_for(qname, ssb, tpch)
