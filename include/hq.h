@@ -234,7 +234,13 @@ typedef enum { HQ_SINK_AGG = 1, HQ_SINK_MATERIALISE = 2 } hq_sink_kind;
  *        one atomic per block and tile (A3, B3, C3) -- the default;
  * ATOMIC = per-row global atomics (A2, B2, C2), kept as an ablation. */
 typedef enum { HQ_RES_LRGP = 0, HQ_RES_ATOMIC = 1 } hq_resolution;
-typedef enum { HQ_EXEC_FUSED = 0, HQ_EXEC_OAAT = 1 } hq_exec;
+/* Execution of a plan:
+ * FUSED        one compound kernel, compiled for this plan with NVRTC (query
+ *              compilation); falls back to FUSED_INTERP
+ *              only if HQ_JIT=0 is set in the environment;
+ * OAAT         operator-at-a-time baseline (Fig 6);
+ * FUSED_INTERP the same compound kernel as a precompiled descriptor interpreter. */
+typedef enum { HQ_EXEC_FUSED = 0, HQ_EXEC_OAAT = 1, HQ_EXEC_FUSED_INTERP = 2 } hq_exec;
 
 typedef struct {
   const hq_table* fact;

@@ -24,7 +24,8 @@ def sources():
 
 
 def headers():
-    return sorted(glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(ROOT, "include", "*.h")))
+    return sorted(glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh")) +
+                  glob.glob(os.path.join(ROOT, "include", "*.h")))
 
 
 def up_to_date() -> bool:
@@ -34,11 +35,24 @@ def up_to_date() -> bool:
     return all(os.path.getmtime(f) <= t for f in sources() + headers())
 
 
+def embed_prelude() -> None:
+    """hq_jit_prelude.cuh -> hq_jit_prelude.inc (a raw string literal for NVRTC)."""
+    src = os.path.join(CSRC, "hq_jit_prelude.cuh")
+    dst = os.path.join(CSRC, "hq_jit_prelude.inc")
+    text = 'R"HQJIT(' + open(src).read() + ')HQJIT"\n'
+    if not os.path.exists(dst) or open(dst).read() != text:
+        with open(dst, "w") as f:
+            f.write(text)
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
+    embed_prelude()
     if not force and up_to_date():
         return SO
+    cudalib = os.path.join(os.path.dirname(os.path.dirname(NVCC)), "lib64")
     cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
-           "-I" + os.path.join(ROOT, "include"), "-o", SO + ".tmp", *sources()]
+           "-I" + os.path.join(ROOT, "include"), "-o", SO + ".tmp", *sources(),
+           "-L" + cudalib, "-lnvrtc", "-Xlinker", "-rpath," + cudalib]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     r = subprocess.run(cmd, capture_output=True, text=True)

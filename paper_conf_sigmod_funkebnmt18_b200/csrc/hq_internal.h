@@ -279,6 +279,12 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r);
 void hq_run_oaat(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
 // shared plan preparation (hq_plan.cu)
 void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
-void hq_build_kplan(hq_ctx* ctx, hq_result* r, hqk::KPlan& kp, int64_t group_cap, int64_t mat_cap);
+void hq_build_kplan(hq_ctx* ctx, hq_result* r, hqk::KPlan& kp, int64_t group_cap, int64_t mat_cap,
+                    bool jit = false);
+// query compilation (hq_jit.cu): NVRTC-specialised fused kernels
+bool hq_jit_enabled();
+void hq_jit_prepare(hq_ctx* ctx, const hqk::KPlan& kp, size_t smem);  // compile (cached) + attributes
+void hq_jit_launch(hq_ctx* ctx, const hqk::KPlan& kp, int grid, size_t smem);
+std::string hq_jit_source(const hqk::KPlan& kp);
 void hq_check_result_faults(hq_ctx* ctx, hq_result* r);
 int hq_type_width(int type);

@@ -1,0 +1,546 @@
+// hq_jit.cu -- query compilation of a fusion operator into a specialised
+// sm_100a kernel with NVRTC (§4.3 code templates + code frame,
+// P:652-704; §5.2 compound-kernel code generation).
+//
+// The validated device plan (KPlan, hq_plan.cu) is turned into CUDA source:
+// the code frame is the same persistent TMA-ring kernel as the interpreter
+// (hq_pipeline.cu) -- producer warp, mbarrier full/empty ring, ragged tiles,
+// LRGP sinks -- but every operator becomes straight-line code with its
+// constants folded, columns loaded from the stage on first use and
+// temporaries (probe payloads, expression results) kept in registers.  The
+// source is compiled once per distinct plan shape (cached by source text),
+// loaded with the driver API (entry points from cudaGetDriverEntryPoint, so
+// libhq does not link libcuda) and launched on the context stream.
+#include <cuda.h>
+#include <nvrtc.h>
+
+#include <climits>
+#include <map>
+#include <mutex>
+#include <set>
+#include <sstream>
+
+#include "hq_internal.h"
+
+using namespace hqk;
+
+// kernel parameters of every generated kernel (mirrored in the generated source)
+#define HQ_JPARAMS_DEF                                                                                         \
+  struct JParams {                                                                                             \
+    long long row_begin, row_end;                                                                              \
+    const char* col[16];                                                                                       \
+    const unsigned* ht[8];                                                                                     \
+    long long* gtab;                                                                                           \
+    unsigned long long gmask;                                                                                  \
+    int glog2, pad;                                                                                            \
+    void* out[8];                                                                                              \
+    long long capacity;                                                                                        \
+    unsigned long long* counter;                                                                               \
+    int* err;                                                                                                  \
+  };
+HQ_JPARAMS_DEF
+#define HQ_XSTR(...) #__VA_ARGS__
+#define HQ_STR(...) HQ_XSTR(__VA_ARGS__)
+
+namespace {
+
+const char* kPrelude =
+#include "hq_jit_prelude.inc"
+    ;
+
+// ---- driver API through the runtime's entry-point query
+typedef CUresult (*PFN_modload)(CUmodule*, const void*);
+typedef CUresult (*PFN_getfn)(CUfunction*, CUmodule, const char*);
+typedef CUresult (*PFN_setattr)(CUfunction, CUfunction_attribute, int);
+typedef CUresult (*PFN_launch)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                               CUstream, void**, void**);
+struct Driver {
+  PFN_modload modload = nullptr;
+  PFN_getfn getfn = nullptr;
+  PFN_setattr setattr = nullptr;
+  PFN_launch launch = nullptr;
+};
+template <class F>
+F entry(const char* name) {
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
+    cudaGetLastError();
+    HQ_THROW(HQ_ERR_CUDA, std::string("driver entry point missing: ") + name);
+  }
+  return (F)fn;
+}
+Driver& driver() {
+  static Driver d;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    d.modload = entry<PFN_modload>("cuModuleLoadData");
+    d.getfn = entry<PFN_getfn>("cuModuleGetFunction");
+    d.setattr = entry<PFN_setattr>("cuFuncSetAttribute");
+    d.launch = entry<PFN_launch>("cuLaunchKernel");
+  });
+  return d;
+}
+
+std::mutex g_mu;
+std::map<std::pair<int, std::string>, CUfunction> g_cache;  // (device, source) -> kernel
+
+// ------------------------------------------------------------------ codegen
+std::string lit(long long v) {
+  if (v == LLONG_MIN) return "HQ_LL_MIN";
+  return std::to_string(v) + "LL";
+}
+const char* ctype(int w) { return w == 1 ? "signed char" : (w == 4 ? "int" : "long long"); }
+
+struct Gen {
+  const KPlan& kp;
+  std::ostringstream o;
+  std::set<int> loaded;        // registers materialised as variables
+  std::map<int, int> stage_k;  // table column -> stage column index
+  explicit Gen(const KPlan& k) : kp(k) {
+    for (int c = 0; c < HQ_MAX_COLS; ++c) {
+      if (!kp.regs[c].in_stage || !kp.regs[c].width) continue;
+      for (int k2 = 0; k2 < kp.ncols; ++k2)
+        if (kp.cols[k2].soff == kp.regs[c].off) stage_k[c] = k2;
+    }
+  }
+  std::string var(int reg) const { return reg < HQ_MAX_COLS ? "c" + std::to_string(reg) : "t" + std::to_string(reg - HQ_MAX_COLS); }
+  int width(int reg) const { return kp.regs[reg].width; }
+  // value of register `reg` for row slot r, as a C++ expression
+  std::string val(int reg) {
+    use(reg);
+    return var(reg) + "[r]";
+  }
+  void use(int reg) {
+    if (loaded.count(reg)) return;
+    if (reg >= HQ_MAX_COLS) HQ_THROW(HQ_ERR_ARG, "jit: temporary read before definition");
+    const KCol& c = kp.cols[stage_k.at(reg)];
+    o << "      " << ctype(c.width) << " " << var(reg) << "[R];\n"
+      << "      { const " << ctype(c.width) << "* b_ = (const " << ctype(c.width) << "*)(st + " << c.soff
+      << "u) + row0;\n#pragma unroll\n        for (int r = 0; r < R; ++r) " << var(reg) << "[r] = b_[r * 32]; }\n";
+    loaded.insert(reg);
+  }
+  void early_exit() { o << "      if (!__any_sync(HQ_FULL, mask)) break;\n"; }
+
+  void filter(const KPred& f, int idx) {
+    std::string cond;
+    if (f.kind == 0) {
+      const bool narrow = width(f.reg) <= 4;
+      std::string v = narrow ? "(int)" + val(f.reg) : "(long long)" + val(f.reg);
+      if (narrow) {
+        if (f.lo32 > f.hi32) cond = "false";
+        else if (f.lo32 == f.hi32) cond = v + " == " + std::to_string(f.lo32);
+        else {
+          std::string a = f.lo32 == INT_MIN ? "" : v + " >= " + std::to_string(f.lo32);
+          std::string b = f.hi32 == INT_MAX ? "" : v + " <= " + std::to_string(f.hi32);
+          cond = a.empty() ? (b.empty() ? "true" : b) : (b.empty() ? a : a + " && " + b);
+        }
+      } else {
+        if (f.lo > f.hi) cond = "false";
+        else {
+          std::string a = f.lo == LLONG_MIN ? "" : v + " >= " + lit(f.lo);
+          std::string b = f.hi == LLONG_MAX ? "" : v + " <= " + lit(f.hi);
+          cond = a.empty() ? (b.empty() ? "true" : b) : (b.empty() ? a : a + " && " + b);
+        }
+      }
+      if (f.neg) cond = "!(" + cond + ")";
+    } else {
+      std::string v = "(unsigned long long)(long long)" + val(f.reg);
+      const std::string bm = "BM_" + std::to_string(idx);
+      cond = "(" + v + " < 256ull && ((" + bm + "[" + v + " >> 6] >> (" + v + " & 63ull)) & 1ull))";
+      bitmaps << "static constexpr __device__ u64 " << bm << "[4] = {" << f.bm[0] << "ull, " << f.bm[1] << "ull, "
+              << f.bm[2] << "ull, " << f.bm[3] << "ull};\n";
+    }
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (!(" << cond << ")) mask &= ~(1u << r);\n";
+    early_exit();
+  }
+
+  void probe(const KProbe& pr, int idx) {
+    const int W = pr.words;
+    const int npay = pr.mode == HQ_PROBE_INNER ? pr.npay : 0;
+    for (int k = 0; k < npay; ++k) {
+      o << "      int " << var(pr.dst[k]) << "[R];\n";
+      loaded.insert(pr.dst[k]);
+    }
+    const std::string key = val(pr.key_reg);
+    o << "      { const u32* ht_ = p.ht[" << idx << "]; u32 found_ = 0u; int kk_[R]; u32 pend_ = 0u; u32 pos_[R];\n"
+      << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n"
+      << "          const long long k_ = (long long)" << key << "; kk_[r] = (int)k_;\n";
+    if (pr.direct) {
+      o << "          const bool ok_ = ((mask >> r) & 1u) && k_ >= " << pr.dmin << "LL && k_ < " << pr.dmin << "LL + "
+        << pr.mask << "LL;\n"
+        << "          pos_[r] = (u32)(k_ - " << pr.dmin << "LL); if (ok_) pend_ |= 1u << r; }\n";
+      o << "        int4 sl_[R];\n#pragma unroll\n        for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) {\n";
+      if (W == 1) o << "          sl_[r].x = __ldg((const int*)ht_ + pos_[r]);\n";
+      else if (W == 2) o << "          const int2 q_ = __ldg((const int2*)ht_ + pos_[r]); sl_[r].x = q_.x; sl_[r].y = q_.y;\n";
+      else o << "          sl_[r] = __ldg((const int4*)ht_ + pos_[r]);\n";
+      o << "        }\n#pragma unroll\n        for (int r = 0; r < R; ++r) if ((pend_ & (1u << r)) && sl_[r].x == kk_[r]) {\n"
+        << "          found_ |= 1u << r;\n";
+      static const char* comp[3] = {"y", "z", "w"};
+      for (int k = 0; k < npay; ++k) o << "          " << var(pr.dst[k]) << "[r] = sl_[r]." << comp[k] << ";\n";
+      o << "        }\n";
+    } else {
+      const int G = W == 1 ? 4 : (W == 2 ? 2 : 1);
+      o << "          const bool ok_ = ((mask >> r) & 1u) && k_ > (long long)HQ_INT_MIN && k_ <= (long long)HQ_INT_MAX;\n"
+        << "          pos_[r] = ((u32)(int)k_ * 0x9E3779B1u) >> " << (32 - pr.log2cap) << "; if (ok_) pend_ |= 1u << r; }\n"
+        << "        while (pend_) {\n          int4 sl_[R];\n"
+        << "#pragma unroll\n          for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) sl_[r] = __ldg((const int4*)ht_ + pos_[r] / "
+        << G << ");\n"
+        << "#pragma unroll\n          for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) {\n"
+        << "            int hit_ = -1; bool stop_ = false; const int first_ = (int)(pos_[r] % " << G << ");\n";
+      const char* keys4[4] = {"x", "y", "z", "w"};
+      for (int j = 0; j < G; ++j) {
+        const char* kc = G == 4 ? keys4[j] : (G == 2 ? (j == 0 ? "x" : "z") : "x");
+        o << "            if (!stop_ && " << j << " >= first_) { if (sl_[r]." << kc << " == kk_[r]) { hit_ = " << j
+          << "; stop_ = true; } else if (sl_[r]." << kc << " == HQ_INT_MIN) stop_ = true; }\n";
+      }
+      o << "            if (hit_ >= 0) { found_ |= 1u << r; pend_ &= ~(1u << r);\n";
+      if (npay > 0) {
+        if (G == 2) o << "              " << var(pr.dst[0]) << "[r] = hit_ == 0 ? sl_[r].y : sl_[r].w;\n";
+        else {
+          static const char* comp[3] = {"y", "z", "w"};
+          for (int k = 0; k < npay; ++k) o << "              " << var(pr.dst[k]) << "[r] = sl_[r]." << comp[k] << ";\n";
+        }
+      }
+      o << "            } else if (stop_) pend_ &= ~(1u << r);\n"
+        << "            else pos_[r] = ((pos_[r] / " << G << " + 1) * " << G << ") & " << pr.mask << "u;\n"
+        << "          }\n        }\n";
+    }
+    o << "        mask = " << (pr.mode == HQ_PROBE_ANTI ? "mask & ~found_" : "mask & found_") << "; }\n";
+    early_exit();
+  }
+
+  std::string operand(const KInsn& in) {
+    if (in.reg < 0) return lit(in.imm);
+    return "(long long)" + val(in.reg);
+  }
+  void compute(const KCompute& c) {
+    // operands first (column loads must not land inside the row loop)
+    std::vector<std::string> ops;
+    for (int k = 0; k < c.n; ++k) ops.push_back(operand(kp.insns[c.first + k]));
+    const std::string dst = var(c.dst);
+    o << "      long long " << dst << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) { long long a_ = 0;\n";
+    for (int k = 0; k < c.n; ++k) {
+      const KInsn& in = kp.insns[c.first + k];
+      const std::string& x = ops[k];
+      switch (in.opc) {
+        case HQ_I_LOAD: o << "        a_ = " << x << ";\n"; break;
+        case HQ_I_ADD: o << "        a_ += " << x << ";\n"; break;
+        case HQ_I_SUB: o << "        a_ -= " << x << ";\n"; break;
+        case HQ_I_RSUB: o << "        a_ = " << x << " - a_;\n"; break;
+        case HQ_I_MUL: o << "        a_ *= " << x << ";\n"; break;
+        default:
+          o << "        { const long long d_ = " << x << "; if (d_ == 0) { if ((mask >> r) & 1u) atomicOr(p.err, F_DIV_ZERO); a_ = 0; }"
+            << " else a_ = a_ " << (in.opc == HQ_I_DIV ? "/" : "%") << " d_; }\n";
+      }
+    }
+    o << "        " << dst << "[r] = a_; }\n";
+    loaded.insert(c.dst);
+  }
+  std::ostringstream bitmaps;
+};
+
+std::string fn_list(const uint8_t* fns, int n) {
+  std::ostringstream s;
+  s << "{";
+  for (int i = 0; i < (n > 0 ? n : 1); ++i) s << (i ? ", " : "") << (i < n ? (int)fns[i] : 0);
+  s << "}";
+  return s.str();
+}
+
+std::string generate(const KPlan& kp) {
+  Gen g(kp);
+  std::ostringstream& o = g.o;
+  const bool c2 = kp.resolution == HQ_RES_ATOMIC;
+  const int sk = kp.sink == HQ_SINK_MATERIALISE ? 2 : (kp.nkeys == 0 ? 0 : 1);
+  // ---------------------------------------------------------------- kernel
+  o << "extern \"C\" __global__ void __launch_bounds__((NW + 1) * 32, 1) hq_jit_kernel(const __grid_constant__ JParams p) {\n"
+    << "  extern __shared__ __align__(128) char smem[];\n"
+    << "  u64* full = (u64*)smem; u64* empty = full + 10;\n"
+    << "  u64* s_base = (u64*)(empty + 10); int* s_wtot = (int*)(s_base + 16); i64* s_red = (i64*)(s_wtot + 16);\n"
+    << "  char* sagg = smem + OFF_AGG; char* stages = smem + OFF_STAGE;\n"
+    << "  (void)s_base; (void)s_wtot; (void)s_red; (void)sagg;\n"
+    << "  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n"
+    << "  const long long first_tile = p.row_begin / T;\n"
+    << "  const long long ntiles = p.row_end > p.row_begin ? (p.row_end + T - 1) / T - first_tile : 0;\n"
+    << "  const long long nj = ntiles > blockIdx.x ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;\n"
+    << "  if (threadIdx.x == 0) { for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], NW); } fence_mbar_init(); }\n";
+  // smem table init
+  if (sk == 1 && kp.smode == SM_LANE) {
+    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * NACC * NW * 32; i += NW * 32) {"
+      << " const int a_ = (int)((i / (NW * 32)) % NACC); t_[i] = a_ == 0 ? 0 : agg_identity(ACC_FN[a_]); } }\n";
+  } else if (sk == 1 && kp.smode == SM_DENSE) {
+    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * VWORDS; i += NW * 32) {"
+      << " const int c_ = (int)(i % VWORDS); t_[i] = c_ == 0 ? 0 : agg_identity(AGG_FN[c_ - 1]); } }\n";
+  } else if (sk == 1 && kp.smode == SM_HASH) {
+    o << "  if (warp < NW) { u64* k_ = (u64*)sagg; i64* e_ = (i64*)sagg + SMEM_CAP;\n"
+      << "    for (u32 i = threadIdx.x; i < SMEM_CAP; i += NW * 32) k_[i] = HQ_EMPTY_KEY;\n"
+      << "    for (u32 i = threadIdx.x; i < SMEM_CAP * VWORDS; i += NW * 32) { const int c_ = (int)(i % VWORDS); e_[i] = c_ == 0 ? 0 : agg_identity(AGG_FN[c_ - 1]); } }\n";
+  }
+  o << "  __syncthreads();\n";
+  // producer
+  o << "  if (warp == NW) {\n    if (lane == 0) {\n      const u64 pol = policy_evict_first();\n"
+    << "      for (long long j = 0; j < nj; ++j) {\n        const int s = (int)(j % S);\n"
+    << "        if (j >= S) mbar_wait(&empty[s], (u32)(((j / S) - 1) & 1));\n"
+    << "        const long long t0 = (first_tile + blockIdx.x + j * gridDim.x) * (long long)T;\n"
+    << "        char* st = stages + (size_t)s * STAGE_STRIDE;\n"
+    << "        if (t0 >= p.row_begin && t0 + T <= p.row_end) {\n          mbar_expect_tx(&full[s], STAGE_BYTES);\n";
+  for (int k = 0; k < kp.ncols; ++k)
+    o << "          tma_load_1d(st + " << kp.cols[k].soff << "u, p.col[" << k << "] + t0 * " << kp.cols[k].width << ", "
+      << kp.tile_rows * kp.cols[k].width << "u, &full[s], pol);\n";
+  o << "        } else mbar_arrive(&full[s]);\n      }\n    }\n    return;\n  }\n";
+  // consumer state
+  o << "  const int row0 = warp * 32 * R + lane;\n";
+  if (sk == 0 && !c2) {
+    o << "  u64 scount_ = 0;\n";
+    for (int a = 0; a < kp.naggs; ++a) o << "  i64 sacc" << a << " = agg_identity(AGG_FN[" << a << "]);\n";
+  }
+  o << "  for (long long j = 0; j < nj; ++j) {\n    const int s = (int)(j % S);\n"
+    << "    mbar_wait(&full[s], (u32)((j / S) & 1));\n"
+    << "    const long long t0 = (first_tile + blockIdx.x + j * gridDim.x) * (long long)T;\n"
+    << "    const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
+    << "    const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
+    << "    const char* st = stages + (size_t)s * STAGE_STRIDE;\n"
+    << "    u32 mask = 0;\n#pragma unroll\n    for (int r = 0; r < R; ++r) { const int row = row0 + r * 32; if (row >= lo && row < hi) mask |= 1u << r; }\n"
+    << "    if (lo > 0 || hi < T) {\n";
+  for (int k = 0; k < kp.ncols; ++k) {
+    const char* ty = ctype(kp.cols[k].width);
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r * 32; ((" << ty
+      << "*)(st + " << kp.cols[k].soff << "u))[row] = ((const " << ty << "*)p.col[" << k << "])[t0 + row]; }\n";
+  }
+  o << "      fence_proxy_async(); __syncwarp();\n    }\n";
+  if (sk == 2)  // output values leave the operator block in registers; the block scan runs after it
+    for (int j = 0; j < kp.nout; ++j) o << "    long long ov" << j << "[R];\n";
+  o << "    do {\n      if (!__any_sync(HQ_FULL, mask)) break;\n";
+  for (int i = 0; i < kp.nops; ++i) {
+    const KOp op = kp.ops[i];
+    if (op.kind == OP_FILTER) g.filter(kp.preds[op.idx], op.idx);
+    else if (op.kind == OP_PROBE) g.probe(kp.probes[op.idx], op.idx);
+    else g.compute(kp.comps[op.idx]);
+  }
+  // ------------------------------------------------------------ sink (tile)
+  auto aggval = [&](int a) -> std::string {
+    if (kp.agg_fn[a] == HQ_AGG_COUNT) return "1LL";
+    return "(i64)" + g.val(kp.agg_reg[a]);
+  };
+  if (sk == 0) {
+    std::vector<std::string> vv;
+    for (int a = 0; a < kp.naggs; ++a) vv.push_back(aggval(a));
+    if (c2) {  // B2: per-row global atomic reduce
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { g_add64(p.gtab, 1);\n";
+      for (int a = 0; a < kp.naggs; ++a) o << "        g_agg(AGG_FN[" << a << "], p.gtab + " << 1 + a << ", " << vv[a] << ", 1);\n";
+      o << "      }\n";
+    } else {
+      o << "      scount_ += __popc(mask);\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) {\n";
+      for (int a = 0; a < kp.naggs; ++a)
+        if (kp.agg_fn[a] != HQ_AGG_COUNT) o << "        sacc" << a << " = agg_combine(AGG_FN[" << a << "], sacc" << a << ", " << vv[a] << ");\n";
+      o << "      }\n";
+    }
+  } else if (sk == 1) {
+    o << "      u64 gk_[R]; bool bad_ = false;\n#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = 0;\n";
+    for (int i = 0; i < kp.nkeys; ++i) {
+      const std::string v = g.val(kp.key_reg[i]);
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kp.key_min[i])
+        << "; if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }"
+        << " gk_[r] += (u64)d_ * " << kp.key_stride[i] << "ull; }\n";
+    }
+    o << "      if (bad_) atomicOr(p.err, F_KEY_DOMAIN);\n";
+    if (kp.smode == SM_LANE) {
+      std::vector<std::string> av(kp.nacc);
+      for (int a = 1; a < kp.nacc; ++a) av[a] = "(i64)" + g.val(kp.acc_reg[a]);
+      o << "      i64* lt_ = (i64*)sagg + threadIdx.x;\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) {\n"
+        << "        i64* e_ = lt_ + gk_[r] * (u64)(NACC * NW * 32);\n        e_[0] += 1;\n";
+      for (int a = 1; a < kp.nacc; ++a)
+        o << "        e_[" << a << " * NW * 32] = agg_combine(ACC_FN[" << a << "], e_[" << a << " * NW * 32], " << av[a] << ");\n";
+      o << "      }\n";
+    } else {
+      std::vector<std::string> vv;
+      for (int a = 0; a < kp.naggs; ++a) vv.push_back(aggval(a));
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) {\n"
+        << "        const bool live_ = (mask >> r) & 1u; const u32 act_ = __ballot_sync(HQ_FULL, live_);\n"
+        << "        if (!act_) continue;\n"
+        << "        i64 v_[NAGGS > 0 ? NAGGS : 1];\n";
+      for (int a = 0; a < kp.naggs; ++a) o << "        v_[" << a << "] = " << vv[a] << ";\n";
+      if (c2) {
+        o << "        if (live_) group_update(p, sagg, gk_[r], false, 1ull, v_);\n      }\n";
+      } else {
+        o << "        const bool sparse_ = __popc(act_) <= 4;\n"
+          << "        const u64 mk_ = live_ ? gk_[r] : HQ_EMPTY_KEY;\n"
+          << "        const u32 peers_ = sparse_ ? ((1u << lane) & act_) : (__match_any_sync(HQ_FULL, mk_) & act_);\n"
+          << "        const bool single_ = live_ && __popc(peers_) == 1;\n"
+          << "        if (single_) group_update(p, sagg, gk_[r], true, 1ull, v_);\n"
+          << "        u32 multi_ = act_ & ~__ballot_sync(HQ_FULL, single_);\n"
+          << "        while (multi_) {\n          const int leader_ = __ffs(multi_) - 1;\n"
+          << "          const u32 grp_ = __shfl_sync(HQ_FULL, peers_, leader_); const bool mine_ = (grp_ >> lane) & 1u;\n"
+          << "          i64 w_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) w_[a] = warp_reduce(AGG_FN[a], mine_ ? v_[a] : agg_identity(AGG_FN[a]));\n"
+          << "          if (lane == leader_) group_update(p, sagg, gk_[r], true, (u64)__popc(grp_), w_);\n"
+          << "          multi_ &= ~grp_;\n        }\n      }\n";
+      }
+    }
+  } else {  // materialise: hand the output values to the block scan below
+    std::vector<std::string> ov;
+    for (int j = 0; j < kp.nout; ++j) ov.push_back(g.val(kp.out_reg[j]));
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) {";
+    for (int j = 0; j < kp.nout; ++j) o << " ov" << j << "[r] = (long long)" << ov[j] << ";";
+    o << " }\n";
+  }
+  o << "    } while (0);\n";
+  if (sk == 2) {
+    // A3 (Fig 25 / P:1069-1072): warp ballots -> block scan over the warps ->
+    // one atomicAdd per block and tile -> writes at local + global offset.
+    // Every consumer warp takes part in every tile (its mask may be empty).
+    o << "    {\n      u32 b_[R]; int wtot_ = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { b_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); wtot_ += __popc(b_[r]); }\n";
+    if (c2) {
+      o << "      (void)wtot_;\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = atomicAdd(p.counter, 1ull);\n";
+    } else {
+      o << "      if (lane == 0) s_wtot[warp] = wtot_;\n      consumer_bar();\n"
+        << "      if (warp == 0) { const int v_ = lane < NW ? s_wtot[lane] : 0; int incl_ = v_;\n"
+        << "#pragma unroll\n        for (int o_ = 1; o_ < 32; o_ <<= 1) { const int t_ = __shfl_up_sync(HQ_FULL, incl_, o_); if (lane >= o_) incl_ += t_; }\n"
+        << "        const int total_ = __shfl_sync(HQ_FULL, incl_, 31); u64 g_ = 0;\n"
+        << "        if (lane == 0 && total_ > 0) g_ = atomicAdd(p.counter, (u64)total_);\n"
+        << "        g_ = __shfl_sync(HQ_FULL, g_, 0); if (lane < NW) s_base[lane] = g_ + (u64)(incl_ - v_); }\n"
+        << "      consumer_bar();\n"
+        << "      const u64 base_ = s_base[warp]; const u32 lt_ = lanemask_lt(); u64 run_ = 0;\n"
+        << "#pragma unroll\n      for (int r = 0; r < R; ++r) { if ((mask >> r) & 1u) { const u64 pos_ = base_ + run_ + __popc(b_[r] & lt_);\n";
+    }
+    o << "        if ((long long)pos_ < p.capacity) {\n";
+    for (int j = 0; j < kp.nout; ++j)
+      o << "          ((" << ctype(kp.out_width[j]) << "*)p.out[" << j << "])[pos_] = (" << ctype(kp.out_width[j]) << ")ov" << j << "[r];\n";
+    o << "        } else atomicOr(p.err, F_CAPACITY); }\n";
+    if (!c2) o << "        run_ += __popc(b_[r]); }\n";
+    o << "    }\n";
+  }
+  o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n  }\n";
+  // ------------------------------------------------------------- sink (end)
+  if (sk == 0 && !c2) {
+    o << "  { u64 c_ = scount_;\n#pragma unroll\n    for (int o_ = 16; o_ > 0; o_ >>= 1) c_ += __shfl_xor_sync(HQ_FULL, c_, o_);\n";
+    for (int a = 0; a < kp.naggs; ++a) o << "    const i64 r" << a << " = warp_reduce(AGG_FN[" << a << "], sacc" << a << ");\n";
+    o << "    if (lane == 0) { s_red[warp * 9] = (i64)c_;";
+    for (int a = 0; a < kp.naggs; ++a) o << " s_red[warp * 9 + " << 1 + a << "] = r" << a << ";";
+    o << " }\n    consumer_bar();\n    if (threadIdx.x == 0) { u64 cnt_ = 0;";
+    for (int a = 0; a < kp.naggs; ++a) o << " i64 x" << a << " = agg_identity(AGG_FN[" << a << "]);";
+    o << "\n      for (int w = 0; w < NW; ++w) { cnt_ += (u64)s_red[w * 9];";
+    for (int a = 0; a < kp.naggs; ++a) o << " x" << a << " = agg_combine(AGG_FN[" << a << "], x" << a << ", s_red[w * 9 + " << 1 + a << "]);";
+    o << " }\n      if (cnt_) { g_add64(p.gtab, (i64)cnt_);";
+    for (int a = 0; a < kp.naggs; ++a) o << " g_agg(AGG_FN[" << a << "], p.gtab + " << 1 + a << ", x" << a << ", cnt_);";
+    o << " } } }\n";
+  } else if (sk == 1 && kp.smode == SM_LANE) {
+    o << "  consumer_bar();\n  { const i64* t_ = (const i64*)sagg;\n"
+      << "    for (u32 g = threadIdx.x; g < SMEM_CAP; g += NW * 32) {\n"
+      << "      const i64* e_ = t_ + (u64)g * NACC * NW * 32; u64 cnt_ = 0;\n"
+      << "      for (int l = 0; l < NW * 32; ++l) cnt_ += (u64)e_[l];\n      if (!cnt_) continue;\n"
+      << "      i64 acc_[NACC];\n#pragma unroll\n      for (int a = 1; a < NACC; ++a) { i64 v = agg_identity(ACC_FN[a]);"
+      << " for (int l = 0; l < NW * 32; ++l) v = agg_combine(ACC_FN[a], v, e_[a * NW * 32 + l]); acc_[a] = v; }\n"
+      << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n";
+    for (int a = 0; a < kp.naggs; ++a)
+      o << "      vals_[" << a << "] = " << (kp.acc_of[a] ? "acc_[" + std::to_string(kp.acc_of[a]) + "]" : std::string("(i64)cnt_")) << ";\n";
+    o << "      group_update(p, sagg, g, false, cnt_, vals_);\n    } }\n";
+  } else if (sk == 1 && kp.smode == SM_DENSE) {
+    o << "  consumer_bar();\n  { const i64* t_ = (const i64*)sagg;\n"
+      << "    for (u32 g = threadIdx.x; g < SMEM_CAP; g += NW * 32) { const i64* e_ = t_ + (u64)g * VWORDS;\n"
+      << "      if (e_[0] != 0) { i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) vals_[a] = e_[1 + a];\n"
+      << "        group_update(p, sagg, g, false, (u64)e_[0], vals_); } } }\n";
+  } else if (sk == 1 && kp.smode == SM_HASH) {
+    o << "  consumer_bar();\n  { const u64* k_ = (const u64*)sagg; const i64* t_ = (const i64*)sagg + SMEM_CAP;\n"
+      << "    for (u32 h = threadIdx.x; h < SMEM_CAP; h += NW * 32) if (k_[h] != HQ_EMPTY_KEY) { const i64* e_ = t_ + (u64)h * VWORDS;\n"
+      << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = e_[1 + a];\n"
+      << "      group_update(p, sagg, k_[h], false, (u64)e_[0], vals_); } }\n";
+  }
+  o << "}\n";
+
+  // ---------------------------------------------------------- constants
+  std::ostringstream h;
+  h << "// generated by libhq (hq_jit.cu) for one fusion operator\n"
+    << "#define NW " << kp.nw << "\n#define R " << kp.R << "\n#define T " << kp.tile_rows << "\n#define S " << kp.nstages
+    << "\n#define STAGE_STRIDE " << kp.stage_stride << "u\n#define STAGE_BYTES " << kp.stage_bytes
+    << "u\n#define OFF_AGG " << kp.off_agg << "u\n#define OFF_STAGE " << kp.off_stage << "u\n"
+    << "#define NAGGS " << kp.naggs << "\n#define VWORDS " << kp.vwords << "\n#define GMODE " << (int)kp.gmode
+    << "\n#define SMODE " << (kp.smode == SM_LANE ? 0 : (int)kp.smode) << "\n#define SMEM_CAP " << kp.smem_cap
+    << "u\n#define SLOG2 " << kp.slog2 << "\n#define NACC " << (kp.nacc > 0 ? kp.nacc : 1) << "\n"
+    << "static constexpr __device__ int AGG_FN[" << (kp.naggs > 0 ? kp.naggs : 1) << "] = " << fn_list(kp.agg_fn, kp.naggs)
+    << ";\n"
+    << "static constexpr __device__ int ACC_FN[" << (kp.nacc > 0 ? kp.nacc : 1) << "] = " << fn_list(kp.acc_fn, kp.nacc) << ";\n"
+    << HQ_STR(HQ_JPARAMS_DEF) << "\n"
+    << kPrelude << "\n"
+    << g.bitmaps.str() << "\n";
+  return h.str() + o.str();
+}
+
+CUfunction compile(hq_ctx* ctx, const std::string& src) {
+  const auto key = std::make_pair(ctx->device, src);
+  {
+    std::lock_guard<std::mutex> gl(g_mu);
+    auto it = g_cache.find(key);
+    if (it != g_cache.end()) return it->second;
+  }
+  nvrtcProgram prog;
+  if (nvrtcCreateProgram(&prog, src.c_str(), "hq_jit_kernel.cu", 0, nullptr, nullptr) != NVRTC_SUCCESS)
+    HQ_THROW(HQ_ERR_CUDA, "nvrtcCreateProgram failed");
+  const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "--device-int128"};
+  const nvrtcResult rc = nvrtcCompileProgram(prog, 4, opts);
+  if (rc != NVRTC_SUCCESS) {
+    size_t n = 0;
+    nvrtcGetProgramLogSize(prog, &n);
+    std::string log(n, '\0');
+    nvrtcGetProgramLog(prog, &log[0]);
+    nvrtcDestroyProgram(&prog);
+    HQ_THROW(HQ_ERR_CUDA, "NVRTC compile failed:\n" + log.substr(0, 4000));
+  }
+  size_t n = 0;
+  nvrtcGetCUBINSize(prog, &n);
+  std::string cubin(n, '\0');
+  nvrtcGetCUBIN(prog, &cubin[0]);
+  nvrtcDestroyProgram(&prog);
+  Driver& d = driver();
+  CUmodule mod;
+  CUfunction fn;
+  if (d.modload(&mod, cubin.data()) != CUDA_SUCCESS) HQ_THROW(HQ_ERR_CUDA, "cuModuleLoadData failed");
+  if (d.getfn(&fn, mod, "hq_jit_kernel") != CUDA_SUCCESS) HQ_THROW(HQ_ERR_CUDA, "cuModuleGetFunction failed");
+  std::lock_guard<std::mutex> gl(g_mu);
+  g_cache[key] = fn;
+  return fn;
+}
+
+}  // namespace
+
+bool hq_jit_enabled() {
+  const char* e = getenv("HQ_JIT");
+  return !(e && e[0] == '0');
+}
+
+std::string hq_jit_source(const KPlan& kp) { return generate(kp); }
+
+namespace {
+thread_local CUfunction t_last_fn = nullptr;  // kernel compiled by the last hq_jit_prepare
+}
+
+void hq_jit_prepare(hq_ctx* ctx, const KPlan& kp, size_t smem) {
+  const std::string src = generate(kp);
+  CUfunction fn = compile(ctx, src);
+  if (driver().setattr(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem) != CUDA_SUCCESS)
+    HQ_THROW(HQ_ERR_CUDA, "cuFuncSetAttribute failed");
+  t_last_fn = fn;
+}
+
+void hq_jit_launch(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
+  CUfunction fn = t_last_fn;
+  if (!fn) HQ_THROW(HQ_ERR_STATE, "jit: hq_jit_prepare not called");
+  Driver& d = driver();
+  JParams jp{};
+  jp.row_begin = kp.row_begin;
+  jp.row_end = kp.row_end;
+  for (int k = 0; k < kp.ncols; ++k) jp.col[k] = kp.cols[k].ptr;
+  for (int i = 0; i < MAX_PROBES; ++i) jp.ht[i] = kp.probes[i].slots;
+  jp.gtab = kp.gtab;
+  jp.gmask = kp.gmask;
+  jp.glog2 = kp.glog2;
+  for (int j = 0; j < kp.nout; ++j) jp.out[j] = kp.out_ptr[j];
+  jp.capacity = kp.capacity;
+  jp.counter = kp.counter;
+  jp.err = kp.err;
+  void* args[] = {&jp};
+  ctx->launches++;
+  if (d.launch(fn, (unsigned)grid, 1, 1, (unsigned)((kp.nw + 1) * 32), 1, 1, (unsigned)smem, (CUstream)ctx->stream, args,
+               nullptr) != CUDA_SUCCESS)
+    HQ_THROW(HQ_ERR_CUDA, "cuLaunchKernel failed");
+}

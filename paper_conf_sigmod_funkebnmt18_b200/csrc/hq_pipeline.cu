@@ -420,7 +420,10 @@ __device__ __forceinline__ void sink_group(const KPlan& p, const char* stage, co
     if (!act) continue;
     const int row = row0 + r * 32;
     const unsigned long long mk = live ? gk[r] : EMPTY_KEY;
-    const uint32_t peers = c2 ? (1u << lane) & act : __match_any_sync(FULLMASK, mk) & act;
+    // few live lanes (selective pipelines): each updates directly; match_any
+    // only pays when many lanes may share a key
+    const bool sparse = c2 || __popc(act) <= 4;
+    const uint32_t peers = sparse ? (1u << lane) & act : __match_any_sync(FULLMASK, mk) & act;
     const bool single = live && __popc(peers) == 1;
     if (single) {  // C2 rows, and keys unique within the warp: direct update
       group_update(p, sagg, gk[r], !c2, 1ull, [&](int a) {

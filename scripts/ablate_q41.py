@@ -61,3 +61,9 @@ for k, sink in [(0, "count"), (1, "count"), (2, "count"), (3, "count"), (4, "cou
     ms = sum(kt) / len(kt)
     print(f"probes={k} sink={sink:5s} kernel {ms:.3f} ms  {rows * 24 / ms / 1e6:.0f} GB/s  rows/clk/SM "
           f"{rows / (ms * 1e-3) / 148 / 1.965e9:.3f}")
+E.resolution = hq.RES_ATOMIC
+ctx.enable_timing(True)
+for _ in range(4):
+    E.run(plan(4, "group")).fetch()
+kt = ctx.kernel_times()[1:]
+print(f"probes=4 sink=group C2 (per-row global atomics) kernel {sum(kt) / len(kt):.3f} ms")

@@ -114,6 +114,16 @@ def test_ssb_q31_materialise_parity(ctx, ssb):
 
 
 @pytest.mark.parametrize("qname", ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q31", "ssb_q41", "tpch_q3"])
+def test_interpreter_parity(ctx, ssb, tpch, qname):
+    """The precompiled descriptor interpreter (HQ_EXEC_FUSED_INTERP) == oracle, so the
+    NVRTC-generated kernels (default FUSED) have an independent GPU twin."""
+    host = host_for(qname, ssb, tpch)
+    kw = {"limit": 0} if qname == "tpch_q3" else {}
+    g = gpu_run(ctx, qname, host, exec_mode=hq.EXEC_FUSED_INTERP, **kw)
+    assert_same(qname, g, oracle_run(qname, host))
+
+
+@pytest.mark.parametrize("qname", ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q31", "ssb_q41", "tpch_q3"])
 def test_operator_at_a_time_parity(ctx, ssb, tpch, qname):
     """The op-at-a-time baseline (a11) of the same plan == oracle (two independent GPU paths)."""
     host = host_for(qname, ssb, tpch)
