@@ -182,8 +182,14 @@ typedef struct {
   int64_t bytes;        /* capacity * slot_words * 4 */
   int64_t key_min;      /* HQ_HT_DIRECT: key stored in slot 0 */
   int32_t layout;       /* HQ_HT_LINEAR or HQ_HT_DIRECT */
+  int32_t pay_min;      /* min / max of payload 0 over the inserted rows (count pass) */
+  int32_t pay_max;
   int32_t reserved;
 } hq_hash_meta;
+/* Direct tables also get a compact derived form (rebuilt on import): a bitmap
+ * of present keys for semi-join tables, or one byte per key (payload - pay_min,
+ * 0xFF = absent) when payload 0 spans <= 255 values; generated kernels stage
+ * small compact tables in shared memory. */
 hq_status hq_hash_info(hq_ctx* ctx, const hq_hash* h, hq_hash_meta* meta);  /* syncs, reports build faults */
 /* Multi-GPU glue: raw device view of the slot array (to broadcast it with NCCL)
  * and import of such a buffer on another device (borrowed, caller keeps it). */

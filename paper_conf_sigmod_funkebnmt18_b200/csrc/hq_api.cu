@@ -294,6 +294,12 @@ hq_status hq_hash_import(hq_ctx* ctx, const hq_hash_meta* meta, void* dev_ptr, h
     while ((1LL << l) < cap) ++l;
     h->log2cap = l;
     h->checked = true;
+    try {
+      hq_build_compact(ctx, h);
+    } catch (...) {
+      h->release();
+      throw;
+    }
     *out = h;
   });
 }

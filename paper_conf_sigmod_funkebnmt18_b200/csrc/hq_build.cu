@@ -58,7 +58,7 @@ __device__ __forceinline__ bool row_passes(const KBuild& b, long long row) {
 
 __global__ void hq_build_count_kernel(const __grid_constant__ KBuild b) {
   unsigned long long c = 0;
-  int kmin = INT_MAX, kmax = INT_MIN;
+  int kmin = INT_MAX, kmax = INT_MIN, pmin = INT_MAX, pmax = INT_MIN;
   for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < b.n; r += (long long)gridDim.x * blockDim.x) {
     if (!row_passes(b, r)) continue;
     ++c;
@@ -67,12 +67,24 @@ __global__ void hq_build_count_kernel(const __grid_constant__ KBuild b) {
       kmin = min(kmin, (int)kv);
       kmax = max(kmax, (int)kv);
     }
+    if (b.npay > 0) {
+      const long long pv = ld_col(b, b.pay_col[0], r);
+      const int pc = pv < (long long)INT_MIN ? INT_MIN : (pv > (long long)INT_MAX ? INT_MAX : (int)pv);
+      pmin = min(pmin, pc);
+      pmax = max(pmax, pc);
+    }
   }
   kmin = __reduce_min_sync(0xffffffffu, kmin);
   kmax = __reduce_max_sync(0xffffffffu, kmax);
+  pmin = __reduce_min_sync(0xffffffffu, pmin);
+  pmax = __reduce_max_sync(0xffffffffu, pmax);
   if ((threadIdx.x & 31) == 0 && kmin <= kmax) {
     atomicMin(b.kminmax, kmin);
     atomicMax(b.kminmax + 1, kmax);
+  }
+  if ((threadIdx.x & 31) == 0 && pmin <= pmax) {
+    atomicMin(b.kminmax + 2, pmin);
+    atomicMax(b.kminmax + 3, pmax);
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
@@ -200,15 +212,17 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   bool direct = false;
   int64_t kmin = 0, range = 0;
   if (keys <= 0) {  // exact count pass (one sync): number and range of the qualifying keys
-    const int init[2] = {INT_MAX, INT_MIN};
-    HQ_CUDA(cudaMemcpyAsync(b.kminmax, init, 8, cudaMemcpyHostToDevice, ctx->stream));
+    const int init[4] = {INT_MAX, INT_MIN, INT_MAX, INT_MIN};
+    HQ_CUDA(cudaMemcpyAsync(b.kminmax, init, 16, cudaMemcpyHostToDevice, ctx->stream));
     if (b.n > 0) { ctx->launches++; hq_build_count_kernel<<<grid, 256, 0, ctx->stream>>>(b); }
     HQ_CUDA(cudaGetLastError());
-    struct { unsigned long long cnt; int kmin, kmax; } st{};
-    HQ_CUDA(cudaMemcpyAsync(&st, b.nkeys, 16, cudaMemcpyDeviceToHost, ctx->stream));
+    struct { unsigned long long cnt; int kmin, kmax, pmin, pmax; } st{};
+    HQ_CUDA(cudaMemcpyAsync(&st, b.nkeys, 24, cudaMemcpyDeviceToHost, ctx->stream));
     HQ_CUDA(cudaStreamSynchronize(ctx->stream));
     HQ_CUDA(cudaMemsetAsync(b.nkeys, 0, 8, ctx->stream));
     keys = (int64_t)st.cnt;
+    h->meta.pay_min = st.pmin;
+    h->meta.pay_max = st.pmax;
     if (keys > 0 && st.kmin <= st.kmax) {
       kmin = st.kmin;
       range = (int64_t)st.kmax - st.kmin + 1;
@@ -243,6 +257,61 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   b.dmin = (int32_t)kmin;
   if (b.n > 0) { ctx->launches++; hq_build_hash_kernel<<<grid, 256, 0, ctx->stream>>>(b); }
   HQ_CUDA(cudaGetLastError());
+  if (direct) hq_build_compact(ctx, h);
+}
+
+namespace {
+// bitmap of present keys: thread per 32-key word
+__global__ void hq_compact_bitmap_kernel(const uint32_t* slots, long long range, uint32_t* out) {
+  const long long nwords = (range + 31) / 32;
+  for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < nwords; w += (long long)gridDim.x * blockDim.x) {
+    uint32_t bits = 0;
+    for (int b = 0; b < 32; ++b) {
+      const long long i = w * 32 + b;
+      if (i < range && (int)slots[i] != INT_MIN) bits |= 1u << b;
+    }
+    out[w] = bits;
+  }
+}
+// one byte per key: payload0 - pay_min, 0xFF = absent (8-B slots {key, payload})
+__global__ void hq_compact_u8_kernel(const uint32_t* slots, long long range, int pay_min, uint32_t* out) {
+  const long long nwords = (range + 3) / 4;
+  for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < nwords; w += (long long)gridDim.x * blockDim.x) {
+    uint32_t v = 0;
+    for (int b = 0; b < 4; ++b) {
+      const long long i = w * 4 + b;
+      uint32_t byte = 0xFFu;
+      if (i < range && (int)slots[2 * i] != INT_MIN) byte = (uint32_t)((int)slots[2 * i + 1] - pay_min) & 0xFFu;
+      v |= byte << (8 * b);
+    }
+    out[w] = v;
+  }
+}
+}  // namespace
+
+// Compact derived form of a direct table (used by generated kernels to stage
+// small probe tables in shared memory): bitmap for semi-joins, bytes for one
+// small payload.  Also run on import (multi-GPU) from the broadcast slots.
+void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
+  h->ckind = 0;
+  h->cbytes = 0;
+  if (h->meta.layout != HQ_HT_DIRECT) return;
+  const long long range = h->meta.capacity;
+  int kind = 0;
+  if (h->meta.npayload == 0) kind = 1;
+  else if (h->meta.npayload == 1 && h->meta.pay_min <= h->meta.pay_max &&
+           (long long)h->meta.pay_max - h->meta.pay_min < 255)
+    kind = 2;
+  if (!kind) return;
+  const long long words = kind == 1 ? (range + 31) / 32 : (range + 3) / 4;
+  h->compact = DevBuf(ctx, (size_t)words * 4 + 16);
+  const int grid = (int)std::max<long long>(1, std::min<long long>((words + 255) / 256, (long long)ctx->num_sms * 8));
+  ctx->launches++;
+  if (kind == 1) hq_compact_bitmap_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->compact.as<uint32_t>());
+  else hq_compact_u8_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>());
+  HQ_CUDA(cudaGetLastError());
+  h->ckind = kind;
+  h->cbytes = words * 4;
 }
 
 // Sync and report build faults (HQ_ERR_DUP_KEY etc.).

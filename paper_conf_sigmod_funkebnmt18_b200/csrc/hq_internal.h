@@ -117,7 +117,13 @@ struct hq_hash : RefObj {
   DevBuf owned;      // slot array (empty when imported)
   DevBuf dstate;     // [0] fault bits (int), [1..2] nkeys (u64) -- see hq_build.cu
   bool checked = false;
+  // compact form of a direct table (hq_build.cu): 1 = bitmap of present keys
+  // (semi-join), 2 = one byte per key (payload0 - pay_min, 0xFF absent)
+  DevBuf compact;
+  int ckind = 0;
+  int64_t cbytes = 0;
 };
+void hq_build_compact(hq_ctx* ctx, hq_hash* h);  // derive hq_hash::compact from the slots
 
 // ------------------------------------------------- device plan (kernel param)
 namespace hqk {
@@ -169,9 +175,13 @@ struct KProbe {
   uint8_t mode;      // hq_probe_mode
   uint8_t npay;
   uint8_t direct;    // 1 = direct-mapped (dense keys)
-  uint8_t pad;
+  uint8_t ckind;     // compact form available (hq_hash::ckind)
   int16_t key_reg;
   int16_t dst[HQ_MAX_PAYLOAD];
+  const void* compact;
+  int32_t pay_min;   // ckind 2: payload = byte + pay_min
+  uint32_t cbytes;
+  uint32_t smem_off; // generated kernels: byte offset of the staged compact table (0 = not staged)
 };
 struct KCompute {
   int16_t dst;
@@ -197,6 +207,7 @@ struct KPlan {
   uint32_t stage_bytes;      // bytes of one stage's columns (= tile_rows * row width)
   uint32_t stage_stride;     // stage spacing in smem (>= stage_bytes, 128-B multiple)
   uint32_t off_tmp, off_agg, off_stage;  // dynamic smem layout
+  uint32_t off_tab, tab_bytes;           // staged compact probe tables (generated kernels)
   int32_t ncols;
   KCol cols[HQ_MAX_COLS];
   KReg regs[NREGS];

@@ -30,6 +30,7 @@ using namespace hqk;
     long long row_begin, row_end;                                                                              \
     const char* col[16];                                                                                       \
     const unsigned* ht[8];                                                                                     \
+    const void* ctab[8];                                                                                       \
     long long* gtab;                                                                                           \
     unsigned long long gmask;                                                                                  \
     int glog2, pad;                                                                                            \
@@ -163,6 +164,26 @@ struct Gen {
       loaded.insert(pr.dst[k]);
     }
     const std::string key = val(pr.key_reg);
+    if (pr.direct && pr.smem_off) {
+      // compact table staged in shared memory: bitmap (semi) or one byte per key
+      o << "      { u32 found_ = 0u;\n#pragma unroll\n        for (int r = 0; r < R; ++r) {\n"
+        << "          const long long k_ = (long long)" << key << ";\n"
+        << "          const u32 d_ = (u32)(k_ - " << pr.dmin << "LL);\n"
+        << "          if (((mask >> r) & 1u) && k_ >= " << pr.dmin << "LL && d_ < " << pr.mask << "u) {\n";
+      if (pr.ckind == 1) {
+        o << "            const u32 w_ = ((const u32*)(smem + " << pr.smem_off << "u))[d_ >> 5];\n"
+          << "            if ((w_ >> (d_ & 31u)) & 1u) found_ |= 1u << r;\n";
+      } else {
+        o << "            const int b_ = ((const unsigned char*)(smem + " << pr.smem_off << "u))[d_];\n"
+          << "            if (b_ != 0xFF) { found_ |= 1u << r;";
+        if (npay > 0) o << " " << var(pr.dst[0]) << "[r] = b_ + (" << pr.pay_min << ");";
+        o << " }\n";
+      }
+      o << "          }\n        }\n"
+        << "        mask = " << (pr.mode == HQ_PROBE_ANTI ? "mask & ~found_" : "mask & found_") << "; }\n";
+      early_exit();
+      return;
+    }
     o << "      { const u32* ht_ = p.ht[" << idx << "]; u32 found_ = 0u; int kk_[R]; u32 pend_ = 0u; u32 pos_[R];\n"
       << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n"
       << "          const long long k_ = (long long)" << key << "; kk_[r] = (int)k_;\n";
@@ -276,6 +297,13 @@ std::string generate(const KPlan& kp) {
     o << "  if (warp < NW) { u64* k_ = (u64*)sagg; i64* e_ = (i64*)sagg + SMEM_CAP;\n"
       << "    for (u32 i = threadIdx.x; i < SMEM_CAP; i += NW * 32) k_[i] = HQ_EMPTY_KEY;\n"
       << "    for (u32 i = threadIdx.x; i < SMEM_CAP * VWORDS; i += NW * 32) { const int c_ = (int)(i % VWORDS); e_[i] = c_ == 0 ? 0 : agg_identity(AGG_FN[c_ - 1]); } }\n";
+  }
+  // staged compact probe tables: one cooperative 16-B copy per CTA
+  for (int i = 0; i < MAX_PROBES; ++i) {
+    const KProbe& pr = kp.probes[i];
+    if (!pr.smem_off) continue;
+    o << "  { const uint4* src_ = (const uint4*)p.ctab[" << i << "]; uint4* dst_ = (uint4*)(smem + " << pr.smem_off << "u);\n"
+      << "    for (u32 x = threadIdx.x; x < " << (pr.cbytes + 15) / 16 << "u; x += blockDim.x) dst_[x] = __ldg(src_ + x); }\n";
   }
   o << "  __syncthreads();\n";
   // producer
@@ -530,7 +558,10 @@ void hq_jit_launch(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
   jp.row_begin = kp.row_begin;
   jp.row_end = kp.row_end;
   for (int k = 0; k < kp.ncols; ++k) jp.col[k] = kp.cols[k].ptr;
-  for (int i = 0; i < MAX_PROBES; ++i) jp.ht[i] = kp.probes[i].slots;
+  for (int i = 0; i < MAX_PROBES; ++i) {
+    jp.ht[i] = kp.probes[i].slots;
+    jp.ctab[i] = kp.probes[i].compact;
+  }
   jp.gtab = kp.gtab;
   jp.gmask = kp.gmask;
   jp.glog2 = kp.glog2;

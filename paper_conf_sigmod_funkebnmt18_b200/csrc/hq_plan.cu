@@ -127,6 +127,11 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.mask = pr.direct ? (uint32_t)op.ht->meta.capacity : (uint32_t)(op.ht->meta.capacity - 1);
       pr.dmin = (int32_t)op.ht->meta.key_min;
       pr.log2cap = (uint8_t)op.ht->log2cap;
+      pr.ckind = (uint8_t)op.ht->ckind;
+      pr.compact = op.ht->compact.p;
+      pr.pay_min = op.ht->meta.pay_min;
+      pr.cbytes = (uint32_t)op.ht->cbytes;
+      pr.smem_off = 0;
       pr.words = (uint8_t)op.ht->meta.slot_words;
       pr.mode = (uint8_t)op.mode;
       const int npay = op.mode == HQ_PROBE_INNER ? op.npayload : 0;
@@ -285,30 +290,62 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     for (int k = 0; k < HQ_MAX_TMP; ++k) tmp_row += (uint32_t)regs[HQ_MAX_COLS + k].width;
 
   kp.nw = kp.smode == SM_LANE ? LANE_NW : NW;
-  if (const char* e = getenv("HQ_DEBUG_NW")) kp.nw = atoi(e);  // debugging aid
-  int chosen_R = 0;
-  for (int R : {4, 2}) {
-    const uint32_t T = (uint32_t)(kp.nw * 32 * R);
-    const uint32_t off_tmp = MISC_BYTES;
-    const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
-    const uint32_t off_stage = align_up(off_agg + agg_smem, 128);
-    const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
-    if (off_stage >= ctx->max_smem) continue;
-    const int S = (int)std::min<int64_t>(MAX_STAGES, (ctx->max_smem - off_stage) / stride);
-    if (S >= 3 || (R == 2 && S >= 2)) {
-      chosen_R = R;
-      kp.R = R;
-      kp.tile_rows = (int32_t)T;
-      kp.nstages = S;
-      kp.stage_bytes = T * rowbytes;
-      kp.stage_stride = stride;
-      kp.off_tmp = off_tmp;
-      kp.off_agg = off_agg;
-      kp.off_stage = off_stage;
-      break;
+  // Generated kernels stage small compact probe tables (bitmaps / byte arrays of
+  // direct tables) in shared memory, earliest probes first (they see the most
+  // rows), as long as the TMA ring keeps >= 3 stages.
+  int staged[MAX_PROBES];
+  int nstaged = 0;
+  if (jit) {
+    uint32_t total = 0;
+    for (int o = 0; o < kp.nops; ++o) {
+      if (kp.ops[o].kind != OP_PROBE) continue;
+      const KProbe& pr = kp.probes[kp.ops[o].idx];
+      if (!pr.ckind || pr.cbytes == 0) continue;
+      const uint32_t b = align_up(pr.cbytes, 128);
+      if (total + b > 96 * 1024) continue;
+      total += b;
+      staged[nstaged++] = kp.ops[o].idx;
     }
   }
+  int chosen_R = 0;
+  for (;;) {
+    uint32_t tab_total = 0;
+    for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
+    for (int R : {4, 2}) {
+      const uint32_t T = (uint32_t)(kp.nw * 32 * R);
+      const uint32_t off_tmp = MISC_BYTES;
+      const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
+      const uint32_t off_tab = align_up(off_agg + agg_smem, 128);
+      const uint32_t off_stage = align_up(off_tab + tab_total, 128);
+      const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
+      if (off_stage >= ctx->max_smem) continue;
+      const int S = (int)std::min<int64_t>(MAX_STAGES, (ctx->max_smem - off_stage) / stride);
+      if (S >= 3 || (R == 2 && S >= 2 && nstaged == 0)) {
+        chosen_R = R;
+        kp.R = R;
+        kp.tile_rows = (int32_t)T;
+        kp.nstages = S;
+        kp.stage_bytes = T * rowbytes;
+        kp.stage_stride = stride;
+        kp.off_tmp = off_tmp;
+        kp.off_agg = off_agg;
+        kp.off_tab = off_tab;
+        kp.tab_bytes = tab_total;
+        kp.off_stage = off_stage;
+        break;
+      }
+    }
+    if (chosen_R || nstaged == 0) break;
+    --nstaged;  // give the last staged table back to the ring
+  }
   if (!chosen_R) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: rows too wide for the shared-memory stage ring");
+  {
+    uint32_t off = kp.off_tab;
+    for (int i = 0; i < nstaged; ++i) {
+      kp.probes[staged[i]].smem_off = off;
+      off += align_up(kp.probes[staged[i]].cbytes, 128);
+    }
+  }
   const uint32_t T = (uint32_t)kp.tile_rows;
   uint32_t soff = 0;
   for (int c = 0; c < F->ncols; ++c) {

@@ -36,7 +36,7 @@ def broadcast_blob(meta: Optional[Sequence[int]], buf: Optional[torch.Tensor], n
     """Broadcast a small int64 meta vector, then a byte buffer whose size is
     meta[nbytes_index].  Non-root ranks pass meta=None, buf=None."""
     rank = dist.get_rank()
-    m = torch.zeros(8, dtype=torch.int64, device=device)
+    m = torch.zeros(16, dtype=torch.int64, device=device)
     if rank == root:
         m[: len(meta)] = torch.tensor(list(meta), dtype=torch.int64)
     dist.broadcast(m, src=root)
@@ -82,14 +82,16 @@ class DistributedEngine(Engine):
             m = h.info()  # syncs, reports build faults before anything is sent
             ptr, _ = h.device_view()
             buf = device_view(ptr, int(m.bytes))
-            meta = [m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout]
+            meta = [m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout,
+                    m.pay_min, m.pay_max]
         else:
             meta, buf = None, None
         meta, buf = broadcast_blob(meta, buf, 4, self.root, self.device)
         if self.rank == self.root:
             return h
         hm = hq.HashMeta()
-        hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout = meta[:7]
+        (hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout,
+         hm.pay_min, hm.pay_max) = meta[:9]
         return self.ctx.import_hash(hm, buf.data_ptr(), keep=buf)
 
     def hash(self, table, key, payload=(), preds=(), expected_rows=0) -> hq.Hash:

@@ -247,6 +247,49 @@ def test_edge_cases(ctx):
         assert res.qualifying() == 0 and len(res.fetch()[0]) == 0
 
 
+@pytest.mark.parametrize("exec_mode", [hq.EXEC_FUSED, hq.EXEC_FUSED_INTERP, hq.EXEC_OAAT])
+@pytest.mark.parametrize("spread", [1, 7, 1000])
+def test_probe_modes(ctx, exec_mode, spread):
+    """semi / anti / inner probes against direct (spread 1, 7) and linear-probing
+    (spread 1000) tables, staged compact or not, vs numpy."""
+    from paper_conf_sigmod_funkebnmt18_b200.engine import PlanBuilder
+    rng = np.random.default_rng(spread)
+    ndim = 5000
+    keys = (np.arange(ndim, dtype=np.int64) * spread + 11).astype(np.int32)
+    sel = rng.random(ndim) < 0.4
+    pay = rng.integers(-3, 40, ndim).astype(np.int32)
+    wide = rng.integers(-10**6, 10**6, ndim).astype(np.int32)
+    dim = ctx.load_columns({"k": keys, "sel": sel.astype(np.int8), "pay": pay, "wide": wide})
+    n = 100_000
+    fk = keys[rng.integers(0, ndim, n)].copy()
+    fk[::17] = 5  # never present
+    vcol = rng.integers(0, 100, n).astype(np.int32)
+    fact = ctx.load_columns({"fk": fk, "v": vcol})
+    pred = [hq.make_pred(1, "=", 1)]
+    h_semi = ctx.build_hash(dim, 0, [], pred)
+    h_one = ctx.build_hash(dim, 0, [2], pred)
+    h_two = ctx.build_hash(dim, 0, [2, 3], pred)
+    present = dict(zip(keys[sel].tolist(), range(int(sel.sum()))))
+    psel, wsel = pay[sel], wide[sel]
+    hit = np.array([k in present for k in fk.tolist()])
+    idx = np.array([present.get(k, 0) for k in fk.tolist()])
+    for mode, ht, payload in (("semi", h_semi, []), ("anti", h_semi, []), ("inner", h_one, ["p"]),
+                              ("inner", h_two, ["p", "w"])):
+        pb = PlanBuilder(fact)
+        pb.probe(ht, "fk", mode, payload)
+        aggs = [("count", None), ("sum", "v")] + [("sum", x) for x in payload]
+        pb.aggregate(aggs=aggs, agg_names=[f"a{i}" for i in range(len(aggs))])
+        pb.plan.exec = exec_mode
+        got = [int(x[0]) for x in ctx.run(pb.plan, keep=pb.keep).fetch()]
+        m = ~hit if mode == "anti" else hit
+        exp = [int(m.sum()), int(vcol[m].astype(np.int64).sum())]
+        if "p" in payload:
+            exp.append(int(psel[idx[m]].astype(np.int64).sum()))
+        if "w" in payload:
+            exp.append(int(wsel[idx[m]].astype(np.int64).sum()))
+        assert got == exp, (mode, payload, got, exp)
+
+
 def test_duplicate_build_key(ctx):
     d = {"k": np.array([1, 2, 2, 3], np.int32), "v": np.array([1, 2, 3, 4], np.int32)}
     t = ctx.load_columns(d)
