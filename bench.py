@@ -145,17 +145,15 @@ def oracle_call(qname, host, nthreads, fact_rows=None):
     return time.perf_counter() - t0
 
 
-def cpu_baseline(qname, host, n_fact, target_s=12.0):
-    """Time the oracle (as it stands) on a bounded prefix sample of the workload."""
+def cpu_baseline(qname, host, n_fact, budget_s=30.0):
+    """Time the oracle (as it stands, all host cores) on the whole workload, or on
+    a prefix sample when the whole would take longer than ~budget_s."""
     cores = os.cpu_count() or 1
     s0 = min(n_fact, 2_000_000)
-    dt = oracle_call(qname, host, cores, s0)
-    rate = s0 / max(dt, 1e-9)
-    s = int(min(n_fact, max(s0, rate * target_s)))
-    if s > s0:
-        dt = oracle_call(qname, host, cores, s)
-    else:
-        s = s0
+    dt0 = oracle_call(qname, host, cores, s0)  # includes the dimension hash-map builds
+    est = dt0 * n_fact / max(s0, 1)
+    s = n_fact if est <= budget_s else max(s0, int(n_fact * budget_s / est))
+    dt = oracle_call(qname, host, cores, s)
     return {"value": s / dt, "unit": "rows/s", "cores": cores, "kind": "oracle",
             "sample": f"first {s} of {n_fact} fact rows (full dimension tables), tuple-at-a-time C++ oracle, "
                       f"{cores} threads, {dt:.2f} s"}
