@@ -184,12 +184,14 @@ typedef struct {
   int32_t layout;       /* HQ_HT_LINEAR or HQ_HT_DIRECT */
   int32_t pay_min;      /* min / max of payload 0 over the inserted rows (count pass) */
   int32_t pay_max;
-  int32_t reserved;
+  int32_t key_max;      /* max key inserted (count pass); key range = [key_min, key_max] */
 } hq_hash_meta;
-/* Direct tables also get a compact derived form (rebuilt on import): a bitmap
- * of present keys for semi-join tables, or one byte per key (payload - pay_min,
- * 0xFF = absent) when payload 0 spans <= 255 values; generated kernels stage
- * small compact tables in shared memory. */
+/* Derived forms (rebuilt on import): direct tables get a compact form -- a
+ * bitmap of present keys for semi-join tables, or one byte per key (payload -
+ * pay_min, 0xFF = absent) when payload 0 spans <= 255 values -- that generated
+ * kernels stage in shared memory; linear tables whose key range fits in 64 MiB
+ * of bits get an exact key-range bitmap that generated kernels test before
+ * touching the slot array (most probe misses then never leave L2). */
 hq_status hq_hash_info(hq_ctx* ctx, const hq_hash* h, hq_hash_meta* meta);  /* syncs, reports build faults */
 /* Multi-GPU glue: raw device view of the slot array (to broadcast it with NCCL)
  * and import of such a buffer on another device (borrowed, caller keeps it). */

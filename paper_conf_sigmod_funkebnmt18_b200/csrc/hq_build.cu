@@ -244,6 +244,7 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   h->meta.bytes = cap * words * 4;
   h->meta.layout = direct ? HQ_HT_DIRECT : HQ_HT_LINEAR;
   h->meta.key_min = kmin;
+  h->meta.key_max = range > 0 ? (int32_t)(kmin + range - 1) : (int32_t)kmin - 1;  // empty range when unknown
   const int64_t nw = cap * words;
   const int fgrid = (int)std::max<int64_t>(1, std::min<int64_t>((nw + 255) / 256, (int64_t)ctx->num_sms * 8));
   ctx->launches++;
@@ -257,7 +258,7 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   b.dmin = (int32_t)kmin;
   if (b.n > 0) { ctx->launches++; hq_build_hash_kernel<<<grid, 256, 0, ctx->stream>>>(b); }
   HQ_CUDA(cudaGetLastError());
-  if (direct) hq_build_compact(ctx, h);
+  hq_build_compact(ctx, h);
 }
 
 namespace {
@@ -271,6 +272,16 @@ __global__ void hq_compact_bitmap_kernel(const uint32_t* slots, long long range,
       if (i < range && (int)slots[i] != INT_MIN) bits |= 1u << b;
     }
     out[w] = bits;
+  }
+}
+// key-range bitmap of a linear table: one bit per key in [kmin, kmin + range)
+__global__ void hq_prefilter_kernel(const uint32_t* slots, long long cap, int words, int kmin, long long range,
+                                    uint32_t* bm) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < cap; i += (long long)gridDim.x * blockDim.x) {
+    const int k = (int)slots[i * words];
+    if (k == INT_MIN) continue;
+    const long long d = (long long)k - kmin;
+    if (d >= 0 && d < range) atomicOr(bm + (d >> 5), 1u << (d & 31));
   }
 }
 // one byte per key: payload0 - pay_min, 0xFF = absent (8-B slots {key, payload})
@@ -295,6 +306,23 @@ __global__ void hq_compact_u8_kernel(const uint32_t* slots, long long range, int
 void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
   h->ckind = 0;
   h->cbytes = 0;
+  h->pf_words = 0;
+  if (h->meta.layout == HQ_HT_LINEAR) {
+    // exact key-range bitmap in front of the slot array (semi-join prefilter)
+    const long long range = (long long)h->meta.key_max - h->meta.key_min + 1;
+    const long long words = (range + 31) / 32;
+    if (range <= 0 || words * 4 > (64LL << 20)) return;
+    h->prefilter = DevBuf(ctx, (size_t)words * 4 + 16);
+    HQ_CUDA(cudaMemsetAsync(h->prefilter.p, 0, (size_t)words * 4 + 16, ctx->stream));
+    const long long cap = h->meta.capacity;
+    const int grid = (int)std::max<long long>(1, std::min<long long>((cap + 255) / 256, (long long)ctx->num_sms * 8));
+    ctx->launches++;
+    hq_prefilter_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, cap, h->meta.slot_words, (int)h->meta.key_min,
+                                                       range, h->prefilter.as<uint32_t>());
+    HQ_CUDA(cudaGetLastError());
+    h->pf_words = words;
+    return;
+  }
   if (h->meta.layout != HQ_HT_DIRECT) return;
   const long long range = h->meta.capacity;
   int kind = 0;

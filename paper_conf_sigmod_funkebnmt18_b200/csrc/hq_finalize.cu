@@ -100,15 +100,16 @@ __device__ __forceinline__ bool row_less(const KSort& s, int a, int b) {
 // Each block sorts one chunk of <= SORT_CHUNK indices (bitonic network in
 // shared memory) and keeps its first `keep` rows.
 __global__ void __launch_bounds__(1024) hq_chunk_sort_kernel(const __grid_constant__ KSort s, const int* in, long long n,
-                                                             int* out, int keep) {
+                                                             int* out, int keep, int net) {
+  // net: power-of-two network size (<= SORT_CHUNK); chunks of `net` rows per block
   __shared__ int idx[SORT_CHUNK];
-  const long long base = (long long)blockIdx.x * SORT_CHUNK;
-  const int cnt = (int)(n - base < SORT_CHUNK ? n - base : SORT_CHUNK);
-  for (int i = threadIdx.x; i < SORT_CHUNK; i += blockDim.x) idx[i] = i < cnt ? (in ? in[base + i] : (int)(base + i)) : -1;
+  const long long base = (long long)blockIdx.x * net;
+  const int cnt = (int)(n - base < net ? n - base : net);
+  for (int i = threadIdx.x; i < net; i += blockDim.x) idx[i] = i < cnt ? (in ? in[base + i] : (int)(base + i)) : -1;
   __syncthreads();
-  for (int k = 2; k <= SORT_CHUNK; k <<= 1) {
+  for (int k = 2; k <= net; k <<= 1) {
     for (int j = k >> 1; j > 0; j >>= 1) {
-      for (int i = threadIdx.x; i < SORT_CHUNK; i += blockDim.x) {
+      for (int i = threadIdx.x; i < net; i += blockDim.x) {
         const int l = i ^ j;
         if (l > i) {
           const int a = idx[i], b = idx[l];
@@ -144,6 +145,13 @@ __global__ void hq_iota_kernel(int* idx, long long n, long long valid) {
 __global__ void hq_gather_kernel(const long long* src, const int* idx, long long n, long long* dst) {
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
     dst[i] = src[idx[i]];
+}
+
+// smallest power-of-two bitonic network (>= 32) that holds n rows
+int net_for(long long n) {
+  int v = 32;
+  while (v < n && v < SORT_CHUNK) v <<= 1;
+  return v;
 }
 
 int grid_for(hq_ctx* ctx, long long n) {
@@ -242,9 +250,10 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
       while (true) {
         const int64_t chunks = (cur_n + SORT_CHUNK - 1) / SORT_CHUNK;
         const int kp = chunks == 1 ? (int)std::min<int64_t>(cur_n, SORT_CHUNK) : keep;
+        const int net = chunks == 1 ? net_for(cur_n) : SORT_CHUNK;
         int* dst = bufs[which];
         ctx->launches++;
-        hq_chunk_sort_kernel<<<(unsigned)chunks, 1024, 0, ctx->stream>>>(s, cur, cur_n, dst, kp);
+        hq_chunk_sort_kernel<<<(unsigned)chunks, std::min(1024, net), 0, ctx->stream>>>(s, cur, cur_n, dst, kp, net);
         HQ_CUDA(cudaGetLastError());
         cur = dst;
         cur_n = chunks * kp;
@@ -254,7 +263,8 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
       sorted = (int*)cur;
     } else if (n <= SORT_CHUNK) {
       ctx->launches++;
-      hq_chunk_sort_kernel<<<1, 1024, 0, ctx->stream>>>(s, nullptr, n, ia.as<int>(), SORT_CHUNK);
+      const int net = net_for(n);
+      hq_chunk_sort_kernel<<<1, std::min(1024, net), 0, ctx->stream>>>(s, nullptr, n, ia.as<int>(), SORT_CHUNK, net);
       HQ_CUDA(cudaGetLastError());
       sorted = ia.as<int>();
     } else {

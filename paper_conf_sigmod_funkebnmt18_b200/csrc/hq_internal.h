@@ -122,6 +122,9 @@ struct hq_hash : RefObj {
   DevBuf compact;
   int ckind = 0;
   int64_t cbytes = 0;
+  // linear tables: exact bitmap over [key_min, key_max] (prefilter before the slots)
+  DevBuf prefilter;
+  int64_t pf_words = 0;
 };
 void hq_build_compact(hq_ctx* ctx, hq_hash* h);  // derive hq_hash::compact from the slots
 
@@ -182,6 +185,9 @@ struct KProbe {
   int32_t pay_min;   // ckind 2: payload = byte + pay_min
   uint32_t cbytes;
   uint32_t smem_off; // generated kernels: byte offset of the staged compact table (0 = not staged)
+  const uint32_t* pf;  // linear tables: key-range bitmap (NULL = none)
+  int32_t pf_min;
+  uint32_t pf_range;
 };
 struct KCompute {
   int16_t dst;

@@ -31,6 +31,7 @@ using namespace hqk;
     const char* col[16];                                                                                       \
     const unsigned* ht[8];                                                                                     \
     const void* ctab[8];                                                                                       \
+    const unsigned* pf[8];                                                                                     \
     long long* gtab;                                                                                           \
     unsigned long long gmask;                                                                                  \
     int glog2, pad;                                                                                            \
@@ -202,8 +203,13 @@ struct Gen {
       o << "        }\n";
     } else {
       const int G = W == 1 ? 4 : (W == 2 ? 2 : 1);
-      o << "          const bool ok_ = ((mask >> r) & 1u) && k_ > (long long)HQ_INT_MIN && k_ <= (long long)HQ_INT_MAX;\n"
-        << "          pos_[r] = ((u32)(int)k_ * 0x9E3779B1u) >> " << (32 - pr.log2cap) << "; if (ok_) pend_ |= 1u << r; }\n"
+      o << "          bool ok_ = ((mask >> r) & 1u) && k_ > (long long)HQ_INT_MIN && k_ <= (long long)HQ_INT_MAX;\n";
+      if (pr.pf) {  // exact key-range bitmap first: misses mostly stop here (L2-resident)
+        o << "          if (ok_) { const long long d_ = k_ - (" << pr.pf_min << "LL);\n"
+          << "            ok_ = d_ >= 0 && d_ < " << pr.pf_range << "LL && ((__ldg(p.pf[" << idx
+          << "] + (d_ >> 5)) >> (d_ & 31)) & 1u); }\n";
+      }
+      o << "          pos_[r] = ((u32)(int)k_ * 0x9E3779B1u) >> " << (32 - pr.log2cap) << "; if (ok_) pend_ |= 1u << r; }\n"
         << "        while (pend_) {\n          int4 sl_[R];\n"
         << "#pragma unroll\n          for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) sl_[r] = __ldg((const int4*)ht_ + pos_[r] / "
         << G << ");\n"
@@ -501,8 +507,17 @@ CUfunction compile(hq_ctx* ctx, const std::string& src) {
     auto it = g_cache.find(key);
     if (it != g_cache.end()) return it->second;
   }
+  // HQ_JIT_DUMP=<dir>: write each generated source there (ncu --resolve-source-file)
+  std::string name = "hq_jit_kernel.cu";
+  if (const char* dir = getenv("HQ_JIT_DUMP")) {
+    name = std::string(dir) + "/hq_jit_" + std::to_string(std::hash<std::string>{}(src) % 1000000007ULL) + ".cu";
+    if (FILE* f = fopen(name.c_str(), "w")) {
+      fwrite(src.data(), 1, src.size(), f);
+      fclose(f);
+    }
+  }
   nvrtcProgram prog;
-  if (nvrtcCreateProgram(&prog, src.c_str(), "hq_jit_kernel.cu", 0, nullptr, nullptr) != NVRTC_SUCCESS)
+  if (nvrtcCreateProgram(&prog, src.c_str(), name.c_str(), 0, nullptr, nullptr) != NVRTC_SUCCESS)
     HQ_THROW(HQ_ERR_CUDA, "nvrtcCreateProgram failed");
   const char* opts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "--device-int128"};
   const nvrtcResult rc = nvrtcCompileProgram(prog, 4, opts);
@@ -561,6 +576,7 @@ void hq_jit_launch(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
   for (int i = 0; i < MAX_PROBES; ++i) {
     jp.ht[i] = kp.probes[i].slots;
     jp.ctab[i] = kp.probes[i].compact;
+    jp.pf[i] = kp.probes[i].pf;
   }
   jp.gtab = kp.gtab;
   jp.gmask = kp.gmask;

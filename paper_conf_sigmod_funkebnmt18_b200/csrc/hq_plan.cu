@@ -132,6 +132,9 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.pay_min = op.ht->meta.pay_min;
       pr.cbytes = (uint32_t)op.ht->cbytes;
       pr.smem_off = 0;
+      pr.pf = op.ht->pf_words ? op.ht->prefilter.as<uint32_t>() : nullptr;
+      pr.pf_min = (int32_t)op.ht->meta.key_min;
+      pr.pf_range = (uint32_t)((int64_t)op.ht->meta.key_max - op.ht->meta.key_min + 1);
       pr.words = (uint8_t)op.ht->meta.slot_words;
       pr.mode = (uint8_t)op.mode;
       const int npay = op.mode == HQ_PROBE_INNER ? op.npayload : 0;

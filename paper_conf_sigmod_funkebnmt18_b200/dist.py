@@ -83,7 +83,7 @@ class DistributedEngine(Engine):
             ptr, _ = h.device_view()
             buf = device_view(ptr, int(m.bytes))
             meta = [m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout,
-                    m.pay_min, m.pay_max]
+                    m.pay_min, m.pay_max, m.key_max]
         else:
             meta, buf = None, None
         meta, buf = broadcast_blob(meta, buf, 4, self.root, self.device)
@@ -91,7 +91,7 @@ class DistributedEngine(Engine):
             return h
         hm = hq.HashMeta()
         (hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout,
-         hm.pay_min, hm.pay_max) = meta[:9]
+         hm.pay_min, hm.pay_max, hm.key_max) = meta[:10]
         return self.ctx.import_hash(hm, buf.data_ptr(), keep=buf)
 
     def hash(self, table, key, payload=(), preds=(), expected_rows=0) -> hq.Hash:
