@@ -296,6 +296,8 @@ typedef struct {
   int64_t qualifying_rows;  /* rows that reached the sink (COUNT(*)) */
   int32_t ncols;
   int32_t types[HQ_MAX_KEYS + HQ_MAX_AGGS]; /* hq_type of each result column */
+  int32_t segment_rows;     /* MATERIALISE: fact rows per LRGP segment (the kernel's tile);
+                               output is ordered within a segment's rows, segments permuted */
 } hq_result_info;
 hq_status hq_result_info_get(hq_ctx* ctx, hq_result* r, hq_result_info* out); /* syncs */
 /* Copy the result into caller host buffers host_cols[c] (capacity_rows rows

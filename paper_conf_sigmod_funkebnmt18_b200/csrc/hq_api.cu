@@ -350,6 +350,7 @@ hq_status hq_result_info_get(hq_ctx* ctx, hq_result* r, hq_result_info* out) {
     out->qualifying_rows = r->qualifying;
     out->ncols = r->ncols;
     for (int c = 0; c < r->ncols; ++c) out->types[c] = r->types[c];
+    out->segment_rows = r->sink == HQ_SINK_MATERIALISE ? r->segment_rows : 0;
   });
 }
 

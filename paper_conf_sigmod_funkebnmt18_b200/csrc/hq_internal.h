@@ -271,6 +271,7 @@ struct hq_result : RefObj {
   // materialise
   std::vector<DevBuf> outcols;
   int64_t capacity = 0;
+  int32_t segment_rows = 0;   // tile rows of the launch that wrote it
   // finalized AGG rows
   bool finalized = false;
   bool checked = false;

@@ -284,7 +284,7 @@ std::string generate(const KPlan& kp) {
   o << "extern \"C\" __global__ void __launch_bounds__((NW + 1) * 32, 1) hq_jit_kernel(const __grid_constant__ JParams p) {\n"
     << "  extern __shared__ __align__(128) char smem[];\n"
     << "  u64* full = (u64*)smem; u64* empty = full + 10;\n"
-    << "  u64* s_base = (u64*)(empty + 10); int* s_wtot = (int*)(s_base + 16); i64* s_red = (i64*)(s_wtot + 16);\n"
+    << "  u64* s_base = (u64*)(empty + 10); int* s_wtot = (int*)(s_base + 32); i64* s_red = (i64*)(s_wtot + 32);\n"
     << "  char* sagg = smem + OFF_AGG; char* stages = smem + OFF_STAGE;\n"
     << "  (void)s_base; (void)s_wtot; (void)s_red; (void)sagg;\n"
     << "  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n"
@@ -390,24 +390,36 @@ std::string generate(const KPlan& kp) {
     } else {
       std::vector<std::string> vv;
       for (int a = 0; a < kp.naggs; ++a) vv.push_back(aggval(a));
-      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) {\n"
-        << "        const bool live_ = (mask >> r) & 1u; const u32 act_ = __ballot_sync(HQ_FULL, live_);\n"
-        << "        if (!act_) continue;\n"
-        << "        i64 v_[NAGGS > 0 ? NAGGS : 1];\n";
-      for (int a = 0; a < kp.naggs; ++a) o << "        v_[" << a << "] = " << vv[a] << ";\n";
+      // warp compaction: the warp's live rows (over all R row slots) move into
+      // consecutive lanes (ballot prefix + __fns + shuffles), so the table updates
+      // of a tile run as parallel rounds of 32 rows instead of R serial slots
+      o << "      i64 va_[NAGGS > 0 ? NAGGS : 1][R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) {";
+      for (int a = 0; a < kp.naggs; ++a) o << " va_[" << a << "][r] = " << vv[a] << ";";
+      o << " }\n"
+        << "      u32 bm_[R]; int pre_[R + 1]; pre_[0] = 0;\n"
+        << "#pragma unroll\n      for (int r = 0; r < R; ++r) { bm_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); pre_[r + 1] = pre_[r] + __popc(bm_[r]); }\n"
+        << "      for (int i0_ = 0; i0_ < pre_[R]; i0_ += 32) {\n"
+        << "        const int t_ = i0_ + lane; const bool live_ = t_ < pre_[R];\n"
+        << "        int rr_ = 0; u32 m_ = bm_[0]; int k_ = t_;\n"
+        << "#pragma unroll\n        for (int r = 1; r < R; ++r) if (t_ >= pre_[r]) { rr_ = r; m_ = bm_[r]; k_ = t_ - pre_[r]; }\n"
+        << "        const int src_ = live_ ? (int)__fns(m_, 0, k_ + 1) : lane;\n"
+        << "        u64 key_ = 0; i64 v_[NAGGS > 0 ? NAGGS : 1];\n"
+        << "#pragma unroll\n        for (int r = 0; r < R; ++r) { const u64 kx_ = __shfl_sync(HQ_FULL, gk_[r], src_); if (r == rr_) key_ = kx_;\n"
+        << "#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) { const i64 x_ = __shfl_sync(HQ_FULL, va_[a][r], src_); if (r == rr_) v_[a] = x_; } }\n"
+        << "        const u32 act_ = __ballot_sync(HQ_FULL, live_);\n";
       if (c2) {
-        o << "        if (live_) group_update(p, sagg, gk_[r], false, 1ull, v_);\n      }\n";
+        o << "        if (live_) group_update(p, sagg, key_, false, 1ull, v_);\n      }\n";
       } else {
         o << "        const bool sparse_ = __popc(act_) <= 4;\n"
-          << "        const u64 mk_ = live_ ? gk_[r] : HQ_EMPTY_KEY;\n"
+          << "        const u64 mk_ = live_ ? key_ : HQ_EMPTY_KEY;\n"
           << "        const u32 peers_ = sparse_ ? ((1u << lane) & act_) : (__match_any_sync(HQ_FULL, mk_) & act_);\n"
           << "        const bool single_ = live_ && __popc(peers_) == 1;\n"
-          << "        if (single_) group_update(p, sagg, gk_[r], true, 1ull, v_);\n"
+          << "        if (single_) group_update(p, sagg, key_, true, 1ull, v_);\n"
           << "        u32 multi_ = act_ & ~__ballot_sync(HQ_FULL, single_);\n"
           << "        while (multi_) {\n          const int leader_ = __ffs(multi_) - 1;\n"
           << "          const u32 grp_ = __shfl_sync(HQ_FULL, peers_, leader_); const bool mine_ = (grp_ >> lane) & 1u;\n"
           << "          i64 w_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) w_[a] = warp_reduce(AGG_FN[a], mine_ ? v_[a] : agg_identity(AGG_FN[a]));\n"
-          << "          if (lane == leader_) group_update(p, sagg, gk_[r], true, (u64)__popc(grp_), w_);\n"
+          << "          if (lane == leader_) group_update(p, sagg, key_, true, (u64)__popc(grp_), w_);\n"
           << "          multi_ &= ~grp_;\n        }\n      }\n";
       }
     }
@@ -472,12 +484,12 @@ std::string generate(const KPlan& kp) {
   } else if (sk == 1 && kp.smode == SM_DENSE) {
     o << "  consumer_bar();\n  { const i64* t_ = (const i64*)sagg;\n"
       << "    for (u32 g = threadIdx.x; g < SMEM_CAP; g += NW * 32) { const i64* e_ = t_ + (u64)g * VWORDS;\n"
-      << "      if (e_[0] != 0) { i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) vals_[a] = e_[1 + a];\n"
+      << "      if (e_[0] != 0) { i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) vals_[a] = AGG_FN[a] == F_COUNT ? e_[0] : e_[1 + a];\n"
       << "        group_update(p, sagg, g, false, (u64)e_[0], vals_); } } }\n";
   } else if (sk == 1 && kp.smode == SM_HASH) {
     o << "  consumer_bar();\n  { const u64* k_ = (const u64*)sagg; const i64* t_ = (const i64*)sagg + SMEM_CAP;\n"
       << "    for (u32 h = threadIdx.x; h < SMEM_CAP; h += NW * 32) if (k_[h] != HQ_EMPTY_KEY) { const i64* e_ = t_ + (u64)h * VWORDS;\n"
-      << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = e_[1 + a];\n"
+      << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = AGG_FN[a] == F_COUNT ? e_[0] : e_[1 + a];\n"
       << "      group_update(p, sagg, k_[h], false, (u64)e_[0], vals_); } }\n";
   }
   o << "}\n";
@@ -557,9 +569,43 @@ namespace {
 thread_local CUfunction t_last_fn = nullptr;  // kernel compiled by the last hq_jit_prepare
 }
 
+namespace {
+// The generated source depends on the plan's shape and constants, not on its
+// runtime arguments (pointers, row range): key the kernel cache on the plan
+// bytes with pointers reduced to null / non-null, so a repeated query skips
+// source generation entirely.
+std::string plan_key(const KPlan& kp) {
+  KPlan k = kp;
+  auto nz = [](const void* p) { return (const char*)(p ? 1 : 0); };
+  k.row_begin = k.row_end = 0;
+  for (auto& c : k.cols) c.ptr = nz(c.ptr);
+  for (auto& pr : k.probes) {
+    pr.slots = (const uint32_t*)nz(pr.slots);
+    pr.compact = nz(pr.compact);
+    pr.pf = (const uint32_t*)nz(pr.pf);
+  }
+  k.gtab = (long long*)nz(k.gtab);
+  for (auto& o : k.out_ptr) o = (void*)nz(o);
+  k.counter = (unsigned long long*)nz(k.counter);
+  k.err = (int*)nz(k.err);
+  return std::string((const char*)&k, sizeof(k));
+}
+std::map<std::pair<int, std::string>, CUfunction> g_plan_cache;
+}  // namespace
+
 void hq_jit_prepare(hq_ctx* ctx, const KPlan& kp, size_t smem) {
-  const std::string src = generate(kp);
-  CUfunction fn = compile(ctx, src);
+  const auto key = std::make_pair(ctx->device, plan_key(kp));
+  CUfunction fn = nullptr;
+  {
+    std::lock_guard<std::mutex> gl(g_mu);
+    auto it = g_plan_cache.find(key);
+    if (it != g_plan_cache.end()) fn = it->second;
+  }
+  if (!fn) {
+    fn = compile(ctx, generate(kp));
+    std::lock_guard<std::mutex> gl(g_mu);
+    g_plan_cache[key] = fn;
+  }
   if (driver().setattr(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, (int)smem) != CUDA_SUCCESS)
     HQ_THROW(HQ_ERR_CUDA, "cuFuncSetAttribute failed");
   t_last_fn = fn;

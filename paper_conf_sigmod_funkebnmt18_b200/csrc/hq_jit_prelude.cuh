@@ -159,9 +159,12 @@ __device__ __forceinline__ void group_update(const JParams& p, char* sagg, u64 k
                                              const i64 (&vals)[NAGGS > 0 ? NAGGS : 1]) {
   const u32 sa = (local && SMODE != 0) ? local_locate(sagg, key) : 0u;
   if (sa) {
-    s_add64(sa, (i64)cnt);
+    // the per-CTA count of a group stays below 2^32: a return-less 32-bit red on
+    // the low word; COUNT aggregates are read from it at the merge
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(sa), "r"((u32)cnt) : "memory");
 #pragma unroll
-    for (int a = 0; a < NAGGS; ++a) s_agg(AGG_FN[a], sa + 8u * (1 + a), vals[a], cnt);
+    for (int a = 0; a < NAGGS; ++a)
+      if (AGG_FN[a] != F_COUNT) s_agg(AGG_FN[a], sa + 8u * (1 + a), vals[a], cnt);
     return;
   }
   i64* e = global_locate(p, key);

@@ -18,7 +18,8 @@ int64_t next_pow2(int64_t x) {
 }
 uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
 
-constexpr uint32_t MISC_BYTES = 2048;  // barriers, block-scan and reduction scratch
+// barriers, block-scan and reduction scratch: full/empty[10], base[32], wtot[32], red[32][9]
+constexpr uint32_t MISC_BYTES = 3072;
 
 struct RegInfo {
   int width = 0;       // 0 = undefined
@@ -293,6 +294,15 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     for (int k = 0; k < HQ_MAX_TMP; ++k) tmp_row += (uint32_t)regs[HQ_MAX_COLS + k].width;
 
   kp.nw = kp.smode == SM_LANE ? LANE_NW : NW;
+  int force_R = 0;
+  if (jit && kp.smode != SM_LANE) {
+    // generated kernels need fewer registers: 31 consumer warps x 2 rows per lane
+    // hides the probe/atomic latency best (sweep on B200, profiles/r01)
+    kp.nw = 31;
+    force_R = 2;
+    if (const char* e = getenv("HQ_JIT_NW")) kp.nw = std::max(1, std::min(31, atoi(e)));
+    if (const char* e = getenv("HQ_JIT_R")) force_R = atoi(e);
+  }
   // Generated kernels stage small compact probe tables (bitmaps / byte arrays of
   // direct tables) in shared memory, earliest probes first (they see the most
   // rows), as long as the TMA ring keeps >= 3 stages.
@@ -314,7 +324,8 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   for (;;) {
     uint32_t tab_total = 0;
     for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
-    for (int R : {4, 2}) {
+    for (int R : {8, 4, 2, 1}) {
+      if (force_R ? R != force_R : (R == 8 || R == 1)) continue;
       const uint32_t T = (uint32_t)(kp.nw * 32 * R);
       const uint32_t off_tmp = MISC_BYTES;
       const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
@@ -323,7 +334,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
       if (off_stage >= ctx->max_smem) continue;
       const int S = (int)std::min<int64_t>(MAX_STAGES, (ctx->max_smem - off_stage) / stride);
-      if (S >= 3 || (R == 2 && S >= 2 && nstaged == 0)) {
+      if (S >= 3 || (R <= 2 && S >= 2 && nstaged == 0)) {
         chosen_R = R;
         kp.R = R;
         kp.tile_rows = (int32_t)T;
@@ -342,6 +353,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     --nstaged;  // give the last staged table back to the ring
   }
   if (!chosen_R) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: rows too wide for the shared-memory stage ring");
+  r->segment_rows = kp.tile_rows;
   {
     uint32_t off = kp.off_tab;
     for (int i = 0; i < nstaged; ++i) {

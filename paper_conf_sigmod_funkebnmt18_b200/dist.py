@@ -49,8 +49,9 @@ def broadcast_blob(meta: Optional[Sequence[int]], buf: Optional[torch.Tensor], n
 
 
 def reduce_partials(t: torch.Tensor, root: int) -> None:
-    """Exact integer SUM of the ranks' partial aggregates onto the root."""
-    dist.reduce(t, dst=root, op=dist.ReduceOp.SUM)
+    """Exact integer SUM of the ranks' partial aggregates (one all-reduce: NCCL
+    over NVLink on the GPUs; gloo in the CPU tests).  Only the root finalizes."""
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
 
 
 class _CudaView:

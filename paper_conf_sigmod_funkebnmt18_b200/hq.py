@@ -95,7 +95,7 @@ class Plan(ctypes.Structure):
 
 class ResultInfo(ctypes.Structure):
     _fields_ = [("nrows", ctypes.c_int64), ("qualifying_rows", ctypes.c_int64), ("ncols", ctypes.c_int32),
-                ("types", ctypes.c_int32 * (MAX_KEYS + MAX_AGGS))]
+                ("types", ctypes.c_int32 * (MAX_KEYS + MAX_AGGS)), ("segment_rows", ctypes.c_int32)]
 
 
 ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)

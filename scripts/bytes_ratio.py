@@ -1,0 +1,88 @@
+#!/usr/bin/env python
+"""DRAM bytes of the fused plan vs the operator-at-a-time plan of the same
+query (the BASELINE.json metric's second half).
+
+Runs every query once per mode under
+  ncu --cache-control all --clock-control none --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum
+and sums the metrics over all kernels of the execution (as the paper summed
+per-kernel nvprof metrics), split into the fact pipeline and the
+rest (hash builds, finalize).  Writes profiles/<round>/bytes_ratio.{json,md}.
+
+    python scripts/bytes_ratio.py --sf 10 --round r01      # on the GPU box
+"""
+import argparse
+import csv
+import io
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+QUERIES = ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q12", "ssb_q13", "ssb_q31", "ssb_q41", "tpch_q3"]
+SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-9, "us": 1e-6, "ms": 1e-3, "s": 1,
+         "nsecond": 1e-9, "usecond": 1e-6, "msecond": 1e-3}
+PIPELINE = ("hq_jit_kernel", "hq_fused_pipeline_kernel", "hq_oaat", "cub::", "DeviceScan")
+
+
+def run(q, sf, mode):
+    log = os.path.join(ROOT, "gpurun_out", f"ncu_{q}_{mode}.csv")
+    cmd = ["ncu", "--cache-control", "all", "--clock-control", "none", "--metrics",
+           "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum", "--csv", "--log-file", log,
+           sys.executable, os.path.join(ROOT, "scripts", "profile_query.py"), "--query", q, "--sf", str(sf),
+           "--reps", "1", "--exec", mode]
+    subprocess.run(cmd, capture_output=True, text=True, timeout=1800)
+    rows = list(csv.reader(io.StringIO(open(log).read())))
+    hi = next(i for i, r in enumerate(rows) if r and r[0] == "ID")
+    h = rows[hi]
+    ik, im, iu, iv = h.index("Kernel Name"), h.index("Metric Name"), h.index("Metric Unit"), h.index("Metric Value")
+    tot = {"pipeline": {}, "other": {}}
+    kernels = set()
+    for r in rows[hi + 1:]:
+        part = "pipeline" if any(p in r[ik] for p in PIPELINE) else "other"
+        v = float(r[iv].replace(",", "")) * SCALE.get(r[iu], 1.0)
+        tot[part][r[im]] = tot[part].get(r[im], 0.0) + v
+        kernels.add((part, r[ik].split("(")[0][:50]))
+    return tot, sorted(kernels)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--sf", type=float, default=10)
+    ap.add_argument("--round", default="r01")
+    ap.add_argument("--queries", default=",".join(QUERIES))
+    a = ap.parse_args()
+    out = {}
+    for q in a.queries.split(","):
+        out[q] = {}
+        for mode in ("fused", "oaat"):
+            tot, kernels = run(q, a.sf, mode)
+            out[q][mode] = {part: {"dram_bytes": d.get("dram__bytes_read.sum", 0) + d.get("dram__bytes_write.sum", 0),
+                                   "time_s": d.get("gpu__time_duration.sum", 0)} for part, d in tot.items()}
+            out[q][mode]["kernels"] = kernels
+        print(q, json.dumps({m: {p: out[q][m][p] for p in ("pipeline", "other")} for m in ("fused", "oaat")}), flush=True)
+    d = os.path.join(ROOT, "gpurun_out")  # copied to profiles/<round>/ after the run
+    os.makedirs(d, exist_ok=True)
+    with open(os.path.join(d, f"bytes_ratio_sf{a.sf:g}.json"), "w") as f:
+        json.dump({"sf": a.sf, "cache_control": "all", "queries": out}, f, indent=1)
+    lines = [f"DRAM bytes (ncu dram__bytes_read.sum + dram__bytes_write.sum, --cache-control all) summed over all kernels "
+             f"of one query execution at SF {a.sf:g}; 'pipeline' = the fact-table pipeline kernels (fused: one generated "
+             "kernel; op-at-a-time: filter/probe/compute/scan/compact/gather/agg kernels), 'all' adds hash builds and finalize.",
+             "", "| query | fused pipeline GB | OAAT pipeline GB | bytes ratio (pipeline) | fused all GB | OAAT all GB | "
+             "bytes ratio (all) | fused pipeline ms | OAAT pipeline ms | kernel-time ratio |",
+             "|---|---|---|---|---|---|---|---|---|---|"]
+    for q, m in out.items():
+        fp, op = m["fused"]["pipeline"], m["oaat"]["pipeline"]
+        fa = fp["dram_bytes"] + m["fused"]["other"]["dram_bytes"]
+        oa = op["dram_bytes"] + m["oaat"]["other"]["dram_bytes"]
+        lines.append(f"| {q} | {fp['dram_bytes'] / 1e9:.3f} | {op['dram_bytes'] / 1e9:.3f} | "
+                     f"{op['dram_bytes'] / max(fp['dram_bytes'], 1):.2f}x | {fa / 1e9:.3f} | {oa / 1e9:.3f} | "
+                     f"{oa / max(fa, 1):.2f}x | {fp['time_s'] * 1e3:.3f} | {op['time_s'] * 1e3:.3f} | "
+                     f"{op['time_s'] / max(fp['time_s'], 1e-12):.2f}x |")
+    with open(os.path.join(d, f"bytes_ratio_sf{a.sf:g}.md"), "w") as f:
+        f.write("\n".join(lines) + "\n")
+    print("\n".join(lines))
+
+
+if __name__ == "__main__":
+    main()

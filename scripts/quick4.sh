@@ -1,0 +1,5 @@
+cd $GRAFT_REPO_ROOT
+timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -5
+timeout 300 python scripts/ablate_q31.py 10
+timeout 300 python scripts/ablate_q41.py 10 | tail -3
+for q in ssb_q31 ssb_q41 tpch_q3 micro_groupby; do timeout 120 python scripts/profile_query.py --query $q --sf 10 --reps 3 2>&1 | tail -1; done

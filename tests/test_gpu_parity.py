@@ -216,7 +216,8 @@ def test_lrgp_positions_segment_ordered(ctx):
     assert res.qualifying() == len(sel) == len(out)
     assert np.array_equal(np.sort(out), sel)  # dense: every slot written exactly once
     # each tile's selected rows occupy one contiguous segment, in row order
-    T = 2048
+    T = res.info().segment_rows
+    assert T > 0 and n > 10 * T
     pos = np.empty(n, np.int64)
     pos[out] = np.arange(len(out))
     tile = sel // T
