@@ -159,6 +159,35 @@ def cpu_baseline(qname, host, n_fact, budget_s=30.0):
                       f"{cores} threads, {dt:.2f} s"}
 
 
+def oaat_timing(qname, host, local, fused_ms, steps=2):
+    """The same query executed operator-at-a-time (Fig 6 baseline, HQ_EXEC_OAAT):
+    device time per step with CUDA events, vs the fused step."""
+    import torch
+    from paper_conf_sigmod_funkebnmt18_b200 import hq
+    from paper_conf_sigmod_funkebnmt18_b200.engine import Engine
+    from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
+    q = QUERIES[qname]
+    dev = torch.device("cuda", local)
+    ctx = hq.Context(local)
+    dtab = {t: {c: torch.from_numpy(np.asarray(a)).to(dev) for c, a in cols.items()} for t, cols in host.items()}
+    tables = {t: ctx.load_columns(cols) for t, cols in dtab.items()}
+    E = Engine(ctx, tables, exec_mode=hq.EXEC_OAAT)
+    q.execute(E)
+    stream = torch.cuda.current_stream(dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(steps):
+        q.execute(E)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    del tables, dtab, E
+    ctx.close()
+    torch.cuda.empty_cache()
+    return {"ms_per_step": ms, "fused_speedup": ms / fused_ms, "steps": steps, "exec": "HQ_EXEC_OAAT"}
+
+
 # --------------------------------------------------------- device measurement
 def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, host=None):
     import torch
@@ -278,7 +307,7 @@ def roofline(q, local_rows, kernel_ms, peak, peak_src):
     achieved = local_rows * bpr / (kernel_ms / 1e3) / 1e9
     return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
             "traffic": traffic, "algorithmic_bytes": local_rows * bpr, "bytes_per_row": bpr,
-            "kernel": "hq_fused_pipeline_kernel", "kernel_ms": kernel_ms, "peak_source": peak_src}
+            "kernel": "hq_jit_kernel (NVRTC-generated fused pipeline)", "kernel_ms": kernel_ms, "peak_source": peak_src}
 
 
 # ----------------------------------------------------------------- arms
@@ -344,6 +373,14 @@ def run_hq(args):
         line["roofline"]["kernel_share_of_step"] = r["kernel_ms"] / r["ms"]
         if world == 1:
             line["cpu_baseline"] = cpu_baseline(args.query, r["host"], r["rows"])
+            line["oaat"] = oaat_timing(args.query, r["host"], local, r["ms"])
+        bp = os.path.join(ROOT, "profiles", "r01", "bytes_ratio_sf10.json")
+        if os.path.exists(bp):
+            br = json.load(open(bp))["queries"].get(args.query)
+            if br:
+                f, o = br["fused"]["pipeline"]["dram_bytes"], br["oaat"]["pipeline"]["dram_bytes"]
+                line["dram_bytes_fused_vs_oaat"] = {"ratio": o / f, "fused_bytes": f, "oaat_bytes": o, "sf": 10,
+                                                    "source": "profiles/r01/bytes_ratio_sf10.json (ncu, --cache-control all)"}
     del r
     if world == 1 and not args.no_extra and args.query == DEFAULT_QUERY:
         per = []
