@@ -335,7 +335,8 @@ std::string generate(const KPlan& kp) {
     << "    const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
     << "    const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
     << "    const char* st = stages + (size_t)s * STAGE_STRIDE;\n"
-    << "    u32 mask = 0;\n#pragma unroll\n    for (int r = 0; r < R; ++r) { const int row = row0 + r * 32; if (row >= lo && row < hi) mask |= 1u << r; }\n"
+    << "    u32 mask = (1u << R) - 1u;\n"
+    << "    if (lo > 0 || hi < T) { mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r * 32; if (row >= lo && row < hi) mask |= 1u << r; } }\n"
     << "    if (lo > 0 || hi < T) {\n";
   for (int k = 0; k < kp.ncols; ++k) {
     const char* ty = ctype(kp.cols[k].width);
@@ -390,23 +391,30 @@ std::string generate(const KPlan& kp) {
     } else {
       std::vector<std::string> vv;
       for (int a = 0; a < kp.naggs; ++a) vv.push_back(aggval(a));
-      // warp compaction: the warp's live rows (over all R row slots) move into
-      // consecutive lanes (ballot prefix + __fns + shuffles), so the table updates
-      // of a tile run as parallel rounds of 32 rows instead of R serial slots
       o << "      i64 va_[NAGGS > 0 ? NAGGS : 1][R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) {";
       for (int a = 0; a < kp.naggs; ++a) o << " va_[" << a << "][r] = " << vv[a] << ";";
-      o << " }\n"
-        << "      u32 bm_[R]; int pre_[R + 1]; pre_[0] = 0;\n"
-        << "#pragma unroll\n      for (int r = 0; r < R; ++r) { bm_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); pre_[r + 1] = pre_[r] + __popc(bm_[r]); }\n"
-        << "      for (int i0_ = 0; i0_ < pre_[R]; i0_ += 32) {\n"
-        << "        const int t_ = i0_ + lane; const bool live_ = t_ < pre_[R];\n"
-        << "        int rr_ = 0; u32 m_ = bm_[0]; int k_ = t_;\n"
-        << "#pragma unroll\n        for (int r = 1; r < R; ++r) if (t_ >= pre_[r]) { rr_ = r; m_ = bm_[r]; k_ = t_ - pre_[r]; }\n"
-        << "        const int src_ = live_ ? (int)__fns(m_, 0, k_ + 1) : lane;\n"
-        << "        u64 key_ = 0; i64 v_[NAGGS > 0 ? NAGGS : 1];\n"
-        << "#pragma unroll\n        for (int r = 0; r < R; ++r) { const u64 kx_ = __shfl_sync(HQ_FULL, gk_[r], src_); if (r == rr_) key_ = kx_;\n"
-        << "#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) { const i64 x_ = __shfl_sync(HQ_FULL, va_[a][r], src_); if (r == rr_) v_[a] = x_; } }\n"
-        << "        const u32 act_ = __ballot_sync(HQ_FULL, live_);\n";
+      o << " }\n";
+      if (kp.R >= 4) {
+        // warp compaction: the warp's live rows (over all R row slots) move into
+        // consecutive lanes (ballot prefix, k-th set bit by popc bisection,
+        // shuffles), so table updates run as rounds of 32 rows instead of R slots
+        o << "      u32 bm_[R]; int pre_[R + 1]; pre_[0] = 0;\n"
+          << "#pragma unroll\n      for (int r = 0; r < R; ++r) { bm_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); pre_[r + 1] = pre_[r] + __popc(bm_[r]); }\n"
+          << "      for (int i0_ = 0; i0_ < pre_[R]; i0_ += 32) {\n"
+          << "        const int t_ = i0_ + lane; const bool live_ = t_ < pre_[R];\n"
+          << "        int rr_ = 0; u32 m_ = bm_[0]; int k_ = t_;\n"
+          << "#pragma unroll\n        for (int r = 1; r < R; ++r) if (t_ >= pre_[r]) { rr_ = r; m_ = bm_[r]; k_ = t_ - pre_[r]; }\n"
+          << "        int src_ = 0;\n#pragma unroll\n        for (int s_ = 16; s_ > 0; s_ >>= 1) { const int c_ = __popc((m_ >> src_) & ((1u << s_) - 1u)); if (k_ >= c_) { k_ -= c_; src_ += s_; } }\n"
+          << "        if (!live_) src_ = lane;\n"
+          << "        u64 key_ = 0; i64 v_[NAGGS > 0 ? NAGGS : 1];\n"
+          << "#pragma unroll\n        for (int r = 0; r < R; ++r) { const u64 kx_ = __shfl_sync(HQ_FULL, gk_[r], src_); if (r == rr_) key_ = kx_;\n"
+          << "#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) { const i64 x_ = __shfl_sync(HQ_FULL, va_[a][r], src_); if (r == rr_) v_[a] = x_; } }\n";
+      } else {
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) {\n"
+          << "        const bool live_ = (mask >> r) & 1u; const u64 key_ = gk_[r];\n"
+          << "        i64 v_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n";
+      }
+      o << "        const u32 act_ = __ballot_sync(HQ_FULL, live_);\n";
       if (c2) {
         o << "        if (live_) group_update(p, sagg, key_, false, 1ull, v_);\n      }\n";
       } else {
