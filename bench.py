@@ -211,7 +211,8 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
     tables = {t: ctx.load_columns(cols) for t, cols in dtab.items()}
 
     def make_engine(tbls):
-        if world > 1:
+        # HQ_FORCE_DIST=1 runs the distributed engine (broadcast + reduce) even at N=1
+        if world > 1 or os.environ.get("HQ_FORCE_DIST") == "1":
             return DistributedEngine(ctx, tbls)
         return Engine(ctx, tbls)
 
@@ -320,10 +321,10 @@ def run_reference(args):
     q = QUERIES[args.query]
     n = hqgen.table_rows(q.fact, args.sf, args.seed)
     cores = os.cpu_count() or 1
-    probe = min(n, 1_000_000)
+    probe = min(n, 2_000_000)
     host = gen_host(q, args.sf, args.seed, (0, probe), with_dims=True, pinned=False)
-    rate = probe / oracle_call(args.query, host, cores)
-    sample = int(min(n, max(probe, rate * 2.0)))  # ~2 s per step
+    est = oracle_call(args.query, host, cores) * n / probe  # upper bound: includes the map builds
+    sample = n if est <= 10.0 else max(probe, int(n * 10.0 / est))  # whole workload, or ~10 s per step
     host = gen_host(q, args.sf, args.seed, (0, sample), with_dims=True, pinned=False)
     for _ in range(args.warmup):
         oracle_call(args.query, host, cores)
@@ -351,7 +352,7 @@ def run_hq(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     torch.cuda.set_device(local)
-    if world > 1:
+    if world > 1 or os.environ.get("HQ_FORCE_DIST") == "1":
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     peak, peak_src = peaks()
     q = QUERIES[args.query]
@@ -397,7 +398,7 @@ def run_hq(args):
         line["per_query"] = per
     if rank == 0:
         print(json.dumps(line), flush=True)
-    if world > 1:
+    if dist.is_initialized():
         dist.barrier()
         dist.destroy_process_group()
 

@@ -304,7 +304,9 @@ hq_status hq_result_info_get(hq_ctx* ctx, hq_result* r, hq_result_info* out); /*
  * each, typed as hq_result_info.types).  Syncs. */
 hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int64_t capacity_rows,
                           int64_t* nrows_out);
-/* Materialised result viewed as a table (borrows the result's buffers). */
+/* Materialised or (finalized, integer-only) aggregation result viewed as a
+ * table (borrows the result's buffers): build input of a later pipeline, or the
+ * input of the root's merge pipeline for distributed hash group-bys. */
 hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out);
 /* Multi-GPU glue for dense AGG results: the raw partial-aggregate array
  * (int64, ngroups x (1+naggs): [count, agg...]) before finalization, so ranks

@@ -375,14 +375,16 @@ hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int
 hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out) {
   return guarded([&] {
     if (!ctx || !r || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
-    if (r->sink != HQ_SINK_MATERIALISE) HQ_THROW(HQ_ERR_STATE, "only materialised results can be viewed as tables");
     hq_finalize_impl(ctx, r);
+    const bool mat = r->sink == HQ_SINK_MATERIALISE;
+    for (int c = 0; c < r->ncols; ++c)
+      if (r->types[c] == HQ_F64) HQ_THROW(HQ_ERR_UNSUPPORTED, "result has fp64 (AVG) columns: not a table");
     hq_table* t = new hq_table();
     t->ctx = ctx;
     t->nrows = r->nrows;
     t->ncols = r->ncols;
     for (int c = 0; c < r->ncols; ++c) {
-      t->cols[c].ptr = r->outcols[c].p;
+      t->cols[c].ptr = mat ? r->outcols[c].p : r->rescols[c].p;
       t->cols[c].type = r->types[c];
       t->cols[c].width = hq_type_width(r->types[c]);
     }

@@ -182,7 +182,8 @@ struct KProbe {
   int16_t key_reg;
   int16_t dst[HQ_MAX_PAYLOAD];
   const void* compact;
-  int32_t pay_min;   // ckind 2: payload = byte + pay_min
+  int32_t pay_min;   // ckind 2: payload = byte + pay_min; range of payload 0 (count pass)
+  int32_t pay_max;
   uint32_t cbytes;
   uint32_t smem_off; // generated kernels: byte offset of the staged compact table (0 = not staged)
   const uint32_t* pf;  // linear tables: key-range bitmap (NULL = none)

@@ -98,6 +98,7 @@ struct Gen {
   const KPlan& kp;
   std::ostringstream o;
   std::set<int> loaded;        // registers materialised as variables
+  std::map<int, std::pair<long long, long long>> known;  // value range of probe payloads (count pass)
   std::map<int, int> stage_k;  // table column -> stage column index
   explicit Gen(const KPlan& k) : kp(k) {
     for (int c = 0; c < HQ_MAX_COLS; ++c) {
@@ -162,6 +163,7 @@ struct Gen {
     const int npay = pr.mode == HQ_PROBE_INNER ? pr.npay : 0;
     for (int k = 0; k < npay; ++k) {
       o << "      int " << var(pr.dst[k]) << "[R];\n";
+      if (k == 0 && pr.pay_min <= pr.pay_max) known[pr.dst[0]] = {pr.pay_min, pr.pay_max};
       loaded.insert(pr.dst[k]);
     }
     const std::string key = val(pr.key_reg);
@@ -375,9 +377,13 @@ std::string generate(const KPlan& kp) {
     o << "      u64 gk_[R]; bool bad_ = false;\n#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = 0;\n";
     for (int i = 0; i < kp.nkeys; ++i) {
       const std::string v = g.val(kp.key_reg[i]);
-      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kp.key_min[i])
-        << "; if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }"
-        << " gk_[r] += (u64)d_ * " << kp.key_stride[i] << "ull; }\n";
+      auto kr = g.known.find(kp.key_reg[i]);
+      const bool in_domain = kr != g.known.end() && kr->second.first >= kp.key_min[i] &&
+                             kr->second.second < kp.key_min[i] + kp.key_card[i];
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kp.key_min[i]) << ";";
+      if (!in_domain)  // payload ranges known from the build's count pass need no domain check
+        o << " if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }";
+      o << " gk_[r] += (u64)d_ * " << kp.key_stride[i] << "ull; }\n";
     }
     o << "      if (bad_) atomicOr(p.err, F_KEY_DOMAIN);\n";
     if (kp.smode == SM_LANE) {

@@ -131,6 +131,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.ckind = (uint8_t)op.ht->ckind;
       pr.compact = op.ht->compact.p;
       pr.pay_min = op.ht->meta.pay_min;
+      pr.pay_max = op.ht->meta.pay_max;
       pr.cbytes = (uint32_t)op.ht->cbytes;
       pr.smem_off = 0;
       pr.pf = op.ht->pf_words ? op.ht->prefilter.as<uint32_t>() : nullptr;

@@ -103,16 +103,75 @@ class DistributedEngine(Engine):
         h = super().hash_from(res, names, key, payload) if self.rank == self.root else None
         return self._share(h)
 
+    @staticmethod
+    def _hash_grouped(P: hq.Plan) -> bool:
+        if P.sink != hq.SINK_AGG or P.nkeys == 0:
+            return False
+        prod = 1
+        for i in range(P.nkeys):
+            prod *= P.key_card[i]
+        return prod > 65536  # libhq's dense/hash switch (hqk::DENSE_LIMIT)
+
     def run(self, pb: PlanBuilder, partitioned: bool = True) -> Optional[hq.Result]:
         if not partitioned and self.rank != self.root:
             return None
+        P = pb.plan
+        if partitioned and self._hash_grouped(P):
+            # ranks keep all their groups; ORDER BY / LIMIT run after the root's merge
+            pb.dist_order = ([(P.order_col[i], P.order_desc[i]) for i in range(P.norder)], P.limit)
+            P.norder, P.limit = 0, 0
         return super().run(pb, partitioned)
 
     def finish(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
-        """Reduce the dense partials onto the root and finalize there."""
-        ptr, nbytes = res.partials_view()
-        t = device_view(ptr, nbytes, torch.int64)
-        reduce_partials(t, self.root)
+        """Dense aggregates: one all-reduce of the partials, root finalizes.
+        Hash group-bys (e.g. TPC-H Q3 by l_orderkey): every rank finalizes its
+        groups, the rows are all-gathered to the root, which merges them with one
+        more fused GROUP BY pipeline on its GPU (and applies ORDER BY / LIMIT)."""
+        if not hasattr(pb, "dist_order"):
+            ptr, nbytes = res.partials_view()
+            t = device_view(ptr, nbytes, torch.int64)
+            reduce_partials(t, self.root)
+            if self.rank != self.root:
+                return None
+            return fetch(res, pb.result_names)
+        return self._merge_groups(res, pb)
+
+    def _merge_groups(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
+        P = pb.plan
+        names = list(pb.result_names)
+        tab = res.as_table(names)  # finalized local groups, device columns
+        cols = []
+        for c in range(len(names)):
+            ptr, _ = tab.column_ptr(c)
+            cols.append(device_view(ptr, max(tab.nrows, 1) * 8, torch.int64)[: tab.nrows])
+        qual = torch.tensor([res.qualifying()], dtype=torch.int64, device=self.device)
+        dist.all_reduce(qual)
+        n = torch.tensor([tab.nrows], dtype=torch.int64, device=self.device)
+        sizes = [torch.zeros_like(n) for _ in range(self.world)]
+        dist.all_gather(sizes, n)
+        sizes = [int(s.item()) for s in sizes]
+        m = max(max(sizes), 1)
+        merged = []
+        for c in cols:
+            pad = torch.zeros(m, dtype=torch.int64, device=self.device)
+            pad[: c.numel()] = c
+            bufs = [torch.empty_like(pad) for _ in range(self.world)]
+            dist.all_gather(bufs, pad)
+            merged.append(torch.cat([b[:s] for b, s in zip(bufs, sizes)]))
         if self.rank != self.root:
             return None
-        return fetch(res, pb.result_names)
+        mt = self.ctx.load_columns({nm: t.contiguous() for nm, t in zip(names, merged)})
+        mb = PlanBuilder(mt)
+        keys = [(names[i], P.key_min[i], P.key_card[i]) for i in range(P.nkeys)]
+        fmap = {hq.AGG_SUM: "sum", hq.AGG_COUNT: "sum", hq.AGG_MIN: "min", hq.AGG_MAX: "max"}
+        aggs = []
+        for a in range(P.naggs):
+            if P.agg_fn[a] not in fmap:
+                raise NotImplementedError("distributed hash group-by merge: AVG needs SUM and COUNT partials")
+            aggs.append((fmap[P.agg_fn[a]], names[P.nkeys + a]))
+        order, limit = pb.dist_order
+        mb.aggregate(keys=keys, aggs=aggs, order=[(names[c], bool(d)) for c, d in order], limit=limit,
+                     group_capacity=max(1024, sum(sizes)), agg_names=names[P.nkeys:])
+        out = fetch(self.ctx.run(mb.plan, keep=mb.keep + [merged]), mb.result_names)
+        out.qualifying = int(qual.item())  # rows that reached the sinks, over all ranks
+        return out

@@ -323,6 +323,13 @@ class Table:
     def col(self, name: str) -> int:
         return self.names.index(name)
 
+    def column_ptr(self, c: int):
+        """(device pointer, hq_type) of column c."""
+        p = ctypes.c_void_p()
+        t = ctypes.c_int32()
+        check(lib().hq_table_column(self.h, c, ctypes.byref(p), ctypes.byref(t)))
+        return p.value, t.value
+
     def free(self) -> None:
         if self.h:
             lib().hq_free_table(self.h)

@@ -12,7 +12,7 @@ import torch.multiprocessing as mp
 pytestmark = pytest.mark.gpu
 
 SF = 0.01
-QS = ["ssb_q41", "ssb_q31", "ssb_q11", "tpch_q6", "tpch_q1"]
+QS = ["ssb_q41", "ssb_q31", "ssb_q11", "tpch_q6", "tpch_q1", "tpch_q3"]
 
 
 def _port():
@@ -87,3 +87,6 @@ def test_two_ranks_on_one_device_match_oracle():
                            "sum_charge", "count_order"])
     for r, avg in zip(root["tpch_q1"], o1.rows(["avg_qty", "avg_price", "avg_disc"])):
         assert all(abs(a - b) <= 1e-9 * abs(b) for a, b in zip(r[6:9], avg))
+    # hash group-by (l_orderkey): ranks' groups all-gathered and merged on the root, then top 10
+    o3 = oracle.tpch_q3(tpch["tpch_customer"], tpch["orders"], tpch["lineitem"])
+    assert root["tpch_q3"] == o3.rows(["l_orderkey", "o_orderdate", "o_shippriority", "revenue", "count"])[:10]
