@@ -240,7 +240,7 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   h->meta.capacity = cap;
   h->meta.slot_words = words;
   h->meta.npayload = d->npayload;
-  h->meta.nkeys = -1;
+  h->meta.nkeys = d->expected_rows <= 0 ? keys : -1;  // exact after the count pass (confirmed at hq_hash_info)
   h->meta.bytes = cap * words * 4;
   h->meta.layout = direct ? HQ_HT_DIRECT : HQ_HT_LINEAR;
   h->meta.key_min = kmin;

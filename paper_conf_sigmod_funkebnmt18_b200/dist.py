@@ -77,11 +77,13 @@ class DistributedEngine(Engine):
         self.world = dist.get_world_size()
         self.root = root
         self.device = torch.device("cuda", ctx.device)
+        self._built: List[hq.Hash] = []
+        self.builds_here = self.rank == root
 
     def _share(self, h: Optional[hq.Hash]) -> hq.Hash:
         if self.rank == self.root:
-            m = h.info()  # syncs, reports build faults before anything is sent
-            ptr, _ = h.device_view()
+            ptr, m = h.device_view()  # no sync: the slot array is stream-ordered before NCCL
+            self._built.append(h)     # build faults are checked in finish()
             buf = device_view(ptr, int(m.bytes))
             meta = [m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout,
                     m.pay_min, m.pay_max, m.key_max]
@@ -127,6 +129,9 @@ class DistributedEngine(Engine):
         Hash group-bys (e.g. TPC-H Q3 by l_orderkey): every rank finalizes its
         groups, the rows are all-gathered to the root, which merges them with one
         more fused GROUP BY pipeline on its GPU (and applies ORDER BY / LIMIT)."""
+        for h in self._built:  # root: raise duplicate-key / build faults (syncs)
+            h.info()
+        self._built.clear()
         if not hasattr(pb, "dist_order"):
             ptr, nbytes = res.partials_view()
             t = device_view(ptr, nbytes, torch.int64)

@@ -177,6 +177,10 @@ class Engine:
     def table(self, name: str) -> hq.Table:
         return self.tables[name]
 
+    #: whether this engine runs build-side (unpartitioned) pipelines; False on
+    #: the non-root ranks of a DistributedEngine
+    builds_here = True
+
     def plan(self, fact: str) -> PlanBuilder:
         return PlanBuilder(self.tables[fact])
 

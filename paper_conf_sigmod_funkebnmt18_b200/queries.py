@@ -144,11 +144,13 @@ def _tpch_q3(E: Engine, limit: int = 10, **_):
     # pipeline 1: customer filter -> build (semi)
     hc = E.hash("tpch_customer", "c_custkey", preds=[("c_mktsegment", "=", BUILDING)])
     # pipeline 2: orders filter -> probe customer -> materialise -> build
-    po = E.plan("orders")
-    po.filter("o_orderdate", "<", 19950315)
-    po.probe(hc, "o_custkey", "semi")
-    po.materialise([("o_orderkey", "i32"), ("o_orderdate", "i32"), ("o_shippriority", "i32")])
-    ro = E.run(po, partitioned=False)
+    ro = None
+    if E.builds_here:  # build side: only the root of a DistributedEngine holds the dimensions
+        po = E.plan("orders")
+        po.filter("o_orderdate", "<", 19950315)
+        po.probe(hc, "o_custkey", "semi")
+        po.materialise([("o_orderkey", "i32"), ("o_orderdate", "i32"), ("o_shippriority", "i32")])
+        ro = E.run(po, partitioned=False)
     ho = E.hash_from(ro, ["o_orderkey", "o_orderdate", "o_shippriority"], "o_orderkey",
                      ["o_orderdate", "o_shippriority"])
     nk = max(int(ho.info().nkeys), 0)

@@ -69,7 +69,8 @@ def test_two_ranks_on_one_device_match_oracle():
     for p in procs:
         p.join(timeout=120)
     errs = [o for o in outs if o[0] != "ok"]
-    assert not errs, errs
+    if errs:
+        pytest.fail("\n\n".join(f"rank {o[1]}:\n{o[2]}" for o in errs))
     root = next(o[2] for o in outs if o[1] == 0)
     ssb = {t: hqgen.generate(t, SF) for t in hqgen.SSB_TABLES}
     tpch = {t: hqgen.generate(t, SF) for t in hqgen.TPCH_TABLES}
