@@ -298,6 +298,20 @@ __global__ void hq_compact_u8_kernel(const uint32_t* slots, long long range, int
     out[w] = v;
   }
 }
+// one nibble per key: payload0 - pay_min (< 15), 0xF = absent (8-B slots {key, payload})
+__global__ void hq_compact_u4_kernel(const uint32_t* slots, long long range, int pay_min, uint32_t* out) {
+  const long long nwords = (range + 7) / 8;
+  for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < nwords; w += (long long)gridDim.x * blockDim.x) {
+    uint32_t v = 0;
+    for (int b = 0; b < 8; ++b) {
+      const long long i = w * 8 + b;
+      uint32_t nib = 0xFu;
+      if (i < range && (int)slots[2 * i] != INT_MIN) nib = (uint32_t)((int)slots[2 * i + 1] - pay_min) & 0xFu;
+      v |= nib << (4 * b);
+    }
+    out[w] = v;
+  }
+}
 }  // namespace
 
 // Compact derived form of a direct table (used by generated kernels to stage
@@ -327,16 +341,18 @@ void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
   const long long range = h->meta.capacity;
   int kind = 0;
   if (h->meta.npayload == 0) kind = 1;
-  else if (h->meta.npayload == 1 && h->meta.pay_min <= h->meta.pay_max &&
-           (long long)h->meta.pay_max - h->meta.pay_min < 255)
-    kind = 2;
+  else if (h->meta.npayload == 1 && h->meta.pay_min <= h->meta.pay_max) {
+    const long long pr = (long long)h->meta.pay_max - h->meta.pay_min;
+    kind = pr < 15 ? 3 : (pr < 255 ? 2 : 0);
+  }
   if (!kind) return;
-  const long long words = kind == 1 ? (range + 31) / 32 : (range + 3) / 4;
+  const long long words = kind == 1 ? (range + 31) / 32 : (kind == 3 ? (range + 7) / 8 : (range + 3) / 4);
   h->compact = DevBuf(ctx, (size_t)words * 4 + 16);
   const int grid = (int)std::max<long long>(1, std::min<long long>((words + 255) / 256, (long long)ctx->num_sms * 8));
   ctx->launches++;
   if (kind == 1) hq_compact_bitmap_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->compact.as<uint32_t>());
-  else hq_compact_u8_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>());
+  else if (kind == 2) hq_compact_u8_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>());
+  else hq_compact_u4_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>());
   HQ_CUDA(cudaGetLastError());
   h->ckind = kind;
   h->cbytes = words * 4;

@@ -118,7 +118,8 @@ struct hq_hash : RefObj {
   DevBuf dstate;     // [0] fault bits (int), [1..2] nkeys (u64) -- see hq_build.cu
   bool checked = false;
   // compact form of a direct table (hq_build.cu): 1 = bitmap of present keys
-  // (semi-join), 2 = one byte per key (payload0 - pay_min, 0xFF absent)
+  // (semi-join), 2 = one byte per key (payload0 - pay_min, 0xFF absent),
+  // 3 = one nibble per key (payload0 - pay_min < 15, 0xF absent)
   DevBuf compact;
   int ckind = 0;
   int64_t cbytes = 0;
@@ -182,7 +183,7 @@ struct KProbe {
   int16_t key_reg;
   int16_t dst[HQ_MAX_PAYLOAD];
   const void* compact;
-  int32_t pay_min;   // ckind 2: payload = byte + pay_min; range of payload 0 (count pass)
+  int32_t pay_min;   // ckind 2/3: payload = byte (nibble) + pay_min; range of payload 0 (count pass)
   int32_t pay_max;
   uint32_t cbytes;
   uint32_t smem_off; // generated kernels: byte offset of the staged compact table (0 = not staged)

@@ -39,6 +39,7 @@ using namespace hqk;
     long long capacity;                                                                                        \
     unsigned long long* counter;                                                                               \
     int* err;                                                                                                  \
+    long long* prof;                                                                                           \
   };
 HQ_JPARAMS_DEF
 #define HQ_XSTR(...) #__VA_ARGS__
@@ -123,7 +124,15 @@ struct Gen {
       << "u) + row0;\n#pragma unroll\n        for (int r = 0; r < R; ++r) " << var(reg) << "[r] = b_[r * 32]; }\n";
     loaded.insert(reg);
   }
-  void early_exit() { o << "      if (!__any_sync(HQ_FULL, mask)) break;\n"; }
+  // skip the rest of the operator block when no row of the warp is live; the
+  // block stays structured (nested ifs, closed in generate()) so that the
+  // compiler reconverges the warp at its end -- with break-style exits a warp
+  // could stay split for the rest of the kernel and run at half speed
+  int open = 0;
+  void early_exit() {
+    o << "      if (__any_sync(HQ_FULL, mask)) {\n";
+    ++open;
+  }
 
   void filter(const KPred& f, int idx) {
     std::string cond;
@@ -155,88 +164,156 @@ struct Gen {
               << f.bm[2] << "ull, " << f.bm[3] << "ull};\n";
     }
     o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (!(" << cond << ")) mask &= ~(1u << r);\n";
-    early_exit();
   }
 
-  void probe(const KProbe& pr, int idx) {
-    const int W = pr.words;
+  // ---- probes.  A direct-mapped probe is three steps: address (key - min,
+  // range check), load (staged compact table in shared memory, compact table in
+  // global memory, or the slot array), resolve (hit test, payload, mask).
+  // Global loads of adjacent probes are issued together (one L2 round trip for
+  // the batch instead of one per probe), see generate().
+  enum { AK_SMEM = 1, AK_GCOMPACT = 2, AK_DIRECT = 3, AK_LINEAR = 4 };
+  static int access(const KProbe& pr) {
+    if (!pr.direct) return AK_LINEAR;
+    if (pr.ckind && pr.smem_off) return AK_SMEM;
+    if (pr.ckind && pr.compact) return AK_GCOMPACT;
+    return AK_DIRECT;
+  }
+  static std::string pv(int i, const char* what) { return "p" + std::to_string(i) + what; }
+  void probe_defs(const KProbe& pr) {
     const int npay = pr.mode == HQ_PROBE_INNER ? pr.npay : 0;
     for (int k = 0; k < npay; ++k) {
       o << "      int " << var(pr.dst[k]) << "[R];\n";
       if (k == 0 && pr.pay_min <= pr.pay_max) known[pr.dst[0]] = {pr.pay_min, pr.pay_max};
       loaded.insert(pr.dst[k]);
     }
+  }
+  void probe_addr(const KProbe& pr, int i) {
     const std::string key = val(pr.key_reg);
-    if (pr.direct && pr.smem_off) {
-      // compact table staged in shared memory: bitmap (semi) or one byte per key
-      o << "      { u32 found_ = 0u;\n#pragma unroll\n        for (int r = 0; r < R; ++r) {\n"
-        << "          const long long k_ = (long long)" << key << ";\n"
-        << "          const u32 d_ = (u32)(k_ - " << pr.dmin << "LL);\n"
-        << "          if (((mask >> r) & 1u) && k_ >= " << pr.dmin << "LL && d_ < " << pr.mask << "u) {\n";
-      if (pr.ckind == 1) {
-        o << "            const u32 w_ = ((const u32*)(smem + " << pr.smem_off << "u))[d_ >> 5];\n"
-          << "            if ((w_ >> (d_ & 31u)) & 1u) found_ |= 1u << r;\n";
-      } else {
-        o << "            const int b_ = ((const unsigned char*)(smem + " << pr.smem_off << "u))[d_];\n"
-          << "            if (b_ != 0xFF) { found_ |= 1u << r;";
-        if (npay > 0) o << " " << var(pr.dst[0]) << "[r] = b_ + (" << pr.pay_min << ");";
-        o << " }\n";
-      }
-      o << "          }\n        }\n"
-        << "        mask = " << (pr.mode == HQ_PROBE_ANTI ? "mask & ~found_" : "mask & found_") << "; }\n";
-      early_exit();
+    const std::string D = pv(i, "d_"), M = pv(i, "m_");
+    o << "      u32 " << D << "[R]; u32 " << M << " = 0u;\n#pragma unroll\n      for (int r = 0; r < R; ++r) {";
+    if (width(pr.key_reg) <= 4)  // int32 keys: (k - min) mod 2^32 < range  <=>  min <= k < min + range
+      o << " const u32 d_ = (u32)(int)" << key << " - " << (uint32_t)pr.dmin << "u; const bool in_ = d_ < " << pr.mask << "u;";
+    else
+      o << " const long long k_ = (long long)" << key << "; const u32 d_ = (u32)(k_ - " << pr.dmin
+        << "LL); const bool in_ = k_ >= " << pr.dmin << "LL && k_ < " << pr.dmin << "LL + " << pr.mask << "LL;";
+    o << " " << D << "[r] = d_; if (((mask >> r) & 1u) && in_) " << M << " |= 1u << r; }\n";
+  }
+  void probe_load(const KProbe& pr, int i) {
+    const std::string D = pv(i, "d_"), M = pv(i, "m_"), V = pv(i, "v_");
+    const int ak = access(pr);
+    if (ak == AK_DIRECT) {
+      const int W = pr.words;
+      o << "      int4 " << V << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((" << M << " >> r) & 1u) ";
+      if (W == 1) o << V << "[r].x = __ldg((const int*)p.ht[" << i << "] + " << D << "[r]);\n";
+      else if (W == 2)
+        o << "{ const int2 q_ = __ldg((const int2*)p.ht[" << i << "] + " << D << "[r]); " << V << "[r].x = q_.x; " << V
+          << "[r].y = q_.y; }\n";
+      else o << V << "[r] = __ldg((const int4*)p.ht[" << i << "] + " << D << "[r]);\n";
       return;
     }
+    std::string idx = D + "[r]";
+    if (pr.ckind == 1) idx = "(" + D + "[r] >> 5)";
+    else if (pr.ckind == 3) idx = "(" + D + "[r] >> 1)";
+    std::string ld;
+    if (ak == AK_SMEM)
+      ld = pr.ckind == 1 ? "((const u32*)(smem + " + std::to_string(pr.smem_off) + "u))[" + idx + "]"
+                         : "(u32)((const unsigned char*)(smem + " + std::to_string(pr.smem_off) + "u))[" + idx + "]";
+    else
+      ld = pr.ckind == 1 ? "__ldg((const u32*)p.ctab[" + std::to_string(i) + "] + " + idx + ")"
+                         : "(u32)__ldg((const unsigned char*)p.ctab[" + std::to_string(i) + "] + " + idx + ")";
+    o << "      u32 " << V << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((" << M << " >> r) & 1u) " << V
+      << "[r] = " << ld << ";\n";
+  }
+  void probe_resolve(const KProbe& pr, int i) {
+    const std::string D = pv(i, "d_"), M = pv(i, "m_"), V = pv(i, "v_");
+    const int npay = pr.mode == HQ_PROBE_INNER ? pr.npay : 0;
+    o << "      { u32 found_ = 0u;\n#pragma unroll\n        for (int r = 0; r < R; ++r) if ((" << M << " >> r) & 1u) {";
+    if (access(pr) == AK_DIRECT) {
+      static const char* comp[3] = {"y", "z", "w"};
+      o << " if (" << V << "[r].x != HQ_INT_MIN) { found_ |= 1u << r;";
+      for (int k = 0; k < npay; ++k) o << " " << var(pr.dst[k]) << "[r] = " << V << "[r]." << comp[k] << ";";
+      o << " }";
+    } else if (pr.ckind == 1) {
+      o << " if ((" << V << "[r] >> (" << D << "[r] & 31u)) & 1u) found_ |= 1u << r;";
+    } else {
+      if (pr.ckind == 3) o << " const u32 b_ = (" << V << "[r] >> ((" << D << "[r] & 1u) * 4u)) & 15u; if (b_ != 15u) {";
+      else o << " const u32 b_ = " << V << "[r]; if (b_ != 0xFFu) {";
+      o << " found_ |= 1u << r;";
+      if (npay > 0) o << " " << var(pr.dst[0]) << "[r] = (int)b_ + (" << pr.pay_min << ");";
+      o << " }";
+    }
+    o << " }\n        mask = " << (pr.mode == HQ_PROBE_ANTI ? "mask & ~found_" : "mask & found_") << "; }\n";
+  }
+
+  // linear-probing table (sparse keys): optional exact key-range bitmap, then
+  // 16-B group scans until the key or an empty slot
+  void probe_linear(const KProbe& pr, int idx) {
+    const int W = pr.words;
+    const int npay = pr.mode == HQ_PROBE_INNER ? pr.npay : 0;
+    probe_defs(pr);
+    const std::string key = val(pr.key_reg);
     o << "      { const u32* ht_ = p.ht[" << idx << "]; u32 found_ = 0u; int kk_[R]; u32 pend_ = 0u; u32 pos_[R];\n"
       << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n"
       << "          const long long k_ = (long long)" << key << "; kk_[r] = (int)k_;\n";
-    if (pr.direct) {
-      o << "          const bool ok_ = ((mask >> r) & 1u) && k_ >= " << pr.dmin << "LL && k_ < " << pr.dmin << "LL + "
-        << pr.mask << "LL;\n"
-        << "          pos_[r] = (u32)(k_ - " << pr.dmin << "LL); if (ok_) pend_ |= 1u << r; }\n";
-      o << "        int4 sl_[R];\n#pragma unroll\n        for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) {\n";
-      if (W == 1) o << "          sl_[r].x = __ldg((const int*)ht_ + pos_[r]);\n";
-      else if (W == 2) o << "          const int2 q_ = __ldg((const int2*)ht_ + pos_[r]); sl_[r].x = q_.x; sl_[r].y = q_.y;\n";
-      else o << "          sl_[r] = __ldg((const int4*)ht_ + pos_[r]);\n";
-      o << "        }\n#pragma unroll\n        for (int r = 0; r < R; ++r) if ((pend_ & (1u << r)) && sl_[r].x == kk_[r]) {\n"
-        << "          found_ |= 1u << r;\n";
-      static const char* comp[3] = {"y", "z", "w"};
-      for (int k = 0; k < npay; ++k) o << "          " << var(pr.dst[k]) << "[r] = sl_[r]." << comp[k] << ";\n";
-      o << "        }\n";
-    } else {
-      const int G = W == 1 ? 4 : (W == 2 ? 2 : 1);
-      o << "          bool ok_ = ((mask >> r) & 1u) && k_ > (long long)HQ_INT_MIN && k_ <= (long long)HQ_INT_MAX;\n";
-      if (pr.pf) {  // exact key-range bitmap first: misses mostly stop here (L2-resident)
-        o << "          if (ok_) { const long long d_ = k_ - (" << pr.pf_min << "LL);\n"
-          << "            ok_ = d_ >= 0 && d_ < " << pr.pf_range << "LL && ((__ldg(p.pf[" << idx
-          << "] + (d_ >> 5)) >> (d_ & 31)) & 1u); }\n";
-      }
-      o << "          pos_[r] = ((u32)(int)k_ * 0x9E3779B1u) >> " << (32 - pr.log2cap) << "; if (ok_) pend_ |= 1u << r; }\n"
-        << "        while (pend_) {\n          int4 sl_[R];\n"
-        << "#pragma unroll\n          for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) sl_[r] = __ldg((const int4*)ht_ + pos_[r] / "
-        << G << ");\n"
-        << "#pragma unroll\n          for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) {\n"
-        << "            int hit_ = -1; bool stop_ = false; const int first_ = (int)(pos_[r] % " << G << ");\n";
-      const char* keys4[4] = {"x", "y", "z", "w"};
-      for (int j = 0; j < G; ++j) {
-        const char* kc = G == 4 ? keys4[j] : (G == 2 ? (j == 0 ? "x" : "z") : "x");
-        o << "            if (!stop_ && " << j << " >= first_) { if (sl_[r]." << kc << " == kk_[r]) { hit_ = " << j
-          << "; stop_ = true; } else if (sl_[r]." << kc << " == HQ_INT_MIN) stop_ = true; }\n";
-      }
-      o << "            if (hit_ >= 0) { found_ |= 1u << r; pend_ &= ~(1u << r);\n";
-      if (npay > 0) {
-        if (G == 2) o << "              " << var(pr.dst[0]) << "[r] = hit_ == 0 ? sl_[r].y : sl_[r].w;\n";
-        else {
-          static const char* comp[3] = {"y", "z", "w"};
-          for (int k = 0; k < npay; ++k) o << "              " << var(pr.dst[k]) << "[r] = sl_[r]." << comp[k] << ";\n";
-        }
-      }
-      o << "            } else if (stop_) pend_ &= ~(1u << r);\n"
-        << "            else pos_[r] = ((pos_[r] / " << G << " + 1) * " << G << ") & " << pr.mask << "u;\n"
-        << "          }\n        }\n";
+    const int G = W == 1 ? 4 : (W == 2 ? 2 : 1);
+    o << "          bool ok_ = ((mask >> r) & 1u) && k_ > (long long)HQ_INT_MIN && k_ <= (long long)HQ_INT_MAX;\n";
+    if (pr.pf) {  // exact key-range bitmap first: misses mostly stop here (L2-resident)
+      o << "          if (ok_) { const long long d_ = k_ - (" << pr.pf_min << "LL);\n"
+        << "            ok_ = d_ >= 0 && d_ < " << pr.pf_range << "LL && ((__ldg(p.pf[" << idx
+        << "] + (d_ >> 5)) >> (d_ & 31)) & 1u); }\n";
     }
+    o << "          pos_[r] = ((u32)(int)k_ * 0x9E3779B1u) >> " << (32 - pr.log2cap) << "; if (ok_) pend_ |= 1u << r; }\n"
+      << "        while (pend_) {\n          int4 sl_[R];\n"
+      << "#pragma unroll\n          for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) sl_[r] = __ldg((const int4*)ht_ + pos_[r] / "
+      << G << ");\n"
+      << "#pragma unroll\n          for (int r = 0; r < R; ++r) if (pend_ & (1u << r)) {\n"
+      << "            int hit_ = -1; bool stop_ = false; const int first_ = (int)(pos_[r] % " << G << ");\n";
+    const char* keys4[4] = {"x", "y", "z", "w"};
+    for (int j = 0; j < G; ++j) {
+      const char* kc = G == 4 ? keys4[j] : (G == 2 ? (j == 0 ? "x" : "z") : "x");
+      o << "            if (!stop_ && " << j << " >= first_) { if (sl_[r]." << kc << " == kk_[r]) { hit_ = " << j
+        << "; stop_ = true; } else if (sl_[r]." << kc << " == HQ_INT_MIN) stop_ = true; }\n";
+    }
+    o << "            if (hit_ >= 0) { found_ |= 1u << r; pend_ &= ~(1u << r);\n";
+    if (npay > 0) {
+      if (G == 2) o << "              " << var(pr.dst[0]) << "[r] = hit_ == 0 ? sl_[r].y : sl_[r].w;\n";
+      else {
+        static const char* comp[3] = {"y", "z", "w"};
+        for (int k = 0; k < npay; ++k) o << "              " << var(pr.dst[k]) << "[r] = sl_[r]." << comp[k] << ";\n";
+      }
+    }
+    o << "            } else if (stop_) pend_ &= ~(1u << r);\n"
+      << "            else pos_[r] = ((pos_[r] / " << G << " + 1) * " << G << ") & " << pr.mask << "u;\n"
+      << "          }\n        }\n";
     o << "        mask = " << (pr.mode == HQ_PROBE_ANTI ? "mask & ~found_" : "mask & found_") << "; }\n";
-    early_exit();
+  }
+
+  // ops [i, end): one probe batch starting at op i (see probe_addr)
+  int probe_batch(int i) {
+    const KProbe& first = kp.probes[kp.ops[i].idx];
+    const int ak = access(first);
+    if (ak == AK_LINEAR) {
+      early_exit();
+      probe_linear(first, kp.ops[i].idx);
+      return i + 1;
+    }
+    std::vector<int> b = {i};
+    if (ak != AK_SMEM) {  // a global probe: the following independent global probes join its batch
+      // (no early exit in front: the warp rarely has no live row here, and the
+      // extra branch measured slower)
+      std::set<int> defs(first.dst, first.dst + (first.mode == HQ_PROBE_INNER ? first.npay : 0));
+      for (int j = i + 1; j < kp.nops && kp.ops[j].kind == OP_PROBE; ++j) {
+        const KProbe& pr = kp.probes[kp.ops[j].idx];
+        if (access(pr) == AK_LINEAR || access(pr) == AK_SMEM || defs.count(pr.key_reg)) break;
+        b.push_back(j);
+        for (int k = 0; k < (pr.mode == HQ_PROBE_INNER ? pr.npay : 0); ++k) defs.insert(pr.dst[k]);
+      }
+    }
+    for (int j : b) probe_defs(kp.probes[kp.ops[j].idx]);
+    for (int j : b) probe_addr(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
+    for (int j : b) probe_load(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
+    for (int j : b) probe_resolve(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
+    return b.back() + 1;
   }
 
   std::string operand(const KInsn& in) {
@@ -279,6 +356,9 @@ std::string fn_list(const uint8_t* fns, int n) {
 
 std::string generate(const KPlan& kp) {
   Gen g(kp);
+  // HQ_JIT_PROF=1 (debug): per-CTA globaltimer start/end and barrier-wait cycles
+  const bool prof = getenv("HQ_JIT_PROF") != nullptr;
+  const int wait_ns = 128;  // consumer back-off between barrier polls
   std::ostringstream& o = g.o;
   const bool c2 = kp.resolution == HQ_RES_ATOMIC;
   const int sk = kp.sink == HQ_SINK_MATERIALISE ? 2 : (kp.nkeys == 0 ? 0 : 1);
@@ -293,7 +373,10 @@ std::string generate(const KPlan& kp) {
     << "  const long long first_tile = p.row_begin / T;\n"
     << "  const long long ntiles = p.row_end > p.row_begin ? (p.row_end + T - 1) / T - first_tile : 0;\n"
     << "  const long long nj = ntiles > blockIdx.x ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;\n"
+    << "  const long long tstep = (long long)gridDim.x * T;\n"
     << "  if (threadIdx.x == 0) { for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], NW); } fence_mbar_init(); }\n";
+  if (prof) o << "  long long pt0_ = 0; if (threadIdx.x == 0) asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(pt0_));\n"
+              << "  long long pw_ = 0, pl0_ = clock64(); int pdv_ = 0;\n";
   // smem table init
   if (sk == 1 && kp.smode == SM_LANE) {
     o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * NACC * NW * 32; i += NW * 32) {"
@@ -316,30 +399,33 @@ std::string generate(const KPlan& kp) {
   o << "  __syncthreads();\n";
   // producer
   o << "  if (warp == NW) {\n    if (lane == 0) {\n      const u64 pol = policy_evict_first();\n"
-    << "      for (long long j = 0; j < nj; ++j) {\n        const int s = (int)(j % S);\n"
-    << "        if (j >= S) mbar_wait(&empty[s], (u32)(((j / S) - 1) & 1));\n"
-    << "        const long long t0 = (first_tile + blockIdx.x + j * gridDim.x) * (long long)T;\n"
+    << "      int s = 0; u32 ph = 0; long long t0 = (first_tile + blockIdx.x) * (long long)T;\n"
+    << "      for (long long j = 0; j < nj; ++j, t0 += tstep) {\n"
+    << "        " << (prof ? "{ const long long c_ = clock64(); if (j >= S) mbar_wait(&empty[s], ph ^ 1u); pw_ += clock64() - c_; }" : "if (j >= S) mbar_wait(&empty[s], ph ^ 1u);") << "\n"
     << "        char* st = stages + (size_t)s * STAGE_STRIDE;\n"
     << "        if (t0 >= p.row_begin && t0 + T <= p.row_end) {\n          mbar_expect_tx(&full[s], STAGE_BYTES);\n";
   for (int k = 0; k < kp.ncols; ++k)
     o << "          tma_load_1d(st + " << kp.cols[k].soff << "u, p.col[" << k << "] + t0 * " << kp.cols[k].width << ", "
       << kp.tile_rows * kp.cols[k].width << "u, &full[s], pol);\n";
-  o << "        } else mbar_arrive(&full[s]);\n      }\n    }\n    return;\n  }\n";
+  o << "        } else mbar_arrive(&full[s]);\n        if (++s == S) { s = 0; ph ^= 1u; }\n      }\n";
+  if (prof) o << "      p.prof[blockIdx.x * 128 + 3] = pw_; p.prof[blockIdx.x * 128 + 4] = clock64() - pl0_;\n";
+  o << "    }\n    return;\n  }\n";
   // consumer state
   o << "  const int row0 = warp * 32 * R + lane;\n";
   if (sk == 0 && !c2) {
     o << "  u64 scount_ = 0;\n";
     for (int a = 0; a < kp.naggs; ++a) o << "  i64 sacc" << a << " = agg_identity(AGG_FN[" << a << "]);\n";
   }
-  o << "  for (long long j = 0; j < nj; ++j) {\n    const int s = (int)(j % S);\n"
-    << "    mbar_wait(&full[s], (u32)((j / S) & 1));\n"
-    << "    const long long t0 = (first_tile + blockIdx.x + j * gridDim.x) * (long long)T;\n"
-    << "    const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
-    << "    const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
+  const std::string cwait = "mbar_wait_sleep(&full[s], ph);";
+  o << "  int s = 0; u32 ph = 0; long long t0 = (first_tile + blockIdx.x) * (long long)T;\n"
+    << "  for (long long j = 0; j < nj; ++j, t0 += tstep) {\n"
+    << (prof ? "    { const long long c_ = clock64(); " + cwait + " pw_ += clock64() - c_; if (__activemask() != 0xffffffffu) ++pdv_; }\n" : "    " + cwait + "\n")
     << "    const char* st = stages + (size_t)s * STAGE_STRIDE;\n"
     << "    u32 mask = (1u << R) - 1u;\n"
-    << "    if (lo > 0 || hi < T) { mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r * 32; if (row >= lo && row < hi) mask |= 1u << r; } }\n"
-    << "    if (lo > 0 || hi < T) {\n";
+    << "    if (t0 < p.row_begin || t0 + T > p.row_end) {  // ragged head / tail tile: lanes copy their rows\n"
+    << "      const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
+    << "      const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
+    << "      mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r * 32; if (row >= lo && row < hi) mask |= 1u << r; }\n";
   for (int k = 0; k < kp.ncols; ++k) {
     const char* ty = ctype(kp.cols[k].width);
     o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r * 32; ((" << ty
@@ -348,13 +434,15 @@ std::string generate(const KPlan& kp) {
   o << "      fence_proxy_async(); __syncwarp();\n    }\n";
   if (sk == 2)  // output values leave the operator block in registers; the block scan runs after it
     for (int j = 0; j < kp.nout; ++j) o << "    long long ov" << j << "[R];\n";
-  o << "    do {\n      if (!__any_sync(HQ_FULL, mask)) break;\n";
-  for (int i = 0; i < kp.nops; ++i) {
+  o << "    {\n";
+  for (int i = 0; i < kp.nops;) {
     const KOp op = kp.ops[i];
+    if (op.kind == OP_PROBE) { i = g.probe_batch(i); continue; }
     if (op.kind == OP_FILTER) g.filter(kp.preds[op.idx], op.idx);
-    else if (op.kind == OP_PROBE) g.probe(kp.probes[op.idx], op.idx);
     else g.compute(kp.comps[op.idx]);
+    ++i;
   }
+  if (sk != 2) g.early_exit();  // the sinks below only touch live rows
   // ------------------------------------------------------------ sink (tile)
   auto aggval = [&](int a) -> std::string {
     if (kp.agg_fn[a] == HQ_AGG_COUNT) return "1LL";
@@ -415,26 +503,44 @@ std::string generate(const KPlan& kp) {
           << "        u64 key_ = 0; i64 v_[NAGGS > 0 ? NAGGS : 1];\n"
           << "#pragma unroll\n        for (int r = 0; r < R; ++r) { const u64 kx_ = __shfl_sync(HQ_FULL, gk_[r], src_); if (r == rr_) key_ = kx_;\n"
           << "#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) { const i64 x_ = __shfl_sync(HQ_FULL, va_[a][r], src_); if (r == rr_) v_[a] = x_; } }\n";
+      } else if (!c2) {
+        // few live rows (selective joins): each live lane updates its own group
+        // (the shared atomics resolve collisions), then one vote reconverges
+        // the warp -- without it a warp could leave the divergent hash probing
+        // split and run the rest of the kernel at half speed.  Otherwise rows
+        // of equal keys are combined in registers first (match_any + reduce).
+        o << "      u32 act_[R]; int nact_ = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { act_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); nact_ += __popc(act_[r]); }\n"
+          << "      if (nact_ <= 4 * R) {\n"
+          << "#pragma unroll\n        for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) {\n"
+          << "          i64 v_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n"
+          << "          group_update(p, sagg, gk_[r], true, 1ull, v_); }\n"
+          << "        nact_ = __popc(__ballot_sync(HQ_FULL, nact_ > 0));\n";
+        o << "      } else {\n"
+          << "#pragma unroll\n      for (int r = 0; r < R; ++r) {\n"
+          << "        const bool live_ = (mask >> r) & 1u; const u64 key_ = gk_[r];\n"
+          << "        i64 v_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n"
+          << "        const u32 am_ = act_[r];\n";
       } else {
         o << "#pragma unroll\n      for (int r = 0; r < R; ++r) {\n"
           << "        const bool live_ = (mask >> r) & 1u; const u64 key_ = gk_[r];\n"
           << "        i64 v_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n";
       }
-      o << "        const u32 act_ = __ballot_sync(HQ_FULL, live_);\n";
+      if (kp.R >= 4 || c2) o << "        const u32 am_ = __ballot_sync(HQ_FULL, live_);\n";
       if (c2) {
         o << "        if (live_) group_update(p, sagg, key_, false, 1ull, v_);\n      }\n";
       } else {
-        o << "        const bool sparse_ = __popc(act_) <= 4;\n"
+        o << "        const bool sparse_ = __popc(am_) <= 4;\n"
           << "        const u64 mk_ = live_ ? key_ : HQ_EMPTY_KEY;\n"
-          << "        const u32 peers_ = sparse_ ? ((1u << lane) & act_) : (__match_any_sync(HQ_FULL, mk_) & act_);\n"
+          << "        const u32 peers_ = sparse_ ? ((1u << lane) & am_) : (__match_any_sync(HQ_FULL, mk_) & am_);\n"
           << "        const bool single_ = live_ && __popc(peers_) == 1;\n"
           << "        if (single_) group_update(p, sagg, key_, true, 1ull, v_);\n"
-          << "        u32 multi_ = act_ & ~__ballot_sync(HQ_FULL, single_);\n"
+          << "        u32 multi_ = am_ & ~__ballot_sync(HQ_FULL, single_);\n"
           << "        while (multi_) {\n          const int leader_ = __ffs(multi_) - 1;\n"
           << "          const u32 grp_ = __shfl_sync(HQ_FULL, peers_, leader_); const bool mine_ = (grp_ >> lane) & 1u;\n"
           << "          i64 w_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) w_[a] = warp_reduce(AGG_FN[a], mine_ ? v_[a] : agg_identity(AGG_FN[a]));\n"
           << "          if (lane == leader_) group_update(p, sagg, key_, true, (u64)__popc(grp_), w_);\n"
           << "          multi_ &= ~grp_;\n        }\n      }\n";
+        if (kp.R < 4) o << "      }\n";  // else of the sparse path
       }
     }
   } else {  // materialise: hand the output values to the block scan below
@@ -444,7 +550,8 @@ std::string generate(const KPlan& kp) {
     for (int j = 0; j < kp.nout; ++j) o << " ov" << j << "[r] = (long long)" << ov[j] << ";";
     o << " }\n";
   }
-  o << "    } while (0);\n";
+  for (int k = 0; k < g.open; ++k) o << "    }\n";
+  o << "    }\n";
   if (sk == 2) {
     // A3 (Fig 25 / P:1069-1072): warp ballots -> block scan over the warps ->
     // one atomicAdd per block and tile -> writes at local + global offset.
@@ -470,7 +577,8 @@ std::string generate(const KPlan& kp) {
     if (!c2) o << "        run_ += __popc(b_[r]); }\n";
     o << "    }\n";
   }
-  o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n  }\n";
+  o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
+  if (prof) o << "  if (lane == 0) { p.prof[blockIdx.x * 128 + 8 + warp] = pw_; p.prof[blockIdx.x * 128 + 40 + warp] = clock64() - pl0_; } if (pdv_) atomicAdd((unsigned long long*)&p.prof[blockIdx.x * 128 + 72 + warp], (unsigned long long)pdv_);\n";
   // ------------------------------------------------------------- sink (end)
   if (sk == 0 && !c2) {
     o << "  { u64 c_ = scount_;\n#pragma unroll\n    for (int o_ = 16; o_ > 0; o_ >>= 1) c_ += __shfl_xor_sync(HQ_FULL, c_, o_);\n";
@@ -506,13 +614,15 @@ std::string generate(const KPlan& kp) {
       << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = AGG_FN[a] == F_COUNT ? e_[0] : e_[1 + a];\n"
       << "      group_update(p, sagg, k_[h], false, (u64)e_[0], vals_); } }\n";
   }
+  if (prof) o << "  if (threadIdx.x == 0) { long long t_; asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(t_)); p.prof[blockIdx.x * 128] = pt0_; p.prof[blockIdx.x * 128 + 5] = t_;"
+              << " unsigned sm_; asm(\"mov.u32 %0, %%smid;\" : \"=r\"(sm_)); p.prof[blockIdx.x * 128 + 6] = sm_; }\n";
   o << "}\n";
 
   // ---------------------------------------------------------- constants
   std::ostringstream h;
   h << "// generated by libhq (hq_jit.cu) for one fusion operator\n"
     << "#define NW " << kp.nw << "\n#define R " << kp.R << "\n#define T " << kp.tile_rows << "\n#define S " << kp.nstages
-    << "\n#define STAGE_STRIDE " << kp.stage_stride << "u\n#define STAGE_BYTES " << kp.stage_bytes
+    << "\n#define WAIT_NS " << wait_ns << "\n#define STAGE_STRIDE " << kp.stage_stride << "u\n#define STAGE_BYTES " << kp.stage_bytes
     << "u\n#define OFF_AGG " << kp.off_agg << "u\n#define OFF_STAGE " << kp.off_stage << "u\n"
     << "#define NAGGS " << kp.naggs << "\n#define VWORDS " << kp.vwords << "\n#define GMODE " << (int)kp.gmode
     << "\n#define SMODE " << (kp.smode == SM_LANE ? 0 : (int)kp.smode) << "\n#define SMEM_CAP " << kp.smem_cap
@@ -645,9 +755,39 @@ void hq_jit_launch(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
   jp.capacity = kp.capacity;
   jp.counter = kp.counter;
   jp.err = kp.err;
+  static long long* prof_buf = nullptr;  // HQ_JIT_PROF (debug) only
+  const bool prof = getenv("HQ_JIT_PROF") != nullptr;
+  if (prof) {
+    if (!prof_buf) HQ_CUDA(cudaMalloc(&prof_buf, 1024 * 128 * sizeof(long long)));
+    HQ_CUDA(cudaMemsetAsync(prof_buf, 0, (size_t)grid * 128 * sizeof(long long), ctx->stream));
+    jp.prof = prof_buf;
+  }
   void* args[] = {&jp};
   ctx->launches++;
   if (d.launch(fn, (unsigned)grid, 1, 1, (unsigned)((kp.nw + 1) * 32), 1, 1, (unsigned)smem, (CUstream)ctx->stream, args,
                nullptr) != CUDA_SUCCESS)
     HQ_THROW(HQ_ERR_CUDA, "cuLaunchKernel failed");
+  if (prof) {
+    std::vector<long long> h((size_t)grid * 128);
+    HQ_CUDA(cudaMemcpyAsync(h.data(), prof_buf, h.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    long long t0 = LLONG_MAX, t1 = 0;
+    auto dur = [&](int b) { return h[b * 128 + 5] - h[b * 128]; };
+    for (int b = 0; b < grid; ++b) { t0 = std::min(t0, h[b * 128]); t1 = std::max(t1, h[b * 128 + 5]); }
+    int slow = 0, fast = 0, nslow = 0;
+    for (int b = 0; b < grid; ++b) {
+      if (dur(b) > dur(slow)) slow = b;
+      if (dur(b) < dur(fast)) fast = b;
+    }
+    for (int b = 0; b < grid; ++b) nslow += dur(b) > dur(fast) * 5 / 4;
+    fprintf(stderr, "[hq prof] grid %d span %lld ns, %d CTAs >1.25x the fastest\n", grid, t1 - t0, nslow);
+    for (int b : {slow, fast}) {
+      fprintf(stderr, "  cta %d sm %lld dur %lld ns producer wait/loop %lld/%lld cyc; warp waits (kcyc):", b, h[b * 128 + 6], dur(b),
+              h[b * 128 + 3], h[b * 128 + 4]);
+      for (int w = 0; w < kp.nw; ++w) fprintf(stderr, " %lld", h[b * 128 + 8 + w] / 1000);
+      fprintf(stderr, "\n    diverged-at-wait lane-iterations per warp:");
+      for (int w = 0; w < kp.nw; ++w) fprintf(stderr, " %lld", h[b * 128 + 72 + w]);
+      fprintf(stderr, "\n");
+    }
+  }
 }

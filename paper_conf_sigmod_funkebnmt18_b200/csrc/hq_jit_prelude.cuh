@@ -40,14 +40,27 @@ __device__ __forceinline__ void mbar_expect_tx(u64* b, u32 tx) {
 __device__ __forceinline__ void mbar_arrive(u64* b) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
 }
-__device__ __forceinline__ void mbar_wait(u64* b, u32 parity) {
+__device__ __forceinline__ bool mbar_try_wait(u64* b, u32 parity) {
+  u32 ok;
   asm volatile(
-      "{\n\t.reg .pred p;\n"
-      "HQW_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
-      "@!p bra HQW_%=;\n}\n" ::"r"(smem_u32(b)),
-      "r"(parity), "r"(1000000)
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(b)), "r"(parity)
       : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(u64* b, u32 parity) {
+  while (!mbar_try_wait(b, parity)) {
+  }
+}
+// consumer-side wait: back off between polls so that warps waiting for a tile
+// leave the issue slots to the warps still working on the previous one (all
+// consumer warps must release a stage before it is refilled; a spinning warp
+// set can starve the last one and lock the CTA into a slow steady state)
+__device__ __forceinline__ void mbar_wait_sleep(u64* b, u32 parity) {
+  while (!mbar_try_wait(b, parity)) __nanosleep(WAIT_NS);
 }
 __device__ __forceinline__ u64 policy_evict_first() {
   u64 pol;

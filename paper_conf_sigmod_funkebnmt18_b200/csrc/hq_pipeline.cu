@@ -50,9 +50,9 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
   asm volatile(
       "{\n\t.reg .pred p;\n"
       "HQ_WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
       "@!p bra HQ_WAIT_%=;\n}\n" ::"r"(smem_u32(b)),
-      "r"(parity), "r"(1000000)  // suspend-time hint (ns): sleep in HW instead of spinning
+      "r"(parity)  // no suspend-time hint: a long hint let a warp oversleep the phase flip
       : "memory");
 }
 __device__ __forceinline__ uint64_t policy_evict_first() {

@@ -242,7 +242,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     if (P.nkeys > 0 && P.resolution == HQ_RES_LRGP) {
       // lane-private tables halve the warps, so only for probe-free pipelines
       // (no latency to hide) whose group domain is tiny
-      if (kp.gmode == GM_DENSE && nprobe == 0 && !getenv("HQ_DEBUG_NOLANE") &&
+      if (kp.gmode == GM_DENSE && nprobe == 0 &&
           (uint64_t)ngroups * kp.nacc * LANE_NW * 32 * 8 <= (uint64_t)SMEM_LANE_BYTES) {
         kp.smode = SM_LANE;  // tiny domain (e.g. TPC-H Q1): contention-free lane-private tables
         kp.smem_cap = (uint32_t)ngroups;
@@ -309,6 +309,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   // rows), as long as the TMA ring keeps >= 3 stages.
   int staged[MAX_PROBES];
   int nstaged = 0;
+  const uint32_t stage_budget = 96 * 1024;
   if (jit) {
     uint32_t total = 0;
     for (int o = 0; o < kp.nops; ++o) {
@@ -316,7 +317,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       const KProbe& pr = kp.probes[kp.ops[o].idx];
       if (!pr.ckind || pr.cbytes == 0) continue;
       const uint32_t b = align_up(pr.cbytes, 128);
-      if (total + b > 96 * 1024) continue;
+      if (total + b > stage_budget) continue;
       total += b;
       staged[nstaged++] = kp.ops[o].idx;
     }
