@@ -241,6 +241,11 @@ struct KPlan {
   uint64_t gmask;            // hash capacity - 1
   int32_t glog2;
   uint32_t smem_cap;         // smem dense groups or smem hash slots
+  // generated kernels: the shared dense table may index a narrowed key domain
+  // (group keys that are probe payloads span only their build-side value range)
+  uint8_t local_keys;
+  int64_t lkey_min[HQ_MAX_KEYS];
+  int64_t lkey_stride[HQ_MAX_KEYS];
   int32_t slog2;
   // SM_LANE: deduplicated accumulators (0 = count; SUM and AVG of one register share)
   int32_t nacc;

@@ -468,10 +468,14 @@ std::string generate(const KPlan& kp) {
       auto kr = g.known.find(kp.key_reg[i]);
       const bool in_domain = kr != g.known.end() && kr->second.first >= kp.key_min[i] &&
                              kr->second.second < kp.key_min[i] + kp.key_card[i];
-      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kp.key_min[i]) << ";";
+      // the shared table may index a narrowed domain (kp.local_keys): only keys
+      // whose payload range is known are narrowed, and those need no check
+      const int64_t kmin = kp.local_keys ? kp.lkey_min[i] : kp.key_min[i];
+      const int64_t kstr = kp.local_keys ? kp.lkey_stride[i] : kp.key_stride[i];
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kmin) << ";";
       if (!in_domain)  // payload ranges known from the build's count pass need no domain check
         o << " if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }";
-      o << " gk_[r] += (u64)d_ * " << kp.key_stride[i] << "ull; }\n";
+      o << " gk_[r] += (u64)d_ * " << kstr << "ull; }\n";
     }
     o << "      if (bad_) atomicOr(p.err, F_KEY_DOMAIN);\n";
     if (kp.smode == SM_LANE) {
@@ -607,7 +611,15 @@ std::string generate(const KPlan& kp) {
     o << "  consumer_bar();\n  { const i64* t_ = (const i64*)sagg;\n"
       << "    for (u32 g = threadIdx.x; g < SMEM_CAP; g += NW * 32) { const i64* e_ = t_ + (u64)g * VWORDS;\n"
       << "      if (e_[0] != 0) { i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) vals_[a] = AGG_FN[a] == F_COUNT ? e_[0] : e_[1 + a];\n"
-      << "        group_update(p, sagg, g, false, (u64)e_[0], vals_); } } }\n";
+      << "        u64 gkey_ = g;\n";
+    if (kp.local_keys) {  // narrowed local index -> declared global key
+      o << "        { u64 rem_ = g; gkey_ = 0;";
+      for (int i = 0; i < kp.nkeys; ++i)
+        o << " { const u64 o_ = rem_ / " << kp.lkey_stride[i] << "ull; rem_ -= o_ * " << kp.lkey_stride[i]
+          << "ull; gkey_ += (o_ + " << (kp.lkey_min[i] - kp.key_min[i]) << "ull) * " << kp.key_stride[i] << "ull; }";
+      o << " }\n";
+    }
+    o << "        group_update(p, sagg, gkey_, false, (u64)e_[0], vals_); } } }\n";
   } else if (sk == 1 && kp.smode == SM_HASH) {
     o << "  consumer_bar();\n  { const u64* k_ = (const u64*)sagg; const i64* t_ = (const i64*)sagg + SMEM_CAP;\n"
       << "    for (u32 h = threadIdx.x; h < SMEM_CAP; h += NW * 32) if (k_[h] != HQ_EMPTY_KEY) { const i64* e_ = t_ + (u64)h * VWORDS;\n"

@@ -237,6 +237,24 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       }
       kp.acc_of[a] = (uint8_t)found;
     }
+    // Generated kernels: a group key that is payload 0 of an inner probe only
+    // takes the payload's value range (count pass), e.g. SSB Q3.1 c_nation of the
+    // ASIA customers spans 14 of the declared 25 values -- the shared table can
+    // be dense over the narrowed domain where the declared one needs a hash.
+    int64_t lmin[HQ_MAX_KEYS], lcard[HQ_MAX_KEYS];
+    __int128 lgroups = 1;
+    for (int i = 0; i < P.nkeys; ++i) {
+      lmin[i] = kp.key_min[i];
+      lcard[i] = kp.key_card[i];
+      for (int q = 0; jit && q < nprobe; ++q) {
+        const KProbe& pr = kp.probes[q];
+        if (pr.mode != HQ_PROBE_INNER || pr.npay < 1 || pr.dst[0] != kp.key_reg[i] || pr.pay_min > pr.pay_max) continue;
+        if (pr.pay_min < kp.key_min[i] || (int64_t)pr.pay_max >= kp.key_min[i] + kp.key_card[i]) continue;
+        lmin[i] = pr.pay_min;
+        lcard[i] = (int64_t)pr.pay_max - pr.pay_min + 1;
+      }
+      lgroups *= lcard[i];
+    }
     // local-resolution table in shared memory
     kp.smode = SM_NONE;
     if (P.nkeys > 0 && P.resolution == HQ_RES_LRGP) {
@@ -251,6 +269,17 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         kp.smode = SM_DENSE;
         kp.smem_cap = (uint32_t)ngroups;
         agg_smem = (uint32_t)(ngroups * kp.vwords * 8);
+      } else if (lgroups < (__int128)ngroups && lgroups * kp.vwords * 8 <= (__int128)SMEM_AGG_BYTES) {
+        kp.smode = SM_DENSE;  // dense over the narrowed domain; merged into the global table by key
+        kp.local_keys = 1;
+        kp.smem_cap = (uint32_t)lgroups;
+        agg_smem = (uint32_t)(lgroups * kp.vwords * 8);
+        int64_t st2 = 1;
+        for (int i = P.nkeys - 1; i >= 0; --i) {
+          kp.lkey_min[i] = lmin[i];
+          kp.lkey_stride[i] = st2;
+          st2 *= lcard[i];
+        }
       } else {
         uint32_t cap = 4096;
         while (cap > 64 && (uint64_t)cap * (kp.vwords + 1) * 8 > (uint64_t)SMEM_AGG_BYTES) cap >>= 1;

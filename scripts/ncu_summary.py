@@ -83,8 +83,11 @@ def main():
                      f"{r.get('dram_write', 0) / 1e6:.2f} | {dram / alg:.3f} | {alg / t / 1e9:.0f} | "
                      f"{r.get('dram_read_bw', 0) / 1e9:.0f} | {r.get('dram_pct', 0):.1f} | {r.get('l2_pct', 0):.1f} | {r.get('warps_active_pct', 0):.1f} | "
                      f"{r.get('issue_active_pct', 0):.1f} | {r.get('regs', 0):.0f} | {r.get('dyn_smem', 0) / 1e3:.0f} |")
-    with open(os.path.join(outdir, "ncu_summary.md"), "a") as f:
-        f.write("\n".join(lines) + "\n")
+    rev = subprocess.run(["git", "-C", ROOT, "rev-parse", "--short", "HEAD"], capture_output=True, text=True).stdout.strip()
+    head = (f"ncu --set full --clock-control none captures of the generated fused kernel (one launch each, "
+            f"cold L2 per replay), code at {rev}. achieved = algorithmic bytes / ncu kernel time.\n\n")
+    with open(os.path.join(outdir, "ncu_summary.md"), "w") as f:
+        f.write(head + "\n".join(lines) + "\n")
     with open(tpath, "w") as f:
         json.dump(traffic, f, indent=1)
     print("\n".join(lines))

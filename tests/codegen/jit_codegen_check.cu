@@ -195,6 +195,15 @@ int main(int argc, char** argv) {
     P.agg_fn[0] = HQ_AGG_SUM; P.agg_reg[0] = 3;
     P.agg_fn[1] = HQ_AGG_COUNT;
     shapes.push_back({"star_smem_hash", P, nullptr});
+    // the same with build-side payload ranges 8..20 (one region's nations):
+    // the shared table becomes dense over the narrowed 13 x 13 x 7 domain
+    hq_hash* na = make_hash(c, HQ_HT_DIRECT, 1, 2, 20000);
+    hq_hash* nb = make_hash(c, HQ_HT_DIRECT, 1, 2, 3000000);
+    na->meta.pay_min = nb->meta.pay_min = 8;
+    na->meta.pay_max = nb->meta.pay_max = 20;
+    P.ops[0] = probe(na, 1, HQ_PROBE_INNER, HQ_TMP(0));
+    P.ops[1] = probe(nb, 0, HQ_PROBE_INNER, HQ_TMP(1));
+    shapes.push_back({"star_narrowed_dense", P, nullptr});
   }
   {  // Q6-like scalar aggregate with an int8 bitmap filter and an i64 expression
     hq_plan P{};

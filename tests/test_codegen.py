@@ -32,7 +32,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     env = {k: v for k, v in os.environ.items() if not k.startswith("HQ_")}
     p = subprocess.run([checker, str(tmp_path)], capture_output=True, text=True, env=env, timeout=600)
     assert p.returncode == 0, p.stdout + p.stderr
-    assert p.stdout.startswith("OK 10 of 10"), p.stdout
+    assert p.stdout.startswith("OK 11 of 11"), p.stdout
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
     star = srcs["star_dense_lrgp"]
@@ -44,3 +44,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "__ldg((const int4*)p.ht[" in srcs["materialise_lrgp"]  # 4-word direct slots
     assert "p.pf[" in srcs["materialise_lrgp"]                     # linear prefilter
     assert "match_any" in srcs["global_hash_groups"] and "pre_[R]" in srcs["global_hash_groups_r4"]
+    # group keys narrowed to the build-side payload ranges: dense shared table + key remap at the merge
+    assert "#define SMODE 2" in srcs["star_smem_hash"]
+    narrowed = srcs["star_narrowed_dense"]
+    assert "#define SMODE 1" in narrowed and "#define SMEM_CAP 1183u" in narrowed and "gkey_ +=" in narrowed
