@@ -173,6 +173,13 @@ typedef struct {
  *    >= keys/0.6; probes scan whole aligned 16-B slot groups per load.
  * Duplicate keys: HQ_ERR_DUP_KEY at hq_hash_info. */
 hq_status hq_build_hash(hq_ctx* ctx, const hq_build_desc* desc, hq_hash** out);
+/* Several builds with ONE host synchronisation (the build
+ * pipelines of a query's dimension tables are independent): the count passes of
+ * all n descriptors run first, their statistics are read back together, then
+ * every table is sized, built and compacted stream-ordered.  descs: n
+ * contiguous descriptors (host memory, read during the call); out: n handles,
+ * all written on HQ_OK, none on error (nothing leaks).  n >= 1. */
+hq_status hq_build_hashes(hq_ctx* ctx, int32_t n, const hq_build_desc* descs, hq_hash** out);
 enum { HQ_HT_LINEAR = 0, HQ_HT_DIRECT = 1 };
 typedef struct {
   int64_t capacity;     /* slots (power of two for HQ_HT_LINEAR, key range for HQ_HT_DIRECT) */

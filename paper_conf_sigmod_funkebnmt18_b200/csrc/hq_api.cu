@@ -5,7 +5,7 @@
 
 #include "hq_internal.h"
 
-void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h);
+void hq_build_hashes_impl(hq_ctx* ctx, int n, const hq_build_desc* d, hq_hash* const* h);
 void hq_hash_check(hq_ctx* ctx, hq_hash* h);
 
 namespace {
@@ -127,6 +127,7 @@ hq_status hq_ctx_destroy(hq_ctx* ctx) {
       cudaEventDestroy(e.second);
     }
     for (auto e : ctx->event_pool) cudaEventDestroy(e);
+    if (ctx->pinned) cudaFreeHost(ctx->pinned);
     delete ctx;
   });
 }
@@ -239,17 +240,24 @@ hq_status hq_free_table(hq_table* t) {
 
 // -------------------------------------------------------------- hash tables
 hq_status hq_build_hash(hq_ctx* ctx, const hq_build_desc* desc, hq_hash** out) {
+  return hq_build_hashes(ctx, 1, desc, out);
+}
+
+hq_status hq_build_hashes(hq_ctx* ctx, int32_t n, const hq_build_desc* descs, hq_hash** out) {
   return guarded([&] {
-    if (!ctx || !desc || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
-    hq_hash* h = new hq_hash();
-    h->ctx = ctx;
+    if (!ctx || !descs || !out || n < 1) HQ_THROW(HQ_ERR_ARG, "NULL argument or n < 1");
+    std::vector<hq_hash*> hs((size_t)n, nullptr);
+    for (auto& h : hs) {
+      h = new hq_hash();
+      h->ctx = ctx;
+    }
     try {
-      hq_build_hash_impl(ctx, desc, h);
+      hq_build_hashes_impl(ctx, n, descs, hs.data());
     } catch (...) {
-      h->release();
+      for (auto* h : hs) h->release();
       throw;
     }
-    *out = h;
+    for (int i = 0; i < n; ++i) out[i] = hs[i];
   });
 }
 
@@ -361,9 +369,15 @@ hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int
     hq_finalize_impl(ctx, r);
     const int64_t n = std::min<int64_t>(r->nrows, capacity_rows);
     if (n > 0 && !host_cols) HQ_THROW(HQ_ERR_ARG, "host_cols is NULL");
+    if (r->host_ready) {  // small result: rows came back with the finalize (no device access)
+      for (int c = 0; c < r->ncols && n > 0; ++c)
+        if (host_cols[c]) std::memcpy(host_cols[c], r->host_rows.data() + (size_t)c * r->nrows, (size_t)n * 8);
+      if (nrows_out) *nrows_out = r->nrows;
+      return;
+    }
     for (int c = 0; c < r->ncols && n > 0; ++c) {
       if (!host_cols[c]) continue;
-      const void* src = r->sink == HQ_SINK_MATERIALISE ? r->outcols[c].p : r->rescols[c].p;
+      const void* src = r->sink == HQ_SINK_MATERIALISE ? r->outcols[c].p : r->rescol[c];
       const size_t w = (size_t)hq_type_width(r->types[c]);
       HQ_CUDA(cudaMemcpyAsync(host_cols[c], src, (size_t)n * w, cudaMemcpyDeviceToHost, ctx->stream));
     }
@@ -384,7 +398,7 @@ hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out) {
     t->nrows = r->nrows;
     t->ncols = r->ncols;
     for (int c = 0; c < r->ncols; ++c) {
-      t->cols[c].ptr = mat ? r->outcols[c].p : r->rescols[c].p;
+      t->cols[c].ptr = mat ? r->outcols[c].p : r->rescol[c];
       t->cols[c].type = r->types[c];
       t->cols[c].width = hq_type_width(r->types[c]);
     }

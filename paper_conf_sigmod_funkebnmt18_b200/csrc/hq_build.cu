@@ -35,7 +35,10 @@ struct KBuild {
   int32_t direct, dmin;
   int* err;
   unsigned long long* nkeys;
-  int* kminmax;      // count pass: [min, max] of the qualifying keys
+  int* kminmax;      // count pass: [min, max] of the qualifying keys, [min, max] of payload 0
+  void* part;        // count pass: per-block partials (CountPart[grid])
+  unsigned* ticket;  // count pass: blocks done
+  int count_inserts; // build pass: accumulate the inserted-key count (no count pass ran)
 };
 
 __device__ __forceinline__ long long ld_col(const KBuild& b, int c, long long row) {
@@ -56,20 +59,84 @@ __device__ __forceinline__ bool row_passes(const KBuild& b, long long row) {
   return true;
 }
 
-__global__ void hq_build_count_kernel(const __grid_constant__ KBuild b) {
+// Both passes give every thread U rows (stride blockDim) with all column loads
+// issued before any is used, and no grid-stride loop: a dimension table's rows
+// are all in flight at once (a grid-stride loop made each thread walk ~10 rows
+// through 2-3 dependent DRAM round trips each).
+constexpr int BUILD_U = 8;
+constexpr int BUILD_BLOCK = 256;
+
+// column c for the thread's U rows: the width dispatch is uniform, the U loads
+// are independent (all in flight)
+__device__ __forceinline__ void ld_rows(const KBuild& b, int c, long long base, long long (&out)[BUILD_U]) {
+  const int w = b.colw[c];
+  const char* p = b.col[c];
+  if (w == 4) {
+#pragma unroll
+    for (int u = 0; u < BUILD_U; ++u) {
+      const long long r = base + (long long)u * BUILD_BLOCK;
+      out[u] = r < b.n ? __ldg((const int*)p + r) : 0;
+    }
+  } else if (w == 8) {
+#pragma unroll
+    for (int u = 0; u < BUILD_U; ++u) {
+      const long long r = base + (long long)u * BUILD_BLOCK;
+      out[u] = r < b.n ? __ldg((const long long*)p + r) : 0;
+    }
+  } else {
+#pragma unroll
+    for (int u = 0; u < BUILD_U; ++u) {
+      const long long r = base + (long long)u * BUILD_BLOCK;
+      out[u] = r < b.n ? (long long)__ldg((const signed char*)p + r) : 0;
+    }
+  }
+}
+// predicates, key and payload 0 of the thread's U rows
+__device__ __forceinline__ void load_rows(const KBuild& b, long long base, bool (&pass)[BUILD_U],
+                                          long long (&kv)[BUILD_U], long long (&pv)[BUILD_U]) {
+  ld_rows(b, b.key_col, base, kv);
+  if (b.npay > 0) ld_rows(b, b.pay_col[0], base, pv);
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u) pass[u] = base + (long long)u * BUILD_BLOCK < b.n;
+  for (int i = 0; i < b.npreds; ++i) {
+    const KBuildPred& f = b.preds[i];
+    long long v[BUILD_U];
+    ld_rows(b, f.col, base, v);
+    if (f.kind == 0) {
+#pragma unroll
+      for (int u = 0; u < BUILD_U; ++u) pass[u] &= (v[u] >= f.lo && v[u] <= f.hi) != (bool)f.neg;
+    } else {
+#pragma unroll
+      for (int u = 0; u < BUILD_U; ++u)
+        pass[u] &= (unsigned long long)v[u] < 256 && ((f.bm[(v[u] >> 6) & 3] >> (v[u] & 63)) & 1ull);
+    }
+  }
+}
+
+// count pass: number of qualifying rows, min/max of their keys and of payload 0.
+// Block partials go to b.part; the last block to finish (ticket) reduces them
+// and writes the totals -- no contended global atomics.
+struct CountPart {
+  unsigned long long cnt;
+  int kmin, kmax, pmin, pmax;
+};
+__global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __grid_constant__ KBuild b) {
   unsigned long long c = 0;
   int kmin = INT_MAX, kmax = INT_MIN, pmin = INT_MAX, pmax = INT_MIN;
-  for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < b.n; r += (long long)gridDim.x * blockDim.x) {
-    if (!row_passes(b, r)) continue;
+  const long long base = (long long)blockIdx.x * BUILD_BLOCK * BUILD_U + threadIdx.x;
+  bool pass[BUILD_U];
+  long long kv[BUILD_U], pv[BUILD_U] = {};
+  load_rows(b, base, pass, kv, pv);
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u) {
+    if (!pass[u]) continue;
     ++c;
-    const long long kv = ld_col(b, b.key_col, r);
-    if (kv > (long long)INT_MIN && kv <= (long long)INT_MAX) {
-      kmin = min(kmin, (int)kv);
-      kmax = max(kmax, (int)kv);
+    if (kv[u] > (long long)INT_MIN && kv[u] <= (long long)INT_MAX) {
+      kmin = min(kmin, (int)kv[u]);
+      kmax = max(kmax, (int)kv[u]);
     }
     if (b.npay > 0) {
-      const long long pv = ld_col(b, b.pay_col[0], r);
-      const int pc = pv < (long long)INT_MIN ? INT_MIN : (pv > (long long)INT_MAX ? INT_MAX : (int)pv);
+      const int pc = pv[u] < (long long)INT_MIN ? INT_MIN : (pv[u] > (long long)INT_MAX ? INT_MAX : (int)pv[u]);
       pmin = min(pmin, pc);
       pmax = max(pmax, pc);
     }
@@ -78,23 +145,53 @@ __global__ void hq_build_count_kernel(const __grid_constant__ KBuild b) {
   kmax = __reduce_max_sync(0xffffffffu, kmax);
   pmin = __reduce_min_sync(0xffffffffu, pmin);
   pmax = __reduce_max_sync(0xffffffffu, pmax);
-  if ((threadIdx.x & 31) == 0 && kmin <= kmax) {
-    atomicMin(b.kminmax, kmin);
-    atomicMax(b.kminmax + 1, kmax);
-  }
-  if ((threadIdx.x & 31) == 0 && pmin <= pmax) {
-    atomicMin(b.kminmax + 2, pmin);
-    atomicMax(b.kminmax + 3, pmax);
-  }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
-  __shared__ unsigned long long red[32];
-  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = c;
+  __shared__ CountPart wp[BUILD_BLOCK / 32];
+  __shared__ bool last;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) wp[w] = {c, kmin, kmax, pmin, pmax};
   __syncthreads();
   if (threadIdx.x == 0) {
-    unsigned long long t = 0;
-    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
-    if (t) atomicAdd(b.nkeys, t);
+    CountPart t{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN};
+    for (int k = 0; k < BUILD_BLOCK / 32; ++k) {
+      t.cnt += wp[k].cnt;
+      t.kmin = min(t.kmin, wp[k].kmin); t.kmax = max(t.kmax, wp[k].kmax);
+      t.pmin = min(t.pmin, wp[k].pmin); t.pmax = max(t.pmax, wp[k].pmax);
+    }
+    ((CountPart*)b.part)[blockIdx.x] = t;
+    __threadfence();
+    last = atomicAdd(b.ticket, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  // last block: reduce every block's partial
+  __threadfence();
+  CountPart t{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN};
+  for (unsigned k = threadIdx.x; k < gridDim.x; k += BUILD_BLOCK) {
+    const volatile CountPart* q = (const volatile CountPart*)b.part + k;
+    t.cnt += q->cnt;
+    t.kmin = min(t.kmin, q->kmin); t.kmax = max(t.kmax, q->kmax);
+    t.pmin = min(t.pmin, q->pmin); t.pmax = max(t.pmax, q->pmax);
+  }
+  t.kmin = __reduce_min_sync(0xffffffffu, t.kmin);
+  t.kmax = __reduce_max_sync(0xffffffffu, t.kmax);
+  t.pmin = __reduce_min_sync(0xffffffffu, t.pmin);
+  t.pmax = __reduce_max_sync(0xffffffffu, t.pmax);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) t.cnt += __shfl_xor_sync(0xffffffffu, t.cnt, o);
+  __syncthreads();
+  if (lane == 0) wp[w] = t;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    CountPart z{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN};
+    for (int k = 0; k < BUILD_BLOCK / 32; ++k) {
+      z.cnt += wp[k].cnt;
+      z.kmin = min(z.kmin, wp[k].kmin); z.kmax = max(z.kmax, wp[k].kmax);
+      z.pmin = min(z.pmin, wp[k].pmin); z.pmax = max(z.pmax, wp[k].pmax);
+    }
+    *b.nkeys = z.cnt;
+    b.kminmax[0] = z.kmin; b.kminmax[1] = z.kmax; b.kminmax[2] = z.pmin; b.kminmax[3] = z.pmax;
   }
 }
 
@@ -103,24 +200,39 @@ __global__ void hq_fill_kernel(uint32_t* p, long long n, uint32_t v) {
     p[i] = v;
 }
 
-__global__ void hq_build_hash_kernel(const __grid_constant__ KBuild b) {
+__global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid_constant__ KBuild b) {
   unsigned long long inserted = 0;
   int fault = 0;
   const uint32_t shift = 32u - b.log2cap;
-  for (long long r = blockIdx.x * (long long)blockDim.x + threadIdx.x; r < b.n; r += (long long)gridDim.x * blockDim.x) {
-    if (!row_passes(b, r)) continue;
-    const long long kv = ld_col(b, b.key_col, r);
-    if (kv <= (long long)INT_MIN || kv > (long long)INT_MAX) {
+  const long long base = (long long)blockIdx.x * BUILD_BLOCK * BUILD_U + threadIdx.x;
+  bool pass[BUILD_U];
+  long long kv[BUILD_U], pv0[BUILD_U] = {};
+  int pay[BUILD_U][HQ_MAX_PAYLOAD] = {};
+  load_rows(b, base, pass, kv, pv0);
+#pragma unroll
+  for (int k = 0; k < HQ_MAX_PAYLOAD; ++k) {
+    if (k >= b.npay) break;
+    long long v[BUILD_U];
+    if (k == 0) {
+#pragma unroll
+      for (int u = 0; u < BUILD_U; ++u) v[u] = pv0[u];
+    } else {
+      ld_rows(b, b.pay_col[k], base, v);
+    }
+#pragma unroll
+    for (int u = 0; u < BUILD_U; ++u) {
+      if (pass[u] && (v[u] < (long long)INT_MIN || v[u] > (long long)INT_MAX)) fault |= HQF_BAD_PAYLOAD;
+      pay[u][k] = (int)v[u];
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u) {
+    if (!pass[u]) continue;
+    if (kv[u] <= (long long)INT_MIN || kv[u] > (long long)INT_MAX) {
       fault |= HQF_BAD_KEY;
       continue;
     }
-    const int key = (int)kv;
-    int pay[HQ_MAX_PAYLOAD] = {0, 0, 0};
-    for (int k = 0; k < b.npay; ++k) {
-      const long long v = ld_col(b, b.pay_col[k], r);
-      if (v < (long long)INT_MIN || v > (long long)INT_MAX) fault |= HQF_BAD_PAYLOAD;
-      pay[k] = (int)v;
-    }
+    const int key = (int)kv[u];
     uint32_t pos = b.direct ? (uint32_t)(key - b.dmin) : ((uint32_t)key * 0x9E3779B1u) >> shift;
     if (b.direct && pos >= b.mask) {  // cannot happen: the range comes from the count pass
       fault |= HQF_HT_FULL;
@@ -131,7 +243,9 @@ __global__ void hq_build_hash_kernel(const __grid_constant__ KBuild b) {
       uint32_t* slot = b.slots + (size_t)pos * b.words;
       const int old = atomicCAS((int*)slot, INT_MIN, key);
       if (old == INT_MIN) {
-        for (int k = 0; k < b.npay; ++k) slot[1 + k] = (uint32_t)pay[k];
+#pragma unroll
+        for (int k = 0; k < HQ_MAX_PAYLOAD; ++k)
+          if (k < b.npay) slot[1 + k] = (uint32_t)pay[u][k];
         ++inserted;
         break;
       }
@@ -144,9 +258,17 @@ __global__ void hq_build_hash_kernel(const __grid_constant__ KBuild b) {
     if (i > b.mask) fault |= HQF_HT_FULL;
   }
   if (fault) atomicOr(b.err, fault);
+  if (!b.count_inserts) return;  // counted builds know their key count already
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) inserted += __shfl_xor_sync(0xffffffffu, inserted, o);
-  if ((threadIdx.x & 31) == 0 && inserted) atomicAdd(b.nkeys, inserted);
+  __shared__ unsigned long long red[BUILD_BLOCK / 32];
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = inserted;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t = 0;
+    for (int k = 0; k < BUILD_BLOCK / 32; ++k) t += red[k];
+    if (t) atomicAdd(b.nkeys, t);
+  }
 }
 
 int64_t next_pow2(int64_t x) {
@@ -180,14 +302,27 @@ void to_kpred(const hq_pred& in, KBuildPred& out, int ncols) {
 
 }  // namespace
 
-// Host side of hq_build_hash (called from hq_api.cu).
-void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
+// Host side of hq_build_hash / hq_build_hashes (called from hq_api.cu).  The
+// builds of one call share ONE host synchronisation: every table's count pass
+// is launched first, their statistics come back together, then the slot arrays
+// are sized, filled, built and compacted (all stream-ordered, no further sync).
+namespace {
+struct BuildState {
+  KBuild b{};
+  int grid = 0;
+  int words = 0;
+  bool counted = false;
+  DevBuf scratch;  // count-pass block partials
+  struct { unsigned long long cnt; int kmin, kmax, pmin, pmax; } st{};
+};
+
+void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& bs) {
   const hq_table* t = d->src;
   if (!t) HQ_THROW(HQ_ERR_ARG, "build: NULL source table");
   if (d->npreds < 0 || d->npreds > HQ_MAX_PREDS) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: too many predicates");
   if (d->npayload < 0 || d->npayload > HQ_MAX_PAYLOAD) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: 0..3 payload columns");
   if (d->key_col < 0 || d->key_col >= t->ncols) HQ_THROW(HQ_ERR_ARG, "build: key column out of range");
-  KBuild b{};
+  KBuild& b = bs.b;
   b.n = t->nrows;
   for (int c = 0; c < t->ncols; ++c) {
     b.col[c] = (const char*)t->cols[c].ptr;
@@ -206,26 +341,35 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   b.err = h->dstate.as<int>();
   b.nkeys = (unsigned long long*)(h->dstate.as<char>() + 8);
   b.kminmax = (int*)(h->dstate.as<char>() + 16);
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((b.n + 255) / 256, (int64_t)ctx->num_sms * 8));
-  int64_t keys = d->expected_rows;
-  const int words = d->npayload == 0 ? 1 : (d->npayload == 1 ? 2 : 4);
-  bool direct = false;
-  int64_t kmin = 0, range = 0;
-  if (keys <= 0) {  // exact count pass (one sync): number and range of the qualifying keys
+  bs.grid = (int)std::max<int64_t>(1, (b.n + BUILD_BLOCK * BUILD_U - 1) / (BUILD_BLOCK * BUILD_U));
+  bs.words = d->npayload == 0 ? 1 : (d->npayload == 1 ? 2 : 4);
+  bs.counted = d->expected_rows <= 0;
+  if (bs.counted) {  // exact count pass: number and range of the qualifying keys
     const int init[4] = {INT_MAX, INT_MIN, INT_MAX, INT_MIN};
     HQ_CUDA(cudaMemcpyAsync(b.kminmax, init, 16, cudaMemcpyHostToDevice, ctx->stream));
-    if (b.n > 0) { ctx->launches++; hq_build_count_kernel<<<grid, 256, 0, ctx->stream>>>(b); }
+    bs.scratch = DevBuf(ctx, (size_t)bs.grid * sizeof(CountPart) + 16);
+    b.part = bs.scratch.p;
+    b.ticket = (unsigned*)(h->dstate.as<char>() + 32);  // zeroed with dstate
+    if (b.n > 0) { ctx->launches++; hq_build_count_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b); }
     HQ_CUDA(cudaGetLastError());
-    struct { unsigned long long cnt; int kmin, kmax, pmin, pmax; } st{};
-    HQ_CUDA(cudaMemcpyAsync(&st, b.nkeys, 24, cudaMemcpyDeviceToHost, ctx->stream));
-    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    HQ_CUDA(cudaMemcpyAsync(&bs.st, b.nkeys, 24, cudaMemcpyDeviceToHost, ctx->stream));
+  }
+}
+
+void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& bs) {
+  KBuild& b = bs.b;
+  const int words = bs.words;
+  int64_t keys = d->expected_rows;
+  bool direct = false;
+  int64_t kmin = 0, range = 0;
+  if (bs.counted) {
     HQ_CUDA(cudaMemsetAsync(b.nkeys, 0, 8, ctx->stream));
-    keys = (int64_t)st.cnt;
-    h->meta.pay_min = st.pmin;
-    h->meta.pay_max = st.pmax;
-    if (keys > 0 && st.kmin <= st.kmax) {
-      kmin = st.kmin;
-      range = (int64_t)st.kmax - st.kmin + 1;
+    keys = (int64_t)bs.st.cnt;
+    h->meta.pay_min = bs.st.pmin;
+    h->meta.pay_max = bs.st.pmax;
+    if (keys > 0 && bs.st.kmin <= bs.st.kmax) {
+      kmin = bs.st.kmin;
+      range = (int64_t)bs.st.kmax - bs.st.kmin + 1;
       // dense keys: direct-mapped slot array (one load per probe)
       direct = range <= (1LL << 30) && (range <= 8 * keys || range * words * 4 <= (2LL << 20));
     }
@@ -240,7 +384,7 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   h->meta.capacity = cap;
   h->meta.slot_words = words;
   h->meta.npayload = d->npayload;
-  h->meta.nkeys = d->expected_rows <= 0 ? keys : -1;  // exact after the count pass (confirmed at hq_hash_info)
+  h->meta.nkeys = bs.counted ? keys : -1;  // exact after the count pass (confirmed at hq_hash_info)
   h->meta.bytes = cap * words * 4;
   h->meta.layout = direct ? HQ_HT_DIRECT : HQ_HT_LINEAR;
   h->meta.key_min = kmin;
@@ -256,22 +400,35 @@ void hq_build_hash_impl(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h) {
   b.words = words;
   b.direct = direct;
   b.dmin = (int32_t)kmin;
-  if (b.n > 0) { ctx->launches++; hq_build_hash_kernel<<<grid, 256, 0, ctx->stream>>>(b); }
+  b.count_inserts = bs.counted ? 0 : 1;
+  if (b.n > 0) { ctx->launches++; hq_build_hash_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b); }
   HQ_CUDA(cudaGetLastError());
   hq_build_compact(ctx, h);
 }
+}  // namespace
+
+void hq_build_hashes_impl(hq_ctx* ctx, int n, const hq_build_desc* d, hq_hash* const* h) {
+  std::vector<BuildState> bs((size_t)n);
+  bool any_count = false;
+  for (int i = 0; i < n; ++i) {
+    build_prepare(ctx, d + i, h[i], bs[i]);
+    any_count = any_count || bs[i].counted;
+  }
+  if (any_count) HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  for (int i = 0; i < n; ++i) build_finish(ctx, d + i, h[i], bs[i]);
+}
 
 namespace {
-// bitmap of present keys: thread per 32-key word
+// bitmap of present keys: a warp reads 32 consecutive slots (coalesced) and
+// one ballot is the word
 __global__ void hq_compact_bitmap_kernel(const uint32_t* slots, long long range, uint32_t* out) {
   const long long nwords = (range + 31) / 32;
-  for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < nwords; w += (long long)gridDim.x * blockDim.x) {
-    uint32_t bits = 0;
-    for (int b = 0; b < 32; ++b) {
-      const long long i = w * 32 + b;
-      if (i < range && (int)slots[i] != INT_MIN) bits |= 1u << b;
-    }
-    out[w] = bits;
+  const int lane = threadIdx.x & 31;
+  const long long wstride = (long long)gridDim.x * (blockDim.x >> 5);
+  for (long long w = blockIdx.x * (long long)(blockDim.x >> 5) + (threadIdx.x >> 5); w < nwords; w += wstride) {
+    const long long i = w * 32 + lane;
+    const uint32_t bits = __ballot_sync(0xffffffffu, i < range && (int)slots[i] != INT_MIN);
+    if (lane == 0) out[w] = bits;
   }
 }
 // key-range bitmap of a linear table: one bit per key in [kmin, kmin + range)
@@ -284,32 +441,35 @@ __global__ void hq_prefilter_kernel(const uint32_t* slots, long long cap, int wo
     if (d >= 0 && d < range) atomicOr(bm + (d >> 5), 1u << (d & 31));
   }
 }
-// one byte per key: payload0 - pay_min, 0xFF = absent (8-B slots {key, payload})
+// one byte per key: payload0 - pay_min, 0xFF = absent (8-B slots {key, payload});
+// thread per key, coalesced 8-B slot reads and byte writes
 __global__ void hq_compact_u8_kernel(const uint32_t* slots, long long range, int pay_min, uint32_t* out) {
-  const long long nwords = (range + 3) / 4;
-  for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < nwords; w += (long long)gridDim.x * blockDim.x) {
-    uint32_t v = 0;
-    for (int b = 0; b < 4; ++b) {
-      const long long i = w * 4 + b;
-      uint32_t byte = 0xFFu;
-      if (i < range && (int)slots[2 * i] != INT_MIN) byte = (uint32_t)((int)slots[2 * i + 1] - pay_min) & 0xFFu;
-      v |= byte << (8 * b);
+  unsigned char* o = (unsigned char*)out;
+  const long long n = (range + 3) / 4 * 4;  // whole words (the tail bytes read as absent)
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    uint32_t byte = 0xFFu;
+    if (i < range) {
+      const uint2 s = ((const uint2*)slots)[i];
+      if ((int)s.x != INT_MIN) byte = (uint32_t)((int)s.y - pay_min) & 0xFFu;
     }
-    out[w] = v;
+    o[i] = (unsigned char)byte;
   }
 }
-// one nibble per key: payload0 - pay_min (< 15), 0xF = absent (8-B slots {key, payload})
+// one nibble per key: payload0 - pay_min (< 15), 0xF = absent (8-B slots
+// {key, payload}); thread per key, eight lanes OR their nibbles into a word
 __global__ void hq_compact_u4_kernel(const uint32_t* slots, long long range, int pay_min, uint32_t* out) {
-  const long long nwords = (range + 7) / 8;
-  for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < nwords; w += (long long)gridDim.x * blockDim.x) {
-    uint32_t v = 0;
-    for (int b = 0; b < 8; ++b) {
-      const long long i = w * 8 + b;
-      uint32_t nib = 0xFu;
-      if (i < range && (int)slots[2 * i] != INT_MIN) nib = (uint32_t)((int)slots[2 * i + 1] - pay_min) & 0xFu;
-      v |= nib << (4 * b);
+  const long long n = (range + 255) / 256 * 256;  // whole warps (the tail reads as absent)
+  const int lane = threadIdx.x & 31;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    uint32_t nib = 0xFu;
+    if (i < range) {
+      const uint2 s = ((const uint2*)slots)[i];
+      if ((int)s.x != INT_MIN) nib = (uint32_t)((int)s.y - pay_min) & 0xFu;
     }
-    out[w] = v;
+    uint32_t v = nib << (4 * (lane & 7));
+#pragma unroll
+    for (int o = 1; o < 8; o <<= 1) v |= __shfl_xor_sync(0xffffffffu, v, o);
+    if ((lane & 7) == 0 && i / 8 < (range + 7) / 8) out[i / 8] = v;
   }
 }
 }  // namespace
@@ -348,7 +508,7 @@ void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
   if (!kind) return;
   const long long words = kind == 1 ? (range + 31) / 32 : (kind == 3 ? (range + 7) / 8 : (range + 3) / 4);
   h->compact = DevBuf(ctx, (size_t)words * 4 + 16);
-  const int grid = (int)std::max<long long>(1, std::min<long long>((words + 255) / 256, (long long)ctx->num_sms * 8));
+  const int grid = (int)std::max<long long>(1, std::min<long long>((range + 255) / 256, (long long)ctx->num_sms * 8));
   ctx->launches++;
   if (kind == 1) hq_compact_bitmap_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->compact.as<uint32_t>());
   else if (kind == 2) hq_compact_u8_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>());
@@ -364,7 +524,7 @@ void hq_hash_check(hq_ctx* ctx, hq_hash* h) {
   int st[4];
   HQ_CUDA(cudaMemcpyAsync(st, h->dstate.p, 16, cudaMemcpyDeviceToHost, ctx->stream));
   HQ_CUDA(cudaStreamSynchronize(ctx->stream));
-  h->meta.nkeys = (int64_t)(*(unsigned long long*)(st + 2));
+  if (h->meta.nkeys < 0) h->meta.nkeys = (int64_t)(*(unsigned long long*)(st + 2));  // expected_rows builds
   h->checked = true;
   if (st[0] & HQF_DUP_KEY) HQ_THROW(HQ_ERR_DUP_KEY, "hash build: duplicate key (join keys must be unique)");
   if (st[0] & HQF_BAD_KEY) HQ_THROW(HQ_ERR_ARG, "hash build: key INT32_MIN or outside int32");

@@ -147,6 +147,113 @@ __global__ void hq_gather_kernel(const long long* src, const int* idx, long long
     dst[i] = src[idx[i]];
 }
 
+// ---- small dense results (SSB/TPC-H aggregates: <= 4,375 groups): compaction,
+// AVG, ORDER BY and LIMIT in ONE block, rows staged to the host with the fault
+// bits in the same copy -- one launch and one host sync per finalize.
+constexpr int SMALL_FIN = 4096;
+constexpr int FIN_THREADS = 1024;
+struct KSmall {
+  KCompact k;                 // k.out: row-major-by-column scratch, capacity ngroups
+  KSort s;                    // over k.out
+  long long limit;            // <= 0: all rows
+  long long* res[MAXRC];      // final columns
+  unsigned long long* stats;  // [0] rows kept, [1] qualifying, [2] fault bits, [3] rows before LIMIT, [4] pipeline faults
+  const int* pipe_err;        // the pipeline's fault word (copied into stats[4])
+};
+__global__ void __launch_bounds__(FIN_THREADS) hq_finalize_small_kernel(const __grid_constant__ KSmall q) {
+  __shared__ int idx[SMALL_FIN];
+  __shared__ int wsum[32];
+  __shared__ int base, tot;
+  __shared__ unsigned long long qual_s;
+  __shared__ int err_s;
+  const KCompact& k = q.k;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  if (tid == 0) { base = 0; qual_s = 0; err_s = 0; }
+  __syncthreads();
+  // 1. ordered compaction of the non-empty groups (block scan of ballots)
+  for (long long g0 = 0; g0 < k.ngroups; g0 += FIN_THREADS) {
+    const long long g = g0 + tid;
+    const bool ne = g < k.ngroups && (k.scalar || k.gtab[g * k.vwords] != 0);
+    const unsigned bal = __ballot_sync(0xffffffffu, ne);
+    if (lane == 0) wsum[w] = __popc(bal);
+    __syncthreads();
+    if (w == 0) {
+      const int v = wsum[lane];
+      int incl = v;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+      }
+      wsum[lane] = incl - v;
+      if (lane == 31) tot = incl;
+    }
+    __syncthreads();
+    if (ne) idx[base + wsum[w] + __popc(bal & ((1u << lane) - 1u))] = (int)g;
+    __syncthreads();
+    if (tid == 0) base += tot;
+    __syncthreads();
+  }
+  const int n = base;
+  // 2. one row per group: decoded keys, aggregates, AVG, int64 guard
+  unsigned long long qsum = 0;
+  bool big = false;
+  for (int i = tid; i < n; i += FIN_THREADS) {
+    const long long g = idx[i];
+    const long long* e = k.gtab + g * k.vwords;
+    const long long cnt = e[0];
+    qsum += (unsigned long long)cnt;
+    for (int c = 0; c < k.nkeys; ++c)
+      k.out[c][i] = k.key_min[c] + (long long)(((unsigned long long)g / (unsigned long long)k.key_stride[c]) % (unsigned long long)k.key_card[c]);
+    for (int a = 0; a < k.naggs; ++a) {
+      const long long v = e[1 + a];
+      long long* o = k.out[k.nkeys + a];
+      if (k.agg_fn[a] == HQ_AGG_AVG) {
+        const double d = cnt ? (double)v / (double)cnt / k.agg_div[a] : __longlong_as_double(0x7ff8000000000000LL);
+        o[i] = __double_as_longlong(d);
+      } else {
+        o[i] = v;
+      }
+      if ((k.agg_fn[a] == HQ_AGG_SUM || k.agg_fn[a] == HQ_AGG_AVG) && (v >= (1LL << 62) || v <= -(1LL << 62))) big = true;
+    }
+  }
+  if (qsum) atomicAdd(&qual_s, qsum);
+  if (big) atomicOr(&err_s, HQF_OVERFLOW);
+  __syncthreads();
+  // 3. ORDER BY (+ group keys, row id: a total order) -- bitonic network in shared memory
+  int net = 32;
+  while (net < n) net <<= 1;
+  for (int i = tid; i < net; i += FIN_THREADS) idx[i] = i < n ? i : -1;
+  __syncthreads();
+  if (n > 1 && (q.s.norder > 0 || k.nkeys > 0)) {
+    for (int kk = 2; kk <= net; kk <<= 1) {
+      for (int j = kk >> 1; j > 0; j >>= 1) {
+        for (int i = tid; i < net; i += FIN_THREADS) {
+          const int l = i ^ j;
+          if (l > i) {
+            const int a = idx[i], b = idx[l];
+            const bool up = (i & kk) == 0;
+            const bool sw = up ? row_less(q.s, b, a) : row_less(q.s, a, b);
+            if (sw) { idx[i] = b; idx[l] = a; }
+          }
+        }
+        __syncthreads();
+      }
+    }
+  }
+  // 4. LIMIT + gather into the result columns
+  const int nf = q.limit > 0 && q.limit < n ? (int)q.limit : n;
+  for (int c = 0; c < k.nkeys + k.naggs; ++c)
+    for (int i = tid; i < nf; i += FIN_THREADS) q.res[c][i] = k.out[c][idx[i]];
+  if (tid == 0) {
+    q.stats[0] = (unsigned long long)nf;
+    q.stats[1] = qual_s;
+    q.stats[2] = (unsigned long long)err_s;
+    q.stats[3] = (unsigned long long)n;
+    q.stats[4] = (unsigned long long)(unsigned)*q.pipe_err;
+  }
+}
+
 // smallest power-of-two bitonic network (>= 32) that holds n rows
 int net_for(long long n) {
   int v = 32;
@@ -160,8 +267,106 @@ int grid_for(hq_ctx* ctx, long long n) {
 
 }  // namespace
 
+namespace {
+void* pinned_staging(hq_ctx* ctx, size_t bytes) {
+  if (ctx->pinned_bytes < bytes) {
+    if (ctx->pinned) HQ_CUDA(cudaFreeHost(ctx->pinned));
+    ctx->pinned = nullptr;
+    ctx->pinned_bytes = 0;
+    const size_t want = std::max<size_t>(bytes, 1 << 20);
+    HQ_CUDA(cudaHostAlloc(&ctx->pinned, want, cudaHostAllocDefault));
+    ctx->pinned_bytes = want;
+  }
+  return ctx->pinned;
+}
+
+// one launch, one sync: fault bits + finalized rows come back together
+bool finalize_small(hq_ctx* ctx, hq_result* r) {
+  const hq_plan& P = r->plan;
+  const int nk = P.nkeys, na = P.naggs, nc = nk + na;
+  if (P.norder < 0 || P.norder > HQ_MAX_ORDER) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: 0..4 ORDER BY columns");
+  for (int i = 0; i < P.norder; ++i)
+    if (P.order_col[i] < 0 || P.order_col[i] >= nc) HQ_THROW(HQ_ERR_ARG, "plan: ORDER BY column out of range");
+  const int64_t ng = std::max<int64_t>(r->ngroups, 1);
+  const int64_t rcap = P.limit > 0 ? std::min<int64_t>(ng, P.limit) : ng;
+  std::vector<DevBuf> cols;
+  for (int c = 0; c < nc; ++c) cols.emplace_back(ctx, (size_t)ng * 8);
+  // [stats: 64 B][column 0: rcap rows][column 1]... -- one D2H copy brings it all back
+  const size_t body = (size_t)nc * rcap * 8;
+  DevBuf pack(ctx, 64 + body);
+  KSmall q{};
+  KCompact& k = q.k;
+  k.gtab = r->gtab.as<long long>();
+  k.ngroups = r->ngroups;
+  k.vwords = r->vwords;
+  k.nkeys = nk;
+  k.naggs = na;
+  k.scalar = nk == 0;
+  int64_t st = 1;
+  for (int i = nk - 1; i >= 0; --i) {
+    k.key_stride[i] = st;
+    st *= P.key_card[i];
+  }
+  for (int i = 0; i < nk; ++i) {
+    k.key_min[i] = P.key_min[i];
+    k.key_card[i] = P.key_card[i];
+    r->types[i] = HQ_I64;
+  }
+  for (int a = 0; a < na; ++a) {
+    k.agg_fn[a] = (uint8_t)P.agg_fn[a];
+    double d = 1.0;
+    for (int s2 = 0; s2 < P.agg_scale[a]; ++s2) d *= 10.0;
+    k.agg_div[a] = d;
+    r->types[nk + a] = P.agg_fn[a] == HQ_AGG_AVG ? HQ_F64 : HQ_I64;
+  }
+  for (int c = 0; c < nc; ++c) {
+    k.out[c] = cols[c].as<long long>();
+    q.s.col[c] = cols[c].as<long long>();
+    q.s.isf[c] = r->types[c] == HQ_F64;
+    q.res[c] = (long long*)(pack.as<char>() + 64 + (size_t)c * rcap * 8);
+  }
+  q.s.norder = P.norder;
+  for (int i = 0; i < P.norder; ++i) {
+    q.s.ocol[i] = P.order_col[i];
+    q.s.odesc[i] = P.order_desc[i];
+  }
+  q.s.nkeys = nk;
+  q.limit = P.limit;
+  q.stats = pack.as<unsigned long long>();
+  q.pipe_err = (const int*)(r->dstate.as<char>() + 8);
+  ctx->launches++;
+  hq_finalize_small_kernel<<<1, FIN_THREADS, 0, ctx->stream>>>(q);
+  HQ_CUDA(cudaGetLastError());
+  char* h = (char*)pinned_staging(ctx, 64 + body);
+  HQ_CUDA(cudaMemcpyAsync(h, pack.p, 64 + body, cudaMemcpyDeviceToHost, ctx->stream));
+  HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  const unsigned long long* sv = (const unsigned long long*)h;
+  if (!r->checked && sv[4]) return false;  // faults: the caller checks (and may re-run), then retries
+  r->checked = true;
+  if (sv[2] & HQF_OVERFLOW) HQ_THROW(HQ_ERR_OVERFLOW, "aggregate exceeds the int64 guard (|v| >= 2^62)");
+  const int64_t nf = (int64_t)sv[0];
+  r->qualifying = (int64_t)sv[1];
+  r->ncols = nc;
+  r->host_rows.assign((size_t)nc * nf, 0);
+  for (int c = 0; c < nc; ++c)
+    std::memcpy(r->host_rows.data() + (size_t)c * nf, h + 64 + (size_t)c * rcap * 8, (size_t)nf * 8);
+  r->host_ready = true;
+  r->rescol.assign((size_t)nc, nullptr);
+  for (int c = 0; c < nc; ++c) r->rescol[c] = pack.as<char>() + 64 + (size_t)c * rcap * 8;
+  r->respack = std::move(pack);
+  r->nrows = nf;
+  r->finalized = true;
+  return true;
+}
+}  // namespace
+
 void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
   if (r->finalized) return;
+  if (r->sink == HQ_SINK_AGG && r->gmode != GM_HASH && r->ngroups <= SMALL_FIN) {
+    if (finalize_small(ctx, r)) return;
+    hq_check_result_faults(ctx, r);  // throws, or re-runs the pipeline with more room
+    if (finalize_small(ctx, r)) return;
+  }
   hq_check_result_faults(ctx, r);
   const hq_plan& P = r->plan;
   if (r->sink == HQ_SINK_MATERIALISE) {
@@ -293,6 +498,8 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
     cols = std::move(out);
   }
   r->rescols = std::move(cols);
+  r->rescol.clear();
+  for (auto& c : r->rescols) r->rescol.push_back(c.p);
   r->nrows = nfinal;
   r->finalized = true;
 }

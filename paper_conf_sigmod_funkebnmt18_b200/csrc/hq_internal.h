@@ -55,6 +55,8 @@ struct hq_ctx {
   int64_t launches = 0;  // kernels this context has launched (hq_ctx_launches)
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> events;  // recorded, not yet read
   std::vector<cudaEvent_t> event_pool;
+  void* pinned = nullptr;  // host staging for small results (cudaHostAlloc, grown on demand)
+  size_t pinned_bytes = 0;
   void* alloc_bytes(size_t bytes);
   void free_bytes(void* p, size_t bytes);
 };
@@ -286,7 +288,11 @@ struct hq_result : RefObj {
   int64_t qualifying = 0;
   int ncols = 0;
   int types[HQ_MAX_KEYS + HQ_MAX_AGGS] = {0};
-  std::vector<DevBuf> rescols;  // finalized result columns (int64 / f64)
+  std::vector<DevBuf> rescols;  // finalized result columns (int64 / f64) ...
+  DevBuf respack;                // ... or packed in one buffer (small results)
+  std::vector<void*> rescol;     // device pointer of each finalized column
+  std::vector<long long> host_rows;  // small results: the finalized rows already on the host
+  bool host_ready = false;           // (column-major, nrows per column)
   ~hq_result() override;
 };
 

@@ -358,7 +358,8 @@ std::string generate(const KPlan& kp) {
   Gen g(kp);
   // HQ_JIT_PROF=1 (debug): per-CTA globaltimer start/end and barrier-wait cycles
   const bool prof = getenv("HQ_JIT_PROF") != nullptr;
-  const int wait_ns = 128;  // consumer back-off between barrier polls
+  int wait_ns = 128;  // consumer back-off between barrier polls (HQ_JIT_WAIT_NS: tuning)
+  if (const char* e = getenv("HQ_JIT_WAIT_NS")) wait_ns = atoi(e);
   std::ostringstream& o = g.o;
   const bool c2 = kp.resolution == HQ_RES_ATOMIC;
   const int sk = kp.sink == HQ_SINK_MATERIALISE ? 2 : (kp.nkeys == 0 ? 0 : 1);

@@ -101,6 +101,10 @@ class DistributedEngine(Engine):
         h = super().hash(table, key, payload, preds, expected_rows) if self.rank == self.root else None
         return self._share(h)
 
+    def hashes(self, specs) -> List[hq.Hash]:
+        hs = super().hashes(specs) if self.rank == self.root else [None] * len(specs)
+        return [self._share(h) for h in hs]
+
     def hash_from(self, res, names, key, payload=()) -> hq.Hash:
         h = super().hash_from(res, names, key, payload) if self.rank == self.root else None
         return self._share(h)

@@ -190,6 +190,16 @@ class Engine:
         ps = [hq.make_pred(t.col(p[0]), *p[1:]) for p in preds]
         return self.ctx.build_hash(t, t.col(key), [t.col(c) for c in payload], ps, expected_rows)
 
+    def hashes(self, specs: Sequence[dict]) -> List[hq.Hash]:
+        """Independent builds (a query's dimension tables) with one host sync:
+        specs = [dict(table=, key=, payload=(), preds=(), expected_rows=0), ...]."""
+        out = []
+        for sp in specs:
+            t = self.tables[sp["table"]]
+            ps = [hq.make_pred(t.col(p[0]), *p[1:]) for p in sp.get("preds", ())]
+            out.append((t, t.col(sp["key"]), [t.col(c) for c in sp.get("payload", ())], ps, sp.get("expected_rows", 0)))
+        return self.ctx.build_hashes(out)
+
     def hash_from(self, res: Optional[hq.Result], names: Sequence[str], key: str,
                   payload: Sequence[str] = ()) -> hq.Hash:
         """Build a hash table from a materialised pipeline result (pipeline breaker)."""

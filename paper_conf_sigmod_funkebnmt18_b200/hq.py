@@ -114,7 +114,7 @@ STRUCTS = {"hq_column": Column, "hq_pred": Pred, "hq_build_desc": BuildDesc, "hq
 EXPORTS = ["hq_ctx_create", "hq_ctx_destroy", "hq_ctx_set_stream", "hq_ctx_sync", "hq_last_error",
            "hq_abi_version", "hq_sizeof", "hq_ctx_enable_timing", "hq_ctx_kernel_times", "hq_ctx_launches",
            "hq_load_columns",
-           "hq_table_info", "hq_table_column", "hq_free_table", "hq_build_hash", "hq_hash_info",
+           "hq_table_info", "hq_table_column", "hq_free_table", "hq_build_hash", "hq_build_hashes", "hq_hash_info",
            "hq_hash_device_view", "hq_hash_import", "hq_free_hash", "hq_run_pipeline", "hq_finalize",
            "hq_result_info_get", "hq_fetch_result", "hq_result_as_table", "hq_result_partials_view",
            "hq_free_result"]
@@ -146,6 +146,7 @@ def lib():
             "hq_load_columns": [vp, P(Column), i32, i64, i32, P(vp)],
             "hq_table_info": [vp, P(i64), P(i32)], "hq_table_column": [vp, i32, P(vp), P(i32)],
             "hq_free_table": [vp], "hq_build_hash": [vp, P(BuildDesc), P(vp)],
+            "hq_build_hashes": [vp, i32, P(BuildDesc), P(vp)],
             "hq_hash_info": [vp, vp, P(HashMeta)], "hq_hash_device_view": [vp, P(vp), P(HashMeta)],
             "hq_hash_import": [vp, P(HashMeta), vp, P(vp)], "hq_free_hash": [vp],
             "hq_run_pipeline": [vp, P(Plan), P(vp)], "hq_finalize": [vp, vp],
@@ -246,9 +247,9 @@ class Context:
     def load_columns(self, cols: Dict[str, object], host_copy: Optional[bool] = None) -> "Table":
         return Table.load(self, cols, host_copy)
 
-    def build_hash(self, src: "Table", key: int, payload: Sequence[int] = (), preds: Sequence[Pred] = (),
-                   expected_rows: int = 0) -> "Hash":
-        d = BuildDesc()
+    @staticmethod
+    def _build_desc(d: "BuildDesc", src: "Table", key: int, payload: Sequence[int], preds: Sequence[Pred],
+                    expected_rows: int) -> None:
         d.src = src.h
         if len(preds) > MAX_PREDS:
             raise ValueError("too many build predicates")
@@ -260,9 +261,24 @@ class Context:
         for i, c in enumerate(payload):
             d.payload_cols[i] = c
         d.expected_rows = expected_rows
+
+    def build_hash(self, src: "Table", key: int, payload: Sequence[int] = (), preds: Sequence[Pred] = (),
+                   expected_rows: int = 0) -> "Hash":
+        d = BuildDesc()
+        self._build_desc(d, src, key, payload, preds, expected_rows)
         h = ctypes.c_void_p()
         check(lib().hq_build_hash(self.h, ctypes.byref(d), ctypes.byref(h)))
         return Hash(self, h, keep=[src])
+
+    def build_hashes(self, specs: Sequence[tuple]) -> List["Hash"]:
+        """Several builds, one host sync: specs = [(src, key, payload, preds, expected_rows), ...]."""
+        n = len(specs)
+        ds = (BuildDesc * n)()
+        for d, (src, key, payload, preds, exp) in zip(ds, specs):
+            self._build_desc(d, src, key, payload, preds, exp)
+        hs = (ctypes.c_void_p * n)()
+        check(lib().hq_build_hashes(self.h, n, ds, hs))
+        return [Hash(self, ctypes.c_void_p(hs[i]), keep=[specs[i][0]]) for i in range(n)]
 
     def import_hash(self, meta: HashMeta, dev_ptr: int, keep=None) -> "Hash":
         h = ctypes.c_void_p()

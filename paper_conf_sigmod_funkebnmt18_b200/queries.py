@@ -97,9 +97,10 @@ def _ssb_q1(v: int):
 
 # ---------------------------------------------------------------- SSB Q3.1
 def _ssb_q31_probes(E: Engine) -> PlanBuilder:
-    hc = E.hash("customer", "c_custkey", payload=["c_nation"], preds=[("c_region", "=", ASIA)])
-    hs = E.hash("supplier", "s_suppkey", payload=["s_nation"], preds=[("s_region", "=", ASIA)])
-    hd = E.hash("date", "d_datekey", payload=["d_year"], preds=[("d_year", "between", 1992, 1997)])
+    hc, hs, hd = E.hashes([
+        dict(table="customer", key="c_custkey", payload=["c_nation"], preds=[("c_region", "=", ASIA)]),
+        dict(table="supplier", key="s_suppkey", payload=["s_nation"], preds=[("s_region", "=", ASIA)]),
+        dict(table="date", key="d_datekey", payload=["d_year"], preds=[("d_year", "between", 1992, 1997)])])
     pb = E.plan("lineorder")
     pb.probe(hs, "lo_suppkey", "inner", ["s_nation"])
     pb.probe(hc, "lo_custkey", "inner", ["c_nation"])
@@ -124,10 +125,11 @@ def _ssb_q31_mat(E: Engine, capacity: int = 0, **_):
 
 # ---------------------------------------------------------------- SSB Q4.1
 def _ssb_q41(E: Engine, **_):
-    hs = E.hash("supplier", "s_suppkey", preds=[("s_region", "=", AMERICA)])
-    hc = E.hash("customer", "c_custkey", payload=["c_nation"], preds=[("c_region", "=", AMERICA)])
-    hp = E.hash("part", "p_partkey", preds=[("p_mfgr", "in", [MFGR1, MFGR2])])
-    hd = E.hash("date", "d_datekey", payload=["d_year"])
+    hs, hc, hp, hd = E.hashes([
+        dict(table="supplier", key="s_suppkey", preds=[("s_region", "=", AMERICA)]),
+        dict(table="customer", key="c_custkey", payload=["c_nation"], preds=[("c_region", "=", AMERICA)]),
+        dict(table="part", key="p_partkey", preds=[("p_mfgr", "in", [MFGR1, MFGR2])]),
+        dict(table="date", key="d_datekey", payload=["d_year"])])
     pb = E.plan("lineorder")
     pb.probe(hs, "lo_suppkey", "semi")
     pb.probe(hc, "lo_custkey", "inner", ["c_nation"])
