@@ -192,6 +192,8 @@ typedef struct {
   int32_t pay_min;      /* min / max of payload 0 over the inserted rows (count pass) */
   int32_t pay_max;
   int32_t key_max;      /* max key inserted (count pass); key range = [key_min, key_max] */
+  uint64_t pay_set[4];  /* payload-0 values present: bit (v & 255) (count pass); exact when
+                         * pay_max - pay_min < 256, all-zero when unknown (expected_rows builds) */
 } hq_hash_meta;
 /* Derived forms (rebuilt on import): direct tables get a compact form -- a
  * bitmap of present keys for semi-join tables, or one byte per key (payload -

@@ -36,6 +36,7 @@ struct KBuild {
   int* err;
   unsigned long long* nkeys;
   int* kminmax;      // count pass: [min, max] of the qualifying keys, [min, max] of payload 0
+  unsigned* pset;    // count pass: payload-0 values present, bit (v & 255) (8 words)
   void* part;        // count pass: per-block partials (CountPart[grid])
   unsigned* ticket;  // count pass: blocks done
   int count_inserts; // build pass: accumulate the inserted-key count (no count pass ran)
@@ -119,10 +120,12 @@ __device__ __forceinline__ void load_rows(const KBuild& b, long long base, bool 
 struct CountPart {
   unsigned long long cnt;
   int kmin, kmax, pmin, pmax;
+  unsigned set[8];  // payload-0 values present, bit (v & 255)
 };
 __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __grid_constant__ KBuild b) {
   unsigned long long c = 0;
   int kmin = INT_MAX, kmax = INT_MIN, pmin = INT_MAX, pmax = INT_MIN;
+  unsigned pset[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};  // registers: constant indices only
   const long long base = (long long)blockIdx.x * BUILD_BLOCK * BUILD_U + threadIdx.x;
   bool pass[BUILD_U];
   long long kv[BUILD_U], pv[BUILD_U] = {};
@@ -139,6 +142,9 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __gri
       const int pc = pv[u] < (long long)INT_MIN ? INT_MIN : (pv[u] > (long long)INT_MAX ? INT_MAX : (int)pv[u]);
       pmin = min(pmin, pc);
       pmax = max(pmax, pc);
+      const int pw = (pc & 255) >> 5;
+#pragma unroll
+      for (int w8 = 0; w8 < 8; ++w8) pset[w8] |= pw == w8 ? 1u << (pc & 31) : 0u;
     }
   }
   kmin = __reduce_min_sync(0xffffffffu, kmin);
@@ -146,19 +152,23 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __gri
   pmin = __reduce_min_sync(0xffffffffu, pmin);
   pmax = __reduce_max_sync(0xffffffffu, pmax);
 #pragma unroll
+  for (int w8 = 0; w8 < 8; ++w8) pset[w8] = __reduce_or_sync(0xffffffffu, pset[w8]);
+#pragma unroll
   for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
   __shared__ CountPart wp[BUILD_BLOCK / 32];
   __shared__ bool last;
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (lane == 0) wp[w] = {c, kmin, kmax, pmin, pmax};
+  if (lane == 0) wp[w] = {c, kmin, kmax, pmin, pmax, {pset[0], pset[1], pset[2], pset[3], pset[4], pset[5], pset[6], pset[7]}};
   __syncthreads();
   if (threadIdx.x == 0) {
-    CountPart t{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN};
+    CountPart t{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN, {}};
     for (int k = 0; k < BUILD_BLOCK / 32; ++k) {
       t.cnt += wp[k].cnt;
       t.kmin = min(t.kmin, wp[k].kmin); t.kmax = max(t.kmax, wp[k].kmax);
       t.pmin = min(t.pmin, wp[k].pmin); t.pmax = max(t.pmax, wp[k].pmax);
     }
+    for (int k = 0; k < BUILD_BLOCK / 32; ++k)
+      for (int w8 = 0; w8 < 8; ++w8) t.set[w8] |= wp[k].set[w8];
     ((CountPart*)b.part)[blockIdx.x] = t;
     __threadfence();
     last = atomicAdd(b.ticket, 1u) == gridDim.x - 1;
@@ -167,13 +177,17 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __gri
   if (!last) return;
   // last block: reduce every block's partial
   __threadfence();
-  CountPart t{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN};
+  CountPart t{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN, {}};
   for (unsigned k = threadIdx.x; k < gridDim.x; k += BUILD_BLOCK) {
     const volatile CountPart* q = (const volatile CountPart*)b.part + k;
     t.cnt += q->cnt;
     t.kmin = min(t.kmin, q->kmin); t.kmax = max(t.kmax, q->kmax);
     t.pmin = min(t.pmin, q->pmin); t.pmax = max(t.pmax, q->pmax);
+#pragma unroll
+    for (int w8 = 0; w8 < 8; ++w8) t.set[w8] |= q->set[w8];
   }
+#pragma unroll
+  for (int w8 = 0; w8 < 8; ++w8) t.set[w8] = __reduce_or_sync(0xffffffffu, t.set[w8]);
   t.kmin = __reduce_min_sync(0xffffffffu, t.kmin);
   t.kmax = __reduce_max_sync(0xffffffffu, t.kmax);
   t.pmin = __reduce_min_sync(0xffffffffu, t.pmin);
@@ -184,14 +198,16 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __gri
   if (lane == 0) wp[w] = t;
   __syncthreads();
   if (threadIdx.x == 0) {
-    CountPart z{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN};
+    CountPart z{0, INT_MAX, INT_MIN, INT_MAX, INT_MIN, {}};
     for (int k = 0; k < BUILD_BLOCK / 32; ++k) {
       z.cnt += wp[k].cnt;
       z.kmin = min(z.kmin, wp[k].kmin); z.kmax = max(z.kmax, wp[k].kmax);
       z.pmin = min(z.pmin, wp[k].pmin); z.pmax = max(z.pmax, wp[k].pmax);
+      for (int w8 = 0; w8 < 8; ++w8) z.set[w8] |= wp[k].set[w8];
     }
     *b.nkeys = z.cnt;
     b.kminmax[0] = z.kmin; b.kminmax[1] = z.kmax; b.kminmax[2] = z.pmin; b.kminmax[3] = z.pmax;
+    for (int w8 = 0; w8 < 8; ++w8) b.pset[w8] = z.set[w8];
   }
 }
 
@@ -313,7 +329,7 @@ struct BuildState {
   int words = 0;
   bool counted = false;
   DevBuf scratch;  // count-pass block partials
-  struct { unsigned long long cnt; int kmin, kmax, pmin, pmax; } st{};
+  struct { unsigned long long cnt; int kmin, kmax, pmin, pmax; unsigned set[8]; } st{};
 };
 
 void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& bs) {
@@ -336,11 +352,12 @@ void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& 
     if (d->payload_cols[k] < 0 || d->payload_cols[k] >= t->ncols) HQ_THROW(HQ_ERR_ARG, "build: payload column out of range");
     b.pay_col[k] = d->payload_cols[k];
   }
-  h->dstate = DevBuf(ctx, 64);
-  HQ_CUDA(cudaMemsetAsync(h->dstate.p, 0, 64, ctx->stream));
+  h->dstate = DevBuf(ctx, 128);
+  HQ_CUDA(cudaMemsetAsync(h->dstate.p, 0, 128, ctx->stream));
   b.err = h->dstate.as<int>();
   b.nkeys = (unsigned long long*)(h->dstate.as<char>() + 8);
   b.kminmax = (int*)(h->dstate.as<char>() + 16);
+  b.pset = (unsigned*)(h->dstate.as<char>() + 64);
   bs.grid = (int)std::max<int64_t>(1, (b.n + BUILD_BLOCK * BUILD_U - 1) / (BUILD_BLOCK * BUILD_U));
   bs.words = d->npayload == 0 ? 1 : (d->npayload == 1 ? 2 : 4);
   bs.counted = d->expected_rows <= 0;
@@ -353,6 +370,7 @@ void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& 
     if (b.n > 0) { ctx->launches++; hq_build_count_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b); }
     HQ_CUDA(cudaGetLastError());
     HQ_CUDA(cudaMemcpyAsync(&bs.st, b.nkeys, 24, cudaMemcpyDeviceToHost, ctx->stream));
+    HQ_CUDA(cudaMemcpyAsync(bs.st.set, b.pset, 32, cudaMemcpyDeviceToHost, ctx->stream));
   }
 }
 
@@ -362,11 +380,14 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   int64_t keys = d->expected_rows;
   bool direct = false;
   int64_t kmin = 0, range = 0;
+  h->meta.pay_min = INT_MAX;  // payload range unknown unless counted
+  h->meta.pay_max = INT_MIN;
   if (bs.counted) {
     HQ_CUDA(cudaMemsetAsync(b.nkeys, 0, 8, ctx->stream));
     keys = (int64_t)bs.st.cnt;
     h->meta.pay_min = bs.st.pmin;
     h->meta.pay_max = bs.st.pmax;
+    for (int k = 0; k < 4; ++k) h->meta.pay_set[k] = (uint64_t)bs.st.set[2 * k] | ((uint64_t)bs.st.set[2 * k + 1] << 32);
     if (keys > 0 && bs.st.kmin <= bs.st.kmax) {
       kmin = bs.st.kmin;
       range = (int64_t)bs.st.kmax - bs.st.kmin + 1;

@@ -189,6 +189,7 @@ struct KProbe {
   int32_t pay_max;
   uint32_t cbytes;
   uint32_t smem_off; // generated kernels: byte offset of the staged compact table (0 = not staged)
+  uint64_t pay_set[4];  // payload-0 values present, bit (v & 255) (hq_hash_meta::pay_set)
   const uint32_t* pf;  // linear tables: key-range bitmap (NULL = none)
   int32_t pf_min;
   uint32_t pf_range;
@@ -246,8 +247,15 @@ struct KPlan {
   // generated kernels: the shared dense table may index a narrowed key domain
   // (group keys that are probe payloads span only their build-side value range)
   uint8_t local_keys;
+  // generated kernels: copy the tile's columns into registers and release the
+  // stage before the operators run (long-latency probes do not hold the ring)
+  uint8_t early_release;
   int64_t lkey_min[HQ_MAX_KEYS];
   int64_t lkey_stride[HQ_MAX_KEYS];
+  // ... and a key whose payload takes few distinct values (SSB Q3.1: 5 ASIA
+  // nations spread over codes 4..24) is indexed by its rank in this set of
+  // values (bit v - lkey_min); all-zero = plain offset v - lkey_min
+  uint64_t lkey_set[HQ_MAX_KEYS][4];
   int32_t slog2;
   // SM_LANE: deduplicated accumulators (0 = count; SUM and AVG of one register share)
   int32_t nacc;

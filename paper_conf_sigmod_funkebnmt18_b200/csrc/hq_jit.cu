@@ -436,6 +436,13 @@ std::string generate(const KPlan& kp) {
   if (sk == 2)  // output values leave the operator block in registers; the block scan runs after it
     for (int j = 0; j < kp.nout; ++j) o << "    long long ov" << j << "[R];\n";
   o << "    {\n";
+  if (kp.early_release) {
+    // every referenced column of the lane's rows into registers, then the stage
+    // goes back to the producer (mbarrier.arrive releases the warp's prior
+    // shared loads); the operators below run on registers only
+    for (const auto& sk2 : g.stage_k) g.use(sk2.first);
+    o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
+  }
   for (int i = 0; i < kp.nops;) {
     const KOp op = kp.ops[i];
     if (op.kind == OP_PROBE) { i = g.probe_batch(i); continue; }
@@ -473,6 +480,20 @@ std::string generate(const KPlan& kp) {
       // whose payload range is known are narrowed, and those need no check
       const int64_t kmin = kp.local_keys ? kp.lkey_min[i] : kp.key_min[i];
       const int64_t kstr = kp.local_keys ? kp.lkey_stride[i] : kp.key_stride[i];
+      const bool ranked = kp.local_keys && (kp.lkey_set[i][0] | kp.lkey_set[i][1] | kp.lkey_set[i][2] | kp.lkey_set[i][3]);
+      if (ranked) {  // index by the rank of the value among the build side's distinct payloads
+        const std::string rk = "RK_" + std::to_string(i);
+        g.bitmaps << "static constexpr __device__ unsigned char " << rk << "[] = {";
+        int64_t n = 0;
+        for (int64_t d = 0; d < 256; ++d) {
+          const bool on = (kp.lkey_set[i][d >> 6] >> (d & 63)) & 1ull;
+          g.bitmaps << (d ? ", " : "") << (on ? n : 255);
+          n += on;
+        }
+        g.bitmaps << "};\n";
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = ((mask >> r) & 1u) ? (long long)" << rk
+          << "[(u32)((long long)" << v << " - " << lit(kmin) << ") & 255u] : 0LL;";
+      } else
       o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kmin) << ";";
       if (!in_domain)  // payload ranges known from the build's count pass need no domain check
         o << " if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }";
@@ -582,7 +603,8 @@ std::string generate(const KPlan& kp) {
     if (!c2) o << "        run_ += __popc(b_[r]); }\n";
     o << "    }\n";
   }
-  o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
+  if (kp.early_release) o << "    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
+  else o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
   if (prof) o << "  if (lane == 0) { p.prof[blockIdx.x * 128 + 8 + warp] = pw_; p.prof[blockIdx.x * 128 + 40 + warp] = clock64() - pl0_; } if (pdv_) atomicAdd((unsigned long long*)&p.prof[blockIdx.x * 128 + 72 + warp], (unsigned long long)pdv_);\n";
   // ------------------------------------------------------------- sink (end)
   if (sk == 0 && !c2) {
@@ -615,9 +637,19 @@ std::string generate(const KPlan& kp) {
       << "        u64 gkey_ = g;\n";
     if (kp.local_keys) {  // narrowed local index -> declared global key
       o << "        { u64 rem_ = g; gkey_ = 0;";
-      for (int i = 0; i < kp.nkeys; ++i)
-        o << " { const u64 o_ = rem_ / " << kp.lkey_stride[i] << "ull; rem_ -= o_ * " << kp.lkey_stride[i]
-          << "ull; gkey_ += (o_ + " << (kp.lkey_min[i] - kp.key_min[i]) << "ull) * " << kp.key_stride[i] << "ull; }";
+      for (int i = 0; i < kp.nkeys; ++i) {
+        const uint64_t* ls = kp.lkey_set[i];
+        o << " { const u64 o_ = rem_ / " << kp.lkey_stride[i] << "ull; rem_ -= o_ * " << kp.lkey_stride[i] << "ull;";
+        if (ls[0] | ls[1] | ls[2] | ls[3]) {  // rank -> value -> offset in the declared domain
+          o << " const long long dv_[] = {";
+          int n = 0;
+          for (int64_t d = 0; d < 256; ++d)
+            if ((ls[d >> 6] >> (d & 63)) & 1ull) o << (n++ ? ", " : "") << (kp.lkey_min[i] + d - kp.key_min[i]) << "LL";
+          o << "}; gkey_ += (u64)dv_[o_] * " << kp.key_stride[i] << "ull; }";
+        } else {
+          o << " gkey_ += (o_ + " << (kp.lkey_min[i] - kp.key_min[i]) << "ull) * " << kp.key_stride[i] << "ull; }";
+        }
+      }
       o << " }\n";
     }
     o << "        group_update(p, sagg, gkey_, false, (u64)e_[0], vals_); } } }\n";

@@ -132,6 +132,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.compact = op.ht->compact.p;
       pr.pay_min = op.ht->meta.pay_min;
       pr.pay_max = op.ht->meta.pay_max;
+      for (int k = 0; k < 4; ++k) pr.pay_set[k] = op.ht->meta.pay_set[k];
       pr.cbytes = (uint32_t)op.ht->cbytes;
       pr.smem_off = 0;
       pr.pf = op.ht->pf_words ? op.ht->prefilter.as<uint32_t>() : nullptr;
@@ -252,6 +253,22 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         if (pr.pay_min < kp.key_min[i] || (int64_t)pr.pay_max >= kp.key_min[i] + kp.key_card[i]) continue;
         lmin[i] = pr.pay_min;
         lcard[i] = (int64_t)pr.pay_max - pr.pay_min + 1;
+        for (int k = 0; k < 4; ++k) kp.lkey_set[i][k] = 0;
+        if (lcard[i] <= 256) {  // distinct payload values (count pass): index by rank
+          int64_t n = 0;
+          uint64_t rel[4] = {0, 0, 0, 0};
+          for (int64_t d = 0; d < lcard[i]; ++d) {
+            const uint32_t v = (uint32_t)(pr.pay_min + d) & 255u;
+            if ((pr.pay_set[v >> 6] >> (v & 63)) & 1ull) {
+              rel[d >> 6] |= 1ull << (d & 63);
+              ++n;
+            }
+          }
+          if (n > 0 && n < lcard[i]) {
+            lcard[i] = n;
+            for (int k = 0; k < 4; ++k) kp.lkey_set[i][k] = rel[k];
+          }
+        }
       }
       lgroups *= lcard[i];
     }
@@ -283,12 +300,21 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       } else {
         uint32_t cap = 4096;
         while (cap > 64 && (uint64_t)cap * (kp.vwords + 1) * 8 > (uint64_t)SMEM_AGG_BYTES) cap >>= 1;
+        // far more groups than the shared table holds (TPC-H Q3: ~10^5-10^6
+        // orderkeys): it would fill up and every later row would scan it before
+        // going to global memory -- update the global table directly (C2)
+        const int64_t expect = group_cap > 0 ? group_cap : P.group_capacity;
+        const char* nl = getenv("HQ_JIT_NOLOCAL");
+        if (jit && kp.gmode == GM_HASH && expect > 4 * (int64_t)cap && !(nl && nl[0] == '0')) {
+          kp.smode = SM_NONE;
+        } else {
         kp.smode = SM_HASH;
         kp.smem_cap = cap;
         int l = 0;
         while ((1u << l) < cap) ++l;
         kp.slog2 = l;
         agg_smem = cap * (kp.vwords + 1) * 8;
+        }
       }
     }
   } else if (P.sink == HQ_SINK_MATERIALISE) {
@@ -384,6 +410,21 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     --nstaged;  // give the last staged table back to the ring
   }
   if (!chosen_R) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: rows too wide for the shared-memory stage ring");
+  kp.early_release = 0;
+  if (jit) {
+    // early stage release when an operator waits on global memory: linear
+    // probes, probes of tables not staged in shared memory, global hash groups
+    bool slow = kp.sink == HQ_SINK_AGG && kp.gmode == GM_HASH && kp.smode == SM_NONE;
+    for (int o = 0; o < kp.nops; ++o) {
+      if (kp.ops[o].kind != OP_PROBE) continue;
+      const KProbe& pr = kp.probes[kp.ops[o].idx];
+      bool staged_here = false;
+      for (int i = 0; i < nstaged; ++i) staged_here = staged_here || staged[i] == kp.ops[o].idx;
+      if (!pr.direct || !staged_here) slow = true;
+    }
+    kp.early_release = slow ? 1 : 0;
+    if (const char* e = getenv("HQ_JIT_EARLY")) kp.early_release = e[0] == '1' ? 1 : 0;
+  }
   r->segment_rows = kp.tile_rows;
   {
     uint32_t off = kp.off_tab;

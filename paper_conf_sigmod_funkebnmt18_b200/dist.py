@@ -31,6 +31,11 @@ def partition(n: int, rank: int, world: int) -> Tuple[int, int]:
     return n * rank // world, n * (rank + 1) // world
 
 
+def _i64(u: int) -> int:
+    """uint64 bit pattern as a signed int64 (torch.int64 transport)."""
+    return u - (1 << 64) if u >= (1 << 63) else u
+
+
 def broadcast_blob(meta: Optional[Sequence[int]], buf: Optional[torch.Tensor], nbytes_index: int,
                    root: int, device) -> Tuple[List[int], torch.Tensor]:
     """Broadcast a small int64 meta vector, then a byte buffer whose size is
@@ -86,7 +91,7 @@ class DistributedEngine(Engine):
             self._built.append(h)     # build faults are checked in finish()
             buf = device_view(ptr, int(m.bytes))
             meta = [m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout,
-                    m.pay_min, m.pay_max, m.key_max]
+                    m.pay_min, m.pay_max, m.key_max] + [_i64(w) for w in m.pay_set]
         else:
             meta, buf = None, None
         meta, buf = broadcast_blob(meta, buf, 4, self.root, self.device)
@@ -95,6 +100,8 @@ class DistributedEngine(Engine):
         hm = hq.HashMeta()
         (hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout,
          hm.pay_min, hm.pay_max, hm.key_max) = meta[:10]
+        for k in range(4):
+            hm.pay_set[k] = meta[10 + k] & 0xFFFFFFFFFFFFFFFF
         return self.ctx.import_hash(hm, buf.data_ptr(), keep=buf)
 
     def hash(self, table, key, payload=(), preds=(), expected_rows=0) -> hq.Hash:

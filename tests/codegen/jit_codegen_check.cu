@@ -204,6 +204,18 @@ int main(int argc, char** argv) {
     P.ops[0] = probe(na, 1, HQ_PROBE_INNER, HQ_TMP(0));
     P.ops[1] = probe(nb, 0, HQ_PROBE_INNER, HQ_TMP(1));
     shapes.push_back({"star_narrowed_dense", P, nullptr});
+    // payloads of five distinct values spread over 4..24 (SSB Q3.1's ASIA
+    // nations): keys indexed by rank, a 5 x 5 x 7 dense shared table
+    hq_hash* ra = make_hash(c, HQ_HT_DIRECT, 1, 2, 20000);
+    hq_hash* rb = make_hash(c, HQ_HT_DIRECT, 1, 2, 3000000);
+    for (hq_hash* h : {ra, rb}) {
+      h->meta.pay_min = 4;
+      h->meta.pay_max = 24;
+      for (int v : {4, 9, 10, 13, 24}) h->meta.pay_set[v >> 6] |= 1ull << (v & 63);
+    }
+    P.ops[0] = probe(ra, 1, HQ_PROBE_INNER, HQ_TMP(0));
+    P.ops[1] = probe(rb, 0, HQ_PROBE_INNER, HQ_TMP(1));
+    shapes.push_back({"star_ranked_dense", P, nullptr});
   }
   {  // Q6-like scalar aggregate with an int8 bitmap filter and an i64 expression
     hq_plan P{};

@@ -32,7 +32,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     env = {k: v for k, v in os.environ.items() if not k.startswith("HQ_")}
     p = subprocess.run([checker, str(tmp_path)], capture_output=True, text=True, env=env, timeout=600)
     assert p.returncode == 0, p.stdout + p.stderr
-    assert p.stdout.startswith("OK 11 of 11"), p.stdout
+    assert p.stdout.startswith("OK 12 of 12"), p.stdout
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
     star = srcs["star_dense_lrgp"]
@@ -48,3 +48,8 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "#define SMODE 2" in srcs["star_smem_hash"]
     narrowed = srcs["star_narrowed_dense"]
     assert "#define SMODE 1" in narrowed and "#define SMEM_CAP 1183u" in narrowed and "gkey_ +=" in narrowed
+    # ... and by the rank among the payloads' distinct values (5 of the 21 codes 4..24)
+    ranked = srcs["star_ranked_dense"]
+    assert "#define SMEM_CAP 175u" in ranked and "RK_0[" in ranked and "RK_1[" in ranked and "dv_[o_]" in ranked
+    # high-cardinality hash group-by skips the shared table (C2 straight to global)
+    assert "#define SMODE 0" in srcs["global_hash_groups"]
