@@ -190,6 +190,7 @@ struct KProbe {
   uint32_t cbytes;
   uint32_t smem_off; // generated kernels: byte offset of the staged compact table (0 = not staged)
   uint64_t pay_set[4];  // payload-0 values present, bit (v & 255) (hq_hash_meta::pay_set)
+  float pass_est;      // expected fraction of probing rows that pass (key density of the build side)
   const uint32_t* pf;  // linear tables: key-range bitmap (NULL = none)
   int32_t pf_min;
   uint32_t pf_range;

@@ -99,6 +99,8 @@ struct Gen {
   const KPlan& kp;
   std::ostringstream o;
   std::set<int> loaded;        // registers materialised as variables
+  std::map<int, std::string> vtype;  // C type of each materialised register
+  std::set<int> dead;          // materialised before the compaction point, not carried over
   std::map<int, std::pair<long long, long long>> known;  // value range of probe payloads (count pass)
   std::map<int, int> stage_k;  // table column -> stage column index
   explicit Gen(const KPlan& k) : kp(k) {
@@ -116,13 +118,27 @@ struct Gen {
     return var(reg) + "[r]";
   }
   void use(int reg) {
+    if (dead.count(reg)) HQ_THROW(HQ_ERR_STATE, "jit: register used after compaction but not carried over");
     if (loaded.count(reg)) return;
     if (reg >= HQ_MAX_COLS) HQ_THROW(HQ_ERR_ARG, "jit: temporary read before definition");
     const KCol& c = kp.cols[stage_k.at(reg)];
-    o << "      " << ctype(c.width) << " " << var(reg) << "[R];\n"
-      << "      { const " << ctype(c.width) << "* b_ = (const " << ctype(c.width) << "*)(st + " << c.soff
-      << "u) + row0;\n#pragma unroll\n        for (int r = 0; r < R; ++r) " << var(reg) << "[r] = b_[r * 32]; }\n";
+    // a lane's R rows are consecutive (row0 .. row0 + R - 1): one vector load
+    // when they span 8 or 16 bytes (stage columns are 16-B aligned)
+    const int vb = compacted_R ? 0 : (int)c.width * kp.R;
+    const char* vt = vb == 16 ? (c.width == 4 ? "int4" : "longlong2") : (vb == 8 ? (c.width == 4 ? "int2" : "long long") : nullptr);
+    o << "      " << ctype(c.width) << " " << var(reg) << "[R];\n";
+    if (vt && c.width >= 4) {
+      o << "      { const " << vt << " q_ = *(const " << vt << "*)((const " << ctype(c.width) << "*)(st + " << c.soff << "u) + row0);";
+      if (vb == 8 && c.width == 8) o << " " << var(reg) << "[0] = q_; }\n";
+      else if (vb == 8) o << " " << var(reg) << "[0] = q_.x; " << var(reg) << "[1] = q_.y; }\n";
+      else if (c.width == 8) o << " " << var(reg) << "[0] = q_.x; " << var(reg) << "[1] = q_.y; }\n";
+      else o << " " << var(reg) << "[0] = q_.x; " << var(reg) << "[1] = q_.y; " << var(reg) << "[2] = q_.z; " << var(reg) << "[3] = q_.w; }\n";
+    } else {
+      o << "      { const " << ctype(c.width) << "* b_ = (const " << ctype(c.width) << "*)(st + " << c.soff
+        << "u) + row0;\n#pragma unroll\n        for (int r = 0; r < R; ++r) " << var(reg) << "[r] = b_[r]; }\n";
+    }
     loaded.insert(reg);
+    vtype[reg] = ctype(c.width);
   }
   // skip the rest of the operator block when no row of the warp is live; the
   // block stays structured (nested ifs, closed in generate()) so that the
@@ -185,6 +201,7 @@ struct Gen {
       o << "      int " << var(pr.dst[k]) << "[R];\n";
       if (k == 0 && pr.pay_min <= pr.pay_max) known[pr.dst[0]] = {pr.pay_min, pr.pay_max};
       loaded.insert(pr.dst[k]);
+      vtype[pr.dst[k]] = "int";
     }
   }
   void probe_addr(const KProbe& pr, int i) {
@@ -342,7 +359,62 @@ struct Gen {
     }
     o << "        " << dst << "[r] = a_; }\n";
     loaded.insert(c.dst);
+    vtype[c.dst] = "long long";
   }
+  // registers read by ops [from, nops) and by the sink
+  std::set<int> uses_from(int from) const {
+    std::set<int> u;
+    for (int j = from; j < kp.nops; ++j) {
+      const KOp& op = kp.ops[j];
+      if (op.kind == OP_FILTER) u.insert(kp.preds[op.idx].reg);
+      else if (op.kind == OP_PROBE) u.insert(kp.probes[op.idx].key_reg);
+      else {
+        const KCompute& c = kp.comps[op.idx];
+        for (int k = 0; k < c.n; ++k)
+          if (kp.insns[c.first + k].reg >= 0) u.insert(kp.insns[c.first + k].reg);
+      }
+    }
+    for (int a = 0; a < kp.naggs; ++a)
+      if (kp.agg_fn[a] != HQ_AGG_COUNT) u.insert(kp.agg_reg[a]);
+    for (int i = 0; i < kp.nkeys; ++i) u.insert(kp.key_reg[i]);
+    return u;
+  }
+  // Warp compaction of the live rows (selection vector in registers): after a
+  // selective probe most of the R row slots are dead, but predicated code pays
+  // for them.  The live rows of the warp's R slots move into consecutive lanes
+  // (ballot prefix, k-th set bit by popc bisection), registers still needed are
+  // shuffled over, and the rest of the pipeline runs in rounds of 32 rows with
+  // ONE row slot (R redefined to 1 in that scope).  Columns not loaded yet are
+  // read from the stage at the compacted row (row0 redefined).
+  void compact(int from) {
+    const int R0 = kp.R;
+    std::vector<int> live;
+    for (int r : uses_from(from))
+      if (loaded.count(r)) live.push_back(r);
+    o << "      {\n      u32 cb_[R]; int cp_[R + 1]; cp_[0] = 0;\n"
+      << "#pragma unroll\n      for (int r = 0; r < R; ++r) { cb_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); cp_[r + 1] = cp_[r] + __popc(cb_[r]); }\n"
+      << "      for (int i0_ = 0; i0_ < cp_[R]; i0_ += 32) {\n"
+      << "        const int ct_ = i0_ + lane; const bool lv_ = ct_ < cp_[R];\n"
+      << "        int rr_ = 0; u32 cm_ = cb_[0]; int ck_ = ct_;\n"
+      << "#pragma unroll\n        for (int r = 1; r < R; ++r) if (ct_ >= cp_[r]) { rr_ = r; cm_ = cb_[r]; ck_ = ct_ - cp_[r]; }\n"
+      << "        int src_ = 0;\n#pragma unroll\n        for (int s_ = 16; s_ > 0; s_ >>= 1) { const int c_ = __popc((cm_ >> src_) & ((1u << s_) - 1u)); if (ck_ >= c_) { ck_ -= c_; src_ += s_; } }\n"
+      << "        if (!lv_) { src_ = lane; rr_ = 0; }\n";
+    for (int r : live) {
+      const std::string& t = vtype.at(r);
+      o << "        " << t << " x_" << var(r) << " = 0;\n#pragma unroll\n        for (int r = 0; r < R; ++r) { const " << t
+        << " y_ = __shfl_sync(HQ_FULL, " << var(r) << "[r], src_); if (r == rr_) x_" << var(r) << " = y_; }\n";
+    }
+    o << "        {\n#undef R\n#define R 1\n"
+      << "        u32 mask = lv_ ? 1u : 0u;\n"
+      << "        const int row0 = warp * 32 * " << R0 << " + src_ * " << R0 << " + rr_;\n";
+    for (int r : live) o << "        " << vtype.at(r) << " " << var(r) << "[R] = {x_" << var(r) << "};\n";
+    std::set<int> keep(live.begin(), live.end());
+    for (int r : loaded)
+      if (!keep.count(r)) dead.insert(r);
+    open += 3;
+    compacted_R = R0;
+  }
+  int compacted_R = 0;  // original R when compact() ran (restored after the scope)
   std::ostringstream bitmaps;
 };
 
@@ -412,24 +484,27 @@ std::string generate(const KPlan& kp) {
   if (prof) o << "      p.prof[blockIdx.x * 128 + 3] = pw_; p.prof[blockIdx.x * 128 + 4] = clock64() - pl0_;\n";
   o << "    }\n    return;\n  }\n";
   // consumer state
-  o << "  const int row0 = warp * 32 * R + lane;\n";
+  o << "  const int row0 = warp * 32 * R + lane * R;  // the lane's rows: row0 .. row0 + R - 1\n";
   if (sk == 0 && !c2) {
     o << "  u64 scount_ = 0;\n";
     for (int a = 0; a < kp.naggs; ++a) o << "  i64 sacc" << a << " = agg_identity(AGG_FN[" << a << "]);\n";
   }
-  const std::string cwait = "mbar_wait_sleep(&full[s], ph);";
+  // HQ_JIT_WAIT=sleep: the older poll + nanosleep loop (A/B)
+  const char* wm = getenv("HQ_JIT_WAIT");
+  const std::string cwait = (wm && std::string(wm) == "sleep") ? "mbar_wait_sleep(&full[s], ph);" : "mbar_wait_suspend(&full[s], ph);";
   o << "  int s = 0; u32 ph = 0; long long t0 = (first_tile + blockIdx.x) * (long long)T;\n"
-    << "  for (long long j = 0; j < nj; ++j, t0 += tstep) {\n"
+    << "  const int njc = (int)nj;\n"
+    << "  for (int j = 0; j < njc; ++j, t0 += tstep) {\n"
     << (prof ? "    { const long long c_ = clock64(); " + cwait + " pw_ += clock64() - c_; if (__activemask() != 0xffffffffu) ++pdv_; }\n" : "    " + cwait + "\n")
     << "    const char* st = stages + (size_t)s * STAGE_STRIDE;\n"
     << "    u32 mask = (1u << R) - 1u;\n"
-    << "    if (t0 < p.row_begin || t0 + T > p.row_end) {  // ragged head / tail tile: lanes copy their rows\n"
+    << "    if ((j == 0 || j == njc - 1) && (t0 < p.row_begin || t0 + T > p.row_end)) {  // ragged head / tail tile: lanes copy their rows\n"
     << "      const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
     << "      const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
-    << "      mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r * 32; if (row >= lo && row < hi) mask |= 1u << r; }\n";
+    << "      mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r; if (row >= lo && row < hi) mask |= 1u << r; }\n";
   for (int k = 0; k < kp.ncols; ++k) {
     const char* ty = ctype(kp.cols[k].width);
-    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r * 32; ((" << ty
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r; ((" << ty
       << "*)(st + " << kp.cols[k].soff << "u))[row] = ((const " << ty << "*)p.col[" << k << "])[t0 + row]; }\n";
   }
   o << "      fence_proxy_async(); __syncwarp();\n    }\n";
@@ -443,13 +518,22 @@ std::string generate(const KPlan& kp) {
     for (const auto& sk2 : g.stage_k) g.use(sk2.first);
     o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
   }
+  // compaction point (Gen::compact): after the first probe that passes at most
+  // half of the rows (build-side key density), aggregation sinks only, R >= 2
+  int cpt = -1;
+  if (sk != 2 && !c2 && kp.R >= 4 && kp.smode != SM_LANE)  // at R = 2 the shuffles cost more than they save (B200)
+    for (int i = 0; i < kp.nops && cpt < 0; ++i)
+      if (kp.ops[i].kind == OP_PROBE && kp.probes[kp.ops[i].idx].pass_est <= 0.5f) cpt = i;
+  if (const char* e = getenv("HQ_JIT_CPT")) cpt = (e[0] == 'o') ? -1 : (sk != 2 ? atoi(e) : -1);
   for (int i = 0; i < kp.nops;) {
+    if (cpt >= 0 && !g.compacted_R && i > cpt) g.compact(i);
     const KOp op = kp.ops[i];
     if (op.kind == OP_PROBE) { i = g.probe_batch(i); continue; }
     if (op.kind == OP_FILTER) g.filter(kp.preds[op.idx], op.idx);
     else g.compute(kp.comps[op.idx]);
     ++i;
   }
+  if (cpt >= 0 && !g.compacted_R) g.compact(kp.nops);
   if (sk != 2) g.early_exit();  // the sinks below only touch live rows
   // ------------------------------------------------------------ sink (tile)
   auto aggval = [&](int a) -> std::string {
@@ -470,35 +554,68 @@ std::string generate(const KPlan& kp) {
       o << "      }\n";
     }
   } else if (sk == 1) {
-    o << "      u64 gk_[R]; bool bad_ = false;\n#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = 0;\n";
+    // local dense / lane-private tables index < 2^32 groups: when no key needs a
+    // domain check the index is computed in 32-bit arithmetic
+    bool all_in = true;
+    std::vector<bool> indom(kp.nkeys);
+    for (int i = 0; i < kp.nkeys; ++i) {
+      auto kr = g.known.find(kp.key_reg[i]);
+      indom[i] = kr != g.known.end() && kr->second.first >= kp.key_min[i] &&
+                 kr->second.second < kp.key_min[i] + kp.key_card[i];
+      all_in = all_in && indom[i];
+    }
+    const bool k32 = all_in && (kp.smode == SM_DENSE || kp.smode == SM_LANE);
+    o << "      u64 gk_[R]; bool bad_ = false;\n";
+    if (k32) o << "      u32 gk32_[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) gk32_[r] = 0u;\n";
+    else o << "#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = 0;\n";
     for (int i = 0; i < kp.nkeys; ++i) {
       const std::string v = g.val(kp.key_reg[i]);
-      auto kr = g.known.find(kp.key_reg[i]);
-      const bool in_domain = kr != g.known.end() && kr->second.first >= kp.key_min[i] &&
-                             kr->second.second < kp.key_min[i] + kp.key_card[i];
       // the shared table may index a narrowed domain (kp.local_keys): only keys
       // whose payload range is known are narrowed, and those need no check
       const int64_t kmin = kp.local_keys ? kp.lkey_min[i] : kp.key_min[i];
       const int64_t kstr = kp.local_keys ? kp.lkey_stride[i] : kp.key_stride[i];
-      const bool ranked = kp.local_keys && (kp.lkey_set[i][0] | kp.lkey_set[i][1] | kp.lkey_set[i][2] | kp.lkey_set[i][3]);
+      const uint64_t* ls = kp.lkey_set[i];
+      const bool ranked = kp.local_keys && (ls[0] | ls[1] | ls[2] | ls[3]);
+      std::string dexpr;  // the key's offset (or rank) in the (narrowed) domain
+      const std::string off32 = "((u32)(long long)" + v + " - " + std::to_string((uint32_t)kmin) + "u)";
       if (ranked) {  // index by the rank of the value among the build side's distinct payloads
-        const std::string rk = "RK_" + std::to_string(i);
-        g.bitmaps << "static constexpr __device__ unsigned char " << rk << "[] = {";
-        int64_t n = 0;
-        for (int64_t d = 0; d < 256; ++d) {
-          const bool on = (kp.lkey_set[i][d >> 6] >> (d & 63)) & 1ull;
-          g.bitmaps << (d ? ", " : "") << (on ? n : 255);
-          n += on;
+        int top = 0;
+        for (int d = 0; d < 256; ++d)
+          if ((ls[d >> 6] >> (d & 63)) & 1ull) top = d + 1;
+        char buf[64];
+        if (top <= 32) {  // rank = popcount of the set below the value
+          snprintf(buf, sizeof buf, "0x%08xu", (unsigned)ls[0]);
+          dexpr = "(u32)__popc(" + std::string(buf) + " & ((1u << (" + off32 + " & 31u)) - 1u))";
+        } else if (top <= 64) {
+          snprintf(buf, sizeof buf, "0x%016llxull", (unsigned long long)ls[0]);
+          dexpr = "(u32)__popcll(" + std::string(buf) + " & ((1ull << (" + off32 + " & 63u)) - 1ull))";
+        } else {
+          const std::string rk = "RK_" + std::to_string(i);
+          g.bitmaps << "static constexpr __device__ unsigned char " << rk << "[] = {";
+          int64_t n = 0;
+          for (int64_t d = 0; d < 256; ++d) {
+            const bool on = (ls[d >> 6] >> (d & 63)) & 1ull;
+            g.bitmaps << (d ? ", " : "") << (on ? n : 255);
+            n += on;
+          }
+          g.bitmaps << "};\n";
+          dexpr = "(((mask >> r) & 1u) ? (u32)" + rk + "[" + off32 + " & 255u] : 0u)";
         }
-        g.bitmaps << "};\n";
-        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = ((mask >> r) & 1u) ? (long long)" << rk
-          << "[(u32)((long long)" << v << " - " << lit(kmin) << ") & 255u] : 0LL;";
-      } else
-      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kmin) << ";";
-      if (!in_domain)  // payload ranges known from the build's count pass need no domain check
+      }
+      if (k32) {
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) gk32_[r] += " << (ranked ? dexpr : off32) << " * "
+          << (uint32_t)kstr << "u;\n";
+        continue;
+      }
+      if (ranked)
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << dexpr << ";";
+      else
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kmin) << ";";
+      if (!indom[i])  // payload ranges known from the build's count pass need no domain check
         o << " if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }";
       o << " gk_[r] += (u64)d_ * " << kstr << "ull; }\n";
     }
+    if (k32) o << "#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = gk32_[r];\n";
     o << "      if (bad_) atomicOr(p.err, F_KEY_DOMAIN);\n";
     if (kp.smode == SM_LANE) {
       std::vector<std::string> av(kp.nacc);
@@ -514,7 +631,9 @@ std::string generate(const KPlan& kp) {
       o << "      i64 va_[NAGGS > 0 ? NAGGS : 1][R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) {";
       for (int a = 0; a < kp.naggs; ++a) o << " va_[" << a << "][r] = " << vv[a] << ";";
       o << " }\n";
-      if (kp.R >= 4) {
+      const char* ce = getenv("HQ_JIT_COMPACT");  // A/B: compaction of R >= 4 row slots
+      const bool wcompact = ce ? ce[0] == '1' : kp.R >= 4;
+      if (wcompact) {
         // warp compaction: the warp's live rows (over all R row slots) move into
         // consecutive lanes (ballot prefix, k-th set bit by popc bisection,
         // shuffles), so table updates run as rounds of 32 rows instead of R slots
@@ -551,7 +670,7 @@ std::string generate(const KPlan& kp) {
           << "        const bool live_ = (mask >> r) & 1u; const u64 key_ = gk_[r];\n"
           << "        i64 v_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n";
       }
-      if (kp.R >= 4 || c2) o << "        const u32 am_ = __ballot_sync(HQ_FULL, live_);\n";
+      if (wcompact || c2) o << "        const u32 am_ = __ballot_sync(HQ_FULL, live_);\n";
       if (c2) {
         o << "        if (live_) group_update(p, sagg, key_, false, 1ull, v_);\n      }\n";
       } else {
@@ -566,7 +685,7 @@ std::string generate(const KPlan& kp) {
           << "          i64 w_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) w_[a] = warp_reduce(AGG_FN[a], mine_ ? v_[a] : agg_identity(AGG_FN[a]));\n"
           << "          if (lane == leader_) group_update(p, sagg, key_, true, (u64)__popc(grp_), w_);\n"
           << "          multi_ &= ~grp_;\n        }\n      }\n";
-        if (kp.R < 4) o << "      }\n";  // else of the sparse path
+        if (!wcompact) o << "      }\n";  // else of the sparse path
       }
     }
   } else {  // materialise: hand the output values to the block scan below
@@ -577,30 +696,35 @@ std::string generate(const KPlan& kp) {
     o << " }\n";
   }
   for (int k = 0; k < g.open; ++k) o << "    }\n";
+  if (g.compacted_R) o << "#undef R\n#define R " << g.compacted_R << "\n";
   o << "    }\n";
   if (sk == 2) {
     // A3 (Fig 25 / P:1069-1072): warp ballots -> block scan over the warps ->
     // one atomicAdd per block and tile -> writes at local + global offset.
     // Every consumer warp takes part in every tile (its mask may be empty).
-    o << "    {\n      u32 b_[R]; int wtot_ = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { b_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); wtot_ += __popc(b_[r]); }\n";
+    // a lane's rows are consecutive: positions in row order are the lane's
+    // exclusive prefix over the warp plus its live rows below r
     if (c2) {
-      o << "      (void)wtot_;\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = atomicAdd(p.counter, 1ull);\n";
+      o << "    {\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = atomicAdd(p.counter, 1ull);\n";
     } else {
-      o << "      if (lane == 0) s_wtot[warp] = wtot_;\n      consumer_bar();\n"
+      o << "    {\n      const int mine_ = __popc(mask); int lin_ = mine_;\n"
+        << "#pragma unroll\n      for (int o_ = 1; o_ < 32; o_ <<= 1) { const int t_ = __shfl_up_sync(HQ_FULL, lin_, o_); if (lane >= o_) lin_ += t_; }\n"
+        << "      const int wtot_ = __shfl_sync(HQ_FULL, lin_, 31);\n"
+        << "      if (lane == 0) s_wtot[warp] = wtot_;\n      consumer_bar();\n"
         << "      if (warp == 0) { const int v_ = lane < NW ? s_wtot[lane] : 0; int incl_ = v_;\n"
         << "#pragma unroll\n        for (int o_ = 1; o_ < 32; o_ <<= 1) { const int t_ = __shfl_up_sync(HQ_FULL, incl_, o_); if (lane >= o_) incl_ += t_; }\n"
         << "        const int total_ = __shfl_sync(HQ_FULL, incl_, 31); u64 g_ = 0;\n"
         << "        if (lane == 0 && total_ > 0) g_ = atomicAdd(p.counter, (u64)total_);\n"
         << "        g_ = __shfl_sync(HQ_FULL, g_, 0); if (lane < NW) s_base[lane] = g_ + (u64)(incl_ - v_); }\n"
         << "      consumer_bar();\n"
-        << "      const u64 base_ = s_base[warp]; const u32 lt_ = lanemask_lt(); u64 run_ = 0;\n"
-        << "#pragma unroll\n      for (int r = 0; r < R; ++r) { if ((mask >> r) & 1u) { const u64 pos_ = base_ + run_ + __popc(b_[r] & lt_);\n";
+        << "      const u64 base_ = s_base[warp] + (u64)(lin_ - mine_);\n"
+        << "#pragma unroll\n      for (int r = 0; r < R; ++r) { if ((mask >> r) & 1u) { const u64 pos_ = base_ + __popc(mask & ((1u << r) - 1u));\n";
     }
     o << "        if ((long long)pos_ < p.capacity) {\n";
     for (int j = 0; j < kp.nout; ++j)
       o << "          ((" << ctype(kp.out_width[j]) << "*)p.out[" << j << "])[pos_] = (" << ctype(kp.out_width[j]) << ")ov" << j << "[r];\n";
     o << "        } else atomicOr(p.err, F_CAPACITY); }\n";
-    if (!c2) o << "        run_ += __popc(b_[r]); }\n";
+    if (!c2) o << "        }\n";
     o << "    }\n";
   }
   if (kp.early_release) o << "    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";

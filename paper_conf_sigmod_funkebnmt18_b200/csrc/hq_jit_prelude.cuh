@@ -62,6 +62,21 @@ __device__ __forceinline__ void mbar_wait(u64* b, u32 parity) {
 __device__ __forceinline__ void mbar_wait_sleep(u64* b, u32 parity) {
   while (!mbar_try_wait(b, parity)) __nanosleep(WAIT_NS);
 }
+// consumer-side wait with a suspend-time hint: the warp is parked by the
+// hardware until the phase completes (or the hint expires) instead of issuing
+// poll/sleep instructions that compete with the working warps
+__device__ __forceinline__ void mbar_wait_suspend(u64* b, u32 parity) {
+  u32 ok;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(ok)
+        : "r"(smem_u32(b)), "r"(parity), "r"(1000000u)
+        : "memory");
+  } while (!ok);
+}
 __device__ __forceinline__ u64 policy_evict_first() {
   u64 pol;
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));

@@ -133,6 +133,12 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.pay_min = op.ht->meta.pay_min;
       pr.pay_max = op.ht->meta.pay_max;
       for (int k = 0; k < 4; ++k) pr.pay_set[k] = op.ht->meta.pay_set[k];
+      {  // uniform foreign keys over the key range: pass fraction = key density (anti: the rest)
+        const double range = (double)op.ht->meta.key_max - (double)op.ht->meta.key_min + 1.0;
+        double est = (op.ht->meta.nkeys >= 0 && range >= 1.0) ? (double)op.ht->meta.nkeys / range : 1.0;
+        est = est > 1.0 ? 1.0 : est;
+        pr.pass_est = (float)(op.mode == HQ_PROBE_ANTI ? 1.0 - est : est);
+      }
       pr.cbytes = (uint32_t)op.ht->cbytes;
       pr.smem_off = 0;
       pr.pf = op.ht->pf_words ? op.ht->prefilter.as<uint32_t>() : nullptr;

@@ -1,0 +1,12 @@
+cd $GRAFT_REPO_ROOT
+timeout 600 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+HQ_JIT_CPT=0 timeout 600 python -m pytest tests/test_gpu_parity.py -m gpu -x -q 2>&1 | tail -2
+for c in auto off; do
+  echo "== CPT=$c"
+  for qs in "ssb_q31 30" "ssb_q41 100" "tpch_q3 30" "ssb_q11 10" "micro_groupby 10"; do
+    set -- $qs
+    if [ $c = auto ]; then timeout 300 python scripts/profile_query.py --query $1 --sf $2 --reps 4 2>&1 | tail -1;
+    else HQ_JIT_CPT=off timeout 300 python scripts/profile_query.py --query $1 --sf $2 --reps 4 2>&1 | tail -1; fi
+  done
+done
+for nwr in "16 4" "31 4"; do set -- $nwr; echo "== NW=$1 R=$2"; for q in ssb_q31 ssb_q41; do HQ_JIT_COMPACT=0 HQ_JIT_NW=$1 HQ_JIT_R=$2 timeout 300 python scripts/profile_query.py --query $q --sf 30 --reps 4 2>&1 | tail -1; done; done

@@ -50,6 +50,6 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "#define SMODE 1" in narrowed and "#define SMEM_CAP 1183u" in narrowed and "gkey_ +=" in narrowed
     # ... and by the rank among the payloads' distinct values (5 of the 21 codes 4..24)
     ranked = srcs["star_ranked_dense"]
-    assert "#define SMEM_CAP 175u" in ranked and "RK_0[" in ranked and "RK_1[" in ranked and "dv_[o_]" in ranked
+    assert "#define SMEM_CAP 175u" in ranked and "__popc(0x00100261u" in ranked and "dv_[o_]" in ranked
     # high-cardinality hash group-by skips the shared table (C2 straight to global)
     assert "#define SMODE 0" in srcs["global_hash_groups"]
