@@ -233,8 +233,10 @@ struct Gen {
     else if (pr.ckind == 3) idx = "(" + D + "[r] >> 1)";
     std::string ld;
     if (ak == AK_SMEM)
-      ld = pr.ckind == 1 ? "((const u32*)(smem + " + std::to_string(pr.smem_off) + "u))[" + idx + "]"
-                         : "(u32)((const unsigned char*)(smem + " + std::to_string(pr.smem_off) + "u))[" + idx + "]";
+      // 32-bit shared-window addresses from a base taken once (a generic
+      // pointer made ptxas re-derive the window from SR_CgaCtaId per probe)
+      ld = pr.ckind == 1 ? "lds_u32(sm0_ + " + std::to_string(pr.smem_off) + "u + (" + idx + ") * 4u)"
+                         : "lds_u8(sm0_ + " + std::to_string(pr.smem_off) + "u + (" + idx + "))";
     else
       ld = pr.ckind == 1 ? "__ldg((const u32*)p.ctab[" + std::to_string(i) + "] + " + idx + ")"
                          : "(u32)__ldg((const unsigned char*)p.ctab[" + std::to_string(i) + "] + " + idx + ")";
@@ -441,6 +443,7 @@ std::string generate(const KPlan& kp) {
     << "  u64* full = (u64*)smem; u64* empty = full + 10;\n"
     << "  u64* s_base = (u64*)(empty + 10); int* s_wtot = (int*)(s_base + 32); i64* s_red = (i64*)(s_wtot + 32);\n"
     << "  char* sagg = smem + OFF_AGG; char* stages = smem + OFF_STAGE;\n"
+    << "  const u32 sm0_ = smem_u32(smem); (void)sm0_;\n"
     << "  (void)s_base; (void)s_wtot; (void)s_red; (void)sagg;\n"
     << "  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n"
     << "  const long long first_tile = p.row_begin / T;\n"

@@ -31,6 +31,17 @@ typedef long long i64;
 #define F_CAPACITY 1
 
 __device__ __forceinline__ u32 smem_u32(const void* p) { return (u32)__cvta_generic_to_shared(p); }
+// loads from read-only shared tables at 32-bit shared-window addresses
+__device__ __forceinline__ u32 lds_u32(u32 a) {
+  u32 v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ u32 lds_u8(u32 a) {
+  u32 v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(a));
+  return v;
+}
 __device__ __forceinline__ void mbar_init(u64* b, u32 count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count) : "memory");
 }

@@ -36,7 +36,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
     star = srcs["star_dense_lrgp"]
-    assert "(const u32*)(smem + " in star            # staged bitmap
+    assert "lds_u32(sm0_ + " in star                 # staged bitmap
     assert "__ldg((const unsigned char*)p.ctab[" in star  # global byte map
     assert "__ldg((const u32*)p.ctab[" in star       # global bitmap
     assert "& 15u" in star                           # staged nibbles
