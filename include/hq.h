@@ -256,8 +256,16 @@ typedef enum { HQ_RES_LRGP = 0, HQ_RES_ATOMIC = 1 } hq_resolution;
  *              compilation); falls back to FUSED_INTERP
  *              only if HQ_JIT=0 is set in the environment;
  * OAAT         operator-at-a-time baseline (Fig 6);
- * FUSED_INTERP the same compound kernel as a precompiled descriptor interpreter. */
-typedef enum { HQ_EXEC_FUSED = 0, HQ_EXEC_OAAT = 1, HQ_EXEC_FUSED_INTERP = 2 } hq_exec;
+ * FUSED_INTERP the same compound kernel as a precompiled descriptor interpreter;
+ * MULTIPASS    multi-pass query compilation (§4, Fig 7-9; Table 4
+ *              A1/B1/C1): a generated count kernel (selections and join probes
+ *              -> one int32 flag per row), a prefix sum over the flags, a
+ *              generated write kernel (projections / aggregation inputs of the
+ *              flagged rows at their prefix-sum positions) and, for AGG sinks,
+ *              library reductions (reduce; radix sort + reduce-by-key).  Same
+ *              results as FUSED (materialised rows in row order); one host
+ *              synchronisation (the qualifying count sizes the outputs). */
+typedef enum { HQ_EXEC_FUSED = 0, HQ_EXEC_OAAT = 1, HQ_EXEC_FUSED_INTERP = 2, HQ_EXEC_MULTIPASS = 3 } hq_exec;
 
 typedef struct {
   const hq_table* fact;

@@ -251,6 +251,13 @@ struct KPlan {
   // generated kernels: copy the tile's columns into registers and release the
   // stage before the operators run (long-latency probes do not hold the ring)
   uint8_t early_release;
+  // multi-pass execution (HQ_EXEC_MULTIPASS, hq_multipass.cu): 1 = count kernel
+  // (relational primitives -> one flag per row), 2 = write kernel (rows whose
+  // flag is set; projections / aggregation inputs written at the prefix-sum
+  // positions); op_skip marks the ops a pass does not execute
+  uint8_t mp_pass;
+  uint8_t op_skip[HQ_MAX_OPS];
+  int16_t mp_flag_reg, mp_pos_reg;  // pass 2: stage registers of the flag and position columns
   int64_t lkey_min[HQ_MAX_KEYS];
   int64_t lkey_stride[HQ_MAX_KEYS];
   // ... and a key whose payload takes few distinct values (SSB Q3.1: 5 ASIA
@@ -300,6 +307,11 @@ struct hq_result : RefObj {
   std::vector<DevBuf> rescols;  // finalized result columns (int64 / f64) ...
   DevBuf respack;                // ... or packed in one buffer (small results)
   std::vector<void*> rescol;     // device pointer of each finalized column
+  // multi-pass execution: per-row flags and prefix-sum positions (int32), the
+  // materialised aggregation inputs (pass 2) and the library-reduction scratch
+  DevBuf mp_flags, mp_pos, mp_keys, mp_vals, mp_scratch;
+  const char* mp_flags_col = nullptr;  // flags / positions indexed by absolute row
+  const char* mp_pos_col = nullptr;
   std::vector<long long> host_rows;  // small results: the finalized rows already on the host
   bool host_ready = false;           // (column-major, nrows per column)
   ~hq_result() override;
@@ -320,7 +332,10 @@ void hq_run_oaat(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
 // shared plan preparation (hq_plan.cu)
 void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
 void hq_build_kplan(hq_ctx* ctx, hq_result* r, hqk::KPlan& kp, int64_t group_cap, int64_t mat_cap,
-                    bool jit = false);
+                    bool jit = false, int mp_pass = 0);
+// multi-pass execution of a plan (hq_multipass.cu): count kernel, prefix sum,
+// write kernel, library reductions (§4, Fig 7-9; A1/B1/C1 of Table 4)
+void hq_run_multipass(hq_ctx* ctx, const hq_plan* plan, hq_result* r, int64_t group_cap = 0);
 // query compilation (hq_jit.cu): NVRTC-specialised fused kernels
 bool hq_jit_enabled();
 void hq_jit_prepare(hq_ctx* ctx, const hqk::KPlan& kp, size_t smem);  // compile (cached) + attributes

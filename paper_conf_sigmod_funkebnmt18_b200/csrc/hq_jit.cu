@@ -321,7 +321,7 @@ struct Gen {
       // (no early exit in front: the warp rarely has no live row here, and the
       // extra branch measured slower)
       std::set<int> defs(first.dst, first.dst + (first.mode == HQ_PROBE_INNER ? first.npay : 0));
-      for (int j = i + 1; j < kp.nops && kp.ops[j].kind == OP_PROBE; ++j) {
+      for (int j = i + 1; j < kp.nops && kp.ops[j].kind == OP_PROBE && !kp.op_skip[j]; ++j) {
         const KProbe& pr = kp.probes[kp.ops[j].idx];
         if (access(pr) == AK_LINEAR || access(pr) == AK_SMEM || defs.count(pr.key_reg)) break;
         b.push_back(j);
@@ -437,6 +437,7 @@ std::string generate(const KPlan& kp) {
   std::ostringstream& o = g.o;
   const bool c2 = kp.resolution == HQ_RES_ATOMIC;
   const int sk = kp.sink == HQ_SINK_MATERIALISE ? 2 : (kp.nkeys == 0 ? 0 : 1);
+  const int mp = kp.mp_pass;  // multi-pass: 1 = count kernel, 2 = write kernel (hq_multipass.cu)
   // ---------------------------------------------------------------- kernel
   o << "extern \"C\" __global__ void __launch_bounds__((NW + 1) * 32, 1) hq_jit_kernel(const __grid_constant__ JParams p) {\n"
     << "  extern __shared__ __align__(128) char smem[];\n"
@@ -500,6 +501,7 @@ std::string generate(const KPlan& kp) {
     << "  for (int j = 0; j < njc; ++j, t0 += tstep) {\n"
     << (prof ? "    { const long long c_ = clock64(); " + cwait + " pw_ += clock64() - c_; if (__activemask() != 0xffffffffu) ++pdv_; }\n" : "    " + cwait + "\n")
     << "    const char* st = stages + (size_t)s * STAGE_STRIDE;\n"
+    << "    const long long tb_ = t0;  // tile start (temporaries t0, t1, ... shadow it below)\n"
     << "    u32 mask = (1u << R) - 1u;\n"
     << "    if ((j == 0 || j == njc - 1) && (t0 < p.row_begin || t0 + T > p.row_end)) {  // ragged head / tail tile: lanes copy their rows\n"
     << "      const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
@@ -521,6 +523,10 @@ std::string generate(const KPlan& kp) {
     for (const auto& sk2 : g.stage_k) g.use(sk2.first);
     o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
   }
+  if (mp == 2) {  // the count kernel's flags select the rows
+    const std::string f = g.val(kp.mp_flag_reg);
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (!" << f << ") mask &= ~(1u << r);\n";
+  }
   // compaction point (Gen::compact): after the first probe that passes at most
   // half of the rows (build-side key density), aggregation sinks only, R >= 2
   int cpt = -1;
@@ -528,8 +534,10 @@ std::string generate(const KPlan& kp) {
     for (int i = 0; i < kp.nops && cpt < 0; ++i)
       if (kp.ops[i].kind == OP_PROBE && kp.probes[kp.ops[i].idx].pass_est <= 0.5f) cpt = i;
   if (const char* e = getenv("HQ_JIT_CPT")) cpt = (e[0] == 'o') ? -1 : (sk != 2 ? atoi(e) : -1);
+  if (mp) cpt = -1;
   for (int i = 0; i < kp.nops;) {
     if (cpt >= 0 && !g.compacted_R && i > cpt) g.compact(i);
+    if (kp.op_skip[i]) { ++i; continue; }  // not executed in this pass
     const KOp op = kp.ops[i];
     if (op.kind == OP_PROBE) { i = g.probe_batch(i); continue; }
     if (op.kind == OP_FILTER) g.filter(kp.preds[op.idx], op.idx);
@@ -537,6 +545,41 @@ std::string generate(const KPlan& kp) {
     ++i;
   }
   if (cpt >= 0 && !g.compacted_R) g.compact(kp.nops);
+  if (mp == 1) {
+    // count kernel (Fig 8): one int32 flag per row of the range, indexed by
+    // absolute row (the flag column's base is offset by the host)
+    o << "      { int* fl_ = (int*)p.out[0];\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long row_ = tb_ + row0 + r;"
+      << " if (row_ >= p.row_begin && row_ < p.row_end) fl_[row_] = (int)((mask >> r) & 1u); } }\n";
+  } else if (mp == 2) {
+    // write kernel (Fig 8): flagged rows write at their prefix-sum position --
+    // the projections (A1) or the aggregation inputs: packed group key, values (B1/C1)
+    const std::string pv = g.val(kp.mp_pos_reg);
+    if (sk == 2) {
+      std::vector<std::string> ov;
+      for (int j = 0; j < kp.nout; ++j) ov.push_back(g.val(kp.out_reg[j]));
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = (u64)(u32)" << pv << ";";
+      for (int j = 0; j < kp.nout; ++j)
+        o << " ((" << ctype(kp.out_width[j]) << "*)p.out[" << j << "])[pos_] = (" << ctype(kp.out_width[j]) << ")" << ov[j] << ";";
+      o << " }\n";
+    } else {
+      o << "      u64 gk_[R]; bool bad_ = false;\n#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = 0;\n";
+      for (int i = 0; i < kp.nkeys; ++i) {
+        const std::string v = g.val(kp.key_reg[i]);
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kp.key_min[i])
+          << "; if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }"
+          << " gk_[r] += (u64)d_ * " << kp.key_stride[i] << "ull; }\n";
+      }
+      o << "      if (bad_) atomicOr(p.err, F_KEY_DOMAIN);\n";
+      std::vector<std::string> vv;
+      for (int a = 0; a < kp.naggs; ++a) vv.push_back(kp.agg_fn[a] == HQ_AGG_COUNT ? std::string() : g.val(kp.agg_reg[a]));
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = (u64)(u32)" << pv << ";";
+      int oc = 0;
+      if (kp.nkeys > 0) o << " ((u64*)p.out[" << oc++ << "])[pos_] = gk_[r];";
+      for (int a = 0; a < kp.naggs; ++a)
+        if (kp.agg_fn[a] != HQ_AGG_COUNT) o << " ((i64*)p.out[" << oc++ << "])[pos_] = (i64)" << vv[a] << ";";
+      o << " }\n";
+    }
+  } else {
   if (sk != 2) g.early_exit();  // the sinks below only touch live rows
   // ------------------------------------------------------------ sink (tile)
   auto aggval = [&](int a) -> std::string {
@@ -698,10 +741,11 @@ std::string generate(const KPlan& kp) {
     for (int j = 0; j < kp.nout; ++j) o << " ov" << j << "[r] = (long long)" << ov[j] << ";";
     o << " }\n";
   }
+  }  // !mp
   for (int k = 0; k < g.open; ++k) o << "    }\n";
   if (g.compacted_R) o << "#undef R\n#define R " << g.compacted_R << "\n";
   o << "    }\n";
-  if (sk == 2) {
+  if (sk == 2 && !mp) {
     // A3 (Fig 25 / P:1069-1072): warp ballots -> block scan over the warps ->
     // one atomicAdd per block and tile -> writes at local + global offset.
     // Every consumer warp takes part in every tile (its mask may be empty).
@@ -734,7 +778,8 @@ std::string generate(const KPlan& kp) {
   else o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
   if (prof) o << "  if (lane == 0) { p.prof[blockIdx.x * 128 + 8 + warp] = pw_; p.prof[blockIdx.x * 128 + 40 + warp] = clock64() - pl0_; } if (pdv_) atomicAdd((unsigned long long*)&p.prof[blockIdx.x * 128 + 72 + warp], (unsigned long long)pdv_);\n";
   // ------------------------------------------------------------- sink (end)
-  if (sk == 0 && !c2) {
+  if (mp) {
+  } else if (sk == 0 && !c2) {
     o << "  { u64 c_ = scount_;\n#pragma unroll\n    for (int o_ = 16; o_ > 0; o_ >>= 1) c_ += __shfl_xor_sync(HQ_FULL, c_, o_);\n";
     for (int a = 0; a < kp.naggs; ++a) o << "    const i64 r" << a << " = warp_reduce(AGG_FN[" << a << "], sacc" << a << ");\n";
     o << "    if (lane == 0) { s_red[warp * 9] = (i64)c_;";

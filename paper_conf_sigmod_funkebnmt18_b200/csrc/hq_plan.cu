@@ -76,7 +76,7 @@ int hq_type_width(int type) {
 }
 
 // Build the device plan; allocates the result's sink buffers on first use.
-void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int64_t mat_cap, bool jit) {
+void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int64_t mat_cap, bool jit, int mp_pass) {
   const hq_plan& P = r->plan;
   const hq_table* F = r->fact;
   std::memset(&kp, 0, sizeof(kp));
@@ -343,13 +343,74 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     HQ_THROW(HQ_ERR_ARG, "plan: bad sink");
   }
 
+  // ---- multi-pass (hq_multipass.cu): which ops a pass executes and which
+  // columns it reads (backward liveness).  Count kernel: selections, probes and
+  // the computes feeding them; write kernel: inner probes and computes whose
+  // results reach the sink, plus the flag and position columns.
+  kp.mp_pass = (uint8_t)mp_pass;
+  kp.mp_flag_reg = kp.mp_pos_reg = -1;
+  int ncols_all = F->ncols;
+  const char* colptr[HQ_MAX_COLS];
+  int colw[HQ_MAX_COLS];
+  for (int c = 0; c < F->ncols; ++c) {
+    colptr[c] = (const char*)F->cols[c].ptr;
+    colw[c] = F->cols[c].width;
+  }
+  if (mp_pass) {
+    if (!jit) HQ_THROW(HQ_ERR_UNSUPPORTED, "multi-pass execution needs generated kernels (HQ_JIT=0 is set)");
+    bool need[NREGS] = {false};
+    if (mp_pass == 2) {
+      if (P.sink == HQ_SINK_MATERIALISE) {
+        for (int j = 0; j < kp.nout; ++j) need[kp.out_reg[j]] = true;
+      } else {
+        for (int i = 0; i < kp.nkeys; ++i) need[kp.key_reg[i]] = true;
+        for (int a = 0; a < kp.naggs; ++a)
+          if (kp.agg_fn[a] != HQ_AGG_COUNT) need[kp.agg_reg[a]] = true;
+      }
+    }
+    for (int o = kp.nops - 1; o >= 0; --o) {
+      const KOp& op = kp.ops[o];
+      bool exec = false;
+      if (op.kind == OP_FILTER) {
+        exec = mp_pass == 1;
+        if (exec) need[kp.preds[op.idx].reg] = true;
+      } else if (op.kind == OP_PROBE) {
+        const KProbe& pr = kp.probes[op.idx];
+        exec = mp_pass == 1;
+        for (int k = 0; mp_pass == 2 && pr.mode == HQ_PROBE_INNER && k < pr.npay; ++k) exec = exec || need[pr.dst[k]];
+        if (exec) need[pr.key_reg] = true;
+      } else {
+        const KCompute& c = kp.comps[op.idx];
+        exec = need[c.dst];
+        for (int k = 0; exec && k < c.n; ++k)
+          if (kp.insns[c.first + k].reg >= 0) need[kp.insns[c.first + k].reg] = true;
+      }
+      kp.op_skip[o] = exec ? 0 : 1;
+    }
+    for (int c = 0; c < F->ncols; ++c) col_used[c] = need[c];
+    if (mp_pass == 2) {
+      if (F->ncols + 2 > HQ_MAX_COLS) HQ_THROW(HQ_ERR_UNSUPPORTED, "multi-pass: no column slots left for flags/positions");
+      kp.mp_flag_reg = (int16_t)F->ncols;
+      kp.mp_pos_reg = (int16_t)(F->ncols + 1);
+      colptr[F->ncols] = r->mp_flags_col;
+      colptr[F->ncols + 1] = r->mp_pos_col;
+      colw[F->ncols] = colw[F->ncols + 1] = 4;
+      col_used[F->ncols] = col_used[F->ncols + 1] = true;
+      ncols_all = F->ncols + 2;
+    }
+    // both passes write plain arrays: no shared pre-aggregation table
+    kp.smode = SM_NONE;
+    kp.local_keys = 0;
+    agg_smem = 0;
+  }
+
   // ---- stage layout: only referenced columns are streamed
   kp.ncols = 0;
   uint32_t rowbytes = 0;
-  for (int c = 0; c < F->ncols; ++c) {
+  for (int c = 0; c < ncols_all; ++c) {
     if (!col_used[c]) continue;
-    if (((uintptr_t)F->cols[c].ptr & 15) != 0) HQ_THROW(HQ_ERR_ARG, "column pointer not 16-byte aligned");
-    rowbytes += (uint32_t)F->cols[c].width;
+    if (((uintptr_t)colptr[c] & 15) != 0) HQ_THROW(HQ_ERR_ARG, "column pointer not 16-byte aligned");
+    rowbytes += (uint32_t)colw[c];
   }
   uint32_t tmp_row = 0;  // generated kernels keep temporaries in registers
   if (!jit)
@@ -441,11 +502,11 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   }
   const uint32_t T = (uint32_t)kp.tile_rows;
   uint32_t soff = 0;
-  for (int c = 0; c < F->ncols; ++c) {
+  for (int c = 0; c < ncols_all; ++c) {
     if (!col_used[c]) continue;
     KCol& kc = kp.cols[kp.ncols++];
-    kc.ptr = (const char*)F->cols[c].ptr;
-    kc.width = (uint32_t)F->cols[c].width;
+    kc.ptr = colptr[c];
+    kc.width = (uint32_t)colw[c];
     kc.soff = soff;
     kp.regs[c] = {soff, (uint8_t)kc.width, 1, {0, 0}};
     soff += T * kc.width;
@@ -498,6 +559,10 @@ void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r) {
     hq_run_oaat(ctx, plan, r);
     return;
   }
+  if (plan->exec == HQ_EXEC_MULTIPASS) {
+    hq_run_multipass(ctx, plan, r);
+    return;
+  }
   if (plan->exec != HQ_EXEC_FUSED && plan->exec != HQ_EXEC_FUSED_INTERP) HQ_THROW(HQ_ERR_ARG, "plan: bad exec mode");
   launch_pipeline(ctx, r, 0, 0);
 }
@@ -516,7 +581,8 @@ void hq_check_result_faults(hq_ctx* ctx, hq_result* r) {
     const bool fixable = (err & (HQF_CAPACITY | HQF_GROUP_FULL)) != 0;
     if (!fixable) break;
     if (attempt >= 3 || r->plan.exec == HQ_EXEC_OAAT) HQ_THROW(HQ_ERR_OVERFLOW, "pipeline: capacity exceeded");
-    if (err & HQF_CAPACITY) launch_pipeline(ctx, r, 0, (int64_t)st.counter);
+    if (r->plan.exec == HQ_EXEC_MULTIPASS) hq_run_multipass(ctx, &r->plan, r, r->ngroups * 4);
+    else if (err & HQF_CAPACITY) launch_pipeline(ctx, r, 0, (int64_t)st.counter);
     else launch_pipeline(ctx, r, r->ngroups * 4, 0);
   }
   r->checked = true;

@@ -31,7 +31,7 @@ I_LOAD, I_ADD, I_SUB, I_RSUB, I_MUL, I_DIV, I_MOD = 1, 2, 3, 4, 5, 6, 7
 AGG_SUM, AGG_COUNT, AGG_MIN, AGG_MAX, AGG_AVG = 1, 2, 3, 4, 5
 SINK_AGG, SINK_MATERIALISE = 1, 2
 RES_LRGP, RES_ATOMIC = 0, 1
-EXEC_FUSED, EXEC_OAAT, EXEC_FUSED_INTERP = 0, 1, 2
+EXEC_FUSED, EXEC_OAAT, EXEC_FUSED_INTERP, EXEC_MULTIPASS = 0, 1, 2, 3
 
 
 def TMP(k: int) -> int:

@@ -24,7 +24,7 @@ def main():
     ap.add_argument("--query", default="ssb_q41")
     ap.add_argument("--sf", type=float, default=10)
     ap.add_argument("--reps", type=int, default=3)
-    ap.add_argument("--exec", default="fused", choices=["fused", "oaat"])
+    ap.add_argument("--exec", default="fused", choices=["fused", "oaat", "multipass"])
     ap.add_argument("--resolution", default="lrgp", choices=["lrgp", "atomic"])
     ap.add_argument("--kw", default="", help="query kwargs k=v,...")
     a = ap.parse_args()
@@ -36,7 +36,7 @@ def main():
     tables = load_tables(ctx, q, a.sf)
     ctx.sync()
     print(f"loaded in {time.time() - t0:.1f}s", flush=True)
-    E = Engine(ctx, tables, exec_mode=hq.EXEC_FUSED if a.exec == "fused" else hq.EXEC_OAAT,
+    E = Engine(ctx, tables, exec_mode={"fused": hq.EXEC_FUSED, "oaat": hq.EXEC_OAAT, "multipass": hq.EXEC_MULTIPASS}[a.exec],
                resolution=hq.RES_LRGP if a.resolution == "lrgp" else hq.RES_ATOMIC)
     ctx.enable_timing(True)
     for i in range(a.reps):

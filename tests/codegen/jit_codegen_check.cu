@@ -111,6 +111,7 @@ struct Shape {
   std::string name;
   hq_plan plan;
   const char* env_r;  // HQ_JIT_R override (nullptr = default)
+  int mp = 0;         // multi-pass kernel: 1 = count, 2 = write
 };
 
 bool compile(const std::string& name, const std::string& src, const char* dump) {
@@ -288,6 +289,23 @@ int main(int argc, char** argv) {
     shapes.push_back({"global_hash_groups_r4", P, "4"});
   }
 
+  // multi-pass count / write kernels (HQ_EXEC_MULTIPASS) of a grouped star
+  // join, a materialising pipeline and a scalar aggregate
+  {
+    std::vector<Shape> mps;
+    for (const Shape& s : shapes) {
+      if (s.name != "star_ranked_dense" && s.name != "materialise_lrgp" && s.name != "scalar_filters") continue;
+      for (int pass : {1, 2}) {
+        Shape m = s;
+        m.name = s.name + "_mp" + std::to_string(pass);
+        m.plan.exec = HQ_EXEC_MULTIPASS;
+        m.mp = pass;
+        mps.push_back(m);
+      }
+    }
+    for (const Shape& m : mps) shapes.push_back(m);
+  }
+
   int ok = 0;
   for (const Shape& s : shapes) {
     if (s.env_r) {  // R = 4 rows per lane needs fewer consumer warps
@@ -302,10 +320,16 @@ int main(int argc, char** argv) {
     r->plan = s.plan;
     r->fact = F;
     r->dstate = DevBuf(c, 32);
+    r->mp_flags_col = (const char*)(uintptr_t)0x7d0000000000ull;
+    r->mp_pos_col = (const char*)(uintptr_t)0x7d8000000000ull;
     std::string src;
     try {
       KPlan kp;
-      hq_build_kplan(c, r, kp, 0, 0, true);
+      hq_build_kplan(c, r, kp, 0, s.mp ? 1000 : 0, true, s.mp);
+      if (s.mp == 1) {
+        kp.nout = 1;
+        kp.out_ptr[0] = (void*)r->mp_flags_col;
+      }
       src = hq_jit_source(kp);
     } catch (const HqError& e) {
       fprintf(stderr, "FAIL %s: plan: %s\n", s.name.c_str(), e.msg.c_str());

@@ -32,7 +32,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     env = {k: v for k, v in os.environ.items() if not k.startswith("HQ_")}
     p = subprocess.run([checker, str(tmp_path)], capture_output=True, text=True, env=env, timeout=600)
     assert p.returncode == 0, p.stdout + p.stderr
-    assert p.stdout.startswith("OK 12 of 12"), p.stdout
+    assert p.stdout.startswith("OK 18 of 18"), p.stdout
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
     star = srcs["star_dense_lrgp"]
@@ -51,5 +51,12 @@ def test_generated_kernels_compile(checker, tmp_path):
     # ... and by the rank among the payloads' distinct values (5 of the 21 codes 4..24)
     ranked = srcs["star_ranked_dense"]
     assert "#define SMEM_CAP 175u" in ranked and "__popc(0x00100261u" in ranked and "dv_[o_]" in ranked
+    # multi-pass (A1/B1/C1): the count kernel writes flags and skips the sink;
+    # the write kernel reads flags + positions, skips filters / semi probes
+    c1 = srcs["star_ranked_dense_mp1"]
+    assert "fl_[row_] = " in c1 and "group_update(" not in c1.split("extern \"C\"")[1]
+    w2 = srcs["materialise_lrgp_mp2"]
+    assert "pos_ = (u64)(u32)" in w2 and "atomicAdd(p.counter" not in w2 and "(int)c4" not in w2
+    assert "((u64*)p.out[0])[pos_] = gk_[r];" in srcs["star_ranked_dense_mp2"]
     # high-cardinality hash group-by skips the shared table (C2 straight to global)
     assert "#define SMODE 0" in srcs["global_hash_groups"]

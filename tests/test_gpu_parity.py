@@ -132,6 +132,48 @@ def test_operator_at_a_time_parity(ctx, ssb, tpch, qname):
     assert_same(qname, g, oracle_run(qname, host))
 
 
+@pytest.mark.parametrize("qname", ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q12", "ssb_q31", "ssb_q41", "tpch_q3"])
+def test_multipass_parity(ctx, ssb, tpch, qname):
+    """Multi-pass query compilation (f1: count kernel -> prefix sum -> write kernel
+    -> library reduce / sort + reduce-by-key; Table 4 A1/B1/C1) == oracle."""
+    host = host_for(qname, ssb, tpch)
+    kw = {"limit": 0} if qname == "tpch_q3" else {}
+    g = gpu_run(ctx, qname, host, exec_mode=hq.EXEC_MULTIPASS, **kw)
+    o = oracle_run(qname, host)
+    assert_same(qname, g, o)
+    assert g.qualifying == o.qualifying
+
+
+def test_multipass_materialise_in_row_order(ctx, ssb):
+    """A1 writes at prefix-sum positions: the output holds the selected
+    rows in input order (no permutation, unlike the atomics of A2/A3)."""
+    g = gpu_run(ctx, "ssb_q31_mat", ssb, exec_mode=hq.EXEC_MULTIPASS)
+    o = oracle_run("ssb_q31_mat", ssb)
+    assert g.qualifying == o.nrows
+    assert sorted(g.rows(["c_nation", "s_nation", "d_year", "lo_revenue"])) == o.rows()
+    n = 300_000
+    rowid = np.arange(n, dtype=np.int32)
+    flag = (np.random.default_rng(5).random(n) < 0.3).astype(np.int32)
+    t = ctx.load_columns({"rowid": rowid, "flag": flag})
+    from paper_conf_sigmod_funkebnmt18_b200.engine import PlanBuilder
+    pb = PlanBuilder(t)
+    pb.filter("flag", "=", 1).materialise([("rowid", "i32")])
+    pb.plan.exec = hq.EXEC_MULTIPASS
+    res = ctx.run(pb.plan, keep=pb.keep)
+    np.testing.assert_array_equal(res.fetch()[0], rowid[flag == 1])
+
+
+@pytest.mark.parametrize("qname", ["ssb_q41", "tpch_q1"])
+def test_multipass_unaligned_range(ctx, ssb, tpch, qname):
+    """Flag/position columns of a range starting at an unaligned row (TMA alignment)."""
+    host = host_for(qname, ssb, tpch)
+    n = len(next(iter(host[QUERIES[qname].fact].values())))
+    rng = (777, n - 5)
+    a = gpu_run(ctx, qname, host, fact_range=rng, exec_mode=hq.EXEC_MULTIPASS)
+    b = gpu_run(ctx, qname, host, fact_range=rng)
+    assert a.rows() == b.rows() and a.qualifying == b.qualifying
+
+
 def test_operator_at_a_time_materialise(ctx, ssb):
     g = gpu_run(ctx, "ssb_q31_mat", ssb, exec_mode=hq.EXEC_OAAT)
     o = oracle_run("ssb_q31_mat", ssb)
