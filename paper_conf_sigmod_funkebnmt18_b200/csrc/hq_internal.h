@@ -245,6 +245,7 @@ struct KPlan {
   uint64_t gmask;            // hash capacity - 1
   int32_t glog2;
   uint32_t smem_cap;         // smem dense groups or smem hash slots
+  uint32_t scopies;          // generated kernels, SM_DENSE: table replicas (warp w updates copy w % scopies)
   // generated kernels: the shared dense table may index a narrowed key domain
   // (group keys that are probe payloads span only their build-side value range)
   uint8_t local_keys;

@@ -459,7 +459,7 @@ std::string generate(const KPlan& kp) {
     o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * NACC * NW * 32; i += NW * 32) {"
       << " const int a_ = (int)((i / (NW * 32)) % NACC); t_[i] = a_ == 0 ? 0 : agg_identity(ACC_FN[a_]); } }\n";
   } else if (sk == 1 && kp.smode == SM_DENSE) {
-    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * VWORDS; i += NW * 32) {"
+    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * VWORDS * SCOPIES; i += NW * 32) {"
       << " const int c_ = (int)(i % VWORDS); t_[i] = c_ == 0 ? 0 : agg_identity(AGG_FN[c_ - 1]); } }\n";
   } else if (sk == 1 && kp.smode == SM_HASH) {
     o << "  if (warp < NW) { u64* k_ = (u64*)sagg; i64* e_ = (i64*)sagg + SMEM_CAP;\n"
@@ -701,7 +701,7 @@ std::string generate(const KPlan& kp) {
         // split and run the rest of the kernel at half speed.  Otherwise rows
         // of equal keys are combined in registers first (match_any + reduce).
         o << "      u32 act_[R]; int nact_ = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { act_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); nact_ += __popc(act_[r]); }\n"
-          << "      if (nact_ <= 4 * R) {\n"
+          << "      if (SCOPIES > 1 || nact_ <= 4 * R) {  // replicated tables: every live lane updates directly\n"
           << "#pragma unroll\n        for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) {\n"
           << "          i64 v_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n"
           << "          group_update(p, sagg, gk_[r], true, 1ull, v_); }\n"
@@ -803,9 +803,13 @@ std::string generate(const KPlan& kp) {
       o << "      vals_[" << a << "] = " << (kp.acc_of[a] ? "acc_[" + std::to_string(kp.acc_of[a]) + "]" : std::string("(i64)cnt_")) << ";\n";
     o << "      group_update(p, sagg, g, false, cnt_, vals_);\n    } }\n";
   } else if (sk == 1 && kp.smode == SM_DENSE) {
+    // the group's entries in every replica are combined first
     o << "  consumer_bar();\n  { const i64* t_ = (const i64*)sagg;\n"
-      << "    for (u32 g = threadIdx.x; g < SMEM_CAP; g += NW * 32) { const i64* e_ = t_ + (u64)g * VWORDS;\n"
-      << "      if (e_[0] != 0) { i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) vals_[a] = AGG_FN[a] == F_COUNT ? e_[0] : e_[1 + a];\n"
+      << "    for (u32 g = threadIdx.x; g < SMEM_CAP; g += NW * 32) { i64 cnt_ = 0; i64 vals_[NAGGS > 0 ? NAGGS : 1];\n"
+      << "#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = agg_identity(AGG_FN[a]);\n"
+      << "      for (u32 c_ = 0; c_ < SCOPIES; ++c_) { const i64* e_ = t_ + ((u64)c_ * SMEM_CAP + g) * VWORDS; cnt_ += e_[0];\n"
+      << "#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) if (AGG_FN[a] != F_COUNT) vals_[a] = agg_combine(AGG_FN[a], vals_[a], e_[1 + a]); }\n"
+      << "      if (cnt_ != 0) {\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) if (AGG_FN[a] == F_COUNT) vals_[a] = cnt_;\n"
       << "        u64 gkey_ = g;\n";
     if (kp.local_keys) {  // narrowed local index -> declared global key
       o << "        { u64 rem_ = g; gkey_ = 0;";
@@ -824,7 +828,7 @@ std::string generate(const KPlan& kp) {
       }
       o << " }\n";
     }
-    o << "        group_update(p, sagg, gkey_, false, (u64)e_[0], vals_); } } }\n";
+    o << "        group_update(p, sagg, gkey_, false, (u64)cnt_, vals_); } } }\n";
   } else if (sk == 1 && kp.smode == SM_HASH) {
     o << "  consumer_bar();\n  { const u64* k_ = (const u64*)sagg; const i64* t_ = (const i64*)sagg + SMEM_CAP;\n"
       << "    for (u32 h = threadIdx.x; h < SMEM_CAP; h += NW * 32) if (k_[h] != HQ_EMPTY_KEY) { const i64* e_ = t_ + (u64)h * VWORDS;\n"
@@ -843,7 +847,7 @@ std::string generate(const KPlan& kp) {
     << "u\n#define OFF_AGG " << kp.off_agg << "u\n#define OFF_STAGE " << kp.off_stage << "u\n"
     << "#define NAGGS " << kp.naggs << "\n#define VWORDS " << kp.vwords << "\n#define GMODE " << (int)kp.gmode
     << "\n#define SMODE " << (kp.smode == SM_LANE ? 0 : (int)kp.smode) << "\n#define SMEM_CAP " << kp.smem_cap
-    << "u\n#define SLOG2 " << kp.slog2 << "\n#define NACC " << (kp.nacc > 0 ? kp.nacc : 1) << "\n"
+    << "u\n#define SCOPIES " << (kp.scopies ? kp.scopies : 1) << "u\n#define SLOG2 " << kp.slog2 << "\n#define NACC " << (kp.nacc > 0 ? kp.nacc : 1) << "\n"
     << "static constexpr __device__ int AGG_FN[" << (kp.naggs > 0 ? kp.naggs : 1) << "] = " << fn_list(kp.agg_fn, kp.naggs)
     << ";\n"
     << "static constexpr __device__ int ACC_FN[" << (kp.nacc > 0 ? kp.nacc : 1) << "] = " << fn_list(kp.acc_fn, kp.nacc) << ";\n"
@@ -919,6 +923,9 @@ std::string plan_key(const KPlan& kp) {
   KPlan k = kp;
   auto nz = [](const void* p) { return (const char*)(p ? 1 : 0); };
   k.row_begin = k.row_end = 0;
+  k.capacity = 0;  // runtime parameters of the launch, not of the source
+  k.gmask = 0;
+  k.glog2 = 0;
   for (auto& c : k.cols) c.ptr = nz(c.ptr);
   for (auto& pr : k.probes) {
     pr.slots = (const uint32_t*)nz(pr.slots);

@@ -8,7 +8,7 @@
 // fences), atomics on group-table entries, warp reductions, and the
 // shared/global group-table lookups.  It expects these generated constants:
 //   NW, R, T, S, STAGE_STRIDE, OFF_TMP, OFF_AGG, OFF_STAGE, STAGE_BYTES,
-//   NAGGS, AGG_FN[], VWORDS, GMODE, SMODE, SMEM_CAP, SLOG2, NACC, ACC_FN[].
+//   NAGGS, AGG_FN[], VWORDS, GMODE, SMODE, SMEM_CAP, SCOPIES, SLOG2, NACC, ACC_FN[].
 typedef unsigned int u32;
 typedef unsigned long long u64;
 typedef long long i64;
@@ -174,7 +174,7 @@ __device__ __forceinline__ i64* global_locate(const JParams& p, u64 key) {
 }
 // shared pre-aggregation table entry (dense or hash), 0 when the hash is full
 __device__ __forceinline__ u32 local_locate(char* sagg, u64 key) {
-  if (SMODE == 1) return smem_u32((i64*)sagg + key * VWORDS);
+  if (SMODE == 1) return smem_u32((i64*)sagg + ((u64)((threadIdx.x >> 5) % SCOPIES) * SMEM_CAP + key) * VWORDS);
   if (SMODE == 2) {
     u64* keys = (u64*)sagg;
     i64* ent = (i64*)sagg + SMEM_CAP;

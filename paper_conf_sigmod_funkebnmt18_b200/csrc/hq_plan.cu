@@ -309,9 +309,10 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         // far more groups than the shared table holds (TPC-H Q3: ~10^5-10^6
         // orderkeys): it would fill up and every later row would scan it before
         // going to global memory -- update the global table directly (C2)
-        const int64_t expect = group_cap > 0 ? group_cap : P.group_capacity;
+        // (a dense domain larger than the table: as many groups as the domain)
+        const int64_t expect = kp.gmode == GM_DENSE ? ngroups : (group_cap > 0 ? group_cap : P.group_capacity);
         const char* nl = getenv("HQ_JIT_NOLOCAL");
-        if (jit && kp.gmode == GM_HASH && expect > 4 * (int64_t)cap && !(nl && nl[0] == '0')) {
+        if (jit && expect > (kp.gmode == GM_DENSE ? 1 : 4) * (int64_t)cap && !(nl && nl[0] == '0')) {
           kp.smode = SM_NONE;
         } else {
         kp.smode = SM_HASH;
@@ -341,6 +342,23 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     kp.capacity = r->capacity;
   } else {
     HQ_THROW(HQ_ERR_ARG, "plan: bad sink");
+  }
+
+  // Generated kernels: replicas of a small dense shared table, so that the 31
+  // consumer warps do not serialise on the same few entries (Exp 2 with 32-512
+  // groups: one table measured 6-9x slower than the tiny lane-private domains)
+  kp.scopies = 1;
+  if (jit && kp.smode == SM_DENSE && !mp_pass) {
+    // every row updates a probe-free pipeline's table; behind selective probes
+    // (star joins: 1-4 % of the rows) contention is low and the shared memory
+    // is worth more to the staged probe tables and the TMA ring
+    const uint64_t one = (uint64_t)kp.smem_cap * kp.vwords * 8;
+    const uint64_t budget = nprobe == 0 ? (uint64_t)SMEM_AGG_BYTES : 4096;
+    uint32_t c = 1;
+    while (c < 31 && one * (c + 1) <= budget) ++c;
+    if (const char* e = getenv("HQ_JIT_SCOPIES")) c = std::max(1, std::min(31, atoi(e)));
+    kp.scopies = c;
+    agg_smem = (uint32_t)(one * c);
   }
 
   // ---- multi-pass (hq_multipass.cu): which ops a pass executes and which

@@ -1,6 +1,8 @@
 #!/usr/bin/env python
-"""DRAM bytes of the fused plan vs the operator-at-a-time plan of the same
-query (the BASELINE.json metric's second half).
+"""DRAM bytes of the fused plan vs the multi-pass and the operator-at-a-time
+plans of the same query (the BASELINE.json metric's second half; SURVEY.md
+§8(d.3); the paper's three execution models, e.g. 8.4 -> 4.4 -> 1.8 GB for SSB
+Q3.1).
 
 Runs every query once per mode under
   ncu --cache-control all --clock-control none --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum
@@ -19,10 +21,11 @@ import subprocess
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-QUERIES = ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q12", "ssb_q13", "ssb_q31", "ssb_q41", "tpch_q3"]
+QUERIES = ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q12", "ssb_q13", "ssb_q31", "ssb_q31_mat", "ssb_q41", "tpch_q3"]
 SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-9, "us": 1e-6, "ms": 1e-3, "s": 1,
          "nsecond": 1e-9, "usecond": 1e-6, "msecond": 1e-3}
-PIPELINE = ("hq_jit_kernel", "hq_fused_pipeline_kernel", "hq_oaat", "cub::", "DeviceScan")
+PIPELINE = ("hq_jit_kernel", "hq_fused_pipeline_kernel", "hq_oaat", "cub::", "DeviceScan", "mp_")
+MODES = ("fused", "multipass", "oaat")
 
 
 def run(q, sf, mode):
@@ -55,30 +58,34 @@ def main():
     out = {}
     for q in a.queries.split(","):
         out[q] = {}
-        for mode in ("fused", "oaat"):
+        for mode in MODES:
             tot, kernels = run(q, a.sf, mode)
             out[q][mode] = {part: {"dram_bytes": d.get("dram__bytes_read.sum", 0) + d.get("dram__bytes_write.sum", 0),
                                    "time_s": d.get("gpu__time_duration.sum", 0)} for part, d in tot.items()}
             out[q][mode]["kernels"] = kernels
-        print(q, json.dumps({m: {p: out[q][m][p] for p in ("pipeline", "other")} for m in ("fused", "oaat")}), flush=True)
+        print(q, json.dumps({m: {p: out[q][m][p] for p in ("pipeline", "other")} for m in MODES}), flush=True)
     d = os.path.join(ROOT, "gpurun_out")  # copied to profiles/<round>/ after the run
     os.makedirs(d, exist_ok=True)
     with open(os.path.join(d, f"bytes_ratio_sf{a.sf:g}.json"), "w") as f:
         json.dump({"sf": a.sf, "cache_control": "all", "queries": out}, f, indent=1)
     lines = [f"DRAM bytes (ncu dram__bytes_read.sum + dram__bytes_write.sum, --cache-control all) summed over all kernels "
              f"of one query execution at SF {a.sf:g}; 'pipeline' = the fact-table pipeline kernels (fused: one generated "
-             "kernel; op-at-a-time: filter/probe/compute/scan/compact/gather/agg kernels), 'all' adds hash builds and finalize.",
-             "", "| query | fused pipeline GB | OAAT pipeline GB | bytes ratio (pipeline) | fused all GB | OAAT all GB | "
-             "bytes ratio (all) | fused pipeline ms | OAAT pipeline ms | kernel-time ratio |",
-             "|---|---|---|---|---|---|---|---|---|---|"]
+             "kernel; multi-pass: generated count + write kernels, CUB scan / reduce / sort, reduce-by-key scatter; "
+             "op-at-a-time: filter/probe/compute/scan/compact/gather/agg kernels), 'all' adds hash builds and finalize. "
+             "Times are ncu kernel durations (cold caches, serialised), summed.",
+             "", "| query | fused GB | multi-pass GB | OAAT GB | MP/fused bytes | OAAT/fused bytes | OAAT/fused bytes (all) "
+             "| fused ms | multi-pass ms | OAAT ms | MP/fused time | OAAT/fused time |",
+             "|---|---|---|---|---|---|---|---|---|---|---|---|"]
     for q, m in out.items():
-        fp, op = m["fused"]["pipeline"], m["oaat"]["pipeline"]
+        fp, mp, op = m["fused"]["pipeline"], m["multipass"]["pipeline"], m["oaat"]["pipeline"]
         fa = fp["dram_bytes"] + m["fused"]["other"]["dram_bytes"]
         oa = op["dram_bytes"] + m["oaat"]["other"]["dram_bytes"]
-        lines.append(f"| {q} | {fp['dram_bytes'] / 1e9:.3f} | {op['dram_bytes'] / 1e9:.3f} | "
-                     f"{op['dram_bytes'] / max(fp['dram_bytes'], 1):.2f}x | {fa / 1e9:.3f} | {oa / 1e9:.3f} | "
-                     f"{oa / max(fa, 1):.2f}x | {fp['time_s'] * 1e3:.3f} | {op['time_s'] * 1e3:.3f} | "
-                     f"{op['time_s'] / max(fp['time_s'], 1e-12):.2f}x |")
+        fb = max(fp["dram_bytes"], 1)
+        ft = max(fp["time_s"], 1e-12)
+        lines.append(f"| {q} | {fp['dram_bytes'] / 1e9:.3f} | {mp['dram_bytes'] / 1e9:.3f} | {op['dram_bytes'] / 1e9:.3f} | "
+                     f"{mp['dram_bytes'] / fb:.2f}x | {op['dram_bytes'] / fb:.2f}x | {oa / max(fa, 1):.2f}x | "
+                     f"{fp['time_s'] * 1e3:.3f} | {mp['time_s'] * 1e3:.3f} | {op['time_s'] * 1e3:.3f} | "
+                     f"{mp['time_s'] / ft:.2f}x | {op['time_s'] / ft:.2f}x |")
     with open(os.path.join(d, f"bytes_ratio_sf{a.sf:g}.md"), "w") as f:
         f.write("\n".join(lines) + "\n")
     print("\n".join(lines))

@@ -45,7 +45,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "p.pf[" in srcs["materialise_lrgp"]                     # linear prefilter
     assert "match_any" in srcs["global_hash_groups"] and "pre_[R]" in srcs["global_hash_groups_r4"]
     # group keys narrowed to the build-side payload ranges: dense shared table + key remap at the merge
-    assert "#define SMODE 2" in srcs["star_smem_hash"]
+    assert "#define SMODE 0" in srcs["star_smem_hash"]  # dense domain larger than any shared table: global (C2 + warp merging)
     narrowed = srcs["star_narrowed_dense"]
     assert "#define SMODE 1" in narrowed and "#define SMEM_CAP 1183u" in narrowed and "gkey_ +=" in narrowed
     # ... and by the rank among the payloads' distinct values (5 of the 21 codes 4..24)
