@@ -159,9 +159,10 @@ def cpu_baseline(qname, host, n_fact, budget_s=30.0):
                       f"{cores} threads, {dt:.2f} s"}
 
 
-def oaat_timing(qname, host, local, fused_ms, steps=2):
-    """The same query executed operator-at-a-time (Fig 6 baseline, HQ_EXEC_OAAT):
-    device time per step with CUDA events, vs the fused step."""
+def exec_timing(qname, host, local, fused_ms, mode="oaat", steps=2):
+    """The same query executed operator-at-a-time (Fig 6 baseline, HQ_EXEC_OAAT)
+    or by multi-pass query compilation (Fig 7-9, HQ_EXEC_MULTIPASS): device time
+    per step with CUDA events, vs the fused step."""
     import torch
     from paper_conf_sigmod_funkebnmt18_b200 import hq
     from paper_conf_sigmod_funkebnmt18_b200.engine import Engine
@@ -171,7 +172,8 @@ def oaat_timing(qname, host, local, fused_ms, steps=2):
     ctx = hq.Context(local)
     dtab = {t: {c: torch.from_numpy(np.asarray(a)).to(dev) for c, a in cols.items()} for t, cols in host.items()}
     tables = {t: ctx.load_columns(cols) for t, cols in dtab.items()}
-    E = Engine(ctx, tables, exec_mode=hq.EXEC_OAAT)
+    em = {"oaat": hq.EXEC_OAAT, "multipass": hq.EXEC_MULTIPASS}[mode]
+    E = Engine(ctx, tables, exec_mode=em)
     q.execute(E)
     stream = torch.cuda.current_stream(dev)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -185,7 +187,8 @@ def oaat_timing(qname, host, local, fused_ms, steps=2):
     del tables, dtab, E
     ctx.close()
     torch.cuda.empty_cache()
-    return {"ms_per_step": ms, "fused_speedup": ms / fused_ms, "steps": steps, "exec": "HQ_EXEC_OAAT"}
+    return {"ms_per_step": ms, "fused_speedup": ms / fused_ms, "steps": steps,
+            "exec": {"oaat": "HQ_EXEC_OAAT", "multipass": "HQ_EXEC_MULTIPASS"}[mode]}
 
 
 # --------------------------------------------------------- device measurement
@@ -374,7 +377,8 @@ def run_hq(args):
         line["roofline"]["kernel_share_of_step"] = r["kernel_ms"] / r["ms"]
         if world == 1:
             line["cpu_baseline"] = cpu_baseline(args.query, r["host"], r["rows"])
-            line["oaat"] = oaat_timing(args.query, r["host"], local, r["ms"])
+            line["oaat"] = exec_timing(args.query, r["host"], local, r["ms"], "oaat")
+            line["multipass"] = exec_timing(args.query, r["host"], local, r["ms"], "multipass")
         bp = os.path.join(ROOT, "profiles", "r01", "bytes_ratio_sf10.json")
         if os.path.exists(bp):
             br = json.load(open(bp))["queries"].get(args.query)
@@ -382,6 +386,9 @@ def run_hq(args):
                 f, o = br["fused"]["pipeline"]["dram_bytes"], br["oaat"]["pipeline"]["dram_bytes"]
                 line["dram_bytes_fused_vs_oaat"] = {"ratio": o / f, "fused_bytes": f, "oaat_bytes": o, "sf": 10,
                                                     "source": "profiles/r01/bytes_ratio_sf10.json (ncu, --cache-control all)"}
+                if "multipass" in br:
+                    m = br["multipass"]["pipeline"]["dram_bytes"]
+                    line["dram_bytes_fused_vs_oaat"].update({"multipass_bytes": m, "multipass_ratio": m / f})
     del r
     if world == 1 and not args.no_extra and args.query == DEFAULT_QUERY:
         per = []
