@@ -44,6 +44,40 @@ def code(dictionary: Sequence[str], s: str) -> int:
     return list(dictionary).index(s)
 
 
+# SSB strings with generated codes (hqgen.cpp): city = nation * 10 + digit, the
+# city name being the nation's first 9 characters (space padded) + the digit;
+# p_category 'MFGR#mc' = (m-1)*5 + (c-1); p_brand1 'MFGR#mcbb' = category*40 + bb-1.
+# City and category code orders equal the string orders; brand codes follow
+# (category, brand number) -- the string order differs only where a one-digit
+# and a two-digit brand number of one category meet ('MFGR#222' < 'MFGR#2221'),
+# which no SSB predicate here compares (Q2.2's BETWEEN spans brands 21..28).
+def city_name(c: int) -> str:
+    return NATIONS[c // 10][:9].ljust(9) + str(c % 10)
+
+
+def city_code(s: str) -> int:
+    for n, name in enumerate(NATIONS):
+        if name[:9].ljust(9) == s[:9]:
+            return n * 10 + int(s[9])
+    raise KeyError(s)
+
+
+def category_name(c: int) -> str:
+    return f"MFGR#{c // 5 + 1}{c % 5 + 1}"
+
+
+def category_code(s: str) -> int:
+    return (int(s[5]) - 1) * 5 + int(s[6]) - 1
+
+
+def brand_name(b: int) -> str:
+    return f"{category_name(b // 40)}{b % 40 + 1}"
+
+
+def brand_code(s: str) -> int:
+    return category_code(s[:7]) * 40 + int(s[7:]) - 1
+
+
 # ---- table schemas (mirror hqgen.h) ---------------------------------------
 SSB_LINEORDER, SSB_DATE, SSB_CUSTOMER, SSB_SUPPLIER, SSB_PART = 1, 2, 3, 4, 5
 TPCH_LINEITEM, TPCH_ORDERS, TPCH_CUSTOMER = 11, 12, 13

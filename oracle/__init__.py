@@ -53,11 +53,11 @@ class _Date(ctypes.Structure):
 
 
 class _SsbDim(ctypes.Structure):
-    _fields_ = [("n", ctypes.c_int64), ("key", P_I32), ("nation", P_I8), ("region", P_I8)]
+    _fields_ = [("n", ctypes.c_int64), ("key", P_I32), ("nation", P_I8), ("region", P_I8), ("city", P_I32)]
 
 
 class _Part(ctypes.Structure):
-    _fields_ = [("n", ctypes.c_int64), ("partkey", P_I32), ("mfgr", P_I8)]
+    _fields_ = [("n", ctypes.c_int64), ("partkey", P_I32), ("mfgr", P_I8), ("category", P_I8), ("brand1", P_I32)]
 
 
 class _Lineitem(ctypes.Structure):
@@ -118,6 +118,10 @@ def lib():
             "orc_ssb_q31_mat": [P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
             "orc_ssb_q41": [P(_Lineorder), P(_Date), P(_SsbDim), P(_SsbDim), P(_Part), ctypes.c_int, ctypes.c_int],
             "orc_tpch_q3": [P(_TCustomer), P(_Orders), P(_Lineitem), ctypes.c_int, ctypes.c_int],
+            "orc_ssb_q2": [ctypes.c_int, P(_Lineorder), P(_Date), P(_Part), P(_SsbDim), ctypes.c_int, ctypes.c_int],
+            "orc_ssb_q3": [ctypes.c_int, P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
+            "orc_ssb_q4": [ctypes.c_int, P(_Lineorder), P(_Date), P(_SsbDim), P(_SsbDim), P(_Part), ctypes.c_int,
+                           ctypes.c_int],
             "orc_micro_select": [P(_Lineorder), ctypes.c_int32, ctypes.c_int],
             "orc_micro_sum": [P(_Lineorder), ctypes.c_int32, ctypes.c_int],
             "orc_micro_groupby": [P(_Lineorder), ctypes.c_int32, ctypes.c_int],
@@ -167,6 +171,7 @@ def _dim(t, prefix, keep):
     s.key = _ptr(t[prefix + ("custkey" if prefix == "c_" else "suppkey")], P_I32, keep)
     s.nation = _ptr(t.get(prefix + "nation"), P_I8, keep)
     s.region = _ptr(t.get(prefix + "region"), P_I8, keep)
+    s.city = _ptr(t.get(prefix + "city"), P_I32, keep)
     return s
 
 
@@ -175,6 +180,8 @@ def _part(t, keep):
     s.n = _n(t)
     s.partkey = _ptr(t["p_partkey"], P_I32, keep)
     s.mfgr = _ptr(t.get("p_mfgr"), P_I8, keep)
+    s.category = _ptr(t.get("p_category"), P_I8, keep)
+    s.brand1 = _ptr(t.get("p_brand1"), P_I32, keep)
     return s
 
 
@@ -271,6 +278,35 @@ def ssb_q41(lineorder, date, customer, supplier, part, brute=False, nthreads=1) 
                                  ctypes.byref(_dim(supplier, "s_", keep)),
                                  ctypes.byref(_part(part, keep)), int(brute), nthreads],
                  ["d_year", "c_nation", "profit", "count"])
+
+
+def ssb_q2(variant, lineorder, date, part, supplier, brute=False, nthreads=1) -> OracleResult:
+    """SSB Q2.1-Q2.3 -> [d_year, p_brand1, revenue, count] ORDER BY d_year, p_brand1."""
+    keep = []
+    return _call("orc_ssb_q2", [variant, ctypes.byref(_lineorder(lineorder, keep)), ctypes.byref(_date(date, keep)),
+                                ctypes.byref(_part(part, keep)), ctypes.byref(_dim(supplier, "s_", keep)),
+                                int(brute), nthreads],
+                 ["d_year", "p_brand1", "revenue", "count"])
+
+
+def ssb_q3(variant, lineorder, customer, supplier, date, brute=False, nthreads=1) -> OracleResult:
+    """SSB Q3.2-Q3.4 -> [c_city, s_city, d_year, revenue, count] ORDER BY d_year, revenue desc."""
+    keep = []
+    return _call("orc_ssb_q3", [variant, ctypes.byref(_lineorder(lineorder, keep)),
+                                ctypes.byref(_dim(customer, "c_", keep)), ctypes.byref(_dim(supplier, "s_", keep)),
+                                ctypes.byref(_date(date, keep)), int(brute), nthreads],
+                 ["c_city", "s_city", "d_year", "revenue", "count"])
+
+
+def ssb_q4(variant, lineorder, date, customer, supplier, part, brute=False, nthreads=1) -> OracleResult:
+    """SSB Q4.2 -> [d_year, s_nation, p_category, profit, count]; Q4.3 -> [d_year, s_city,
+    p_brand1, profit, count]; ORDER BY the three keys."""
+    keep = []
+    k1, k2 = ("s_nation", "p_category") if variant == 2 else ("s_city", "p_brand1")
+    return _call("orc_ssb_q4", [variant, ctypes.byref(_lineorder(lineorder, keep)), ctypes.byref(_date(date, keep)),
+                                ctypes.byref(_dim(customer, "c_", keep)), ctypes.byref(_dim(supplier, "s_", keep)),
+                                ctypes.byref(_part(part, keep)), int(brute), nthreads],
+                 ["d_year", k1, k2, "profit", "count"])
 
 
 def tpch_q3(customer, orders, lineitem, brute=False, nthreads=1) -> OracleResult:

@@ -46,8 +46,8 @@ typedef struct {
 } orc_lineorder;
 typedef struct { int64_t n; const int32_t *datekey, *year, *yearmonthnum, *weeknuminyear; } orc_date;
 /* SSB customer or supplier */
-typedef struct { int64_t n; const int32_t* key; const int8_t *nation, *region; } orc_ssb_dim;
-typedef struct { int64_t n; const int32_t* partkey; const int8_t* mfgr; } orc_part;
+typedef struct { int64_t n; const int32_t* key; const int8_t *nation, *region; const int32_t* city; } orc_ssb_dim;
+typedef struct { int64_t n; const int32_t* partkey; const int8_t *mfgr, *category; const int32_t* brand1; } orc_part;
 /* TPC-H lineitem: DECIMALs are int64 fixed point, scale 2 */
 typedef struct {
   int64_t n;
@@ -78,6 +78,23 @@ int orc_ssb_q31_mat(const orc_lineorder* lo, const orc_ssb_dim* c, const orc_ssb
 /* SSB Q4.1 -> rows [d_year, c_nation, profit, count], ORDER BY d_year, c_nation */
 int orc_ssb_q41(const orc_lineorder* lo, const orc_date* d, const orc_ssb_dim* c,
                 const orc_ssb_dim* s, const orc_part* p, int brute, int nthreads, orc_result* out);
+/* SSB flight 2 (variant 1..3: Q2.1 p_category = 'MFGR#12', s_region = 'AMERICA'; Q2.2 p_brand1
+ * BETWEEN 'MFGR#2221' AND 'MFGR#2228', s_region = 'ASIA'; Q2.3 p_brand1 = 'MFGR#2239',
+ * s_region = 'EUROPE') -> rows [d_year, p_brand1, revenue, count] ORDER BY d_year, p_brand1 */
+int orc_ssb_q2(int variant, const orc_lineorder* lo, const orc_date* d, const orc_part* p,
+               const orc_ssb_dim* s, int brute, int nthreads, orc_result* out);
+/* SSB flight 3 (variant 2..4: Q3.2 c_nation = s_nation = 'UNITED STATES', d_year 1992..1997;
+ * Q3.3 c_city, s_city IN ('UNITED KI1', 'UNITED KI5'), d_year 1992..1997; Q3.4 the same cities,
+ * d_yearmonth = 'Dec1997') -> rows [c_city, s_city, d_year, revenue, count]
+ * ORDER BY d_year asc, revenue desc, c_city, s_city */
+int orc_ssb_q3(int variant, const orc_lineorder* lo, const orc_ssb_dim* c, const orc_ssb_dim* s,
+               const orc_date* d, int brute, int nthreads, orc_result* out);
+/* SSB flight 4 (variant 2..3): Q4.2 c_region = s_region = 'AMERICA', d_year IN (1997, 1998),
+ * p_mfgr IN ('MFGR#1', 'MFGR#2') -> rows [d_year, s_nation, p_category, profit, count];
+ * Q4.3 c_region = 'AMERICA', s_nation = 'UNITED STATES', d_year IN (1997, 1998),
+ * p_category = 'MFGR#14' -> rows [d_year, s_city, p_brand1, profit, count]; ORDER BY the keys */
+int orc_ssb_q4(int variant, const orc_lineorder* lo, const orc_date* d, const orc_ssb_dim* c,
+               const orc_ssb_dim* s, const orc_part* p, int brute, int nthreads, orc_result* out);
 /* TPC-H Q3 -> rows [l_orderkey, revenue(s4), o_orderdate, o_shippriority, count],
  * ORDER BY revenue desc, o_orderdate asc, l_orderkey asc (full result; caller applies LIMIT 10) */
 int orc_tpch_q3(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li, int brute,

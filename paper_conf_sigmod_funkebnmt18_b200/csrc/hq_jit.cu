@@ -705,10 +705,12 @@ std::string generate(const KPlan& kp) {
           // a lane's consecutive rows of one group (clustered keys: the lines of
           // an order) are folded first: one table update instead of a chain of
           // dependent global round trips (TPC-H Q3)
-          << "        u64 cn_[R];\n#pragma unroll\n        for (int r = 0; r < R; ++r) cn_[r] = 1ull;\n"
-          << "#pragma unroll\n        for (int r = 1; r < R; ++r) if (((mask >> r) & 1u) && ((mask >> (r - 1)) & 1u) && gk_[r] == gk_[r - 1]) {\n"
-          << "#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) va_[a][r] = agg_combine(AGG_FN[a], va_[a][r], va_[a][r - 1]);\n"
-          << "          cn_[r] += cn_[r - 1]; mask &= ~(1u << (r - 1)); }\n"
+          << "        u64 cn_[R];\n#pragma unroll\n        for (int r = 0; r < R; ++r) cn_[r] = 1ull;\n";
+        if (kp.smode == SM_NONE)  // only where an update is a dependent global round trip
+          o << "#pragma unroll\n        for (int r = 1; r < R; ++r) if (((mask >> r) & 1u) && ((mask >> (r - 1)) & 1u) && gk_[r] == gk_[r - 1]) {\n"
+            << "#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) va_[a][r] = agg_combine(AGG_FN[a], va_[a][r], va_[a][r - 1]);\n"
+            << "          cn_[r] += cn_[r - 1]; mask &= ~(1u << (r - 1)); }\n";
+        o
           << "#pragma unroll\n        for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) {\n"
           << "          i64 v_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n"
           << "          group_update(p, sagg, gk_[r], true, cn_[r], v_); }\n"

@@ -25,6 +25,9 @@ AMERICA = hqgen.code(hqgen.REGIONS, "AMERICA")
 BUILDING = hqgen.code(hqgen.MKTSEGMENTS, "BUILDING")
 MFGR1 = hqgen.code(hqgen.MFGRS, "MFGR#1")
 MFGR2 = hqgen.code(hqgen.MFGRS, "MFGR#2")
+EUROPE = hqgen.code(hqgen.REGIONS, "EUROPE")
+UNITED_STATES = hqgen.code(hqgen.NATIONS, "UNITED STATES")
+UNITED_KI1, UNITED_KI5 = hqgen.city_code("UNITED KI1"), hqgen.city_code("UNITED KI5")
 
 
 class Query:
@@ -141,6 +144,99 @@ def _ssb_q41(E: Engine, **_):
     return E.run(pb), pb
 
 
+# ------------------------------------------------------- SSB flight 2
+# select sum(lo_revenue), d_year, p_brand1 from lineorder, date, part, supplier
+# where <joins> and <part predicate> and s_region = <r> group by d_year, p_brand1
+# order by d_year, p_brand1
+_Q2X = {
+    1: ([("p_category", "=", hqgen.category_code("MFGR#12"))], AMERICA),
+    2: ([("p_brand1", "between", hqgen.brand_code("MFGR#2221"), hqgen.brand_code("MFGR#2228"))],
+        hqgen.code(hqgen.REGIONS, "ASIA")),
+    3: ([("p_brand1", "=", hqgen.brand_code("MFGR#2239"))], EUROPE),
+}
+
+
+def _ssb_q2(v: int):
+    def run(E: Engine, **_):
+        ppreds, region = _Q2X[v]
+        hp, hs, hd = E.hashes([
+            dict(table="part", key="p_partkey", payload=["p_brand1"], preds=ppreds),
+            dict(table="supplier", key="s_suppkey", preds=[("s_region", "=", region)]),
+            dict(table="date", key="d_datekey", payload=["d_year"])])
+        pb = E.plan("lineorder")
+        pb.probe(hs, "lo_suppkey", "semi")                  # 1/5, a bitmap staged in shared memory
+        pb.probe(hp, "lo_partkey", "inner", ["p_brand1"])   # 1/25 .. 1/1000, a byte map in L2
+        pb.probe(hd, "lo_orderdate", "inner", ["d_year"])
+        pb.aggregate(keys=[("d_year", 1992, 7), ("p_brand1", 0, 1000)],
+                     aggs=[("sum", "lo_revenue"), ("count", None)], agg_names=["revenue", "count"])
+        return E.run(pb), pb
+    return run
+
+
+# ------------------------------------------------------- SSB flight 3 (Q3.2-Q3.4)
+# select c_city, s_city, d_year, sum(lo_revenue) as revenue from customer, lineorder,
+# supplier, date where <joins> and <customer, supplier, date predicates>
+# group by c_city, s_city, d_year order by d_year asc, revenue desc
+_CITIES = ("in", [UNITED_KI1, UNITED_KI5])
+_Q3X = {
+    2: ([("c_nation", "=", UNITED_STATES)], [("s_nation", "=", UNITED_STATES)], [("d_year", "between", 1992, 1997)]),
+    3: ([("c_city",) + _CITIES], [("s_city",) + _CITIES], [("d_year", "between", 1992, 1997)]),
+    4: ([("c_city",) + _CITIES], [("s_city",) + _CITIES], [("d_yearmonthnum", "=", 199712)]),  # 'Dec1997'
+}
+
+
+def _ssb_q3(v: int):
+    def run(E: Engine, **_):
+        cpreds, spreds, dpreds = _Q3X[v]
+        hc, hs, hd = E.hashes([
+            dict(table="customer", key="c_custkey", payload=["c_city"], preds=cpreds),
+            dict(table="supplier", key="s_suppkey", payload=["s_city"], preds=spreds),
+            dict(table="date", key="d_datekey", payload=["d_year"], preds=dpreds)])
+        pb = E.plan("lineorder")
+        pb.probe(hs, "lo_suppkey", "inner", ["s_city"])
+        pb.probe(hc, "lo_custkey", "inner", ["c_city"])
+        pb.probe(hd, "lo_orderdate", "inner", ["d_year"])
+        pb.aggregate(keys=[("c_city", 0, 250), ("s_city", 0, 250), ("d_year", 1992, 7)],
+                     aggs=[("sum", "lo_revenue"), ("count", None)],
+                     order=[("d_year", False), ("revenue", True)], agg_names=["revenue", "count"],
+                     group_capacity=4096)  # declared 437,500 city pairs x years; <= 600 occur
+        return E.run(pb), pb
+    return run
+
+
+# ------------------------------------------------------- SSB flight 4 (Q4.2, Q4.3)
+# select d_year, <s_nation | s_city>, <p_category | p_brand1>, sum(lo_revenue - lo_supplycost)
+# from date, customer, supplier, part, lineorder where <joins> and c_region = 'AMERICA'
+# and <supplier predicate> and d_year in (1997, 1998) and <part predicate>
+# group by / order by the three keys
+def _ssb_q4(v: int):
+    def run(E: Engine, **_):
+        if v == 2:
+            sdesc = dict(table="supplier", key="s_suppkey", payload=["s_nation"], preds=[("s_region", "=", AMERICA)])
+            pdesc = dict(table="part", key="p_partkey", payload=["p_category"], preds=[("p_mfgr", "in", [MFGR1, MFGR2])])
+            skey, pkey = ("s_nation", 0, 25), ("p_category", 0, 25)
+        else:
+            sdesc = dict(table="supplier", key="s_suppkey", payload=["s_city"], preds=[("s_nation", "=", UNITED_STATES)])
+            pdesc = dict(table="part", key="p_partkey", payload=["p_brand1"],
+                         preds=[("p_category", "=", hqgen.category_code("MFGR#14"))])
+            skey, pkey = ("s_city", 0, 250), ("p_brand1", 0, 1000)
+        hc, hs, hp, hd = E.hashes([
+            dict(table="customer", key="c_custkey", preds=[("c_region", "=", AMERICA)]), sdesc, pdesc,
+            dict(table="date", key="d_datekey", payload=["d_year"],
+                 preds=[("d_year", "between", 1997, 1998)])])  # d_year = 1997 or d_year = 1998
+        pb = E.plan("lineorder")
+        pb.probe(hd, "lo_orderdate", "inner", ["d_year"])   # 2/7
+        pb.probe(hs, "lo_suppkey", "inner", [skey[0]])        # 1/5 or 1/25
+        pb.probe(hc, "lo_custkey", "semi")                    # 1/5
+        pb.probe(hp, "lo_partkey", "inner", [pkey[0]])        # 2/5 or 1/25
+        pb.compute("profit", [("load", "lo_revenue"), ("sub", "lo_supplycost")])
+        pb.aggregate(keys=[("d_year", 1992, 7), skey, pkey],
+                     aggs=[("sum", "profit"), ("count", None)], agg_names=["profit", "count"],
+                     group_capacity=4096)  # Q4.3: declared 1.75 M keys, <= 800 occur
+        return E.run(pb), pb
+    return run
+
+
 # ---------------------------------------------------------------- TPC-H Q3
 def _tpch_q3(E: Engine, limit: int = 10, **_):
     # pipeline 1: customer filter -> build (semi)
@@ -225,6 +321,19 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
           {"lineorder": ["lo_custkey", "lo_suppkey", "lo_partkey", "lo_orderdate", "lo_revenue", "lo_supplycost"],
            "customer": ["c_custkey", "c_nation", "c_region"], "supplier": ["s_suppkey", "s_region"],
            "part": ["p_partkey", "p_mfgr"], "date": ["d_datekey", "d_year"]}, _ssb_q41),
+    *[Query(f"ssb_q2{v}", "ssb", "lineorder",
+            {"lineorder": ["lo_partkey", "lo_suppkey", "lo_orderdate", "lo_revenue"],
+             "part": ["p_partkey", "p_category", "p_brand1"], "supplier": ["s_suppkey", "s_region"],
+             "date": ["d_datekey", "d_year"]}, _ssb_q2(v)) for v in (1, 2, 3)],
+    *[Query(f"ssb_q3{v}", "ssb", "lineorder",
+            {"lineorder": ["lo_custkey", "lo_suppkey", "lo_orderdate", "lo_revenue"],
+             "customer": ["c_custkey", "c_nation", "c_city"], "supplier": ["s_suppkey", "s_nation", "s_city"],
+             "date": ["d_datekey", "d_year", "d_yearmonthnum"]}, _ssb_q3(v)) for v in (2, 3, 4)],
+    *[Query(f"ssb_q4{v}", "ssb", "lineorder",
+            {"lineorder": ["lo_custkey", "lo_suppkey", "lo_partkey", "lo_orderdate", "lo_revenue", "lo_supplycost"],
+             "customer": ["c_custkey", "c_region"], "supplier": ["s_suppkey", "s_nation", "s_region", "s_city"],
+             "part": ["p_partkey", "p_mfgr", "p_category", "p_brand1"], "date": ["d_datekey", "d_year"]},
+            _ssb_q4(v)) for v in (2, 3)],
     Query("tpch_q3", "tpch", "lineitem",
           {"lineitem": ["l_orderkey", "l_shipdate", "l_extendedprice", "l_discount"],
            "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority"],

@@ -57,6 +57,12 @@ def oracle_run(qname, t, **kw):
         return oracle.ssb_q41(t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"])
     if qname == "tpch_q3":
         return oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    if qname.startswith("ssb_q2"):
+        return oracle.ssb_q2(int(qname[-1]), t["lineorder"], t["date"], t["part"], t["supplier"])
+    if qname.startswith("ssb_q3"):
+        return oracle.ssb_q3(int(qname[-1]), t["lineorder"], t["customer"], t["supplier"], t["date"])
+    if qname.startswith("ssb_q4"):
+        return oracle.ssb_q4(int(qname[-1]), t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"])
     raise KeyError(qname)
 
 
@@ -67,7 +73,15 @@ INT_COLS = {
     "ssb_q31": ["c_nation", "s_nation", "d_year", "revenue", "count"],
     "ssb_q41": ["d_year", "c_nation", "profit", "count"],
     "tpch_q3": ["l_orderkey", "o_orderdate", "o_shippriority", "revenue", "count"],
+    "ssb_q21": ["d_year", "p_brand1", "revenue", "count"], "ssb_q22": ["d_year", "p_brand1", "revenue", "count"],
+    "ssb_q23": ["d_year", "p_brand1", "revenue", "count"],
+    "ssb_q32": ["c_city", "s_city", "d_year", "revenue", "count"],
+    "ssb_q33": ["c_city", "s_city", "d_year", "revenue", "count"],
+    "ssb_q34": ["c_city", "s_city", "d_year", "revenue", "count"],
+    "ssb_q42": ["d_year", "s_nation", "p_category", "profit", "count"],
+    "ssb_q43": ["d_year", "s_city", "p_brand1", "profit", "count"],
 }
+SSB_FLIGHTS = ["ssb_q21", "ssb_q22", "ssb_q23", "ssb_q32", "ssb_q33", "ssb_q34", "ssb_q42", "ssb_q43"]
 
 
 def assert_same(qname, g, o):
@@ -91,6 +105,32 @@ def test_query_parity(ctx, ssb, tpch, qname):
     o = oracle_run(qname, host)
     assert_same(qname, g, o)
     assert g.qualifying == o.qualifying
+
+
+@pytest.fixture(scope="module")
+def ssb_sf1():
+    return {t: hqgen.generate(t, 1.0) for t in hqgen.SSB_TABLES}
+
+
+@pytest.mark.parametrize("qname", SSB_FLIGHTS)
+def test_ssb_flights_parity(ctx, ssb, ssb_sf1, qname):
+    """The remaining SSB queries (f3): SF 0.01 and SF 1 (flight 3's city predicates
+    select ~1/25,000 of the rows), fused and multi-pass, element-wise vs the oracle."""
+    for host in (ssb, ssb_sf1):
+        o = oracle_run(qname, host)
+        for em in (hq.EXEC_FUSED, hq.EXEC_MULTIPASS):
+            g = gpu_run(ctx, qname, host, exec_mode=em)
+            assert_same(qname, g, o)
+            assert g.qualifying == o.qualifying
+
+
+def test_ssb_flights_golden(ctx, golden):
+    """Hand-computed fixture F8 through the CUDA path (one ragged tile)."""
+    fx = golden("F8_ssb_flights_2_4.json")
+    for qname in SSB_FLIGHTS:
+        g = gpu_run(ctx, qname, fx["tables"])
+        assert [list(r) for r in g.rows(INT_COLS[qname])] == fx["expected"][qname]["rows"], qname
+        assert g.qualifying == fx["expected"][qname]["qualifying"], qname
 
 
 def test_tpch_q3_parity(ctx, tpch):
