@@ -546,10 +546,9 @@ std::string generate(const KPlan& kp) {
   }
   if (cpt >= 0 && !g.compacted_R) g.compact(kp.nops);
   if (mp == 1) {
-    // count kernel (Fig 8): one int32 flag per row of the range, indexed by
-    // absolute row (the flag column's base is offset by the host)
-    o << "      { int* fl_ = (int*)p.out[0];\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long row_ = tb_ + row0 + r;"
-      << " if (row_ >= p.row_begin && row_ < p.row_end) fl_[row_] = (int)((mask >> r) & 1u); } }\n";
+    // count kernel: the flags are written below, after the early-exit blocks
+    // close -- every row of the range gets its flag, also in a warp whose rows
+    // all died before a linear probe (the buffer is not cleared)
   } else if (mp == 2) {
     // write kernel (Fig 8): flagged rows write at their prefix-sum position --
     // the projections (A1) or the aggregation inputs: packed group key, values (B1/C1)
@@ -752,6 +751,9 @@ std::string generate(const KPlan& kp) {
   }
   }  // !mp
   for (int k = 0; k < g.open; ++k) o << "    }\n";
+  if (mp == 1)  // count kernel (Fig 8): one int32 flag per row, indexed by absolute row (base offset by the host)
+    o << "      { int* fl_ = (int*)p.out[0];\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long row_ = tb_ + row0 + r;"
+      << " if (row_ >= p.row_begin && row_ < p.row_end) fl_[row_] = (int)((mask >> r) & 1u); } }\n";
   if (g.compacted_R) o << "#undef R\n#define R " << g.compacted_R << "\n";
   o << "    }\n";
   if (sk == 2 && !mp) {

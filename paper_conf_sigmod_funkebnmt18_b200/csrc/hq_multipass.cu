@@ -19,6 +19,8 @@
 #include <cub/device/device_scan.cuh>
 
 #include <climits>
+#include <cstdio>
+#include <vector>
 
 #include "hq_device.cuh"
 #include "hq_internal.h"
@@ -147,7 +149,21 @@ void hq_run_multipass(hq_ctx* ctx, const hq_plan* plan, hq_result* r, int64_t gr
     for (int a = 0; a < nvals; ++a) k2.out_ptr[oc++] = r->mp_vals.as<long long>() + (size_t)a * m;
     k2.nout = oc;
   }
+  const bool dbg = getenv("HQ_MP_DEBUG") != nullptr;
+  if (dbg && agg && k2.nkeys > 0 && nq > 0) HQ_CUDA(cudaMemsetAsync(r->mp_keys.p, 0xFF, (size_t)nq * 8, st));
   if (nq > 0) launch_generated(ctx, k2);
+  if (dbg && agg && k2.nkeys > 0 && nq > 0) {  // every position written exactly once, keys in the domain
+    std::vector<unsigned long long> hk((size_t)nq);
+    HQ_CUDA(cudaMemcpyAsync(hk.data(), r->mp_keys.p, (size_t)nq * 8, cudaMemcpyDeviceToHost, st));
+    HQ_CUDA(cudaStreamSynchronize(st));
+    long long unwritten = 0, bad = 0;
+    for (auto k : hk) {
+      unwritten += k == ~0ULL;
+      bad += k != ~0ULL && k2.gmode != GM_HASH && (long long)k >= r->ngroups;
+    }
+    fprintf(stderr, "[hq multipass] nq %lld unwritten %lld out-of-domain %lld (ngroups %lld)\n", nq, unwritten, bad,
+            (long long)r->ngroups);
+  }
 
   if (agg && nq > 0) {
     const size_t m = (size_t)nq;

@@ -52,12 +52,13 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--sf", type=float, default=30)
     ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--queries", default=",".join(SSB))
     a = ap.parse_args()
     torch.cuda.set_device(0)
     ctx = hq.Context(0)
     host = {t: hqgen.generate(t, a.sf) for t in hqgen.SSB_TABLES}
     rows = []
-    for name in SSB:
+    for name in a.queries.split(","):
         q = QUERIES[name]
         tables = load_tables(ctx, q, a.sf, host=host)
         n = int(tables[q.fact].nrows)

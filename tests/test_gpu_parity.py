@@ -119,6 +119,7 @@ def test_ssb_flights_parity(ctx, ssb, ssb_sf1, qname):
     for host in (ssb, ssb_sf1):
         o = oracle_run(qname, host)
         for em in (hq.EXEC_FUSED, hq.EXEC_MULTIPASS):
+            poison_device_pool()
             g = gpu_run(ctx, qname, host, exec_mode=em)
             assert_same(qname, g, o)
             assert g.qualifying == o.qualifying
@@ -172,10 +173,34 @@ def test_operator_at_a_time_parity(ctx, ssb, tpch, qname):
     assert_same(qname, g, oracle_run(qname, host))
 
 
+def poison_device_pool(nbytes=1 << 30, byte=0x01):
+    """Fill and free a block of the device's default stream-ordered memory pool (the
+    one libhq allocates from, release threshold raised by hq_ctx_create) so that the
+    next allocations start with garbage rather than fresh zeroed pages: a kernel that
+    leaves part of a buffer unwritten then shows up."""
+    import ctypes
+    import glob
+    rt = None
+    for cand in ["libcudart.so"] + sorted(glob.glob("/usr/local/cuda/lib64/libcudart.so*")):
+        try:
+            rt = ctypes.CDLL(cand)
+            break
+        except OSError:
+            continue
+    assert rt is not None, "libcudart not found"
+    p = ctypes.c_void_p()
+    assert rt.cudaMallocAsync(ctypes.byref(p), ctypes.c_size_t(nbytes), None) == 0
+    assert rt.cudaMemsetAsync(p, byte, ctypes.c_size_t(nbytes), None) == 0
+    assert rt.cudaFreeAsync(p, None) == 0
+    assert rt.cudaDeviceSynchronize() == 0
+
+
 @pytest.mark.parametrize("qname", ["tpch_q6", "tpch_q1", "ssb_q11", "ssb_q12", "ssb_q31", "ssb_q41", "tpch_q3"])
 def test_multipass_parity(ctx, ssb, tpch, qname):
     """Multi-pass query compilation (f1: count kernel -> prefix sum -> write kernel
-    -> library reduce / sort + reduce-by-key; Table 4 A1/B1/C1) == oracle."""
+    -> library reduce / sort + reduce-by-key; Table 4 A1/B1/C1) == oracle, on
+    poisoned pool memory (every flag and position must be written)."""
+    poison_device_pool()
     host = host_for(qname, ssb, tpch)
     kw = {"limit": 0} if qname == "tpch_q3" else {}
     g = gpu_run(ctx, qname, host, exec_mode=hq.EXEC_MULTIPASS, **kw)
