@@ -128,6 +128,7 @@ hq_status hq_ctx_destroy(hq_ctx* ctx) {
     }
     for (auto e : ctx->event_pool) cudaEventDestroy(e);
     if (ctx->pinned) cudaFreeHost(ctx->pinned);
+    if (ctx->pinned_build) cudaFreeHost(ctx->pinned_build);
     delete ctx;
   });
 }

@@ -330,6 +330,7 @@ struct BuildState {
   bool counted = false;
   DevBuf scratch;  // count-pass block partials
   struct { unsigned long long cnt; int kmin, kmax, pmin, pmax; unsigned set[8]; } st{};
+  void* host_st = nullptr;  // this build's slot in hq_ctx::pinned_build (st's layout)
 };
 
 void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& bs) {
@@ -362,15 +363,16 @@ void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& 
   bs.words = d->npayload == 0 ? 1 : (d->npayload == 1 ? 2 : 4);
   bs.counted = d->expected_rows <= 0;
   if (bs.counted) {  // exact count pass: number and range of the qualifying keys
-    const int init[4] = {INT_MAX, INT_MIN, INT_MAX, INT_MIN};
-    HQ_CUDA(cudaMemcpyAsync(b.kminmax, init, 16, cudaMemcpyHostToDevice, ctx->stream));
+    // (kminmax needs no initial values: the count kernel's last block writes
+    // them; an empty table has count 0 and its range is never read)
     bs.scratch = DevBuf(ctx, (size_t)bs.grid * sizeof(CountPart) + 16);
     b.part = bs.scratch.p;
     b.ticket = (unsigned*)(h->dstate.as<char>() + 32);  // zeroed with dstate
     if (b.n > 0) { ctx->launches++; hq_build_count_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b); }
     HQ_CUDA(cudaGetLastError());
-    HQ_CUDA(cudaMemcpyAsync(&bs.st, b.nkeys, 24, cudaMemcpyDeviceToHost, ctx->stream));
-    HQ_CUDA(cudaMemcpyAsync(bs.st.set, b.pset, 32, cudaMemcpyDeviceToHost, ctx->stream));
+    // statistics -> pinned staging (truly asynchronous copies; read after the one sync)
+    HQ_CUDA(cudaMemcpyAsync(bs.host_st, b.nkeys, 24, cudaMemcpyDeviceToHost, ctx->stream));
+    HQ_CUDA(cudaMemcpyAsync((char*)bs.host_st + 24, b.pset, 32, cudaMemcpyDeviceToHost, ctx->stream));
   }
 }
 
@@ -431,11 +433,24 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
 void hq_build_hashes_impl(hq_ctx* ctx, int n, const hq_build_desc* d, hq_hash* const* h) {
   std::vector<BuildState> bs((size_t)n);
   bool any_count = false;
+  const size_t slot = 64;
+  static_assert(sizeof(BuildState::st) <= 64, "stats slot");
+  if (ctx->pinned_build_bytes < (size_t)n * slot) {
+    if (ctx->pinned_build) HQ_CUDA(cudaFreeHost(ctx->pinned_build));
+    ctx->pinned_build = nullptr;
+    ctx->pinned_build_bytes = 0;
+    const size_t want = std::max<size_t>((size_t)n * slot, 16 * slot);
+    HQ_CUDA(cudaHostAlloc(&ctx->pinned_build, want, cudaHostAllocDefault));
+    ctx->pinned_build_bytes = want;
+  }
   for (int i = 0; i < n; ++i) {
+    bs[i].host_st = (char*)ctx->pinned_build + (size_t)i * slot;
     build_prepare(ctx, d + i, h[i], bs[i]);
     any_count = any_count || bs[i].counted;
   }
   if (any_count) HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  for (int i = 0; i < n; ++i)
+    if (bs[i].counted) std::memcpy(&bs[i].st, bs[i].host_st, sizeof(bs[i].st));
   for (int i = 0; i < n; ++i) build_finish(ctx, d + i, h[i], bs[i]);
 }
 

@@ -57,6 +57,8 @@ struct hq_ctx {
   std::vector<cudaEvent_t> event_pool;
   void* pinned = nullptr;  // host staging for small results (cudaHostAlloc, grown on demand)
   size_t pinned_bytes = 0;
+  void* pinned_build = nullptr;  // host staging of the builds' count-pass statistics
+  size_t pinned_build_bytes = 0;
   void* alloc_bytes(size_t bytes);
   void free_bytes(void* p, size_t bytes);
 };
