@@ -80,7 +80,7 @@ def brand_code(s: str) -> int:
 
 # ---- table schemas (mirror hqgen.h) ---------------------------------------
 SSB_LINEORDER, SSB_DATE, SSB_CUSTOMER, SSB_SUPPLIER, SSB_PART = 1, 2, 3, 4, 5
-TPCH_LINEITEM, TPCH_ORDERS, TPCH_CUSTOMER = 11, 12, 13
+TPCH_LINEITEM, TPCH_ORDERS, TPCH_CUSTOMER, TPCH_SUPPLIER, TPCH_NATION, TPCH_REGION = 11, 12, 13, 14, 15, 16
 
 SCHEMAS: Dict[int, list] = {
     SSB_LINEORDER: [("lo_orderkey", "i4"), ("lo_linenumber", "i4"), ("lo_custkey", "i4"),
@@ -95,18 +95,22 @@ SCHEMAS: Dict[int, list] = {
     TPCH_LINEITEM: [("l_orderkey", "i4"), ("l_partkey", "i4"), ("l_quantity", "i8"),
                     ("l_extendedprice", "i8"), ("l_discount", "i8"), ("l_tax", "i8"),
                     ("l_returnflag", "i1"), ("l_linestatus", "i1"), ("l_shipdate", "i4"),
-                    ("l_receiptdate", "i4"), ("l_linenumber", "i4")],
+                    ("l_receiptdate", "i4"), ("l_linenumber", "i4"), ("l_suppkey", "i4")],
     TPCH_ORDERS: [("o_orderkey", "i4"), ("o_custkey", "i4"), ("o_orderdate", "i4"),
                   ("o_shippriority", "i4")],
     TPCH_CUSTOMER: [("c_custkey", "i4"), ("c_mktsegment", "i1"), ("c_nationkey", "i1")],
+    TPCH_SUPPLIER: [("s_suppkey", "i4"), ("s_nationkey", "i1")],
+    TPCH_NATION: [("n_nationkey", "i1"), ("n_regionkey", "i1")],
+    TPCH_REGION: [("r_regionkey", "i1")],
 }
 TABLE_NAMES = {
     "lineorder": SSB_LINEORDER, "date": SSB_DATE, "customer": SSB_CUSTOMER,
     "supplier": SSB_SUPPLIER, "part": SSB_PART, "lineitem": TPCH_LINEITEM,
-    "orders": TPCH_ORDERS, "tpch_customer": TPCH_CUSTOMER,
+    "orders": TPCH_ORDERS, "tpch_customer": TPCH_CUSTOMER, "tpch_supplier": TPCH_SUPPLIER,
+    "nation": TPCH_NATION, "region": TPCH_REGION,
 }
 SSB_TABLES = ["lineorder", "date", "customer", "supplier", "part"]
-TPCH_TABLES = ["lineitem", "orders", "tpch_customer"]
+TPCH_TABLES = ["lineitem", "orders", "tpch_customer", "tpch_supplier", "nation", "region"]
 
 
 def _build() -> None:

@@ -167,9 +167,12 @@ const int kW_D[D_NCOLS] = {4, 4, 4, 4};
 const int kW_C[C_NCOLS] = {4, 1, 1, 4};
 const int kW_S[S_NCOLS] = {4, 1, 1, 4};
 const int kW_P[P_NCOLS] = {4, 1, 1, 4};
-const int kW_L[L_NCOLS] = {4, 4, 8, 8, 8, 8, 1, 1, 4, 4, 4};
+const int kW_L[L_NCOLS] = {4, 4, 8, 8, 8, 8, 1, 1, 4, 4, 4, 4};
 const int kW_O[O_NCOLS] = {4, 4, 4, 4};
 const int kW_TC[TC_NCOLS] = {4, 1, 1};
+const int kW_TS[TS_NCOLS] = {4, 1};
+const int kW_N[N_NCOLS] = {1, 1};
+const int kW_R[R_NCOLS] = {1};
 
 const int* widths(int table, int* ncols) {
   switch (table) {
@@ -181,6 +184,9 @@ const int* widths(int table, int* ncols) {
     case HQG_TPCH_LINEITEM: *ncols = L_NCOLS; return kW_L;
     case HQG_TPCH_ORDERS: *ncols = O_NCOLS; return kW_O;
     case HQG_TPCH_CUSTOMER: *ncols = TC_NCOLS; return kW_TC;
+    case HQG_TPCH_SUPPLIER: *ncols = TS_NCOLS; return kW_TS;
+    case HQG_TPCH_NATION: *ncols = N_NCOLS; return kW_N;
+    case HQG_TPCH_REGION: *ncols = R_NCOLS; return kW_R;
   }
   *ncols = 0;
   return nullptr;
@@ -240,6 +246,7 @@ void l_line(const Out& o, double sf, uint64_t seed, int64_t i, int j, int64_t ro
       case L_SHIPDATE: v = yyyymmdd((int32_t)shipday()); break;
       case L_RECEIPTDATE: v = yyyymmdd((int32_t)rcptday()); break;
       case L_LINENUMBER: v = j + 1; break;
+      case L_SUPPKEY: v = uni(seed, S(T, L_SUPPKEY), q, 1, scaled(10000.0, sf)); break;
     }
     put(o, k, row, v, kW_L[o.cols[k]]);
   }
@@ -313,6 +320,18 @@ void gen_dim(int table, double sf, uint64_t seed, int64_t a, int64_t b, const Ou
           else if (c == TC_MKTSEGMENT) { v = uni(seed, S(table, TC_MKTSEGMENT), (uint64_t)r, 0, 4); w = 1; }
           else { v = uni(seed, S(table, TC_NATIONKEY), (uint64_t)r, 0, 24); w = 1; }
           break;
+        case HQG_TPCH_SUPPLIER:
+          if (c == TS_SUPPKEY) v = r + 1;
+          else { v = uni(seed, S(table, TS_NATIONKEY), (uint64_t)r, 0, 24); w = 1; }
+          break;
+        case HQG_TPCH_NATION:
+          v = c == N_NATIONKEY ? r : kNationRegion[r];
+          w = 1;
+          break;
+        case HQG_TPCH_REGION:
+          v = r;
+          w = 1;
+          break;
       }
       put(o, k, r, v, w);
     }
@@ -327,6 +346,9 @@ int64_t dim_rows(int table, double sf) {
     case HQG_SSB_PART: return ssb_parts(sf);
     case HQG_TPCH_ORDERS: return n_orders(sf);
     case HQG_TPCH_CUSTOMER: return scaled(150000.0, sf);
+    case HQG_TPCH_SUPPLIER: return scaled(10000.0, sf);
+    case HQG_TPCH_NATION: return 25;
+    case HQG_TPCH_REGION: return 5;
   }
   return -1;
 }

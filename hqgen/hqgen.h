@@ -36,7 +36,10 @@ enum {
   HQG_SSB_PART = 5,
   HQG_TPCH_LINEITEM = 11,
   HQG_TPCH_ORDERS = 12,
-  HQG_TPCH_CUSTOMER = 13
+  HQG_TPCH_CUSTOMER = 13,
+  HQG_TPCH_SUPPLIER = 14,
+  HQG_TPCH_NATION = 15,
+  HQG_TPCH_REGION = 16
 };
 
 /* SSB lineorder columns (all int32) */
@@ -56,12 +59,18 @@ enum { P_PARTKEY = 0, P_MFGR, P_CATEGORY, P_BRAND1, P_NCOLS };
 /* TPC-H lineitem */
 enum {
   L_ORDERKEY = 0, L_PARTKEY, L_QUANTITY, L_EXTENDEDPRICE, L_DISCOUNT, L_TAX,
-  L_RETURNFLAG, L_LINESTATUS, L_SHIPDATE, L_RECEIPTDATE, L_LINENUMBER, L_NCOLS
+  L_RETURNFLAG, L_LINESTATUS, L_SHIPDATE, L_RECEIPTDATE, L_LINENUMBER, L_SUPPKEY, L_NCOLS
 };
 /* TPC-H orders */
 enum { O_ORDERKEY = 0, O_CUSTKEY, O_ORDERDATE, O_SHIPPRIORITY, O_NCOLS };
 /* TPC-H customer */
 enum { TC_CUSTKEY = 0, TC_MKTSEGMENT, TC_NATIONKEY, TC_NCOLS };
+/* TPC-H supplier (10 K * SF rows): suppkey i32, nationkey i8 (uniform over the 25 nations) */
+enum { TS_SUPPKEY = 0, TS_NATIONKEY, TS_NCOLS };
+/* TPC-H nation (25 rows): nationkey i8 = the name's dictionary code, regionkey i8 */
+enum { N_NATIONKEY = 0, N_REGIONKEY, N_NCOLS };
+/* TPC-H region (5 rows): regionkey i8 = the name's dictionary code */
+enum { R_REGIONKEY = 0, R_NCOLS };
 
 /* Number of rows of a table at scale factor sf (lineorder/lineitem count
  * the 1..7 lines of every order, computed once and cached). <0 on error. */

@@ -63,7 +63,7 @@ class _Part(ctypes.Structure):
 class _Lineitem(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("orderkey", P_I32), ("quantity", P_I64),
                 ("extendedprice", P_I64), ("discount", P_I64), ("tax", P_I64),
-                ("returnflag", P_I8), ("linestatus", P_I8), ("shipdate", P_I32)]
+                ("returnflag", P_I8), ("linestatus", P_I8), ("shipdate", P_I32), ("suppkey", P_I32)]
 
 
 class _Orders(ctypes.Structure):
@@ -72,7 +72,19 @@ class _Orders(ctypes.Structure):
 
 
 class _TCustomer(ctypes.Structure):
-    _fields_ = [("n", ctypes.c_int64), ("custkey", P_I32), ("mktsegment", P_I8)]
+    _fields_ = [("n", ctypes.c_int64), ("custkey", P_I32), ("mktsegment", P_I8), ("nationkey", P_I8)]
+
+
+class _TSupplier(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("suppkey", P_I32), ("nationkey", P_I8)]
+
+
+class _Nation(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("nationkey", P_I8), ("regionkey", P_I8)]
+
+
+class _Region(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("regionkey", P_I8)]
 
 
 class OracleError(RuntimeError):
@@ -118,6 +130,8 @@ def lib():
             "orc_ssb_q31_mat": [P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
             "orc_ssb_q41": [P(_Lineorder), P(_Date), P(_SsbDim), P(_SsbDim), P(_Part), ctypes.c_int, ctypes.c_int],
             "orc_tpch_q3": [P(_TCustomer), P(_Orders), P(_Lineitem), ctypes.c_int, ctypes.c_int],
+            "orc_tpch_q5": [P(_TCustomer), P(_Orders), P(_Lineitem), P(_TSupplier), P(_Nation), P(_Region),
+                            ctypes.c_int, ctypes.c_int],
             "orc_ssb_q2": [ctypes.c_int, P(_Lineorder), P(_Date), P(_Part), P(_SsbDim), ctypes.c_int, ctypes.c_int],
             "orc_ssb_q3": [ctypes.c_int, P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
             "orc_ssb_q4": [ctypes.c_int, P(_Lineorder), P(_Date), P(_SsbDim), P(_SsbDim), P(_Part), ctypes.c_int,
@@ -194,6 +208,7 @@ def _lineitem(t, keep):
     s.returnflag = _ptr(t.get("l_returnflag"), P_I8, keep)
     s.linestatus = _ptr(t.get("l_linestatus"), P_I8, keep)
     s.shipdate = _ptr(t.get("l_shipdate"), P_I32, keep)
+    s.suppkey = _ptr(t.get("l_suppkey"), P_I32, keep)
     return s
 
 
@@ -210,6 +225,30 @@ def _tcust(t, keep):
     s.n = _n(t)
     s.custkey = _ptr(t["c_custkey"], P_I32, keep)
     s.mktsegment = _ptr(t.get("c_mktsegment"), P_I8, keep)
+    s.nationkey = _ptr(t.get("c_nationkey"), P_I8, keep)
+    return s
+
+
+def _tsupp(t, keep):
+    s = _TSupplier()
+    s.n = _n(t)
+    s.suppkey = _ptr(t["s_suppkey"], P_I32, keep)
+    s.nationkey = _ptr(t.get("s_nationkey"), P_I8, keep)
+    return s
+
+
+def _nation(t, keep):
+    s = _Nation()
+    s.n = _n(t)
+    s.nationkey = _ptr(t["n_nationkey"], P_I8, keep)
+    s.regionkey = _ptr(t.get("n_regionkey"), P_I8, keep)
+    return s
+
+
+def _region(t, keep):
+    s = _Region()
+    s.n = _n(t)
+    s.regionkey = _ptr(t["r_regionkey"], P_I8, keep)
     return s
 
 
@@ -315,6 +354,16 @@ def tpch_q3(customer, orders, lineitem, brute=False, nthreads=1) -> OracleResult
                                  ctypes.byref(_orders(orders, keep)),
                                  ctypes.byref(_lineitem(lineitem, keep)), int(brute), nthreads],
                  ["l_orderkey", "revenue", "o_orderdate", "o_shippriority", "count"])
+
+
+def tpch_q5(customer, orders, lineitem, supplier, nation, region, brute=False, nthreads=1) -> OracleResult:
+    """TPC-H Q5 -> [n_name, revenue (scale 4), count] ORDER BY revenue desc."""
+    keep = []
+    return _call("orc_tpch_q5", [ctypes.byref(_tcust(customer, keep)), ctypes.byref(_orders(orders, keep)),
+                                 ctypes.byref(_lineitem(lineitem, keep)), ctypes.byref(_tsupp(supplier, keep)),
+                                 ctypes.byref(_nation(nation, keep)), ctypes.byref(_region(region, keep)),
+                                 int(brute), nthreads],
+                 ["n_name", "revenue", "count"])
 
 
 def micro_select(lineorder, x, nthreads=1) -> OracleResult:

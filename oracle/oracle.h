@@ -55,9 +55,13 @@ typedef struct {
   const int64_t *quantity, *extendedprice, *discount, *tax;
   const int8_t *returnflag, *linestatus;
   const int32_t* shipdate;
+  const int32_t* suppkey;
 } orc_lineitem;
 typedef struct { int64_t n; const int32_t *orderkey, *custkey, *orderdate, *shippriority; } orc_orders;
-typedef struct { int64_t n; const int32_t* custkey; const int8_t* mktsegment; } orc_tpch_customer;
+typedef struct { int64_t n; const int32_t* custkey; const int8_t *mktsegment, *nationkey; } orc_tpch_customer;
+typedef struct { int64_t n; const int32_t* suppkey; const int8_t* nationkey; } orc_tpch_supplier;
+typedef struct { int64_t n; const int8_t *nationkey, *regionkey; } orc_nation;
+typedef struct { int64_t n; const int8_t* regionkey; } orc_region;
 
 /* TPC-H Q6 -> 1 row: [revenue (scale 4), count] */
 int orc_tpch_q6(const orc_lineitem* li, int nthreads, orc_result* out);
@@ -99,6 +103,11 @@ int orc_ssb_q4(int variant, const orc_lineorder* lo, const orc_date* d, const or
  * ORDER BY revenue desc, o_orderdate asc, l_orderkey asc (full result; caller applies LIMIT 10) */
 int orc_tpch_q3(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li, int brute,
                 int nthreads, orc_result* out);
+/* TPC-H Q5 (region 'ASIA', order year 1994) -> rows [n_name (nation code), revenue (scale 4),
+ * count] ORDER BY revenue desc, n_name */
+int orc_tpch_q5(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li,
+                const orc_tpch_supplier* s, const orc_nation* n, const orc_region* r, int brute, int nthreads,
+                orc_result* out);
 /* PAPER.md Fig 16 "Query 1": revenue = lo_extendedprice*lo_discount+lo_tax
  * where lo_quantity between 25-x and 25+x -> rows [revenue] sorted (a multiset) */
 int orc_micro_select(const orc_lineorder* lo, int32_t x, int nthreads, orc_result* out);

@@ -266,6 +266,49 @@ def _tpch_q3(E: Engine, limit: int = 10, **_):
     return res, pl
 
 
+# ---------------------------------------------------------------- TPC-H Q5
+# select n_name, sum(l_extendedprice * (1 - l_discount)) as revenue
+# from customer, orders, lineitem, supplier, nation, region
+# where c_custkey = o_custkey and l_orderkey = o_orderkey and l_suppkey = s_suppkey
+#   and c_nationkey = s_nationkey and s_nationkey = n_nationkey and n_regionkey = r_regionkey
+#   and r_name = 'ASIA' and o_orderdate >= '1994-01-01' and o_orderdate < '1995-01-01'
+# group by n_name order by revenue desc
+def _tpch_q5(E: Engine, **_):
+    asia = hqgen.code(hqgen.REGIONS, "ASIA")  # r_name = 'ASIA' (region key = its name's code)
+    # pipeline 1: region filter -> build; pipeline 2: nation -> probe region -> materialise -> build
+    hr = E.hash("region", "r_regionkey", preds=[("r_regionkey", "=", asia)])
+    hc, hs = E.hashes([dict(table="tpch_customer", key="c_custkey", payload=["c_nationkey"]),
+                       dict(table="tpch_supplier", key="s_suppkey", payload=["s_nationkey"])])
+    rn = ro = None
+    if E.builds_here:  # build side: only the root of a DistributedEngine holds the dimensions
+        pn = E.plan("nation")
+        pn.probe(hr, "n_regionkey", "semi")
+        pn.materialise([("n_nationkey", "i32")])
+        rn = E.run(pn, partitioned=False)
+        # pipeline 3: orders filter -> probe customer -> materialise -> build
+        po = E.plan("orders")
+        po.filter("o_orderdate", "between", 19940101, 19950101 - 1)
+        po.probe(hc, "o_custkey", "inner", ["c_nationkey"])
+        po.materialise([("o_orderkey", "i32"), ("c_nationkey", "i32")])
+        ro = E.run(po, partitioned=False)
+    hn = E.hash_from(rn, ["n_nationkey"], "n_nationkey")
+    ho = E.hash_from(ro, ["o_orderkey", "c_nationkey"], "o_orderkey", ["c_nationkey"])
+    # pipeline 4: lineitem -> probe orders, supplier -> c_nationkey = s_nationkey -> probe nation -> group
+    pl = E.plan("lineitem")
+    pl.probe(ho, "l_orderkey", "inner", ["c_nationkey"])   # ~1/7 of the rows (order year)
+    pl.probe(hs, "l_suppkey", "inner", ["s_nationkey"])
+    pl.compute("dn", [("load", "c_nationkey"), ("sub", "s_nationkey")])
+    pl.filter("dn", "=", 0)                                # c_nationkey = s_nationkey
+    pl.probe(hn, "s_nationkey", "semi")                    # the nation is in ASIA
+    pl.compute("n_name", [("load", "s_nationkey")])        # n_name = the nation's code
+    pl.compute("rev", [("load", "l_discount"), ("rsub", 100), ("mul", "l_extendedprice")])  # scale 4
+    pl.aggregate(keys=[("n_name", 0, 25)], aggs=[("sum", "rev"), ("count", None)],
+                 order=[("revenue", True)], agg_names=["revenue", "count"])
+    res = E.run(pl)
+    pl.keep += [rn, ro, hn, ho]
+    return res, pl
+
+
 # ------------------------------------------------ paper micro queries (f2)
 def _micro_select(E: Engine, x: int = 5, resolution=None, **_):
     """PAPER.md Fig 16 'Query 1': selection + projection, materialised."""
@@ -338,6 +381,11 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
           {"lineitem": ["l_orderkey", "l_shipdate", "l_extendedprice", "l_discount"],
            "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority"],
            "tpch_customer": ["c_custkey", "c_mktsegment"]}, _tpch_q3),
+    Query("tpch_q5", "tpch", "lineitem",
+          {"lineitem": ["l_orderkey", "l_suppkey", "l_extendedprice", "l_discount"],
+           "orders": ["o_orderkey", "o_custkey", "o_orderdate"], "tpch_customer": ["c_custkey", "c_nationkey"],
+           "tpch_supplier": ["s_suppkey", "s_nationkey"], "nation": ["n_nationkey", "n_regionkey"],
+           "region": ["r_regionkey"]}, _tpch_q5),
     Query("micro_select", "ssb", "lineorder",
           {"lineorder": ["lo_quantity", "lo_extendedprice", "lo_discount", "lo_tax"]}, _micro_select),
     Query("micro_sum", "ssb", "lineorder",

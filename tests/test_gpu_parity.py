@@ -57,6 +57,8 @@ def oracle_run(qname, t, **kw):
         return oracle.ssb_q41(t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"])
     if qname == "tpch_q3":
         return oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    if qname == "tpch_q5":
+        return oracle.tpch_q5(t["tpch_customer"], t["orders"], t["lineitem"], t["tpch_supplier"], t["nation"], t["region"])
     if qname.startswith("ssb_q2"):
         return oracle.ssb_q2(int(qname[-1]), t["lineorder"], t["date"], t["part"], t["supplier"])
     if qname.startswith("ssb_q3"):
@@ -80,6 +82,7 @@ INT_COLS = {
     "ssb_q34": ["c_city", "s_city", "d_year", "revenue", "count"],
     "ssb_q42": ["d_year", "s_nation", "p_category", "profit", "count"],
     "ssb_q43": ["d_year", "s_city", "p_brand1", "profit", "count"],
+    "tpch_q5": ["n_name", "revenue", "count"],
 }
 SSB_FLIGHTS = ["ssb_q21", "ssb_q22", "ssb_q23", "ssb_q32", "ssb_q33", "ssb_q34", "ssb_q42", "ssb_q43"]
 
@@ -132,6 +135,26 @@ def test_ssb_flights_golden(ctx, golden):
         g = gpu_run(ctx, qname, fx["tables"])
         assert [list(r) for r in g.rows(INT_COLS[qname])] == fx["expected"][qname]["rows"], qname
         assert g.qualifying == fx["expected"][qname]["qualifying"], qname
+
+
+@pytest.mark.parametrize("sf", [0.01, 1.0])
+def test_tpch_q5_parity(ctx, tpch, sf):
+    """TPC-H Q5 (f3): four pipelines (region build, nation and orders pipelines feeding
+    builds, the lineitem probe pipeline with a join predicate across two probes),
+    fused and multi-pass, vs the oracle; and the hand-computed fixture F9."""
+    host = tpch if sf == 0.01 else {t: hqgen.generate(t, sf) for t in hqgen.TPCH_TABLES}
+    o = oracle_run("tpch_q5", host)
+    for em in (hq.EXEC_FUSED, hq.EXEC_MULTIPASS):
+        g = gpu_run(ctx, "tpch_q5", host, exec_mode=em)
+        assert_same("tpch_q5", g, o)
+        assert g.qualifying == o.qualifying
+
+
+def test_tpch_q5_golden(ctx, golden):
+    fx = golden("F9_tpch_q5.json")
+    g = gpu_run(ctx, "tpch_q5", fx["tables"])
+    assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"]
+    assert g.qualifying == fx["expected"]["qualifying"]
 
 
 def test_tpch_q3_parity(ctx, tpch):
@@ -335,8 +358,10 @@ def test_lrgp_positions_segment_ordered(ctx):
         assert p[-1] - p[0] == e - s - 1 and np.all(np.diff(p) == 1)
 
 
-def test_edge_cases(ctx):
+@pytest.mark.parametrize("exec_mode", [hq.EXEC_FUSED, hq.EXEC_MULTIPASS])
+def test_edge_cases(ctx, exec_mode):
     from paper_conf_sigmod_funkebnmt18_b200.engine import PlanBuilder
+    poison_device_pool(1 << 26)
     # empty table, all-filtered, empty range
     for n in (0, 1, 33, 2048, 2049):
         a = np.arange(n, dtype=np.int32)
@@ -344,6 +369,7 @@ def test_edge_cases(ctx):
         pb = PlanBuilder(t)
         pb.filter("a", ">=", 0).aggregate(aggs=[("sum", "b"), ("count", None), ("min", "b"), ("max", "b")],
                                           agg_names=["s", "c", "mn", "mx"])
+        pb.plan.exec = exec_mode
         res = ctx.run(pb.plan, keep=pb.keep)
         s, c, mn, mx = [x[0] for x in res.fetch()]
         assert (s, c) == (int((a * 7).sum()), n)
@@ -351,8 +377,18 @@ def test_edge_cases(ctx):
             assert (mn, mx) == (0, 7 * (n - 1))
         pb = PlanBuilder(t)
         pb.filter("a", "<", 0).materialise([("b", "i64")])
+        pb.plan.exec = exec_mode
         res = ctx.run(pb.plan, keep=pb.keep)
         assert res.qualifying() == 0 and len(res.fetch()[0]) == 0
+        # grouped: a % 5 over every row (C1 sort path on the multi-pass side)
+        pb = PlanBuilder(t)
+        pb.compute("k", [("load", "a"), ("mod", 5)])
+        pb.aggregate(keys=[("k", 0, 5)], aggs=[("sum", "b"), ("count", None)], agg_names=["s", "c"])
+        pb.plan.exec = exec_mode
+        res = ctx.run(pb.plan, keep=pb.keep)
+        got = list(zip(*[x.tolist() for x in res.fetch()]))
+        exp = [(k, int((a[a % 5 == k] * 7).sum()), int((a % 5 == k).sum())) for k in range(5) if (a % 5 == k).any()]
+        assert got == exp
 
 
 @pytest.mark.parametrize("exec_mode", [hq.EXEC_FUSED, hq.EXEC_FUSED_INTERP, hq.EXEC_OAAT])
