@@ -108,6 +108,12 @@ int orc_tpch_q3(const orc_tpch_customer* c, const orc_orders* o, const orc_linei
 int orc_tpch_q5(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li,
                 const orc_tpch_supplier* s, const orc_nation* n, const orc_region* r, int brute, int nthreads,
                 orc_result* out);
+/* TPC-H Q10 (returned items; order quarter 1993-10-01 .. 1993-12-31, l_returnflag = 'R') ->
+ * rows [c_custkey, n_name, revenue (scale 4), count] ORDER BY revenue desc, c_custkey (full
+ * result; the caller applies LIMIT 20).  c_name, c_acctbal, c_phone, c_address, c_comment are
+ * functionally dependent on c_custkey and not generated (R18). */
+int orc_tpch_q10(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li, const orc_nation* n,
+                 int brute, int nthreads, orc_result* out);
 /* PAPER.md Fig 16 "Query 1": revenue = lo_extendedprice*lo_discount+lo_tax
  * where lo_quantity between 25-x and 25+x -> rows [revenue] sorted (a multiset) */
 int orc_micro_select(const orc_lineorder* lo, int32_t x, int nthreads, orc_result* out);

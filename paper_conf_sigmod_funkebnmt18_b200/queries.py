@@ -309,6 +309,41 @@ def _tpch_q5(E: Engine, **_):
     return res, pl
 
 
+# ---------------------------------------------------------------- TPC-H Q10
+# select c_custkey, c_name, sum(l_extendedprice * (1 - l_discount)) as revenue, c_acctbal,
+#   n_name, c_address, c_phone, c_comment from customer, orders, lineitem, nation
+# where c_custkey = o_custkey and l_orderkey = o_orderkey and o_orderdate >= '1993-10-01'
+#   and o_orderdate < '1994-01-01' and l_returnflag = 'R' and c_nationkey = n_nationkey
+# group by c_custkey, c_name, c_acctbal, c_phone, n_name, c_address, c_comment
+# order by revenue desc limit 20
+# (R18: the customer attributes besides c_custkey and n_name depend on c_custkey)
+def _tpch_q10(E: Engine, limit: int = 20, **_):
+    hc, hn = E.hashes([dict(table="tpch_customer", key="c_custkey", payload=["c_nationkey"]),
+                       dict(table="nation", key="n_nationkey")])
+    ro = None
+    if E.builds_here:
+        po = E.plan("orders")
+        po.filter("o_orderdate", "between", 19931001, 19940101 - 1)
+        po.probe(hc, "o_custkey", "inner", ["c_nationkey"])
+        po.materialise([("o_orderkey", "i32"), ("o_custkey", "i32"), ("c_nationkey", "i32")])
+        ro = E.run(po, partitioned=False)
+    ho = E.hash_from(ro, ["o_orderkey", "o_custkey", "c_nationkey"], "o_orderkey", ["o_custkey", "c_nationkey"])
+    nk = max(int(ho.info().nkeys), 0)
+    pl = E.plan("lineitem")
+    pl.filter("l_returnflag", "=", hqgen.code(hqgen.RETURNFLAGS, "R"))
+    pl.probe(ho, "l_orderkey", "inner", ["o_custkey", "c_nationkey"])
+    pl.probe(hn, "c_nationkey", "semi")
+    pl.compute("c_custkey", [("load", "o_custkey")])
+    pl.compute("n_name", [("load", "c_nationkey")])
+    pl.compute("rev", [("load", "l_discount"), ("rsub", 100), ("mul", "l_extendedprice")])  # scale 4
+    pl.aggregate(keys=[("c_custkey", 0, 1 << 31), ("n_name", 0, 25)], aggs=[("sum", "rev"), ("count", None)],
+                 order=[("revenue", True)], limit=limit, group_capacity=max(1024, nk),
+                 agg_names=["revenue", "count"])
+    res = E.run(pl)
+    pl.keep += [ro, ho]
+    return res, pl
+
+
 # ------------------------------------------------ paper micro queries (f2)
 def _micro_select(E: Engine, x: int = 5, resolution=None, **_):
     """PAPER.md Fig 16 'Query 1': selection + projection, materialised."""
@@ -386,6 +421,10 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
            "orders": ["o_orderkey", "o_custkey", "o_orderdate"], "tpch_customer": ["c_custkey", "c_nationkey"],
            "tpch_supplier": ["s_suppkey", "s_nationkey"], "nation": ["n_nationkey", "n_regionkey"],
            "region": ["r_regionkey"]}, _tpch_q5),
+    Query("tpch_q10", "tpch", "lineitem",
+          {"lineitem": ["l_orderkey", "l_returnflag", "l_extendedprice", "l_discount"],
+           "orders": ["o_orderkey", "o_custkey", "o_orderdate"], "tpch_customer": ["c_custkey", "c_nationkey"],
+           "nation": ["n_nationkey"]}, _tpch_q10),
     Query("micro_select", "ssb", "lineorder",
           {"lineorder": ["lo_quantity", "lo_extendedprice", "lo_discount", "lo_tax"]}, _micro_select),
     Query("micro_sum", "ssb", "lineorder",

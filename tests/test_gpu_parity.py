@@ -57,6 +57,8 @@ def oracle_run(qname, t, **kw):
         return oracle.ssb_q41(t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"])
     if qname == "tpch_q3":
         return oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    if qname == "tpch_q10":
+        return oracle.tpch_q10(t["tpch_customer"], t["orders"], t["lineitem"], t["nation"])
     if qname == "tpch_q5":
         return oracle.tpch_q5(t["tpch_customer"], t["orders"], t["lineitem"], t["tpch_supplier"], t["nation"], t["region"])
     if qname.startswith("ssb_q2"):
@@ -83,6 +85,7 @@ INT_COLS = {
     "ssb_q42": ["d_year", "s_nation", "p_category", "profit", "count"],
     "ssb_q43": ["d_year", "s_city", "p_brand1", "profit", "count"],
     "tpch_q5": ["n_name", "revenue", "count"],
+    "tpch_q10": ["c_custkey", "n_name", "revenue", "count"],
 }
 SSB_FLIGHTS = ["ssb_q21", "ssb_q22", "ssb_q23", "ssb_q32", "ssb_q33", "ssb_q34", "ssb_q42", "ssb_q43"]
 
@@ -153,6 +156,26 @@ def test_tpch_q5_parity(ctx, tpch, sf):
 def test_tpch_q5_golden(ctx, golden):
     fx = golden("F9_tpch_q5.json")
     g = gpu_run(ctx, "tpch_q5", fx["tables"])
+    assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"]
+    assert g.qualifying == fx["expected"]["qualifying"]
+
+
+@pytest.mark.parametrize("sf", [0.01, 1.0])
+def test_tpch_q10_parity(ctx, tpch, sf):
+    """TPC-H Q10 (f3): hash group-by over c_custkey behind two probes, top 20; the full
+    pre-LIMIT set under the total order, fused and multi-pass; fixture F10."""
+    host = tpch if sf == 0.01 else {t: hqgen.generate(t, sf) for t in hqgen.TPCH_TABLES}
+    o = oracle_run("tpch_q10", host)
+    for em in (hq.EXEC_FUSED, hq.EXEC_MULTIPASS):
+        full = gpu_run(ctx, "tpch_q10", host, exec_mode=em, limit=0)
+        assert_same("tpch_q10", full, o)
+        top = gpu_run(ctx, "tpch_q10", host, exec_mode=em)
+        assert top.rows(INT_COLS["tpch_q10"]) == o.rows(INT_COLS["tpch_q10"])[:20]
+
+
+def test_tpch_q10_golden(ctx, golden):
+    fx = golden("F10_tpch_q10.json")
+    g = gpu_run(ctx, "tpch_q10", fx["tables"])
     assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"]
     assert g.qualifying == fx["expected"]["qualifying"]
 
