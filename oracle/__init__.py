@@ -130,6 +130,8 @@ def lib():
             "orc_ssb_q31_mat": [P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
             "orc_ssb_q41": [P(_Lineorder), P(_Date), P(_SsbDim), P(_SsbDim), P(_Part), ctypes.c_int, ctypes.c_int],
             "orc_tpch_q3": [P(_TCustomer), P(_Orders), P(_Lineitem), ctypes.c_int, ctypes.c_int],
+            "orc_tpch_q7": [P(_TCustomer), P(_Orders), P(_Lineitem), P(_TSupplier), P(_Nation),
+                            ctypes.c_int, ctypes.c_int],
             "orc_tpch_q10": [P(_TCustomer), P(_Orders), P(_Lineitem), P(_Nation), ctypes.c_int, ctypes.c_int],
             "orc_tpch_q5": [P(_TCustomer), P(_Orders), P(_Lineitem), P(_TSupplier), P(_Nation), P(_Region),
                             ctypes.c_int, ctypes.c_int],
@@ -365,6 +367,16 @@ def tpch_q5(customer, orders, lineitem, supplier, nation, region, brute=False, n
                                  ctypes.byref(_nation(nation, keep)), ctypes.byref(_region(region, keep)),
                                  int(brute), nthreads],
                  ["n_name", "revenue", "count"])
+
+
+def tpch_q7(customer, orders, lineitem, supplier, nation, brute=False, nthreads=1) -> OracleResult:
+    """TPC-H Q7 -> [supp_nation, cust_nation, l_year, revenue (scale 4), count]
+    ORDER BY supp_nation, cust_nation, l_year."""
+    keep = []
+    return _call("orc_tpch_q7", [ctypes.byref(_tcust(customer, keep)), ctypes.byref(_orders(orders, keep)),
+                                 ctypes.byref(_lineitem(lineitem, keep)), ctypes.byref(_tsupp(supplier, keep)),
+                                 ctypes.byref(_nation(nation, keep)), int(brute), nthreads],
+                 ["supp_nation", "cust_nation", "l_year", "revenue", "count"])
 
 
 def tpch_q10(customer, orders, lineitem, nation, brute=False, nthreads=1) -> OracleResult:

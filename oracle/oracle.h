@@ -114,6 +114,11 @@ int orc_tpch_q5(const orc_tpch_customer* c, const orc_orders* o, const orc_linei
  * functionally dependent on c_custkey and not generated (R18). */
 int orc_tpch_q10(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li, const orc_nation* n,
                  int brute, int nthreads, orc_result* out);
+/* TPC-H Q7 (volume shipping between FRANCE and GERMANY, ship years 1995-1996) ->
+ * rows [supp_nation, cust_nation, l_year, revenue (scale 4), count]
+ * ORDER BY supp_nation, cust_nation, l_year (n_name = the nation's code, R18) */
+int orc_tpch_q7(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li,
+                const orc_tpch_supplier* s, const orc_nation* n, int brute, int nthreads, orc_result* out);
 /* PAPER.md Fig 16 "Query 1": revenue = lo_extendedprice*lo_discount+lo_tax
  * where lo_quantity between 25-x and 25+x -> rows [revenue] sorted (a multiset) */
 int orc_micro_select(const orc_lineorder* lo, int32_t x, int nthreads, orc_result* out);

@@ -309,6 +309,53 @@ def _tpch_q5(E: Engine, **_):
     return res, pl
 
 
+# ---------------------------------------------------------------- TPC-H Q7
+# select supp_nation, cust_nation, l_year, sum(volume) as revenue
+# from (select n1.n_name as supp_nation, n2.n_name as cust_nation, extract(year from l_shipdate) as l_year,
+#              l_extendedprice * (1 - l_discount) as volume
+#       from supplier, lineitem, orders, customer, nation n1, nation n2
+#       where s_suppkey = l_suppkey and o_orderkey = l_orderkey and c_custkey = o_custkey
+#         and s_nationkey = n1.n_nationkey and c_nationkey = n2.n_nationkey
+#         and ((n1.n_name = 'FRANCE' and n2.n_name = 'GERMANY') or (n1.n_name = 'GERMANY' and n2.n_name = 'FRANCE'))
+#         and l_shipdate between date '1995-01-01' and date '1996-12-31') as shipping
+# group by supp_nation, cust_nation, l_year order by supp_nation, cust_nation, l_year
+# The disjunction is (n1, n2 both in {FRANCE, GERMANY}) and n1 != n2; each half is pushed
+# into its build (n_name = nation key, R18), the inequality stays in the pipeline.
+def _tpch_q7(E: Engine, **_):
+    pair = ("in", [hqgen.code(hqgen.NATIONS, "FRANCE"), hqgen.code(hqgen.NATIONS, "GERMANY")])
+    hs, hc, hn = E.hashes([dict(table="tpch_supplier", key="s_suppkey", payload=["s_nationkey"],
+                                preds=[("s_nationkey",) + pair]),
+                           dict(table="tpch_customer", key="c_custkey", payload=["c_nationkey"],
+                                preds=[("c_nationkey",) + pair]),
+                           dict(table="nation", key="n_nationkey", preds=[("n_nationkey",) + pair])])
+    ro = None
+    if E.builds_here:
+        po = E.plan("orders")
+        po.probe(hc, "o_custkey", "inner", ["c_nationkey"])   # 2/25 of the orders
+        po.materialise([("o_orderkey", "i32"), ("c_nationkey", "i32")])
+        ro = E.run(po, partitioned=False)
+    ho = E.hash_from(ro, ["o_orderkey", "c_nationkey"], "o_orderkey", ["c_nationkey"])
+    pl = E.plan("lineitem")
+    pl.filter("l_shipdate", "between", 19950101, 19961231)  # ~30 %
+    pl.probe(hs, "l_suppkey", "inner", ["s_nationkey"])     # 2/25
+    pl.probe(ho, "l_orderkey", "inner", ["c_nationkey"])    # 2/25
+    pl.compute("dn", [("load", "s_nationkey"), ("sub", "c_nationkey")])
+    pl.filter("dn", "!=", 0)                                # FRANCE -> GERMANY or GERMANY -> FRANCE
+    pl.probe(hn, "s_nationkey", "semi")                     # n1
+    pl.probe(hn, "c_nationkey", "semi")                     # n2
+    pl.compute("l_year", [("load", "l_shipdate"), ("div", 10000)])
+    pl.compute("rev", [("load", "l_discount"), ("rsub", 100), ("mul", "l_extendedprice")])  # scale 4
+    pl.aggregate(keys=[("s_nationkey", 0, 25), ("c_nationkey", 0, 25), ("l_year", 1995, 2)],
+                 aggs=[("sum", "rev"), ("count", None)],
+                 order=[("s_nationkey", False), ("c_nationkey", False), ("l_year", False)],
+                 agg_names=["revenue", "count"])
+    pb_names = ["supp_nation", "cust_nation", "l_year", "revenue", "count"]
+    res = E.run(pl)
+    pl.result_names = pb_names
+    pl.keep += [ro, ho]
+    return res, pl
+
+
 # ---------------------------------------------------------------- TPC-H Q10
 # select c_custkey, c_name, sum(l_extendedprice * (1 - l_discount)) as revenue, c_acctbal,
 #   n_name, c_address, c_phone, c_comment from customer, orders, lineitem, nation
@@ -421,6 +468,10 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
            "orders": ["o_orderkey", "o_custkey", "o_orderdate"], "tpch_customer": ["c_custkey", "c_nationkey"],
            "tpch_supplier": ["s_suppkey", "s_nationkey"], "nation": ["n_nationkey", "n_regionkey"],
            "region": ["r_regionkey"]}, _tpch_q5),
+    Query("tpch_q7", "tpch", "lineitem",
+          {"lineitem": ["l_orderkey", "l_suppkey", "l_shipdate", "l_extendedprice", "l_discount"],
+           "orders": ["o_orderkey", "o_custkey"], "tpch_customer": ["c_custkey", "c_nationkey"],
+           "tpch_supplier": ["s_suppkey", "s_nationkey"], "nation": ["n_nationkey"]}, _tpch_q7),
     Query("tpch_q10", "tpch", "lineitem",
           {"lineitem": ["l_orderkey", "l_returnflag", "l_extendedprice", "l_discount"],
            "orders": ["o_orderkey", "o_custkey", "o_orderdate"], "tpch_customer": ["c_custkey", "c_nationkey"],

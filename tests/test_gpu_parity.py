@@ -57,6 +57,8 @@ def oracle_run(qname, t, **kw):
         return oracle.ssb_q41(t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"])
     if qname == "tpch_q3":
         return oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    if qname == "tpch_q7":
+        return oracle.tpch_q7(t["tpch_customer"], t["orders"], t["lineitem"], t["tpch_supplier"], t["nation"])
     if qname == "tpch_q10":
         return oracle.tpch_q10(t["tpch_customer"], t["orders"], t["lineitem"], t["nation"])
     if qname == "tpch_q5":
@@ -86,6 +88,7 @@ INT_COLS = {
     "ssb_q43": ["d_year", "s_city", "p_brand1", "profit", "count"],
     "tpch_q5": ["n_name", "revenue", "count"],
     "tpch_q10": ["c_custkey", "n_name", "revenue", "count"],
+    "tpch_q7": ["supp_nation", "cust_nation", "l_year", "revenue", "count"],
 }
 SSB_FLIGHTS = ["ssb_q21", "ssb_q22", "ssb_q23", "ssb_q32", "ssb_q33", "ssb_q34", "ssb_q42", "ssb_q43"]
 
@@ -156,6 +159,27 @@ def test_tpch_q5_parity(ctx, tpch, sf):
 def test_tpch_q5_golden(ctx, golden):
     fx = golden("F9_tpch_q5.json")
     g = gpu_run(ctx, "tpch_q5", fx["tables"])
+    assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"]
+    assert g.qualifying == fx["expected"]["qualifying"]
+
+
+@pytest.mark.parametrize("sf", [0.01, 1.0])
+def test_tpch_q7_parity(ctx, tpch, sf):
+    """TPC-H Q7 (f3): two filtered builds, the orders pipeline feeding a build, the
+    lineitem pipeline with an inequality across two probe payloads and two semi-probes
+    of one table; fused and multi-pass; fixture F11."""
+    host = tpch if sf == 0.01 else {t: hqgen.generate(t, sf) for t in hqgen.TPCH_TABLES}
+    o = oracle_run("tpch_q7", host)
+    assert o.nrows == 4
+    for em in (hq.EXEC_FUSED, hq.EXEC_MULTIPASS):
+        g = gpu_run(ctx, "tpch_q7", host, exec_mode=em)
+        assert_same("tpch_q7", g, o)
+        assert g.qualifying == o.qualifying
+
+
+def test_tpch_q7_golden(ctx, golden):
+    fx = golden("F11_tpch_q7.json")
+    g = gpu_run(ctx, "tpch_q7", fx["tables"])
     assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"]
     assert g.qualifying == fx["expected"]["qualifying"]
 
