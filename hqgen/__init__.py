@@ -38,6 +38,15 @@ MFGRS = ["MFGR#1", "MFGR#2", "MFGR#3", "MFGR#4", "MFGR#5"]
 MKTSEGMENTS = ["AUTOMOBILE", "BUILDING", "FURNITURE", "HOUSEHOLD", "MACHINERY"]
 RETURNFLAGS = ["A", "N", "R"]
 LINESTATUS = ["F", "O"]
+ORDERSTATUS = ["F", "O", "P"]
+ORDERPRIORITIES = ["1-URGENT", "2-HIGH", "3-MEDIUM", "4-NOT SPECIFIED", "5-LOW"]
+SHIPMODES = ["AIR", "FOB", "MAIL", "RAIL", "REG AIR", "SHIP", "TRUCK"]
+SHIPINSTRUCTS = ["COLLECT COD", "DELIVER IN PERSON", "NONE", "TAKE BACK RETURN"]
+# TPC-H p_brand 'Brand#MN' (M, N in 1..5) = (M-1)*5 + N-1; p_container = the 40
+# 'SIZE TYPE' strings (TPC-H 4.2.2.13) in string order
+BRANDS = [f"Brand#{m}{n}" for m in range(1, 6) for n in range(1, 6)]
+CONTAINERS = sorted(f"{a} {b}" for a in ["SM", "LG", "MED", "JUMBO", "WRAP"]
+                    for b in ["CASE", "BOX", "BAG", "JAR", "PKG", "PACK", "CAN", "DRUM"])
 
 
 def code(dictionary: Sequence[str], s: str) -> int:
@@ -81,6 +90,7 @@ def brand_code(s: str) -> int:
 # ---- table schemas (mirror hqgen.h) ---------------------------------------
 SSB_LINEORDER, SSB_DATE, SSB_CUSTOMER, SSB_SUPPLIER, SSB_PART = 1, 2, 3, 4, 5
 TPCH_LINEITEM, TPCH_ORDERS, TPCH_CUSTOMER, TPCH_SUPPLIER, TPCH_NATION, TPCH_REGION = 11, 12, 13, 14, 15, 16
+TPCH_PART, TPCH_PARTSUPP = 17, 18
 
 SCHEMAS: Dict[int, list] = {
     SSB_LINEORDER: [("lo_orderkey", "i4"), ("lo_linenumber", "i4"), ("lo_custkey", "i4"),
@@ -95,22 +105,26 @@ SCHEMAS: Dict[int, list] = {
     TPCH_LINEITEM: [("l_orderkey", "i4"), ("l_partkey", "i4"), ("l_quantity", "i8"),
                     ("l_extendedprice", "i8"), ("l_discount", "i8"), ("l_tax", "i8"),
                     ("l_returnflag", "i1"), ("l_linestatus", "i1"), ("l_shipdate", "i4"),
-                    ("l_receiptdate", "i4"), ("l_linenumber", "i4"), ("l_suppkey", "i4")],
+                    ("l_receiptdate", "i4"), ("l_linenumber", "i4"), ("l_suppkey", "i4"),
+                    ("l_commitdate", "i4"), ("l_shipmode", "i1"), ("l_shipinstruct", "i1")],
     TPCH_ORDERS: [("o_orderkey", "i4"), ("o_custkey", "i4"), ("o_orderdate", "i4"),
-                  ("o_shippriority", "i4")],
+                  ("o_shippriority", "i4"), ("o_orderpriority", "i1"), ("o_totalprice", "i8"),
+                  ("o_orderstatus", "i1")],
     TPCH_CUSTOMER: [("c_custkey", "i4"), ("c_mktsegment", "i1"), ("c_nationkey", "i1")],
     TPCH_SUPPLIER: [("s_suppkey", "i4"), ("s_nationkey", "i1")],
     TPCH_NATION: [("n_nationkey", "i1"), ("n_regionkey", "i1")],
     TPCH_REGION: [("r_regionkey", "i1")],
+    TPCH_PART: [("p_partkey", "i4"), ("p_brand", "i1"), ("p_container", "i1"), ("p_size", "i4")],
+    TPCH_PARTSUPP: [("ps_partkey", "i4"), ("ps_suppkey", "i4"), ("ps_supplycost", "i8")],
 }
 TABLE_NAMES = {
     "lineorder": SSB_LINEORDER, "date": SSB_DATE, "customer": SSB_CUSTOMER,
     "supplier": SSB_SUPPLIER, "part": SSB_PART, "lineitem": TPCH_LINEITEM,
     "orders": TPCH_ORDERS, "tpch_customer": TPCH_CUSTOMER, "tpch_supplier": TPCH_SUPPLIER,
-    "nation": TPCH_NATION, "region": TPCH_REGION,
+    "nation": TPCH_NATION, "region": TPCH_REGION, "tpch_part": TPCH_PART, "partsupp": TPCH_PARTSUPP,
 }
 SSB_TABLES = ["lineorder", "date", "customer", "supplier", "part"]
-TPCH_TABLES = ["lineitem", "orders", "tpch_customer", "tpch_supplier", "nation", "region"]
+TPCH_TABLES = ["lineitem", "orders", "tpch_customer", "tpch_supplier", "nation", "region", "tpch_part", "partsupp"]
 
 
 def _build() -> None:

@@ -167,8 +167,10 @@ const int kW_D[D_NCOLS] = {4, 4, 4, 4};
 const int kW_C[C_NCOLS] = {4, 1, 1, 4};
 const int kW_S[S_NCOLS] = {4, 1, 1, 4};
 const int kW_P[P_NCOLS] = {4, 1, 1, 4};
-const int kW_L[L_NCOLS] = {4, 4, 8, 8, 8, 8, 1, 1, 4, 4, 4, 4};
-const int kW_O[O_NCOLS] = {4, 4, 4, 4};
+const int kW_L[L_NCOLS] = {4, 4, 8, 8, 8, 8, 1, 1, 4, 4, 4, 4, 4, 1, 1};
+const int kW_O[O_NCOLS] = {4, 4, 4, 4, 1, 8, 1};
+const int kW_TP[TP_NCOLS] = {4, 1, 1, 4};
+const int kW_PS[PS_NCOLS] = {4, 4, 8};
 const int kW_TC[TC_NCOLS] = {4, 1, 1};
 const int kW_TS[TS_NCOLS] = {4, 1};
 const int kW_N[N_NCOLS] = {1, 1};
@@ -187,6 +189,8 @@ const int* widths(int table, int* ncols) {
     case HQG_TPCH_SUPPLIER: *ncols = TS_NCOLS; return kW_TS;
     case HQG_TPCH_NATION: *ncols = N_NCOLS; return kW_N;
     case HQG_TPCH_REGION: *ncols = R_NCOLS; return kW_R;
+    case HQG_TPCH_PART: *ncols = TP_NCOLS; return kW_TP;
+    case HQG_TPCH_PARTSUPP: *ncols = PS_NCOLS; return kW_PS;
   }
   *ncols = 0;
   return nullptr;
@@ -220,36 +224,76 @@ void lo_line(const Out& o, double sf, uint64_t seed, int64_t i, int j, int64_t r
   }
 }
 
-// TPC-H lineitem line
-void l_line(const Out& o, double sf, uint64_t seed, int64_t i, int j, int64_t row) {
-  const int T = HQG_TPCH_LINEITEM;
-  const uint64_t q = (uint64_t)i * 8 + (uint64_t)j;
-  const int64_t odate = uni(seed, S(HQG_TPCH_ORDERS, O_ORDERDATE), (uint64_t)i, 0, kTpchODays - 1);
+// TPC-H lineitem line values (i = order index, j = line index within order);
+// the orders' o_totalprice / o_orderstatus are derived from the same values.
+struct TLine {
+  double sf;
+  uint64_t seed;
+  int64_t i;
+  uint64_t q;
+  int64_t odate;
   int64_t pk = -1, qty = -1, ship = -1, rcpt = -1;
-  auto partkey = [&] { if (pk < 0) pk = uni(seed, S(T, L_PARTKEY), q, 1, scaled(200000.0, sf)); return pk; };
-  auto quantity = [&] { if (qty < 0) qty = uni(seed, S(T, L_QUANTITY), q, 1, 50); return qty; };
-  auto shipday = [&] { if (ship < 0) ship = odate + uni(seed, S(T, L_SHIPDATE), q, 1, 121); return ship; };
-  auto rcptday = [&] { if (rcpt < 0) rcpt = shipday() + uni(seed, S(T, L_RECEIPTDATE), q, 1, 30); return rcpt; };
+  TLine(double sf_, uint64_t seed_, int64_t i_, int j)
+      : sf(sf_), seed(seed_), i(i_), q((uint64_t)i_ * 8 + (uint64_t)j),
+        odate(uni(seed_, S(HQG_TPCH_ORDERS, O_ORDERDATE), (uint64_t)i_, 0, kTpchODays - 1)) {}
+  static const int T = HQG_TPCH_LINEITEM;
+  int64_t partkey() { if (pk < 0) pk = uni(seed, S(T, L_PARTKEY), q, 1, scaled(200000.0, sf)); return pk; }
+  int64_t quantity() { if (qty < 0) qty = uni(seed, S(T, L_QUANTITY), q, 1, 50); return qty; }
+  int64_t shipday() { if (ship < 0) ship = odate + uni(seed, S(T, L_SHIPDATE), q, 1, 121); return ship; }
+  int64_t rcptday() { if (rcpt < 0) rcpt = shipday() + uni(seed, S(T, L_RECEIPTDATE), q, 1, 30); return rcpt; }
+  int64_t discount() { return uni(seed, S(T, L_DISCOUNT), q, 0, 10); }
+  int64_t tax() { return uni(seed, S(T, L_TAX), q, 0, 8); }
+  int64_t extendedprice() { return quantity() * (int64_t)retailprice(partkey()); }
+  int64_t suppkey() {  // one of the part's four partsupp suppliers (TPC-H 4.2.3)
+    const int64_t ns = scaled(10000.0, sf);
+    return ps_supplier(partkey(), uni(seed, S(T, L_SUPPKEY), q, 0, 3), ns);
+  }
+  static int64_t ps_supplier(int64_t pk, int64_t k, int64_t ns) {
+    return (pk + k * (ns / 4 + (pk - 1) / ns)) % ns + 1;
+  }
+};
+
+void l_line(const Out& o, double sf, uint64_t seed, int64_t i, int j, int64_t row) {
+  TLine L(sf, seed, i, j);
+  const int T = HQG_TPCH_LINEITEM;
+  const uint64_t q = L.q;
   for (int k = 0; k < o.ncols; ++k) {
     int64_t v = 0;
     switch (o.cols[k]) {
       case L_ORDERKEY: v = orderkey(i); break;
-      case L_PARTKEY: v = partkey(); break;
-      case L_QUANTITY: v = quantity() * 100; break;                               // scale 2
-      case L_EXTENDEDPRICE: v = quantity() * (int64_t)retailprice(partkey()); break;  // cents
-      case L_DISCOUNT: v = uni(seed, S(T, L_DISCOUNT), q, 0, 10); break;           // hundredths
-      case L_TAX: v = uni(seed, S(T, L_TAX), q, 0, 8); break;                      // hundredths
+      case L_PARTKEY: v = L.partkey(); break;
+      case L_QUANTITY: v = L.quantity() * 100; break;  // scale 2
+      case L_EXTENDEDPRICE: v = L.extendedprice(); break;  // cents
+      case L_DISCOUNT: v = L.discount(); break;  // hundredths
+      case L_TAX: v = L.tax(); break;            // hundredths
       case L_RETURNFLAG:  // A=0, N=1, R=2 ; spec 4.2.3: R or A if receipt <= CURRENTDATE
-        v = rcptday() <= kCurrentDay ? (uni(seed, S(T, L_RETURNFLAG), q, 0, 1) ? 2 : 0) : 1;
+        v = L.rcptday() <= kCurrentDay ? (uni(seed, S(T, L_RETURNFLAG), q, 0, 1) ? 2 : 0) : 1;
         break;
-      case L_LINESTATUS: v = shipday() > kCurrentDay ? 1 : 0; break;  // F=0, O=1
-      case L_SHIPDATE: v = yyyymmdd((int32_t)shipday()); break;
-      case L_RECEIPTDATE: v = yyyymmdd((int32_t)rcptday()); break;
+      case L_LINESTATUS: v = L.shipday() > kCurrentDay ? 1 : 0; break;  // F=0, O=1
+      case L_SHIPDATE: v = yyyymmdd((int32_t)L.shipday()); break;
+      case L_RECEIPTDATE: v = yyyymmdd((int32_t)L.rcptday()); break;
       case L_LINENUMBER: v = j + 1; break;
-      case L_SUPPKEY: v = uni(seed, S(T, L_SUPPKEY), q, 1, scaled(10000.0, sf)); break;
+      case L_SUPPKEY: v = L.suppkey(); break;
+      case L_COMMITDATE: v = yyyymmdd((int32_t)(L.odate + uni(seed, S(T, L_COMMITDATE), q, 30, 90))); break;
+      case L_SHIPMODE: v = uni(seed, S(T, L_SHIPMODE), q, 0, 6); break;
+      case L_SHIPINSTRUCT: v = uni(seed, S(T, L_SHIPINSTRUCT), q, 0, 3); break;
     }
     put(o, k, row, v, kW_L[o.cols[k]]);
   }
+}
+
+// o_totalprice (cents) and o_orderstatus (F=0, O=1, P=2) of order i from its lines
+void order_lines(double sf, uint64_t seed, int64_t i, int64_t* total, int64_t* status) {
+  const int n = nlines(HQG_TPCH_LINEITEM, seed, i);
+  int64_t t = 0;
+  int nopen = 0;
+  for (int j = 0; j < n; ++j) {
+    TLine L(sf, seed, i, j);
+    t += L.extendedprice() * (100 + L.tax()) * (100 - L.discount()) / 10000;
+    nopen += L.shipday() > kCurrentDay;
+  }
+  *total = t;
+  *status = nopen == 0 ? 0 : (nopen == n ? 1 : 2);
 }
 
 void gen_lines(int table, double sf, uint64_t seed, int64_t a, int64_t b, const Out& o,
@@ -313,7 +357,12 @@ void gen_dim(int table, double sf, uint64_t seed, int64_t a, int64_t b, const Ou
           else if (c == O_CUSTKEY) v = uni(seed, S(table, O_CUSTKEY), (uint64_t)r, 1, scaled(150000.0, sf));
           else if (c == O_ORDERDATE)
             v = yyyymmdd((int32_t)uni(seed, S(table, O_ORDERDATE), (uint64_t)r, 0, kTpchODays - 1));
-          else v = 0;  // o_shippriority
+          else if (c == O_ORDERPRIORITY) { v = uni(seed, S(table, O_ORDERPRIORITY), (uint64_t)r, 0, 4); w = 1; }
+          else if (c == O_TOTALPRICE || c == O_ORDERSTATUS) {
+            int64_t tot, st;
+            order_lines(sf, seed, r, &tot, &st);
+            if (c == O_TOTALPRICE) { v = tot; w = 8; } else { v = st; w = 1; }
+          } else v = 0;  // o_shippriority
           break;
         case HQG_TPCH_CUSTOMER:
           if (c == TC_CUSTKEY) v = r + 1;
@@ -332,6 +381,21 @@ void gen_dim(int table, double sf, uint64_t seed, int64_t a, int64_t b, const Ou
           v = r;
           w = 1;
           break;
+        case HQG_TPCH_PART:
+          if (c == TP_PARTKEY) v = r + 1;
+          else if (c == TP_BRAND) {  // Brand#MN: M uniform 1..5, N uniform 1..5
+            v = uni(seed, S(table, TP_BRAND), (uint64_t)r, 0, 4) * 5 + uni(seed, S(table, 40), (uint64_t)r, 0, 4);
+            w = 1;
+          } else if (c == TP_CONTAINER) { v = uni(seed, S(table, TP_CONTAINER), (uint64_t)r, 0, 39); w = 1; }
+          else v = uni(seed, S(table, TP_SIZE), (uint64_t)r, 1, 50);
+          break;
+        case HQG_TPCH_PARTSUPP: {
+          const int64_t pk = r / 4 + 1;
+          if (c == PS_PARTKEY) v = pk;
+          else if (c == PS_SUPPKEY) v = TLine::ps_supplier(pk, r % 4, scaled(10000.0, sf));
+          else { v = uni(seed, S(table, PS_SUPPLYCOST), (uint64_t)r, 100, 100000); w = 8; }
+          break;
+        }
       }
       put(o, k, r, v, w);
     }
@@ -349,6 +413,8 @@ int64_t dim_rows(int table, double sf) {
     case HQG_TPCH_SUPPLIER: return scaled(10000.0, sf);
     case HQG_TPCH_NATION: return 25;
     case HQG_TPCH_REGION: return 5;
+    case HQG_TPCH_PART: return scaled(200000.0, sf);
+    case HQG_TPCH_PARTSUPP: return 4 * scaled(200000.0, sf);
   }
   return -1;
 }

@@ -39,7 +39,9 @@ enum {
   HQG_TPCH_CUSTOMER = 13,
   HQG_TPCH_SUPPLIER = 14,
   HQG_TPCH_NATION = 15,
-  HQG_TPCH_REGION = 16
+  HQG_TPCH_REGION = 16,
+  HQG_TPCH_PART = 17,
+  HQG_TPCH_PARTSUPP = 18
 };
 
 /* SSB lineorder columns (all int32) */
@@ -59,10 +61,20 @@ enum { P_PARTKEY = 0, P_MFGR, P_CATEGORY, P_BRAND1, P_NCOLS };
 /* TPC-H lineitem */
 enum {
   L_ORDERKEY = 0, L_PARTKEY, L_QUANTITY, L_EXTENDEDPRICE, L_DISCOUNT, L_TAX,
-  L_RETURNFLAG, L_LINESTATUS, L_SHIPDATE, L_RECEIPTDATE, L_LINENUMBER, L_SUPPKEY, L_NCOLS
+  L_RETURNFLAG, L_LINESTATUS, L_SHIPDATE, L_RECEIPTDATE, L_LINENUMBER, L_SUPPKEY,
+  L_COMMITDATE,   /* i32 yyyymmdd: o_orderdate + U[30, 90] (TPC-H 4.2.3) */
+  L_SHIPMODE,     /* i8 code of AIR, FOB, MAIL, RAIL, REG AIR, SHIP, TRUCK (uniform) */
+  L_SHIPINSTRUCT, /* i8 code of COLLECT COD, DELIVER IN PERSON, NONE, TAKE BACK RETURN (uniform) */
+  L_NCOLS
 };
 /* TPC-H orders */
-enum { O_ORDERKEY = 0, O_CUSTKEY, O_ORDERDATE, O_SHIPPRIORITY, O_NCOLS };
+enum {
+  O_ORDERKEY = 0, O_CUSTKEY, O_ORDERDATE, O_SHIPPRIORITY,
+  O_ORDERPRIORITY, /* i8 code of 1-URGENT .. 5-LOW (uniform) */
+  O_TOTALPRICE,    /* i64 cents: sum over the order's lines of l_extendedprice*(100+l_tax)*(100-l_discount)/10^4 */
+  O_ORDERSTATUS,   /* i8 code of F, O, P: all lines F / all lines O / mixed (TPC-H 4.2.3) */
+  O_NCOLS
+};
 /* TPC-H customer */
 enum { TC_CUSTKEY = 0, TC_MKTSEGMENT, TC_NATIONKEY, TC_NCOLS };
 /* TPC-H supplier (10 K * SF rows): suppkey i32, nationkey i8 (uniform over the 25 nations) */
@@ -71,6 +83,13 @@ enum { TS_SUPPKEY = 0, TS_NATIONKEY, TS_NCOLS };
 enum { N_NATIONKEY = 0, N_REGIONKEY, N_NCOLS };
 /* TPC-H region (5 rows): regionkey i8 = the name's dictionary code */
 enum { R_REGIONKEY = 0, R_NCOLS };
+/* TPC-H part (200 K * SF rows): partkey i32, brand i8 ('Brand#MN' = (M-1)*5 + N-1, M, N in 1..5),
+ * container i8 (code of the 40 'SIZE TYPE' strings in string order), size i32 (1..50) */
+enum { TP_PARTKEY = 0, TP_BRAND, TP_CONTAINER, TP_SIZE, TP_NCOLS };
+/* TPC-H partsupp (4 rows per part): partkey i32, suppkey i32 (TPC-H 4.2.3: the part's
+ * i-th supplier (partkey + i*(S/4 + (partkey-1)/S)) mod S + 1), supplycost i64 cents 100..100000.
+ * l_suppkey is one of its l_partkey's four suppliers, chosen uniformly. */
+enum { PS_PARTKEY = 0, PS_SUPPKEY, PS_SUPPLYCOST, PS_NCOLS };
 
 /* Number of rows of a table at scale factor sf (lineorder/lineitem count
  * the 1..7 lines of every order, computed once and cached). <0 on error. */

@@ -210,7 +210,12 @@ hq_status hq_free_hash(hq_hash* h);
 
 /* ------------------------------------------------------------------ plans */
 typedef enum { HQ_OP_FILTER = 1, HQ_OP_PROBE = 2, HQ_OP_COMPUTE = 3 } hq_op_kind;
-typedef enum { HQ_PROBE_INNER = 0, HQ_PROBE_SEMI = 1, HQ_PROBE_ANTI = 2 } hq_probe_mode;
+/* INNER: row survives on a match, payload words -> payload_dst temps.
+ * SEMI / ANTI: row survives on a match / on no match (EXISTS / NOT EXISTS).
+ * OUTER: LEFT OUTER JOIN: the row always survives; payload_dst temps get the
+ *        matching slot's payload words, or 0 when the key is absent
+ *        (COALESCE(payload, 0)); build keys are unique, so at most one match. */
+typedef enum { HQ_PROBE_INNER = 0, HQ_PROBE_SEMI = 1, HQ_PROBE_ANTI = 2, HQ_PROBE_OUTER = 3 } hq_probe_mode;
 /* Expression code: an accumulator machine evaluated per row in int64.
  * operand = register `reg`, or the immediate `imm` when reg < 0. */
 typedef enum {
@@ -220,7 +225,19 @@ typedef enum {
   HQ_I_RSUB,     /* acc = operand - acc      */
   HQ_I_MUL,      /* acc = acc * operand      */
   HQ_I_DIV,      /* acc = acc / operand (C truncation; /0 -> HQ_ERR_ARG) */
-  HQ_I_MOD       /* acc = acc % operand (C semantics; %0 -> HQ_ERR_ARG) */
+  HQ_I_MOD,      /* acc = acc % operand (C semantics; %0 -> HQ_ERR_ARG) */
+  /* Predicate instructions (boolean acc, 0/1): acc = (acc != 0 && reg CMP imm).
+   * They read BOTH fields: reg (>= 0, a column or temp) and the constant imm, so a
+   * conjunction over several registers is one expression (e.g. one disjunct of
+   * TPC-H Q19's WHERE clause). */
+  HQ_I_AND_EQ,   /* acc = acc && reg == imm */
+  HQ_I_AND_NE,   /* acc = acc && reg != imm */
+  HQ_I_AND_LT,   /* acc = acc && reg <  imm */
+  HQ_I_AND_LE,   /* acc = acc && reg <= imm */
+  HQ_I_AND_GT,   /* acc = acc && reg >  imm */
+  HQ_I_AND_GE,   /* acc = acc && reg >= imm */
+  HQ_I_AND_IN,   /* acc = acc && 0 <= reg < 64 && bit reg of (uint64)imm (IN-list over codes < 64) */
+  HQ_I_OR        /* acc = acc || operand != 0 (disjunction with another predicate temp) */
 } hq_opcode;
 typedef struct {
   int32_t opc;

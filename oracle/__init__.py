@@ -63,12 +63,19 @@ class _Part(ctypes.Structure):
 class _Lineitem(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("orderkey", P_I32), ("quantity", P_I64),
                 ("extendedprice", P_I64), ("discount", P_I64), ("tax", P_I64),
-                ("returnflag", P_I8), ("linestatus", P_I8), ("shipdate", P_I32), ("suppkey", P_I32)]
+                ("returnflag", P_I8), ("linestatus", P_I8), ("shipdate", P_I32), ("suppkey", P_I32),
+                ("partkey", P_I32), ("commitdate", P_I32), ("receiptdate", P_I32),
+                ("shipmode", P_I8), ("shipinstruct", P_I8)]
 
 
 class _Orders(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("orderkey", P_I32), ("custkey", P_I32),
-                ("orderdate", P_I32), ("shippriority", P_I32)]
+                ("orderdate", P_I32), ("shippriority", P_I32), ("orderpriority", P_I8),
+                ("totalprice", P_I64), ("orderstatus", P_I8)]
+
+
+class _TPart(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("partkey", P_I32), ("brand", P_I8), ("container", P_I8), ("size", P_I32)]
 
 
 class _TCustomer(ctypes.Structure):
@@ -130,6 +137,12 @@ def lib():
             "orc_ssb_q31_mat": [P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
             "orc_ssb_q41": [P(_Lineorder), P(_Date), P(_SsbDim), P(_SsbDim), P(_Part), ctypes.c_int, ctypes.c_int],
             "orc_tpch_q3": [P(_TCustomer), P(_Orders), P(_Lineitem), ctypes.c_int, ctypes.c_int],
+            "orc_tpch_q4": [P(_Orders), P(_Lineitem), ctypes.c_int, ctypes.c_int],
+            "orc_tpch_q13": [P(_TCustomer), P(_Orders), ctypes.c_int],
+            "orc_tpch_q17": [P(_TPart), P(_Lineitem), ctypes.c_int],
+            "orc_tpch_q18": [P(_TCustomer), P(_Orders), P(_Lineitem), ctypes.c_int],
+            "orc_tpch_q19": [P(_TPart), P(_Lineitem), ctypes.c_int, ctypes.c_int],
+            "orc_tpch_q21": [ctypes.c_int, P(_TSupplier), P(_Orders), P(_Lineitem), P(_Nation), ctypes.c_int],
             "orc_tpch_q7": [P(_TCustomer), P(_Orders), P(_Lineitem), P(_TSupplier), P(_Nation),
                             ctypes.c_int, ctypes.c_int],
             "orc_tpch_q10": [P(_TCustomer), P(_Orders), P(_Lineitem), P(_Nation), ctypes.c_int, ctypes.c_int],
@@ -212,6 +225,10 @@ def _lineitem(t, keep):
     s.linestatus = _ptr(t.get("l_linestatus"), P_I8, keep)
     s.shipdate = _ptr(t.get("l_shipdate"), P_I32, keep)
     s.suppkey = _ptr(t.get("l_suppkey"), P_I32, keep)
+    for f in ("partkey", "commitdate", "receiptdate"):
+        setattr(s, f, _ptr(t.get("l_" + f), P_I32, keep))
+    s.shipmode = _ptr(t.get("l_shipmode"), P_I8, keep)
+    s.shipinstruct = _ptr(t.get("l_shipinstruct"), P_I8, keep)
     return s
 
 
@@ -220,6 +237,19 @@ def _orders(t, keep):
     s.n = _n(t)
     for f in ("orderkey", "custkey", "orderdate", "shippriority"):
         setattr(s, f, _ptr(t.get("o_" + f), P_I32, keep))
+    s.orderpriority = _ptr(t.get("o_orderpriority"), P_I8, keep)
+    s.totalprice = _ptr(t.get("o_totalprice"), P_I64, keep)
+    s.orderstatus = _ptr(t.get("o_orderstatus"), P_I8, keep)
+    return s
+
+
+def _tpart(t, keep):
+    s = _TPart()
+    s.n = _n(t)
+    s.partkey = _ptr(t["p_partkey"], P_I32, keep)
+    s.brand = _ptr(t.get("p_brand"), P_I8, keep)
+    s.container = _ptr(t.get("p_container"), P_I8, keep)
+    s.size = _ptr(t.get("p_size"), P_I32, keep)
     return s
 
 
@@ -377,6 +407,52 @@ def tpch_q7(customer, orders, lineitem, supplier, nation, brute=False, nthreads=
                                  ctypes.byref(_lineitem(lineitem, keep)), ctypes.byref(_tsupp(supplier, keep)),
                                  ctypes.byref(_nation(nation, keep)), int(brute), nthreads],
                  ["supp_nation", "cust_nation", "l_year", "revenue", "count"])
+
+
+def tpch_q4(orders, lineitem, brute=False, nthreads=1) -> OracleResult:
+    """TPC-H Q4 -> [o_orderpriority, order_count] ORDER BY o_orderpriority."""
+    keep = []
+    return _call("orc_tpch_q4", [ctypes.byref(_orders(orders, keep)), ctypes.byref(_lineitem(lineitem, keep)),
+                                 int(brute), nthreads], ["o_orderpriority", "order_count"])
+
+
+def tpch_q13(customer, orders, brute=False) -> OracleResult:
+    """TPC-H Q13 (App F: no LIKE) -> [c_count, custdist] ORDER BY custdist desc, c_count desc."""
+    keep = []
+    return _call("orc_tpch_q13", [ctypes.byref(_tcust(customer, keep)), ctypes.byref(_orders(orders, keep)),
+                                  int(brute)], ["c_count", "custdist"])
+
+
+def tpch_q17(part, lineitem, brute=False) -> OracleResult:
+    """TPC-H Q17 (unnested) -> 1 row [sum_extendedprice (cents), count]; avg_yearly = sum / 7.0."""
+    keep = []
+    return _call("orc_tpch_q17", [ctypes.byref(_tpart(part, keep)), ctypes.byref(_lineitem(lineitem, keep)),
+                                  int(brute)], ["sum_extendedprice", "count"])
+
+
+def tpch_q18(customer, orders, lineitem, brute=False) -> OracleResult:
+    """TPC-H Q18 -> [c_custkey, o_orderkey, o_orderdate, o_totalprice, sum_qty, count]
+    ORDER BY o_totalprice desc, o_orderdate, o_orderkey (full result)."""
+    keep = []
+    return _call("orc_tpch_q18", [ctypes.byref(_tcust(customer, keep)), ctypes.byref(_orders(orders, keep)),
+                                  ctypes.byref(_lineitem(lineitem, keep)), int(brute)],
+                 ["c_custkey", "o_orderkey", "o_orderdate", "o_totalprice", "sum_qty", "count"])
+
+
+def tpch_q19(part, lineitem, brute=False, nthreads=1) -> OracleResult:
+    """TPC-H Q19 -> 1 row [revenue (scale 4), count]."""
+    keep = []
+    return _call("orc_tpch_q19", [ctypes.byref(_tpart(part, keep)), ctypes.byref(_lineitem(lineitem, keep)),
+                                  int(brute), nthreads], ["revenue", "count"])
+
+
+def tpch_q21(supplier, orders, lineitem, nation, variant=0, brute=False) -> OracleResult:
+    """TPC-H Q21 -> [s_suppkey, numwait] ORDER BY numwait desc, s_suppkey (full result);
+    variant 1 = PAPER.md App F's EXISTS in place of NOT EXISTS."""
+    keep = []
+    return _call("orc_tpch_q21", [int(variant), ctypes.byref(_tsupp(supplier, keep)),
+                                  ctypes.byref(_orders(orders, keep)), ctypes.byref(_lineitem(lineitem, keep)),
+                                  ctypes.byref(_nation(nation, keep)), int(brute)], ["s_suppkey", "numwait"])
 
 
 def tpch_q10(customer, orders, lineitem, nation, brute=False, nthreads=1) -> OracleResult:

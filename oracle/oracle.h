@@ -56,8 +56,18 @@ typedef struct {
   const int8_t *returnflag, *linestatus;
   const int32_t* shipdate;
   const int32_t* suppkey;
+  const int32_t *partkey, *commitdate, *receiptdate;
+  const int8_t *shipmode, *shipinstruct;
 } orc_lineitem;
-typedef struct { int64_t n; const int32_t *orderkey, *custkey, *orderdate, *shippriority; } orc_orders;
+typedef struct {
+  int64_t n;
+  const int32_t *orderkey, *custkey, *orderdate, *shippriority;
+  const int8_t* orderpriority;
+  const int64_t* totalprice;
+  const int8_t* orderstatus;
+} orc_orders;
+/* TPC-H part: brand 'Brand#MN' = (M-1)*5 + N-1; container = code in string order (hqgen) */
+typedef struct { int64_t n; const int32_t* partkey; const int8_t *brand, *container; const int32_t* size; } orc_tpch_part;
 typedef struct { int64_t n; const int32_t* custkey; const int8_t *mktsegment, *nationkey; } orc_tpch_customer;
 typedef struct { int64_t n; const int32_t* suppkey; const int8_t* nationkey; } orc_tpch_supplier;
 typedef struct { int64_t n; const int8_t *nationkey, *regionkey; } orc_nation;
@@ -127,6 +137,28 @@ int orc_micro_sum(const orc_lineorder* lo, int32_t x, int nthreads, orc_result* 
 /* Fig 26: select sum(lo_extendedprice), lo_orderkey % x group by lo_orderkey % x
  * -> rows [lo_orderkey % x, sum, count] ORDER BY key */
 int orc_micro_groupby(const orc_lineorder* lo, int32_t x, int nthreads, orc_result* out);
+
+/* TPC-H Q4 (order priority checking) -> rows [o_orderpriority, order_count] ORDER BY
+ * o_orderpriority; qualifying = orders counted */
+int orc_tpch_q4(const orc_orders* o, const orc_lineitem* li, int brute, int nthreads, orc_result* out);
+/* TPC-H Q13 without the o_comment LIKE (App F) -> rows [c_count,
+ * custdist] ORDER BY custdist desc, c_count desc; qualifying = customers */
+int orc_tpch_q13(const orc_tpch_customer* c, const orc_orders* o, int brute, orc_result* out);
+/* TPC-H Q17, the correlated subquery unnested (App F) -> 1 row [sum_extendedprice
+ * (cents), count]; avg_yearly = sum_extendedprice / 7.0 (R19) */
+int orc_tpch_q17(const orc_tpch_part* p, const orc_lineitem* li, int brute, orc_result* out);
+/* TPC-H Q18 (large volume customer) -> rows [c_custkey, o_orderkey, o_orderdate, o_totalprice,
+ * sum_qty (scale 2), count] ORDER BY o_totalprice desc, o_orderdate, o_orderkey (full result;
+ * the caller applies LIMIT 100); c_name depends on c_custkey (R18) */
+int orc_tpch_q18(const orc_tpch_customer* c, const orc_orders* o, const orc_lineitem* li, int brute,
+                 orc_result* out);
+/* TPC-H Q19 (discounted revenue) -> 1 row [revenue (scale 4), count] */
+int orc_tpch_q19(const orc_tpch_part* p, const orc_lineitem* li, int brute, int nthreads, orc_result* out);
+/* TPC-H Q21 (suppliers who kept orders waiting; variant 0: the TPC-H text, the third
+ * subquery NOT EXISTS; variant 1: PAPER.md App F's EXISTS) -> rows
+ * [s_suppkey, numwait] ORDER BY numwait desc, s_suppkey (s_name depends on s_suppkey, R18) */
+int orc_tpch_q21(int variant, const orc_tpch_supplier* s, const orc_orders* o, const orc_lineitem* li,
+                 const orc_nation* n, int brute, orc_result* out);
 
 void orc_free(orc_result* r);
 

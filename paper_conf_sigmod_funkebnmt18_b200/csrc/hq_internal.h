@@ -13,6 +13,28 @@
 
 #include "hq.h"
 
+// probes whose payload words reach registers (INNER, and OUTER with 0 on a miss)
+__host__ __device__ inline bool hq_probe_has_payload(int mode) {
+  return mode == HQ_PROBE_INNER || mode == HQ_PROBE_OUTER;
+}
+
+// predicate instructions of the expression machine (hq.h HQ_I_AND_* / HQ_I_OR):
+// acc is boolean, o the register operand (OR: register or immediate), imm the constant
+__host__ __device__ inline long long hq_pred_insn(int opc, long long acc, long long o, long long imm) {
+  bool c;
+  switch (opc) {
+    case HQ_I_AND_EQ: c = o == imm; break;
+    case HQ_I_AND_NE: c = o != imm; break;
+    case HQ_I_AND_LT: c = o < imm; break;
+    case HQ_I_AND_LE: c = o <= imm; break;
+    case HQ_I_AND_GT: c = o > imm; break;
+    case HQ_I_AND_GE: c = o >= imm; break;
+    case HQ_I_AND_IN: c = o >= 0 && o < 64 && (((unsigned long long)imm >> o) & 1ull); break;
+    default: return (acc != 0 || o != 0) ? 1 : 0;  // HQ_I_OR
+  }
+  return (acc != 0 && c) ? 1 : 0;
+}
+
 // ---------------------------------------------------------------- errors
 struct HqError {
   hq_status code;

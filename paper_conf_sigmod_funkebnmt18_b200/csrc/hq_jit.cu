@@ -196,13 +196,20 @@ struct Gen {
   }
   static std::string pv(int i, const char* what) { return "p" + std::to_string(i) + what; }
   void probe_defs(const KProbe& pr) {
-    const int npay = pr.mode == HQ_PROBE_INNER ? pr.npay : 0;
+    const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
+    const bool outer = pr.mode == HQ_PROBE_OUTER;  // a miss leaves 0
     for (int k = 0; k < npay; ++k) {
-      o << "      int " << var(pr.dst[k]) << "[R];\n";
-      if (k == 0 && pr.pay_min <= pr.pay_max) known[pr.dst[0]] = {pr.pay_min, pr.pay_max};
+      o << "      int " << var(pr.dst[k]) << (outer ? "[R] = {};\n" : "[R];\n");
+      if (k == 0 && pr.pay_min <= pr.pay_max)
+        known[pr.dst[0]] = {outer ? std::min(pr.pay_min, 0) : pr.pay_min, outer ? std::max(pr.pay_max, 0) : pr.pay_max};
       loaded.insert(pr.dst[k]);
       vtype[pr.dst[k]] = "int";
     }
+  }
+  static const char* mask_after(const KProbe& pr) {
+    if (pr.mode == HQ_PROBE_ANTI) return "mask & ~found_";
+    if (pr.mode == HQ_PROBE_OUTER) return "mask; (void)found_";
+    return "mask & found_";
   }
   void probe_addr(const KProbe& pr, int i) {
     const std::string key = val(pr.key_reg);
@@ -245,7 +252,7 @@ struct Gen {
   }
   void probe_resolve(const KProbe& pr, int i) {
     const std::string D = pv(i, "d_"), M = pv(i, "m_"), V = pv(i, "v_");
-    const int npay = pr.mode == HQ_PROBE_INNER ? pr.npay : 0;
+    const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
     o << "      { u32 found_ = 0u;\n#pragma unroll\n        for (int r = 0; r < R; ++r) if ((" << M << " >> r) & 1u) {";
     if (access(pr) == AK_DIRECT) {
       static const char* comp[3] = {"y", "z", "w"};
@@ -261,14 +268,14 @@ struct Gen {
       if (npay > 0) o << " " << var(pr.dst[0]) << "[r] = (int)b_ + (" << pr.pay_min << ");";
       o << " }";
     }
-    o << " }\n        mask = " << (pr.mode == HQ_PROBE_ANTI ? "mask & ~found_" : "mask & found_") << "; }\n";
+    o << " }\n        mask = " << mask_after(pr) << "; }\n";
   }
 
   // linear-probing table (sparse keys): optional exact key-range bitmap, then
   // 16-B group scans until the key or an empty slot
   void probe_linear(const KProbe& pr, int idx) {
     const int W = pr.words;
-    const int npay = pr.mode == HQ_PROBE_INNER ? pr.npay : 0;
+    const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
     probe_defs(pr);
     const std::string key = val(pr.key_reg);
     o << "      { const u32* ht_ = p.ht[" << idx << "]; u32 found_ = 0u; int kk_[R]; u32 pend_ = 0u; u32 pos_[R];\n"
@@ -304,7 +311,7 @@ struct Gen {
     o << "            } else if (stop_) pend_ &= ~(1u << r);\n"
       << "            else pos_[r] = ((pos_[r] / " << G << " + 1) * " << G << ") & " << pr.mask << "u;\n"
       << "          }\n        }\n";
-    o << "        mask = " << (pr.mode == HQ_PROBE_ANTI ? "mask & ~found_" : "mask & found_") << "; }\n";
+    o << "        mask = " << mask_after(pr) << "; }\n";
   }
 
   // ops [i, end): one probe batch starting at op i (see probe_addr)
@@ -320,12 +327,12 @@ struct Gen {
     if (ak != AK_SMEM) {  // a global probe: the following independent global probes join its batch
       // (no early exit in front: the warp rarely has no live row here, and the
       // extra branch measured slower)
-      std::set<int> defs(first.dst, first.dst + (first.mode == HQ_PROBE_INNER ? first.npay : 0));
+      std::set<int> defs(first.dst, first.dst + (hq_probe_has_payload(first.mode) ? first.npay : 0));
       for (int j = i + 1; j < kp.nops && kp.ops[j].kind == OP_PROBE && !kp.op_skip[j]; ++j) {
         const KProbe& pr = kp.probes[kp.ops[j].idx];
         if (access(pr) == AK_LINEAR || access(pr) == AK_SMEM || defs.count(pr.key_reg)) break;
         b.push_back(j);
-        for (int k = 0; k < (pr.mode == HQ_PROBE_INNER ? pr.npay : 0); ++k) defs.insert(pr.dst[k]);
+        for (int k = 0; k < (hq_probe_has_payload(pr.mode) ? pr.npay : 0); ++k) defs.insert(pr.dst[k]);
       }
     }
     for (int j : b) probe_defs(kp.probes[kp.ops[j].idx]);
@@ -354,6 +361,16 @@ struct Gen {
         case HQ_I_SUB: o << "        a_ -= " << x << ";\n"; break;
         case HQ_I_RSUB: o << "        a_ = " << x << " - a_;\n"; break;
         case HQ_I_MUL: o << "        a_ *= " << x << ";\n"; break;
+        case HQ_I_AND_EQ: case HQ_I_AND_NE: case HQ_I_AND_LT: case HQ_I_AND_LE: case HQ_I_AND_GT: case HQ_I_AND_GE: {
+          static const char* cmp[6] = {"==", "!=", "<", "<=", ">", ">="};
+          o << "        a_ = (a_ != 0 && " << x << " " << cmp[in.opc - HQ_I_AND_EQ] << " " << lit(in.imm) << ") ? 1 : 0;\n";
+          break;
+        }
+        case HQ_I_AND_IN:
+          o << "        { const long long v_ = " << x << "; a_ = (a_ != 0 && v_ >= 0 && v_ < 64 && ((" << (unsigned long long)in.imm
+            << "ULL >> v_) & 1ull)) ? 1 : 0; }\n";
+          break;
+        case HQ_I_OR: o << "        a_ = (a_ != 0 || " << x << " != 0) ? 1 : 0;\n"; break;
         default:
           o << "        { const long long d_ = " << x << "; if (d_ == 0) { if ((mask >> r) & 1u) atomicOr(p.err, F_DIV_ZERO); a_ = 0; }"
             << " else a_ = a_ " << (in.opc == HQ_I_DIV ? "/" : "%") << " d_; }\n";

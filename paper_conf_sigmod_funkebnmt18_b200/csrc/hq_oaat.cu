@@ -81,7 +81,7 @@ __global__ void hq_oaat_probe(const char* key, int w, KProbe pr, long long n, in
         }
       }
     }
-    flags[i] = pr.mode == HQ_PROBE_ANTI ? !hit : hit;
+    flags[i] = pr.mode == HQ_PROBE_ANTI ? !hit : (pr.mode == HQ_PROBE_OUTER ? 1 : hit);  // OUTER: payload 0 on a miss
     if (pr.npay > 0) p0[i] = pay[0];
     if (pr.npay > 1) p1[i] = pay[1];
     if (pr.npay > 2) p2[i] = pay[2];
@@ -118,6 +118,8 @@ __global__ void hq_oaat_compute(KInsn const* __restrict__ code, int ninsn, KIn i
         case HQ_I_SUB: acc -= o; break;
         case HQ_I_RSUB: acc = o - acc; break;
         case HQ_I_MUL: acc *= o; break;
+        case HQ_I_AND_EQ: case HQ_I_AND_NE: case HQ_I_AND_LT: case HQ_I_AND_LE: case HQ_I_AND_GT: case HQ_I_AND_GE:
+        case HQ_I_AND_IN: case HQ_I_OR: acc = hq_pred_insn(c[k].opc, acc, o, c[k].imm); break;
         default:
           if (o == 0) { atomicOr(err, HQF_DIV_ZERO); acc = 0; }
           else acc = c[k].opc == HQ_I_DIV ? acc / o : acc % o;

@@ -189,10 +189,18 @@ __device__ __forceinline__ uint32_t probe_rows(const KPlan& p, const KProbe& pr,
       pos[r] = ((uint32_t)(int)kv[r] * 0x9E3779B1u) >> (32u - pr.log2cap);
     }
   }
-  const bool inner = pr.mode == HQ_PROBE_INNER;
+  const bool inner = hq_probe_has_payload(pr.mode);
   int* dst0 = (int*)(tmp + p.regs[pr.dst[0]].off) + row0;
   int* dst1 = (int*)(tmp + p.regs[pr.dst[W > 2 ? 1 : 0]].off) + row0;
   int* dst2 = (int*)(tmp + p.regs[pr.dst[W > 2 ? 2 : 0]].off) + row0;
+  if (W > 1 && pr.mode == HQ_PROBE_OUTER) {  // LEFT OUTER: a miss leaves payload 0
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (pr.npay > 0) dst0[r * 32] = 0;
+      if (W > 2 && pr.npay > 1) dst1[r * 32] = 0;
+      if (W > 2 && pr.npay > 2) dst2[r * 32] = 0;
+    }
+  }
   constexpr int G = W == 1 ? 4 : (W == 2 ? 2 : 1);  // slots per 16-B group
   while (pending) {
     int4 sl[R];
@@ -248,6 +256,7 @@ __device__ __forceinline__ uint32_t probe_rows(const KPlan& p, const KProbe& pr,
     }
   }
   if (pr.mode == HQ_PROBE_ANTI) return mask & ~found;
+  if (pr.mode == HQ_PROBE_OUTER) return mask;
   return mask & found;
 }
 
@@ -301,6 +310,11 @@ __device__ __forceinline__ void op_compute(const KPlan& p, int idx, const char* 
       case HQ_I_MUL:
 #pragma unroll
         for (int r = 0; r < R; ++r) acc[r] *= o[r];
+        break;
+      case HQ_I_AND_EQ: case HQ_I_AND_NE: case HQ_I_AND_LT: case HQ_I_AND_LE: case HQ_I_AND_GT: case HQ_I_AND_GE:
+      case HQ_I_AND_IN: case HQ_I_OR:
+#pragma unroll
+        for (int r = 0; r < R; ++r) acc[r] = hq_pred_insn(in.opc, acc[r], o[r], in.imm);
         break;
       default: {  // DIV / MOD
         bool bad = false;

@@ -120,7 +120,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     } else if (op.kind == HQ_OP_PROBE) {
       if (nprobe >= MAX_PROBES) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: too many probes");
       if (!op.ht) HQ_THROW(HQ_ERR_ARG, "plan: probe without hash table");
-      if (op.mode < HQ_PROBE_INNER || op.mode > HQ_PROBE_ANTI) HQ_THROW(HQ_ERR_ARG, "plan: bad probe mode");
+      if (op.mode < HQ_PROBE_INNER || op.mode > HQ_PROBE_OUTER) HQ_THROW(HQ_ERR_ARG, "plan: bad probe mode");
       KProbe& pr = kp.probes[nprobe];
       pr.key_reg = (int16_t)use(op.key_reg, "probe key");
       pr.slots = op.ht->slots;
@@ -137,7 +137,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         const double range = (double)op.ht->meta.key_max - (double)op.ht->meta.key_min + 1.0;
         double est = (op.ht->meta.nkeys >= 0 && range >= 1.0) ? (double)op.ht->meta.nkeys / range : 1.0;
         est = est > 1.0 ? 1.0 : est;
-        pr.pass_est = (float)(op.mode == HQ_PROBE_ANTI ? 1.0 - est : est);
+        pr.pass_est = (float)(op.mode == HQ_PROBE_ANTI ? 1.0 - est : (op.mode == HQ_PROBE_OUTER ? 1.0 : est));
       }
       pr.cbytes = (uint32_t)op.ht->cbytes;
       pr.smem_off = 0;
@@ -146,7 +146,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.pf_range = (uint32_t)((int64_t)op.ht->meta.key_max - op.ht->meta.key_min + 1);
       pr.words = (uint8_t)op.ht->meta.slot_words;
       pr.mode = (uint8_t)op.mode;
-      const int npay = op.mode == HQ_PROBE_INNER ? op.npayload : 0;
+      const int npay = hq_probe_has_payload(op.mode) ? op.npayload : 0;
       if (npay < 0 || npay > op.ht->meta.npayload) HQ_THROW(HQ_ERR_ARG, "plan: probe asks for more payload words than the table holds");
       pr.npay = (uint8_t)npay;
       for (int k = 0; k < npay; ++k) pr.dst[k] = (int16_t)def(op.payload_dst[k], 4, "probe payload");
@@ -161,7 +161,9 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       c.n = (uint8_t)op.ninsn;
       for (int k = 0; k < op.ninsn; ++k) {
         const hq_insn& in = op.code[k];
-        if (in.opc < HQ_I_LOAD || in.opc > HQ_I_MOD) HQ_THROW(HQ_ERR_ARG, "plan: bad opcode");
+        if (in.opc < HQ_I_LOAD || in.opc > HQ_I_OR) HQ_THROW(HQ_ERR_ARG, "plan: bad opcode");
+        if (in.opc >= HQ_I_AND_EQ && in.opc <= HQ_I_AND_IN && in.reg < 0)
+          HQ_THROW(HQ_ERR_ARG, "plan: predicate instruction needs a register operand");
         KInsn& ki = kp.insns[ninsn++];
         ki.opc = (uint8_t)in.opc;
         ki.reg = in.reg < 0 ? (int16_t)-1 : (int16_t)use(in.reg, "expression");
@@ -395,7 +397,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       } else if (op.kind == OP_PROBE) {
         const KProbe& pr = kp.probes[op.idx];
         exec = mp_pass == 1;
-        for (int k = 0; mp_pass == 2 && pr.mode == HQ_PROBE_INNER && k < pr.npay; ++k) exec = exec || need[pr.dst[k]];
+        for (int k = 0; mp_pass == 2 && hq_probe_has_payload(pr.mode) && k < pr.npay; ++k) exec = exec || need[pr.dst[k]];
         if (exec) need[pr.key_reg] = true;
       } else {
         const KCompute& c = kp.comps[op.idx];

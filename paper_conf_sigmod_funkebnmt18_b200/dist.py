@@ -112,8 +112,8 @@ class DistributedEngine(Engine):
         hs = super().hashes(specs) if self.rank == self.root else [None] * len(specs)
         return [self._share(h) for h in hs]
 
-    def hash_from(self, res, names, key, payload=()) -> hq.Hash:
-        h = super().hash_from(res, names, key, payload) if self.rank == self.root else None
+    def hash_from(self, res, names, key, payload=(), preds=()) -> hq.Hash:
+        h = super().hash_from(res, names, key, payload, preds) if self.rank == self.root else None
         return self._share(h)
 
     @staticmethod

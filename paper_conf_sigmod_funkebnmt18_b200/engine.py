@@ -18,7 +18,8 @@ import numpy as np
 from . import hq
 
 _OPC = {"load": hq.I_LOAD, "add": hq.I_ADD, "sub": hq.I_SUB, "rsub": hq.I_RSUB, "mul": hq.I_MUL,
-        "div": hq.I_DIV, "mod": hq.I_MOD}
+        "div": hq.I_DIV, "mod": hq.I_MOD, "and_eq": hq.I_AND_EQ, "and_ne": hq.I_AND_NE, "and_lt": hq.I_AND_LT,
+        "and_le": hq.I_AND_LE, "and_gt": hq.I_AND_GT, "and_ge": hq.I_AND_GE, "and_in": hq.I_AND_IN, "or": hq.I_OR}
 _AGG = {"sum": hq.AGG_SUM, "count": hq.AGG_COUNT, "min": hq.AGG_MIN, "max": hq.AGG_MAX, "avg": hq.AGG_AVG}
 _TYPES = {"i8": hq.HQ_I8, "i32": hq.HQ_I32, "i64": hq.HQ_I64}
 
@@ -70,7 +71,7 @@ class PlanBuilder:
         op.kind = hq.OP_PROBE
         op.ht = ht.h
         op.key_reg = self.reg(key)
-        op.mode = {"inner": hq.PROBE_INNER, "semi": hq.PROBE_SEMI, "anti": hq.PROBE_ANTI}[mode]
+        op.mode = {"inner": hq.PROBE_INNER, "semi": hq.PROBE_SEMI, "anti": hq.PROBE_ANTI, "outer": hq.PROBE_OUTER}[mode]
         op.npayload = len(payload)
         for i, name in enumerate(payload):
             op.payload_dst[i] = self._new_tmp(name)
@@ -78,16 +79,29 @@ class PlanBuilder:
         return self
 
     def compute(self, dst: str, code: Sequence[Tuple[str, object]]) -> "PlanBuilder":
-        """code: accumulator-machine program, e.g. [("load","a"), ("rsub",100), ("mul","b")]."""
+        """code: accumulator-machine program, e.g. [("load","a"), ("rsub",100), ("mul","b")].
+        Predicate instructions name a register and a constant: ("and_le", "p_size", 5),
+        ("and_in", "p_container", [codes...]) (a conjunction; "or" joins a predicate temp)."""
         op = self._op()
         op.kind = hq.OP_COMPUTE
         if len(code) > hq.MAX_INSN:
             raise ValueError("expression too long")
         op.ninsn = len(code)
-        for i, (opc, arg) in enumerate(code):
+        for i, (opc, arg, *const) in enumerate(code):
             ins = op.code[i]
             ins.opc = _OPC[opc]
-            if isinstance(arg, str):
+            if const:  # predicate instruction: register arg, constant (or IN-list) const[0]
+                c = const[0]
+                if opc == "and_in":
+                    m = 0
+                    for v in c:
+                        if not 0 <= int(v) < 64:
+                            raise ValueError("and_in values must be codes 0..63")
+                        m |= 1 << int(v)
+                    c = m - (1 << 64) if m >= (1 << 63) else m
+                ins.reg = self.reg(arg)
+                ins.imm = int(c)
+            elif isinstance(arg, str):
                 ins.reg = self.reg(arg)
             else:
                 ins.reg = -1
@@ -201,10 +215,12 @@ class Engine:
         return self.ctx.build_hashes(out)
 
     def hash_from(self, res: Optional[hq.Result], names: Sequence[str], key: str,
-                  payload: Sequence[str] = ()) -> hq.Hash:
-        """Build a hash table from a materialised pipeline result (pipeline breaker)."""
+                  payload: Sequence[str] = (), preds: Sequence[Tuple] = ()) -> hq.Hash:
+        """Build a hash table from a materialised (or aggregated) pipeline result
+        (pipeline breaker); preds filter its rows (e.g. a HAVING clause)."""
         t = res.as_table(list(names))
-        return self.ctx.build_hash(t, t.col(key), [t.col(c) for c in payload])
+        ps = [hq.make_pred(t.col(p[0]), *p[1:]) for p in preds]
+        return self.ctx.build_hash(t, t.col(key), [t.col(c) for c in payload], ps)
 
     def run(self, pb: PlanBuilder, partitioned: bool = True) -> Optional[hq.Result]:
         P = pb.plan

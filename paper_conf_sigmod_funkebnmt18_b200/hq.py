@@ -26,8 +26,9 @@ MAX_OUT, MAX_TMP, MAX_INSN, MAX_PREDS, MAX_ORDER = 8, 8, 16, 8, 4
 HQ_HOST_COPY, HQ_DEVICE_BORROW = 1, 2
 EQ, NE, LT, LE, GT, GE, BETWEEN, IN_BITMAP = 1, 2, 3, 4, 5, 6, 7, 8
 OP_FILTER, OP_PROBE, OP_COMPUTE = 1, 2, 3
-PROBE_INNER, PROBE_SEMI, PROBE_ANTI = 0, 1, 2
+PROBE_INNER, PROBE_SEMI, PROBE_ANTI, PROBE_OUTER = 0, 1, 2, 3
 I_LOAD, I_ADD, I_SUB, I_RSUB, I_MUL, I_DIV, I_MOD = 1, 2, 3, 4, 5, 6, 7
+I_AND_EQ, I_AND_NE, I_AND_LT, I_AND_LE, I_AND_GT, I_AND_GE, I_AND_IN, I_OR = 8, 9, 10, 11, 12, 13, 14, 15
 AGG_SUM, AGG_COUNT, AGG_MIN, AGG_MAX, AGG_AVG = 1, 2, 3, 4, 5
 SINK_AGG, SINK_MATERIALISE = 1, 2
 RES_LRGP, RES_ATOMIC = 0, 1

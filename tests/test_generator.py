@@ -26,7 +26,7 @@ def test_deterministic(table):
         assert any(not np.array_equal(a[k], c[k]) for k in a)
 
 
-@pytest.mark.parametrize("table", ["lineorder", "lineitem", "orders", "tpch_customer", "supplier"])
+@pytest.mark.parametrize("table", ["lineorder", "lineitem", "orders", "tpch_customer", "supplier", "tpch_part", "partsupp"])
 def test_partition_invariance(table):
     full = hqgen.generate(table, 0.01)
     n = hqgen.table_rows(table, 0.01)
@@ -138,3 +138,40 @@ def test_tpch_lineitem_rules():
     assert abs(share[0] - 0.246) < 0.02 and abs(share[4] - 0.246) < 0.02   # A/F, R/F
     assert abs(share[3] - 0.487) < 0.03                                     # N/O
     assert share[2] < 0.03                                                  # N/F
+
+
+def test_tpch_derived_columns():
+    """Columns of the TPC-H Q4/Q9/Q13/Q17/Q18/Q19/Q21 plans (TPC-H 4.2.3 rules as
+    DESIGN.md §3 states them), checked against the lines with pandas."""
+    import pandas as pd
+    sf = 0.05
+    li = pd.DataFrame(hqgen.generate("lineitem", sf))
+    o = pd.DataFrame(hqgen.generate("orders", sf))
+    p = pd.DataFrame(hqgen.generate("tpch_part", sf))
+    ps = pd.DataFrame(hqgen.generate("partsupp", sf))
+    ns = hqgen.table_rows("tpch_supplier", sf)
+    to_day = lambda v: (pd.to_datetime(v.astype(str), format="%Y%m%d") - pd.Timestamp(EPOCH)).dt.days
+    j = li.merge(o, left_on="l_orderkey", right_on="o_orderkey")
+    d = to_day(j.l_commitdate) - to_day(j.o_orderdate)
+    assert d.min() == 30 and d.max() == 90
+    # o_totalprice = sum of the lines' extendedprice * (1 + tax) * (1 - discount), per line in cents
+    j = j.assign(charge=j.l_extendedprice * (100 + j.l_tax) * (100 - j.l_discount) // 10000,
+                 open=(j.l_linestatus == 1).astype(int), one=1)
+    g = j.groupby("o_orderkey").agg(tp=("charge", "sum"), op=("open", "sum"), n=("one", "sum"),
+                                    o_totalprice=("o_totalprice", "first"), st=("o_orderstatus", "first"))
+    assert (g.tp == g.o_totalprice).all()
+    exp = np.where(g.op == 0, 0, np.where(g.op == g.n, 1, 2))            # F, O, P
+    assert (g.st.values == exp).all()
+    assert len(g) == len(o)                                             # every order has lines
+    assert set(o.o_orderpriority) == set(range(5)) and set(li.l_shipmode) == set(range(7))
+    assert set(li.l_shipinstruct) == set(range(4))
+    # part: brand / container / size domains; partsupp: 4 distinct suppliers per part, and
+    # every (l_partkey, l_suppkey) is one partsupp row
+    assert set(p.p_brand) == set(range(25)) and set(p.p_container) == set(range(40))
+    assert p.p_size.min() == 1 and p.p_size.max() == 50 and (p.p_partkey == np.arange(1, len(p) + 1)).all()
+    assert len(ps) == 4 * len(p) and (ps.groupby("ps_partkey").ps_suppkey.nunique() == 4).all()
+    assert ps.ps_suppkey.between(1, ns).all() and ps.ps_supplycost.between(100, 100000).all()
+    m = li.merge(ps, left_on=["l_partkey", "l_suppkey"], right_on=["ps_partkey", "ps_suppkey"])
+    assert len(m) == len(li)
+    assert hqgen.BRANDS[hqgen.code(hqgen.BRANDS, "Brand#23")] == "Brand#23" and hqgen.BRANDS == sorted(hqgen.BRANDS)
+    assert len(hqgen.CONTAINERS) == 40 and hqgen.CONTAINERS == sorted(hqgen.CONTAINERS)
