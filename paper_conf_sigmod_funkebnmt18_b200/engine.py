@@ -198,6 +198,14 @@ class Engine:
     def plan(self, fact: str) -> PlanBuilder:
         return PlanBuilder(self.tables[fact])
 
+    def plan_over(self, res: hq.Result, names: Sequence[str]) -> PlanBuilder:
+        """A pipeline over a finalized aggregation (or materialised) result, e.g. the
+        outer GROUP BY of TPC-H Q13 or a HAVING / derived predicate; run it with
+        partitioned=False."""
+        pb = PlanBuilder(res.as_table(list(names)))
+        pb.keep.append(res)
+        return pb
+
     def hash(self, table: str, key: str, payload: Sequence[str] = (),
              preds: Sequence[Tuple] = (), expected_rows: int = 0) -> hq.Hash:
         t = self.tables[table]

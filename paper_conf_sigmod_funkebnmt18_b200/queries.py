@@ -391,6 +391,208 @@ def _tpch_q10(E: Engine, limit: int = 20, **_):
     return res, pl
 
 
+# ------------------------------------------------------- TPC-H Q4, Q13, Q17, Q18, Q19, Q21
+# Single-device plans (multi-GPU: DESIGN.md §7).  Correlated and nested subqueries
+# become pipelines whose aggregation results feed builds or further pipelines
+# (pipeline breakers); functionally dependent attributes (R18) ride along
+# as MIN aggregates of their group.
+_KEY32 = 1 << 31
+
+
+def _orders_estimate(E: Engine) -> int:
+    return max(1024, E.table("lineitem").nrows // 4)  # 1..7 lines per order, 4 on average
+
+
+# select o_orderpriority, count(*) as order_count from orders
+# where o_orderdate >= date '1993-07-01' and o_orderdate < date '1993-10-01'
+#   and exists (select * from lineitem where l_orderkey = o_orderkey and l_commitdate < l_receiptdate)
+# group by o_orderpriority order by o_orderpriority
+def _tpch_q4(E: Engine, **_):
+    # the quarter's orders -> build (3.8 % of the orders, payload o_orderpriority)
+    ho = E.hash("orders", "o_orderkey", payload=["o_orderpriority"],
+                preds=[("o_orderdate", "between", 19930701, 19931001 - 1)])
+    nk = max(int(ho.info().nkeys), 0)
+    # lineitem: late lines probe the quarter's orders; GROUP BY l_orderkey = the EXISTS (one row per order)
+    pl = E.plan("lineitem")
+    pl.compute("late", [("load", "l_receiptdate"), ("sub", "l_commitdate")])
+    pl.filter("late", ">", 0)                                   # l_commitdate < l_receiptdate
+    pl.probe(ho, "l_orderkey", "inner", ["o_orderpriority"])
+    pl.aggregate(keys=[("l_orderkey", 0, _KEY32), ("o_orderpriority", 0, 5)], aggs=[("count", None)],
+                 group_capacity=max(1024, nk), agg_names=["lines"])
+    rl = E.run(pl, partitioned=False)
+    # orders per priority over the distinct order keys
+    pg = E.plan_over(rl, ["l_orderkey", "o_orderpriority", "lines"])
+    pg.aggregate(keys=[("o_orderpriority", 0, 5)], aggs=[("count", None)],
+                 order=[("o_orderpriority", False)], agg_names=["order_count"])
+    return E.run(pg, partitioned=False), pg
+
+
+# select c_count, count(*) as custdist
+# from (select c_custkey, count(o_orderkey) from customer left outer join orders on c_custkey = o_custkey
+#       group by c_custkey) as c_orders (c_custkey, c_count)
+# group by c_count order by custdist desc, c_count desc            (App F: no o_comment LIKE)
+def _tpch_q13(E: Engine, **_):
+    po = E.plan("orders")
+    po.aggregate(keys=[("o_custkey", 0, _KEY32)], aggs=[("count", None)],
+                 group_capacity=max(1024, E.table("tpch_customer").nrows), agg_names=["n"])
+    ro = E.run(po, partitioned=False)
+    hn = E.hash_from(ro, ["o_custkey", "n"], "o_custkey", ["n"])
+    maxn = max(int(hn.info().pay_max), 0)
+    pc = E.plan("tpch_customer")
+    pc.probe(hn, "c_custkey", "outer", ["c_count"])            # LEFT OUTER JOIN: 0 orders -> 0
+    pc.aggregate(keys=[("c_count", 0, maxn + 1)], aggs=[("count", None)],
+                 order=[("custdist", True), ("c_count", True)], agg_names=["custdist"])
+    res = E.run(pc, partitioned=False)
+    pc.keep += [ro, hn]
+    return res, pc
+
+
+# select sum(l_extendedprice) / 7.0 as avg_yearly from lineitem, part
+# where p_partkey = l_partkey and p_brand = 'Brand#23' and p_container = 'MED BOX'
+#   and l_quantity < (select 0.2 * avg(l_quantity) from lineitem where l_partkey = p_partkey)
+# unnested (App F): pipeline 1 aggregates the subquery per selected part, pipeline 2
+# tests l_quantity < 0.2 * sum / cnt as 5 * l_quantity * cnt - sum < 0 (exact integers, R19).
+def _tpch_q17(E: Engine, **_):
+    hp = E.hash("tpch_part", "p_partkey", preds=[("p_brand", "=", hqgen.code(hqgen.BRANDS, "Brand#23")),
+                                                 ("p_container", "=", hqgen.code(hqgen.CONTAINERS, "MED BOX"))])
+    p1 = E.plan("lineitem")
+    p1.probe(hp, "l_partkey", "semi")
+    p1.aggregate(keys=[("l_partkey", 0, _KEY32)], aggs=[("sum", "l_quantity"), ("count", None)],
+                 group_capacity=max(1024, int(hp.info().nkeys)), agg_names=["sum_qty", "cnt"])
+    r1 = E.run(p1, partitioned=False)
+    ha = E.hash_from(r1, ["l_partkey", "sum_qty", "cnt"], "l_partkey", ["sum_qty", "cnt"])
+    p2 = E.plan("lineitem")
+    p2.probe(ha, "l_partkey", "inner", ["sum_qty", "cnt"])
+    p2.compute("d", [("load", "l_quantity"), ("mul", 5), ("mul", "cnt"), ("sub", "sum_qty")])
+    p2.filter("d", "<", 0)
+    p2.aggregate(aggs=[("sum", "l_extendedprice"), ("count", None)], agg_names=["sum_extendedprice", "count"])
+    res = E.run(p2, partitioned=False)
+    p2.keep += [r1, hp]
+    return res, p2
+
+
+# select c_name, c_custkey, o_orderkey, o_orderdate, o_totalprice, sum(l_quantity)
+# from customer, orders, lineitem
+# where o_orderkey in (select l_orderkey from lineitem group by l_orderkey having sum(l_quantity) > 300)
+#   and c_custkey = o_custkey and o_orderkey = l_orderkey
+# group by c_name, c_custkey, o_orderkey, o_orderdate, o_totalprice
+# order by o_totalprice desc, o_orderdate limit 100
+def _tpch_q18(E: Engine, limit: int = 100, **_):
+    # the IN subquery: GROUP BY l_orderkey over all of lineitem, HAVING as the build predicate
+    p1 = E.plan("lineitem")
+    p1.aggregate(keys=[("l_orderkey", 0, _KEY32)], aggs=[("sum", "l_quantity")],
+                 group_capacity=_orders_estimate(E), agg_names=["sum_qty"])
+    r1 = E.run(p1, partitioned=False)
+    hb = E.hash_from(r1, ["l_orderkey", "sum_qty"], "l_orderkey", preds=[("sum_qty", ">", 30000)])
+    hc = E.hash("tpch_customer", "c_custkey")
+    po = E.plan("orders")
+    po.probe(hb, "o_orderkey", "semi")
+    po.probe(hc, "o_custkey", "semi")
+    po.materialise([("o_orderkey", "i32"), ("o_custkey", "i32"), ("o_orderdate", "i32"), ("o_totalprice", "i64")])
+    ro = E.run(po, partitioned=False)
+    ho = E.hash_from(ro, ["o_orderkey", "o_custkey", "o_orderdate", "o_totalprice"], "o_orderkey",
+                     ["o_custkey", "o_orderdate", "o_totalprice"])
+    pl = E.plan("lineitem")
+    pl.probe(ho, "l_orderkey", "inner", ["o_custkey", "o_orderdate", "o_totalprice"])
+    pl.aggregate(keys=[("l_orderkey", 0, _KEY32)],
+                 aggs=[("min", "o_custkey"), ("min", "o_orderdate"), ("min", "o_totalprice"),
+                       ("sum", "l_quantity"), ("count", None)],
+                 order=[("o_totalprice", True), ("o_orderdate", False)], limit=limit,
+                 group_capacity=max(1024, int(ho.info().nkeys)),
+                 agg_names=["c_custkey", "o_orderdate", "o_totalprice", "sum_qty", "count"])
+    res = E.run(pl, partitioned=False)
+    pl.result_names = ["o_orderkey"] + pl.result_names[1:]
+    pl.keep += [r1, hb, ro, ho]
+    return res, pl
+
+
+# select sum(l_extendedprice * (1 - l_discount)) as revenue from lineitem, part
+# where (p_partkey = l_partkey and p_brand = 'Brand#12' and p_container in ('SM CASE', 'SM BOX', 'SM PACK', 'SM PKG')
+#        and l_quantity >= 1 and l_quantity <= 1 + 10 and p_size between 1 and 5
+#        and l_shipmode in ('AIR', 'AIR REG') and l_shipinstruct = 'DELIVER IN PERSON')
+#    or (... 'Brand#23' ... ('MED BAG', 'MED BOX', 'MED PKG', 'MED PACK') ... 10 .. 20 ... size 1 .. 10 ...)
+#    or (... 'Brand#34' ... ('LG CASE', 'LG BOX', 'LG PACK', 'LG PKG') ... 20 .. 30 ... size 1 .. 15 ...)
+# The conjuncts common to the three disjuncts are filters / the part build's superset
+# predicate; each disjunct is one predicate expression over the probe payloads (HQ_I_AND_*).
+_Q19 = [("Brand#12", ["SM CASE", "SM BOX", "SM PACK", "SM PKG"], 1, 5),
+        ("Brand#23", ["MED BAG", "MED BOX", "MED PKG", "MED PACK"], 10, 10),
+        ("Brand#34", ["LG CASE", "LG BOX", "LG PACK", "LG PKG"], 20, 15)]
+
+
+def _tpch_q19(E: Engine, **_):
+    brands = [hqgen.code(hqgen.BRANDS, b) for b, *_ in _Q19]
+    conts = [[hqgen.code(hqgen.CONTAINERS, c) for c in cs] for _, cs, *_ in _Q19]
+    hp = E.hash("tpch_part", "p_partkey", payload=["p_brand", "p_container", "p_size"],
+                preds=[("p_brand", "in", brands), ("p_container", "in", sum(conts, [])),
+                       ("p_size", "between", 1, 15)])
+    modes = [hqgen.code(hqgen.SHIPMODES, m) for m in ("AIR", "AIR REG") if m in hqgen.SHIPMODES]  # R19
+    pl = E.plan("lineitem")
+    pl.filter("l_shipinstruct", "=", hqgen.code(hqgen.SHIPINSTRUCTS, "DELIVER IN PERSON"))
+    pl.filter("l_shipmode", "in", modes)
+    pl.filter("l_quantity", "between", 100, 3000)               # the union of the three ranges
+    pl.probe(hp, "l_partkey", "inner", ["p_brand", "p_container", "p_size"])
+    for k, (brand, cs, (_, _, qlo, size)) in enumerate(zip(brands, conts, _Q19)):
+        code = [("load", 1), ("and_eq", "p_brand", brand), ("and_in", "p_container", cs),
+                ("and_ge", "l_quantity", qlo * 100), ("and_le", "l_quantity", (qlo + 10) * 100),
+                ("and_ge", "p_size", 1), ("and_le", "p_size", size)]
+        code += [("or", f"b{j}") for j in range(k)]
+        pl.compute(f"b{k}", code)
+    pl.filter("b2", "!=", 0)
+    pl.compute("rev", [("load", "l_discount"), ("rsub", 100), ("mul", "l_extendedprice")])  # scale 4
+    pl.aggregate(aggs=[("sum", "rev"), ("count", None)], agg_names=["revenue", "count"])
+    return E.run(pl, partitioned=False), pl
+
+
+# select s_name, count(*) as numwait from supplier, lineitem l1, orders, nation
+# where s_suppkey = l1.l_suppkey and o_orderkey = l1.l_orderkey and o_orderstatus = 'F'
+#   and l1.l_receiptdate > l1.l_commitdate
+#   and exists (select * from lineitem l2 where l2.l_orderkey = l1.l_orderkey and l2.l_suppkey <> l1.l_suppkey)
+#   and not exists (select * from lineitem l3 where l3.l_orderkey = l1.l_orderkey
+#                   and l3.l_suppkey <> l1.l_suppkey and l3.l_receiptdate > l3.l_commitdate)
+#   and s_nationkey = n_nationkey and n_name = 'SAUDI ARABIA'
+# group by s_name order by numwait desc, s_name limit 100
+# variant 1: App F's EXISTS for the third subquery.  l1's supplier belongs to
+# both subqueries' supplier sets, so "another supplier exists" <=> min(l_suppkey) <> max(l_suppkey)
+# over the order's lines (l2) / late lines (l3): two GROUP BY l_orderkey pipelines (R20).
+def _tpch_q21(E: Engine, variant: int = 0, limit: int = 100, **_):
+    saudi = hqgen.code(hqgen.NATIONS, "SAUDI ARABIA")
+    hs, hn, ho = E.hashes([dict(table="tpch_supplier", key="s_suppkey", payload=["s_nationkey"],
+                                preds=[("s_nationkey", "=", saudi)]),
+                           dict(table="nation", key="n_nationkey", preds=[("n_nationkey", "=", saudi)]),
+                           dict(table="orders", key="o_orderkey",
+                                preds=[("o_orderstatus", "=", hqgen.code(hqgen.ORDERSTATUS, "F"))])])
+    sets = []
+    for late in (False, True):  # l2: all lines of the order; l3: its late lines
+        pb = E.plan("lineitem")
+        if late:
+            pb.compute("late", [("load", "l_receiptdate"), ("sub", "l_commitdate")])
+            pb.filter("late", ">", 0)
+        pb.aggregate(keys=[("l_orderkey", 0, _KEY32)], aggs=[("min", "l_suppkey"), ("max", "l_suppkey")],
+                     group_capacity=_orders_estimate(E), agg_names=["smin", "smax"])
+        r = E.run(pb, partitioned=False)
+        pm = E.plan_over(r, ["l_orderkey", "smin", "smax"])
+        pm.compute("d", [("load", "smax"), ("sub", "smin")])
+        pm.filter("d", "=" if (late and variant == 0) else "!=", 0)
+        pm.materialise([("l_orderkey", "i32")])
+        sets.append(E.hash_from(E.run(pm, partitioned=False), ["l_orderkey"], "l_orderkey"))
+    h2, h3 = sets
+    pl = E.plan("lineitem")
+    pl.compute("late", [("load", "l_receiptdate"), ("sub", "l_commitdate")])
+    pl.filter("late", ">", 0)                                   # l1.l_receiptdate > l1.l_commitdate
+    pl.probe(hs, "l_suppkey", "inner", ["s_nationkey"])         # 1/25
+    pl.probe(hn, "s_nationkey", "semi")
+    pl.probe(ho, "l_orderkey", "semi")                          # o_orderstatus = 'F'
+    pl.probe(h2, "l_orderkey", "semi")                          # exists l2
+    pl.probe(h3, "l_orderkey", "semi")                          # not exists l3 (variant 1: exists)
+    nsupp = E.table("tpch_supplier").nrows
+    pl.aggregate(keys=[("l_suppkey", 1, max(nsupp, 1))], aggs=[("count", None)],
+                 order=[("numwait", True), ("l_suppkey", False)], limit=limit, agg_names=["numwait"])
+    res = E.run(pl, partitioned=False)
+    pl.result_names = ["s_suppkey", "numwait"]
+    pl.keep += sets
+    return res, pl
+
+
 # ------------------------------------------------ paper micro queries (f2)
 def _micro_select(E: Engine, x: int = 5, resolution=None, **_):
     """PAPER.md Fig 16 'Query 1': selection + projection, materialised."""
@@ -476,6 +678,25 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
           {"lineitem": ["l_orderkey", "l_returnflag", "l_extendedprice", "l_discount"],
            "orders": ["o_orderkey", "o_custkey", "o_orderdate"], "tpch_customer": ["c_custkey", "c_nationkey"],
            "nation": ["n_nationkey"]}, _tpch_q10),
+    Query("tpch_q4", "tpch", "lineitem",
+          {"lineitem": ["l_orderkey", "l_commitdate", "l_receiptdate"],
+           "orders": ["o_orderkey", "o_orderdate", "o_orderpriority"]}, _tpch_q4),
+    Query("tpch_q13", "tpch", "orders",
+          {"orders": ["o_custkey"], "tpch_customer": ["c_custkey"]}, _tpch_q13),
+    Query("tpch_q17", "tpch", "lineitem",
+          {"lineitem": ["l_partkey", "l_quantity", "l_extendedprice"],
+           "tpch_part": ["p_partkey", "p_brand", "p_container"]}, _tpch_q17),
+    Query("tpch_q18", "tpch", "lineitem",
+          {"lineitem": ["l_orderkey", "l_quantity"],
+           "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_totalprice"],
+           "tpch_customer": ["c_custkey"]}, _tpch_q18),
+    Query("tpch_q19", "tpch", "lineitem",
+          {"lineitem": ["l_partkey", "l_quantity", "l_extendedprice", "l_discount", "l_shipmode", "l_shipinstruct"],
+           "tpch_part": ["p_partkey", "p_brand", "p_container", "p_size"]}, _tpch_q19),
+    Query("tpch_q21", "tpch", "lineitem",
+          {"lineitem": ["l_orderkey", "l_suppkey", "l_commitdate", "l_receiptdate"],
+           "orders": ["o_orderkey", "o_orderstatus"], "tpch_supplier": ["s_suppkey", "s_nationkey"],
+           "nation": ["n_nationkey"]}, _tpch_q21),
     Query("micro_select", "ssb", "lineorder",
           {"lineorder": ["lo_quantity", "lo_extendedprice", "lo_discount", "lo_tax"]}, _micro_select),
     Query("micro_sum", "ssb", "lineorder",

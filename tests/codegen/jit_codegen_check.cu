@@ -289,12 +289,35 @@ int main(int argc, char** argv) {
     shapes.push_back({"global_hash_groups_r4", P, "4"});
   }
 
+  {  // LEFT OUTER probes (byte map, linear, direct) and predicate expressions (TPC-H Q13 / Q19 shapes)
+    hq_plan P{};
+    P.fact = F;
+    P.row_end = -1;
+    P.ops[P.nops++] = probe(byte_big, 0, HQ_PROBE_OUTER, HQ_TMP(0));
+    P.ops[P.nops++] = probe(lin_1, 1, HQ_PROBE_OUTER, HQ_TMP(1));
+    P.ops[P.nops++] = probe(direct2, 2, HQ_PROBE_OUTER, HQ_TMP(2));
+    P.ops[P.nops++] = compute(HQ_TMP(3), {{HQ_I_LOAD, -1, 1}, {HQ_I_AND_EQ, HQ_TMP(0), 3}, {HQ_I_AND_IN, 7, 0x0F0F},
+                                          {HQ_I_AND_LE, 5, 7}});
+    P.ops[P.nops++] = compute(HQ_TMP(4), {{HQ_I_LOAD, -1, 1}, {HQ_I_AND_GE, HQ_TMP(1), 2}, {HQ_I_AND_NE, 4, 9},
+                                          {HQ_I_AND_LT, 5, 3}, {HQ_I_AND_GT, 6, 0}, {HQ_I_OR, HQ_TMP(3), 0}});
+    P.ops[P.nops++] = filter(HQ_TMP(4), HQ_NE, 0);
+    P.sink = HQ_SINK_AGG;
+    P.nkeys = 1;
+    P.key_reg[0] = HQ_TMP(0); P.key_card[0] = 25;
+    P.naggs = 2;
+    P.agg_fn[0] = HQ_AGG_SUM; P.agg_reg[0] = 6;
+    P.agg_fn[1] = HQ_AGG_COUNT;
+    shapes.push_back({"outer_predicates", P, nullptr});
+  }
+
   // multi-pass count / write kernels (HQ_EXEC_MULTIPASS) of a grouped star
   // join, a materialising pipeline and a scalar aggregate
   {
     std::vector<Shape> mps;
     for (const Shape& s : shapes) {
-      if (s.name != "star_ranked_dense" && s.name != "materialise_lrgp" && s.name != "scalar_filters") continue;
+      if (s.name != "star_ranked_dense" && s.name != "materialise_lrgp" && s.name != "scalar_filters" &&
+          s.name != "outer_predicates")
+        continue;
       for (int pass : {1, 2}) {
         Shape m = s;
         m.name = s.name + "_mp" + std::to_string(pass);

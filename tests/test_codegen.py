@@ -32,7 +32,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     env = {k: v for k, v in os.environ.items() if not k.startswith("HQ_")}
     p = subprocess.run([checker, str(tmp_path)], capture_output=True, text=True, env=env, timeout=600)
     assert p.returncode == 0, p.stdout + p.stderr
-    assert p.stdout.startswith("OK 18 of 18"), p.stdout
+    assert p.stdout.startswith("OK 21 of 21"), p.stdout
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
     star = srcs["star_dense_lrgp"]
@@ -60,3 +60,8 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "((u64*)p.out[0])[pos_] = gk_[r];" in srcs["star_ranked_dense_mp2"]
     # high-cardinality hash group-by skips the shared table (C2 straight to global)
     assert "#define SMODE 0" in srcs["global_hash_groups"]
+    # LEFT OUTER probes keep the row and default the payload to 0; predicate instructions
+    op = srcs["outer_predicates"]
+    assert "[R] = {};" in op and "mask; (void)found_" in op
+    assert "(a_ != 0 && " in op and "3855ULL >> v_" in op and "(a_ != 0 || " in op
+    assert "mask; (void)found_" not in srcs["outer_predicates_mp2"].split("extern \"C\"")[0]

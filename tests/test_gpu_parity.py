@@ -57,6 +57,18 @@ def oracle_run(qname, t, **kw):
         return oracle.ssb_q41(t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"])
     if qname == "tpch_q3":
         return oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    if qname == "tpch_q4":
+        return oracle.tpch_q4(t["orders"], t["lineitem"])
+    if qname == "tpch_q13":
+        return oracle.tpch_q13(t["tpch_customer"], t["orders"])
+    if qname == "tpch_q17":
+        return oracle.tpch_q17(t["tpch_part"], t["lineitem"])
+    if qname == "tpch_q18":
+        return oracle.tpch_q18(t["tpch_customer"], t["orders"], t["lineitem"])
+    if qname == "tpch_q19":
+        return oracle.tpch_q19(t["tpch_part"], t["lineitem"])
+    if qname == "tpch_q21":
+        return oracle.tpch_q21(t["tpch_supplier"], t["orders"], t["lineitem"], t["nation"], variant=kw.get("variant", 0))
     if qname == "tpch_q7":
         return oracle.tpch_q7(t["tpch_customer"], t["orders"], t["lineitem"], t["tpch_supplier"], t["nation"])
     if qname == "tpch_q10":
@@ -89,6 +101,12 @@ INT_COLS = {
     "tpch_q5": ["n_name", "revenue", "count"],
     "tpch_q10": ["c_custkey", "n_name", "revenue", "count"],
     "tpch_q7": ["supp_nation", "cust_nation", "l_year", "revenue", "count"],
+    "tpch_q4": ["o_orderpriority", "order_count"],
+    "tpch_q13": ["c_count", "custdist"],
+    "tpch_q17": ["sum_extendedprice", "count"],
+    "tpch_q18": ["c_custkey", "o_orderkey", "o_orderdate", "o_totalprice", "sum_qty", "count"],
+    "tpch_q19": ["revenue", "count"],
+    "tpch_q21": ["s_suppkey", "numwait"],
 }
 SSB_FLIGHTS = ["ssb_q21", "ssb_q22", "ssb_q23", "ssb_q32", "ssb_q33", "ssb_q34", "ssb_q42", "ssb_q43"]
 
@@ -532,3 +550,59 @@ def test_sf1_parity_multi_tile(ctx):
              "ssb_q31": lambda: oracle.ssb_q31(host["lineorder"], host["customer"], host["supplier"], host["date"], nthreads=8),
              "ssb_q11": lambda: oracle.ssb_q1(1, host["lineorder"], host["date"], nthreads=8)}[qname]()
         assert_same(qname, g, o)
+
+
+# ------------------------------------------- TPC-H Q4, Q13, Q17, Q18, Q19, Q21 (f3)
+ALL_EXEC = [hq.EXEC_FUSED, hq.EXEC_FUSED_INTERP, hq.EXEC_MULTIPASS, hq.EXEC_OAAT]
+LIMITED = {"tpch_q18": 100, "tpch_q21": 100}
+
+
+@pytest.fixture(scope="module")
+def tpch1():
+    return {t: hqgen.generate(t, 1.0) for t in hqgen.TPCH_TABLES}
+
+
+@pytest.mark.parametrize("qname", ["tpch_q4", "tpch_q13", "tpch_q17", "tpch_q18", "tpch_q19", "tpch_q21"])
+@pytest.mark.parametrize("sf", [0.01, 1.0])
+def test_tpch_f3_parity(ctx, tpch, tpch1, qname, sf):
+    """Multi-pipeline plans (aggregation results feeding builds and pipelines, LEFT OUTER
+    probes, predicate expressions): every execution model vs the oracle; full pre-LIMIT
+    sets under the total order, then the LIMIT."""
+    host = tpch if sf == 0.01 else tpch1
+    o = oracle_run(qname, host)
+    if sf == 1.0:
+        assert o.nrows > 0 and o.qualifying > 0
+    kw = {"limit": 0} if qname in LIMITED else {}
+    for em in ALL_EXEC:
+        g = gpu_run(ctx, qname, host, exec_mode=em, **kw)
+        assert_same(qname, g, o)
+        assert g.qualifying == o.qualifying, (em, g.qualifying, o.qualifying)
+        if qname in LIMITED and em == hq.EXEC_FUSED:
+            top = gpu_run(ctx, qname, host, exec_mode=em)
+            assert top.rows(INT_COLS[qname]) == o.rows(INT_COLS[qname])[:LIMITED[qname]]
+
+
+@pytest.mark.parametrize("sf", [0.01, 1.0])
+def test_tpch_q21_appf_parity(ctx, tpch, tpch1, sf):
+    """PAPER.md App F's Q21 (EXISTS in place of NOT EXISTS)."""
+    host = tpch if sf == 0.01 else tpch1
+    o = oracle_run("tpch_q21", host, variant=1)
+    for em in (hq.EXEC_FUSED, hq.EXEC_MULTIPASS):
+        g = gpu_run(ctx, "tpch_q21", host, exec_mode=em, variant=1, limit=0)
+        assert_same("tpch_q21", g, o)
+        assert g.qualifying == o.qualifying
+
+
+@pytest.mark.parametrize("fx_name,qname", [("F12_tpch_q4.json", "tpch_q4"), ("F13_tpch_q13.json", "tpch_q13"),
+                                            ("F14_tpch_q17.json", "tpch_q17"), ("F15_tpch_q18.json", "tpch_q18"),
+                                            ("F16_tpch_q19.json", "tpch_q19"), ("F17_tpch_q21.json", "tpch_q21")])
+def test_tpch_f3_golden(ctx, golden, fx_name, qname):
+    """Hand-computed fixtures F12-F17 through the CUDA path, every execution model."""
+    fx = golden(fx_name)
+    for em in ALL_EXEC:
+        g = gpu_run(ctx, qname, fx["tables"], exec_mode=em)
+        assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"], (qname, em)
+        assert g.qualifying == fx["expected"]["qualifying"], (qname, em)
+    if qname == "tpch_q21":
+        g = gpu_run(ctx, qname, fx["tables"], variant=1)
+        assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["appf"]["rows"]
