@@ -133,6 +133,17 @@ typedef struct {
 } hq_column;
 #define HQ_HOST_COPY 1     /* library allocates device memory and copies (async; host buffer must stay valid until the next ctx sync) */
 #define HQ_DEVICE_BORROW 2 /* data are device pointers kept alive by the caller */
+/* HQ_HOST_STREAM: data are HOST pointers kept alive (and unchanged) by the caller until
+ * every pipeline over the table has completed; nothing is copied at load time.  A
+ * pipeline whose fact table is such a table runs as batch processing (§3,
+ * P:220-305; Exp 5): blocks of rows are copied over the host link into a
+ * double-buffered device ring on a copy stream while the compound kernel processes the
+ * previous block on the context stream, and the sink's state (group table, output
+ * counter) carries over the blocks, so the result equals the HBM-resident run.  Pinned
+ * host memory (cudaHostAlloc / cudaHostRegister) is needed for the copies to overlap.
+ * Only fused execution streams (HQ_EXEC_FUSED / HQ_EXEC_FUSED_INTERP); hash builds and
+ * hq_table_column need device tables (HQ_ERR_UNSUPPORTED). */
+#define HQ_HOST_STREAM 3
 hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int64_t nrows,
                           int32_t flags, hq_table** out);
 hq_status hq_table_info(const hq_table* t, int64_t* nrows, int32_t* ncols);
@@ -321,6 +332,12 @@ typedef struct {
 /* Enqueue the pipeline (async).  The plan is copied; hash tables and the fact
  * table it references are retained by the result. */
 hq_status hq_run_pipeline(hq_ctx* ctx, const hq_plan* plan, hq_result** out);
+/* Batch processing over an HQ_HOST_STREAM fact table with an explicit block size:
+ * block_rows > 0 is rounded up to the kernel's tile (hq_run_pipeline uses
+ * HQ_STREAM_BLOCK_ROWS).  Device memory: 2 x block_rows x (bytes of the referenced
+ * columns).  HQ_ERR_ARG when the fact table is not HQ_HOST_STREAM. */
+#define HQ_STREAM_BLOCK_ROWS (1 << 24)
+hq_status hq_run_pipeline_streamed(hq_ctx* ctx, const hq_plan* plan, int64_t block_rows, hq_result** out);
 /* Post-process an AGG result in place (compaction, AVG, ORDER BY, LIMIT);
  * idempotent; implied by hq_result_info_get / hq_fetch_result. */
 hq_status hq_finalize(hq_ctx* ctx, hq_result* r);

@@ -129,6 +129,14 @@ hq_status hq_ctx_destroy(hq_ctx* ctx) {
     for (auto e : ctx->event_pool) cudaEventDestroy(e);
     if (ctx->pinned) cudaFreeHost(ctx->pinned);
     if (ctx->pinned_build) cudaFreeHost(ctx->pinned_build);
+    if (ctx->copy_stream) {
+      cudaStreamSynchronize(ctx->copy_stream);
+      cudaStreamDestroy(ctx->copy_stream);
+    }
+    for (int i = 0; i < 2; ++i) {
+      if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
+      if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
+    }
     delete ctx;
   });
 }
@@ -186,7 +194,8 @@ hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int
     if (!ctx || !out || (!cols && ncols > 0)) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     if (ncols < 0 || ncols > HQ_MAX_COLS) HQ_THROW(HQ_ERR_UNSUPPORTED, "tables have 0..16 columns");
     if (nrows < 0) HQ_THROW(HQ_ERR_ARG, "nrows < 0");
-    if (flags != HQ_HOST_COPY && flags != HQ_DEVICE_BORROW) HQ_THROW(HQ_ERR_ARG, "flags must be HQ_HOST_COPY or HQ_DEVICE_BORROW");
+    if (flags != HQ_HOST_COPY && flags != HQ_DEVICE_BORROW && flags != HQ_HOST_STREAM)
+      HQ_THROW(HQ_ERR_ARG, "flags must be HQ_HOST_COPY, HQ_DEVICE_BORROW or HQ_HOST_STREAM");
     hq_table* t = new hq_table();
     t->ctx = ctx;
     t->nrows = nrows;
@@ -204,6 +213,9 @@ hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int
           t->owned.emplace_back(ctx, (bytes + 255) / 256 * 256 + 256);
           if (bytes) HQ_CUDA(cudaMemcpyAsync(t->owned.back().p, cols[c].data, bytes, cudaMemcpyHostToDevice, ctx->stream));
           t->cols[c].ptr = t->owned.back().p;
+        } else if (flags == HQ_HOST_STREAM) {  // stays on the host; pipelines stream it in blocks
+          t->host_stream = true;
+          t->cols[c].ptr = cols[c].data;
         } else {
           if (((uintptr_t)cols[c].data & 15) != 0) HQ_THROW(HQ_ERR_ARG, "device column pointer must be 16-byte aligned");
           t->cols[c].ptr = cols[c].data;
@@ -228,6 +240,7 @@ hq_status hq_table_info(const hq_table* t, int64_t* nrows, int32_t* ncols) {
 hq_status hq_table_column(const hq_table* t, int32_t col, const void** dev_ptr, int32_t* type) {
   return guarded([&] {
     if (!t || col < 0 || col >= t->ncols) HQ_THROW(HQ_ERR_ARG, "bad table/column");
+    if (t->host_stream) HQ_THROW(HQ_ERR_UNSUPPORTED, "HQ_HOST_STREAM table: its columns are not in device memory");
     if (dev_ptr) *dev_ptr = t->cols[col].ptr;
     if (type) *type = t->cols[col].type;
   });
@@ -320,11 +333,11 @@ hq_status hq_free_hash(hq_hash* h) {
 }
 
 // ---------------------------------------------------------------- pipelines
-hq_status hq_run_pipeline(hq_ctx* ctx, const hq_plan* plan, hq_result** out) {
-  return guarded([&] {
+static void run_pipeline(hq_ctx* ctx, const hq_plan* plan, int64_t block_rows, hq_result** out) {
     if (!ctx || !plan || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     if (!plan->fact) HQ_THROW(HQ_ERR_ARG, "plan: fact table is NULL");
     hq_result* r = new hq_result();
+    if (plan->fact->host_stream) r->stream_block = block_rows > 0 ? block_rows : HQ_STREAM_BLOCK_ROWS;
     r->fact = const_cast<hq_table*>(plan->fact);
     r->fact->retain();
     for (int o = 0; o < plan->nops && o < HQ_MAX_OPS; ++o)
@@ -340,6 +353,18 @@ hq_status hq_run_pipeline(hq_ctx* ctx, const hq_plan* plan, hq_result** out) {
       throw;
     }
     *out = r;
+}
+
+hq_status hq_run_pipeline(hq_ctx* ctx, const hq_plan* plan, hq_result** out) {
+  return guarded([&] { run_pipeline(ctx, plan, 0, out); });
+}
+
+hq_status hq_run_pipeline_streamed(hq_ctx* ctx, const hq_plan* plan, int64_t block_rows, hq_result** out) {
+  return guarded([&] {
+    if (plan && plan->fact && !plan->fact->host_stream)
+      HQ_THROW(HQ_ERR_ARG, "hq_run_pipeline_streamed: the fact table is not HQ_HOST_STREAM");
+    if (block_rows < 0) HQ_THROW(HQ_ERR_ARG, "block_rows < 0");
+    run_pipeline(ctx, plan, block_rows, out);
   });
 }
 
@@ -390,7 +415,7 @@ hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int
 hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out) {
   return guarded([&] {
     if (!ctx || !r || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
-    hq_finalize_impl(ctx, r);
+    hq_finalize_impl(ctx, r, /*unordered=*/true);
     const bool mat = r->sink == HQ_SINK_MATERIALISE;
     for (int c = 0; c < r->ncols; ++c)
       if (r->types[c] == HQ_F64) HQ_THROW(HQ_ERR_UNSUPPORTED, "result has fp64 (AVG) columns: not a table");

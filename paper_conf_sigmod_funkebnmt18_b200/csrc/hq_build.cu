@@ -336,6 +336,7 @@ struct BuildState {
 void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& bs) {
   const hq_table* t = d->src;
   if (!t) HQ_THROW(HQ_ERR_ARG, "build: NULL source table");
+  if (t->host_stream) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: the source is an HQ_HOST_STREAM (host) table");
   if (d->npreds < 0 || d->npreds > HQ_MAX_PREDS) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: too many predicates");
   if (d->npayload < 0 || d->npayload > HQ_MAX_PAYLOAD) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: 0..3 payload columns");
   if (d->key_col < 0 || d->key_col >= t->ncols) HQ_THROW(HQ_ERR_ARG, "build: key column out of range");

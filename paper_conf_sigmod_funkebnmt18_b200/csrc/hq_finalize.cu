@@ -3,6 +3,8 @@
 // compiled kernels): compaction of the global group table into rows, AVG,
 // ORDER BY with a total tie-break, LIMIT.  Runs on the device of the context
 // (GPU 0 in the multi-GPU flow).
+#include <cub/device/device_radix_sort.cuh>
+
 #include <algorithm>
 #include <climits>
 #include <cstring>
@@ -142,18 +144,23 @@ __global__ void __launch_bounds__(1024) hq_chunk_sort_kernel(const __grid_consta
   for (int i = m + threadIdx.x; i < keep; i += blockDim.x) out[(long long)blockIdx.x * keep + i] = -1;
 }
 
-// one step of a global bitonic sort over a power-of-two index array
-__global__ void hq_bitonic_step_kernel(const __grid_constant__ KSort s, int* idx, long long n, long long j, long long k) {
+// Radix-sort key of one ORDER BY / group-key column in row order idx (NULL =
+// identity): an unsigned image whose ascending order is the column's order.
+// Group keys: v - key_min (< key_card, so only the low bits are sorted); order
+// columns: int64 with the sign bit flipped, fp64 by the IEEE total-order map,
+// bitwise NOT for DESC.
+__global__ void hq_sortkey_kernel(const long long* __restrict__ col, const int* __restrict__ idx, long long n,
+                                  int mode, long long kmin, int desc, unsigned long long* __restrict__ out) {
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
-    const long long l = i ^ j;
-    if (l > i) {
-      const int a = idx[i], b = idx[l];
-      const bool up = (i & k) == 0;
-      const bool sw = up ? row_less(s, b, a) : row_less(s, a, b);
-      if (sw) { idx[i] = b; idx[l] = a; }
-    }
+    const long long v = col[idx ? idx[i] : i];
+    unsigned long long t;
+    if (mode == 0) t = (unsigned long long)(v - kmin);                 // group key
+    else if (mode == 1) t = (unsigned long long)v ^ 0x8000000000000000ull;  // int64
+    else t = v < 0 ? ~(unsigned long long)v : (unsigned long long)v ^ 0x8000000000000000ull;  // fp64 bits
+    out[i] = desc ? ~t : t;
   }
 }
+
 __global__ void hq_iota_kernel(int* idx, long long n, long long valid) {
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
     idx[i] = i < valid ? (int)i : -1;
@@ -376,7 +383,51 @@ bool finalize_small(hq_ctx* ctx, hq_result* r) {
 }
 }  // namespace
 
-void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
+// Stable LSD radix sort of the rows by (ORDER BY columns, then the group keys
+// ascending): one CUB radix pass per column, least significant first; returns
+// the sorted row order in `idx` (n entries).
+static void radix_order(hq_ctx* ctx, const hq_plan& P, const std::vector<DevBuf>& cols, const int* types, int64_t n,
+                        DevBuf& idx) {
+  DevBuf kb[2] = {DevBuf(ctx, (size_t)n * 8), DevBuf(ctx, (size_t)n * 8)};
+  DevBuf ib(ctx, (size_t)n * 4);
+  idx = DevBuf(ctx, (size_t)n * 4);
+  size_t tmp_bytes = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, kb[0].as<unsigned long long>(), kb[1].as<unsigned long long>(),
+                                  ib.as<int>(), idx.as<int>(), (int)n, 0, 64, ctx->stream);
+  DevBuf tmp(ctx, tmp_bytes + 16);
+  bool first = true;
+  auto pass = [&](int c, int mode, long long kmin, int desc, int bits) {
+    ctx->launches++;
+    hq_sortkey_kernel<<<grid_for(ctx, n), 256, 0, ctx->stream>>>(cols[c].as<long long>(), first ? nullptr : idx.as<int>(), n,
+                                                                 mode, kmin, desc, kb[0].as<unsigned long long>());
+    if (first) {
+      ctx->launches++;
+      hq_iota_kernel<<<grid_for(ctx, n), 256, 0, ctx->stream>>>(ib.as<int>(), n, n);
+    } else {
+      HQ_CUDA(cudaMemcpyAsync(ib.p, idx.p, (size_t)n * 4, cudaMemcpyDeviceToDevice, ctx->stream));
+    }
+    size_t tb = tmp_bytes;
+    ctx->launches++;
+    HQ_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, kb[0].as<unsigned long long>(), kb[1].as<unsigned long long>(),
+                                            ib.as<int>(), idx.as<int>(), (int)n, 0, bits, ctx->stream));
+    first = false;
+  };
+  for (int i = P.nkeys - 1; i >= 0; --i) {  // tie-break: group keys ascending (R7)
+    int bits = 1;
+    while (bits < 64 && (1ull << bits) < (unsigned long long)P.key_card[i]) ++bits;
+    pass(i, 0, P.key_min[i], 0, bits);
+  }
+  for (int i = P.norder - 1; i >= 0; --i) {
+    const int c = P.order_col[i];
+    pass(c, types[c] == HQ_F64 ? 2 : 1, 0, P.order_desc[i] ? 1 : 0, 64);
+  }
+  if (first) {  // no sort column: identity order
+    ctx->launches++;
+    hq_iota_kernel<<<grid_for(ctx, n), 256, 0, ctx->stream>>>(idx.as<int>(), n, n);
+  }
+}
+
+void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered) {
   if (r->finalized) return;
   if (r->sink == HQ_SINK_AGG && r->gmode != GM_HASH && r->ngroups <= SMALL_FIN) {
     if (finalize_small(ctx, r)) return;
@@ -444,7 +495,9 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
   int64_t nfinal = n;
   if (P.limit > 0) nfinal = std::min<int64_t>(nfinal, P.limit);
   // ---- ORDER BY (+ LIMIT)
-  if ((P.norder > 0 || nk > 0) && n > 1) {
+  // a pure GROUP BY (no ORDER BY, no LIMIT) viewed as a table keeps the group-table order
+  const bool sort = (P.norder > 0 || nk > 0) && n > 1 && !(unordered && P.norder == 0 && P.limit <= 0);
+  if (sort) {
     KSort s{};
     for (int c = 0; c < nc; ++c) {
       s.col[c] = cols[c].as<long long>();
@@ -488,17 +541,8 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r) {
       hq_chunk_sort_kernel<<<1, std::min(1024, net), 0, ctx->stream>>>(s, nullptr, n, ia.as<int>(), SORT_CHUNK, net);
       HQ_CUDA(cudaGetLastError());
       sorted = ia.as<int>();
-    } else {
-      int64_t N = 1;
-      while (N < n) N <<= 1;
-      ia = DevBuf(ctx, (size_t)N * 4);
-      ctx->launches++;
-      hq_iota_kernel<<<grid_for(ctx, N), 256, 0, ctx->stream>>>(ia.as<int>(), N, n);
-      for (int64_t kk = 2; kk <= N; kk <<= 1)
-        for (int64_t j = kk >> 1; j > 0; j >>= 1) {
-          ctx->launches++;
-          hq_bitonic_step_kernel<<<grid_for(ctx, N), 256, 0, ctx->stream>>>(s, ia.as<int>(), N, j, kk);
-        }
+    } else {  // large results: stable LSD radix sort, one CUB pass per sort column
+      radix_order(ctx, P, cols, r->types, n, ia);
       HQ_CUDA(cudaGetLastError());
       sorted = ia.as<int>();
     }

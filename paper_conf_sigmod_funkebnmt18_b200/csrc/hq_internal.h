@@ -81,6 +81,10 @@ struct hq_ctx {
   size_t pinned_bytes = 0;
   void* pinned_build = nullptr;  // host staging of the builds' count-pass statistics
   size_t pinned_build_bytes = 0;
+  // batch processing of HQ_HOST_STREAM tables: host->device copies run on their own
+  // stream, ordered against the pipeline kernels by events (created on first use)
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_copied[2] = {nullptr, nullptr}, ev_consumed[2] = {nullptr, nullptr};
   void* alloc_bytes(size_t bytes);
   void free_bytes(void* p, size_t bytes);
 };
@@ -132,6 +136,7 @@ struct hq_table : RefObj {
   TableCol cols[HQ_MAX_COLS];
   std::vector<DevBuf> owned;
   hq_result* backing = nullptr;  // retained when the table views a result
+  bool host_stream = false;      // HQ_HOST_STREAM: cols[].ptr are caller-owned host pointers
   ~hq_table() override;
 };
 
@@ -337,6 +342,8 @@ struct hq_result : RefObj {
   DevBuf mp_flags, mp_pos, mp_keys, mp_vals, mp_scratch;
   const char* mp_flags_col = nullptr;  // flags / positions indexed by absolute row
   const char* mp_pos_col = nullptr;
+  int64_t stream_block = 0;  // > 0: batch processing of a host-resident fact table, rows per block
+  DevBuf ring;               // its double-buffered device blocks
   std::vector<long long> host_rows;  // small results: the finalized rows already on the host
   bool host_ready = false;           // (column-major, nrows per column)
   ~hq_result() override;
@@ -351,7 +358,8 @@ int64_t fused_smem_bytes(const KPlan& kp);
 }  // namespace hqk
 
 // finalize: compaction + AVG + ORDER BY + LIMIT (hq_finalize.cu)
-void hq_finalize_impl(hq_ctx* ctx, hq_result* r);
+// unordered: a pure GROUP BY (no ORDER BY / LIMIT) skips the sort (hq_result_as_table)
+void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered = false);
 // op-at-a-time execution of a plan (hq_oaat.cu)
 void hq_run_oaat(hq_ctx* ctx, const hq_plan* plan, hq_result* r);
 // shared plan preparation (hq_plan.cu)

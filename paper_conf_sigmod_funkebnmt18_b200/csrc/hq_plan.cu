@@ -429,7 +429,8 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   uint32_t rowbytes = 0;
   for (int c = 0; c < ncols_all; ++c) {
     if (!col_used[c]) continue;
-    if (((uintptr_t)colptr[c] & 15) != 0) HQ_THROW(HQ_ERR_ARG, "column pointer not 16-byte aligned");
+    // (host-streamed columns are copied into 256-B aligned ring slots)
+    if (!F->host_stream && ((uintptr_t)colptr[c] & 15) != 0) HQ_THROW(HQ_ERR_ARG, "column pointer not 16-byte aligned");
     rowbytes += (uint32_t)colw[c];
   }
   uint32_t tmp_row = 0;  // generated kernels keep temporaries in registers
@@ -542,6 +543,52 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   kp.err = (int*)(r->dstate.as<char>() + 8);
 }
 
+// Batch processing (§3; Exp 5) of an HQ_HOST_STREAM
+// fact table: block b's referenced columns are copied host -> device into ring slot
+// b % 2 on ctx->copy_stream while the compound kernel of block b - 1 runs on the
+// context stream (copy of b waits for the kernel of b - 2 to release the slot).  The
+// kernels see block-local rows [0, rows of the block); the sink state (group table,
+// output counter, fault bits) is initialised once by the caller and carries over.
+static void launch_streamed(hq_ctx* ctx, hq_result* r, const KPlan& kp, bool jit, size_t smem) {
+  const long long T = kp.tile_rows;
+  const int64_t B = std::max<int64_t>(T, (r->stream_block + T - 1) / T * T);
+  size_t slot_off[HQ_MAX_COLS + 1] = {0};
+  for (int k = 0; k < kp.ncols; ++k) slot_off[k + 1] = slot_off[k] + ((size_t)B * kp.cols[k].width + 511) / 256 * 256;
+  const size_t slot_bytes = std::max<size_t>(slot_off[kp.ncols], 256);
+  if (!r->ring.p || r->ring.bytes < 2 * slot_bytes) r->ring = DevBuf(ctx, 2 * slot_bytes);
+  if (!ctx->copy_stream) {
+    HQ_CUDA(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      HQ_CUDA(cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming));
+      HQ_CUDA(cudaEventCreateWithFlags(&ctx->ev_consumed[i], cudaEventDisableTiming));
+    }
+  }
+  // the ring may still be read by earlier work on the context stream
+  for (int i = 0; i < 2; ++i) HQ_CUDA(cudaEventRecord(ctx->ev_consumed[i], ctx->stream));
+  int64_t b = 0;
+  for (int64_t s = kp.row_begin; s < kp.row_end; s += B, ++b) {
+    const int64_t e = std::min<int64_t>(s + B, kp.row_end);
+    const int slot = (int)(b & 1);
+    char* base = r->ring.as<char>() + (size_t)slot * slot_bytes;
+    HQ_CUDA(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_consumed[slot], 0));
+    KPlan kb = kp;
+    kb.row_begin = 0;
+    kb.row_end = e - s;
+    for (int k = 0; k < kp.ncols; ++k) {
+      const size_t w = kp.cols[k].width;
+      HQ_CUDA(cudaMemcpyAsync(base + slot_off[k], (const char*)kp.cols[k].ptr + (size_t)s * w, (size_t)(e - s) * w,
+                              cudaMemcpyHostToDevice, ctx->copy_stream));
+      kb.cols[k].ptr = base + slot_off[k];
+    }
+    HQ_CUDA(cudaEventRecord(ctx->ev_copied[slot], ctx->copy_stream));
+    HQ_CUDA(cudaStreamWaitEvent(ctx->stream, ctx->ev_copied[slot], 0));
+    const int grid = (int)std::max<long long>(1, std::min<long long>((e - s + T - 1) / T, ctx->num_sms));
+    if (jit) hq_jit_launch(ctx, kb, grid, smem);
+    else launch_fused(ctx, kb, grid, smem);
+    HQ_CUDA(cudaEventRecord(ctx->ev_consumed[slot], ctx->stream));
+  }
+}
+
 static void launch_pipeline(hq_ctx* ctx, hq_result* r, int64_t group_cap, int64_t mat_cap) {
   const bool jit = r->plan.exec == HQ_EXEC_FUSED && hq_jit_enabled();
   KPlan kp;
@@ -562,7 +609,8 @@ static void launch_pipeline(hq_ctx* ctx, hq_result* r, int64_t group_cap, int64_
   }
   if (jit) hq_jit_prepare(ctx, kp, smem);  // compile (cached) outside the timed launch
   if (ctx->timing) HQ_CUDA(cudaEventRecord(e0, ctx->stream));
-  if (jit) hq_jit_launch(ctx, kp, grid, smem);
+  if (r->stream_block > 0) launch_streamed(ctx, r, kp, jit, smem);
+  else if (jit) hq_jit_launch(ctx, kp, grid, smem);
   else launch_fused(ctx, kp, grid, smem);
   if (ctx->timing) {
     HQ_CUDA(cudaEventRecord(e1, ctx->stream));
@@ -575,6 +623,8 @@ void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r) {
   r->plan = *plan;
   r->sink = plan->sink;
   r->dstate = DevBuf(ctx, 32);
+  if (r->fact->host_stream && plan->exec != HQ_EXEC_FUSED && plan->exec != HQ_EXEC_FUSED_INTERP)
+    HQ_THROW(HQ_ERR_UNSUPPORTED, "HQ_HOST_STREAM fact tables stream through the fused kernel only");
   if (plan->exec == HQ_EXEC_OAAT) {
     hq_run_oaat(ctx, plan, r);
     return;

@@ -181,12 +181,14 @@ class Engine:
     """
 
     def __init__(self, ctx: hq.Context, tables: Dict[str, hq.Table], exec_mode: int = hq.EXEC_FUSED,
-                 resolution: int = hq.RES_LRGP, fact_range: Optional[Tuple[int, int]] = None):
+                 resolution: int = hq.RES_LRGP, fact_range: Optional[Tuple[int, int]] = None,
+                 stream_block: Optional[int] = None):
         self.ctx = ctx
         self.tables = tables
         self.exec_mode = exec_mode
         self.resolution = resolution
         self.fact_range = fact_range
+        self.stream_block = stream_block  # rows per block for host-streamed fact tables
 
     def table(self, name: str) -> hq.Table:
         return self.tables[name]
@@ -236,7 +238,8 @@ class Engine:
         P.resolution = self.resolution
         if partitioned and self.fact_range is not None:
             P.row_begin, P.row_end = self.fact_range
-        return self.ctx.run(P, keep=pb.keep)
+        block = self.stream_block if getattr(pb.fact, "host_stream", False) else None
+        return self.ctx.run(P, keep=pb.keep, block_rows=block)
 
     def finish(self, res: hq.Result, pb: PlanBuilder) -> QueryResult:
         return fetch(res, pb.result_names)

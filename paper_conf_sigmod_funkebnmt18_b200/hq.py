@@ -23,7 +23,8 @@ HQ_ERR_UNSUPPORTED, HQ_ERR_OVERFLOW, HQ_ERR_STATE, HQ_ERR_NO_DEVICE = -5, -6, -7
 HQ_I8, HQ_I32, HQ_I64, HQ_F64 = 1, 3, 4, 5
 MAX_COLS, MAX_OPS, MAX_PAYLOAD, MAX_KEYS, MAX_AGGS = 16, 16, 3, 4, 8
 MAX_OUT, MAX_TMP, MAX_INSN, MAX_PREDS, MAX_ORDER = 8, 8, 16, 8, 4
-HQ_HOST_COPY, HQ_DEVICE_BORROW = 1, 2
+HQ_HOST_COPY, HQ_DEVICE_BORROW, HQ_HOST_STREAM = 1, 2, 3
+STREAM_BLOCK_ROWS = 1 << 24
 EQ, NE, LT, LE, GT, GE, BETWEEN, IN_BITMAP = 1, 2, 3, 4, 5, 6, 7, 8
 OP_FILTER, OP_PROBE, OP_COMPUTE = 1, 2, 3
 PROBE_INNER, PROBE_SEMI, PROBE_ANTI, PROBE_OUTER = 0, 1, 2, 3
@@ -116,7 +117,8 @@ EXPORTS = ["hq_ctx_create", "hq_ctx_destroy", "hq_ctx_set_stream", "hq_ctx_sync"
            "hq_abi_version", "hq_sizeof", "hq_ctx_enable_timing", "hq_ctx_kernel_times", "hq_ctx_launches",
            "hq_load_columns",
            "hq_table_info", "hq_table_column", "hq_free_table", "hq_build_hash", "hq_build_hashes", "hq_hash_info",
-           "hq_hash_device_view", "hq_hash_import", "hq_free_hash", "hq_run_pipeline", "hq_finalize",
+           "hq_hash_device_view", "hq_hash_import", "hq_free_hash", "hq_run_pipeline", "hq_run_pipeline_streamed",
+           "hq_finalize",
            "hq_result_info_get", "hq_fetch_result", "hq_result_as_table", "hq_result_partials_view",
            "hq_free_result"]
 
@@ -151,6 +153,7 @@ def lib():
             "hq_hash_info": [vp, vp, P(HashMeta)], "hq_hash_device_view": [vp, P(vp), P(HashMeta)],
             "hq_hash_import": [vp, P(HashMeta), vp, P(vp)], "hq_free_hash": [vp],
             "hq_run_pipeline": [vp, P(Plan), P(vp)], "hq_finalize": [vp, vp],
+            "hq_run_pipeline_streamed": [vp, P(Plan), i64, P(vp)],
             "hq_result_info_get": [vp, vp, P(ResultInfo)],
             "hq_fetch_result": [vp, vp, P(vp), i64, P(i64)],
             "hq_result_as_table": [vp, vp, P(vp)],
@@ -245,8 +248,11 @@ class Context:
             pass
 
     # -- objects
-    def load_columns(self, cols: Dict[str, object], host_copy: Optional[bool] = None) -> "Table":
-        return Table.load(self, cols, host_copy)
+    def load_columns(self, cols: Dict[str, object], host_copy: Optional[bool] = None,
+                     stream: bool = False) -> "Table":
+        """stream=True: the host arrays stay where they are (HQ_HOST_STREAM); pipelines over
+        the table stream it in blocks (pin them, e.g. torch pinned CPU tensors, to overlap)."""
+        return Table.load(self, cols, host_copy, stream)
 
     @staticmethod
     def _build_desc(d: "BuildDesc", src: "Table", key: int, payload: Sequence[int], preds: Sequence[Pred],
@@ -286,24 +292,35 @@ class Context:
         check(lib().hq_hash_import(self.h, ctypes.byref(meta), ctypes.c_void_p(dev_ptr), ctypes.byref(h)))
         return Hash(self, h, keep=[keep])
 
-    def run(self, plan: Plan, keep=()) -> "Result":
+    def run(self, plan: Plan, keep=(), block_rows: Optional[int] = None) -> "Result":
+        """Enqueue a pipeline.  block_rows: batch processing of an HQ_HOST_STREAM fact
+        table with this many rows per block (None: the library default)."""
         h = ctypes.c_void_p()
-        check(lib().hq_run_pipeline(self.h, ctypes.byref(plan), ctypes.byref(h)))
+        if block_rows is None:
+            check(lib().hq_run_pipeline(self.h, ctypes.byref(plan), ctypes.byref(h)))
+        else:
+            check(lib().hq_run_pipeline_streamed(self.h, ctypes.byref(plan), int(block_rows), ctypes.byref(h)))
         return Result(self, h, keep=list(keep))
 
 
 class Table:
-    def __init__(self, ctx: Context, h, nrows: int, names: List[str], keep=None):
+    def __init__(self, ctx: Context, h, nrows: int, names: List[str], keep=None, host_stream: bool = False):
         self.ctx, self.h, self.nrows, self.names, self._keep = ctx, h, nrows, names, keep
+        self.host_stream = host_stream
 
     @classmethod
-    def load(cls, ctx: Context, cols: Dict[str, object], host_copy: Optional[bool] = None) -> "Table":
-        """cols: name -> numpy array (host copy) or torch CUDA tensor (borrowed)."""
+    def load(cls, ctx: Context, cols: Dict[str, object], host_copy: Optional[bool] = None,
+             stream: bool = False) -> "Table":
+        """cols: name -> numpy array (host copy) or torch CUDA tensor (borrowed); with
+        stream=True, numpy arrays or torch CPU (pinned) tensors that stay on the host."""
         names = list(cols)
         if not names:
             raise ValueError("empty table")
         arrs = list(cols.values())
         is_dev = [hasattr(a, "is_cuda") and a.is_cuda for a in arrs]
+        if stream and any(is_dev):
+            raise ValueError("stream=True takes host columns")
+        arrs = [a.numpy() if stream and hasattr(a, "numpy") else a for a in arrs]  # torch CPU -> zero-copy view
         if any(is_dev) and not all(is_dev):
             raise ValueError("mix of host and device columns")
         dev = all(is_dev)
@@ -332,10 +349,11 @@ class Table:
             carr[i].type = dt
             carr[i].data = ptr
         h = ctypes.c_void_p()
-        flags = HQ_DEVICE_BORROW if dev else HQ_HOST_COPY
+        flags = HQ_HOST_STREAM if stream else (HQ_DEVICE_BORROW if dev else HQ_HOST_COPY)
         check(lib().hq_load_columns(ctx.h, carr, len(names), n, flags, ctypes.byref(h)))
-        # host copies are async: keep the host arrays until the next sync
-        return cls(ctx, h, n, names, keep=keep)
+        # host copies are async: keep the host arrays until the next sync (streamed
+        # tables: for the table's lifetime)
+        return cls(ctx, h, n, names, keep=keep, host_stream=stream)
 
     def col(self, name: str) -> int:
         return self.names.index(name)

@@ -708,10 +708,11 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
 
 def load_tables(ctx: hq.Context, query: Query, sf: float, seed: int = hqgen.DEFAULT_SEED,
                 fact_range: Optional[tuple] = None, host: Optional[Dict[str, Dict]] = None,
-                skip_dims: bool = False) -> Dict[str, hq.Table]:
+                skip_dims: bool = False, stream_fact: bool = False) -> Dict[str, hq.Table]:
     """Generate (or take from ``host``) the referenced columns and load them onto
     the context's device.  fact_range: rows of the fact table to load (a range
-    partition).  skip_dims: load only the fact table (non-root ranks)."""
+    partition).  skip_dims: load only the fact table (non-root ranks).  stream_fact:
+    leave the fact table in host memory (HQ_HOST_STREAM, batch processing)."""
     tables = {}
     for t, cols in query.columns.items():
         if skip_dims and t != query.fact:
@@ -721,5 +722,5 @@ def load_tables(ctx: hq.Context, query: Query, sf: float, seed: int = hqgen.DEFA
         else:
             rr = fact_range if t == query.fact else None
             data = hqgen.generate(t, sf, seed, columns=cols, row_range=rr)
-        tables[t] = ctx.load_columns(data)
+        tables[t] = ctx.load_columns(data, stream=stream_fact and t == query.fact)
     return tables
