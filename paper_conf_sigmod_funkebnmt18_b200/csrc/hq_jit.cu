@@ -89,6 +89,9 @@ std::mutex g_mu;
 std::map<std::pair<int, std::string>, CUfunction> g_cache;  // (device, source) -> kernel
 
 // ------------------------------------------------------------------ codegen
+// per-warp scratch words at the end of the kernel's misc header (MISC_BYTES = 3072 in
+// hq_plan.cu; barriers, block-scan and scalar-reduction slots use < 2,800 B)
+constexpr unsigned MISC_DEP = 3072 - 128;
 std::string lit(long long v) {
   if (v == LLONG_MIN) return "HQ_LL_MIN";
   return std::to_string(v) + "LL";
@@ -538,7 +541,27 @@ std::string generate(const KPlan& kp) {
     // goes back to the producer (mbarrier.arrive releases the warp's prior
     // shared loads); the operators below run on registers only
     for (const auto& sk2 : g.stage_k) g.use(sk2.first);
-    o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
+    // The arrive must not overtake the lanes' shared loads of the stage (the
+    // producer's next TMA overwrites it): measured on B200, a bare __syncwarp +
+    // arrive let ~1 % of SSB Q4.1 runs read a refilled value.  Every lane folds
+    // its loaded registers, a ballot over the fold completes only after all
+    // loads did, and lane 0 stores the ballot before its (release) arrive.
+    const char* rf = getenv("HQ_JIT_RELFIX");  // A/B: dep (default), fence, none
+    const std::string fix = rf ? rf : "dep";
+    if (fix == "dep") {
+      o << "    { u32 f_ = 0u;\n#pragma unroll\n      for (int r = 0; r < R; ++r) f_ ^= 0u";
+      for (const auto& sk2 : g.stage_k) {
+        const std::string v = g.var(sk2.first) + "[r]";
+        if (g.width(sk2.first) == 8) o << " ^ (u32)" << v << " ^ (u32)((u64)" << v << " >> 32)";
+        else o << " ^ (u32)" << v;
+      }
+      o << ";\n      const u32 b_ = __ballot_sync(HQ_FULL, f_ == 0x9E3779B9u);\n"
+        << "      if (lane == 0) { *(volatile u32*)(smem + " << (MISC_DEP) << "u + 4u * warp) = b_; mbar_arrive(&empty[s]); } }\n";
+    } else if (fix == "fence") {
+      o << "    fence_proxy_async(); __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
+    } else {
+      o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
+    }
   }
   if (mp == 2) {  // the count kernel's flags select the rows
     const std::string f = g.val(kp.mp_flag_reg);
