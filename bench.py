@@ -259,13 +259,16 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
 
     res = {"ms": ms, "kernel_ms": kms, "launches": launches, "clocks": clk.summary(), "rows": n,
            "local_rows": b - a, "result": out}
-    # ---- e2e: host (pinned) buffers through the public API, H2D inside the timed region
+    # ---- e2e: host (pinned) buffers through the public API, H2D inside the timed region.
+    # Dimension tables are copied (HQ_HOST_COPY); the fact table streams from its pinned
+    # host buffers through the fused kernel in blocks (HQ_HOST_STREAM, batch processing:
+    # block b+1 crosses the host link while block b is processed, SURVEY.md §8(f) f4 i).
     if with_e2e:
         e2e_steps = max(1, min(steps, 3))
         h2d = sum(arr.nbytes for cols in host.values() for arr in cols.values())
 
         def e2e_step():
-            tb = {t: ctx.load_columns(cols) for t, cols in host.items()}
+            tb = {t: ctx.load_columns(cols, stream=(t == q.fact)) for t, cols in host.items()}
             Eng = make_engine(tb)
             r, pb = q.run(Eng)
             o = Eng.finish(r, pb)
@@ -290,7 +293,9 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
         res["e2e"] = {"value": n / (ems / 1e3), "unit": "rows/s", "h2d_bytes_per_step": int(h2d),
-                      "d2h_bytes_per_step": int(d2h), "ms_per_step": ems, "steps": e2e_steps}
+                      "d2h_bytes_per_step": int(d2h), "ms_per_step": ems, "steps": e2e_steps,
+                      "mode": f"fact table streamed from pinned host memory (HQ_HOST_STREAM, {hq.STREAM_BLOCK_ROWS}-row "
+                              "blocks, copies overlapped with the fused kernel); dimensions HQ_HOST_COPY"}
     res["host"] = host
     del tables, dtab, E
     ctx.close()
