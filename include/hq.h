@@ -174,6 +174,11 @@ typedef struct {
   int32_t payload_cols[HQ_MAX_PAYLOAD];
   int64_t expected_rows; /* >0: capacity sized for this many keys (no count pass, no host sync);
                             <=0: a count pass sizes the table exactly (one ctx sync) */
+  int32_t composite;     /* != 0: two-column join key (key_col, payload_cols[0]) (TPC-H Q9's
+                            (ps_partkey, ps_suppkey)): the slot is hashed on key_col, stores the
+                            second key as payload word 0 and the remaining payload columns after
+                            it; key_col alone need not be unique, the pairs must be (not checked).
+                            Always HQ_HT_LINEAR; npayload >= 1. */
 } hq_build_desc;
 /* Slot = {int32 key, payload...} of 4, 8 or 16 bytes, empty key INT32_MIN,
  * claimed with one atomicCAS on the key.  Two layouts:
@@ -205,6 +210,7 @@ typedef struct {
   int32_t key_max;      /* max key inserted (count pass); key range = [key_min, key_max] */
   uint64_t pay_set[4];  /* payload-0 values present: bit (v & 255) (count pass); exact when
                          * pay_max - pay_min < 256, all-zero when unknown (expected_rows builds) */
+  int32_t composite;    /* built with hq_build_desc::composite (payload word 0 = second key) */
 } hq_hash_meta;
 /* Derived forms (rebuilt on import): direct tables get a compact form -- a
  * bitmap of present keys for semi-join tables, or one byte per key (payload -
@@ -270,6 +276,9 @@ typedef struct {
   int32_t dst;
   int32_t ninsn;
   hq_insn code[HQ_MAX_INSN];
+  /* PROBE of a composite table: register holding the second key (compared with the
+   * slot's payload word 0); payload_dst[k] then receive payload words 1 + k. */
+  int32_t key2_reg;
 } hq_op;
 
 typedef enum { HQ_AGG_SUM = 1, HQ_AGG_COUNT, HQ_AGG_MIN, HQ_AGG_MAX, HQ_AGG_AVG } hq_agg_fn;

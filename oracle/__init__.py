@@ -74,6 +74,10 @@ class _Orders(ctypes.Structure):
                 ("totalprice", P_I64), ("orderstatus", P_I8)]
 
 
+class _Partsupp(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("partkey", P_I32), ("suppkey", P_I32), ("supplycost", P_I64)]
+
+
 class _TPart(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("partkey", P_I32), ("brand", P_I8), ("container", P_I8), ("size", P_I32)]
 
@@ -137,6 +141,8 @@ def lib():
             "orc_ssb_q31_mat": [P(_Lineorder), P(_SsbDim), P(_SsbDim), P(_Date), ctypes.c_int, ctypes.c_int],
             "orc_ssb_q41": [P(_Lineorder), P(_Date), P(_SsbDim), P(_SsbDim), P(_Part), ctypes.c_int, ctypes.c_int],
             "orc_tpch_q3": [P(_TCustomer), P(_Orders), P(_Lineitem), ctypes.c_int, ctypes.c_int],
+            "orc_tpch_q9": [P(_TPart), P(_TSupplier), P(_Lineitem), P(_Partsupp), P(_Orders), P(_Nation),
+                            ctypes.c_int32, ctypes.c_int, ctypes.c_int],
             "orc_tpch_q4": [P(_Orders), P(_Lineitem), ctypes.c_int, ctypes.c_int],
             "orc_tpch_q13": [P(_TCustomer), P(_Orders), ctypes.c_int],
             "orc_tpch_q17": [P(_TPart), P(_Lineitem), ctypes.c_int],
@@ -407,6 +413,31 @@ def tpch_q7(customer, orders, lineitem, supplier, nation, brute=False, nthreads=
                                  ctypes.byref(_lineitem(lineitem, keep)), ctypes.byref(_tsupp(supplier, keep)),
                                  ctypes.byref(_nation(nation, keep)), int(brute), nthreads],
                  ["supp_nation", "cust_nation", "l_year", "revenue", "count"])
+
+
+def _partsupp(t, keep):
+    s = _Partsupp()
+    s.n = _n(t)
+    s.partkey = _ptr(t["ps_partkey"], P_I32, keep)
+    s.suppkey = _ptr(t["ps_suppkey"], P_I32, keep)
+    s.supplycost = _ptr(t["ps_supplycost"], P_I64, keep)
+    return s
+
+
+def q9_pmax(nparts: int) -> int:
+    """DESIGN.md R19: App F's p_partkey filter for p_name like '%green%' keeps the LIKE's
+    selectivity, 5 of 92 colour words: p_partkey <= |part| * 5 // 92."""
+    return int(nparts) * 5 // 92
+
+
+def tpch_q9(part, supplier, lineitem, partsupp, orders, nation, pmax=None, brute=False, nthreads=1) -> OracleResult:
+    """TPC-H Q9 (App F) -> [nation, o_year, sum_profit (scale 4), count] ORDER BY nation, o_year desc."""
+    keep = []
+    pmax = q9_pmax(_n(part)) if pmax is None else int(pmax)
+    return _call("orc_tpch_q9", [ctypes.byref(_tpart(part, keep)), ctypes.byref(_tsupp(supplier, keep)),
+                                 ctypes.byref(_lineitem(lineitem, keep)), ctypes.byref(_partsupp(partsupp, keep)),
+                                 ctypes.byref(_orders(orders, keep)), ctypes.byref(_nation(nation, keep)), pmax,
+                                 int(brute), nthreads], ["nation", "o_year", "sum_profit", "count"])
 
 
 def tpch_q4(orders, lineitem, brute=False, nthreads=1) -> OracleResult:

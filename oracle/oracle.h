@@ -66,6 +66,8 @@ typedef struct {
   const int64_t* totalprice;
   const int8_t* orderstatus;
 } orc_orders;
+/* TPC-H partsupp (4 rows per part): supplycost int64 cents */
+typedef struct { int64_t n; const int32_t *partkey, *suppkey; const int64_t* supplycost; } orc_partsupp;
 /* TPC-H part: brand 'Brand#MN' = (M-1)*5 + N-1; container = code in string order (hqgen) */
 typedef struct { int64_t n; const int32_t* partkey; const int8_t *brand, *container; const int32_t* size; } orc_tpch_part;
 typedef struct { int64_t n; const int32_t* custkey; const int8_t *mktsegment, *nationkey; } orc_tpch_customer;
@@ -159,6 +161,12 @@ int orc_tpch_q19(const orc_tpch_part* p, const orc_lineitem* li, int brute, int 
  * [s_suppkey, numwait] ORDER BY numwait desc, s_suppkey (s_name depends on s_suppkey, R18) */
 int orc_tpch_q21(int variant, const orc_tpch_supplier* s, const orc_orders* o, const orc_lineitem* li,
                  const orc_nation* n, int brute, orc_result* out);
+
+/* TPC-H Q9 (product type profit) with PAPER.md App F's rewrite of p_name like '%green%' as a
+ * filter on p_partkey (R19: p_partkey <= pmax) -> rows [nation, o_year,
+ * sum_profit (scale 4), count] ORDER BY nation, o_year desc */
+int orc_tpch_q9(const orc_tpch_part* p, const orc_tpch_supplier* s, const orc_lineitem* li, const orc_partsupp* ps,
+                const orc_orders* o, const orc_nation* n, int32_t pmax, int brute, int nthreads, orc_result* out);
 
 void orc_free(orc_result* r);
 

@@ -40,6 +40,7 @@ struct KBuild {
   void* part;        // count pass: per-block partials (CountPart[grid])
   unsigned* ticket;  // count pass: blocks done
   int count_inserts; // build pass: accumulate the inserted-key count (no count pass ran)
+  int composite;     // two-column key: equal key_col values take separate slots (no dup check)
 };
 
 __device__ __forceinline__ long long ld_col(const KBuild& b, int c, long long row) {
@@ -265,7 +266,7 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid
         ++inserted;
         break;
       }
-      if (old == key || b.direct) {
+      if (!b.composite && (old == key || b.direct)) {
         fault |= HQF_DUP_KEY;  // join keys must be unique (R6)
         break;
       }
@@ -350,6 +351,8 @@ void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& 
   for (int i = 0; i < d->npreds; ++i) to_kpred(d->preds[i], b.preds[i], t->ncols);
   b.key_col = d->key_col;
   b.npay = d->npayload;
+  b.composite = d->composite != 0;
+  if (b.composite && d->npayload < 1) HQ_THROW(HQ_ERR_ARG, "build: a composite key needs payload_cols[0] (the second key)");
   for (int k = 0; k < d->npayload; ++k) {
     if (d->payload_cols[k] < 0 || d->payload_cols[k] >= t->ncols) HQ_THROW(HQ_ERR_ARG, "build: payload column out of range");
     b.pay_col[k] = d->payload_cols[k];
@@ -395,7 +398,7 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
       kmin = bs.st.kmin;
       range = (int64_t)bs.st.kmax - bs.st.kmin + 1;
       // dense keys: direct-mapped slot array (one load per probe)
-      direct = range <= (1LL << 30) && (range <= 8 * keys || range * words * 4 <= (2LL << 20));
+      direct = !b.composite && range <= (1LL << 30) && (range <= 8 * keys || range * words * 4 <= (2LL << 20));
     }
   }
   const int64_t cap = direct ? range : std::max<int64_t>(16, next_pow2((keys * 5 + 2) / 3));  // load <= 0.6
@@ -408,6 +411,7 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   h->meta.capacity = cap;
   h->meta.slot_words = words;
   h->meta.npayload = d->npayload;
+  h->meta.composite = b.composite;
   h->meta.nkeys = bs.counted ? keys : -1;  // exact after the count pass (confirmed at hq_hash_info)
   h->meta.bytes = cap * words * 4;
   h->meta.layout = direct ? HQ_HT_DIRECT : HQ_HT_LINEAR;

@@ -223,6 +223,8 @@ struct KProbe {
   const uint32_t* pf;  // linear tables: key-range bitmap (NULL = none)
   int32_t pf_min;
   uint32_t pf_range;
+  uint8_t composite;   // two-column key: slot word 1 must equal key2_reg; payloads from word 2
+  int16_t key2_reg;
 };
 struct KCompute {
   int16_t dst;

@@ -281,9 +281,14 @@ struct Gen {
     const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
     probe_defs(pr);
     const std::string key = val(pr.key_reg);
-    o << "      { const u32* ht_ = p.ht[" << idx << "]; u32 found_ = 0u; int kk_[R]; u32 pend_ = 0u; u32 pos_[R];\n"
+    // composite keys: the slot's word 1 must also equal the second key (TPC-H Q9)
+    const bool cmp2 = pr.composite;
+    const std::string key2 = cmp2 ? val(pr.key2_reg) : std::string();
+    o << "      { const u32* ht_ = p.ht[" << idx << "]; u32 found_ = 0u; int kk_[R]; u32 pend_ = 0u; u32 pos_[R];"
+      << (cmp2 ? " int kk2_[R];" : "") << "\n"
       << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n"
       << "          const long long k_ = (long long)" << key << "; kk_[r] = (int)k_;\n";
+    if (cmp2) o << "          kk2_[r] = (int)(long long)" << key2 << ";\n";
     const int G = W == 1 ? 4 : (W == 2 ? 2 : 1);
     o << "          bool ok_ = ((mask >> r) & 1u) && k_ > (long long)HQ_INT_MIN && k_ <= (long long)HQ_INT_MAX;\n";
     if (pr.pf) {  // exact key-range bitmap first: misses mostly stop here (L2-resident)
@@ -300,7 +305,9 @@ struct Gen {
     const char* keys4[4] = {"x", "y", "z", "w"};
     for (int j = 0; j < G; ++j) {
       const char* kc = G == 4 ? keys4[j] : (G == 2 ? (j == 0 ? "x" : "z") : "x");
-      o << "            if (!stop_ && " << j << " >= first_) { if (sl_[r]." << kc << " == kk_[r]) { hit_ = " << j
+      const char* k2c = G == 2 ? (j == 0 ? "y" : "w") : "y";  // composite: the slot's word 1
+      const std::string m2 = cmp2 ? std::string(" && sl_[r].") + k2c + " == kk2_[r]" : std::string();
+      o << "            if (!stop_ && " << j << " >= first_) { if (sl_[r]." << kc << " == kk_[r]" << m2 << ") { hit_ = " << j
         << "; stop_ = true; } else if (sl_[r]." << kc << " == HQ_INT_MIN) stop_ = true; }\n";
     }
     o << "            if (hit_ >= 0) { found_ |= 1u << r; pend_ &= ~(1u << r);\n";
@@ -308,7 +315,8 @@ struct Gen {
       if (G == 2) o << "              " << var(pr.dst[0]) << "[r] = hit_ == 0 ? sl_[r].y : sl_[r].w;\n";
       else {
         static const char* comp[3] = {"y", "z", "w"};
-        for (int k = 0; k < npay; ++k) o << "              " << var(pr.dst[k]) << "[r] = sl_[r]." << comp[k] << ";\n";
+        for (int k = 0; k < npay; ++k)
+          o << "              " << var(pr.dst[k]) << "[r] = sl_[r]." << comp[k + (cmp2 ? 1 : 0)] << ";\n";
       }
     }
     o << "            } else if (stop_) pend_ &= ~(1u << r);\n"
@@ -389,7 +397,10 @@ struct Gen {
     for (int j = from; j < kp.nops; ++j) {
       const KOp& op = kp.ops[j];
       if (op.kind == OP_FILTER) u.insert(kp.preds[op.idx].reg);
-      else if (op.kind == OP_PROBE) u.insert(kp.probes[op.idx].key_reg);
+      else if (op.kind == OP_PROBE) {
+        u.insert(kp.probes[op.idx].key_reg);
+        if (kp.probes[op.idx].composite) u.insert(kp.probes[op.idx].key2_reg);
+      }
       else {
         const KCompute& c = kp.comps[op.idx];
         for (int k = 0; k < c.n; ++k)

@@ -52,9 +52,11 @@ __global__ void hq_oaat_filter(const char* in, int w, KPred f, long long n, int*
   }
 }
 // join probe primitive: flag + payload per row
-__global__ void hq_oaat_probe(const char* key, int w, KProbe pr, long long n, int* flags, int* p0, int* p1, int* p2) {
+__global__ void hq_oaat_probe(const char* key, int w, const char* key2, int w2, KProbe pr, long long n, int* flags,
+                              int* p0, int* p1, int* p2) {
   GRID_STRIDE(i, n) {
     const long long kv = ldw(key, w, i);
+    const int k2 = pr.composite ? (int)ldw(key2, w2, i) : 0;  // composite: slot word 1 = second key
     int hit = 0, pay[3] = {0, 0, 0};
     if (kv > (long long)INT_MIN && kv <= (long long)INT_MAX) {
       const int k = (int)kv;
@@ -71,9 +73,9 @@ __global__ void hq_oaat_probe(const char* key, int w, KProbe pr, long long n, in
         uint32_t pos = ((uint32_t)k * 0x9E3779B1u) >> (32u - pr.log2cap);
         for (uint32_t t = 0; t <= pr.mask; ++t) {
           const uint32_t* s = pr.slots + (size_t)pos * pr.words;
-          if ((int)s[0] == k) {
+          if ((int)s[0] == k && (!pr.composite || (int)s[1] == k2)) {
             hit = 1;
-            for (int j = 0; j < pr.npay; ++j) pay[j] = (int)s[1 + j];
+            for (int j = 0; j < pr.npay; ++j) pay[j] = (int)s[1 + pr.composite + j];
             break;
           }
           if ((int)s[0] == INT_MIN) break;
@@ -290,11 +292,13 @@ void hq_run_oaat(hq_ctx* ctx, const hq_plan* plan, hq_result* r) {
     } else if (op.kind == OP_PROBE) {
       const KProbe& pr = kp.probes[op.idx];
       Mat& in = get(pr.key_reg);
+      const Mat* in2 = pr.composite ? &get(pr.key2_reg) : nullptr;
       DevBuf flags(ctx, (size_t)std::max<long long>(n, 1) * 4);
       DevBuf pay[3];
       for (int j = 0; j < pr.npay; ++j) pay[j] = DevBuf(ctx, (size_t)std::max<long long>(n, 1) * 4);
       ctx->launches++;
-      hq_oaat_probe<<<grid_for(ctx, n), 256, 0, st>>>(in.p, in.w, pr, n, flags.as<int>(), pay[0].as<int>(),
+      hq_oaat_probe<<<grid_for(ctx, n), 256, 0, st>>>(in.p, in.w, in2 ? in2->p : nullptr, in2 ? in2->w : 4, pr, n,
+                                                      flags.as<int>(), pay[0].as<int>(),
                                                       pay[1].as<int>(), pay[2].as<int>());
       for (int j = 0; j < pr.npay; ++j) {
         Mat& m = mats[pr.dst[j]];

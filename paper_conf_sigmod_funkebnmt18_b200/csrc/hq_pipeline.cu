@@ -175,7 +175,7 @@ __device__ __forceinline__ uint32_t op_filter(const KPlan& p, int idx, const cha
 // order, so a warp's round count is rarely more than one.
 template <int R, int W>
 __device__ __forceinline__ uint32_t probe_rows(const KPlan& p, const KProbe& pr, const long long (&kv)[R],
-                                               char* tmp, int row0, uint32_t mask) {
+                                               const long long (&kv2)[R], char* tmp, int row0, uint32_t mask) {
   uint32_t pending = mask, found = 0;
   uint32_t pos[R];
 #pragma unroll
@@ -230,7 +230,7 @@ __device__ __forceinline__ uint32_t probe_rows(const KPlan& p, const KProbe& pr,
 #pragma unroll
         for (int j = 0; j < G; ++j) {
           if (!stop && j >= first) {
-            if (sk[j] == key) { hit = j; stop = true; }
+            if (sk[j] == key && (!pr.composite || (G == 1 ? sl[r].y : sp0[j]) == (int)kv2[r])) { hit = j; stop = true; }
             else if (sk[j] == INT_MIN) stop = true;
           }
         }
@@ -243,9 +243,14 @@ __device__ __forceinline__ uint32_t probe_rows(const KPlan& p, const KProbe& pr,
 #pragma unroll
             for (int j = 1; j < G; ++j)
               if (hit == j) v0 = sp0[j];
-            if (pr.npay > 0) dst0[r * 32] = v0;
-            if (W > 2 && pr.npay > 1) dst1[r * 32] = sp1;
-            if (W > 2 && pr.npay > 2) dst2[r * 32] = sp2;
+            if (pr.composite) {  // word 1 is the second key: payloads are words 2, 3
+              if (W > 2 && pr.npay > 0) dst0[r * 32] = sp1;
+              if (W > 2 && pr.npay > 1) dst1[r * 32] = sp2;
+            } else {
+              if (pr.npay > 0) dst0[r * 32] = v0;
+              if (W > 2 && pr.npay > 1) dst1[r * 32] = sp1;
+              if (W > 2 && pr.npay > 2) dst2[r * 32] = sp2;
+            }
           }
         } else if (stop) {
           pending &= ~(1u << r);
@@ -264,11 +269,12 @@ template <int R>
 __device__ __forceinline__ uint32_t op_probe(const KPlan& p, int idx, const char* stage, char* tmp, int row0,
                                              uint32_t mask) {
   const KProbe& pr = p.probes[idx];
-  long long kv[R];
+  long long kv[R], kv2[R];
   load_rows<R>(p, pr.key_reg, stage, tmp, row0, kv);
-  if (pr.words == 1) return probe_rows<R, 1>(p, pr, kv, tmp, row0, mask);
-  if (pr.words == 2) return probe_rows<R, 2>(p, pr, kv, tmp, row0, mask);
-  return probe_rows<R, 4>(p, pr, kv, tmp, row0, mask);
+  if (pr.composite) load_rows<R>(p, pr.key2_reg, stage, tmp, row0, kv2);
+  if (pr.words == 1) return probe_rows<R, 1>(p, pr, kv, kv2, tmp, row0, mask);
+  if (pr.words == 2) return probe_rows<R, 2>(p, pr, kv, kv2, tmp, row0, mask);
+  return probe_rows<R, 4>(p, pr, kv, kv2, tmp, row0, mask);
 }
 
 // Projection / arithmetic (revenue[wp] = price[tid]*discount[tid]):

@@ -147,7 +147,16 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.words = (uint8_t)op.ht->meta.slot_words;
       pr.mode = (uint8_t)op.mode;
       const int npay = hq_probe_has_payload(op.mode) ? op.npayload : 0;
-      if (npay < 0 || npay > op.ht->meta.npayload) HQ_THROW(HQ_ERR_ARG, "plan: probe asks for more payload words than the table holds");
+      pr.composite = op.ht->meta.composite ? 1 : 0;
+      pr.key2_reg = 0;
+      if (pr.composite) {  // two-column key: payload word 0 is the second key
+        pr.key2_reg = (int16_t)use(op.key2_reg, "probe second key");
+        pr.pay_min = 1;  // payload ranges of the count pass describe the second key, not the payloads
+        pr.pay_max = 0;
+        for (int k = 0; k < 4; ++k) pr.pay_set[k] = 0;
+      }
+      if (npay < 0 || npay > op.ht->meta.npayload - pr.composite)
+        HQ_THROW(HQ_ERR_ARG, "plan: probe asks for more payload words than the table holds");
       pr.npay = (uint8_t)npay;
       for (int k = 0; k < npay; ++k) pr.dst[k] = (int16_t)def(op.payload_dst[k], 4, "probe payload");
       kp.ops[o] = {OP_PROBE, (uint8_t)nprobe++};
@@ -399,6 +408,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         exec = mp_pass == 1;
         for (int k = 0; mp_pass == 2 && hq_probe_has_payload(pr.mode) && k < pr.npay; ++k) exec = exec || need[pr.dst[k]];
         if (exec) need[pr.key_reg] = true;
+        if (exec && pr.composite) need[pr.key2_reg] = true;
       } else {
         const KCompute& c = kp.comps[op.idx];
         exec = need[c.dst];

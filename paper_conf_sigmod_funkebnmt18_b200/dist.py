@@ -91,7 +91,7 @@ class DistributedEngine(Engine):
             self._built.append(h)     # build faults are checked in finish()
             buf = device_view(ptr, int(m.bytes))
             meta = [m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout,
-                    m.pay_min, m.pay_max, m.key_max] + [_i64(w) for w in m.pay_set]
+                    m.pay_min, m.pay_max, m.key_max] + [_i64(w) for w in m.pay_set] + [m.composite]
         else:
             meta, buf = None, None
         meta, buf = broadcast_blob(meta, buf, 4, self.root, self.device)
@@ -102,10 +102,11 @@ class DistributedEngine(Engine):
          hm.pay_min, hm.pay_max, hm.key_max) = meta[:10]
         for k in range(4):
             hm.pay_set[k] = meta[10 + k] & 0xFFFFFFFFFFFFFFFF
+        hm.composite = meta[14]
         return self.ctx.import_hash(hm, buf.data_ptr(), keep=buf)
 
-    def hash(self, table, key, payload=(), preds=(), expected_rows=0) -> hq.Hash:
-        h = super().hash(table, key, payload, preds, expected_rows) if self.rank == self.root else None
+    def hash(self, table, key, payload=(), preds=(), expected_rows=0, key2=None) -> hq.Hash:
+        h = super().hash(table, key, payload, preds, expected_rows, key2) if self.rank == self.root else None
         return self._share(h)
 
     def hashes(self, specs) -> List[hq.Hash]:

@@ -66,11 +66,15 @@ class PlanBuilder:
         op.filter = hq.make_pred(self.reg(col), cmp, lo, hi)
         return self
 
-    def probe(self, ht: hq.Hash, key: str, mode: str = "inner", payload: Sequence[str] = ()) -> "PlanBuilder":
+    def probe(self, ht: hq.Hash, key: str, mode: str = "inner", payload: Sequence[str] = (),
+              key2: Optional[str] = None) -> "PlanBuilder":
+        """key2: the second key register of a composite (two-column) join key."""
         op = self._op()
         op.kind = hq.OP_PROBE
         op.ht = ht.h
         op.key_reg = self.reg(key)
+        if key2 is not None:
+            op.key2_reg = self.reg(key2)
         op.mode = {"inner": hq.PROBE_INNER, "semi": hq.PROBE_SEMI, "anti": hq.PROBE_ANTI, "outer": hq.PROBE_OUTER}[mode]
         op.npayload = len(payload)
         for i, name in enumerate(payload):
@@ -209,10 +213,12 @@ class Engine:
         return pb
 
     def hash(self, table: str, key: str, payload: Sequence[str] = (),
-             preds: Sequence[Tuple] = (), expected_rows: int = 0) -> hq.Hash:
+             preds: Sequence[Tuple] = (), expected_rows: int = 0, key2: Optional[str] = None) -> hq.Hash:
+        """key2: second column of a composite join key (e.g. (ps_partkey, ps_suppkey))."""
         t = self.tables[table]
         ps = [hq.make_pred(t.col(p[0]), *p[1:]) for p in preds]
-        return self.ctx.build_hash(t, t.col(key), [t.col(c) for c in payload], ps, expected_rows)
+        return self.ctx.build_hash(t, t.col(key), [t.col(c) for c in payload], ps, expected_rows,
+                                   None if key2 is None else t.col(key2))
 
     def hashes(self, specs: Sequence[dict]) -> List[hq.Hash]:
         """Independent builds (a query's dimension tables) with one host sync:
@@ -221,7 +227,9 @@ class Engine:
         for sp in specs:
             t = self.tables[sp["table"]]
             ps = [hq.make_pred(t.col(p[0]), *p[1:]) for p in sp.get("preds", ())]
-            out.append((t, t.col(sp["key"]), [t.col(c) for c in sp.get("payload", ())], ps, sp.get("expected_rows", 0)))
+            k2 = sp.get("key2")
+            out.append((t, t.col(sp["key"]), [t.col(c) for c in sp.get("payload", ())], ps, sp.get("expected_rows", 0),
+                        None if k2 is None else t.col(k2)))
         return self.ctx.build_hashes(out)
 
     def hash_from(self, res: Optional[hq.Result], names: Sequence[str], key: str,

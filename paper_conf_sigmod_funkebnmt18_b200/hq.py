@@ -59,14 +59,15 @@ class Pred(ctypes.Structure):
 class BuildDesc(ctypes.Structure):
     _fields_ = [("src", ctypes.c_void_p), ("npreds", ctypes.c_int32), ("preds", Pred * MAX_PREDS),
                 ("key_col", ctypes.c_int32), ("npayload", ctypes.c_int32),
-                ("payload_cols", ctypes.c_int32 * MAX_PAYLOAD), ("expected_rows", ctypes.c_int64)]
+                ("payload_cols", ctypes.c_int32 * MAX_PAYLOAD), ("expected_rows", ctypes.c_int64),
+                ("composite", ctypes.c_int32)]
 
 
 class HashMeta(ctypes.Structure):
     _fields_ = [("capacity", ctypes.c_int64), ("slot_words", ctypes.c_int32), ("npayload", ctypes.c_int32),
                 ("nkeys", ctypes.c_int64), ("bytes", ctypes.c_int64), ("key_min", ctypes.c_int64),
                 ("layout", ctypes.c_int32), ("pay_min", ctypes.c_int32), ("pay_max", ctypes.c_int32),
-                ("key_max", ctypes.c_int32), ("pay_set", ctypes.c_uint64 * 4)]
+                ("key_max", ctypes.c_int32), ("pay_set", ctypes.c_uint64 * 4), ("composite", ctypes.c_int32)]
 
 
 class Insn(ctypes.Structure):
@@ -77,7 +78,7 @@ class Op(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("filter", Pred), ("ht", ctypes.c_void_p),
                 ("key_reg", ctypes.c_int32), ("mode", ctypes.c_int32), ("npayload", ctypes.c_int32),
                 ("payload_dst", ctypes.c_int32 * MAX_PAYLOAD), ("dst", ctypes.c_int32),
-                ("ninsn", ctypes.c_int32), ("code", Insn * MAX_INSN)]
+                ("ninsn", ctypes.c_int32), ("code", Insn * MAX_INSN), ("key2_reg", ctypes.c_int32)]
 
 
 class Plan(ctypes.Structure):
@@ -256,8 +257,13 @@ class Context:
 
     @staticmethod
     def _build_desc(d: "BuildDesc", src: "Table", key: int, payload: Sequence[int], preds: Sequence[Pred],
-                    expected_rows: int) -> None:
+                    expected_rows: int, key2: Optional[int] = None) -> None:
+        """key2: second key column of a composite (two-column) join key; it is stored
+        as payload word 0, ahead of `payload`."""
         d.src = src.h
+        if key2 is not None:
+            payload = [key2] + list(payload)
+            d.composite = 1
         if len(preds) > MAX_PREDS:
             raise ValueError("too many build predicates")
         d.npreds = len(preds)
@@ -270,9 +276,9 @@ class Context:
         d.expected_rows = expected_rows
 
     def build_hash(self, src: "Table", key: int, payload: Sequence[int] = (), preds: Sequence[Pred] = (),
-                   expected_rows: int = 0) -> "Hash":
+                   expected_rows: int = 0, key2: Optional[int] = None) -> "Hash":
         d = BuildDesc()
-        self._build_desc(d, src, key, payload, preds, expected_rows)
+        self._build_desc(d, src, key, payload, preds, expected_rows, key2)
         h = ctypes.c_void_p()
         check(lib().hq_build_hash(self.h, ctypes.byref(d), ctypes.byref(h)))
         return Hash(self, h, keep=[src])
@@ -281,8 +287,8 @@ class Context:
         """Several builds, one host sync: specs = [(src, key, payload, preds, expected_rows), ...]."""
         n = len(specs)
         ds = (BuildDesc * n)()
-        for d, (src, key, payload, preds, exp) in zip(ds, specs):
-            self._build_desc(d, src, key, payload, preds, exp)
+        for d, spec in zip(ds, specs):
+            self._build_desc(d, *spec)
         hs = (ctypes.c_void_p * n)()
         check(lib().hq_build_hashes(self.h, n, ds, hs))
         return [Hash(self, ctypes.c_void_p(hs[i]), keep=[specs[i][0]]) for i in range(n)]

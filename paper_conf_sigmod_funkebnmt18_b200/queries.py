@@ -593,6 +593,43 @@ def _tpch_q21(E: Engine, variant: int = 0, limit: int = 100, **_):
     return res, pl
 
 
+# select nation, o_year, sum(amount) as sum_profit
+# from (select n_name as nation, extract(year from o_orderdate) as o_year,
+#              l_extendedprice * (1 - l_discount) - ps_supplycost * l_quantity as amount
+#       from part, supplier, lineitem, partsupp, orders, nation
+#       where s_suppkey = l_suppkey and ps_suppkey = l_suppkey and ps_partkey = l_partkey
+#         and p_partkey = l_partkey and o_orderkey = l_orderkey and s_nationkey = n_nationkey
+#         and p_name like '%green%') as profit
+# group by nation, o_year order by nation, o_year desc
+# App F: the LIKE becomes a filter on p_partkey, p_partkey <= |part| * 5 // 92 (R19),
+# pushed into the partsupp build through p_partkey = ps_partkey.  partsupp is joined on its
+# two-column key (ps_partkey, ps_suppkey): a composite hash table (hq_build_desc::composite).
+def _tpch_q9(E: Engine, pmax: Optional[int] = None, **_):
+    if pmax is None:
+        pmax = E.table("tpch_part").nrows * 5 // 92
+    hp, hps, hs, hn, ho = E.hashes([
+        dict(table="tpch_part", key="p_partkey", preds=[("p_partkey", "<=", pmax)]),
+        dict(table="partsupp", key="ps_partkey", key2="ps_suppkey", payload=["ps_supplycost"],
+             preds=[("ps_partkey", "<=", pmax)]),
+        dict(table="tpch_supplier", key="s_suppkey", payload=["s_nationkey"]),
+        dict(table="nation", key="n_nationkey"),
+        dict(table="orders", key="o_orderkey", payload=["o_orderdate"])])
+    pl = E.plan("lineitem")
+    pl.probe(hp, "l_partkey", "semi")                                           # 5/92
+    pl.probe(hps, "l_partkey", "inner", ["ps_supplycost"], key2="l_suppkey")
+    pl.probe(hs, "l_suppkey", "inner", ["s_nationkey"])
+    pl.probe(hn, "s_nationkey", "semi")
+    pl.probe(ho, "l_orderkey", "inner", ["o_orderdate"])
+    pl.compute("o_year", [("load", "o_orderdate"), ("div", 10000)])
+    pl.compute("cost", [("load", "ps_supplycost"), ("mul", "l_quantity")])   # scale 4
+    pl.compute("amount", [("load", "l_discount"), ("rsub", 100), ("mul", "l_extendedprice"), ("sub", "cost")])
+    pl.aggregate(keys=[("s_nationkey", 0, 25), ("o_year", 1992, 7)], aggs=[("sum", "amount"), ("count", None)],
+                 order=[("s_nationkey", False), ("o_year", True)], agg_names=["sum_profit", "count"])
+    res = E.run(pl)
+    pl.result_names = ["nation"] + pl.result_names[1:]
+    return res, pl
+
+
 # ------------------------------------------------ paper micro queries (f2)
 def _micro_select(E: Engine, x: int = 5, resolution=None, **_):
     """PAPER.md Fig 16 'Query 1': selection + projection, materialised."""
@@ -681,6 +718,11 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
     Query("tpch_q4", "tpch", "lineitem",
           {"lineitem": ["l_orderkey", "l_commitdate", "l_receiptdate"],
            "orders": ["o_orderkey", "o_orderdate", "o_orderpriority"]}, _tpch_q4),
+    Query("tpch_q9", "tpch", "lineitem",
+          {"lineitem": ["l_orderkey", "l_partkey", "l_suppkey", "l_quantity", "l_extendedprice", "l_discount"],
+           "orders": ["o_orderkey", "o_orderdate"], "tpch_part": ["p_partkey"],
+           "partsupp": ["ps_partkey", "ps_suppkey", "ps_supplycost"], "tpch_supplier": ["s_suppkey", "s_nationkey"],
+           "nation": ["n_nationkey"]}, _tpch_q9),
     Query("tpch_q13", "tpch", "orders",
           {"orders": ["o_custkey"], "tpch_customer": ["c_custkey"]}, _tpch_q13),
     Query("tpch_q17", "tpch", "lineitem",

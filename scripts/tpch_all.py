@@ -25,7 +25,7 @@ from paper_conf_sigmod_funkebnmt18_b200 import hq  # noqa: E402
 from paper_conf_sigmod_funkebnmt18_b200.engine import Engine  # noqa: E402
 from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES, load_tables  # noqa: E402
 
-TPCH = ["tpch_q1", "tpch_q3", "tpch_q4", "tpch_q5", "tpch_q6", "tpch_q7", "tpch_q10", "tpch_q13", "tpch_q17",
+TPCH = ["tpch_q1", "tpch_q3", "tpch_q4", "tpch_q5", "tpch_q6", "tpch_q7", "tpch_q9", "tpch_q10", "tpch_q13", "tpch_q17",
         "tpch_q18", "tpch_q19", "tpch_q21"]
 
 

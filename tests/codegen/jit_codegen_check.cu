@@ -310,13 +310,34 @@ int main(int argc, char** argv) {
     shapes.push_back({"outer_predicates", P, nullptr});
   }
 
+  {  // composite (two-column) join key in a linear table: slot {k1, k2, payload, -} (TPC-H Q9)
+    hq_hash* comp = make_hash(c, HQ_HT_LINEAR, 2, 0, 800000, true);
+    comp->meta.composite = 1;
+    hq_plan P{};
+    P.fact = F;
+    P.row_end = -1;
+    hq_op pc = probe(comp, 1, HQ_PROBE_INNER, HQ_TMP(0));
+    pc.key2_reg = 2;
+    P.ops[P.nops++] = pc;
+    hq_op ps = probe(comp, 3, HQ_PROBE_SEMI);
+    ps.key2_reg = 0;
+    P.ops[P.nops++] = ps;
+    P.sink = HQ_SINK_AGG;
+    P.nkeys = 1;
+    P.key_reg[0] = 7; P.key_card[0] = 16;
+    P.naggs = 2;
+    P.agg_fn[0] = HQ_AGG_SUM; P.agg_reg[0] = HQ_TMP(0);
+    P.agg_fn[1] = HQ_AGG_COUNT;
+    shapes.push_back({"composite_probe", P, nullptr});
+  }
+
   // multi-pass count / write kernels (HQ_EXEC_MULTIPASS) of a grouped star
   // join, a materialising pipeline and a scalar aggregate
   {
     std::vector<Shape> mps;
     for (const Shape& s : shapes) {
       if (s.name != "star_ranked_dense" && s.name != "materialise_lrgp" && s.name != "scalar_filters" &&
-          s.name != "outer_predicates")
+          s.name != "outer_predicates" && s.name != "composite_probe")
         continue;
       for (int pass : {1, 2}) {
         Shape m = s;

@@ -32,7 +32,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     env = {k: v for k, v in os.environ.items() if not k.startswith("HQ_")}
     p = subprocess.run([checker, str(tmp_path)], capture_output=True, text=True, env=env, timeout=600)
     assert p.returncode == 0, p.stdout + p.stderr
-    assert p.stdout.startswith("OK 21 of 21"), p.stdout
+    assert p.stdout.startswith("OK 24 of 24"), p.stdout
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
     star = srcs["star_dense_lrgp"]
@@ -65,3 +65,6 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "[R] = {};" in op and "mask; (void)found_" in op
     assert "(a_ != 0 && " in op and "3855ULL >> v_" in op and "(a_ != 0 || " in op
     assert "mask; (void)found_" not in srcs["outer_predicates_mp2"].split("extern \"C\"")[0]
+    # composite keys: the slot's word 1 is compared with the second key, payloads start at word 2
+    cp = srcs["composite_probe"]
+    assert "kk2_[r] = (int)(long long)c2[r];" in cp and "sl_[r].y == kk2_[r]" in cp and "= sl_[r].z;" in cp

@@ -12,7 +12,7 @@ import torch.multiprocessing as mp
 pytestmark = pytest.mark.gpu
 
 SF = 0.01
-QS = ["ssb_q41", "ssb_q31", "ssb_q11", "tpch_q6", "tpch_q1", "tpch_q3", "tpch_q5", "ssb_q43", "tpch_q7"]
+QS = ["ssb_q41", "ssb_q31", "ssb_q11", "tpch_q6", "tpch_q1", "tpch_q3", "tpch_q5", "ssb_q43", "tpch_q7", "tpch_q9"]
 
 
 def _port():
@@ -81,6 +81,8 @@ def test_two_ranks_on_one_device_match_oracle():
         "tpch_q6": oracle.tpch_q6(tpch["lineitem"]).rows(),
         "tpch_q5": oracle.tpch_q5(tpch["tpch_customer"], tpch["orders"], tpch["lineitem"], tpch["tpch_supplier"],
                                   tpch["nation"], tpch["region"]).rows(),
+        "tpch_q9": oracle.tpch_q9(tpch["tpch_part"], tpch["tpch_supplier"], tpch["lineitem"], tpch["partsupp"],
+                                  tpch["orders"], tpch["nation"]).rows(),
         "tpch_q7": oracle.tpch_q7(tpch["tpch_customer"], tpch["orders"], tpch["lineitem"], tpch["tpch_supplier"],
                                   tpch["nation"]).rows(),
         "ssb_q43": oracle.ssb_q4(3, ssb["lineorder"], ssb["date"], ssb["customer"], ssb["supplier"], ssb["part"]).rows(),

@@ -57,6 +57,9 @@ def oracle_run(qname, t, **kw):
         return oracle.ssb_q41(t["lineorder"], t["date"], t["customer"], t["supplier"], t["part"])
     if qname == "tpch_q3":
         return oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    if qname == "tpch_q9":
+        return oracle.tpch_q9(t["tpch_part"], t["tpch_supplier"], t["lineitem"], t["partsupp"], t["orders"], t["nation"],
+                              pmax=kw.get("pmax"))
     if qname == "tpch_q4":
         return oracle.tpch_q4(t["orders"], t["lineitem"])
     if qname == "tpch_q13":
@@ -102,6 +105,7 @@ INT_COLS = {
     "tpch_q10": ["c_custkey", "n_name", "revenue", "count"],
     "tpch_q7": ["supp_nation", "cust_nation", "l_year", "revenue", "count"],
     "tpch_q4": ["o_orderpriority", "order_count"],
+    "tpch_q9": ["nation", "o_year", "sum_profit", "count"],
     "tpch_q13": ["c_count", "custdist"],
     "tpch_q17": ["sum_extendedprice", "count"],
     "tpch_q18": ["c_custkey", "o_orderkey", "o_orderdate", "o_totalprice", "sum_qty", "count"],
@@ -562,7 +566,7 @@ def tpch1():
     return {t: hqgen.generate(t, 1.0) for t in hqgen.TPCH_TABLES}
 
 
-@pytest.mark.parametrize("qname", ["tpch_q4", "tpch_q13", "tpch_q17", "tpch_q18", "tpch_q19", "tpch_q21"])
+@pytest.mark.parametrize("qname", ["tpch_q4", "tpch_q9", "tpch_q13", "tpch_q17", "tpch_q18", "tpch_q19", "tpch_q21"])
 @pytest.mark.parametrize("sf", [0.01, 1.0])
 def test_tpch_f3_parity(ctx, tpch, tpch1, qname, sf):
     """Multi-pipeline plans (aggregation results feeding builds and pipelines, LEFT OUTER
@@ -623,3 +627,12 @@ def test_repeated_runs_identical(ctx):
     E = Engine(ctx, {t: ctx.load_columns({c: host[t][c] for c in cs}) for t, cs in q.columns.items()})
     bad = sum(q.execute(E).rows(cols) != o.rows() for _ in range(300))
     assert bad == 0, f"{bad}/300 runs differ from the oracle"
+
+
+def test_tpch_q9_golden(ctx, golden):
+    """Fixture F18 (composite partsupp key) through every execution model."""
+    fx = golden("F18_tpch_q9.json")
+    for em in ALL_EXEC:
+        g = gpu_run(ctx, "tpch_q9", fx["tables"], exec_mode=em, pmax=fx["params"]["pmax"])
+        assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"], em
+        assert g.qualifying == fx["expected"]["qualifying"]
