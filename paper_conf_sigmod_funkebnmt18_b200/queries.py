@@ -605,8 +605,8 @@ def _tpch_q21(E: Engine, variant: int = 0, limit: int = 100, **_):
 # pushed into the partsupp build through p_partkey = ps_partkey.  partsupp is joined on its
 # two-column key (ps_partkey, ps_suppkey): a composite hash table (hq_build_desc::composite).
 def _tpch_q9(E: Engine, pmax: Optional[int] = None, **_):
-    if pmax is None:
-        pmax = E.table("tpch_part").nrows * 5 // 92
+    if pmax is None:  # only the ranks that build need it (non-root ranks hold no dimension tables)
+        pmax = E.table("tpch_part").nrows * 5 // 92 if E.builds_here else 0
     hp, hps, hs, hn, ho = E.hashes([
         dict(table="tpch_part", key="p_partkey", preds=[("p_partkey", "<=", pmax)]),
         dict(table="partsupp", key="ps_partkey", key2="ps_suppkey", payload=["ps_supplycost"],
