@@ -137,6 +137,14 @@ hq_status hq_ctx_destroy(hq_ctx* ctx) {
       if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
       if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
     }
+    for (int i = 0; i < hq_ctx::NSIDE; ++i) {
+      if (ctx->side[i]) {
+        cudaStreamSynchronize(ctx->side[i]);
+        cudaStreamDestroy(ctx->side[i]);
+      }
+      if (ctx->ev_join[i]) cudaEventDestroy(ctx->ev_join[i]);
+    }
+    if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
     delete ctx;
   });
 }

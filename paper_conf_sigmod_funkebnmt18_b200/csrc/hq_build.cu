@@ -448,15 +448,57 @@ void hq_build_hashes_impl(hq_ctx* ctx, int n, const hq_build_desc* d, hq_hash* c
     HQ_CUDA(cudaHostAlloc(&ctx->pinned_build, want, cudaHostAllocDefault));
     ctx->pinned_build_bytes = want;
   }
-  for (int i = 0; i < n; ++i) {
-    bs[i].host_st = (char*)ctx->pinned_build + (size_t)i * slot;
-    build_prepare(ctx, d + i, h[i], bs[i]);
-    any_count = any_count || bs[i].counted;
+  // Independent builds run concurrently: build i is enqueued on side stream i % NSIDE,
+  // forked from the context stream by an event and joined back by another, so the
+  // small dimension tables' kernels overlap instead of queueing behind each other.
+  // Every allocation of a build is made while ctx->stream points at its side stream
+  // (stream-ordered); the join makes the context stream wait for all of them.  With
+  // caller allocator hooks (which may not order frees across streams) builds stay on
+  // the context stream.
+  const int nside = (n > 1 && !ctx->has_alloc) ? std::min(n, hq_ctx::NSIDE) : 0;
+  if (nside && !ctx->ev_fork) {
+    HQ_CUDA(cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming));
+    for (int k = 0; k < hq_ctx::NSIDE; ++k) {
+      HQ_CUDA(cudaStreamCreateWithFlags(&ctx->side[k], cudaStreamNonBlocking));
+      HQ_CUDA(cudaEventCreateWithFlags(&ctx->ev_join[k], cudaEventDisableTiming));
+    }
   }
-  if (any_count) HQ_CUDA(cudaStreamSynchronize(ctx->stream));
-  for (int i = 0; i < n; ++i)
-    if (bs[i].counted) std::memcpy(&bs[i].st, bs[i].host_st, sizeof(bs[i].st));
-  for (int i = 0; i < n; ++i) build_finish(ctx, d + i, h[i], bs[i]);
+  cudaStream_t main = ctx->stream;
+  auto fork = [&] {
+    if (!nside) return;
+    HQ_CUDA(cudaEventRecord(ctx->ev_fork, main));
+    for (int k = 0; k < nside; ++k) HQ_CUDA(cudaStreamWaitEvent(ctx->side[k], ctx->ev_fork, 0));
+  };
+  auto join = [&] {
+    ctx->stream = main;
+    if (!nside) return;
+    for (int k = 0; k < nside; ++k) {
+      HQ_CUDA(cudaEventRecord(ctx->ev_join[k], ctx->side[k]));
+      HQ_CUDA(cudaStreamWaitEvent(main, ctx->ev_join[k], 0));
+    }
+  };
+  try {
+    fork();
+    for (int i = 0; i < n; ++i) {
+      bs[i].host_st = (char*)ctx->pinned_build + (size_t)i * slot;
+      if (nside) ctx->stream = ctx->side[i % nside];
+      build_prepare(ctx, d + i, h[i], bs[i]);
+      any_count = any_count || bs[i].counted;
+    }
+    join();
+    if (any_count) HQ_CUDA(cudaStreamSynchronize(main));
+    for (int i = 0; i < n; ++i)
+      if (bs[i].counted) std::memcpy(&bs[i].st, bs[i].host_st, sizeof(bs[i].st));
+    fork();
+    for (int i = 0; i < n; ++i) {
+      if (nside) ctx->stream = ctx->side[i % nside];
+      build_finish(ctx, d + i, h[i], bs[i]);
+    }
+    join();
+  } catch (...) {
+    ctx->stream = main;
+    throw;
+  }
 }
 
 namespace {

@@ -85,6 +85,11 @@ struct hq_ctx {
   // stream, ordered against the pipeline kernels by events (created on first use)
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_copied[2] = {nullptr, nullptr}, ev_consumed[2] = {nullptr, nullptr};
+  // concurrent hash builds (hq_build_hashes): side streams forked from / joined to
+  // the context stream by events (created on first use)
+  static constexpr int NSIDE = 4;
+  cudaStream_t side[NSIDE] = {};
+  cudaEvent_t ev_fork = nullptr, ev_join[NSIDE] = {};
   void* alloc_bytes(size_t bytes);
   void free_bytes(void* p, size_t bytes);
 };
