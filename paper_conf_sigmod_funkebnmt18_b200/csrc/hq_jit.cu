@@ -106,6 +106,7 @@ struct Gen {
   std::set<int> dead;          // materialised before the compaction point, not carried over
   std::map<int, std::pair<long long, long long>> known;  // value range of probe payloads (count pass)
   std::map<int, int> stage_k;  // table column -> stage column index
+  std::set<int> vec_loaded;    // stage columns read with ONE vector load per lane (all R rows)
   explicit Gen(const KPlan& k) : kp(k) {
     for (int c = 0; c < HQ_MAX_COLS; ++c) {
       if (!kp.regs[c].in_stage || !kp.regs[c].width) continue;
@@ -131,6 +132,7 @@ struct Gen {
     const char* vt = vb == 16 ? (c.width == 4 ? "int4" : "longlong2") : (vb == 8 ? (c.width == 4 ? "int2" : "long long") : nullptr);
     o << "      " << ctype(c.width) << " " << var(reg) << "[R];\n";
     if (vt && c.width >= 4) {
+      vec_loaded.insert(reg);
       o << "      { const " << vt << " q_ = *(const " << vt << "*)((const " << ctype(c.width) << "*)(st + " << c.soff << "u) + row0);";
       if (vb == 8 && c.width == 8) o << " " << var(reg) << "[0] = q_; }\n";
       else if (vb == 8) o << " " << var(reg) << "[0] = q_.x; " << var(reg) << "[1] = q_.y; }\n";
@@ -560,13 +562,21 @@ std::string generate(const KPlan& kp) {
     const char* rf = getenv("HQ_JIT_RELFIX");  // A/B: dep (default), fence, none
     const std::string fix = rf ? rf : "dep";
     if (fix == "dep") {
-      o << "    { u32 f_ = 0u;\n#pragma unroll\n      for (int r = 0; r < R; ++r) f_ ^= 0u";
-      for (const auto& sk2 : g.stage_k) {
-        const std::string v = g.var(sk2.first) + "[r]";
-        if (g.width(sk2.first) == 8) o << " ^ (u32)" << v << " ^ (u32)((u64)" << v << " >> 32)";
-        else o << " ^ (u32)" << v;
+      // one destination register per shared load instruction: a vector load
+      // completes all its registers together, so element 0 stands for it
+      o << "    { u32 f_ = 0u";
+      for (const auto& sk2 : g.stage_k)
+        if (g.vec_loaded.count(sk2.first)) o << " ^ (u32)" << g.var(sk2.first) << "[0]";
+      o << ";\n";
+      bool scalar = false;
+      for (const auto& sk2 : g.stage_k) scalar = scalar || !g.vec_loaded.count(sk2.first);
+      if (scalar) {
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) f_ ^= 0u";
+        for (const auto& sk2 : g.stage_k)
+          if (!g.vec_loaded.count(sk2.first)) o << " ^ (u32)" << g.var(sk2.first) << "[r]";
+        o << ";\n";
       }
-      o << ";\n      const u32 b_ = __ballot_sync(HQ_FULL, f_ == 0x9E3779B9u);\n"
+      o << "      const u32 b_ = __ballot_sync(HQ_FULL, f_ == 0x9E3779B9u);\n"
         << "      if (lane == 0) { *(volatile u32*)(smem + " << (MISC_DEP) << "u + 4u * warp) = b_; mbar_arrive(&empty[s]); } }\n";
     } else if (fix == "fence") {
       o << "    fence_proxy_async(); __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
