@@ -475,12 +475,28 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       staged[nstaged++] = kp.ops[o].idx;
     }
   }
+  // Generated kernels whose probes all read shared-memory-staged tables (or that
+  // have none) wait on no global round trip per row: 4 rows per lane halve the
+  // per-tile overhead (mbarrier waits, loop, votes) and stream faster (SSB Q1.1
+  // SF30 0.428 -> 0.395 ms); probes that wait on global memory keep 2 rows per
+  // lane, and R = 4 applies only when the ring still holds 3 stages with every
+  // table staged (SSB Q3.1 at R = 4 lost its staged tables: 0.61 -> 1.85 ms).
+  bool prefer4 = false;
+  if (jit && force_R == 2 && !getenv("HQ_JIT_R")) {
+    prefer4 = true;
+    for (int o = 0; o < kp.nops; ++o) {
+      if (kp.ops[o].kind != OP_PROBE) continue;
+      bool st = false;
+      for (int i = 0; i < nstaged; ++i) st = st || staged[i] == kp.ops[o].idx;
+      prefer4 = prefer4 && st && kp.probes[kp.ops[o].idx].direct;
+    }
+  }
   int chosen_R = 0;
   for (;;) {
     uint32_t tab_total = 0;
     for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
     for (int R : {8, 4, 2, 1}) {
-      if (force_R ? R != force_R : (R == 8 || R == 1)) continue;
+      if (prefer4 ? (R != 4 && R != 2) : (force_R ? R != force_R : (R == 8 || R == 1))) continue;
       const uint32_t T = (uint32_t)(kp.nw * 32 * R);
       const uint32_t off_tmp = MISC_BYTES;
       const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
