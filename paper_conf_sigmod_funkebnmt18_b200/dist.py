@@ -127,8 +127,11 @@ class DistributedEngine(Engine):
         return prod > 65536  # libhq's dense/hash switch (hqk::DENSE_LIMIT)
 
     def run(self, pb: PlanBuilder, partitioned: bool = True) -> Optional[hq.Result]:
-        if not partitioned and self.rank != self.root:
-            return None
+        if not partitioned:
+            pb.root_only = True  # a build-side or post-merge pipeline: the root's result is complete
+            if self.rank != self.root:
+                return None
+            return super().run(pb, partitioned)
         P = pb.plan
         if partitioned and self._hash_grouped(P):
             # ranks keep all their groups; ORDER BY / LIMIT run after the root's merge
@@ -144,6 +147,8 @@ class DistributedEngine(Engine):
         for h in self._built:  # root: raise duplicate-key / build faults (syncs)
             h.info()
         self._built.clear()
+        if getattr(pb, "root_only", False):  # no collective: the root ran the whole pipeline
+            return fetch(res, pb.result_names) if self.rank == self.root else None
         if not hasattr(pb, "dist_order"):
             ptr, nbytes = res.partials_view()
             t = device_view(ptr, nbytes, torch.int64)
@@ -153,7 +158,34 @@ class DistributedEngine(Engine):
             return fetch(res, pb.result_names)
         return self._merge_groups(res, pb)
 
+    def gather(self, res: Optional[hq.Result], pb: PlanBuilder) -> Optional[hq.Result]:
+        """Complete result of a partitioned pipeline whose aggregation feeds a later build
+        or root-side pipeline (e.g. TPC-H Q18's GROUP BY l_orderkey ... HAVING): hash
+        group-bys are merged on the root (all-gather of the ranks' groups + one fused merge
+        pipeline; an order split by the range partition is combined there), dense ones are
+        summed with one all-reduce.  Returns the device result on the root, None elsewhere."""
+        if getattr(pb, "root_only", False):
+            return res
+        if hasattr(pb, "dist_order"):
+            merged = self._merge_device(res, pb)
+            return merged[0] if merged is not None else None
+        ptr, nbytes = res.partials_view()
+        reduce_partials(device_view(ptr, nbytes, torch.int64), self.root)
+        return res if self.rank == self.root else None
+
     def _merge_groups(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
+        merged = self._merge_device(res, pb)
+        if merged is None:
+            return None
+        out_res, mb, qual = merged
+        out = fetch(out_res, mb.result_names)
+        out.qualifying = qual  # rows that reached the sinks, over all ranks
+        return out
+
+    def _merge_device(self, res: hq.Result, pb: PlanBuilder):
+        """All-gather the ranks' finalized groups; the root merges them with one fused
+        GROUP BY pipeline (ORDER BY / LIMIT applied there).  Root: (result, plan, qualifying
+        rows over all ranks); other ranks: None."""
         P = pb.plan
         names = list(pb.result_names)
         tab = res.as_table(names)  # finalized local groups, device columns
@@ -189,6 +221,5 @@ class DistributedEngine(Engine):
         order, limit = pb.dist_order
         mb.aggregate(keys=keys, aggs=aggs, order=[(names[c], bool(d)) for c, d in order], limit=limit,
                      group_capacity=max(1024, sum(sizes)), agg_names=names[P.nkeys:])
-        out = fetch(self.ctx.run(mb.plan, keep=mb.keep + [merged]), mb.result_names)
-        out.qualifying = int(qual.item())  # rows that reached the sinks, over all ranks
-        return out
+        mb.root_only = True
+        return self.ctx.run(mb.plan, keep=mb.keep + [merged]), mb, int(qual.item())

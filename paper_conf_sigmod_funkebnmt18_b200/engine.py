@@ -251,3 +251,8 @@ class Engine:
 
     def finish(self, res: hq.Result, pb: PlanBuilder) -> QueryResult:
         return fetch(res, pb.result_names)
+
+    def gather(self, res: Optional[hq.Result], pb: PlanBuilder) -> Optional[hq.Result]:
+        """The complete result of a partitioned pipeline whose aggregation feeds a later
+        build or pipeline (an intermediate GROUP BY): on one device, the result itself."""
+        return res

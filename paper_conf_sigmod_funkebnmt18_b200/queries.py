@@ -392,11 +392,21 @@ def _tpch_q10(E: Engine, limit: int = 20, **_):
 
 
 # ------------------------------------------------------- TPC-H Q4, Q13, Q17, Q18, Q19, Q21
-# Single-device plans (multi-GPU: DESIGN.md §7).  Correlated and nested subqueries
-# become pipelines whose aggregation results feed builds or further pipelines
-# (pipeline breakers); functionally dependent attributes (R18) ride along
-# as MIN aggregates of their group.
+# Correlated and nested subqueries become pipelines whose aggregation results feed
+# builds or further pipelines (pipeline breakers); functionally dependent
+# attributes (R18) ride along as MIN aggregates of their group.  Multi-GPU (DESIGN.md
+# §7): fact pipelines run over each rank's range partition; E.gather completes an
+# intermediate GROUP BY on the root (an order split by the partition is merged there),
+# whose builds are broadcast; root-side pipelines finish the query on the root.
 _KEY32 = 1 << 31
+
+
+class _RootOnly:
+    """What a non-root rank returns for a query the root finishes alone."""
+    root_only = True
+
+    def __init__(self, names):
+        self.result_names, self.keep = list(names), []
 
 
 def _orders_estimate(E: Engine) -> int:
@@ -419,7 +429,9 @@ def _tpch_q4(E: Engine, **_):
     pl.probe(ho, "l_orderkey", "inner", ["o_orderpriority"])
     pl.aggregate(keys=[("l_orderkey", 0, _KEY32), ("o_orderpriority", 0, 5)], aggs=[("count", None)],
                  group_capacity=max(1024, nk), agg_names=["lines"])
-    rl = E.run(pl, partitioned=False)
+    rl = E.gather(E.run(pl), pl)
+    if rl is None:  # non-root rank: the root finishes the query
+        return None, _RootOnly(["o_orderpriority", "order_count"])
     # orders per priority over the distinct order keys
     pg = E.plan_over(rl, ["l_orderkey", "o_orderpriority", "lines"])
     pg.aggregate(keys=[("o_orderpriority", 0, 5)], aggs=[("count", None)],
@@ -434,10 +446,12 @@ def _tpch_q4(E: Engine, **_):
 def _tpch_q13(E: Engine, **_):
     po = E.plan("orders")
     po.aggregate(keys=[("o_custkey", 0, _KEY32)], aggs=[("count", None)],
-                 group_capacity=max(1024, E.table("tpch_customer").nrows), agg_names=["n"])
-    ro = E.run(po, partitioned=False)
+                 group_capacity=max(1024, E.table("orders").nrows // 4), agg_names=["n"])
+    ro = E.gather(E.run(po), po)
     hn = E.hash_from(ro, ["o_custkey", "n"], "o_custkey", ["n"])
     maxn = max(int(hn.info().pay_max), 0)
+    if not E.builds_here:  # the customer table (the outer join's preserved side) is on the root
+        return None, _RootOnly(["c_count", "custdist"])
     pc = E.plan("tpch_customer")
     pc.probe(hn, "c_custkey", "outer", ["c_count"])            # LEFT OUTER JOIN: 0 orders -> 0
     pc.aggregate(keys=[("c_count", 0, maxn + 1)], aggs=[("count", None)],
@@ -459,14 +473,14 @@ def _tpch_q17(E: Engine, **_):
     p1.probe(hp, "l_partkey", "semi")
     p1.aggregate(keys=[("l_partkey", 0, _KEY32)], aggs=[("sum", "l_quantity"), ("count", None)],
                  group_capacity=max(1024, int(hp.info().nkeys)), agg_names=["sum_qty", "cnt"])
-    r1 = E.run(p1, partitioned=False)
+    r1 = E.gather(E.run(p1), p1)
     ha = E.hash_from(r1, ["l_partkey", "sum_qty", "cnt"], "l_partkey", ["sum_qty", "cnt"])
     p2 = E.plan("lineitem")
     p2.probe(ha, "l_partkey", "inner", ["sum_qty", "cnt"])
     p2.compute("d", [("load", "l_quantity"), ("mul", 5), ("mul", "cnt"), ("sub", "sum_qty")])
     p2.filter("d", "<", 0)
     p2.aggregate(aggs=[("sum", "l_extendedprice"), ("count", None)], agg_names=["sum_extendedprice", "count"])
-    res = E.run(p2, partitioned=False)
+    res = E.run(p2)
     p2.keep += [r1, hp]
     return res, p2
 
@@ -482,14 +496,16 @@ def _tpch_q18(E: Engine, limit: int = 100, **_):
     p1 = E.plan("lineitem")
     p1.aggregate(keys=[("l_orderkey", 0, _KEY32)], aggs=[("sum", "l_quantity")],
                  group_capacity=_orders_estimate(E), agg_names=["sum_qty"])
-    r1 = E.run(p1, partitioned=False)
+    r1 = E.gather(E.run(p1), p1)
     hb = E.hash_from(r1, ["l_orderkey", "sum_qty"], "l_orderkey", preds=[("sum_qty", ">", 30000)])
     hc = E.hash("tpch_customer", "c_custkey")
-    po = E.plan("orders")
-    po.probe(hb, "o_orderkey", "semi")
-    po.probe(hc, "o_custkey", "semi")
-    po.materialise([("o_orderkey", "i32"), ("o_custkey", "i32"), ("o_orderdate", "i32"), ("o_totalprice", "i64")])
-    ro = E.run(po, partitioned=False)
+    ro = None
+    if E.builds_here:  # build side: the orders pipeline runs where the dimensions are
+        po = E.plan("orders")
+        po.probe(hb, "o_orderkey", "semi")
+        po.probe(hc, "o_custkey", "semi")
+        po.materialise([("o_orderkey", "i32"), ("o_custkey", "i32"), ("o_orderdate", "i32"), ("o_totalprice", "i64")])
+        ro = E.run(po, partitioned=False)
     ho = E.hash_from(ro, ["o_orderkey", "o_custkey", "o_orderdate", "o_totalprice"], "o_orderkey",
                      ["o_custkey", "o_orderdate", "o_totalprice"])
     pl = E.plan("lineitem")
@@ -500,7 +516,7 @@ def _tpch_q18(E: Engine, limit: int = 100, **_):
                  order=[("o_totalprice", True), ("o_orderdate", False)], limit=limit,
                  group_capacity=max(1024, int(ho.info().nkeys)),
                  agg_names=["c_custkey", "o_orderdate", "o_totalprice", "sum_qty", "count"])
-    res = E.run(pl, partitioned=False)
+    res = E.run(pl)
     pl.result_names = ["o_orderkey"] + pl.result_names[1:]
     pl.keep += [r1, hb, ro, ho]
     return res, pl
@@ -540,7 +556,7 @@ def _tpch_q19(E: Engine, **_):
     pl.filter("b2", "!=", 0)
     pl.compute("rev", [("load", "l_discount"), ("rsub", 100), ("mul", "l_extendedprice")])  # scale 4
     pl.aggregate(aggs=[("sum", "rev"), ("count", None)], agg_names=["revenue", "count"])
-    return E.run(pl, partitioned=False), pl
+    return E.run(pl), pl
 
 
 # select s_name, count(*) as numwait from supplier, lineitem l1, orders, nation
@@ -569,12 +585,15 @@ def _tpch_q21(E: Engine, variant: int = 0, limit: int = 100, **_):
             pb.filter("late", ">", 0)
         pb.aggregate(keys=[("l_orderkey", 0, _KEY32)], aggs=[("min", "l_suppkey"), ("max", "l_suppkey")],
                      group_capacity=_orders_estimate(E), agg_names=["smin", "smax"])
-        r = E.run(pb, partitioned=False)
-        pm = E.plan_over(r, ["l_orderkey", "smin", "smax"])
-        pm.compute("d", [("load", "smax"), ("sub", "smin")])
-        pm.filter("d", "=" if (late and variant == 0) else "!=", 0)
-        pm.materialise([("l_orderkey", "i32")])
-        sets.append(E.hash_from(E.run(pm, partitioned=False), ["l_orderkey"], "l_orderkey"))
+        r = E.gather(E.run(pb), pb)
+        mat = None
+        if r is not None:  # the derived predicate runs on the merged groups (root)
+            pm = E.plan_over(r, ["l_orderkey", "smin", "smax"])
+            pm.compute("d", [("load", "smax"), ("sub", "smin")])
+            pm.filter("d", "=" if (late and variant == 0) else "!=", 0)
+            pm.materialise([("l_orderkey", "i32")])
+            mat = E.run(pm, partitioned=False)
+        sets.append(E.hash_from(mat, ["l_orderkey"], "l_orderkey"))
     h2, h3 = sets
     pl = E.plan("lineitem")
     pl.compute("late", [("load", "l_receiptdate"), ("sub", "l_commitdate")])
@@ -584,10 +603,11 @@ def _tpch_q21(E: Engine, variant: int = 0, limit: int = 100, **_):
     pl.probe(ho, "l_orderkey", "semi")                          # o_orderstatus = 'F'
     pl.probe(h2, "l_orderkey", "semi")                          # exists l2
     pl.probe(h3, "l_orderkey", "semi")                          # not exists l3 (variant 1: exists)
-    nsupp = E.table("tpch_supplier").nrows
-    pl.aggregate(keys=[("l_suppkey", 1, max(nsupp, 1))], aggs=[("count", None)],
+    ms = hs.info()  # the surviving rows' suppliers are the build's keys (same meta on every rank)
+    pl.aggregate(keys=[("l_suppkey", int(ms.key_min), max(int(ms.key_max) - int(ms.key_min) + 1, 1))],
+                 aggs=[("count", None)],
                  order=[("numwait", True), ("l_suppkey", False)], limit=limit, agg_names=["numwait"])
-    res = E.run(pl, partitioned=False)
+    res = E.run(pl)
     pl.result_names = ["s_suppkey", "numwait"]
     pl.keep += sets
     return res, pl

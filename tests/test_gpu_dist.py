@@ -12,7 +12,8 @@ import torch.multiprocessing as mp
 pytestmark = pytest.mark.gpu
 
 SF = 0.01
-QS = ["ssb_q41", "ssb_q31", "ssb_q11", "tpch_q6", "tpch_q1", "tpch_q3", "tpch_q5", "ssb_q43", "tpch_q7", "tpch_q9"]
+QS = ["ssb_q41", "ssb_q31", "ssb_q11", "tpch_q6", "tpch_q1", "tpch_q3", "tpch_q5", "ssb_q43", "tpch_q7", "tpch_q9", "tpch_q4", "tpch_q13",
+      "tpch_q17", "tpch_q18", "tpch_q19", "tpch_q21"]
 
 
 def _port():
@@ -23,7 +24,9 @@ def _port():
     return p
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, qs=None, sf=None):
+    qs = QS if qs is None else qs
+    sf = SF if sf is None else sf
     try:
         import torch
         import torch.distributed as dist
@@ -39,11 +42,11 @@ def _worker(rank, world, port, q):
         dist.init_process_group("gloo", rank=rank, world_size=world)
         ctx = hq.Context(0)
         out = {}
-        for qn in QS:
+        for qn in qs:
             qq = QUERIES[qn]
-            n = hqgen.table_rows(qq.fact, SF)
+            n = hqgen.table_rows(qq.fact, sf)
             rng = partition(n, rank, world)
-            tables = load_tables(ctx, qq, SF, fact_range=rng, skip_dims=rank != 0)
+            tables = load_tables(ctx, qq, sf, fact_range=rng, skip_dims=rank != 0)
             E = DistributedEngine(ctx, tables)
             res, pb = qq.run(E)
             r = E.finish(res, pb)
@@ -81,6 +84,13 @@ def test_two_ranks_on_one_device_match_oracle():
         "tpch_q6": oracle.tpch_q6(tpch["lineitem"]).rows(),
         "tpch_q5": oracle.tpch_q5(tpch["tpch_customer"], tpch["orders"], tpch["lineitem"], tpch["tpch_supplier"],
                                   tpch["nation"], tpch["region"]).rows(),
+        "tpch_q4": oracle.tpch_q4(tpch["orders"], tpch["lineitem"]).rows(),
+        "tpch_q13": oracle.tpch_q13(tpch["tpch_customer"], tpch["orders"]).rows(),
+        "tpch_q17": oracle.tpch_q17(tpch["tpch_part"], tpch["lineitem"]).rows(),
+        "tpch_q18": oracle.tpch_q18(tpch["tpch_customer"], tpch["orders"], tpch["lineitem"]).rows(
+            ["o_orderkey", "c_custkey", "o_orderdate", "o_totalprice", "sum_qty", "count"])[:100],
+        "tpch_q19": oracle.tpch_q19(tpch["tpch_part"], tpch["lineitem"]).rows(),
+        "tpch_q21": oracle.tpch_q21(tpch["tpch_supplier"], tpch["orders"], tpch["lineitem"], tpch["nation"]).rows()[:100],
         "tpch_q9": oracle.tpch_q9(tpch["tpch_part"], tpch["tpch_supplier"], tpch["lineitem"], tpch["partsupp"],
                                   tpch["orders"], tpch["nation"]).rows(),
         "tpch_q7": oracle.tpch_q7(tpch["tpch_customer"], tpch["orders"], tpch["lineitem"], tpch["tpch_supplier"],
@@ -98,3 +108,42 @@ def test_two_ranks_on_one_device_match_oracle():
     # hash group-by (l_orderkey): ranks' groups all-gathered and merged on the root, then top 10
     o3 = oracle.tpch_q3(tpch["tpch_customer"], tpch["orders"], tpch["lineitem"])
     assert root["tpch_q3"] == o3.rows(["l_orderkey", "o_orderdate", "o_shippriority", "revenue", "count"])[:10]
+
+
+F3 = ["tpch_q4", "tpch_q13", "tpch_q17", "tpch_q18", "tpch_q19", "tpch_q21"]
+
+
+def test_two_ranks_tpch_multi_pipeline_sf1():
+    """The multi-pipeline TPC-H plans at SF 1 (non-empty Q17/Q18/Q19 results) over two
+    ranks: intermediate GROUP BYs over the lineitem / orders partitions are gathered and
+    merged on the root (orders split by the range partition are combined), their builds
+    broadcast, and the root finishes; the root's rows equal the oracle's."""
+    import hqgen
+    import oracle
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, F3, 1.0)) for r in range(2)]
+    for p in procs:
+        p.start()
+    outs = [q.get(timeout=900) for _ in procs]
+    for p in procs:
+        p.join(timeout=120)
+    errs = [o for o in outs if o[0] != "ok"]
+    if errs:
+        pytest.fail("\n\n".join(f"rank {o[1]}:\n{o[2]}" for o in errs))
+    root = next(o[2] for o in outs if o[1] == 0)
+    assert all(o[2][qn] is None for o in outs if o[1] != 0 for qn in F3)
+    t = {x: hqgen.generate(x, 1.0) for x in hqgen.TPCH_TABLES}
+    exp = {
+        "tpch_q4": oracle.tpch_q4(t["orders"], t["lineitem"]).rows(),
+        "tpch_q13": oracle.tpch_q13(t["tpch_customer"], t["orders"]).rows(),
+        "tpch_q17": oracle.tpch_q17(t["tpch_part"], t["lineitem"]).rows(),
+        "tpch_q18": oracle.tpch_q18(t["tpch_customer"], t["orders"], t["lineitem"]).rows(
+            ["o_orderkey", "c_custkey", "o_orderdate", "o_totalprice", "sum_qty", "count"])[:100],
+        "tpch_q19": oracle.tpch_q19(t["tpch_part"], t["lineitem"]).rows(),
+        "tpch_q21": oracle.tpch_q21(t["tpch_supplier"], t["orders"], t["lineitem"], t["nation"]).rows()[:100],
+    }
+    for qn, rows in exp.items():
+        assert root[qn] == rows, qn
+        assert len(rows) > 0, qn
