@@ -147,6 +147,11 @@ typedef struct {
 hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int64_t nrows,
                           int32_t flags, hq_table** out);
 hq_status hq_table_info(const hq_table* t, int64_t* nrows, int32_t* ncols);
+/* Column statistics for the planner: min and max of column `col` over all rows (one
+ * device reduction, syncs the context).  An empty table gives *min > *max.  Used to
+ * declare tight GROUP BY key domains (a dense group table needs no hash claim, see
+ * hq_plan::key_card). */
+hq_status hq_column_range(hq_ctx* ctx, const hq_table* t, int32_t col, int64_t* min, int64_t* max);
 hq_status hq_table_column(const hq_table* t, int32_t col, const void** dev_ptr, int32_t* type);
 hq_status hq_free_table(hq_table* t);
 
@@ -315,7 +320,10 @@ typedef struct {
   int32_t ntmp_types;         /* unused, must be 0 */
   /* AGG sink: GROUP BY key_reg[] (each value v must satisfy key_min <= v <
    * key_min + key_card; the packed index sum((v-min)*stride) selects a dense
-   * table when prod(card) <= 65536, else a global hash table); aggregates. */
+   * table when prod(card) <= 65536, else a global hash table -- or, for fused
+   * execution, a dense global table when prod(card) <= 2^28 and its size is at
+   * most twice the hash table's: a group update is then two fire-and-forget
+   * atomics instead of a claim round trip); aggregates. */
   int32_t nkeys;
   int32_t key_reg[HQ_MAX_KEYS];
   int64_t key_min[HQ_MAX_KEYS];

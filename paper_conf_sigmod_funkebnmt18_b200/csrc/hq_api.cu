@@ -237,6 +237,14 @@ hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int
   });
 }
 
+hq_status hq_column_range(hq_ctx* ctx, const hq_table* t, int32_t col, int64_t* min, int64_t* max) {
+  return guarded([&] {
+    if (!ctx || !t || !min || !max) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    if (col < 0 || col >= t->ncols) HQ_THROW(HQ_ERR_ARG, "column out of range");
+    hq_column_range_impl(ctx, t, col, min, max);
+  });
+}
+
 hq_status hq_table_info(const hq_table* t, int64_t* nrows, int32_t* ncols) {
   return guarded([&] {
     if (!t) HQ_THROW(HQ_ERR_ARG, "table is NULL");

@@ -614,3 +614,45 @@ void hq_hash_check(hq_ctx* ctx, hq_hash* h) {
   if (st[0] & HQF_BAD_PAYLOAD) HQ_THROW(HQ_ERR_ARG, "hash build: payload outside int32");
   if (st[0] & HQF_HT_FULL) HQ_THROW(HQ_ERR_OVERFLOW, "hash build: table full (expected_rows too small)");
 }
+
+// ------------------------------------------------------------ column statistics
+namespace {
+__global__ void hq_column_range_kernel(const char* col, int w, long long n, long long* out) {
+  long long mn = LLONG_MAX, mx = LLONG_MIN;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    const long long v = w == 4 ? (long long)((const int*)col)[i] : (w == 8 ? ((const long long*)col)[i] : (long long)((const signed char*)col)[i]);
+    mn = v < mn ? v : mn;
+    mx = v > mx ? v : mx;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const long long a = __shfl_xor_sync(0xffffffffu, mn, o), b = __shfl_xor_sync(0xffffffffu, mx, o);
+    mn = a < mn ? a : mn;
+    mx = b > mx ? b : mx;
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMin(out, mn);
+    atomicMax(out + 1, mx);
+  }
+}
+}  // namespace
+
+void hq_column_range_impl(hq_ctx* ctx, const hq_table* t, int col, int64_t* mn, int64_t* mx) {
+  if (t->host_stream) HQ_THROW(HQ_ERR_UNSUPPORTED, "column range: HQ_HOST_STREAM table");
+  DevBuf out(ctx, 16);
+  const long long init[2] = {LLONG_MAX, LLONG_MIN};
+  long long* h = (long long*)pinned_staging(ctx, 16);
+  std::memcpy(h, init, 16);
+  HQ_CUDA(cudaMemcpyAsync(out.p, h, 16, cudaMemcpyHostToDevice, ctx->stream));
+  if (t->nrows > 0) {
+    const int grid = (int)std::max<long long>(1, std::min<long long>((t->nrows + 255) / 256, (long long)ctx->num_sms * 8));
+    ctx->launches++;
+    hq_column_range_kernel<<<grid, 256, 0, ctx->stream>>>((const char*)t->cols[col].ptr, t->cols[col].width, t->nrows,
+                                                          out.as<long long>());
+    HQ_CUDA(cudaGetLastError());
+  }
+  HQ_CUDA(cudaMemcpyAsync(h, out.p, 16, cudaMemcpyDeviceToHost, ctx->stream));
+  HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  *mn = h[0];
+  *mx = h[1];
+}

@@ -33,52 +33,93 @@ struct KCompact {
   int scalar;
 };
 
-// one warp-aggregated atomic per 32 entries for the output rows and one for the
-// qualifying count (a per-entry atomic on one address serialised: TPC-H Q3's
-// 2 M-slot hash table took 0.33 ms)
-__global__ void hq_compact_kernel(const __grid_constant__ KCompact k) {
-  const uint32_t stride = k.vwords + (k.hash ? 1 : 0);
-  const int lane = threadIdx.x & 31;
-  const long long span = (k.ngroups + 31) / 32 * 32;  // whole warps take part in the ballots
-  for (long long g = blockIdx.x * (long long)blockDim.x + threadIdx.x; g < span;
-       g += (long long)gridDim.x * blockDim.x) {
-    const long long* e = k.gtab + g * stride;
-    unsigned long long key = (unsigned long long)g;
-    bool live = g < k.ngroups;
-    if (live && k.hash) {
-      key = (unsigned long long)e[0];
-      ++e;
-      live = key != EMPTY_KEY;
+// write one live group entry as result row `row` (keys decoded from the packed index)
+__device__ __forceinline__ void compact_emit(const KCompact& k, const long long* e, unsigned long long key,
+                                             long long cnt, unsigned long long row) {
+  for (int i = 0; i < k.nkeys; ++i)
+    k.out[i][row] = k.key_min[i] + (long long)((key / (unsigned long long)k.key_stride[i]) % (unsigned long long)k.key_card[i]);
+  bool big = false;
+  for (int a = 0; a < k.naggs; ++a) {
+    const long long v = e[1 + a];
+    long long* o = k.out[k.nkeys + a];
+    if (k.agg_fn[a] == HQ_AGG_AVG) {
+      const double d = cnt ? (double)v / (double)cnt / k.agg_div[a] : __longlong_as_double(0x7ff8000000000000LL);
+      o[row] = __double_as_longlong(d);
+    } else {
+      o[row] = v;
     }
-    const long long cnt = live ? e[0] : 0;
-    live = live && (cnt != 0 || k.scalar);
-    const unsigned m = __ballot_sync(0xffffffffu, live);
-    unsigned long long q = live ? (unsigned long long)cnt : 0ull;
+    if ((k.agg_fn[a] == HQ_AGG_SUM || k.agg_fn[a] == HQ_AGG_AVG) && (v >= (1LL << 62) || v <= -(1LL << 62))) big = true;
+  }
+  if (big) atomicOr(k.err, HQF_OVERFLOW);
+}
+
+// Compaction of the group table into result rows: a block takes tiles of
+// blockDim x COMPACT_PER_THREAD entries, scans its live-entry counts in shared
+// memory and claims its output range with ONE atomic per tile (a warp-level
+// atomic on the single row counter serialised: a 60 M-entry dense table -- TPC-H
+// Q18's GROUP BY l_orderkey -- spent 4 ms in 1.9 M same-address atomics).
+constexpr int COMPACT_PER_THREAD = 8;
+__global__ void __launch_bounds__(256) hq_compact_kernel(const __grid_constant__ KCompact k) {
+  const uint32_t stride = k.vwords + (k.hash ? 1 : 0);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  __shared__ unsigned long long s_cnt[32], s_qual[32], s_base;
+  const long long tile = (long long)blockDim.x * COMPACT_PER_THREAD;
+  for (long long t0 = blockIdx.x * tile; t0 < k.ngroups; t0 += (long long)gridDim.x * tile) {
+    unsigned live = 0;
+    int nl = 0;
+    unsigned long long q = 0;
+#pragma unroll
+    for (int c = 0; c < COMPACT_PER_THREAD; ++c) {
+      const long long g = t0 + (long long)c * blockDim.x + threadIdx.x;
+      if (g >= k.ngroups) continue;
+      const long long* e = k.gtab + g * stride;
+      bool l = true;
+      if (k.hash) {
+        l = (unsigned long long)e[0] != EMPTY_KEY;
+        ++e;
+      }
+      const long long cnt = l ? e[0] : 0;
+      l = l && (cnt != 0 || k.scalar);
+      if (l) {
+        live |= 1u << c;
+        ++nl;
+        q += (unsigned long long)cnt;
+      }
+    }
+    int incl = nl;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int t = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += t;
+    }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) q += __shfl_xor_sync(0xffffffffu, q, o);
-    unsigned long long base = 0;
-    if (lane == 0 && m) {
-      base = atomicAdd(k.nout, (unsigned long long)__popc(m));
-      atomicAdd(k.nout + 1, q);
-    }
-    base = __shfl_sync(0xffffffffu, base, 0);
-    if (!live) continue;
-    const unsigned long long row = base + __popc(m & ((1u << lane) - 1u));
-    for (int i = 0; i < k.nkeys; ++i)
-      k.out[i][row] = k.key_min[i] + (long long)((key / (unsigned long long)k.key_stride[i]) % (unsigned long long)k.key_card[i]);
-    bool big = false;
-    for (int a = 0; a < k.naggs; ++a) {
-      const long long v = e[1 + a];
-      long long* o = k.out[k.nkeys + a];
-      if (k.agg_fn[a] == HQ_AGG_AVG) {
-        const double d = cnt ? (double)v / (double)cnt / k.agg_div[a] : __longlong_as_double(0x7ff8000000000000LL);
-        o[row] = __double_as_longlong(d);
-      } else {
-        o[row] = v;
+    if (lane == 31) s_cnt[warp] = (unsigned long long)incl;
+    if (lane == 0) s_qual[warp] = q;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long tot = 0, qt = 0;
+      for (int w = 0; w < nw; ++w) {
+        const unsigned long long c = s_cnt[w];
+        s_cnt[w] = tot;  // exclusive prefix of the warps
+        tot += c;
+        qt += s_qual[w];
       }
-      if ((k.agg_fn[a] == HQ_AGG_SUM || k.agg_fn[a] == HQ_AGG_AVG) && (v >= (1LL << 62) || v <= -(1LL << 62))) big = true;
+      s_base = tot ? atomicAdd(k.nout, tot) : 0ull;
+      if (qt) atomicAdd(k.nout + 1, qt);
     }
-    if (big) atomicOr(k.err, HQF_OVERFLOW);
+    __syncthreads();
+    unsigned long long row = s_base + s_cnt[warp] + (unsigned long long)(incl - nl);
+#pragma unroll
+    for (int c = 0; c < COMPACT_PER_THREAD; ++c) {
+      if (!((live >> c) & 1u)) continue;
+      const long long g = t0 + (long long)c * blockDim.x + threadIdx.x;
+      const long long* e = k.gtab + g * stride;
+      unsigned long long key = (unsigned long long)g;
+      if (k.hash) key = (unsigned long long)*e++;
+      compact_emit(k, e, key, e[0], row++);
+    }
+    __syncthreads();  // s_cnt / s_base are reused by the next tile
   }
 }
 
@@ -117,6 +158,7 @@ __device__ __forceinline__ bool row_less(const KSort& s, int a, int b) {
 
 // Each block sorts one chunk of <= SORT_CHUNK indices (bitonic network in
 // shared memory) and keeps its first `keep` rows.
+
 __global__ void __launch_bounds__(1024) hq_chunk_sort_kernel(const __grid_constant__ KSort s, const int* in, long long n,
                                                              int* out, int keep, int net) {
   // net: power-of-two network size (<= SORT_CHUNK); chunks of `net` rows per block
@@ -290,7 +332,7 @@ int grid_for(hq_ctx* ctx, long long n) {
 
 }  // namespace
 
-namespace {
+// per-context pinned host staging (small results, column statistics)
 void* pinned_staging(hq_ctx* ctx, size_t bytes) {
   if (ctx->pinned_bytes < bytes) {
     if (ctx->pinned) HQ_CUDA(cudaFreeHost(ctx->pinned));
@@ -303,6 +345,7 @@ void* pinned_staging(hq_ctx* ctx, size_t bytes) {
   return ctx->pinned;
 }
 
+namespace {
 // one launch, one sync: fault bits + finalized rows come back together
 bool finalize_small(hq_ctx* ctx, hq_result* r) {
   const hq_plan& P = r->plan;
@@ -311,7 +354,9 @@ bool finalize_small(hq_ctx* ctx, hq_result* r) {
   for (int i = 0; i < P.norder; ++i)
     if (P.order_col[i] < 0 || P.order_col[i] >= nc) HQ_THROW(HQ_ERR_ARG, "plan: ORDER BY column out of range");
   const int64_t ng = std::max<int64_t>(r->ngroups, 1);
-  const int64_t rcap = P.limit > 0 ? std::min<int64_t>(ng, P.limit) : ng;
+  // columns start 16-B aligned (an even row count): the result may become the fact
+  // table of a later pipeline (hq_result_as_table), whose stage loads need it
+  const int64_t rcap = ((P.limit > 0 ? std::min<int64_t>(ng, P.limit) : ng) + 1) / 2 * 2;
   std::vector<DevBuf> cols;
   for (int c = 0; c < nc; ++c) cols.emplace_back(ctx, (size_t)ng * 8);
   // [stats: 64 B][column 0: rcap rows][column 1]... -- one D2H copy brings it all back

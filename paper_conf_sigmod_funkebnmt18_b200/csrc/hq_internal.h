@@ -177,6 +177,7 @@ constexpr int MAX_INSNS = 64;
 constexpr int NREGS = HQ_MAX_COLS + HQ_MAX_TMP;
 constexpr int SMEM_AGG_BYTES = 32 * 1024;
 constexpr int64_t DENSE_LIMIT = 65536;
+constexpr int64_t DENSE_GLOBAL_LIMIT = 1LL << 28;  // dense global group tables (fused execution)
 constexpr unsigned long long EMPTY_KEY = ~0ULL;
 
 enum : uint8_t { OP_FILTER = 1, OP_PROBE = 2, OP_COMPUTE = 3 };
@@ -365,6 +366,8 @@ int64_t fused_smem_bytes(const KPlan& kp);
 }  // namespace hqk
 
 // finalize: compaction + AVG + ORDER BY + LIMIT (hq_finalize.cu)
+void hq_column_range_impl(hq_ctx* ctx, const hq_table* t, int col, int64_t* mn, int64_t* mx);
+void* pinned_staging(hq_ctx* ctx, size_t bytes);  // hq_finalize.cu: per-context pinned host buffer
 // unordered: a pure GROUP BY (no ORDER BY / LIMIT) skips the sort (hq_result_as_table)
 void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered = false);
 // op-at-a-time execution of a plan (hq_oaat.cu)

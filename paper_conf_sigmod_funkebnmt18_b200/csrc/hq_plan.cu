@@ -216,10 +216,19 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       kp.agg_reg[a] = P.agg_fn[a] == HQ_AGG_COUNT ? (int16_t)0 : (int16_t)use(P.agg_reg[a], "aggregate");
     }
     kp.vwords = 1 + P.naggs;
+    // a dense global table for a tight but large key domain (fused execution): no hash
+    // claim round trip per group update, when it is at most twice the hash table's size
+    auto dense_global = [&](int64_t ng) {
+      if (P.exec != HQ_EXEC_FUSED && P.exec != HQ_EXEC_FUSED_INTERP) return false;
+      if (ng > DENSE_GLOBAL_LIMIT) return false;
+      int64_t hcap = group_cap > 0 ? group_cap : (P.group_capacity > 0 ? P.group_capacity : std::min<int64_t>(ng, 1 << 20));
+      hcap = std::max<int64_t>(1024, next_pow2(hcap * 2));
+      return (__int128)ng * kp.vwords <= (__int128)2 * hcap * (kp.vwords + 1);
+    };
     if (P.nkeys == 0) {
       kp.gmode = GM_SCALAR;
       r->ngroups = 1;
-    } else if (ngroups <= DENSE_LIMIT) {
+    } else if (ngroups <= DENSE_LIMIT || dense_global(ngroups)) {
       kp.gmode = GM_DENSE;
       r->ngroups = ngroups;
     } else {

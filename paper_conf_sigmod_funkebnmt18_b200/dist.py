@@ -124,6 +124,8 @@ class DistributedEngine(Engine):
         prod = 1
         for i in range(P.nkeys):
             prod *= P.key_card[i]
+        if any(P.agg_fn[a] in (hq.AGG_MIN, hq.AGG_MAX) for a in range(P.naggs)):
+            return True  # MIN / MAX partials do not combine with a SUM all-reduce: merge the groups
         return prod > 65536  # libhq's dense/hash switch (hqk::DENSE_LIMIT)
 
     def run(self, pb: PlanBuilder, partitioned: bool = True) -> Optional[hq.Result]:
@@ -157,6 +159,15 @@ class DistributedEngine(Engine):
                 return None
             return fetch(res, pb.result_names)
         return self._merge_groups(res, pb)
+
+    def key_domain(self, table: str, col: str):
+        """The key domain over ALL ranks' partitions (min / max all-reduced), so every rank
+        declares the same group table."""
+        lo, hi = self.tables[table].column_range(col)
+        t = torch.tensor([-lo, hi], dtype=torch.int64, device=self.device)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        lo, hi = -int(t[0].item()), int(t[1].item())
+        return (0, 1) if lo > hi else (lo, hi - lo + 1)
 
     def gather(self, res: Optional[hq.Result], pb: PlanBuilder) -> Optional[hq.Result]:
         """Complete result of a partitioned pipeline whose aggregation feeds a later build

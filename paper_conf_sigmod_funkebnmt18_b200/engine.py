@@ -252,6 +252,12 @@ class Engine:
     def finish(self, res: hq.Result, pb: PlanBuilder) -> QueryResult:
         return fetch(res, pb.result_names)
 
+    def key_domain(self, table: str, col: str) -> Tuple[int, int]:
+        """(min, cardinality) of a column, for declaring a tight GROUP BY key domain
+        (lets libhq use a dense group table for large groupings, hq.h key_card)."""
+        lo, hi = self.tables[table].column_range(col)
+        return (0, 1) if lo > hi else (lo, hi - lo + 1)
+
     def gather(self, res: Optional[hq.Result], pb: PlanBuilder) -> Optional[hq.Result]:
         """The complete result of a partitioned pipeline whose aggregation feeds a later
         build or pipeline (an intermediate GROUP BY): on one device, the result itself."""

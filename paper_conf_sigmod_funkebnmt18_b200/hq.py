@@ -116,7 +116,7 @@ STRUCTS = {"hq_column": Column, "hq_pred": Pred, "hq_build_desc": BuildDesc, "hq
 # every symbol include/hq.h declares
 EXPORTS = ["hq_ctx_create", "hq_ctx_destroy", "hq_ctx_set_stream", "hq_ctx_sync", "hq_last_error",
            "hq_abi_version", "hq_sizeof", "hq_ctx_enable_timing", "hq_ctx_kernel_times", "hq_ctx_launches",
-           "hq_load_columns",
+           "hq_load_columns", "hq_column_range",
            "hq_table_info", "hq_table_column", "hq_free_table", "hq_build_hash", "hq_build_hashes", "hq_hash_info",
            "hq_hash_device_view", "hq_hash_import", "hq_free_hash", "hq_run_pipeline", "hq_run_pipeline_streamed",
            "hq_finalize",
@@ -155,6 +155,7 @@ def lib():
             "hq_hash_import": [vp, P(HashMeta), vp, P(vp)], "hq_free_hash": [vp],
             "hq_run_pipeline": [vp, P(Plan), P(vp)], "hq_finalize": [vp, vp],
             "hq_run_pipeline_streamed": [vp, P(Plan), i64, P(vp)],
+            "hq_column_range": [vp, vp, i32, P(i64), P(i64)],
             "hq_result_info_get": [vp, vp, P(ResultInfo)],
             "hq_fetch_result": [vp, vp, P(vp), i64, P(i64)],
             "hq_result_as_table": [vp, vp, P(vp)],
@@ -363,6 +364,12 @@ class Table:
 
     def col(self, name: str) -> int:
         return self.names.index(name)
+
+    def column_range(self, name: str):
+        """(min, max) of a column (device reduction; syncs).  Empty: min > max."""
+        lo, hi = ctypes.c_int64(), ctypes.c_int64()
+        check(lib().hq_column_range(self.ctx.h, self.h, self.col(name), ctypes.byref(lo), ctypes.byref(hi)))
+        return lo.value, hi.value
 
     def column_ptr(self, c: int):
         """(device pointer, hq_type) of column c."""

@@ -445,7 +445,7 @@ def _tpch_q4(E: Engine, **_):
 # group by c_count order by custdist desc, c_count desc            (App F: no o_comment LIKE)
 def _tpch_q13(E: Engine, **_):
     po = E.plan("orders")
-    po.aggregate(keys=[("o_custkey", 0, _KEY32)], aggs=[("count", None)],
+    po.aggregate(keys=[("o_custkey",) + E.key_domain("orders", "o_custkey")], aggs=[("count", None)],
                  group_capacity=max(1024, E.table("orders").nrows // 4), agg_names=["n"])
     ro = E.gather(E.run(po), po)
     hn = E.hash_from(ro, ["o_custkey", "n"], "o_custkey", ["n"])
@@ -471,7 +471,8 @@ def _tpch_q17(E: Engine, **_):
                                                  ("p_container", "=", hqgen.code(hqgen.CONTAINERS, "MED BOX"))])
     p1 = E.plan("lineitem")
     p1.probe(hp, "l_partkey", "semi")
-    p1.aggregate(keys=[("l_partkey", 0, _KEY32)], aggs=[("sum", "l_quantity"), ("count", None)],
+    p1.aggregate(keys=[("l_partkey",) + E.key_domain("lineitem", "l_partkey")],
+                 aggs=[("sum", "l_quantity"), ("count", None)],
                  group_capacity=max(1024, int(hp.info().nkeys)), agg_names=["sum_qty", "cnt"])
     r1 = E.gather(E.run(p1), p1)
     ha = E.hash_from(r1, ["l_partkey", "sum_qty", "cnt"], "l_partkey", ["sum_qty", "cnt"])
@@ -494,7 +495,7 @@ def _tpch_q17(E: Engine, **_):
 def _tpch_q18(E: Engine, limit: int = 100, **_):
     # the IN subquery: GROUP BY l_orderkey over all of lineitem, HAVING as the build predicate
     p1 = E.plan("lineitem")
-    p1.aggregate(keys=[("l_orderkey", 0, _KEY32)], aggs=[("sum", "l_quantity")],
+    p1.aggregate(keys=[("l_orderkey",) + E.key_domain("lineitem", "l_orderkey")], aggs=[("sum", "l_quantity")],
                  group_capacity=_orders_estimate(E), agg_names=["sum_qty"])
     r1 = E.gather(E.run(p1), p1)
     hb = E.hash_from(r1, ["l_orderkey", "sum_qty"], "l_orderkey", preds=[("sum_qty", ">", 30000)])
@@ -578,12 +579,13 @@ def _tpch_q21(E: Engine, variant: int = 0, limit: int = 100, **_):
                            dict(table="orders", key="o_orderkey",
                                 preds=[("o_orderstatus", "=", hqgen.code(hqgen.ORDERSTATUS, "F"))])])
     sets = []
+    okeys = E.key_domain("lineitem", "l_orderkey")
     for late in (False, True):  # l2: all lines of the order; l3: its late lines
         pb = E.plan("lineitem")
         if late:
             pb.compute("late", [("load", "l_receiptdate"), ("sub", "l_commitdate")])
             pb.filter("late", ">", 0)
-        pb.aggregate(keys=[("l_orderkey", 0, _KEY32)], aggs=[("min", "l_suppkey"), ("max", "l_suppkey")],
+        pb.aggregate(keys=[("l_orderkey",) + okeys], aggs=[("min", "l_suppkey"), ("max", "l_suppkey")],
                      group_capacity=_orders_estimate(E), agg_names=["smin", "smax"])
         r = E.gather(E.run(pb), pb)
         mat = None
