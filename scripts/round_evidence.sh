@@ -15,4 +15,6 @@ done
 timeout 900 python scripts/tpch_all.py --sf 10 > gpurun_out/tpch_all.log 2>&1; tail -3 gpurun_out/tpch_all.log
 timeout 900 python scripts/stream_sweep.py --query ssb_q41 --sf 30 > gpurun_out/stream_sweep.log 2>&1; tail -3 gpurun_out/stream_sweep.log
 timeout 600 python scripts/stress_stream.py ssb_q41 30 4194304 60 200 2>&1 | tail -3
+timeout 900 python scripts/ssb_all.py --sf 30 --reps 5 > gpurun_out/ssb_all.log 2>&1; tail -3 gpurun_out/ssb_all.log
+timeout 1800 python scripts/bytes_ratio.py --sf 10 > gpurun_out/bytes_ratio.log 2>&1; tail -3 gpurun_out/bytes_ratio.log
 ls gpurun_out
