@@ -798,15 +798,25 @@ std::string generate(const KPlan& kp) {
           // updates the table in ONE pass, so the global round trips of a warp's
           // groups overlap instead of queueing one per group (TPC-H Q18/Q21:
           // GROUP BY l_orderkey, ~16 groups per warp)
-          << "        u32 multi_ = am_ & ~__ballot_sync(HQ_FULL, single_);\n"
-          << "        bool upd_ = single_; u64 uc_ = 1ull;\n"
-          << "        while (multi_) {\n          const int leader_ = __ffs(multi_) - 1;\n"
-          << "          const u32 grp_ = __shfl_sync(HQ_FULL, peers_, leader_); const bool mine_ = (grp_ >> lane) & 1u;\n"
-          << "          i64 w_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) w_[a] = warp_reduce(AGG_FN[a], mine_ ? v_[a] : agg_identity(AGG_FN[a]));\n"
-          << "          if (lane == leader_) {\n#pragma unroll\n            for (int a = 0; a < NAGGS; ++a) v_[a] = w_[a];\n"
-          << "            uc_ = (u64)__popc(grp_); upd_ = true; }\n"
-          << "          multi_ &= ~grp_;\n        }\n"
-          << "        if (upd_) group_update(p, sagg, key_, true, uc_, v_);\n      }\n";
+          << "        u32 multi_ = am_ & ~__ballot_sync(HQ_FULL, single_);\n";
+        const char* op1 = getenv("HQ_JIT_ONEPASS");  // A/B: 0 = one update per group inside the loop
+        if (op1 && op1[0] == '0') {
+          o << "        if (single_) group_update(p, sagg, key_, true, 1ull, v_);\n"
+            << "        while (multi_) {\n          const int leader_ = __ffs(multi_) - 1;\n"
+            << "          const u32 grp_ = __shfl_sync(HQ_FULL, peers_, leader_); const bool mine_ = (grp_ >> lane) & 1u;\n"
+            << "          i64 w_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) w_[a] = warp_reduce(AGG_FN[a], mine_ ? v_[a] : agg_identity(AGG_FN[a]));\n"
+            << "          if (lane == leader_) group_update(p, sagg, key_, true, (u64)__popc(grp_), w_);\n"
+            << "          multi_ &= ~grp_;\n        }\n      }\n";
+        } else {
+          o << "        bool upd_ = single_; u64 uc_ = 1ull;\n"
+            << "        while (multi_) {\n          const int leader_ = __ffs(multi_) - 1;\n"
+            << "          const u32 grp_ = __shfl_sync(HQ_FULL, peers_, leader_); const bool mine_ = (grp_ >> lane) & 1u;\n"
+            << "          i64 w_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) w_[a] = warp_reduce(AGG_FN[a], mine_ ? v_[a] : agg_identity(AGG_FN[a]));\n"
+            << "          if (lane == leader_) {\n#pragma unroll\n            for (int a = 0; a < NAGGS; ++a) v_[a] = w_[a];\n"
+            << "            uc_ = (u64)__popc(grp_); upd_ = true; }\n"
+            << "          multi_ &= ~grp_;\n        }\n"
+            << "        if (upd_) group_update(p, sagg, key_, true, uc_, v_);\n      }\n";
+        }
         if (!wcompact) o << "      }\n";  // else of the sparse path
       }
     }
