@@ -799,8 +799,12 @@ std::string generate(const KPlan& kp) {
           // groups overlap instead of queueing one per group (TPC-H Q18/Q21:
           // GROUP BY l_orderkey, ~16 groups per warp)
           << "        u32 multi_ = am_ & ~__ballot_sync(HQ_FULL, single_);\n";
-        const char* op1 = getenv("HQ_JIT_ONEPASS");  // A/B: 0 = one update per group inside the loop
-        if (op1 && op1[0] == '0') {
+        // one pass only where an update is a global round trip (C2 straight to global):
+        // with a shared-memory table the per-group updates are cheap and the extra
+        // live registers cost ~1.5 % (SSB Q3.1 / Q4.1); HQ_JIT_ONEPASS=0/1 forces (A/B)
+        const char* op1 = getenv("HQ_JIT_ONEPASS");
+        const bool onepass = op1 ? op1[0] == '1' : kp.smode == SM_NONE;
+        if (!onepass) {
           o << "        if (single_) group_update(p, sagg, key_, true, 1ull, v_);\n"
             << "        while (multi_) {\n          const int leader_ = __ffs(multi_) - 1;\n"
             << "          const u32 grp_ = __shfl_sync(HQ_FULL, peers_, leader_); const bool mine_ = (grp_ >> lane) & 1u;\n"
