@@ -636,3 +636,29 @@ def test_tpch_q9_golden(ctx, golden):
         g = gpu_run(ctx, "tpch_q9", fx["tables"], exec_mode=em, pmax=fx["params"]["pmax"])
         assert [list(r) for r in g.rows(fx["expected"]["columns"])] == fx["expected"]["rows"], em
         assert g.qualifying == fx["expected"]["qualifying"]
+
+
+@pytest.mark.parametrize("qname,sf", [("ssb_q41", 100.0), ("ssb_q31", 30.0), ("tpch_q3", 30.0), ("tpch_q1", 10.0)])
+def test_bench_configs_full_size(ctx, qname, sf):
+    """BASELINE.json's configs at their full sizes, in the launch configuration bench.py
+    times (generated fused kernel, default plan), element by element against the oracle
+    (all host cores): the bench's workloads are the ones the parity covers."""
+    import os
+    from paper_conf_sigmod_funkebnmt18_b200.queries import load_tables
+    q = QUERIES[qname]
+    tabs = hqgen.SSB_TABLES if q.bench == "ssb" else hqgen.TPCH_TABLES
+    host = {t: hqgen.generate(t, sf, columns=q.columns[t]) for t in q.columns if t in tabs}
+    nt = os.cpu_count() or 1
+    if qname == "ssb_q41":
+        o = oracle.ssb_q41(host["lineorder"], host["date"], host["customer"], host["supplier"], host["part"], nthreads=nt)
+    elif qname == "ssb_q31":
+        o = oracle.ssb_q31(host["lineorder"], host["customer"], host["supplier"], host["date"], nthreads=nt)
+    elif qname == "tpch_q3":
+        o = oracle.tpch_q3(host["tpch_customer"], host["orders"], host["lineitem"], nthreads=nt)
+    else:
+        o = oracle.tpch_q1(host["lineitem"], nthreads=nt)
+    E = Engine(ctx, load_tables(ctx, q, sf, host=host))
+    g = q.execute(E, **({"limit": 0} if qname == "tpch_q3" else {}))
+    assert_same(qname, g, o)
+    assert g.qualifying == o.qualifying
+    del E
