@@ -99,20 +99,22 @@ def _ssb_q1(v: int):
 
 
 # ---------------------------------------------------------------- SSB Q3.1
-def _ssb_q31_probes(E: Engine) -> PlanBuilder:
+def _ssb_q31_probes(E: Engine, porder: str = "scd") -> PlanBuilder:
     hc, hs, hd = E.hashes([
         dict(table="customer", key="c_custkey", payload=["c_nation"], preds=[("c_region", "=", ASIA)]),
         dict(table="supplier", key="s_suppkey", payload=["s_nation"], preds=[("s_region", "=", ASIA)]),
         dict(table="date", key="d_datekey", payload=["d_year"], preds=[("d_year", "between", 1992, 1997)])])
     pb = E.plan("lineorder")
-    pb.probe(hs, "lo_suppkey", "inner", ["s_nation"])
-    pb.probe(hc, "lo_custkey", "inner", ["c_nation"])
-    pb.probe(hd, "lo_orderdate", "inner", ["d_year"])
+    probes = {"s": (hs, "lo_suppkey", ["s_nation"]), "c": (hc, "lo_custkey", ["c_nation"]),
+              "d": (hd, "lo_orderdate", ["d_year"])}
+    for k in porder:  # probe order (result-invariant, R14)
+        h, key, pay = probes[k]
+        pb.probe(h, key, "inner", pay)
     return pb
 
 
-def _ssb_q31(E: Engine, **_):
-    pb = _ssb_q31_probes(E)
+def _ssb_q31(E: Engine, porder: str = "scd", **_):
+    pb = _ssb_q31_probes(E, porder)
     pb.aggregate(keys=[("c_nation", 0, 25), ("s_nation", 0, 25), ("d_year", 1992, 7)],
                  aggs=[("sum", "lo_revenue"), ("count", None)],
                  order=[("d_year", False), ("revenue", True)], agg_names=["revenue", "count"])
