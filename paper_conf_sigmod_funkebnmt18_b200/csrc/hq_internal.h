@@ -177,6 +177,11 @@ constexpr int MAX_INSNS = 64;
 constexpr int NREGS = HQ_MAX_COLS + HQ_MAX_TMP;
 constexpr int SMEM_AGG_BYTES = 32 * 1024;
 constexpr int64_t DENSE_LIMIT = 65536;
+// shared-memory header of the fused kernels (mbarriers, block-scan and scalar-reduction
+// slots, < 2,800 B) and, in its last 128 B, the per-warp words of the stage-release
+// dependency (hq_jit.cu)
+constexpr uint32_t MISC_BYTES = 3072;
+constexpr uint32_t MISC_DEP = MISC_BYTES - 128;
 constexpr int64_t DENSE_GLOBAL_LIMIT = 1LL << 28;  // dense global group tables (fused execution)
 constexpr unsigned long long EMPTY_KEY = ~0ULL;
 

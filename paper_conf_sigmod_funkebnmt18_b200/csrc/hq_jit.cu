@@ -89,9 +89,6 @@ std::mutex g_mu;
 std::map<std::pair<int, std::string>, CUfunction> g_cache;  // (device, source) -> kernel
 
 // ------------------------------------------------------------------ codegen
-// per-warp scratch words at the end of the kernel's misc header (MISC_BYTES = 3072 in
-// hq_plan.cu; barriers, block-scan and scalar-reduction slots use < 2,800 B)
-constexpr unsigned MISC_DEP = 3072 - 128;
 std::string lit(long long v) {
   if (v == LLONG_MIN) return "HQ_LL_MIN";
   return std::to_string(v) + "LL";

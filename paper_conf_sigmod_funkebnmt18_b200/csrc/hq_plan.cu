@@ -19,7 +19,6 @@ int64_t next_pow2(int64_t x) {
 uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
 
 // barriers, block-scan and reduction scratch: full/empty[10], base[32], wtot[32], red[32][9]
-constexpr uint32_t MISC_BYTES = 3072;
 
 struct RegInfo {
   int width = 0;       // 0 = undefined
