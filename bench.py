@@ -154,9 +154,14 @@ def cpu_baseline(qname, host, n_fact, budget_s=30.0):
     est = dt0 * n_fact / max(s0, 1)
     s = n_fact if est <= budget_s else max(s0, int(n_fact * budget_s / est))
     dt = oracle_call(qname, host, cores, s)
+    # the oracle single-threaded too (a bounded prefix)
+    s1 = min(n_fact, 4_000_000)
+    dt1 = oracle_call(qname, host, 1, s1)
     return {"value": s / dt, "unit": "rows/s", "cores": cores, "kind": "oracle",
             "sample": f"first {s} of {n_fact} fact rows (full dimension tables), tuple-at-a-time C++ oracle, "
-                      f"{cores} threads, {dt:.2f} s"}
+                      f"{cores} threads, {dt:.2f} s",
+            "single_thread": {"value": s1 / dt1, "unit": "rows/s", "cores": 1,
+                              "sample": f"first {s1} fact rows, 1 thread, {dt1:.2f} s"}}
 
 
 def exec_timing(qname, host, local, fused_ms, mode="oaat", steps=2):
