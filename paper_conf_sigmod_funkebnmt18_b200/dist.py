@@ -85,37 +85,53 @@ class DistributedEngine(Engine):
         self._built: List[hq.Hash] = []
         self.builds_here = self.rank == root
 
-    def _share(self, h: Optional[hq.Hash]) -> hq.Hash:
+    def _share_many(self, hs: Sequence[Optional[hq.Hash]]) -> List[hq.Hash]:
+        """Broadcast several root-built tables: ONE broadcast of all their metadata (the
+        root sends what it knows on the host; only the other ranks read it back), then one
+        asynchronous broadcast per slot array, then the imports -- instead of a metadata
+        broadcast and host read per table (each a stream sync)."""
+        n = len(hs)
+        meta = torch.zeros((max(n, 1), 16), dtype=torch.int64, device=self.device)
+        views = []
         if self.rank == self.root:
-            ptr, m = h.device_view()  # no sync: the slot array is stream-ordered before NCCL
-            self._built.append(h)     # build faults are checked in finish()
-            buf = device_view(ptr, int(m.bytes))
-            meta = [m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout,
-                    m.pay_min, m.pay_max, m.key_max] + [_i64(w) for w in m.pay_set] + [m.composite]
-        else:
-            meta, buf = None, None
-        meta, buf = broadcast_blob(meta, buf, 4, self.root, self.device)
+            rows = []
+            for h in hs:
+                ptr, m = h.device_view()
+                self._built.append(h)  # build faults are checked in finish()
+                views.append(device_view(ptr, int(m.bytes)))
+                rows.append([m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout,
+                             m.pay_min, m.pay_max, m.key_max] + [_i64(w) for w in m.pay_set] + [m.composite, 0])
+            meta[:n] = torch.tensor(rows, dtype=torch.int64)
+        dist.broadcast(meta, src=self.root)
         if self.rank == self.root:
-            return h
-        hm = hq.HashMeta()
-        (hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout,
-         hm.pay_min, hm.pay_max, hm.key_max) = meta[:10]
-        for k in range(4):
-            hm.pay_set[k] = meta[10 + k] & 0xFFFFFFFFFFFFFFFF
-        hm.composite = meta[14]
-        return self.ctx.import_hash(hm, buf.data_ptr(), keep=buf)
+            for v in views:
+                dist.broadcast(v, src=self.root)
+            return list(hs)
+        rows = meta.cpu().tolist()
+        out = []
+        for r in rows[:n]:
+            buf = torch.empty(int(r[4]), dtype=torch.uint8, device=self.device)
+            dist.broadcast(buf, src=self.root)
+            hm = hq.HashMeta()
+            (hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout,
+             hm.pay_min, hm.pay_max, hm.key_max) = r[:10]
+            for k in range(4):
+                hm.pay_set[k] = r[10 + k] & 0xFFFFFFFFFFFFFFFF
+            hm.composite = r[14]
+            out.append(self.ctx.import_hash(hm, buf.data_ptr(), keep=buf))
+        return out
 
     def hash(self, table, key, payload=(), preds=(), expected_rows=0, key2=None) -> hq.Hash:
         h = super().hash(table, key, payload, preds, expected_rows, key2) if self.rank == self.root else None
-        return self._share(h)
+        return self._share_many([h])[0]
 
     def hashes(self, specs) -> List[hq.Hash]:
         hs = super().hashes(specs) if self.rank == self.root else [None] * len(specs)
-        return [self._share(h) for h in hs]
+        return self._share_many(hs)
 
     def hash_from(self, res, names, key, payload=(), preds=()) -> hq.Hash:
         h = super().hash_from(res, names, key, payload, preds) if self.rank == self.root else None
-        return self._share(h)
+        return self._share_many([h])[0]
 
     @staticmethod
     def _hash_grouped(P: hq.Plan) -> bool:
