@@ -290,9 +290,16 @@ typedef enum { HQ_AGG_SUM = 1, HQ_AGG_COUNT, HQ_AGG_MIN, HQ_AGG_MAX, HQ_AGG_AVG 
 typedef enum { HQ_SINK_AGG = 1, HQ_SINK_MATERIALISE = 2 } hq_sink_kind;
 /* Reduction technique of the sink (Table 4):
  * LRGP = local resolution in registers/shared memory + global propagation with
- *        one atomic per block and tile (A3, B3, C3) -- the default;
- * ATOMIC = per-row global atomics (A2, B2, C2), kept as an ablation. */
-typedef enum { HQ_RES_LRGP = 0, HQ_RES_ATOMIC = 1 } hq_resolution;
+ *        one atomic per block and tile (A3, B3, C3) -- the default; its local
+ *        resolution is SIMD-style (warp shuffles/ballots, App C "SIMD Reduction");
+ * ATOMIC = per-row global atomics (A2, B2, C2), kept as an ablation;
+ * WE = local resolution by work-efficient (Blelloch) trees in shared memory with one
+ *        barrier per level, one pre-aggregate / write offset per workgroup and tile
+ *        (App C "Work-Efficient Reduction", Fig 24): A3-WE exclusive scan
+ *        of the row flags, B3-WE tree reduction, C3-WE sort by key + segmented scan +
+ *        atomic hash reduce of each segment.  Generated fused kernels
+ *        only (HQ_EXEC_FUSED; HQ_ERR_UNSUPPORTED otherwise); an ablation. */
+typedef enum { HQ_RES_LRGP = 0, HQ_RES_ATOMIC = 1, HQ_RES_WE = 2 } hq_resolution;
 /* Execution of a plan:
  * FUSED        one compound kernel, compiled for this plan with NVRTC (query
  *              compilation); falls back to FUSED_INTERP
@@ -380,6 +387,32 @@ hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out);
  * (int64, ngroups x (1+naggs): [count, agg...]) before finalization, so ranks
  * can sum it with NCCL; only SUM/COUNT/AVG plans (HQ_ERR_UNSUPPORTED else). */
 hq_status hq_result_partials_view(hq_result* r, void** dev_ptr, size_t* bytes);
+/* Rebuild the dense partial-aggregate array of `r` from the caller's device buffer
+ * (same layout as hq_result_partials_view: ngroups x (1+naggs) int64), e.g. after the
+ * ranks' partials were summed into a buffer of their own: copies `bytes` bytes into
+ * the result's group table on the ctx stream (async).  The result must not be
+ * finalized yet; bytes must equal the view's size (HQ_ERR_ARG).  (The reduce itself
+ * may also run in place on the view, which needs no call.) */
+hq_status hq_result_from_partials(hq_ctx* ctx, hq_result* r, const void* dev_ptr, size_t bytes);
+
+/* Fault words gathered on the device, without a host synchronisation, so that a
+ * multi-rank caller can combine every rank's faults with the collective it runs
+ * anyway and raise on all ranks or on none (a fault seen by one rank alone would
+ * leave the others blocked in the next collective).  Writes HQ_FAULT_WORDS int64 to
+ * the device buffer dev_out (async, ctx stream): word k (k < 16) = 1 if fault bit k
+ * is set in any of the hashes' build fault words, word 16 + k = 1 if bit k is set in
+ * any of the results' pipeline fault words, 0 otherwise -- so a SUM reduce over the
+ * ranks keeps "some rank saw fault k" as word k != 0.  Imported hashes (no build on
+ * this device) contribute nothing.  nh / nr may be 0. */
+#define HQ_FAULT_WORDS 32
+hq_status hq_gather_faults(hq_ctx* ctx, const hq_hash* const* hashes, int32_t nh, const hq_result* const* results,
+                           int32_t nr, int64_t* dev_out);
+/* Map HQ_FAULT_WORDS host words (as written by hq_gather_faults, possibly summed over
+ * ranks) to a status: HQ_OK when no error fault is set, else the status a syncing call
+ * would raise for it (HQ_ERR_DUP_KEY, HQ_ERR_ARG, HQ_ERR_OVERFLOW), with the message in
+ * hq_last_error().  The re-runnable pipeline faults (group table full, materialise
+ * capacity) are not errors here: the owning result re-runs at its own finalize. */
+hq_status hq_raise_faults(const int64_t* host_words);
 hq_status hq_free_result(hq_result* r);
 
 #ifdef __cplusplus

@@ -45,22 +45,46 @@ def embed_prelude() -> None:
             f.write(text)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    embed_prelude()
-    if not force and up_to_date():
-        return SO
-    cudalib = os.path.join(os.path.dirname(os.path.dirname(NVCC)), "lib64")
-    cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
-           "-I" + os.path.join(ROOT, "include"), "-o", SO + ".tmp", *sources(),
-           "-L" + cudalib, "-lnvrtc", "-Xlinker", "-rpath," + cudalib]
+def _compile(src: str, obj: str, verbose: bool) -> None:
+    cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "-c",
+           "-I" + os.path.join(ROOT, "include"), "-o", obj + ".tmp", src]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
-        raise RuntimeError("nvcc failed building libhq.so")
+        raise RuntimeError(f"nvcc failed compiling {os.path.basename(src)}")
     if verbose:
         sys.stderr.write(r.stderr)
+    os.replace(obj + ".tmp", obj)
+
+
+def build(force: bool = False, verbose: bool = False) -> str:
+    """One object per CUDA source, compiled in parallel (a source is recompiled when it
+    or any header is newer than its object), then linked into libhq.so."""
+    from concurrent.futures import ThreadPoolExecutor
+    embed_prelude()
+    if not force and up_to_date():
+        return SO
+    objdir = os.path.join(ROOT, "build", "libhq")
+    os.makedirs(objdir, exist_ok=True)
+    hdr_t = max([os.path.getmtime(h) for h in headers()] + [0.0])
+    jobs = []
+    objs = []
+    for src in sources():
+        obj = os.path.join(objdir, os.path.basename(src)[:-3] + ".o")
+        objs.append(obj)
+        if force or not os.path.exists(obj) or os.path.getmtime(obj) < max(os.path.getmtime(src), hdr_t):
+            jobs.append((src, obj))
+    with ThreadPoolExecutor(max_workers=max(1, min(len(jobs), os.cpu_count() or 1))) as ex:
+        for f in [ex.submit(_compile, s2, o, verbose) for s2, o in jobs]:
+            f.result()
+    cudalib = os.path.join(os.path.dirname(os.path.dirname(NVCC)), "lib64")
+    cmd = [NVCC, *ARCH, "-shared", "-o", SO + ".tmp", *objs, "-L" + cudalib, "-lnvrtc", "-Xlinker", "-rpath," + cudalib]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError("nvcc failed linking libhq.so")
     os.replace(SO + ".tmp", SO)
     return SO
 

@@ -464,6 +464,52 @@ hq_status hq_result_partials_view(hq_result* r, void** dev_ptr, size_t* bytes) {
   });
 }
 
+hq_status hq_result_from_partials(hq_ctx* ctx, hq_result* r, const void* dev_ptr, size_t bytes) {
+  return guarded([&] {
+    if (!ctx || !r || !dev_ptr) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    void* p = nullptr;
+    size_t n = 0;
+    const hq_status st = hq_result_partials_view(r, &p, &n);
+    if (st != HQ_OK) HQ_THROW(st, g_last_error);
+    if (bytes != n) HQ_THROW(HQ_ERR_ARG, "hq_result_from_partials: size differs from the partials view");
+    if (p != dev_ptr && n > 0) HQ_CUDA(cudaMemcpyAsync(p, dev_ptr, n, cudaMemcpyDeviceToDevice, ctx->stream));
+  });
+}
+
+hq_status hq_gather_faults(hq_ctx* ctx, const hq_hash* const* hashes, int32_t nh, const hq_result* const* results,
+                           int32_t nr, int64_t* dev_out) {
+  return guarded([&] {
+    if (!ctx || !dev_out || nh < 0 || nr < 0) HQ_THROW(HQ_ERR_ARG, "NULL argument or negative count");
+    if ((nh > 0 && !hashes) || (nr > 0 && !results)) HQ_THROW(HQ_ERR_ARG, "NULL handle array");
+    std::vector<const int*> hw, rw;
+    for (int i = 0; i < nh; ++i) {
+      if (!hashes[i]) HQ_THROW(HQ_ERR_ARG, "NULL hash");
+      if (hashes[i]->dstate.p) hw.push_back(hashes[i]->dstate.as<int>());  // imported tables: no build here
+    }
+    for (int i = 0; i < nr; ++i) {
+      if (!results[i]) HQ_THROW(HQ_ERR_ARG, "NULL result");
+      if (results[i]->dstate.p) rw.push_back((const int*)(results[i]->dstate.as<char>() + 8));
+    }
+    hq_launch_gather_faults(ctx, hw, rw, (long long*)dev_out);
+  });
+}
+
+hq_status hq_raise_faults(const int64_t* w) {
+  return guarded([&] {
+    if (!w) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    auto b = [&](int bit) { return w[bit] != 0; };
+    auto pb = [&](int flag) { int k = 0; while ((1 << k) != flag) ++k; return w[16 + k] != 0; };
+    auto hb = [&](int flag) { int k = 0; while ((1 << k) != flag) ++k; return b(k); };
+    if (hb(HQF_DUP_KEY)) HQ_THROW(HQ_ERR_DUP_KEY, "hash build: duplicate key (join keys must be unique)");
+    if (hb(HQF_BAD_KEY)) HQ_THROW(HQ_ERR_ARG, "hash build: key INT32_MIN or outside int32");
+    if (hb(HQF_BAD_PAYLOAD)) HQ_THROW(HQ_ERR_ARG, "hash build: payload outside int32");
+    if (hb(HQF_HT_FULL)) HQ_THROW(HQ_ERR_OVERFLOW, "hash build: table full (expected_rows too small)");
+    if (pb(HQF_DIV_ZERO)) HQ_THROW(HQ_ERR_ARG, "pipeline: division by zero");
+    if (pb(HQF_KEY_DOMAIN)) HQ_THROW(HQ_ERR_ARG, "pipeline: group key outside its declared [min, min+card)");
+    if (pb(HQF_OVERFLOW)) HQ_THROW(HQ_ERR_OVERFLOW, "aggregate exceeds the int64 guard (|v| >= 2^62)");
+  });
+}
+
 hq_status hq_free_result(hq_result* r) {
   return guarded([&] {
     if (r) r->release();

@@ -632,3 +632,37 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered) {
   r->nrows = nfinal;
   r->finalized = true;
 }
+
+// ------------------------------------------------------------- fault words
+namespace {
+constexpr int GF_MAX = 256;
+struct KGather {
+  const int* w[GF_MAX];
+  int nh, nr;
+  long long* out;
+};
+// word k < 16: bit k of any hash's build fault word; word 16 + k: bit k of any
+// result's pipeline fault word (hq.h hq_gather_faults)
+__global__ void hq_gather_faults_kernel(const __grid_constant__ KGather g) {
+  const int k = threadIdx.x;
+  int hb = 0, rb = 0;
+  for (int i = 0; i < g.nh; ++i) hb |= *(volatile const int*)g.w[i];
+  for (int i = 0; i < g.nr; ++i) rb |= *(volatile const int*)g.w[g.nh + i];
+  if (k < 16) g.out[k] = (hb >> k) & 1;
+  else if (k < 32) g.out[k] = (rb >> (k - 16)) & 1;
+}
+}  // namespace
+
+void hq_launch_gather_faults(hq_ctx* ctx, const std::vector<const int*>& hw, const std::vector<const int*>& rw,
+                             long long* out) {
+  if (hw.size() + rw.size() > (size_t)GF_MAX) HQ_THROW(HQ_ERR_UNSUPPORTED, "hq_gather_faults: more than 256 handles");
+  KGather g{};
+  g.nh = (int)hw.size();
+  g.nr = (int)rw.size();
+  for (size_t i = 0; i < hw.size(); ++i) g.w[i] = hw[i];
+  for (size_t i = 0; i < rw.size(); ++i) g.w[hw.size() + i] = rw[i];
+  g.out = out;
+  ctx->launches++;
+  hq_gather_faults_kernel<<<1, 32, 0, ctx->stream>>>(g);
+  HQ_CUDA(cudaGetLastError());
+}

@@ -372,7 +372,10 @@ int64_t fused_smem_bytes(const KPlan& kp);
 
 // finalize: compaction + AVG + ORDER BY + LIMIT (hq_finalize.cu)
 void hq_column_range_impl(hq_ctx* ctx, const hq_table* t, int col, int64_t* mn, int64_t* mx);
-void* pinned_staging(hq_ctx* ctx, size_t bytes);  // hq_finalize.cu: per-context pinned host buffer
+void* pinned_staging(hq_ctx* ctx, size_t bytes);
+// hq_finalize.cu: OR of fault words into HQ_FAULT_WORDS int64 (hq_gather_faults)
+void hq_launch_gather_faults(hq_ctx* ctx, const std::vector<const int*>& hw, const std::vector<const int*>& rw,
+                             long long* out);  // hq_finalize.cu: per-context pinned host buffer
 // unordered: a pure GROUP BY (no ORDER BY / LIMIT) skips the sort (hq_result_as_table)
 void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered = false);
 // op-at-a-time execution of a plan (hq_oaat.cu)

@@ -458,6 +458,106 @@ std::string fn_list(const uint8_t* fns, int n) {
   return s.str();
 }
 
+// Resolution:WE tile code (App C, "Work-Efficient Reduction", Fig 24,
+// P:1989-2029; Table 4 A3/B3/C3): every consumer thread takes part (NT = NW * 32 is a
+// power of two for WE plans, hq_plan.cu), one consumer barrier per tree level.
+//  B3-WE: up-sweep of the threads' tile partials -> one global atomic per tile;
+//  A3-WE: Blelloch exclusive scan of the threads' row counts -> one atomicAdd per tile,
+//         rows written at base + scan + their rank among the thread's rows;
+//  C3-WE: bitonic sort of the tile's (key, count, values) by key, a work-efficient
+//         segmented scan with (f1,v1)+(f2,v2) = (f1|f2, f2 ? v2 : v1+v2), and every
+//         segment's last entry updates the global group table (atomic hash reduce).
+void gen_we_tile(std::ostringstream& o, const KPlan& kp, int sk) {
+  const int NT = kp.nw * 32;
+  if (NT & (NT - 1)) HQ_THROW(HQ_ERR_STATE, "jit: Resolution:WE needs a power-of-two thread count");
+  const std::string nt = std::to_string(NT);
+  o << "    { const int tid_ = threadIdx.x;\n";
+  if (sk == 0) {
+    o << "      i64* wr_ = (i64*)(smem + OFF_AGG);  // [1 + NAGGS][NT]: count, aggregates\n"
+      << "      wr_[tid_] = (i64)wc_;\n";
+    for (int a = 0; a < kp.naggs; ++a) o << "      wr_[" << (1 + a) * NT << " + tid_] = wa_[" << a << "];\n";
+    o << "      for (int d_ = 1; d_ < " << nt << "; d_ <<= 1) {\n        consumer_bar();\n"
+      << "        const int i_ = (tid_ + 1) * 2 * d_ - 1;\n        if (i_ < " << nt << ") { wr_[i_] += wr_[i_ - d_];";
+    for (int a = 0; a < kp.naggs; ++a)
+      o << " wr_[" << (1 + a) * NT << " + i_] = agg_combine(AGG_FN[" << a << "], wr_[" << (1 + a) * NT << " + i_ - d_], wr_["
+        << (1 + a) * NT << " + i_]);";
+    o << " }\n      }\n      consumer_bar();\n"
+      << "      if (tid_ == 0 && wr_[" << NT - 1 << "] != 0) { const u64 cnt_ = (u64)wr_[" << NT - 1 << "]; g_add64(p.gtab, (i64)cnt_);";
+    for (int a = 0; a < kp.naggs; ++a)
+      o << " g_agg(AGG_FN[" << a << "], p.gtab + " << 1 + a << ", wr_[" << (1 + a) * NT + NT - 1 << "], cnt_);";
+    o << " }\n      consumer_bar();  // the next tile rewrites the tree\n    }\n";
+    return;
+  }
+  if (sk == 2) {
+    o << "      int* ws_ = (int*)(smem + OFF_AGG);\n      const u32 msk_ = mask;\n      ws_[tid_] = __popc(msk_);\n"
+      << "      for (int d_ = 1; d_ < " << nt << "; d_ <<= 1) { consumer_bar(); const int i_ = (tid_ + 1) * 2 * d_ - 1;"
+      << " if (i_ < " << nt << ") ws_[i_] += ws_[i_ - d_]; }\n      consumer_bar();\n"
+      << "      if (tid_ == 0) { const int tot_ = ws_[" << NT - 1 << "]; s_base[0] = tot_ > 0 ? atomicAdd(p.counter, (u64)tot_) : 0ull;"
+      << " ws_[" << NT - 1 << "] = 0; }\n"
+      << "      for (int d_ = " << NT / 2 << "; d_ >= 1; d_ >>= 1) { consumer_bar(); const int i_ = (tid_ + 1) * 2 * d_ - 1;"
+      << " if (i_ < " << nt << ") { const int t_ = ws_[i_ - d_]; ws_[i_ - d_] = ws_[i_]; ws_[i_] += t_; } }\n"
+      << "      consumer_bar();\n      const u64 base_ = s_base[0] + (u64)ws_[tid_];\n"
+      << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((msk_ >> r) & 1u) { const u64 pos_ = base_ + __popc(msk_ & ((1u << r) - 1u));\n"
+      << "        if ((long long)pos_ < p.capacity) {\n";
+    for (int j = 0; j < kp.nout; ++j)
+      o << "          ((" << ctype(kp.out_width[j]) << "*)p.out[" << j << "])[pos_] = (" << ctype(kp.out_width[j]) << ")ov" << j << "[r];\n";
+    o << "        } else atomicOr(p.err, F_CAPACITY); }\n      consumer_bar();  // s_base / the scan are rewritten by the next tile\n    }\n";
+    return;
+  }
+  // C3-WE over N = NT * R entries
+  const int N = NT * kp.R;
+  const std::string n = std::to_string(N);
+  const int na = kp.naggs;
+  o << "      u64* wk_s = (u64*)(smem + OFF_AGG); i64* wn_ = (i64*)(wk_s + " << N << "); i64* wv_s = wn_ + " << N
+    << "; int* wf_ = (int*)(wv_s + " << (size_t)N * (na > 0 ? na : 1) << ");\n"
+    << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const int e_ = tid_ * R + r; const bool l_ = (wm_ >> r) & 1u;"
+    << " wk_s[e_] = l_ ? wk_[r] : HQ_EMPTY_KEY; wn_[e_] = l_ ? 1 : 0;";
+  for (int a = 0; a < na; ++a) o << " wv_s[" << a * N << " + e_] = l_ ? wv_[" << a << "][r] : agg_identity(AGG_FN[" << a << "]);";
+  o << " }\n";
+  // bitonic sort by key (empty keys = ~0 sort last)
+  o << "      for (int k_ = 2; k_ <= " << n << "; k_ <<= 1)\n        for (int j_ = k_ >> 1; j_ > 0; j_ >>= 1) {\n          consumer_bar();\n"
+    << "          for (int e_ = tid_; e_ < " << n << "; e_ += " << nt << ") { const int q_ = e_ ^ j_; if (q_ > e_) {\n"
+    << "            const u64 a_ = wk_s[e_], b_ = wk_s[q_];\n"
+    << "            if ((a_ > b_) == ((e_ & k_) == 0)) { wk_s[e_] = b_; wk_s[q_] = a_; { const i64 x_ = wn_[e_]; wn_[e_] = wn_[q_]; wn_[q_] = x_; }";
+  for (int a = 0; a < na; ++a)
+    o << " { const i64 x_ = wv_s[" << a * N << " + e_]; wv_s[" << a * N << " + e_] = wv_s[" << a * N << " + q_]; wv_s[" << a * N
+      << " + q_] = x_; }";
+  o << " } } }\n        }\n      consumer_bar();\n";
+  // head flags, then the segmented up-sweep: node i = op(left, node)
+  o << "      for (int e_ = tid_; e_ < " << n << "; e_ += " << nt << ") wf_[e_] = (e_ == 0 || wk_s[e_] != wk_s[e_ - 1]) ? 1 : 0;\n"
+    << "      for (int d_ = 1; d_ < " << n << "; d_ <<= 1) {\n        consumer_bar();\n"
+    << "        for (int t_ = tid_; t_ < " << n << " / (2 * d_); t_ += " << nt << ") { const int i_ = (t_ + 1) * 2 * d_ - 1, l_ = i_ - d_;\n"
+    << "          if (!wf_[i_]) { wn_[i_] += wn_[l_];";
+  for (int a = 0; a < na; ++a)
+    o << " wv_s[" << a * N << " + i_] = agg_combine(AGG_FN[" << a << "], wv_s[" << a * N << " + l_], wv_s[" << a * N << " + i_]);";
+  o << " }\n          wf_[i_] |= wf_[l_]; }\n      }\n      consumer_bar();\n"
+    // the root is the last segment's total; then it becomes the identity for the down-sweep
+    << "      if (tid_ == 0) { s_red[0] = wn_[" << N - 1 << "];";
+  for (int a = 0; a < na; ++a) o << " s_red[" << 1 + a << "] = wv_s[" << a * N + N - 1 << "];";
+  o << " wf_[" << N - 1 << "] = 0; wn_[" << N - 1 << "] = 0;";
+  for (int a = 0; a < na; ++a) o << " wv_s[" << a * N + N - 1 << "] = agg_identity(AGG_FN[" << a << "]);";
+  o << " }\n"
+    // down-sweep: left <- parent prefix; right <- op(parent prefix, left total)
+    << "      for (int d_ = " << N / 2 << "; d_ >= 1; d_ >>= 1) {\n        consumer_bar();\n"
+    << "        for (int t_ = tid_; t_ < " << n << " / (2 * d_); t_ += " << nt << ") { const int i_ = (t_ + 1) * 2 * d_ - 1, l_ = i_ - d_;\n"
+    << "          const int tf_ = wf_[l_]; const i64 tn_ = wn_[l_]; wf_[l_] = wf_[i_]; wn_[l_] = wn_[i_];";
+  for (int a = 0; a < na; ++a)
+    o << " const i64 tv" << a << "_ = wv_s[" << a * N << " + l_]; wv_s[" << a * N << " + l_] = wv_s[" << a * N << " + i_];";
+  o << "\n          wf_[i_] |= tf_;\n          if (tf_) { wn_[i_] = tn_;";
+  for (int a = 0; a < na; ++a) o << " wv_s[" << a * N << " + i_] = tv" << a << "_;";
+  o << " } else { wn_[i_] += tn_;";
+  for (int a = 0; a < na; ++a)
+    o << " wv_s[" << a * N << " + i_] = agg_combine(AGG_FN[" << a << "], wv_s[" << a * N << " + i_], tv" << a << "_);";
+  o << " } }\n      }\n      consumer_bar();\n"
+    // every segment's last entry: its total is the exclusive prefix of the next entry
+    << "      for (int e_ = tid_; e_ < " << n << "; e_ += " << nt << ") { const u64 key_ = wk_s[e_];\n"
+    << "        if (key_ == HQ_EMPTY_KEY || (e_ + 1 < " << n << " && wk_s[e_ + 1] == key_)) continue;\n"
+    << "        const bool last_ = e_ + 1 == " << n << "; i64 v_[NAGGS > 0 ? NAGGS : 1];\n"
+    << "        const u64 cnt_ = (u64)(last_ ? s_red[0] : wn_[e_ + 1]);\n";
+  for (int a = 0; a < na; ++a) o << "        v_[" << a << "] = last_ ? s_red[" << 1 + a << "] : wv_s[" << a * N << " + e_ + 1];\n";
+  o << "        group_update(p, sagg, key_, false, cnt_, v_); }\n      consumer_bar();  // the next tile rewrites the sort buffers\n    }\n";
+}
+
 std::string generate(const KPlan& kp) {
   Gen g(kp);
   // HQ_JIT_PROF=1 (debug): per-CTA globaltimer start/end and barrier-wait cycles
@@ -466,6 +566,10 @@ std::string generate(const KPlan& kp) {
   if (const char* e = getenv("HQ_JIT_WAIT_NS")) wait_ns = atoi(e);
   std::ostringstream& o = g.o;
   const bool c2 = kp.resolution == HQ_RES_ATOMIC;
+  // Resolution:WE (App C, Fig 24): per tile, a work-efficient
+  // (Blelloch) tree in shared memory with one consumer barrier per level produces one
+  // pre-aggregate / write offset per workgroup (the CTA) for global propagation
+  const bool we = kp.resolution == HQ_RES_WE;
   const int sk = kp.sink == HQ_SINK_MATERIALISE ? 2 : (kp.nkeys == 0 ? 0 : 1);
   const int mp = kp.mp_pass;  // multi-pass: 1 = count kernel, 2 = write kernel (hq_multipass.cu)
   // ---------------------------------------------------------------- kernel
@@ -519,7 +623,7 @@ std::string generate(const KPlan& kp) {
   o << "    }\n    return;\n  }\n";
   // consumer state
   o << "  const int row0 = warp * 32 * R + lane * R;  // the lane's rows: row0 .. row0 + R - 1\n";
-  if (sk == 0 && !c2) {
+  if (sk == 0 && !c2 && !we) {
     o << "  u64 scount_ = 0;\n";
     for (int a = 0; a < kp.naggs; ++a) o << "  i64 sacc" << a << " = agg_identity(AGG_FN[" << a << "]);\n";
   }
@@ -545,6 +649,11 @@ std::string generate(const KPlan& kp) {
   o << "      fence_proxy_async(); __syncwarp();\n    }\n";
   if (sk == 2)  // output values leave the operator block in registers; the block scan runs after it
     for (int j = 0; j < kp.nout; ++j) o << "    long long ov" << j << "[R];\n";
+  if (we && sk == 0 && !mp) {  // the tile's per-thread partials leave the operator block for the WE tree
+    o << "    u32 wc_ = 0u; i64 wa_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n    for (int a = 0; a < NAGGS; ++a) wa_[a] = agg_identity(AGG_FN[a]);\n";
+  } else if (we && sk == 1 && !mp) {  // the tile's live (key, values) leave it for the WE sort + segmented scan
+    o << "    u32 wm_ = 0u; u64 wk_[R]; i64 wv_[NAGGS > 0 ? NAGGS : 1][R];\n";
+  }
   o << "    {\n";
   if (kp.early_release) {
     // every referenced column of the lane's rows into registers, then the stage
@@ -646,7 +755,12 @@ std::string generate(const KPlan& kp) {
   if (sk == 0) {
     std::vector<std::string> vv;
     for (int a = 0; a < kp.naggs; ++a) vv.push_back(aggval(a));
-    if (c2) {  // B2: per-row global atomic reduce
+    if (we) {  // B3-WE: the thread's partial over its R rows of this tile
+      o << "      wc_ = __popc(mask);\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) {\n";
+      for (int a = 0; a < kp.naggs; ++a)
+        if (kp.agg_fn[a] != HQ_AGG_COUNT) o << "        wa_[" << a << "] = agg_combine(AGG_FN[" << a << "], wa_[" << a << "], " << vv[a] << ");\n";
+      o << "      }\n";
+    } else if (c2) {  // B2: per-row global atomic reduce
       o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { g_add64(p.gtab, 1);\n";
       for (int a = 0; a < kp.naggs; ++a) o << "        g_agg(AGG_FN[" << a << "], p.gtab + " << 1 + a << ", " << vv[a] << ", 1);\n";
       o << "      }\n";
@@ -720,7 +834,13 @@ std::string generate(const KPlan& kp) {
     }
     if (k32) o << "#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = gk32_[r];\n";
     o << "      if (bad_) atomicOr(p.err, F_KEY_DOMAIN);\n";
-    if (kp.smode == SM_LANE) {
+    if (we) {  // C3-WE: hand the live rows' keys and values to the tile's sort below
+      std::vector<std::string> vv;
+      for (int a = 0; a < kp.naggs; ++a) vv.push_back(aggval(a));
+      o << "      wm_ = mask;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { wk_[r] = gk_[r];";
+      for (int a = 0; a < kp.naggs; ++a) o << " wv_[" << a << "][r] = " << vv[a] << ";";
+      o << " }\n";
+    } else if (kp.smode == SM_LANE) {
       std::vector<std::string> av(kp.nacc);
       for (int a = 1; a < kp.nacc; ++a) av[a] = "(i64)" + g.val(kp.acc_reg[a]);
       o << "      i64* lt_ = (i64*)sagg + threadIdx.x;\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) {\n"
@@ -835,7 +955,8 @@ std::string generate(const KPlan& kp) {
       << " if (row_ >= p.row_begin && row_ < p.row_end) fl_[row_] = (int)((mask >> r) & 1u); } }\n";
   if (g.compacted_R) o << "#undef R\n#define R " << g.compacted_R << "\n";
   o << "    }\n";
-  if (sk == 2 && !mp) {
+  if (we && !mp) gen_we_tile(o, kp, sk);
+  if (sk == 2 && !mp && !we) {
     // A3 (Fig 25 / P:1069-1072): warp ballots -> block scan over the warps ->
     // one atomicAdd per block and tile -> writes at local + global offset.
     // Every consumer warp takes part in every tile (its mask may be empty).
@@ -869,7 +990,7 @@ std::string generate(const KPlan& kp) {
   if (prof) o << "  if (lane == 0) { p.prof[blockIdx.x * 128 + 8 + warp] = pw_; p.prof[blockIdx.x * 128 + 40 + warp] = clock64() - pl0_; } if (pdv_) atomicAdd((unsigned long long*)&p.prof[blockIdx.x * 128 + 72 + warp], (unsigned long long)pdv_);\n";
   // ------------------------------------------------------------- sink (end)
   if (mp) {
-  } else if (sk == 0 && !c2) {
+  } else if (sk == 0 && !c2 && !we) {
     o << "  { u64 c_ = scount_;\n#pragma unroll\n    for (int o_ = 16; o_ > 0; o_ >>= 1) c_ += __shfl_xor_sync(HQ_FULL, c_, o_);\n";
     for (int a = 0; a < kp.naggs; ++a) o << "    const i64 r" << a << " = warp_reduce(AGG_FN[" << a << "], sacc" << a << ");\n";
     o << "    if (lane == 0) { s_red[warp * 9] = (i64)c_;";

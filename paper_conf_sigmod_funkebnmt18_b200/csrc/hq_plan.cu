@@ -187,7 +187,11 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   // ---- sink
   kp.sink = P.sink;
   kp.resolution = P.resolution;
-  if (P.resolution != HQ_RES_LRGP && P.resolution != HQ_RES_ATOMIC) HQ_THROW(HQ_ERR_ARG, "plan: bad resolution");
+  if (P.resolution != HQ_RES_LRGP && P.resolution != HQ_RES_ATOMIC && P.resolution != HQ_RES_WE)
+    HQ_THROW(HQ_ERR_ARG, "plan: bad resolution");
+  const bool we = P.resolution == HQ_RES_WE;
+  if (we && (!jit || mp_pass))
+    HQ_THROW(HQ_ERR_UNSUPPORTED, "Resolution:WE is implemented by the generated fused kernel only (HQ_EXEC_FUSED)");
   uint32_t agg_smem = 0;
   if (P.sink == HQ_SINK_AGG) {
     if (P.nkeys < 0 || P.nkeys > HQ_MAX_KEYS) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: 0..4 group keys");
@@ -380,6 +384,16 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     agg_smem = (uint32_t)(one * c);
   }
 
+  // Resolution:WE (hq_jit.cu gen_we_tile): 16 consumer warps (a power-of-two tree),
+  // the tile's scratch in the aggregation region: B3 [1 + naggs][512] int64, A3 [512]
+  // int32, C3 512 x (key, count, naggs values, head flag) at one row per lane
+  if (we) {
+    const uint32_t nt = (uint32_t)NW * 32;
+    if (P.sink == HQ_SINK_MATERIALISE) agg_smem = nt * 4;
+    else if (P.nkeys == 0) agg_smem = (1u + (uint32_t)P.naggs) * nt * 8;
+    else agg_smem = nt * (8u + 8u + 8u * (uint32_t)std::max(P.naggs, 1) + 4u);
+  }
+
   // ---- multi-pass (hq_multipass.cu): which ops a pass executes and which
   // columns it reads (backward liveness).  Count kernel: selections, probes and
   // the computes feeding them; write kernel: inner probes and computes whose
@@ -465,6 +479,10 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     if (const char* e = getenv("HQ_JIT_NW")) kp.nw = std::max(1, std::min(31, atoi(e)));
     if (const char* e = getenv("HQ_JIT_R")) force_R = atoi(e);
   }
+  if (we) {  // the WE trees need a power-of-two thread count; C3-WE sorts one row per lane
+    kp.nw = NW;
+    force_R = (P.sink == HQ_SINK_AGG && P.nkeys > 0) ? 1 : 2;
+  }
   // Generated kernels stage small compact probe tables (bitmaps / byte arrays of
   // direct tables) in shared memory, earliest probes first (they see the most
   // rows), as long as the TMA ring keeps >= 3 stages.
@@ -490,7 +508,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   // lane, and R = 4 applies only when the ring still holds 3 stages with every
   // table staged (SSB Q3.1 at R = 4 lost its staged tables: 0.61 -> 1.85 ms).
   bool prefer4 = false;
-  if (jit && force_R == 2 && !getenv("HQ_JIT_R")) {
+  if (jit && force_R == 2 && !getenv("HQ_JIT_R") && !we) {
     prefer4 = true;
     for (int o = 0; o < kp.nops; ++o) {
       if (kp.ops[o].kind != OP_PROBE) continue;

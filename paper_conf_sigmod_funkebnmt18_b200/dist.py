@@ -17,6 +17,8 @@ new (north_star).
 """
 from __future__ import annotations
 
+import os
+import sys
 from typing import List, Optional, Sequence, Tuple
 
 import torch
@@ -36,21 +38,61 @@ def _i64(u: int) -> int:
     return u - (1 << 64) if u >= (1 << 63) else u
 
 
-def broadcast_blob(meta: Optional[Sequence[int]], buf: Optional[torch.Tensor], nbytes_index: int,
-                   root: int, device) -> Tuple[List[int], torch.Tensor]:
-    """Broadcast a small int64 meta vector, then a byte buffer whose size is
-    meta[nbytes_index].  Non-root ranks pass meta=None, buf=None."""
+# hq_hash_meta <-> one int64 row of the metadata broadcast (column 15 is spare)
+META_COLS = 16
+
+
+def meta_row(m: hq.HashMeta) -> List[int]:
+    return ([m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout, m.pay_min, m.pay_max,
+             m.key_max] + [_i64(w) for w in m.pay_set] + [m.composite, 0])
+
+
+def meta_from_row(r: Sequence[int]) -> hq.HashMeta:
+    hm = hq.HashMeta()
+    (hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout,
+     hm.pay_min, hm.pay_max, hm.key_max) = [int(x) for x in r[:10]]
+    for k in range(4):
+        hm.pay_set[k] = int(r[10 + k]) & 0xFFFFFFFFFFFFFFFF
+    hm.composite = int(r[14])
+    return hm
+
+
+class RootError(hq.HQError):
+    """Raised on the ranks that did not fail when the root's build (or another rank's
+    pipeline) did: every rank raises, none is left waiting in a collective."""
+
+
+def broadcast_tables(rows: Optional[List[List[int]]], bufs: Optional[List[torch.Tensor]], n: int, root: int,
+                     device, err: Optional[BaseException] = None) -> Tuple[List[List[int]], List[torch.Tensor]]:
+    """Broadcast n root-built tables: ONE broadcast of an (n+1) x 16 int64 metadata block
+    (row n = the root's status: error code or 0), then one broadcast per byte buffer
+    (row[4] bytes each).  Root: rows / bufs given (bufs are sent in place); other ranks:
+    None, buffers are allocated here.  A root-side error is broadcast before the root
+    re-raises it, so the other ranks raise RootError instead of blocking in the next
+    collective."""
     rank = dist.get_rank()
-    m = torch.zeros(16, dtype=torch.int64, device=device)
+    meta = torch.zeros((n + 1, META_COLS), dtype=torch.int64, device=device)
     if rank == root:
-        m[: len(meta)] = torch.tensor(list(meta), dtype=torch.int64)
-    dist.broadcast(m, src=root)
-    meta_out = [int(x) for x in m.tolist()]
-    nbytes = meta_out[nbytes_index]
-    if rank != root:
-        buf = torch.empty(nbytes, dtype=torch.uint8, device=device)
-    dist.broadcast(buf, src=root)
-    return meta_out, buf
+        if err is not None:
+            meta[n, 0] = getattr(err, "code", hq.HQ_ERR_STATE) or hq.HQ_ERR_STATE
+        elif n:
+            meta[:n] = torch.tensor(rows, dtype=torch.int64)
+    dist.broadcast(meta, src=root)
+    if rank == root:
+        if err is not None:
+            raise err
+        for b in bufs:
+            dist.broadcast(b, src=root)
+        return rows, bufs
+    m = meta.cpu().tolist()
+    if m[n][0] != 0:
+        raise RootError(int(m[n][0]), "hash build failed on the root rank")
+    out = []
+    for r in m[:n]:
+        b = torch.empty(int(r[4]), dtype=torch.uint8, device=device)
+        dist.broadcast(b, src=root)
+        out.append(b)
+    return m[:n], out
 
 
 def reduce_partials(t: torch.Tensor, root: int) -> None:
@@ -84,54 +126,51 @@ class DistributedEngine(Engine):
         self.device = torch.device("cuda", ctx.device)
         self._built: List[hq.Hash] = []
         self.builds_here = self.rank == root
+        # HQ_DIST_FAULT_TRACE=1 (debug): re-read every root build's fault word after the
+        # final fetch and report the ones that changed since the build
+        self._trace: Optional[List[Tuple[str, hq.Hash, List[int]]]] = (
+            [] if os.environ.get("HQ_DIST_FAULT_TRACE") == "1" else None)
 
-    def _share_many(self, hs: Sequence[Optional[hq.Hash]]) -> List[hq.Hash]:
-        """Broadcast several root-built tables: ONE broadcast of all their metadata (the
-        root sends what it knows on the host; only the other ranks read it back), then one
-        asynchronous broadcast per slot array, then the imports -- instead of a metadata
-        broadcast and host read per table (each a stream sync)."""
-        n = len(hs)
-        meta = torch.zeros((max(n, 1), 16), dtype=torch.int64, device=self.device)
-        views = []
+    def _share_many(self, hs: Optional[Sequence[hq.Hash]], n: int, err: Optional[BaseException] = None) -> List[hq.Hash]:
+        """Broadcast n root-built tables (broadcast_tables: one metadata broadcast, one
+        asynchronous broadcast per slot array, no host read on the root) and import them
+        on the other ranks.  Build faults are not read here (that would sync per table):
+        the root's fault words travel with the pipeline's reduce (_reduce_checked)."""
         if self.rank == self.root:
-            rows = []
-            for h in hs:
-                ptr, m = h.device_view()
-                self._built.append(h)  # build faults are checked in finish()
-                views.append(device_view(ptr, int(m.bytes)))
-                rows.append([m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout,
-                             m.pay_min, m.pay_max, m.key_max] + [_i64(w) for w in m.pay_set] + [m.composite, 0])
-            meta[:n] = torch.tensor(rows, dtype=torch.int64)
-        dist.broadcast(meta, src=self.root)
-        if self.rank == self.root:
-            for v in views:
-                dist.broadcast(v, src=self.root)
+            rows, views = [], []
+            if err is None:
+                for h in hs:
+                    ptr, m = h.device_view()
+                    self._built.append(h)
+                    if self._trace is not None:
+                        self._trace.append((f"build#{len(self._trace)} rows={m.nkeys} cap={m.capacity}", h,
+                                            self._faults_of(h)))
+                    views.append(device_view(ptr, int(m.bytes)))
+                    rows.append(meta_row(m))
+            broadcast_tables(rows, views, n, self.root, self.device, err)
             return list(hs)
-        rows = meta.cpu().tolist()
-        out = []
-        for r in rows[:n]:
-            buf = torch.empty(int(r[4]), dtype=torch.uint8, device=self.device)
-            dist.broadcast(buf, src=self.root)
-            hm = hq.HashMeta()
-            (hm.capacity, hm.slot_words, hm.npayload, hm.nkeys, hm.bytes, hm.key_min, hm.layout,
-             hm.pay_min, hm.pay_max, hm.key_max) = r[:10]
-            for k in range(4):
-                hm.pay_set[k] = r[10 + k] & 0xFFFFFFFFFFFFFFFF
-            hm.composite = r[14]
-            out.append(self.ctx.import_hash(hm, buf.data_ptr(), keep=buf))
-        return out
+        rows, bufs = broadcast_tables(None, None, n, self.root, self.device)
+        return [self.ctx.import_hash(meta_from_row(r), b.data_ptr(), keep=b) for r, b in zip(rows, bufs)]
+
+    def _root_build(self, fn, n: int):
+        hs, err = None, None
+        if self.rank == self.root:
+            try:
+                hs = fn()
+            except hq.HQError as e:
+                err = e
+        return self._share_many(hs, n, err)
 
     def hash(self, table, key, payload=(), preds=(), expected_rows=0, key2=None) -> hq.Hash:
-        h = super().hash(table, key, payload, preds, expected_rows, key2) if self.rank == self.root else None
-        return self._share_many([h])[0]
+        return self._root_build(lambda: [super(DistributedEngine, self).hash(table, key, payload, preds,
+                                                                             expected_rows, key2)], 1)[0]
 
     def hashes(self, specs) -> List[hq.Hash]:
-        hs = super().hashes(specs) if self.rank == self.root else [None] * len(specs)
-        return self._share_many(hs)
+        return self._root_build(lambda: super(DistributedEngine, self).hashes(specs), len(specs))
 
     def hash_from(self, res, names, key, payload=(), preds=()) -> hq.Hash:
-        h = super().hash_from(res, names, key, payload, preds) if self.rank == self.root else None
-        return self._share_many([h])[0]
+        return self._root_build(lambda: [super(DistributedEngine, self).hash_from(res, names, key, payload,
+                                                                                  preds)], 1)[0]
 
     @staticmethod
     def _hash_grouped(P: hq.Plan) -> bool:
@@ -157,24 +196,63 @@ class DistributedEngine(Engine):
             P.norder, P.limit = 0, 0
         return super().run(pb, partitioned)
 
+    def _faults_of(self, h: hq.Hash) -> List[int]:
+        st = torch.zeros(hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
+        self.ctx.gather_faults([h], [], st.data_ptr())
+        return st.tolist()
+
+    def _trace_report(self, where: str) -> None:
+        if not self._trace:
+            return
+        for label, h, before in self._trace:
+            now = self._faults_of(h)
+            if now != before:
+                print(f"[hq dist trace] rank {self.rank} {where}: {label} fault words {before} -> {now}",
+                      file=sys.stderr, flush=True)
+        self._trace.clear()
+
+    def _reduce_checked(self, res: hq.Result) -> None:
+        """ONE all-reduce of [dense partials | fault words]: the partials are summed
+        (exact int64), and the fault words -- the root's build faults and every rank's
+        pipeline faults, gathered on the device (hq_gather_faults) -- are summed too, so
+        every rank sees every rank's faults and raises, or none does.  One host read of
+        the 32 fault words at the end; no per-table synchronisation."""
+        ptr, nbytes = res.partials_view()
+        n = nbytes // 8
+        red = torch.empty(n + hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
+        red[:n].copy_(device_view(ptr, nbytes, torch.int64))
+        built, self._built = self._built, []
+        self.ctx.gather_faults(built, [res], red.data_ptr() + n * 8)
+        reduce_partials(red, self.root)
+        res.from_partials(red.data_ptr(), nbytes)
+        hq.raise_faults(red[n:].tolist())
+
+    def _root_only_checked(self, res: Optional[hq.Result]) -> None:
+        """A root-only final pipeline: the root's build and pipeline faults are shared
+        with one small all-reduce, so that all ranks raise together."""
+        st = torch.zeros(hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
+        built, self._built = self._built, []
+        if self.rank == self.root:
+            self.ctx.gather_faults(built, [res] if res is not None else [], st.data_ptr())
+        dist.all_reduce(st)
+        hq.raise_faults(st.tolist())
+
     def finish(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
-        """Dense aggregates: one all-reduce of the partials, root finalizes.
-        Hash group-bys (e.g. TPC-H Q3 by l_orderkey): every rank finalizes its
-        groups, the rows are all-gathered to the root, which merges them with one
-        more fused GROUP BY pipeline on its GPU (and applies ORDER BY / LIMIT)."""
-        for h in self._built:  # root: raise duplicate-key / build faults (syncs)
-            h.info()
-        self._built.clear()
-        if getattr(pb, "root_only", False):  # no collective: the root ran the whole pipeline
-            return fetch(res, pb.result_names) if self.rank == self.root else None
-        if not hasattr(pb, "dist_order"):
-            ptr, nbytes = res.partials_view()
-            t = device_view(ptr, nbytes, torch.int64)
-            reduce_partials(t, self.root)
-            if self.rank != self.root:
-                return None
-            return fetch(res, pb.result_names)
-        return self._merge_groups(res, pb)
+        """Dense aggregates: one all-reduce of the partials (with every rank's fault
+        words), root finalizes.  Hash group-bys (e.g. TPC-H Q3 by l_orderkey): every rank
+        finalizes its groups, the rows are all-gathered to the root, which merges them
+        with one more fused GROUP BY pipeline on its GPU (and applies ORDER BY / LIMIT)."""
+        if getattr(pb, "root_only", False):  # no data collective: the root ran the whole pipeline
+            self._root_only_checked(res)
+            out = fetch(res, pb.result_names) if self.rank == self.root else None
+        elif not hasattr(pb, "dist_order"):
+            self._reduce_checked(res)
+            out = fetch(res, pb.result_names) if self.rank == self.root else None
+        else:
+            out = self._merge_groups(res, pb)
+        if self._trace is not None:
+            self._trace_report("after fetch")
+        return out
 
     def key_domain(self, table: str, col: str):
         """The key domain over ALL ranks' partitions (min / max all-reduced), so every rank
@@ -196,8 +274,7 @@ class DistributedEngine(Engine):
         if hasattr(pb, "dist_order"):
             merged = self._merge_device(res, pb)
             return merged[0] if merged is not None else None
-        ptr, nbytes = res.partials_view()
-        reduce_partials(device_view(ptr, nbytes, torch.int64), self.root)
+        self._reduce_checked(res)
         return res if self.rank == self.root else None
 
     def _merge_groups(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
@@ -212,31 +289,48 @@ class DistributedEngine(Engine):
     def _merge_device(self, res: hq.Result, pb: PlanBuilder):
         """All-gather the ranks' finalized groups; the root merges them with one fused
         GROUP BY pipeline (ORDER BY / LIMIT applied there).  Root: (result, plan, qualifying
-        rows over all ranks); other ranks: None."""
+        rows over all ranks); other ranks: None.  A rank whose local finalize fails (a
+        pipeline fault) still takes part in the status all-reduce, then every rank raises."""
         P = pb.plan
         names = list(pb.result_names)
-        tab = res.as_table(names)  # finalized local groups, device columns
-        cols = []
-        for c in range(len(names)):
-            ptr, _ = tab.column_ptr(c)
-            cols.append(device_view(ptr, max(tab.nrows, 1) * 8, torch.int64)[: tab.nrows])
-        qual = torch.tensor([res.qualifying()], dtype=torch.int64, device=self.device)
-        dist.all_reduce(qual)
-        n = torch.tensor([tab.nrows], dtype=torch.int64, device=self.device)
+        # status = [qualifying rows, ranks that failed, fault words...], one SUM all-reduce
+        st = torch.zeros(2 + hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
+        built, self._built = self._built, []
+        self.ctx.gather_faults(built, [], st.data_ptr() + 16)  # the root's build faults
+        err, tab, nrows = None, None, 0
+        try:
+            tab = res.as_table(names)  # finalized local groups (re-runs a full group table)
+            nrows = tab.nrows
+            st[0] = res.qualifying()
+        except hq.HQError as e:
+            err = e
+            st[1] = 1
+        dist.all_reduce(st)
+        stl = st.tolist()
+        if err is not None:
+            raise err
+        if stl[1]:
+            raise RootError(hq.HQ_ERR_STATE, "pipeline failed on another rank")
+        hq.raise_faults(stl[2:])
+        qual = int(stl[0])
+        ncol = len(names)
+        n = torch.tensor([nrows], dtype=torch.int64, device=self.device)
         sizes = [torch.zeros_like(n) for _ in range(self.world)]
         dist.all_gather(sizes, n)
         sizes = [int(s.item()) for s in sizes]
         m = max(max(sizes), 1)
-        merged = []
-        for c in cols:
-            pad = torch.zeros(m, dtype=torch.int64, device=self.device)
-            pad[: c.numel()] = c
-            bufs = [torch.empty_like(pad) for _ in range(self.world)]
-            dist.all_gather(bufs, pad)
-            merged.append(torch.cat([b[:s] for b, s in zip(bufs, sizes)]))
+        # ONE all-gather of the packed [ncol, m] group rows
+        pad = torch.zeros((ncol, m), dtype=torch.int64, device=self.device)
+        for c in range(ncol):
+            ptr, _ = tab.column_ptr(c)
+            if nrows:
+                pad[c, :nrows] = device_view(ptr, nrows * 8, torch.int64)
+        bufs = [torch.empty_like(pad) for _ in range(self.world)]
+        dist.all_gather(bufs, pad)
         if self.rank != self.root:
             return None
-        mt = self.ctx.load_columns({nm: t.contiguous() for nm, t in zip(names, merged)})
+        merged = [torch.cat([b[c, :s] for b, s in zip(bufs, sizes)]).contiguous() for c in range(ncol)]
+        mt = self.ctx.load_columns({nm: t for nm, t in zip(names, merged)})
         mb = PlanBuilder(mt)
         keys = [(names[i], P.key_min[i], P.key_card[i]) for i in range(P.nkeys)]
         fmap = {hq.AGG_SUM: "sum", hq.AGG_COUNT: "sum", hq.AGG_MIN: "min", hq.AGG_MAX: "max"}
@@ -249,4 +343,4 @@ class DistributedEngine(Engine):
         mb.aggregate(keys=keys, aggs=aggs, order=[(names[c], bool(d)) for c, d in order], limit=limit,
                      group_capacity=max(1024, sum(sizes)), agg_names=names[P.nkeys:])
         mb.root_only = True
-        return self.ctx.run(mb.plan, keep=mb.keep + [merged]), mb, int(qual.item())
+        return self.ctx.run(mb.plan, keep=mb.keep + [merged]), mb, qual

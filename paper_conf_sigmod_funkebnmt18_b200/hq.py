@@ -32,7 +32,7 @@ I_LOAD, I_ADD, I_SUB, I_RSUB, I_MUL, I_DIV, I_MOD = 1, 2, 3, 4, 5, 6, 7
 I_AND_EQ, I_AND_NE, I_AND_LT, I_AND_LE, I_AND_GT, I_AND_GE, I_AND_IN, I_OR = 8, 9, 10, 11, 12, 13, 14, 15
 AGG_SUM, AGG_COUNT, AGG_MIN, AGG_MAX, AGG_AVG = 1, 2, 3, 4, 5
 SINK_AGG, SINK_MATERIALISE = 1, 2
-RES_LRGP, RES_ATOMIC = 0, 1
+RES_LRGP, RES_ATOMIC, RES_WE = 0, 1, 2
 EXEC_FUSED, EXEC_OAAT, EXEC_FUSED_INTERP, EXEC_MULTIPASS = 0, 1, 2, 3
 
 
@@ -121,7 +121,8 @@ EXPORTS = ["hq_ctx_create", "hq_ctx_destroy", "hq_ctx_set_stream", "hq_ctx_sync"
            "hq_hash_device_view", "hq_hash_import", "hq_free_hash", "hq_run_pipeline", "hq_run_pipeline_streamed",
            "hq_finalize",
            "hq_result_info_get", "hq_fetch_result", "hq_result_as_table", "hq_result_partials_view",
-           "hq_free_result"]
+           "hq_result_from_partials", "hq_gather_faults", "hq_raise_faults", "hq_free_result"]
+FAULT_WORDS = 32
 
 
 class HQError(RuntimeError):
@@ -160,6 +161,9 @@ def lib():
             "hq_fetch_result": [vp, vp, P(vp), i64, P(i64)],
             "hq_result_as_table": [vp, vp, P(vp)],
             "hq_result_partials_view": [vp, P(vp), P(ctypes.c_size_t)], "hq_free_result": [vp],
+            "hq_result_from_partials": [vp, vp, vp, ctypes.c_size_t],
+            "hq_gather_faults": [vp, P(vp), i32, P(vp), i32, vp],
+            "hq_raise_faults": [P(i64)],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -298,6 +302,13 @@ class Context:
         h = ctypes.c_void_p()
         check(lib().hq_hash_import(self.h, ctypes.byref(meta), ctypes.c_void_p(dev_ptr), ctypes.byref(h)))
         return Hash(self, h, keep=[keep])
+
+    def gather_faults(self, hashes: Sequence["Hash"], results: Sequence["Result"], dev_out: int) -> None:
+        """Enqueue the OR of the hashes' build and the results' pipeline fault words into
+        FAULT_WORDS int64 at device address dev_out (no host sync; hq_gather_faults)."""
+        hs = (ctypes.c_void_p * max(len(hashes), 1))(*[h.h for h in hashes])
+        rs = (ctypes.c_void_p * max(len(results), 1))(*[r.h for r in results])
+        check(lib().hq_gather_faults(self.h, hs, len(hashes), rs, len(results), ctypes.c_void_p(dev_out)))
 
     def run(self, plan: Plan, keep=(), block_rows: Optional[int] = None) -> "Result":
         """Enqueue a pipeline.  block_rows: batch processing of an HQ_HOST_STREAM fact
@@ -452,6 +463,10 @@ class Result:
         check(lib().hq_result_partials_view(self.h, ctypes.byref(p), ctypes.byref(n)))
         return p.value, n.value
 
+    def from_partials(self, dev_ptr: int, nbytes: int) -> None:
+        """Copy reduced partials back into the result's group table (hq_result_from_partials)."""
+        check(lib().hq_result_from_partials(self.ctx.h, self.h, ctypes.c_void_p(dev_ptr), nbytes))
+
     def free(self) -> None:
         if self.h:
             lib().hq_free_result(self.h)
@@ -462,6 +477,12 @@ class Result:
             self.free()
         except Exception:
             pass
+
+
+def raise_faults(words: Sequence[int]) -> None:
+    """Raise the HQError a set of gathered (and rank-summed) fault words maps to."""
+    arr = (ctypes.c_int64 * FAULT_WORDS)(*[int(w) for w in words])
+    check(lib().hq_raise_faults(arr))
 
 
 # ---- plan construction helpers ----------------------------------------------

@@ -1,0 +1,84 @@
+#!/usr/bin/env python
+"""GPU timeline of one query step (CUPTI through torch.profiler): every kernel and
+memcpy of the step with its start offset and duration, the idle gaps between them,
+and the CUDA runtime calls that block the host (stream syncs) -- where the time
+outside the fused kernel goes.
+
+    python scripts/step_trace.py --query ssb_q41 --sf 100 [--steps 3] [--json out.json]
+"""
+import argparse
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+from paper_conf_sigmod_funkebnmt18_b200 import hq  # noqa: E402
+from paper_conf_sigmod_funkebnmt18_b200.engine import Engine  # noqa: E402
+from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES, load_tables  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--query", default="ssb_q41")
+    ap.add_argument("--sf", type=float, default=10)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--json", default="")
+    a = ap.parse_args()
+    torch.cuda.set_device(0)
+    q = QUERIES[a.query]
+    ctx = hq.Context(0)
+    tables = load_tables(ctx, q, a.sf)
+    ctx.sync()
+    E = Engine(ctx, tables)
+    for _ in range(3):
+        q.execute(E)
+    torch.cuda.synchronize()
+    from torch.profiler import ProfilerActivity, profile
+    marks = []
+    with profile(activities=[ProfilerActivity.CPU, ProfilerActivity.CUDA]) as prof:
+        for _ in range(a.steps):
+            torch.cuda.synchronize()
+            with torch.profiler.record_function("hq_step"):
+                q.execute(E)
+            torch.cuda.synchronize()
+    evs = prof.events()
+    steps = sorted([e for e in evs if e.name == "hq_step"], key=lambda e: e.time_range.start)
+    gpu = sorted([e for e in evs if e.device_type == torch.autograd.DeviceType.CUDA],
+                 key=lambda e: e.time_range.start)
+    syncs = [e for e in evs if e.device_type == torch.autograd.DeviceType.CPU and "Synchronize" in e.name]
+    out = []
+    for si, st in enumerate(steps):
+        t0, t1 = st.time_range.start, st.time_range.end
+        ks = [e for e in gpu if t0 <= e.time_range.start <= t1]
+        ss = [e for e in syncs if t0 <= e.time_range.start <= t1]
+        rows = []
+        prev = None
+        busy = 0.0
+        for e in ks:
+            s, d = e.time_range.start - t0, e.time_range.end - e.time_range.start
+            gap = (e.time_range.start - prev) if prev is not None else s
+            prev = max(prev or 0, e.time_range.end)
+            busy += d
+            rows.append({"name": e.name[:70], "start_us": s, "dur_us": d, "gap_before_us": gap})
+        rec = {"step": si, "host_us": t1 - t0, "gpu_busy_us": busy, "n_gpu_ops": len(ks),
+               "syncs": [{"name": x.name, "start_us": x.time_range.start - t0,
+                          "dur_us": x.time_range.end - x.time_range.start} for x in ss], "ops": rows}
+        out.append(rec)
+        print(f"step {si}: host {rec['host_us']:.1f} us, GPU busy {busy:.1f} us over {len(ks)} ops, "
+              f"{len(ss)} host syncs ({sum(x['dur_us'] for x in rec['syncs']):.1f} us blocked)")
+        if si == len(steps) - 1:
+            for r in rows:
+                print(f"  +{r['start_us']:9.1f} us  gap {r['gap_before_us']:8.1f}  dur {r['dur_us']:9.1f}  {r['name']}")
+            for x in rec["syncs"]:
+                print(f"  sync at +{x['start_us']:.1f} us for {x['dur_us']:.1f} us ({x['name']})")
+    if a.json:
+        with open(a.json, "w") as f:
+            json.dump({"query": a.query, "sf": a.sf, "steps": out}, f, indent=1)
+
+
+if __name__ == "__main__":
+    main()

@@ -331,6 +331,22 @@ int main(int argc, char** argv) {
     shapes.push_back({"composite_probe", P, nullptr});
   }
 
+  // Resolution:WE (App C, Fig 24) variants: B3-WE tree, A3-WE scan, C3-WE sort +
+  // segmented scan into a dense and into a hash global table
+  {
+    std::vector<Shape> wes;
+    for (const Shape& s : shapes) {
+      if (s.name != "star_ranked_dense" && s.name != "materialise_lrgp" && s.name != "scalar_filters" &&
+          s.name != "global_hash_groups")
+        continue;
+      Shape w = s;
+      w.name = s.name + "_we";
+      w.plan.resolution = HQ_RES_WE;
+      wes.push_back(w);
+    }
+    for (const Shape& w : wes) shapes.push_back(w);
+  }
+
   // multi-pass count / write kernels (HQ_EXEC_MULTIPASS) of a grouped star
   // join, a materialising pipeline and a scalar aggregate
   {

@@ -32,7 +32,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     env = {k: v for k, v in os.environ.items() if not k.startswith("HQ_")}
     p = subprocess.run([checker, str(tmp_path)], capture_output=True, text=True, env=env, timeout=600)
     assert p.returncode == 0, p.stdout + p.stderr
-    assert p.stdout.startswith("OK 24 of 24"), p.stdout
+    assert p.stdout.startswith("OK 28 of 28"), p.stdout
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
     star = srcs["star_dense_lrgp"]

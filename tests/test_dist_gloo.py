@@ -2,7 +2,9 @@
 range-partition / broadcast / reduce functions the NCCL path uses
 (paper_conf_sigmod_funkebnmt18_b200.dist), with a TEST-ONLY numpy stand-in for
 the device engine's partial aggregates.  Pins: the reduced partials of the two
-ranks equal the oracle on the whole table; broadcast blobs arrive intact."""
+ranks equal the oracle on the whole table; broadcast tables (metadata rows and
+buffers) arrive intact for 0, 1 and 3 tables; a root-side build error makes every
+rank raise."""
 import os
 import socket
 
@@ -13,7 +15,9 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 import hqgen
-from paper_conf_sigmod_funkebnmt18_b200.dist import broadcast_blob, partition, reduce_partials
+from paper_conf_sigmod_funkebnmt18_b200 import hq
+from paper_conf_sigmod_funkebnmt18_b200.dist import (RootError, broadcast_tables, meta_from_row, meta_row, partition,
+                                                     reduce_partials)
 
 SF = 0.01
 
@@ -42,6 +46,18 @@ def _q41_partials(lo, c, s, p, d):
     return t
 
 
+def _stub_meta(k, nbytes):
+    """A hash-table metadata record with every field set (pay_set words with bit 63 on)."""
+    m = hq.HashMeta()
+    m.capacity, m.slot_words, m.npayload, m.nkeys = 1 << (10 + k), 2, 1, 1000 + k
+    m.bytes, m.key_min, m.layout = nbytes, -5 - k, k % 2
+    m.pay_min, m.pay_max, m.key_max = -3, 200 + k, 99999
+    for i in range(4):
+        m.pay_set[i] = (1 << 63) | (0x0123456789ABCDEF >> i) | k
+    m.composite = k % 2
+    return m
+
+
 def _worker(rank, world, port, q):
     try:
         os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -51,14 +67,34 @@ def _worker(rank, world, port, q):
         a, b = partition(n, rank, world)
         lo = hqgen.generate("lineorder", SF, row_range=(a, b))
         dims = {t: hqgen.generate(t, SF) for t in ("customer", "supplier", "part", "date")}
-        # root "builds" and broadcasts a blob (the hash-table slot array on GPUs)
+        # root "builds" and broadcasts tables (the hash-table slot arrays on GPUs): n = 0, 1, 3
         blob = np.ascontiguousarray(dims["customer"]["c_custkey"][dims["customer"]["c_region"] == 1]).view(np.uint8)
+        for nt in (0, 1, 3):
+            blobs = [np.roll(blob, k).copy() for k in range(nt)]
+            metas = [_stub_meta(k, x.nbytes) for k, x in enumerate(blobs)]
+            if rank == 0:
+                rows, bufs = broadcast_tables([meta_row(m) for m in metas], [torch.from_numpy(x) for x in blobs], nt, 0,
+                                              "cpu")
+            else:
+                rows, bufs = broadcast_tables(None, None, nt, 0, "cpu")
+            assert len(rows) == len(bufs) == nt
+            for m, r, buf, ref in zip(metas, rows, bufs, blobs):
+                got = meta_from_row(r)
+                assert bytes(got) == bytes(m)  # every field, pay_set bit 63 included
+                assert np.array_equal(buf.numpy(), ref)
+        # a root-side build error: the root re-raises it, the other rank raises RootError
         if rank == 0:
-            meta, buf = broadcast_blob([7, 2, 1, 0, blob.nbytes], torch.from_numpy(blob.copy()), 4, 0, "cpu")
+            try:
+                broadcast_tables(None, None, 2, 0, "cpu", err=hq.HQError(hq.HQ_ERR_DUP_KEY, "dup"))
+                raise AssertionError("root did not re-raise")
+            except hq.HQError as e:
+                assert e.code == hq.HQ_ERR_DUP_KEY and not isinstance(e, RootError)
         else:
-            meta, buf = broadcast_blob(None, None, 4, 0, "cpu")
-        assert meta[:5] == [7, 2, 1, 0, blob.nbytes]
-        assert np.array_equal(buf.numpy(), blob)
+            try:
+                broadcast_tables(None, None, 2, 0, "cpu")
+                raise AssertionError("rank 1 did not raise")
+            except RootError as e:
+                assert e.code == hq.HQ_ERR_DUP_KEY
         part = torch.from_numpy(_q41_partials(lo, dims["customer"], dims["supplier"], dims["part"], dims["date"]).ravel().copy())
         reduce_partials(part, 0)
         if rank == 0:

@@ -638,7 +638,8 @@ def test_tpch_q9_golden(ctx, golden):
         assert g.qualifying == fx["expected"]["qualifying"]
 
 
-@pytest.mark.parametrize("qname,sf", [("ssb_q41", 100.0), ("ssb_q31", 30.0), ("tpch_q3", 30.0), ("tpch_q1", 10.0)])
+@pytest.mark.parametrize("qname,sf", [("ssb_q41", 100.0), ("ssb_q31", 30.0), ("tpch_q3", 30.0), ("tpch_q1", 10.0),
+                                      ("ssb_q11", 10.0), ("ssb_q12", 10.0), ("ssb_q13", 10.0), ("tpch_q6", 10.0)])
 def test_bench_configs_full_size(ctx, qname, sf):
     """BASELINE.json's configs at their full sizes, in the launch configuration bench.py
     times (generated fused kernel, default plan), element by element against the oracle
@@ -655,6 +656,10 @@ def test_bench_configs_full_size(ctx, qname, sf):
         o = oracle.ssb_q31(host["lineorder"], host["customer"], host["supplier"], host["date"], nthreads=nt)
     elif qname == "tpch_q3":
         o = oracle.tpch_q3(host["tpch_customer"], host["orders"], host["lineitem"], nthreads=nt)
+    elif qname.startswith("ssb_q1"):
+        o = oracle.ssb_q1(int(qname[-1]), host["lineorder"], host["date"], nthreads=nt)
+    elif qname == "tpch_q6":
+        o = oracle.tpch_q6(host["lineitem"], nthreads=nt)
     else:
         o = oracle.tpch_q1(host["lineitem"], nthreads=nt)
     E = Engine(ctx, load_tables(ctx, q, sf, host=host))
