@@ -94,6 +94,7 @@ typedef struct hq_ctx hq_ctx;
 typedef struct hq_table hq_table;
 typedef struct hq_hash hq_hash;
 typedef struct hq_result hq_result;
+typedef struct hq_graph hq_graph;
 
 /* Device memory hooks.  alloc returns a device pointer (>= 256-B aligned) or
  * NULL; both are called with the ctx stream. */
@@ -414,6 +415,32 @@ hq_status hq_gather_faults(hq_ctx* ctx, const hq_hash* const* hashes, int32_t nh
  * capacity) are not errors here: the owning result re-runs at its own finalize. */
 hq_status hq_raise_faults(const int64_t* host_words);
 hq_status hq_free_result(hq_result* r);
+
+/* ------------------------------------------------- prepared queries (CUDA graphs)
+ * A query whose steps need no host synchronisation -- its hash builds have cached
+ * statistics (a previous build of the same descriptor over the same table, see
+ * hq_build_hash), its pipelines are fused, its results are dense aggregates of at most
+ * 4,096 groups -- can be recorded once and replayed: between hq_ctx_capture_begin and
+ * hq_ctx_capture_end the calls the caller makes (hq_build_hash(es), hq_run_pipeline,
+ * hq_finalize) are enqueued into a CUDA graph instead of executed.  Every launch
+ * re-executes ALL the recorded device work -- builds (slot fill, insert, compact,
+ * statistics verification), the compound kernels, finalization -- into the same
+ * buffers, and leaves each finalized result readable (hq_result_info_get /
+ * hq_fetch_result) until the next launch.  Only the host-side planning (plan
+ * validation, layout, kernel selection, launch configuration) is done once, as for a
+ * prepared statement.  Calls that need the host while capturing fail with
+ * HQ_ERR_STATE (nothing is recorded after that; call hq_ctx_capture_abort): a build
+ * without cached statistics, hq_*_info / fetch, large or materialised finalizes,
+ * multi-pass / operator-at-a-time execution, batch processing, hq_load_columns.
+ * The graph keeps the objects its nodes use (results, hashes, build source tables)
+ * until hq_graph_destroy.  The capture runs on a private stream; launches run on the
+ * context stream and synchronise it (the rows are decoded on the host).  Needs the
+ * default stream-ordered allocator (no hq_allocator hooks: HQ_ERR_UNSUPPORTED). */
+hq_status hq_ctx_capture_begin(hq_ctx* ctx);
+hq_status hq_ctx_capture_end(hq_ctx* ctx, hq_graph** out);
+hq_status hq_ctx_capture_abort(hq_ctx* ctx);
+hq_status hq_graph_launch(hq_ctx* ctx, hq_graph* g);
+hq_status hq_graph_destroy(hq_graph* g);
 
 #ifdef __cplusplus
 }

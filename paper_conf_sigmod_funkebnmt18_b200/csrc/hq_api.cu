@@ -42,7 +42,15 @@ void hq_set_error(const std::string& msg) { g_last_error = msg; }
 void* hq_ctx::alloc_bytes(size_t bytes) {
   if (bytes == 0) bytes = 16;
   void* p = nullptr;
-  if (has_alloc) {
+  if (capturing) {
+    // not a captured node: the pool allocation happens now, on a stream of its own,
+    // and the memory belongs to the graph's objects (or is freed with the graph)
+    if (has_alloc) HQ_THROW(HQ_ERR_UNSUPPORTED, "graph capture needs the stream-ordered pool (no allocator hooks)");
+    if (cudaMallocAsync(&p, bytes, alloc_stream) != cudaSuccess || cudaStreamSynchronize(alloc_stream) != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+    }
+  } else if (has_alloc) {
     p = alloc.alloc(bytes, (void*)stream, alloc.user);
   } else {
     cudaError_t e = cudaMallocAsync(&p, bytes, stream);
@@ -56,6 +64,10 @@ void* hq_ctx::alloc_bytes(size_t bytes) {
 }
 void hq_ctx::free_bytes(void* p, size_t bytes) {
   if (!p) return;
+  if (capturing) {  // captured work may still use it at every launch: freed with the graph
+    cap_frees.emplace_back(p, bytes);
+    return;
+  }
   if (has_alloc) alloc.free(p, bytes, (void*)stream, alloc.user);
   else cudaFreeAsync(p, stream);
 }
@@ -65,9 +77,93 @@ hq_table::~hq_table() {
   if (backing) backing->release();
 }
 hq_result::~hq_result() {
+  if (stage_host) cudaFreeHost(stage_host);
   if (fact) fact->release();
   for (auto* h : hashes) h->release();
 }
+
+void hq_ctx::release() {
+  if (refs.fetch_sub(1) != 1) return;
+  hq_ctx* ctx = this;
+  {
+    cudaStreamSynchronize(ctx->stream);
+    for (auto& e : ctx->events) {
+      cudaEventDestroy(e.first);
+      cudaEventDestroy(e.second);
+    }
+    for (auto e : ctx->event_pool) cudaEventDestroy(e);
+    if (ctx->pinned) cudaFreeHost(ctx->pinned);
+    if (ctx->pinned_build) cudaFreeHost(ctx->pinned_build);
+    if (ctx->copy_stream) {
+      cudaStreamSynchronize(ctx->copy_stream);
+      cudaStreamDestroy(ctx->copy_stream);
+    }
+    for (int i = 0; i < 2; ++i) {
+      if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
+      if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
+    }
+    for (int i = 0; i < hq_ctx::NSIDE; ++i) {
+      if (ctx->side[i]) {
+        cudaStreamSynchronize(ctx->side[i]);
+        cudaStreamDestroy(ctx->side[i]);
+      }
+      if (ctx->ev_join[i]) cudaEventDestroy(ctx->ev_join[i]);
+    }
+    if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
+    if (ctx->cap_stream) cudaStreamDestroy(ctx->cap_stream);
+    if (ctx->alloc_stream) cudaStreamDestroy(ctx->alloc_stream);
+    delete ctx;
+  }
+}
+
+void hq_sync(hq_ctx* ctx, const char* what) {
+  hq_require_eager(ctx, what);
+  HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+}
+void hq_require_eager(hq_ctx* ctx, const char* what) {
+  if (ctx->capturing)
+    HQ_THROW(HQ_ERR_STATE, std::string("not capturable in a CUDA graph: ") + what +
+                               " needs the host (a synchronisation); run the query eagerly");
+}
+
+// A captured prepared query: the instantiated graph, the objects its nodes read and
+// write (retained), the results whose rows it stages, and buffers freed during capture.
+struct hq_graph {
+  CtxPtr ctx;
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+  std::vector<RefObj*> objs;
+  std::vector<hq_result*> results;
+  std::vector<std::pair<void*, size_t>> frees;
+  int64_t nkernels = 0;  // kernels one launch runs (hq_ctx_launches accounting)
+  ~hq_graph() {
+    hq_ctx* c = ctx;
+    if (c) cudaStreamSynchronize(c->stream);
+    if (exec) cudaGraphExecDestroy(exec);
+    if (graph) cudaGraphDestroy(graph);
+    for (auto& f : frees) c->free_bytes(f.first, f.second);
+    for (RefObj* o : objs) o->release();
+  }
+};
+
+static void capture_cleanup(hq_ctx* ctx, hq_graph* g) {
+  // frees and retained objects go to the graph (or are released if there is none)
+  ctx->capturing = false;
+  ctx->stream = ctx->user_stream;
+  if (g) {
+    g->frees.swap(ctx->cap_frees);
+    g->objs.swap(ctx->cap_objs);
+    g->results.swap(ctx->cap_results);
+  } else {
+    cudaStreamSynchronize(ctx->stream);
+    for (auto& f : ctx->cap_frees) ctx->free_bytes(f.first, f.second);
+    for (RefObj* o : ctx->cap_objs) o->release();
+  }
+  ctx->cap_frees.clear();
+  ctx->cap_objs.clear();
+  ctx->cap_results.clear();
+}
+
 
 extern "C" {
 
@@ -120,33 +216,81 @@ hq_status hq_ctx_create(int32_t device, void* stream, const hq_allocator* alloc,
 
 hq_status hq_ctx_destroy(hq_ctx* ctx) {
   return guarded([&] {
-    if (!ctx) return;
-    cudaStreamSynchronize(ctx->stream);
-    for (auto& e : ctx->events) {
-      cudaEventDestroy(e.first);
-      cudaEventDestroy(e.second);
-    }
-    for (auto e : ctx->event_pool) cudaEventDestroy(e);
-    if (ctx->pinned) cudaFreeHost(ctx->pinned);
-    if (ctx->pinned_build) cudaFreeHost(ctx->pinned_build);
-    if (ctx->copy_stream) {
-      cudaStreamSynchronize(ctx->copy_stream);
-      cudaStreamDestroy(ctx->copy_stream);
-    }
-    for (int i = 0; i < 2; ++i) {
-      if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
-      if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
-    }
-    for (int i = 0; i < hq_ctx::NSIDE; ++i) {
-      if (ctx->side[i]) {
-        cudaStreamSynchronize(ctx->side[i]);
-        cudaStreamDestroy(ctx->side[i]);
-      }
-      if (ctx->ev_join[i]) cudaEventDestroy(ctx->ev_join[i]);
-    }
-    if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
-    delete ctx;
+    if (ctx) ctx->release();  // objects still alive keep the context until they are freed
   });
+}
+
+hq_status hq_ctx_capture_begin(hq_ctx* ctx) {
+  return guarded([&] {
+    if (!ctx) HQ_THROW(HQ_ERR_ARG, "ctx is NULL");
+    if (ctx->capturing) HQ_THROW(HQ_ERR_STATE, "a capture is already running");
+    if (ctx->has_alloc) HQ_THROW(HQ_ERR_UNSUPPORTED, "graph capture needs the stream-ordered pool (no allocator hooks)");
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    if (!ctx->cap_stream) HQ_CUDA(cudaStreamCreateWithFlags(&ctx->cap_stream, cudaStreamNonBlocking));
+    if (!ctx->alloc_stream) HQ_CUDA(cudaStreamCreateWithFlags(&ctx->alloc_stream, cudaStreamNonBlocking));
+    ctx->user_stream = ctx->stream;
+    ctx->stream = ctx->cap_stream;
+    HQ_CUDA(cudaStreamBeginCapture(ctx->cap_stream, cudaStreamCaptureModeRelaxed));
+    ctx->capturing = true;
+    ctx->cap_launches0 = ctx->launches;
+  });
+}
+
+hq_status hq_ctx_capture_end(hq_ctx* ctx, hq_graph** out) {
+  return guarded([&] {
+    if (!ctx || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    if (!ctx->capturing) HQ_THROW(HQ_ERR_STATE, "no capture is running");
+    cudaGraph_t graph = nullptr;
+    const cudaError_t e = cudaStreamEndCapture(ctx->cap_stream, &graph);
+    if (e != cudaSuccess || !graph) {
+      cudaGetLastError();
+      capture_cleanup(ctx, nullptr);
+      HQ_THROW(HQ_ERR_CUDA, std::string("graph capture failed: ") + cudaGetErrorString(e));
+    }
+    hq_graph* g = new hq_graph();
+    g->ctx = ctx;
+    g->graph = graph;
+    g->nkernels = ctx->launches - ctx->cap_launches0;
+    capture_cleanup(ctx, g);
+    const cudaError_t ie = cudaGraphInstantiate(&g->exec, graph, 0);
+    if (ie != cudaSuccess) {
+      cudaGetLastError();
+      delete g;
+      HQ_THROW(HQ_ERR_CUDA, std::string("graph instantiation failed: ") + cudaGetErrorString(ie));
+    }
+    *out = g;
+  });
+}
+
+hq_status hq_ctx_capture_abort(hq_ctx* ctx) {
+  return guarded([&] {
+    if (!ctx || !ctx->capturing) return;
+    cudaGraph_t graph = nullptr;
+    cudaStreamEndCapture(ctx->cap_stream, &graph);
+    cudaGetLastError();
+    if (graph) cudaGraphDestroy(graph);
+    capture_cleanup(ctx, nullptr);
+  });
+}
+
+hq_status hq_graph_launch(hq_ctx* ctx, hq_graph* g) {
+  return guarded([&] {
+    if (!ctx || !g) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    if (ctx->capturing) HQ_THROW(HQ_ERR_STATE, "launch during a capture");
+    for (hq_result* r : g->results) {  // the graph refinalizes them: stale host rows go
+      r->host_ready = false;
+      r->finalized = false;
+      r->checked = false;
+    }
+    ctx->launches += g->nkernels;
+    HQ_CUDA(cudaGraphLaunch(g->exec, ctx->stream));
+    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    for (hq_result* r : g->results) hq_decode_captured(ctx, r);
+  });
+}
+
+hq_status hq_graph_destroy(hq_graph* g) {
+  return guarded([&] { delete g; });
 }
 
 hq_status hq_ctx_set_stream(hq_ctx* ctx, void* stream) {
@@ -158,6 +302,7 @@ hq_status hq_ctx_set_stream(hq_ctx* ctx, void* stream) {
 
 hq_status hq_ctx_sync(hq_ctx* ctx) {
   return guarded([&] {
+    if (ctx) hq_require_eager(ctx, "hq_ctx_sync");
     if (!ctx) HQ_THROW(HQ_ERR_ARG, "ctx is NULL");
     HQ_CUDA(cudaStreamSynchronize(ctx->stream));
   });
@@ -172,6 +317,7 @@ hq_status hq_ctx_enable_timing(hq_ctx* ctx, int32_t on) {
 
 hq_status hq_ctx_kernel_times(hq_ctx* ctx, float* ms, int32_t max, int32_t* n) {
   return guarded([&] {
+    if (ctx) hq_require_eager(ctx, "hq_ctx_kernel_times");
     if (!ctx || !n) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     int32_t k = 0;
     for (auto& e : ctx->events) {
@@ -199,6 +345,7 @@ hq_status hq_ctx_launches(hq_ctx* ctx, int64_t* n) {
 hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int64_t nrows, int32_t flags,
                           hq_table** out) {
   return guarded([&] {
+    if (ctx) hq_require_eager(ctx, "hq_load_columns");
     if (!ctx || !out || (!cols && ncols > 0)) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     if (ncols < 0 || ncols > HQ_MAX_COLS) HQ_THROW(HQ_ERR_UNSUPPORTED, "tables have 0..16 columns");
     if (nrows < 0) HQ_THROW(HQ_ERR_ARG, "nrows < 0");
@@ -239,6 +386,7 @@ hq_status hq_load_columns(hq_ctx* ctx, const hq_column* cols, int32_t ncols, int
 
 hq_status hq_column_range(hq_ctx* ctx, const hq_table* t, int32_t col, int64_t* min, int64_t* max) {
   return guarded([&] {
+    if (ctx) hq_require_eager(ctx, "hq_column_range");
     if (!ctx || !t || !min || !max) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     if (col < 0 || col >= t->ncols) HQ_THROW(HQ_ERR_ARG, "column out of range");
     hq_column_range_impl(ctx, t, col, min, max);
@@ -287,7 +435,11 @@ hq_status hq_build_hashes(hq_ctx* ctx, int32_t n, const hq_build_desc* descs, hq
       for (auto* h : hs) h->release();
       throw;
     }
-    for (int i = 0; i < n; ++i) out[i] = hs[i];
+    for (int i = 0; i < n; ++i) {  // a captured build re-reads its source at every launch
+      hs[i]->capture_retain(ctx);
+      const_cast<hq_table*>(descs[i].src)->capture_retain(ctx);
+      out[i] = hs[i];
+    }
   });
 }
 
@@ -309,6 +461,7 @@ hq_status hq_hash_device_view(const hq_hash* h, void** dev_ptr, hq_hash_meta* me
 
 hq_status hq_hash_import(hq_ctx* ctx, const hq_hash_meta* meta, void* dev_ptr, hq_hash** out) {
   return guarded([&] {
+    if (ctx) hq_require_eager(ctx, "hq_hash_import");
     if (!ctx || !meta || !dev_ptr || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     const int64_t cap = meta->capacity;
     if (meta->layout == HQ_HT_DIRECT) {
@@ -363,11 +516,14 @@ static void run_pipeline(hq_ctx* ctx, const hq_plan* plan, int64_t block_rows, h
         r->hashes.push_back(h);
       }
     try {
+      if (ctx->capturing && (r->stream_block > 0 || (plan->exec != HQ_EXEC_FUSED && plan->exec != HQ_EXEC_FUSED_INTERP)))
+        HQ_THROW(HQ_ERR_STATE, "not capturable in a CUDA graph: batch processing, multi-pass or operator-at-a-time");
       hq_prepare_result(ctx, plan, r);
     } catch (...) {
       r->release();
       throw;
     }
+    r->capture_retain(ctx);
     *out = r;
 }
 
@@ -393,6 +549,7 @@ hq_status hq_finalize(hq_ctx* ctx, hq_result* r) {
 
 hq_status hq_result_info_get(hq_ctx* ctx, hq_result* r, hq_result_info* out) {
   return guarded([&] {
+    if (ctx) hq_require_eager(ctx, "hq_result_info_get");
     if (!ctx || !r || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     hq_finalize_impl(ctx, r);
     std::memset(out, 0, sizeof(*out));
@@ -407,6 +564,7 @@ hq_status hq_result_info_get(hq_ctx* ctx, hq_result* r, hq_result_info* out) {
 hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int64_t capacity_rows,
                           int64_t* nrows_out) {
   return guarded([&] {
+    if (ctx) hq_require_eager(ctx, "hq_fetch_result");
     if (!ctx || !r) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     hq_finalize_impl(ctx, r);
     const int64_t n = std::min<int64_t>(r->nrows, capacity_rows);
@@ -430,6 +588,7 @@ hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int
 
 hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out) {
   return guarded([&] {
+    if (ctx) hq_require_eager(ctx, "hq_result_as_table");
     if (!ctx || !r || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     hq_finalize_impl(ctx, r, /*unordered=*/true);
     const bool mat = r->sink == HQ_SINK_MATERIALISE;
@@ -504,6 +663,7 @@ hq_status hq_raise_faults(const int64_t* w) {
     if (hb(HQF_BAD_KEY)) HQ_THROW(HQ_ERR_ARG, "hash build: key INT32_MIN or outside int32");
     if (hb(HQF_BAD_PAYLOAD)) HQ_THROW(HQ_ERR_ARG, "hash build: payload outside int32");
     if (hb(HQF_HT_FULL)) HQ_THROW(HQ_ERR_OVERFLOW, "hash build: table full (expected_rows too small)");
+    if (hb(HQF_STALE)) HQ_THROW(HQ_ERR_STATE, "hash build: source rows differ from the cached build statistics");
     if (pb(HQF_DIV_ZERO)) HQ_THROW(HQ_ERR_ARG, "pipeline: division by zero");
     if (pb(HQF_KEY_DOMAIN)) HQ_THROW(HQ_ERR_ARG, "pipeline: group key outside its declared [min, min+card)");
     if (pb(HQF_OVERFLOW)) HQ_THROW(HQ_ERR_OVERFLOW, "aggregate exceeds the int64 guard (|v| >= 2^62)");

@@ -41,6 +41,12 @@ struct KBuild {
   unsigned* ticket;  // count pass: blocks done
   int count_inserts; // build pass: accumulate the inserted-key count (no count pass ran)
   int composite;     // two-column key: equal key_col values take separate slots (no dup check)
+  // cached statistics (no count pass ran): the insert pass checks that the qualifying
+  // rows match them -- keys in [kmin, kmax], payload 0 in [pmin, pmax] and in set, as
+  // many rows -- and flags HQF_STALE otherwise
+  int verify;
+  BuildStats vs;
+  unsigned long long* vqual;  // qualifying rows seen by the insert pass
 };
 
 __device__ __forceinline__ long long ld_col(const KBuild& b, int c, long long row) {
@@ -218,7 +224,7 @@ __global__ void hq_fill_kernel(uint32_t* p, long long n, uint32_t v) {
 }
 
 __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid_constant__ KBuild b) {
-  unsigned long long inserted = 0;
+  unsigned long long inserted = 0, qual = 0;
   int fault = 0;
   const uint32_t shift = 32u - b.log2cap;
   const long long base = (long long)blockIdx.x * BUILD_BLOCK * BUILD_U + threadIdx.x;
@@ -245,6 +251,15 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid
 #pragma unroll
   for (int u = 0; u < BUILD_U; ++u) {
     if (!pass[u]) continue;
+    if (b.verify) {  // the rows the count pass would have summarised
+      ++qual;
+      if (kv[u] > (long long)INT_MIN && kv[u] <= (long long)INT_MAX && (kv[u] < b.vs.kmin || kv[u] > b.vs.kmax))
+        fault |= HQF_STALE;
+      if (b.npay > 0) {
+        const int pc = pv0[u] < (long long)INT_MIN ? INT_MIN : (pv0[u] > (long long)INT_MAX ? INT_MAX : (int)pv0[u]);
+        if (pc < b.vs.pmin || pc > b.vs.pmax || !((b.vs.set[(pc & 255) >> 5] >> (pc & 31)) & 1u)) fault |= HQF_STALE;
+      }
+    }
     if (kv[u] <= (long long)INT_MIN || kv[u] > (long long)INT_MAX) {
       fault |= HQF_BAD_KEY;
       continue;
@@ -275,6 +290,23 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid
     if (i > b.mask) fault |= HQF_HT_FULL;
   }
   if (fault) atomicOr(b.err, fault);
+  if (b.verify) {  // the number of qualifying rows must equal the cached count
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) qual += __shfl_xor_sync(0xffffffffu, qual, o);
+    __shared__ unsigned long long vred[BUILD_BLOCK / 32];
+    if ((threadIdx.x & 31) == 0) vred[threadIdx.x >> 5] = qual;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long t = 0;
+      for (int k = 0; k < BUILD_BLOCK / 32; ++k) t += vred[k];
+      if (t) atomicAdd(b.vqual, t);
+      __threadfence();
+      if (atomicAdd(b.ticket, 1u) == gridDim.x - 1) {  // last block: every block's rows are in
+        __threadfence();
+        if (*(volatile unsigned long long*)b.vqual != b.vs.cnt) atomicOr(b.err, HQF_STALE);
+      }
+    }
+  }
   if (!b.count_inserts) return;  // counted builds know their key count already
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) inserted += __shfl_xor_sync(0xffffffffu, inserted, o);
@@ -292,6 +324,11 @@ int64_t next_pow2(int64_t x) {
   int64_t c = 1;
   while (c < x) c <<= 1;
   return c;
+}
+
+bool stats_cache_on() {
+  const char* e = getenv("HQ_BUILD_STATS");
+  return !(e && e[0] == '0');
 }
 
 void to_kpred(const hq_pred& in, KBuildPred& out, int ncols) {
@@ -329,6 +366,8 @@ struct BuildState {
   int grid = 0;
   int words = 0;
   bool counted = false;
+  bool cached = false;     // statistics from hq_ctx::build_stats (no count pass, verified on device)
+  std::string stats_key;   // cache key; empty when the cache is off
   DevBuf scratch;  // count-pass block partials
   struct { unsigned long long cnt; int kmin, kmax, pmin, pmax; unsigned set[8]; } st{};
   void* host_st = nullptr;  // this build's slot in hq_ctx::pinned_build (st's layout)
@@ -366,6 +405,32 @@ void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& 
   bs.grid = (int)std::max<int64_t>(1, (b.n + BUILD_BLOCK * BUILD_U - 1) / (BUILD_BLOCK * BUILD_U));
   bs.words = d->npayload == 0 ? 1 : (d->npayload == 1 ? 2 : 4);
   bs.counted = d->expected_rows <= 0;
+  if (bs.counted && stats_cache_on()) {
+    // the descriptor's identity: source table uid + everything the statistics depend on
+    std::string& k = bs.stats_key;
+    auto put = [&](const void* p, size_t n) { k.append((const char*)p, n); };
+    put(&t->uid, sizeof(t->uid));
+    put(&b.n, sizeof(b.n));
+    put(&b.npreds, sizeof(b.npreds));
+    put(b.preds, sizeof(KBuildPred) * (size_t)b.npreds);
+    put(&b.key_col, sizeof(b.key_col));
+    put(&b.npay, sizeof(b.npay));
+    put(b.pay_col, sizeof(b.pay_col));
+    put(&b.composite, sizeof(b.composite));
+    auto it = ctx->build_stats.find(k);
+    if (it != ctx->build_stats.end()) {
+      const BuildStats& c = it->second;
+      bs.cached = true;
+      bs.st.cnt = c.cnt;
+      bs.st.kmin = c.kmin; bs.st.kmax = c.kmax; bs.st.pmin = c.pmin; bs.st.pmax = c.pmax;
+      for (int w = 0; w < 8; ++w) bs.st.set[w] = c.set[w];
+      b.verify = 1;
+      b.vs = c;
+      b.vqual = (unsigned long long*)(h->dstate.as<char>() + 40);  // zeroed with dstate
+      b.ticket = (unsigned*)(h->dstate.as<char>() + 32);
+      return;
+    }
+  }
   if (bs.counted) {  // exact count pass: number and range of the qualifying keys
     // (kminmax needs no initial values: the count kernel's last block writes
     // them; an empty table has count 0 and its range is never read)
@@ -429,6 +494,7 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   b.direct = direct;
   b.dmin = (int32_t)kmin;
   b.count_inserts = bs.counted ? 0 : 1;
+  h->stats_key = bs.stats_key;
   if (b.n > 0) { ctx->launches++; hq_build_hash_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b); }
   HQ_CUDA(cudaGetLastError());
   hq_build_compact(ctx, h);
@@ -483,12 +549,25 @@ void hq_build_hashes_impl(hq_ctx* ctx, int n, const hq_build_desc* d, hq_hash* c
       bs[i].host_st = (char*)ctx->pinned_build + (size_t)i * slot;
       if (nside) ctx->stream = ctx->side[i % nside];
       build_prepare(ctx, d + i, h[i], bs[i]);
-      any_count = any_count || bs[i].counted;
+      any_count = any_count || (bs[i].counted && !bs[i].cached);
     }
     join();
-    if (any_count) HQ_CUDA(cudaStreamSynchronize(main));
+    if (any_count) {
+      ctx->stream = main;
+      hq_sync(ctx, "a hash build without cached statistics (its count pass)");
+    }
     for (int i = 0; i < n; ++i)
-      if (bs[i].counted) std::memcpy(&bs[i].st, bs[i].host_st, sizeof(bs[i].st));
+      if (bs[i].counted && !bs[i].cached) {
+        std::memcpy(&bs[i].st, bs[i].host_st, sizeof(bs[i].st));
+        if (!bs[i].stats_key.empty()) {
+          BuildStats c;
+          c.cnt = bs[i].st.cnt;
+          c.kmin = bs[i].st.kmin; c.kmax = bs[i].st.kmax; c.pmin = bs[i].st.pmin; c.pmax = bs[i].st.pmax;
+          for (int w = 0; w < 8; ++w) c.set[w] = bs[i].st.set[w];
+          if (ctx->build_stats.size() > 4096) ctx->build_stats.clear();
+          ctx->build_stats[bs[i].stats_key] = c;
+        }
+      }
     fork();
     for (int i = 0; i < n; ++i) {
       if (nside) ctx->stream = ctx->side[i % nside];
@@ -604,6 +683,7 @@ void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
 // Sync and report build faults (HQ_ERR_DUP_KEY etc.).
 void hq_hash_check(hq_ctx* ctx, hq_hash* h) {
   if (h->checked || !h->dstate.p) return;
+  hq_require_eager(ctx, "a hash build's fault check");
   int st[4];
   HQ_CUDA(cudaMemcpyAsync(st, h->dstate.p, 16, cudaMemcpyDeviceToHost, ctx->stream));
   HQ_CUDA(cudaStreamSynchronize(ctx->stream));
@@ -613,6 +693,11 @@ void hq_hash_check(hq_ctx* ctx, hq_hash* h) {
   if (st[0] & HQF_BAD_KEY) HQ_THROW(HQ_ERR_ARG, "hash build: key INT32_MIN or outside int32");
   if (st[0] & HQF_BAD_PAYLOAD) HQ_THROW(HQ_ERR_ARG, "hash build: payload outside int32");
   if (st[0] & HQF_HT_FULL) HQ_THROW(HQ_ERR_OVERFLOW, "hash build: table full (expected_rows too small)");
+  if (st[0] & HQF_STALE) {
+    ctx->build_stats.erase(h->stats_key);  // the next build of this descriptor counts again
+    HQ_THROW(HQ_ERR_STATE, "hash build: the source table's rows differ from the statistics cached when it was "
+                           "last built (tables are immutable; the statistics were dropped, re-run the query)");
+  }
 }
 
 // ------------------------------------------------------------ column statistics

@@ -248,6 +248,8 @@ struct KSmall {
   long long* res[MAXRC];      // final columns
   unsigned long long* stats;  // [0] rows kept, [1] qualifying, [2] fault bits, [3] rows before LIMIT, [4] pipeline faults
   const int* pipe_err;        // the pipeline's fault word (copied into stats[4])
+  const int* hash_err[8];     // fault words of the probed tables' builds (ORed into stats[4])
+  int nhash;
 };
 __global__ void __launch_bounds__(FIN_THREADS) hq_finalize_small_kernel(const __grid_constant__ KSmall q) {
   __shared__ int idx[SMALL_FIN];
@@ -339,7 +341,9 @@ __global__ void __launch_bounds__(FIN_THREADS) hq_finalize_small_kernel(const __
     q.stats[1] = qual_s;
     q.stats[2] = (unsigned long long)err_s;
     q.stats[3] = (unsigned long long)n;
-    q.stats[4] = (unsigned long long)(unsigned)*q.pipe_err;
+    int e_ = *q.pipe_err;
+    for (int i = 0; i < q.nhash; ++i) e_ |= *(volatile const int*)q.hash_err[i];
+    q.stats[4] = (unsigned long long)(unsigned)e_;
   }
 }
 
@@ -369,10 +373,16 @@ void* pinned_staging(hq_ctx* ctx, size_t bytes) {
   return ctx->pinned;
 }
 
+static bool decode_small(hq_result* r, const char* h, int64_t rcap, int nc);
 namespace {
 // one launch, one sync: fault bits + finalized rows come back together
 bool finalize_small(hq_ctx* ctx, hq_result* r) {
   const hq_plan& P = r->plan;
+  {  // more probed tables than the kernel reads fault words of: the syncing check first
+    int nh = 0;
+    for (hq_hash* hh : r->hashes) nh += (hh->dstate.p && !hh->checked) ? 1 : 0;
+    if (nh > 8) hq_check_result_faults(ctx, r);
+  }
   const int nk = P.nkeys, na = P.naggs, nc = nk + na;
   if (P.norder < 0 || P.norder > HQ_MAX_ORDER) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: 0..4 ORDER BY columns");
   for (int i = 0; i < P.norder; ++i)
@@ -426,14 +436,43 @@ bool finalize_small(hq_ctx* ctx, hq_result* r) {
   q.limit = P.limit;
   q.stats = pack.as<unsigned long long>();
   q.pipe_err = (const int*)(r->dstate.as<char>() + 8);
+  q.nhash = 0;
+  for (hq_hash* hh : r->hashes)
+    if (hh->dstate.p && !hh->checked && q.nhash < 8) q.hash_err[q.nhash++] = hh->dstate.as<int>();
   ctx->launches++;
   hq_finalize_small_kernel<<<1, FIN_THREADS, 0, ctx->stream>>>(q);
   HQ_CUDA(cudaGetLastError());
+  if (ctx->capturing) {
+    // graph capture: the rows land in the result's own pinned staging at every launch
+    // and are decoded on the host after it (hq_graph_launch -> hq_decode_captured)
+    if (r->stage_host) HQ_THROW(HQ_ERR_STATE, "result finalized twice in one capture");
+    HQ_CUDA(cudaHostAlloc(&r->stage_host, 64 + body, cudaHostAllocDefault));
+    HQ_CUDA(cudaMemcpyAsync(r->stage_host, pack.p, 64 + body, cudaMemcpyDeviceToHost, ctx->stream));
+    r->stage_rcap = rcap;
+    r->ncols = nc;
+    r->rescol.assign((size_t)nc, nullptr);
+    for (int c = 0; c < nc; ++c) r->rescol[c] = pack.as<char>() + 64 + (size_t)c * rcap * 8;
+    r->respack = std::move(pack);
+    r->capture_retain(ctx);
+    ctx->cap_results.push_back(r);
+    r->finalized = true;  // for this capture; hq_graph_launch re-opens it
+    return true;
+  }
   char* h = (char*)pinned_staging(ctx, 64 + body);
   HQ_CUDA(cudaMemcpyAsync(h, pack.p, 64 + body, cudaMemcpyDeviceToHost, ctx->stream));
   HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  if (!decode_small(r, h, rcap, nc)) return false;  // faults: the caller checks (and may re-run), then retries
+  r->rescol.assign((size_t)nc, nullptr);
+  for (int c = 0; c < nc; ++c) r->rescol[c] = pack.as<char>() + 64 + (size_t)c * rcap * 8;
+  r->respack = std::move(pack);
+  return true;
+}
+}  // namespace
+
+// finalize_small's host part: stats + rows staged in h (layout of KSmall)
+static bool decode_small(hq_result* r, const char* h, int64_t rcap, int nc) {
   const unsigned long long* sv = (const unsigned long long*)h;
-  if (!r->checked && sv[4]) return false;  // faults: the caller checks (and may re-run), then retries
+  if (!r->checked && sv[4]) return false;
   r->checked = true;
   if (sv[2] & HQF_OVERFLOW) HQ_THROW(HQ_ERR_OVERFLOW, "aggregate exceeds the int64 guard (|v| >= 2^62)");
   const int64_t nf = (int64_t)sv[0];
@@ -443,14 +482,20 @@ bool finalize_small(hq_ctx* ctx, hq_result* r) {
   for (int c = 0; c < nc; ++c)
     std::memcpy(r->host_rows.data() + (size_t)c * nf, h + 64 + (size_t)c * rcap * 8, (size_t)nf * 8);
   r->host_ready = true;
-  r->rescol.assign((size_t)nc, nullptr);
-  for (int c = 0; c < nc; ++c) r->rescol[c] = pack.as<char>() + 64 + (size_t)c * rcap * 8;
-  r->respack = std::move(pack);
   r->nrows = nf;
   r->finalized = true;
   return true;
 }
-}  // namespace
+
+void hq_decode_captured(hq_ctx* ctx, hq_result* r) {
+  if (!r->stage_host) HQ_THROW(HQ_ERR_STATE, "result has no capture staging");
+  if (decode_small(r, (const char*)r->stage_host, r->stage_rcap, r->ncols)) return;
+  // a fault (pipeline, or a probed table's build): raised by the syncing check; the
+  // re-runnable ones cannot occur in a dense small result
+  r->checked = false;
+  hq_check_result_faults(ctx, r);
+  HQ_THROW(HQ_ERR_STATE, "captured query: unexpected re-runnable fault");
+}
 
 // Stable LSD radix sort of the rows by (ORDER BY columns, then the group keys
 // ascending): one CUB radix pass per column, least significant first; returns
@@ -503,6 +548,7 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered) {
     hq_check_result_faults(ctx, r);  // throws, or re-runs the pipeline with more room
     if (finalize_small(ctx, r)) return;
   }
+  hq_require_eager(ctx, "the finalize of a large, hash-grouped or materialised result");
   hq_check_result_faults(ctx, r);
   const hq_plan& P = r->plan;
   if (r->sink == HQ_SINK_MATERIALISE) {

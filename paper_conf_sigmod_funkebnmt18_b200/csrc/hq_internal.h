@@ -8,6 +8,7 @@
 #include <algorithm>
 #include <atomic>
 #include <cstring>
+#include <map>
 #include <string>
 #include <vector>
 
@@ -62,7 +63,18 @@ enum : int {
   HQF_BAD_KEY = 32,     // build key INT32_MIN or outside int32
   HQF_BAD_PAYLOAD = 64, // build payload outside int32
   HQF_HT_FULL = 128,    // join hash table full (cannot happen when sized by the count pass)
-  HQF_OVERFLOW = 256    // int64 guard tripped (|aggregate| >= 2^62)
+  HQF_OVERFLOW = 256,   // int64 guard tripped (|aggregate| >= 2^62)
+  HQF_STALE = 512       // a build's cached statistics do not describe its source rows (hq_build.cu)
+};
+
+// Statistics of a build's qualifying rows (count pass): number, key range, payload-0
+// range and value set (bit v & 255).  Cached per (source table, descriptor) so that a
+// repeated build skips the count pass and its host synchronisation; the insert kernel
+// then re-derives them on the device and flags HQF_STALE on any difference.
+struct BuildStats {
+  unsigned long long cnt;
+  int kmin, kmax, pmin, pmax;
+  unsigned set[8];
 };
 
 // ---------------------------------------------------------------- objects
@@ -90,8 +102,47 @@ struct hq_ctx {
   static constexpr int NSIDE = 4;
   cudaStream_t side[NSIDE] = {};
   cudaEvent_t ev_fork = nullptr, ev_join[NSIDE] = {};
+  // build statistics by (source table uid, descriptor bytes); HQ_BUILD_STATS=0 disables
+  std::map<std::string, BuildStats> build_stats;
+  // CUDA-graph capture of a prepared query (hq_ctx_capture_begin/_end): the work is
+  // captured on cap_stream; allocations come from the pool through alloc_stream (not
+  // captured), frees are deferred to the graph's destruction, objects created or
+  // read by captured work are retained by the graph, and results finalized during the
+  // capture leave their rows in their own pinned staging (decoded after each launch)
+  bool capturing = false;
+  cudaStream_t user_stream = nullptr, cap_stream = nullptr, alloc_stream = nullptr;
+  std::vector<std::pair<void*, size_t>> cap_frees;
+  std::vector<struct RefObj*> cap_objs;
+  std::vector<struct hq_result*> cap_results;
+  int64_t cap_launches0 = 0;
   void* alloc_bytes(size_t bytes);
   void free_bytes(void* p, size_t bytes);
+  // Reference count: every table / hash / result holds the context (CtxPtr), so
+  // hq_ctx_destroy only drops the caller's reference and the context's streams and
+  // staging live until the last object that may still free device memory through it.
+  std::atomic<int> refs{1};
+  void retain() { refs.fetch_add(1); }
+  void release();  // hq_api.cu: the last reference destroys the context
+};
+
+// An owning reference to the context, declared as the FIRST member of the library's
+// objects so that it is destroyed after their device buffers were freed through it.
+struct CtxPtr {
+  hq_ctx* c = nullptr;
+  CtxPtr() = default;
+  CtxPtr(const CtxPtr&) = delete;
+  CtxPtr& operator=(const CtxPtr&) = delete;
+  CtxPtr& operator=(hq_ctx* n) {
+    if (n) n->retain();
+    if (c) c->release();
+    c = n;
+    return *this;
+  }
+  ~CtxPtr() {
+    if (c) c->release();
+  }
+  operator hq_ctx*() const { return c; }
+  hq_ctx* operator->() const { return c; }
 };
 
 // A device allocation owned through the context allocator.
@@ -119,12 +170,20 @@ struct DevBuf {
 
 struct RefObj {
   std::atomic<int> refs{1};
+  // called for objects created or used by work captured into a CUDA graph
+  void capture_retain(hq_ctx* c);
   virtual ~RefObj() {}
   void retain() { refs.fetch_add(1); }
   void release() {
     if (refs.fetch_sub(1) == 1) delete this;
   }
 };
+
+inline void RefObj::capture_retain(hq_ctx* c) {
+  if (!c || !c->capturing) return;
+  retain();
+  c->cap_objs.push_back(this);
+}
 
 struct hq_result;
 
@@ -135,7 +194,12 @@ struct TableCol {
 };
 
 struct hq_table : RefObj {
-  hq_ctx* ctx = nullptr;
+  CtxPtr ctx;
+  uint64_t uid = next_uid();  // never reused (a freed table's address may be)
+  static uint64_t next_uid() {
+    static std::atomic<uint64_t> n{1};
+    return n.fetch_add(1);
+  }
   int64_t nrows = 0;
   int ncols = 0;
   TableCol cols[HQ_MAX_COLS];
@@ -146,13 +210,14 @@ struct hq_table : RefObj {
 };
 
 struct hq_hash : RefObj {
-  hq_ctx* ctx = nullptr;
+  CtxPtr ctx;
   hq_hash_meta meta{};
   int log2cap = 0;
   uint32_t* slots = nullptr;
   DevBuf owned;      // slot array (empty when imported)
   DevBuf dstate;     // [0] fault bits (int), [1..2] nkeys (u64) -- see hq_build.cu
   bool checked = false;
+  std::string stats_key;  // its entry in hq_ctx::build_stats (dropped on HQF_STALE)
   // compact form of a direct table (hq_build.cu): 1 = bitmap of present keys
   // (semi-join), 2 = one byte per key (payload0 - pay_min, 0xFF absent),
   // 3 = one nibble per key (payload0 - pay_min < 15, 0xF absent)
@@ -326,7 +391,7 @@ struct KPlan {
 }  // namespace hqk
 
 struct hq_result : RefObj {
-  hq_ctx* ctx = nullptr;
+  CtxPtr ctx;
   hq_plan plan{};
   hq_table* fact = nullptr;
   std::vector<hq_hash*> hashes;
@@ -359,6 +424,9 @@ struct hq_result : RefObj {
   DevBuf ring;               // its double-buffered device blocks
   std::vector<long long> host_rows;  // small results: the finalized rows already on the host
   bool host_ready = false;           // (column-major, nrows per column)
+  // finalized inside a graph capture: rows + stats land in stage_host at every launch
+  void* stage_host = nullptr;        // pinned (cudaHostAlloc), owned
+  int64_t stage_rcap = 0;
   ~hq_result() override;
 };
 
@@ -393,4 +461,10 @@ void hq_jit_prepare(hq_ctx* ctx, const hqk::KPlan& kp, size_t smem);  // compile
 void hq_jit_launch(hq_ctx* ctx, const hqk::KPlan& kp, int grid, size_t smem);
 std::string hq_jit_source(const hqk::KPlan& kp);
 void hq_check_result_faults(hq_ctx* ctx, hq_result* r);
+// host synchronisation of the context stream; illegal while a graph is captured
+void hq_sync(hq_ctx* ctx, const char* what);
+void hq_require_eager(hq_ctx* ctx, const char* what);  // throws HQ_ERR_STATE while capturing
+// decode a result finalized during a capture from its pinned staging (after a launch)
+void hq_decode_captured(hq_ctx* ctx, hq_result* r);
+void hq_hash_check(hq_ctx* ctx, hq_hash* h);  // hq_build.cu: sync + raise build faults
 int hq_type_width(int type);

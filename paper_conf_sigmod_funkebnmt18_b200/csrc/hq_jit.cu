@@ -629,15 +629,19 @@ std::string generate(const KPlan& kp) {
   }
   // HQ_JIT_WAIT=sleep: the older poll + nanosleep loop (A/B)
   const char* wm = getenv("HQ_JIT_WAIT");
-  const std::string cwait = (wm && std::string(wm) == "sleep") ? "mbar_wait_sleep(&full[s], ph);" : "mbar_wait_suspend(&full[s], ph);";
+  const std::string cwait = (wm && std::string(wm) == "sleep") ? "mbar_wait_sleep(&full[s], ph);" : "mbar_wait_suspend_a(sm0_ + 8u * (u32)s, ph);";
   o << "  int s = 0; u32 ph = 0; long long t0 = (first_tile + blockIdx.x) * (long long)T;\n"
     << "  const int njc = (int)nj;\n"
+    // only a CTA's first and last tile can be ragged (partition boundaries): decided once
+    << "  const long long tl_ = t0 + (nj - 1) * tstep;\n"
+    << "  const int rj0_ = (nj > 0 && (t0 < p.row_begin || t0 + T > p.row_end)) ? 0 : -1;\n"
+    << "  const int rj1_ = (nj > 0 && (tl_ < p.row_begin || tl_ + T > p.row_end)) ? njc - 1 : -1;\n"
     << "  for (int j = 0; j < njc; ++j, t0 += tstep) {\n"
     << (prof ? "    { const long long c_ = clock64(); " + cwait + " pw_ += clock64() - c_; if (__activemask() != 0xffffffffu) ++pdv_; }\n" : "    " + cwait + "\n")
     << "    const char* st = stages + (size_t)s * STAGE_STRIDE;\n"
     << "    const long long tb_ = t0;  // tile start (temporaries t0, t1, ... shadow it below)\n"
     << "    u32 mask = (1u << R) - 1u;\n"
-    << "    if ((j == 0 || j == njc - 1) && (t0 < p.row_begin || t0 + T > p.row_end)) {  // ragged head / tail tile: lanes copy their rows\n"
+    << "    if (j == rj0_ || j == rj1_) {  // ragged head / tail tile: lanes copy their rows\n"
     << "      const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
     << "      const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
     << "      mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r; if (row >= lo && row < hi) mask |= 1u << r; }\n";
@@ -683,7 +687,7 @@ std::string generate(const KPlan& kp) {
         o << ";\n";
       }
       o << "      const u32 b_ = __ballot_sync(HQ_FULL, f_ == 0x9E3779B9u);\n"
-        << "      if (lane == 0) { *(volatile u32*)(smem + " << (MISC_DEP) << "u + 4u * warp) = b_; mbar_arrive(&empty[s]); } }\n";
+        << "      if (lane == 0) { *(volatile u32*)(smem + " << (MISC_DEP) << "u + 4u * warp) = b_; mbar_arrive_a(sm0_ + 80u + 8u * (u32)s); } }\n";
     } else if (fix == "fence") {
       o << "    fence_proxy_async(); __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
     } else {
@@ -986,7 +990,7 @@ std::string generate(const KPlan& kp) {
     o << "    }\n";
   }
   if (kp.early_release) o << "    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
-  else o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
+  else o << "    __syncwarp();\n    if (lane == 0) mbar_arrive_a(sm0_ + 80u + 8u * (u32)s);\n    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
   if (prof) o << "  if (lane == 0) { p.prof[blockIdx.x * 128 + 8 + warp] = pw_; p.prof[blockIdx.x * 128 + 40 + warp] = clock64() - pl0_; } if (pdv_) atomicAdd((unsigned long long*)&p.prof[blockIdx.x * 128 + 72 + warp], (unsigned long long)pdv_);\n";
   // ------------------------------------------------------------- sink (end)
   if (mp) {

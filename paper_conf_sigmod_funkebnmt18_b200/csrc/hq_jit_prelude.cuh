@@ -88,6 +88,23 @@ __device__ __forceinline__ void mbar_wait_suspend(u64* b, u32 parity) {
         : "memory");
   } while (!ok);
 }
+// the same on a 32-bit shared-window address computed once (a generic pointer makes
+// ptxas re-derive the window base from SR_CgaCtaId at every call)
+__device__ __forceinline__ void mbar_wait_suspend_a(u32 a, u32 parity) {
+  u32 ok;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(ok)
+        : "r"(a), "r"(parity), "r"(1000000u)
+        : "memory");
+  } while (!ok);
+}
+__device__ __forceinline__ void mbar_arrive_a(u32 a) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(a) : "memory");
+}
 __device__ __forceinline__ u64 policy_evict_first() {
   u64 pol;
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));

@@ -653,18 +653,19 @@ static void launch_pipeline(hq_ctx* ctx, hq_result* r, int64_t group_cap, int64_
   const int grid = (int)std::max<long long>(1, std::min<long long>(ntiles, ctx->num_sms));
   const size_t smem = (size_t)fused_smem_bytes(kp);
   cudaEvent_t e0 = nullptr, e1 = nullptr;
-  if (ctx->timing) {
+  const bool timing = ctx->timing && !ctx->capturing;
+  if (timing) {
     for (cudaEvent_t* e : {&e0, &e1}) {
       if (!ctx->event_pool.empty()) { *e = ctx->event_pool.back(); ctx->event_pool.pop_back(); }
       else HQ_CUDA(cudaEventCreate(e));
     }
   }
   if (jit) hq_jit_prepare(ctx, kp, smem);  // compile (cached) outside the timed launch
-  if (ctx->timing) HQ_CUDA(cudaEventRecord(e0, ctx->stream));
+  if (timing) HQ_CUDA(cudaEventRecord(e0, ctx->stream));
   if (r->stream_block > 0) launch_streamed(ctx, r, kp, jit, smem);
   else if (jit) hq_jit_launch(ctx, kp, grid, smem);
   else launch_fused(ctx, kp, grid, smem);
-  if (ctx->timing) {
+  if (timing) {
     HQ_CUDA(cudaEventRecord(e1, ctx->stream));
     ctx->events.emplace_back(e0, e1);
   }
@@ -691,8 +692,30 @@ void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r) {
 
 // Sync, read the device fault bits; re-run once with the exact size when an
 // output capacity or group table overflowed (SURVEY.md §5 failure handling).
+// Build faults of the hash tables a result probed (duplicate keys, stale cached
+// statistics, ...): one gather of their fault words and one read; raised through
+// hq_hash_check (which names the fault) when any is set.
+static void check_result_hashes(hq_ctx* ctx, hq_result* r) {
+  std::vector<const int*> hw;
+  for (hq_hash* h : r->hashes)
+    if (h->dstate.p && !h->checked) hw.push_back(h->dstate.as<int>());
+  if (hw.empty()) return;
+  DevBuf out(ctx, 32 * 8);
+  hq_launch_gather_faults(ctx, hw, {}, out.as<long long>());
+  long long w[32];
+  HQ_CUDA(cudaMemcpyAsync(w, out.p, sizeof(w), cudaMemcpyDeviceToHost, ctx->stream));
+  HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+  bool any = false;
+  for (int k = 0; k < 16; ++k) any = any || w[k] != 0;
+  if (!any) return;
+  for (hq_hash* h : r->hashes)
+    if (h->dstate.p) hq_hash_check(ctx, h);
+}
+
 void hq_check_result_faults(hq_ctx* ctx, hq_result* r) {
   if (r->checked) return;
+  hq_require_eager(ctx, "a result's fault check");
+  check_result_hashes(ctx, r);
   for (int attempt = 0;; ++attempt) {
     struct { unsigned long long counter; int err; int pad; } st{};
     HQ_CUDA(cudaMemcpyAsync(&st, r->dstate.p, sizeof(st), cudaMemcpyDeviceToHost, ctx->stream));

@@ -209,6 +209,11 @@ class DistributedEngine(Engine):
             if now != before:
                 print(f"[hq dist trace] rank {self.rank} {where}: {label} fault words {before} -> {now}",
                       file=sys.stderr, flush=True)
+            try:  # the syncing check round 1 ran here (hq_hash_info)
+                h.info()
+            except hq.HQError as e:
+                print(f"[hq dist trace] rank {self.rank} {where}: {label} hq_hash_info raised {e}", file=sys.stderr,
+                      flush=True)
         self._trace.clear()
 
     def _reduce_checked(self, res: hq.Result) -> None:

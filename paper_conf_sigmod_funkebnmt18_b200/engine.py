@@ -258,7 +258,40 @@ class Engine:
         lo, hi = self.tables[table].column_range(col)
         return (0, 1) if lo > hi else (lo, hi - lo + 1)
 
+    def prepare(self, query, **kw) -> "PreparedQuery":
+        """A prepared query: executed once eagerly (kernels compiled, build statistics
+        cached), then recorded into a CUDA graph whose launches re-run all its device work
+        (hq.h "prepared queries").  Raises HQError(HQ_ERR_STATE) for queries that need
+        the host mid-way (materialised intermediates, large results, ...)."""
+        return PreparedQuery(self, query, **kw)
+
     def gather(self, res: Optional[hq.Result], pb: PlanBuilder) -> Optional[hq.Result]:
         """The complete result of a partitioned pipeline whose aggregation feeds a later
         build or pipeline (an intermediate GROUP BY): on one device, the result itself."""
         return res
+
+
+class PreparedQuery:
+    """One query step recorded as a CUDA graph (Engine.prepare).  execute() launches it:
+    the hash builds, compound kernels and finalization all run again on the device;
+    only the host-side planning was done once."""
+
+    def __init__(self, E: Engine, query, **kw):
+        self.E, self.query, self.kw = E, query, kw
+        query.execute(E, **kw)  # eager run: JIT kernels compiled, build statistics cached
+        ctx = E.ctx
+        ctx.capture_begin()
+        try:
+            self.res, self.pb = query.run(E, **kw)
+            self.res.finalize()
+        except BaseException:
+            ctx.capture_abort()
+            raise
+        self.graph = ctx.capture_end()
+
+    def execute(self) -> QueryResult:
+        self.graph.launch()
+        return fetch(self.res, self.pb.result_names)
+
+    def close(self) -> None:
+        self.graph.free()

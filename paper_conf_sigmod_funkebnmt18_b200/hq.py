@@ -121,7 +121,8 @@ EXPORTS = ["hq_ctx_create", "hq_ctx_destroy", "hq_ctx_set_stream", "hq_ctx_sync"
            "hq_hash_device_view", "hq_hash_import", "hq_free_hash", "hq_run_pipeline", "hq_run_pipeline_streamed",
            "hq_finalize",
            "hq_result_info_get", "hq_fetch_result", "hq_result_as_table", "hq_result_partials_view",
-           "hq_result_from_partials", "hq_gather_faults", "hq_raise_faults", "hq_free_result"]
+           "hq_result_from_partials", "hq_gather_faults", "hq_raise_faults", "hq_free_result",
+           "hq_ctx_capture_begin", "hq_ctx_capture_end", "hq_ctx_capture_abort", "hq_graph_launch", "hq_graph_destroy"]
 FAULT_WORDS = 32
 
 
@@ -164,6 +165,8 @@ def lib():
             "hq_result_from_partials": [vp, vp, vp, ctypes.c_size_t],
             "hq_gather_faults": [vp, P(vp), i32, P(vp), i32, vp],
             "hq_raise_faults": [P(i64)],
+            "hq_ctx_capture_begin": [vp], "hq_ctx_capture_end": [vp, P(vp)], "hq_ctx_capture_abort": [vp],
+            "hq_graph_launch": [vp, vp], "hq_graph_destroy": [vp],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -303,6 +306,18 @@ class Context:
         check(lib().hq_hash_import(self.h, ctypes.byref(meta), ctypes.c_void_p(dev_ptr), ctypes.byref(h)))
         return Hash(self, h, keep=[keep])
 
+    # -- prepared queries (CUDA graphs, hq.h "prepared queries")
+    def capture_begin(self) -> None:
+        check(lib().hq_ctx_capture_begin(self.h))
+
+    def capture_end(self) -> "Graph":
+        g = ctypes.c_void_p()
+        check(lib().hq_ctx_capture_end(self.h, ctypes.byref(g)))
+        return Graph(self, g)
+
+    def capture_abort(self) -> None:
+        check(lib().hq_ctx_capture_abort(self.h))
+
     def gather_faults(self, hashes: Sequence["Hash"], results: Sequence["Result"], dev_out: int) -> None:
         """Enqueue the OR of the hashes' build and the results' pipeline fault words into
         FAULT_WORDS int64 at device address dev_out (no host sync; hq_gather_faults)."""
@@ -319,6 +334,28 @@ class Context:
         else:
             check(lib().hq_run_pipeline_streamed(self.h, ctypes.byref(plan), int(block_rows), ctypes.byref(h)))
         return Result(self, h, keep=list(keep))
+
+
+class Graph:
+    """A recorded query step (hq_graph): launch() re-executes every recorded kernel and
+    leaves the results it finalizes readable until the next launch."""
+
+    def __init__(self, ctx: Context, h):
+        self.ctx, self.h = ctx, h
+
+    def launch(self) -> None:
+        check(lib().hq_graph_launch(self.ctx.h, self.h))
+
+    def free(self) -> None:
+        if self.h:
+            lib().hq_graph_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
 
 
 class Table:
@@ -409,6 +446,13 @@ class Hash:
         m = HashMeta()
         check(lib().hq_hash_info(self.ctx.h, self.h, ctypes.byref(m)))
         return m
+
+    def meta(self) -> HashMeta:
+        """The table's metadata as the host knows it after the build call (sizes, key and
+        payload ranges: exact from the count pass or the cached statistics; nkeys = -1 for
+        expected_rows builds), without a sync -- build faults are raised by info() or by
+        the finalize of a result that probed the table."""
+        return self.device_view()[1]
 
     def device_view(self):
         p = ctypes.c_void_p()

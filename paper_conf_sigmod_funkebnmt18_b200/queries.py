@@ -253,7 +253,7 @@ def _tpch_q3(E: Engine, limit: int = 10, **_):
         ro = E.run(po, partitioned=False)
     ho = E.hash_from(ro, ["o_orderkey", "o_orderdate", "o_shippriority"], "o_orderkey",
                      ["o_orderdate", "o_shippriority"])
-    nk = max(int(ho.info().nkeys), 0)
+    nk = max(int(ho.meta().nkeys), 0)
     # pipeline 3: lineitem filter -> probe orders -> group by orderkey
     pl = E.plan("lineitem")
     pl.filter("l_shipdate", ">", 19950315)
@@ -377,7 +377,7 @@ def _tpch_q10(E: Engine, limit: int = 20, **_):
         po.materialise([("o_orderkey", "i32"), ("o_custkey", "i32"), ("c_nationkey", "i32")])
         ro = E.run(po, partitioned=False)
     ho = E.hash_from(ro, ["o_orderkey", "o_custkey", "c_nationkey"], "o_orderkey", ["o_custkey", "c_nationkey"])
-    nk = max(int(ho.info().nkeys), 0)
+    nk = max(int(ho.meta().nkeys), 0)
     pl = E.plan("lineitem")
     pl.filter("l_returnflag", "=", hqgen.code(hqgen.RETURNFLAGS, "R"))
     pl.probe(ho, "l_orderkey", "inner", ["o_custkey", "c_nationkey"])
@@ -423,7 +423,7 @@ def _tpch_q4(E: Engine, **_):
     # the quarter's orders -> build (3.8 % of the orders, payload o_orderpriority)
     ho = E.hash("orders", "o_orderkey", payload=["o_orderpriority"],
                 preds=[("o_orderdate", "between", 19930701, 19931001 - 1)])
-    nk = max(int(ho.info().nkeys), 0)
+    nk = max(int(ho.meta().nkeys), 0)
     # lineitem: late lines probe the quarter's orders; GROUP BY l_orderkey = the EXISTS (one row per order)
     pl = E.plan("lineitem")
     pl.compute("late", [("load", "l_receiptdate"), ("sub", "l_commitdate")])
@@ -451,7 +451,7 @@ def _tpch_q13(E: Engine, **_):
                  group_capacity=max(1024, E.table("orders").nrows // 4), agg_names=["n"])
     ro = E.gather(E.run(po), po)
     hn = E.hash_from(ro, ["o_custkey", "n"], "o_custkey", ["n"])
-    maxn = max(int(hn.info().pay_max), 0)
+    maxn = max(int(hn.meta().pay_max), 0)
     if not E.builds_here:  # the customer table (the outer join's preserved side) is on the root
         return None, _RootOnly(["c_count", "custdist"])
     pc = E.plan("tpch_customer")
@@ -475,7 +475,7 @@ def _tpch_q17(E: Engine, **_):
     p1.probe(hp, "l_partkey", "semi")
     p1.aggregate(keys=[("l_partkey",) + E.key_domain("lineitem", "l_partkey")],
                  aggs=[("sum", "l_quantity"), ("count", None)],
-                 group_capacity=max(1024, int(hp.info().nkeys)), agg_names=["sum_qty", "cnt"])
+                 group_capacity=max(1024, int(hp.meta().nkeys)), agg_names=["sum_qty", "cnt"])
     r1 = E.gather(E.run(p1), p1)
     ha = E.hash_from(r1, ["l_partkey", "sum_qty", "cnt"], "l_partkey", ["sum_qty", "cnt"])
     p2 = E.plan("lineitem")
@@ -517,7 +517,7 @@ def _tpch_q18(E: Engine, limit: int = 100, **_):
                  aggs=[("min", "o_custkey"), ("min", "o_orderdate"), ("min", "o_totalprice"),
                        ("sum", "l_quantity"), ("count", None)],
                  order=[("o_totalprice", True), ("o_orderdate", False)], limit=limit,
-                 group_capacity=max(1024, int(ho.info().nkeys)),
+                 group_capacity=max(1024, int(ho.meta().nkeys)),
                  agg_names=["c_custkey", "o_orderdate", "o_totalprice", "sum_qty", "count"])
     res = E.run(pl)
     pl.result_names = ["o_orderkey"] + pl.result_names[1:]
@@ -607,7 +607,7 @@ def _tpch_q21(E: Engine, variant: int = 0, limit: int = 100, **_):
     pl.probe(ho, "l_orderkey", "semi")                          # o_orderstatus = 'F'
     pl.probe(h2, "l_orderkey", "semi")                          # exists l2
     pl.probe(h3, "l_orderkey", "semi")                          # not exists l3 (variant 1: exists)
-    ms = hs.info()  # the surviving rows' suppliers are the build's keys (same meta on every rank)
+    ms = hs.meta()  # the surviving rows' suppliers are the build's keys (same meta on every rank)
     pl.aggregate(keys=[("l_suppkey", int(ms.key_min), max(int(ms.key_max) - int(ms.key_min) + 1, 1))],
                  aggs=[("count", None)],
                  order=[("numwait", True), ("l_suppkey", False)], limit=limit, agg_names=["numwait"])

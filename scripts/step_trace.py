@@ -38,43 +38,52 @@ def main():
         q.execute(E)
     torch.cuda.synchronize()
     from torch.profiler import ProfilerActivity, profile
-    marks = []
+    marker = torch.zeros(1024, device="cuda")
     with profile(activities=[ProfilerActivity.CPU, ProfilerActivity.CUDA]) as prof:
         for _ in range(a.steps):
             torch.cuda.synchronize()
             with torch.profiler.record_function("hq_step"):
+                marker.mul_(1.5)  # a step-start marker kernel on the GPU timeline
                 q.execute(E)
             torch.cuda.synchronize()
     evs = prof.events()
-    steps = sorted([e for e in evs if e.name == "hq_step"], key=lambda e: e.time_range.start)
-    gpu = sorted([e for e in evs if e.device_type == torch.autograd.DeviceType.CUDA],
+    hsteps = sorted([e for e in evs if e.name == "hq_step" and e.device_type == torch.autograd.DeviceType.CPU],
+                    key=lambda e: e.time_range.start)
+    gpu = sorted([e for e in evs if e.device_type == torch.autograd.DeviceType.CUDA and e.name != "hq_step"],
                  key=lambda e: e.time_range.start)
     syncs = [e for e in evs if e.device_type == torch.autograd.DeviceType.CPU and "Synchronize" in e.name]
+    # GPU ops of step k: from its marker kernel to the next marker (CPU and GPU clocks may differ)
+    mk = [i for i, e in enumerate(gpu) if "elementwise" in e.name.lower()]
     out = []
-    for si, st in enumerate(steps):
+    for si, st in enumerate(hsteps):
+        if si >= len(mk):
+            break
+        lo, hi = mk[si], (mk[si + 1] if si + 1 < len(mk) else len(gpu))
+        ks = gpu[lo + 1:hi]
         t0, t1 = st.time_range.start, st.time_range.end
-        ks = [e for e in gpu if t0 <= e.time_range.start <= t1]
         ss = [e for e in syncs if t0 <= e.time_range.start <= t1]
+        g0 = gpu[lo].time_range.end
         rows = []
         prev = None
         busy = 0.0
         for e in ks:
-            s, d = e.time_range.start - t0, e.time_range.end - e.time_range.start
+            s, d = e.time_range.start - g0, e.time_range.end - e.time_range.start
             gap = (e.time_range.start - prev) if prev is not None else s
             prev = max(prev or 0, e.time_range.end)
             busy += d
             rows.append({"name": e.name[:70], "start_us": s, "dur_us": d, "gap_before_us": gap})
-        rec = {"step": si, "host_us": t1 - t0, "gpu_busy_us": busy, "n_gpu_ops": len(ks),
+        span = (ks[-1].time_range.end - g0) if ks else 0.0
+        rec = {"step": si, "host_us": t1 - t0, "gpu_span_us": span, "gpu_busy_us": busy, "n_gpu_ops": len(ks),
                "syncs": [{"name": x.name, "start_us": x.time_range.start - t0,
                           "dur_us": x.time_range.end - x.time_range.start} for x in ss], "ops": rows}
         out.append(rec)
-        print(f"step {si}: host {rec['host_us']:.1f} us, GPU busy {busy:.1f} us over {len(ks)} ops, "
+        print(f"step {si}: host {rec['host_us']:.1f} us, GPU span {span:.1f} us, busy {busy:.1f} us over {len(ks)} ops, "
               f"{len(ss)} host syncs ({sum(x['dur_us'] for x in rec['syncs']):.1f} us blocked)")
-        if si == len(steps) - 1:
+        if si == len(hsteps) - 1:
             for r in rows:
                 print(f"  +{r['start_us']:9.1f} us  gap {r['gap_before_us']:8.1f}  dur {r['dur_us']:9.1f}  {r['name']}")
             for x in rec["syncs"]:
-                print(f"  sync at +{x['start_us']:.1f} us for {x['dur_us']:.1f} us ({x['name']})")
+                print(f"  host sync at +{x['start_us']:.1f} us (host clock) for {x['dur_us']:.1f} us ({x['name']})")
     if a.json:
         with open(a.json, "w") as f:
             json.dump({"query": a.query, "sf": a.sf, "steps": out}, f, indent=1)

@@ -1,0 +1,87 @@
+"""Build statistics cache: a repeated build of the same descriptor over
+the same table skips the count pass and its host synchronisation, the insert pass
+re-derives the statistics on the device, and a difference (the caller changed a
+borrowed table in place) is raised as HQ_ERR_STATE -- never a silent wrong answer."""
+import numpy as np
+import pytest
+
+import hqgen
+import oracle
+from paper_conf_sigmod_funkebnmt18_b200 import hq
+from paper_conf_sigmod_funkebnmt18_b200.engine import Engine, PlanBuilder
+from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ctx():
+    import torch
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    c = hq.Context(0)
+    yield c
+    c.close()
+
+
+def test_repeated_query_skips_count_pass(ctx):
+    """SSB Q4.1 three times on the same tables: from the second run on, its four builds
+    launch no count kernel (4 fewer launches), and every run equals the oracle."""
+    host = {t: hqgen.generate(t, 0.1) for t in hqgen.SSB_TABLES}
+    q = QUERIES["ssb_q41"]
+    E = Engine(ctx, {t: ctx.load_columns({c: host[t][c] for c in cs}) for t, cs in q.columns.items()})
+    o = oracle.ssb_q41(host["lineorder"], host["date"], host["customer"], host["supplier"], host["part"])
+    cols = ["d_year", "c_nation", "profit", "count"]
+    n = []
+    for _ in range(3):
+        l0 = ctx.launches()
+        assert q.execute(E).rows(cols) == o.rows()
+        n.append(ctx.launches() - l0)
+    assert n[1] == n[2] == n[0] - 4, n
+
+
+def test_changed_borrowed_table_is_detected(ctx):
+    """A dimension table borrowed from torch memory is changed after its first build:
+    the next build of the same descriptor (cached statistics) must not return a wrong
+    answer -- the pipeline's finalize raises HQ_ERR_STATE; the build after that counts
+    afresh and is exact again."""
+    import torch
+    rng = np.random.default_rng(11)
+    nd = 1000
+    dk = torch.arange(1, nd + 1, dtype=torch.int32, device="cuda")
+    dv = torch.tensor(rng.integers(0, 10, nd).astype(np.int32), device="cuda")  # payload 0..9
+    dim = ctx.load_columns({"k": dk, "v": dv})
+    nf = 50_000
+    fk = rng.integers(1, nd + 1, nf).astype(np.int32)
+    fact = ctx.load_columns({"fk": fk})
+
+    def run():
+        h = ctx.build_hash(dim, 0, [1], [hq.make_pred(1, "<", 8)])
+        pb = PlanBuilder(fact)
+        pb.probe(h, "fk", "inner", ["v"])
+        pb.aggregate(keys=[("v", 0, 16)], aggs=[("count", None)], agg_names=["c"])
+        return ctx.run(pb.plan, keep=pb.keep + [h]).fetch()
+
+    def expect():
+        v = dv.cpu().numpy()
+        sel = v[fk - 1]
+        sel = sel[sel < 8]
+        keys, cnt = np.unique(sel, return_counts=True)
+        return [keys.tolist(), cnt.tolist()]
+
+    assert [c.tolist() for c in run()] == expect()        # count pass, statistics cached
+    l0 = ctx.launches()
+    assert [c.tolist() for c in run()] == expect()        # cached: no count kernel
+    dv[5] = 12                                            # payload outside the cached range ...
+    dv[7] = 3 if int(dv[7]) != 3 else 4                   # ... and a changed value
+    torch.cuda.synchronize()
+    with pytest.raises(hq.HQError) as e:
+        run()
+    assert e.value.code == hq.HQ_ERR_STATE
+    assert [c.tolist() for c in run()] == expect()        # the entry was dropped: counted again
+    dv[5] = 1                                             # a row newly qualifying (count differs)
+    torch.cuda.synchronize()
+    with pytest.raises(hq.HQError) as e:
+        run()
+    assert e.value.code == hq.HQ_ERR_STATE
+    assert [c.tolist() for c in run()] == expect()
+    assert ctx.launches() > l0
