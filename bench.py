@@ -234,36 +234,70 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
         if world > 1:
             dist.barrier()
 
+    stream = torch.cuda.current_stream(dev)
+
+    def timed(run_step, k):
+        """k steps between a barrier + sync on both sides; CUDA events on the stream
+        between the steps (per-step times for the median / min)."""
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(k + 1)]
+        barrier()
+        torch.cuda.synchronize()
+        ev[0].record(stream)
+        o = None
+        for i in range(k):
+            o = run_step()
+            ev[i + 1].record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        per = [ev[i].elapsed_time(ev[i + 1]) for i in range(k)]
+        return ev[0].elapsed_time(ev[k]) / k, per, o
+
     for _ in range(warmup):
         out = step(E)
+    # eager steps (the plan built by the host every step), with the fused kernels timed
     ctx.kernel_times()
     ctx.enable_timing(True)
     l0 = ctx.launches()
-    stream = torch.cuda.current_stream(dev)
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
-        barrier()
-        torch.cuda.synchronize()
-        e0.record(stream)
-        for _ in range(steps):
-            out = step(E)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        barrier()
-    ms = e0.elapsed_time(e1) / steps
-    launches = ctx.launches() - l0
+        ms_eager, per_eager, out = timed(lambda: step(E), steps)
+    launches_eager = ctx.launches() - l0
     kt = ctx.kernel_times()
     ctx.enable_timing(False)
     per_step = max(1, len(kt) // steps)
-    fact_kt = kt[per_step - 1::per_step]  # the fact-table pipeline is the last fused launch of a step
+    # the dominant kernel: the longest fused launch of each step (the fact-table pipeline)
+    fact_kt = [max(kt[i:i + per_step]) for i in range(0, per_step * steps, per_step)] if kt else []
     kms = statistics.mean(fact_kt) if fact_kt else float("nan")
+    # prepared query (CUDA graph of the whole step: builds + fused pipeline + finalize
+    # re-executed every launch; include/hq.h "prepared queries") where the plan is static
+    prep = None
+    if world == 1 and os.environ.get("HQ_BENCH_EAGER") != "1" and os.environ.get("HQ_FORCE_DIST") != "1":
+        try:
+            pq = E.prepare(q)
+            for _ in range(warmup):
+                pq.execute()
+            l1 = ctx.launches()
+            with ClockSampler(local) as clk2:
+                ms_prep, per_prep, out_p = timed(pq.execute, steps)
+            if out_p.rows() != out.rows():
+                raise RuntimeError("prepared result differs from the eager one")
+            prep = {"ms": ms_prep, "per": per_prep, "launches": ctx.launches() - l1, "clocks": clk2.summary()}
+            pq.close()
+        except Exception as e:  # noqa: BLE001 -- a query the graph cannot hold runs eagerly
+            prep = {"error": str(e)[:200]}
+    ms, per, launches, clocks = ms_eager, per_eager, launches_eager, clk.summary()
+    mode = "eager"
+    if prep and "ms" in prep:
+        ms, per, launches, clocks, mode = prep["ms"], prep["per"], prep["launches"], prep["clocks"], "prepared"
     if world > 1:
         t = torch.tensor([ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
 
-    res = {"ms": ms, "kernel_ms": kms, "launches": launches, "clocks": clk.summary(), "rows": n,
-           "local_rows": b - a, "result": out}
+    res = {"ms": ms, "kernel_ms": kms, "launches": launches, "clocks": clocks, "rows": n,
+           "local_rows": b - a, "result": out, "mode": mode, "step_ms_median": statistics.median(per),
+           "step_ms_min": min(per), "eager": {"ms_per_step": ms_eager, "median": statistics.median(per_eager),
+                                               "min": min(per_eager), "launches": launches_eager},
+           "prepared": prep}
     # ---- e2e: host (pinned) buffers through the public API, H2D inside the timed region.
     # Dimension tables are copied (HQ_HOST_COPY); the fact table streams from its pinned
     # host buffers through the fused kernel in blocks (HQ_HOST_STREAM, batch processing:
@@ -306,6 +340,30 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
     ctx.close()
     torch.cuda.empty_cache()
     return res
+
+
+def bytes_ratio(qname, sf):
+    """Fused vs multi-pass vs operator-at-a-time DRAM bytes of this query, as measured by
+    scripts/bytes_ratio.py under ncu at the bench's scale factor (profiles/r02), with the
+    paper's GTX 970 figures beside it."""
+    for rel in ("profiles/r02/bytes_ratio_bench_sfs.json", "profiles/r01/bytes_ratio_sf10.json"):
+        p = os.path.join(ROOT, rel)
+        if not os.path.exists(p):
+            continue
+        br = json.load(open(p))["queries"].get(qname)
+        if not br:
+            continue
+        f, o = br["fused"]["pipeline"]["dram_bytes"], br["oaat"]["pipeline"]["dram_bytes"]
+        ft, ot = br["fused"]["pipeline"]["time_s"], br["oaat"]["pipeline"]["time_s"]
+        out = {"ratio": o / f, "fused_bytes": f, "oaat_bytes": o, "kernel_time_ratio": ot / max(ft, 1e-12),
+               "sf": br.get("sf", 10), "bench_sf": sf, "source": rel + " (scripts/bytes_ratio.py: ncu, --cache-control all)",
+               "paper": "up to 7.5x memory volume and 9.5x kernel time, fused vs operator-at-a-time, GTX 970 "
+                        "(PAPER.md P:40-42)"}
+        if "multipass" in br:
+            m = br["multipass"]["pipeline"]["dram_bytes"]
+            out.update({"multipass_bytes": m, "multipass_ratio": m / f})
+        return out
+    return None
 
 
 def roofline(q, local_rows, kernel_ms, peak, peak_src):
@@ -375,13 +433,16 @@ def run_hq(args):
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "rows/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": r["ms"], "higher_is_better": True,
-                "scaling": "strong" if world > 1 else "strong", "vs_baseline": None, "dtype": "int64",
+                "scaling": "strong", "vs_baseline": None, "dtype": "int64",
                 "data": "synthetic (hqgen TPC-H/SSB-shaped generator, seed %d)" % args.seed,
                 "config": {"workload": f"{args.query}_sf{args.sf:g}", "query": args.query, "sf": args.sf,
                            "fact_rows": r["rows"], "fact_bytes": r["rows"] * q.fact_bytes_per_row(),
                            "l2": "inputs larger than L2 (no flush needed)",
                            "parallelism": f"fact range partition dp{world}, dimension HTs broadcast, 1 reduce",
-                           "step": "hash builds + fused pipeline + reduce + finalize/fetch"},
+                           "step": "hash builds + fused pipeline + reduce + finalize/fetch",
+                           "step_mode": r["mode"] + (" (CUDA graph of the whole step; every kernel re-executed per step)"
+                                                     if r["mode"] == "prepared" else "")},
+                "step_ms_median": r["step_ms_median"], "step_ms_min": r["step_ms_min"], "eager": r["eager"],
                 "roofline": roofline(q, r["local_rows"], r["kernel_ms"], peak, peak_src),
                 "e2e": r.get("e2e"), "gpu_launches": r["launches"], "clocks": r["clocks"]}
         line["roofline"]["kernel_share_of_step"] = r["kernel_ms"] / r["ms"]
@@ -389,16 +450,7 @@ def run_hq(args):
             line["cpu_baseline"] = cpu_baseline(args.query, r["host"], r["rows"])
             line["oaat"] = exec_timing(args.query, r["host"], local, r["ms"], "oaat")
             line["multipass"] = exec_timing(args.query, r["host"], local, r["ms"], "multipass")
-        bp = os.path.join(ROOT, "profiles", "r01", "bytes_ratio_sf10.json")
-        if os.path.exists(bp):
-            br = json.load(open(bp))["queries"].get(args.query)
-            if br:
-                f, o = br["fused"]["pipeline"]["dram_bytes"], br["oaat"]["pipeline"]["dram_bytes"]
-                line["dram_bytes_fused_vs_oaat"] = {"ratio": o / f, "fused_bytes": f, "oaat_bytes": o, "sf": 10,
-                                                    "source": "profiles/r01/bytes_ratio_sf10.json (ncu, --cache-control all)"}
-                if "multipass" in br:
-                    m = br["multipass"]["pipeline"]["dram_bytes"]
-                    line["dram_bytes_fused_vs_oaat"].update({"multipass_bytes": m, "multipass_ratio": m / f})
+        line["dram_bytes_fused_vs_oaat"] = bytes_ratio(args.query, args.sf)
     del r
     if world == 1 and not args.no_extra and args.query == DEFAULT_QUERY:
         per = []
@@ -407,8 +459,12 @@ def run_hq(args):
                 x = measure(qn, sf, args.steps, args.warmup, args.seed, 0, 1, local, with_e2e=False)
                 qq = QUERIES[qn]
                 per.append({"query": qn, "sf": sf, "fact_rows": x["rows"], "value": x["rows"] / (x["ms"] / 1e3),
-                            "unit": "rows/s", "ms_per_step": x["ms"],
-                            "roofline": roofline(qq, x["local_rows"], x["kernel_ms"], peak, peak_src)})
+                            "unit": "rows/s", "ms_per_step": x["ms"], "step_mode": x["mode"],
+                            "step_ms_median": x["step_ms_median"], "step_ms_min": x["step_ms_min"],
+                            "eager_ms_per_step": x["eager"]["ms_per_step"],
+                            "step_over_kernel": x["ms"] / x["kernel_ms"],
+                            "roofline": roofline(qq, x["local_rows"], x["kernel_ms"], peak, peak_src),
+                            "dram_bytes_fused_vs_oaat": bytes_ratio(qn, sf)})
                 del x
             except Exception as e:  # noqa: BLE001
                 per.append({"query": qn, "sf": sf, "error": str(e)[:200]})

@@ -420,7 +420,7 @@ hq_status hq_free_result(hq_result* r);
  * A query whose steps need no host synchronisation -- its hash builds have cached
  * statistics (a previous build of the same descriptor over the same table, see
  * hq_build_hash), its pipelines are fused, its results are dense aggregates of at most
- * 4,096 groups -- can be recorded once and replayed: between hq_ctx_capture_begin and
+ * 8,192 groups -- can be recorded once and replayed: between hq_ctx_capture_begin and
  * hq_ctx_capture_end the calls the caller makes (hq_build_hash(es), hq_run_pipeline,
  * hq_finalize) are enqueued into a CUDA graph instead of executed.  Every launch
  * re-executes ALL the recorded device work -- builds (slot fill, insert, compact,

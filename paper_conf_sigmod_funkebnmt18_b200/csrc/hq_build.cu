@@ -603,16 +603,25 @@ __global__ void hq_prefilter_kernel(const uint32_t* slots, long long cap, int wo
     if (d >= 0 && d < range) atomicOr(bm + (d >> 5), 1u << (d & 31));
   }
 }
-// one byte per key: payload0 - pay_min, 0xFF = absent (8-B slots {key, payload});
-// thread per key, coalesced 8-B slot reads and byte writes
-__global__ void hq_compact_u8_kernel(const uint32_t* slots, long long range, int pay_min, uint32_t* out) {
+// one byte per key: payload0 - pay_min, or its rank in the payload set when a LUT is
+// given (sparse value sets: the generated kernel then indexes a ranked group key with
+// the byte itself); 0xFF = absent (8-B slots {key, payload}); thread per key,
+// coalesced 8-B slot reads and byte writes
+struct RankLut {
+  unsigned char r[256];
+};
+__global__ void hq_compact_u8_kernel(const uint32_t* slots, long long range, int pay_min, uint32_t* out, int use_lut,
+                                     const __grid_constant__ RankLut lut) {
   unsigned char* o = (unsigned char*)out;
   const long long n = (range + 3) / 4 * 4;  // whole words (the tail bytes read as absent)
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
     uint32_t byte = 0xFFu;
     if (i < range) {
       const uint2 s = ((const uint2*)slots)[i];
-      if ((int)s.x != INT_MIN) byte = (uint32_t)((int)s.y - pay_min) & 0xFFu;
+      if ((int)s.x != INT_MIN) {
+        byte = (uint32_t)((int)s.y - pay_min) & 0xFFu;
+        if (use_lut) byte = lut.r[byte];
+      }
     }
     o[i] = (unsigned char)byte;
   }
@@ -641,6 +650,7 @@ __global__ void hq_compact_u4_kernel(const uint32_t* slots, long long range, int
 // small payload.  Also run on import (multi-GPU) from the broadcast slots.
 void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
   h->ckind = 0;
+  h->crank = 0;
   h->cbytes = 0;
   h->pf_words = 0;
   if (h->meta.layout == HQ_HT_LINEAR) {
@@ -673,7 +683,19 @@ void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
   const int grid = (int)std::max<long long>(1, std::min<long long>((range + 255) / 256, (long long)ctx->num_sms * 8));
   ctx->launches++;
   if (kind == 1) hq_compact_bitmap_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->compact.as<uint32_t>());
-  else if (kind == 2) hq_compact_u8_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>());
+  else if (kind == 2) {
+    // a sparse payload-value set (SSB Q3.1's five ASIA nations among codes 8..24): rank-code
+    RankLut lut{};
+    int n = 0, span = h->meta.pay_max - h->meta.pay_min + 1;
+    for (int d = 0; d < span; ++d) {
+      const uint32_t v = (uint32_t)(h->meta.pay_min + d) & 255u;
+      lut.r[d] = (unsigned char)0xFF;
+      if ((h->meta.pay_set[v >> 6] >> (v & 63)) & 1ull) lut.r[d] = (unsigned char)n++;
+    }
+    h->crank = (n > 0 && n < span && span <= 255 && !getenv("HQ_NO_RANKMAP")) ? 1 : 0;
+    hq_compact_u8_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>(),
+                                                        h->crank, lut);
+  }
   else hq_compact_u4_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>());
   HQ_CUDA(cudaGetLastError());
   h->ckind = kind;

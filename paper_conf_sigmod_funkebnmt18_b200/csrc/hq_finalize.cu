@@ -236,10 +236,182 @@ __global__ void hq_gather_kernel(const long long* src, const int* idx, long long
     dst[i] = src[idx[i]];
 }
 
+// ---- top-k of a large group table (ORDER BY ... LIMIT k, k <= TOPK_MAX): the table
+// is read once, no compaction.  Pass 1: every block sorts a chunk of table entries
+// (live ones only) under the result order and keeps its first k entry indices, and
+// sums the groups' counts; pass 2 (one block): sorts the blocks' candidates, keeps k,
+// decodes those k rows and stages rows + statistics for ONE host copy.
+constexpr int TOPK_MAX = 256;
+struct KTopK {
+  KCompact k;       // the group table and its decoding (k.out unused)
+  KSort s;          // s.norder / ocol / odesc / nkeys (s.col unused)
+  int keep;         // rows kept per chunk (= limit)
+  int* cand;        // pass 1 output: gridDim x keep entry indices (-1 = none)
+  unsigned long long* stats;  // [0] rows kept, [1] qualifying, [2] fault bits, [3] live groups, [4] pipeline faults
+  long long* res[MAXRC];      // final columns (keep rows each)
+  const int* pipe_err;
+  const int* hash_err[8];
+  int nhash;
+};
+__device__ __forceinline__ const long long* tk_entry(const KCompact& k, long long g) {
+  return k.gtab + g * (k.vwords + (k.hash ? 1 : 0)) + (k.hash ? 1 : 0);
+}
+__device__ __forceinline__ bool tk_live(const KCompact& k, long long g) {
+  const long long* e = k.gtab + g * (k.vwords + (k.hash ? 1 : 0));
+  if (k.hash && (unsigned long long)e[0] == EMPTY_KEY) return false;
+  return (k.hash ? e[1] : e[0]) != 0;
+}
+// result column c of the group at table entry g (keys decoded, AVG as fp64 bits)
+__device__ __forceinline__ long long tk_col(const KCompact& k, long long g, int c) {
+  const long long* e = tk_entry(k, g);
+  if (c < k.nkeys) {
+    const unsigned long long key = k.hash ? (unsigned long long)e[-1] : (unsigned long long)g;
+    return k.key_min[c] + (long long)((key / (unsigned long long)k.key_stride[c]) % (unsigned long long)k.key_card[c]);
+  }
+  const int a = c - k.nkeys;
+  const long long v = e[1 + a];
+  if (k.agg_fn[a] == HQ_AGG_AVG) {
+    const long long cnt = e[0];
+    const double d = cnt ? (double)v / (double)cnt / k.agg_div[a] : __longlong_as_double(0x7ff8000000000000LL);
+    return __double_as_longlong(d);
+  }
+  return v;
+}
+__device__ __forceinline__ int tk_cmp(const KCompact& k, const KSort& s, int c, long long a, long long b) {
+  const long long x = tk_col(k, a, c), y = tk_col(k, b, c);
+  if (s.isf[c]) {
+    const double dx = __longlong_as_double(x), dy = __longlong_as_double(y);
+    return dx < dy ? -1 : (dx > dy ? 1 : 0);
+  }
+  return x < y ? -1 : (x > y ? 1 : 0);
+}
+// the total order of hq_finalize (ORDER BY, then group keys, then entry index)
+__device__ __forceinline__ bool tk_less(const KCompact& k, const KSort& s, long long a, long long b) {
+  if (a < 0) return false;
+  if (b < 0) return true;
+  for (int i = 0; i < s.norder; ++i) {
+    int c = tk_cmp(k, s, s.ocol[i], a, b);
+    if (s.odesc[i]) c = -c;
+    if (c) return c < 0;
+  }
+  for (int i = 0; i < s.nkeys; ++i) {
+    const int c = tk_cmp(k, s, i, a, b);
+    if (c) return c < 0;
+  }
+  return a < b;
+}
+// bitonic sort of idx[0..net) (entry indices, -1 sorts last) under tk_less; the first
+// ORDER BY column travels as an order-preserving key so most comparisons stay in smem
+__device__ void tk_sort(const KCompact& k, const KSort& s, long long* idx, unsigned long long* pk, int net) {
+  const int c0 = s.norder > 0 ? s.ocol[0] : 0;
+  const bool d0 = s.norder > 0 && s.odesc[0];
+  for (int i = threadIdx.x; i < net; i += blockDim.x) {
+    unsigned long long t = ~0ull;
+    if (idx[i] >= 0) {
+      const long long v = tk_col(k, idx[i], c0);
+      t = s.isf[c0] ? (v < 0 ? ~(unsigned long long)v : (unsigned long long)v ^ 0x8000000000000000ull)
+                    : (unsigned long long)v ^ 0x8000000000000000ull;
+      if (d0) t = ~t;
+      if (s.norder == 0 && s.nkeys == 0) t = 0;
+    }
+    pk[i] = t;
+  }
+  __syncthreads();
+  for (int kk = 2; kk <= net; kk <<= 1) {
+    for (int j = kk >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < net; i += blockDim.x) {
+        const int l = i ^ j;
+        if (l > i) {
+          const long long a = idx[i], b = idx[l];
+          const unsigned long long ka = pk[i], kb = pk[l];
+          const bool up = (i & kk) == 0;
+          const bool b_lt_a = kb != ka ? kb < ka : tk_less(k, s, b, a);
+          const bool a_lt_b = kb != ka ? ka < kb : tk_less(k, s, a, b);
+          if (up ? b_lt_a : a_lt_b) { idx[i] = b; idx[l] = a; pk[i] = kb; pk[l] = ka; }
+        }
+      }
+      __syncthreads();
+    }
+  }
+}
+__global__ void __launch_bounds__(1024) hq_topk1_kernel(const __grid_constant__ KTopK q) {
+  __shared__ long long idx[SORT_CHUNK];
+  __shared__ unsigned long long pk[SORT_CHUNK];
+  __shared__ unsigned long long qual_s, live_s;
+  const KCompact& k = q.k;
+  if (threadIdx.x == 0) { qual_s = 0; live_s = 0; }
+  // chunk of SORT_CHUNK - keep entries; the block's running top-k occupies idx[0..keep)
+  const long long chunk = SORT_CHUNK - q.keep;
+  const long long per = (k.ngroups + gridDim.x - 1) / gridDim.x;
+  const long long g0 = (long long)blockIdx.x * per, g1 = g0 + per < k.ngroups ? g0 + per : k.ngroups;
+  for (int i = threadIdx.x; i < q.keep; i += blockDim.x) idx[i] = -1;
+  unsigned long long qsum = 0, lsum = 0;
+  for (long long c0 = g0; c0 < g1; c0 += chunk) {
+    __syncthreads();
+    for (int i = threadIdx.x; i < (int)chunk; i += blockDim.x) {
+      const long long g = c0 + i;
+      const bool live = g < g1 && tk_live(k, g);
+      if (live) {
+        qsum += (unsigned long long)tk_entry(k, g)[0];
+        ++lsum;
+      }
+      idx[q.keep + i] = live ? g : -1;
+    }
+    __syncthreads();
+    tk_sort(k, q.s, idx, pk, SORT_CHUNK);
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < q.keep; i += blockDim.x) q.cand[(long long)blockIdx.x * q.keep + i] = (int)idx[i];
+  if (qsum) atomicAdd(&qual_s, qsum);
+  if (lsum) atomicAdd(&live_s, lsum);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    if (qual_s) atomicAdd(q.stats + 1, qual_s);
+    if (live_s) atomicAdd(q.stats + 3, live_s);
+  }
+}
+__global__ void __launch_bounds__(1024) hq_topk2_kernel(const __grid_constant__ KTopK q, int ncand) {
+  __shared__ long long idx[SORT_CHUNK];
+  __shared__ unsigned long long pk[SORT_CHUNK];
+  __shared__ int err_s;
+  const KCompact& k = q.k;
+  if (threadIdx.x == 0) err_s = 0;
+  // candidates in rounds of SORT_CHUNK - keep, the running top-k in idx[0..keep)
+  const int chunk = SORT_CHUNK - q.keep;
+  for (int i = threadIdx.x; i < q.keep; i += blockDim.x) idx[i] = -1;
+  for (int c0 = 0; c0 < ncand; c0 += chunk) {
+    __syncthreads();
+    for (int i = threadIdx.x; i < chunk; i += blockDim.x) idx[q.keep + i] = c0 + i < ncand ? q.cand[c0 + i] : -1;
+    __syncthreads();
+    tk_sort(k, q.s, idx, pk, SORT_CHUNK);
+  }
+  __syncthreads();
+  const int nc = k.nkeys + k.naggs;
+  for (int i = threadIdx.x; i < q.keep; i += blockDim.x) {
+    const long long g = idx[i];
+    if (g < 0) continue;
+    for (int c = 0; c < nc; ++c) q.res[c][i] = tk_col(k, g, c);
+    for (int a = 0; a < k.naggs; ++a) {
+      const long long v = tk_entry(k, g)[1 + a];
+      if ((k.agg_fn[a] == HQ_AGG_SUM || k.agg_fn[a] == HQ_AGG_AVG) && (v >= (1LL << 62) || v <= -(1LL << 62)))
+        atomicOr(&err_s, HQF_OVERFLOW);
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned long long live = q.stats[3];
+    q.stats[0] = live < (unsigned long long)q.keep ? live : (unsigned long long)q.keep;
+    q.stats[2] = (unsigned long long)err_s;
+    int e_ = *q.pipe_err;
+    for (int i = 0; i < q.nhash; ++i) e_ |= *(volatile const int*)q.hash_err[i];
+    q.stats[4] = (unsigned long long)(unsigned)e_;
+  }
+}
+
 // ---- small dense results (SSB/TPC-H aggregates: <= 4,375 groups): compaction,
 // AVG, ORDER BY and LIMIT in ONE block, rows staged to the host with the fault
 // bits in the same copy -- one launch and one host sync per finalize.
-constexpr int SMALL_FIN = 4096;
+constexpr int SMALL_FIN = 8192;  // (SSB Q3.1 declares 4,375 groups)
 constexpr int FIN_THREADS = 1024;
 struct KSmall {
   KCompact k;                 // k.out: row-major-by-column scratch, capacity ngroups
@@ -497,6 +669,73 @@ void hq_decode_captured(hq_ctx* ctx, hq_result* r) {
   HQ_THROW(HQ_ERR_STATE, "captured query: unexpected re-runnable fault");
 }
 
+// ORDER BY ... LIMIT k (k <= TOPK_MAX) of a large group table: two launches, one host
+// copy (rows + statistics), no compaction of the whole table (hq_topk1/2_kernel).
+static bool finalize_topk(hq_ctx* ctx, hq_result* r) {
+  const hq_plan& P = r->plan;
+  const int nk = P.nkeys, na = P.naggs, nc = nk + na;
+  if (P.norder < 0 || P.norder > HQ_MAX_ORDER) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: 0..4 ORDER BY columns");
+  for (int i = 0; i < P.norder; ++i)
+    if (P.order_col[i] < 0 || P.order_col[i] >= nc) HQ_THROW(HQ_ERR_ARG, "plan: ORDER BY column out of range");
+  KTopK q{};
+  KCompact& k = q.k;
+  k.gtab = r->gtab.as<long long>();
+  k.ngroups = r->ngroups;
+  k.vwords = r->vwords;
+  k.hash = r->gmode == GM_HASH;
+  k.nkeys = nk;
+  k.naggs = na;
+  int64_t st = 1;
+  for (int i = nk - 1; i >= 0; --i) {
+    k.key_stride[i] = st;
+    st *= P.key_card[i];
+  }
+  for (int i = 0; i < nk; ++i) {
+    k.key_min[i] = P.key_min[i];
+    k.key_card[i] = P.key_card[i];
+    r->types[i] = HQ_I64;
+  }
+  for (int a = 0; a < na; ++a) {
+    k.agg_fn[a] = (uint8_t)P.agg_fn[a];
+    double d = 1.0;
+    for (int s2 = 0; s2 < P.agg_scale[a]; ++s2) d *= 10.0;
+    k.agg_div[a] = d;
+    r->types[nk + a] = P.agg_fn[a] == HQ_AGG_AVG ? HQ_F64 : HQ_I64;
+  }
+  for (int c = 0; c < nc; ++c) q.s.isf[c] = r->types[c] == HQ_F64;
+  q.s.norder = P.norder;
+  for (int i = 0; i < P.norder; ++i) {
+    q.s.ocol[i] = P.order_col[i];
+    q.s.odesc[i] = P.order_desc[i];
+  }
+  q.s.nkeys = nk;
+  q.keep = (int)P.limit;
+  const int64_t rcap = (P.limit + 1) / 2 * 2;
+  const size_t body = (size_t)nc * rcap * 8;
+  DevBuf pack(ctx, 64 + body);
+  HQ_CUDA(cudaMemsetAsync(pack.p, 0, 64, ctx->stream));
+  q.stats = pack.as<unsigned long long>();
+  for (int c = 0; c < nc; ++c) q.res[c] = (long long*)(pack.as<char>() + 64 + (size_t)c * rcap * 8);
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)ctx->num_sms * 2, (r->ngroups + 4095) / 4096));
+  DevBuf cand(ctx, (size_t)grid * q.keep * 4 + 16);
+  q.cand = cand.as<int>();
+  q.pipe_err = (const int*)(r->dstate.as<char>() + 8);
+  for (hq_hash* hh : r->hashes)
+    if (hh->dstate.p && !hh->checked && q.nhash < 8) q.hash_err[q.nhash++] = hh->dstate.as<int>();
+  ctx->launches += 2;
+  hq_topk1_kernel<<<grid, 1024, 0, ctx->stream>>>(q);
+  hq_topk2_kernel<<<1, 1024, 0, ctx->stream>>>(q, grid * q.keep);
+  HQ_CUDA(cudaGetLastError());
+  char* h = (char*)pinned_staging(ctx, 64 + body);
+  HQ_CUDA(cudaMemcpyAsync(h, pack.p, 64 + body, cudaMemcpyDeviceToHost, ctx->stream));
+  hq_sync(ctx, "a top-k finalize");
+  if (!decode_small(r, h, rcap, nc)) return false;
+  r->rescol.assign((size_t)nc, nullptr);
+  for (int c = 0; c < nc; ++c) r->rescol[c] = pack.as<char>() + 64 + (size_t)c * rcap * 8;
+  r->respack = std::move(pack);
+  return true;
+}
+
 // Stable LSD radix sort of the rows by (ORDER BY columns, then the group keys
 // ascending): one CUB radix pass per column, least significant first; returns
 // the sorted row order in `idx` (n entries).
@@ -549,6 +788,12 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered) {
     if (finalize_small(ctx, r)) return;
   }
   hq_require_eager(ctx, "the finalize of a large, hash-grouped or materialised result");
+  if (r->sink == HQ_SINK_AGG && r->plan.limit > 0 && r->plan.limit <= TOPK_MAX && r->plan.nkeys > 0 &&
+      !getenv("HQ_NO_TOPK")) {
+    if (finalize_topk(ctx, r)) return;
+    hq_check_result_faults(ctx, r);  // throws, or re-runs the pipeline with a larger group table
+    if (finalize_topk(ctx, r)) return;
+  }
   hq_check_result_faults(ctx, r);
   const hq_plan& P = r->plan;
   if (r->sink == HQ_SINK_MATERIALISE) {

@@ -223,6 +223,7 @@ struct hq_hash : RefObj {
   // 3 = one nibble per key (payload0 - pay_min < 15, 0xF absent)
   DevBuf compact;
   int ckind = 0;
+  int crank = 0;  // ckind 2 holds the rank of payload 0 in meta.pay_set instead of payload - pay_min
   int64_t cbytes = 0;
   // linear tables: exact bitmap over [key_min, key_max] (prefilter before the slots)
   DevBuf prefilter;
@@ -301,6 +302,7 @@ struct KProbe {
   uint32_t pf_range;
   uint8_t composite;   // two-column key: slot word 1 must equal key2_reg; payloads from word 2
   int16_t key2_reg;
+  uint8_t crank;       // ckind 2: the byte is the payload's RANK in pay_set (sparse value sets)
 };
 struct KCompute {
   int16_t dst;
@@ -348,6 +350,10 @@ struct KPlan {
   int16_t agg_reg[HQ_MAX_AGGS];
   uint8_t gmode, smode;
   uint32_t vwords;           // 1 + naggs: [count, agg...] per group
+  // generated kernels' shared pre-aggregation entries: [count, non-COUNT aggs...]
+  // (COUNT aggregates read the count word); lcol[a] = the aggregate's word
+  uint32_t lvwords;
+  uint8_t lcol[HQ_MAX_AGGS];
   long long* gtab;           // global dense table or hash entries [key, count, agg...]
   uint64_t gmask;            // hash capacity - 1
   int32_t glog2;

@@ -116,8 +116,15 @@ struct Gen {
   // value of register `reg` for row slot r, as a C++ expression
   std::string val(int reg) {
     use(reg);
+    auto rk = rank_of.find(reg);
+    // rank -> value (a dead row's register may hold anything: the index is masked to the table)
+    if (rk != rank_of.end()) return "RV_" + std::to_string(rk->second) + "[(u32)" + var(reg) + "[r] & 255u]";
     return var(reg) + "[r]";
   }
+  // payload registers holding the payload's rank in its build's value set (rank-coded
+  // byte maps, hq_build_compact): register -> probe index (RV_<i> maps rank -> value)
+  std::map<int, int> rank_of;
+  std::set<int> rank_probe;  // rank-coded probes whose payload is decoded to its value at the probe
   void use(int reg) {
     if (dead.count(reg)) HQ_THROW(HQ_ERR_STATE, "jit: register used after compaction but not carried over");
     if (loaded.count(reg)) return;
@@ -148,9 +155,35 @@ struct Gen {
   // could stay split for the rest of the kernel and run at half speed
   int open = 0;
   void early_exit() {
+    sync_mask();  // mask must be right on the path that skips the block
     o << "      if (__any_sync(HQ_FULL, mask)) {\n";
     ++open;
   }
+  // Row liveness inside the operator section: one bool per row slot (al_[r], kept in
+  // predicate registers) for filters and direct probes, and the R-bit `mask` the sinks,
+  // votes and linear probes use; whichever was written last is synced on demand.
+  enum { LIVE_BOTH = 0, LIVE_AL = 1, LIVE_MASK = 2 };
+  int live = LIVE_MASK;
+  bool al_declared = false;
+  void begin_al() {
+    if (!al_declared) {
+      o << "      bool al_[R];\n";
+      al_declared = true;
+      live = LIVE_MASK;
+    }
+    sync_al();
+  }
+  void sync_al() {
+    if (live != LIVE_MASK) return;
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) al_[r] = (mask >> r) & 1u;\n";
+    live = LIVE_BOTH;
+  }
+  void sync_mask() {
+    if (live != LIVE_AL) return;
+    o << "      mask = 0u;\n#pragma unroll\n      for (int r = 0; r < R; ++r) mask |= (u32)al_[r] << r;\n";
+    live = LIVE_BOTH;
+  }
+  void mask_written() { live = LIVE_MASK; }
 
   void filter(const KPred& f, int idx) {
     std::string cond;
@@ -181,7 +214,9 @@ struct Gen {
       bitmaps << "static constexpr __device__ u64 " << bm << "[4] = {" << f.bm[0] << "ull, " << f.bm[1] << "ull, "
               << f.bm[2] << "ull, " << f.bm[3] << "ull};\n";
     }
-    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (!(" << cond << ")) mask &= ~(1u << r);\n";
+    sync_al();
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) al_[r] = al_[r] && (" << cond << ");\n";
+    live = LIVE_AL;
   }
 
   // ---- probes.  A direct-mapped probe is three steps: address (key - min,
@@ -197,9 +232,22 @@ struct Gen {
     return AK_DIRECT;
   }
   static std::string pv(int i, const char* what) { return "p" + std::to_string(i) + what; }
-  void probe_defs(const KProbe& pr) {
+  void probe_defs(const KProbe& pr, int idx = -1) {
     const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
     const bool outer = pr.mode == HQ_PROBE_OUTER;  // a miss leaves 0
+    if (npay > 0 && idx >= 0 && access(pr) != AK_DIRECT && access(pr) != AK_LINEAR && pr.ckind == 2 && pr.crank) {
+      // a rank-coded byte map: the register keeps the rank (an OUTER probe's 0 default
+      // is a value, so there the byte is mapped back at the probe instead)
+      if (!outer) rank_of[pr.dst[0]] = idx;
+      else rank_probe.insert(idx);
+      bitmaps << "static constexpr __device__ int RV_" << idx << "[256] = {";
+      int n = 0;
+      for (int d = 0; d <= pr.pay_max - pr.pay_min; ++d) {
+        const uint32_t v = (uint32_t)(pr.pay_min + d) & 255u;
+        if ((pr.pay_set[v >> 6] >> (v & 63)) & 1ull) bitmaps << (n++ ? ", " : "") << (pr.pay_min + d);
+      }
+      bitmaps << "};\n";
+    }
     for (int k = 0; k < npay; ++k) {
       o << "      int " << var(pr.dst[k]) << (outer ? "[R] = {};\n" : "[R];\n");
       if (k == 0 && pr.pay_min <= pr.pay_max)
@@ -216,20 +264,21 @@ struct Gen {
   void probe_addr(const KProbe& pr, int i) {
     const std::string key = val(pr.key_reg);
     const std::string D = pv(i, "d_"), M = pv(i, "m_");
-    o << "      u32 " << D << "[R]; u32 " << M << " = 0u;\n#pragma unroll\n      for (int r = 0; r < R; ++r) {";
+    sync_al();
+    o << "      u32 " << D << "[R]; bool " << M << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) {";
     if (width(pr.key_reg) <= 4)  // int32 keys: (k - min) mod 2^32 < range  <=>  min <= k < min + range
       o << " const u32 d_ = (u32)(int)" << key << " - " << (uint32_t)pr.dmin << "u; const bool in_ = d_ < " << pr.mask << "u;";
     else
       o << " const long long k_ = (long long)" << key << "; const u32 d_ = (u32)(k_ - " << pr.dmin
         << "LL); const bool in_ = k_ >= " << pr.dmin << "LL && k_ < " << pr.dmin << "LL + " << pr.mask << "LL;";
-    o << " " << D << "[r] = d_; if (((mask >> r) & 1u) && in_) " << M << " |= 1u << r; }\n";
+    o << " " << D << "[r] = d_; " << M << "[r] = al_[r] && in_; }\n";
   }
   void probe_load(const KProbe& pr, int i) {
     const std::string D = pv(i, "d_"), M = pv(i, "m_"), V = pv(i, "v_");
     const int ak = access(pr);
     if (ak == AK_DIRECT) {
       const int W = pr.words;
-      o << "      int4 " << V << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((" << M << " >> r) & 1u) ";
+      o << "      int4 " << V << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) if (" << M << "[r]) ";
       if (W == 1) o << V << "[r].x = __ldg((const int*)p.ht[" << i << "] + " << D << "[r]);\n";
       else if (W == 2)
         o << "{ const int2 q_ = __ldg((const int2*)p.ht[" << i << "] + " << D << "[r]); " << V << "[r].x = q_.x; " << V
@@ -249,33 +298,41 @@ struct Gen {
     else
       ld = pr.ckind == 1 ? "__ldg((const u32*)p.ctab[" + std::to_string(i) + "] + " + idx + ")"
                          : "(u32)__ldg((const unsigned char*)p.ctab[" + std::to_string(i) + "] + " + idx + ")";
-    o << "      u32 " << V << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) if ((" << M << " >> r) & 1u) " << V
+    o << "      u32 " << V << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) if (" << M << "[r]) " << V
       << "[r] = " << ld << ";\n";
   }
   void probe_resolve(const KProbe& pr, int i) {
     const std::string D = pv(i, "d_"), M = pv(i, "m_"), V = pv(i, "v_");
     const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
-    o << "      { u32 found_ = 0u;\n#pragma unroll\n        for (int r = 0; r < R; ++r) if ((" << M << " >> r) & 1u) {";
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { bool f_ = false; if (" << M << "[r]) {";
     if (access(pr) == AK_DIRECT) {
       static const char* comp[3] = {"y", "z", "w"};
-      o << " if (" << V << "[r].x != HQ_INT_MIN) { found_ |= 1u << r;";
+      o << " if (" << V << "[r].x != HQ_INT_MIN) { f_ = true;";
       for (int k = 0; k < npay; ++k) o << " " << var(pr.dst[k]) << "[r] = " << V << "[r]." << comp[k] << ";";
       o << " }";
     } else if (pr.ckind == 1) {
-      o << " if ((" << V << "[r] >> (" << D << "[r] & 31u)) & 1u) found_ |= 1u << r;";
+      o << " f_ = (" << V << "[r] >> (" << D << "[r] & 31u)) & 1u;";
     } else {
       if (pr.ckind == 3) o << " const u32 b_ = (" << V << "[r] >> ((" << D << "[r] & 1u) * 4u)) & 15u; if (b_ != 15u) {";
       else o << " const u32 b_ = " << V << "[r]; if (b_ != 0xFFu) {";
-      o << " found_ |= 1u << r;";
-      if (npay > 0) o << " " << var(pr.dst[0]) << "[r] = (int)b_ + (" << pr.pay_min << ");";
+      o << " f_ = true;";
+      if (npay > 0 && rank_of.count(pr.dst[0])) o << " " << var(pr.dst[0]) << "[r] = (int)b_;";  // the rank
+      else if (npay > 0 && rank_probe.count(i)) o << " " << var(pr.dst[0]) << "[r] = RV_" << i << "[b_ & 255u];";
+      else if (npay > 0) o << " " << var(pr.dst[0]) << "[r] = (int)b_ + (" << pr.pay_min << ");";
       o << " }";
     }
-    o << " }\n        mask = " << mask_after(pr) << "; }\n";
+    o << " }";
+    if (pr.mode == HQ_PROBE_ANTI) o << " al_[r] = al_[r] && !f_;";
+    else if (pr.mode == HQ_PROBE_OUTER) o << " (void)f_;";
+    else o << " al_[r] = al_[r] && f_;";  // (a batched probe's address step saw the liveness before the batch)
+    o << " }\n";
+    live = LIVE_AL;
   }
 
   // linear-probing table (sparse keys): optional exact key-range bitmap, then
   // 16-B group scans until the key or an empty slot
   void probe_linear(const KProbe& pr, int idx) {
+    sync_mask();
     const int W = pr.words;
     const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
     probe_defs(pr);
@@ -322,6 +379,7 @@ struct Gen {
       << "            else pos_[r] = ((pos_[r] / " << G << " + 1) * " << G << ") & " << pr.mask << "u;\n"
       << "          }\n        }\n";
     o << "        mask = " << mask_after(pr) << "; }\n";
+    mask_written();
   }
 
   // ops [i, end): one probe batch starting at op i (see probe_addr)
@@ -345,7 +403,7 @@ struct Gen {
         for (int k = 0; k < (hq_probe_has_payload(pr.mode) ? pr.npay : 0); ++k) defs.insert(pr.dst[k]);
       }
     }
-    for (int j : b) probe_defs(kp.probes[kp.ops[j].idx]);
+    for (int j : b) probe_defs(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
     for (int j : b) probe_addr(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
     for (int j : b) probe_load(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
     for (int j : b) probe_resolve(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
@@ -357,6 +415,7 @@ struct Gen {
     return "(long long)" + val(in.reg);
   }
   void compute(const KCompute& c) {
+    sync_mask();  // DIV / MOD flag faults of live rows only
     // operands first (column loads must not land inside the row loop)
     std::vector<std::string> ops;
     for (int k = 0; k < c.n; ++k) ops.push_back(operand(kp.insns[c.first + k]));
@@ -419,6 +478,7 @@ struct Gen {
   // ONE row slot (R redefined to 1 in that scope).  Columns not loaded yet are
   // read from the stage at the compacted row (row0 redefined).
   void compact(int from) {
+    sync_mask();
     const int R0 = kp.R;
     std::vector<int> live;
     for (int r : uses_from(from))
@@ -445,10 +505,26 @@ struct Gen {
       if (!keep.count(r)) dead.insert(r);
     open += 3;
     compacted_R = R0;
+    mask_written();
   }
   int compacted_R = 0;  // original R when compact() ran (restored after the scope)
   std::ostringstream bitmaps;
 };
+
+// LCOL[a]: the shared-table word of aggregate a (0 = the count word, for COUNT);
+// LFN[c]: the aggregate function of word c (for its identity)
+std::string lcol_tables(const KPlan& kp) {
+  std::ostringstream s;
+  s << "static constexpr __device__ int LCOL[" << (kp.naggs > 0 ? kp.naggs : 1) << "] = {";
+  for (int a = 0; a < (kp.naggs > 0 ? kp.naggs : 1); ++a) s << (a ? ", " : "") << (a < kp.naggs ? (int)kp.lcol[a] : 0);
+  s << "};\nstatic constexpr __device__ int LFN[" << (kp.lvwords > 0 ? kp.lvwords : 1) << "] = {";
+  std::vector<int> fn(kp.lvwords > 0 ? kp.lvwords : 1, HQ_AGG_COUNT);
+  for (int a = 0; a < kp.naggs; ++a)
+    if (kp.lcol[a]) fn[kp.lcol[a]] = kp.agg_fn[a];
+  for (size_t c = 0; c < fn.size(); ++c) s << (c ? ", " : "") << fn[c];
+  s << "};\n";
+  return s.str();
+}
 
 std::string fn_list(const uint8_t* fns, int n) {
   std::ostringstream s;
@@ -593,12 +669,12 @@ std::string generate(const KPlan& kp) {
     o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * NACC * NW * 32; i += NW * 32) {"
       << " const int a_ = (int)((i / (NW * 32)) % NACC); t_[i] = a_ == 0 ? 0 : agg_identity(ACC_FN[a_]); } }\n";
   } else if (sk == 1 && kp.smode == SM_DENSE) {
-    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * VWORDS * SCOPIES; i += NW * 32) {"
-      << " const int c_ = (int)(i % VWORDS); t_[i] = c_ == 0 ? 0 : agg_identity(AGG_FN[c_ - 1]); } }\n";
+    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * LVWORDS * SCOPIES; i += NW * 32) {"
+      << " const int c_ = (int)(i % LVWORDS); t_[i] = c_ == 0 ? 0 : agg_identity(LFN[c_]); } }\n";
   } else if (sk == 1 && kp.smode == SM_HASH) {
     o << "  if (warp < NW) { u64* k_ = (u64*)sagg; i64* e_ = (i64*)sagg + SMEM_CAP;\n"
       << "    for (u32 i = threadIdx.x; i < SMEM_CAP; i += NW * 32) k_[i] = HQ_EMPTY_KEY;\n"
-      << "    for (u32 i = threadIdx.x; i < SMEM_CAP * VWORDS; i += NW * 32) { const int c_ = (int)(i % VWORDS); e_[i] = c_ == 0 ? 0 : agg_identity(AGG_FN[c_ - 1]); } }\n";
+      << "    for (u32 i = threadIdx.x; i < SMEM_CAP * LVWORDS; i += NW * 32) { const int c_ = (int)(i % LVWORDS); e_[i] = c_ == 0 ? 0 : agg_identity(LFN[c_]); } }\n";
   }
   // staged compact probe tables: one cooperative 16-B copy per CTA
   for (int i = 0; i < MAX_PROBES; ++i) {
@@ -706,6 +782,7 @@ std::string generate(const KPlan& kp) {
       if (kp.ops[i].kind == OP_PROBE && kp.probes[kp.ops[i].idx].pass_est <= 0.5f) cpt = i;
   if (const char* e = getenv("HQ_JIT_CPT")) cpt = (e[0] == 'o') ? -1 : (sk != 2 ? atoi(e) : -1);
   if (mp) cpt = -1;
+  g.begin_al();
   for (int i = 0; i < kp.nops;) {
     if (cpt >= 0 && !g.compacted_R && i > cpt) g.compact(i);
     if (kp.op_skip[i]) { ++i; continue; }  // not executed in this pass
@@ -716,6 +793,7 @@ std::string generate(const KPlan& kp) {
     ++i;
   }
   if (cpt >= 0 && !g.compacted_R) g.compact(kp.nops);
+  g.sync_mask();  // the sinks, the block scan and the count kernel's flags read mask
   if (mp == 1) {
     // count kernel: the flags are written below, after the early-exit blocks
     // close -- every row of the range gets its flag, also in a warp whose rows
@@ -799,7 +877,10 @@ std::string generate(const KPlan& kp) {
       const bool ranked = kp.local_keys && (ls[0] | ls[1] | ls[2] | ls[3]);
       std::string dexpr;  // the key's offset (or rank) in the (narrowed) domain
       const std::string off32 = "((u32)(long long)" + v + " - " + std::to_string((uint32_t)kmin) + "u)";
-      if (ranked) {  // index by the rank of the value among the build side's distinct payloads
+      auto rkr = g.rank_of.find(kp.key_reg[i]);
+      if (ranked && rkr != g.rank_of.end() && kp.probes[rkr->second].pay_min == kmin) {
+        dexpr = "(u32)" + g.var(kp.key_reg[i]) + "[r]";  // the byte map holds the rank already
+      } else if (ranked) {  // index by the rank of the value among the build side's distinct payloads
         int top = 0;
         for (int d = 0; d < 256; ++d)
           if ((ls[d >> 6] >> (d & 63)) & 1ull) top = d + 1;
@@ -1022,8 +1103,8 @@ std::string generate(const KPlan& kp) {
     o << "  consumer_bar();\n  { const i64* t_ = (const i64*)sagg;\n"
       << "    for (u32 g = threadIdx.x; g < SMEM_CAP; g += NW * 32) { i64 cnt_ = 0; i64 vals_[NAGGS > 0 ? NAGGS : 1];\n"
       << "#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = agg_identity(AGG_FN[a]);\n"
-      << "      for (u32 c_ = 0; c_ < SCOPIES; ++c_) { const i64* e_ = t_ + ((u64)c_ * SMEM_CAP + g) * VWORDS; cnt_ += e_[0];\n"
-      << "#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) if (AGG_FN[a] != F_COUNT) vals_[a] = agg_combine(AGG_FN[a], vals_[a], e_[1 + a]); }\n"
+      << "      for (u32 c_ = 0; c_ < SCOPIES; ++c_) { const i64* e_ = t_ + ((u64)c_ * SMEM_CAP + g) * LVWORDS; cnt_ += e_[0];\n"
+      << "#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) if (AGG_FN[a] != F_COUNT) vals_[a] = agg_combine(AGG_FN[a], vals_[a], e_[LCOL[a]]); }\n"
       << "      if (cnt_ != 0) {\n#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) if (AGG_FN[a] == F_COUNT) vals_[a] = cnt_;\n"
       << "        u64 gkey_ = g;\n";
     if (kp.local_keys) {  // narrowed local index -> declared global key
@@ -1046,8 +1127,8 @@ std::string generate(const KPlan& kp) {
     o << "        group_update(p, sagg, gkey_, false, (u64)cnt_, vals_); } } }\n";
   } else if (sk == 1 && kp.smode == SM_HASH) {
     o << "  consumer_bar();\n  { const u64* k_ = (const u64*)sagg; const i64* t_ = (const i64*)sagg + SMEM_CAP;\n"
-      << "    for (u32 h = threadIdx.x; h < SMEM_CAP; h += NW * 32) if (k_[h] != HQ_EMPTY_KEY) { const i64* e_ = t_ + (u64)h * VWORDS;\n"
-      << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = AGG_FN[a] == F_COUNT ? e_[0] : e_[1 + a];\n"
+      << "    for (u32 h = threadIdx.x; h < SMEM_CAP; h += NW * 32) if (k_[h] != HQ_EMPTY_KEY) { const i64* e_ = t_ + (u64)h * LVWORDS;\n"
+      << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = AGG_FN[a] == F_COUNT ? e_[0] : e_[LCOL[a]];\n"
       << "      group_update(p, sagg, k_[h], false, (u64)e_[0], vals_); } }\n";
   }
   if (prof) o << "  if (threadIdx.x == 0) { long long t_; asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(t_)); p.prof[blockIdx.x * 128] = pt0_; p.prof[blockIdx.x * 128 + 5] = t_;"
@@ -1066,6 +1147,7 @@ std::string generate(const KPlan& kp) {
     << "static constexpr __device__ int AGG_FN[" << (kp.naggs > 0 ? kp.naggs : 1) << "] = " << fn_list(kp.agg_fn, kp.naggs)
     << ";\n"
     << "static constexpr __device__ int ACC_FN[" << (kp.nacc > 0 ? kp.nacc : 1) << "] = " << fn_list(kp.acc_fn, kp.nacc) << ";\n"
+    << "#define LVWORDS " << kp.lvwords << "\n" << lcol_tables(kp)
     << HQ_STR(HQ_JPARAMS_DEF) << "\n"
     << kPrelude << "\n"
     << g.bitmaps.str() << "\n";

@@ -191,7 +191,7 @@ __device__ __forceinline__ i64* global_locate(const JParams& p, u64 key) {
 }
 // shared pre-aggregation table entry (dense or hash), 0 when the hash is full
 __device__ __forceinline__ u32 local_locate(char* sagg, u64 key) {
-  if (SMODE == 1) return smem_u32((i64*)sagg + ((u64)((threadIdx.x >> 5) % SCOPIES) * SMEM_CAP + key) * VWORDS);
+  if (SMODE == 1) return smem_u32((i64*)sagg + ((u64)((threadIdx.x >> 5) % SCOPIES) * SMEM_CAP + key) * LVWORDS);
   if (SMODE == 2) {
     u64* keys = (u64*)sagg;
     i64* ent = (i64*)sagg + SMEM_CAP;
@@ -204,7 +204,7 @@ __device__ __forceinline__ u32 local_locate(char* sagg, u64 key) {
         const u64 old = atomicCAS(keys + h, HQ_EMPTY_KEY, key);
         hit = old == HQ_EMPTY_KEY || old == key;
       }
-      if (hit) return smem_u32(ent + (u64)h * VWORDS);
+      if (hit) return smem_u32(ent + (u64)h * LVWORDS);
       h = (h + 1) & (SMEM_CAP - 1);
     }
   }
@@ -220,7 +220,7 @@ __device__ __forceinline__ void group_update(const JParams& p, char* sagg, u64 k
     asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(sa), "r"((u32)cnt) : "memory");
 #pragma unroll
     for (int a = 0; a < NAGGS; ++a)
-      if (AGG_FN[a] != F_COUNT) s_agg(AGG_FN[a], sa + 8u * (1 + a), vals[a], cnt);
+      if (AGG_FN[a] != F_COUNT) s_agg(AGG_FN[a], sa + 8u * LCOL[a], vals[a], cnt);
     return;
   }
   i64* e = global_locate(p, key);

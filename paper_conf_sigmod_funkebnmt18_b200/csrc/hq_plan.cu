@@ -128,6 +128,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.dmin = (int32_t)op.ht->meta.key_min;
       pr.log2cap = (uint8_t)op.ht->log2cap;
       pr.ckind = (uint8_t)op.ht->ckind;
+      pr.crank = (uint8_t)op.ht->crank;
       pr.compact = op.ht->compact.p;
       pr.pay_min = op.ht->meta.pay_min;
       pr.pay_max = op.ht->meta.pay_max;
@@ -219,6 +220,11 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       kp.agg_reg[a] = P.agg_fn[a] == HQ_AGG_COUNT ? (int16_t)0 : (int16_t)use(P.agg_reg[a], "aggregate");
     }
     kp.vwords = 1 + P.naggs;
+    kp.lvwords = 1;
+    for (int a = 0; a < P.naggs; ++a) {  // interpreter: the global layout; generated: COUNTs share word 0
+      if (jit && P.agg_fn[a] == HQ_AGG_COUNT) kp.lcol[a] = 0;
+      else kp.lcol[a] = (uint8_t)kp.lvwords++;
+    }
     // a dense global table for a tight but large key domain (fused execution): no hash
     // claim round trip per group update, when it is at most twice the hash table's size
     auto dense_global = [&](int64_t ng) {
@@ -301,7 +307,28 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       }
       lgroups *= lcard[i];
     }
-    // local-resolution table in shared memory
+    // local-resolution table in shared memory: 32 KB, or for a probe-free generated
+    // kernel (nothing else competes for shared memory) whatever the TMA ring leaves
+    // with 3 stages of the 2-rows-per-lane tile (Exp 2: up to 8,192 groups
+    // keep their pre-aggregation in shared memory)
+    uint64_t agg_budget = SMEM_AGG_BYTES;
+    if (jit && nprobe == 0 && !mp_pass) {
+      uint32_t rb = 0;
+      for (int c = 0; c < F->ncols; ++c) rb += col_used[c] ? (uint32_t)F->cols[c].width : 0u;
+      const uint64_t stage = align_up(31u * 32u * 2u * std::max<uint32_t>(rb, 1u), 128);
+      const uint64_t avail = ctx->max_smem > MISC_BYTES + 3 * stage + 1024 ? ctx->max_smem - MISC_BYTES - 3 * stage - 1024 : 0;
+      agg_budget = std::max<uint64_t>(agg_budget, avail / 128 * 128);
+    }
+    const uint32_t lvw = kp.lvwords;
+    // a group key narrowed to the rank of a rank-coded byte map (hq_build_compact) indexes
+    // the shared table with the probe's byte itself: prefer the narrowed table then
+    bool ranked_narrow = false;
+    for (int i = 0; jit && i < P.nkeys; ++i) {
+      if (!(kp.lkey_set[i][0] | kp.lkey_set[i][1] | kp.lkey_set[i][2] | kp.lkey_set[i][3])) continue;
+      for (int q = 0; q < nprobe; ++q)
+        if (kp.probes[q].dst[0] == kp.key_reg[i] && kp.probes[q].crank && kp.probes[q].ckind == 2 && kp.probes[q].npay > 0)
+          ranked_narrow = true;
+    }
     kp.smode = SM_NONE;
     if (P.nkeys > 0 && P.resolution == HQ_RES_LRGP) {
       // lane-private tables halve the warps, so only for probe-free pipelines
@@ -311,15 +338,15 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         kp.smode = SM_LANE;  // tiny domain (e.g. TPC-H Q1): contention-free lane-private tables
         kp.smem_cap = (uint32_t)ngroups;
         agg_smem = (uint32_t)(ngroups * kp.nacc * LANE_NW * 32 * 8);
-      } else if (kp.gmode == GM_DENSE && (uint64_t)ngroups * kp.vwords * 8 <= (uint64_t)SMEM_AGG_BYTES) {
+      } else if (kp.gmode == GM_DENSE && (uint64_t)ngroups * lvw * 8 <= agg_budget && !(ranked_narrow && lgroups < (__int128)ngroups)) {
         kp.smode = SM_DENSE;
         kp.smem_cap = (uint32_t)ngroups;
-        agg_smem = (uint32_t)(ngroups * kp.vwords * 8);
-      } else if (lgroups < (__int128)ngroups && lgroups * kp.vwords * 8 <= (__int128)SMEM_AGG_BYTES) {
+        agg_smem = (uint32_t)(ngroups * lvw * 8);
+      } else if (lgroups < (__int128)ngroups && lgroups * lvw * 8 <= (__int128)agg_budget) {
         kp.smode = SM_DENSE;  // dense over the narrowed domain; merged into the global table by key
         kp.local_keys = 1;
         kp.smem_cap = (uint32_t)lgroups;
-        agg_smem = (uint32_t)(lgroups * kp.vwords * 8);
+        agg_smem = (uint32_t)(lgroups * lvw * 8);
         int64_t st2 = 1;
         for (int i = P.nkeys - 1; i >= 0; --i) {
           kp.lkey_min[i] = lmin[i];
@@ -327,8 +354,8 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
           st2 *= lcard[i];
         }
       } else {
-        uint32_t cap = 4096;
-        while (cap > 64 && (uint64_t)cap * (kp.vwords + 1) * 8 > (uint64_t)SMEM_AGG_BYTES) cap >>= 1;
+        uint32_t cap = agg_budget > SMEM_AGG_BYTES ? 16384 : 4096;
+        while (cap > 64 && (uint64_t)cap * (lvw + 1) * 8 > agg_budget) cap >>= 1;
         // far more groups than the shared table holds (TPC-H Q3: ~10^5-10^6
         // orderkeys): it would fill up and every later row would scan it before
         // going to global memory -- update the global table directly (C2)
@@ -343,7 +370,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         int l = 0;
         while ((1u << l) < cap) ++l;
         kp.slog2 = l;
-        agg_smem = cap * (kp.vwords + 1) * 8;
+        agg_smem = cap * (lvw + 1) * 8;
         }
       }
     }
@@ -375,7 +402,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     // every row updates a probe-free pipeline's table; behind selective probes
     // (star joins: 1-4 % of the rows) contention is low and the shared memory
     // is worth more to the staged probe tables and the TMA ring
-    const uint64_t one = (uint64_t)kp.smem_cap * kp.vwords * 8;
+    const uint64_t one = (uint64_t)kp.smem_cap * kp.lvwords * 8;
     const uint64_t budget = nprobe == 0 ? (uint64_t)SMEM_AGG_BYTES : 4096;
     uint32_t c = 1;
     while (c < 31 && one * (c + 1) <= budget) ++c;

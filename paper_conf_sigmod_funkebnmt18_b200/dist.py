@@ -62,14 +62,23 @@ class RootError(hq.HQError):
     pipeline) did: every rank raises, none is left waiting in a collective."""
 
 
+def _offsets(rows: Sequence[Sequence[int]]) -> Tuple[List[int], int]:
+    """Byte offsets of the tables' slot arrays in the packed broadcast buffer (256-B aligned)."""
+    offs, tot = [], 0
+    for r in rows:
+        offs.append(tot)
+        tot += (int(r[4]) + 255) // 256 * 256
+    return offs, tot
+
+
 def broadcast_tables(rows: Optional[List[List[int]]], bufs: Optional[List[torch.Tensor]], n: int, root: int,
                      device, err: Optional[BaseException] = None) -> Tuple[List[List[int]], List[torch.Tensor]]:
-    """Broadcast n root-built tables: ONE broadcast of an (n+1) x 16 int64 metadata block
-    (row n = the root's status: error code or 0), then one broadcast per byte buffer
-    (row[4] bytes each).  Root: rows / bufs given (bufs are sent in place); other ranks:
-    None, buffers are allocated here.  A root-side error is broadcast before the root
-    re-raises it, so the other ranks raise RootError instead of blocking in the next
-    collective."""
+    """Broadcast n root-built tables with TWO collectives: an (n+1) x 16 int64 metadata
+    block (row n = the root's status: error code or 0), then ONE byte buffer holding every
+    slot array at 256-B aligned offsets (the root packs them with device copies; the
+    other ranks get views into it).  Root: rows / bufs given; other ranks: None.  A
+    root-side error is broadcast before the root re-raises it, so the other ranks raise
+    RootError instead of blocking in the next collective."""
     rank = dist.get_rank()
     meta = torch.zeros((n + 1, META_COLS), dtype=torch.int64, device=device)
     if rank == root:
@@ -81,18 +90,24 @@ def broadcast_tables(rows: Optional[List[List[int]]], bufs: Optional[List[torch.
     if rank == root:
         if err is not None:
             raise err
-        for b in bufs:
-            dist.broadcast(b, src=root)
+        if n == 0:
+            return rows, bufs
+        offs, tot = _offsets(rows)
+        packed = torch.empty(tot, dtype=torch.uint8, device=device)
+        for o, b in zip(offs, bufs):
+            packed[o:o + b.numel()].copy_(b)
+        dist.broadcast(packed, src=root)
         return rows, bufs
     m = meta.cpu().tolist()
     if m[n][0] != 0:
         raise RootError(int(m[n][0]), "hash build failed on the root rank")
-    out = []
-    for r in m[:n]:
-        b = torch.empty(int(r[4]), dtype=torch.uint8, device=device)
-        dist.broadcast(b, src=root)
-        out.append(b)
-    return m[:n], out
+    rows = m[:n]
+    if n == 0:
+        return rows, []
+    offs, tot = _offsets(rows)
+    packed = torch.empty(tot, dtype=torch.uint8, device=device)
+    dist.broadcast(packed, src=root)
+    return rows, [packed[o:o + int(r[4])] for o, r in zip(offs, rows)]
 
 
 def reduce_partials(t: torch.Tensor, root: int) -> None:
@@ -150,7 +165,7 @@ class DistributedEngine(Engine):
             broadcast_tables(rows, views, n, self.root, self.device, err)
             return list(hs)
         rows, bufs = broadcast_tables(None, None, n, self.root, self.device)
-        return [self.ctx.import_hash(meta_from_row(r), b.data_ptr(), keep=b) for r, b in zip(rows, bufs)]
+        return [self.ctx.import_hash(meta_from_row(r), b.data_ptr(), keep=b) for r, b in zip(rows, bufs)]  # views keep the buffer
 
     def _root_build(self, fn, n: int):
         hs, err = None, None

@@ -15,7 +15,7 @@ from typing import Dict, List, Optional, Sequence
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(_PKG, "libhq.so")
+SO_PATH = os.environ.get("HQ_LIB_PATH") or os.path.join(_PKG, "libhq.so")  # override: debugging only
 
 # ---- constants (mirror hq.h) ----------------------------------------------
 HQ_OK, HQ_ERR_ARG, HQ_ERR_CUDA, HQ_ERR_OOM, HQ_ERR_DUP_KEY = 0, -1, -2, -3, -4
@@ -169,7 +169,9 @@ def lib():
             "hq_graph_launch": [vp, vp], "hq_graph_destroy": [vp],
         }
         for name, args in sig.items():
-            f = getattr(L, name)
+            f = getattr(L, name, None)
+            if f is None:  # an older library (HQ_LIB_PATH): the call is unavailable
+                continue
             f.argtypes = args
             f.restype = ctypes.c_int32
         L.hq_last_error.restype = ctypes.c_char_p

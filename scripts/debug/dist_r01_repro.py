@@ -25,11 +25,67 @@ def worker(rank, world, port, q, reps):
     from paper_conf_sigmod_funkebnmt18_b200.engine import fetch
     from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES, load_tables
 
+    trace = os.environ.get("HQ_REPRO_TRACE") == "1"
+    log_t = torch.zeros((256, 32), dtype=torch.int64, device="cuda") if trace else None
+    labels = []
+
+    def probe(E, what):
+        """Enqueue (no sync) a read of every root build's fault words at this stream point."""
+        if not trace or E.rank != 0 or len(labels) >= 256:
+            return
+        hs = list(E._built) + [h for h in E._extra]
+        E.ctx.gather_faults(hs, [], log_t[len(labels)].data_ptr())
+        labels.append((what, len(hs)))
+
+    if os.environ.get("HQ_REPRO_CLONE") == "1":
+        # experiment: the root broadcasts torch-owned copies of its slot arrays instead of
+        # the library-owned arrays themselves (gloo then never writes the root's tables)
+        orig_bcast = dist_r01.dist.broadcast
+
+        def bcast_clone(t, src=0, **kw):
+            if dist.get_rank() == src and t.dtype == torch.uint8:
+                c = t.clone()
+                return orig_bcast(c, src=src, **kw)
+            return orig_bcast(t, src=src, **kw)
+        dist_r01.dist.broadcast = bcast_clone
+
     class Late(dist_r01.DistributedEngine):
+        def __init__(self, *a, **k):
+            super().__init__(*a, **k)
+            self._extra = []
+
+        def hash(self, *a, **k):
+            h = super().hash(*a, **k)
+            probe(self, "hash")
+            return h
+
+        def hashes(self, *a, **k):
+            hs = super().hashes(*a, **k)
+            probe(self, "hashes")
+            return hs
+
+        def hash_from(self, *a, **k):
+            h = super().hash_from(*a, **k)
+            probe(self, "hash_from")
+            return h
+
+        def run(self, *a, **k):
+            r = super().run(*a, **k)
+            probe(self, "run")
+            return r
+
+        def gather(self, *a, **k):
+            r = super().gather(*a, **k)
+            probe(self, "gather")
+            return r
+
         def finish(self, res, pb):
             built = list(self._built)
             self._built.clear()
+            self._extra = built
+            probe(self, "finish:start")
             out = super().finish(res, pb)  # the round-1 finish with an empty check list
+            probe(self, "finish:after-fetch")
             faults = []
             for i, h in enumerate(built):
                 try:
@@ -58,6 +114,15 @@ def worker(rank, world, port, q, reps):
                 faults = [("exception", repr(e)[:300])]
             if faults:
                 log.append((rep, qn, faults))
+            if trace and rank == 0 and faults:
+                torch.cuda.synchronize()
+                lt = log_t.cpu().tolist()
+                for i, (what, nh) in enumerate(labels):
+                    bits = [k for k in range(16) if lt[i][k]]
+                    log.append(("trace", qn, i, what, nh, bits))
+            labels.clear()
+            if trace:
+                log_t.zero_()
     q.put((rank, log))
     dist.barrier()
     dist.destroy_process_group()

@@ -213,6 +213,7 @@ int main(int argc, char** argv) {
       h->meta.pay_min = 4;
       h->meta.pay_max = 24;
       for (int v : {4, 9, 10, 13, 24}) h->meta.pay_set[v >> 6] |= 1ull << (v & 63);
+      h->crank = 1;  // rank-coded byte maps (hq_build_compact)
     }
     P.ops[0] = probe(ra, 1, HQ_PROBE_INNER, HQ_TMP(0));
     P.ops[1] = probe(rb, 0, HQ_PROBE_INNER, HQ_TMP(1));
@@ -290,6 +291,10 @@ int main(int argc, char** argv) {
   }
 
   {  // LEFT OUTER probes (byte map, linear, direct) and predicate expressions (TPC-H Q13 / Q19 shapes)
+    // the byte map rank-coded over a sparse payload set (Q13's orders-per-customer counts)
+    byte_big = make_hash(c, HQ_HT_DIRECT, 1, 2, 3000000);
+    for (int v : {1, 2, 5, 7, 24}) byte_big->meta.pay_set[v >> 6] |= 1ull << (v & 63);
+    byte_big->crank = 1;
     hq_plan P{};
     P.fact = F;
     P.row_end = -1;

@@ -50,7 +50,10 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "#define SMODE 1" in narrowed and "#define SMEM_CAP 1183u" in narrowed and "gkey_ +=" in narrowed
     # ... and by the rank among the payloads' distinct values (5 of the 21 codes 4..24)
     ranked = srcs["star_ranked_dense"]
-    assert "#define SMEM_CAP 175u" in ranked and "__popc(0x00100261u" in ranked and "dv_[o_]" in ranked
+    assert "#define SMEM_CAP 175u" in ranked and "dv_[o_]" in ranked
+    # rank-coded byte maps: the probe stores the rank, the group index uses it directly,
+    # and RV_ maps it back to the value where the value is needed
+    assert "RV_0[256] = {4, 9, 10, 13, 24}" in ranked and "__popc(0x00100261u" not in ranked
     # multi-pass (A1/B1/C1): the count kernel writes flags and skips the sink;
     # the write kernel reads flags + positions, skips filters / semi probes
     c1 = srcs["star_ranked_dense_mp1"]
@@ -62,9 +65,10 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "#define SMODE 0" in srcs["global_hash_groups"]
     # LEFT OUTER probes keep the row and default the payload to 0; predicate instructions
     op = srcs["outer_predicates"]
-    assert "[R] = {};" in op and "mask; (void)found_" in op
+    assert "[R] = {};" in op and "(void)f_" in op
+    assert "= RV_0[b_ & 255u];" in op  # a rank-coded byte map decoded at an OUTER probe
     assert "(a_ != 0 && " in op and "3855ULL >> v_" in op and "(a_ != 0 || " in op
-    assert "mask; (void)found_" not in srcs["outer_predicates_mp2"].split("extern \"C\"")[0]
+    assert "(void)f_" not in srcs["outer_predicates_mp2"].split("extern \"C\"")[0]
     # composite keys: the slot's word 1 is compared with the second key, payloads start at word 2
     cp = srcs["composite_probe"]
     assert "kk2_[r] = (int)(long long)c2[r];" in cp and "sl_[r].y == kk2_[r]" in cp and "= sl_[r].z;" in cp
