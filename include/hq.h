@@ -217,13 +217,23 @@ typedef struct {
   uint64_t pay_set[4];  /* payload-0 values present: bit (v & 255) (count pass); exact when
                          * pay_max - pay_min < 256, all-zero when unknown (expected_rows builds) */
   int32_t composite;    /* built with hq_build_desc::composite (payload word 0 = second key) */
+  int32_t compact_kind; /* hq_hash_device_view / hq_hash_import: 0 = the buffer is the slot array; 1 / 2 / 3 =
+                         * the buffer is the compact form of a direct table (1 bitmap of present keys, 2 one
+                         * byte per key, 3 one nibble per key; see below) -- tables whose only consumers
+                         * read that form are built straight into it */
 } hq_hash_meta;
 /* Derived forms (rebuilt on import): direct tables get a compact form -- a
  * bitmap of present keys for semi-join tables, or one byte per key (payload -
- * pay_min, 0xFF = absent) when payload 0 spans <= 255 values -- that generated
- * kernels stage in shared memory; linear tables whose key range fits in 64 MiB
- * of bits get an exact key-range bitmap that generated kernels test before
- * touching the slot array (most probe misses then never leave L2). */
+ * pay_min, or the payload's rank among the present payload values when they are a
+ * sparse set; 0xFF = absent) when payload 0 spans < 255 values, or one nibble per
+ * key when it spans < 15 -- that generated kernels stage in shared memory.  Such a
+ * direct table is built straight into its compact form (one atomic per row, duplicate
+ * keys detected by it); its slot array is derived only if a consumer that reads slots
+ * (precompiled interpreter, operator-at-a-time) probes it.  hq_hash_device_view then
+ * returns the compact form (meta.compact_kind != 0), which hq_hash_import accepts.
+ * Linear tables whose key range fits in 64 MiB of bits get an exact key-range
+ * bitmap that generated kernels test before touching the slot array (most probe
+ * misses then never leave L2). */
 hq_status hq_hash_info(hq_ctx* ctx, const hq_hash* h, hq_hash_meta* meta);  /* syncs, reports build faults */
 /* Multi-GPU glue: raw device view of the slot array (to broadcast it with NCCL)
  * and import of such a buffer on another device (borrowed, caller keeps it). */

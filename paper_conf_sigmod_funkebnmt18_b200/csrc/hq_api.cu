@@ -454,8 +454,16 @@ hq_status hq_hash_info(hq_ctx* ctx, const hq_hash* h, hq_hash_meta* meta) {
 hq_status hq_hash_device_view(const hq_hash* h, void** dev_ptr, hq_hash_meta* meta) {
   return guarded([&] {
     if (!h) HQ_THROW(HQ_ERR_ARG, "hash is NULL");
-    if (dev_ptr) *dev_ptr = h->slots;
-    if (meta) *meta = h->meta;
+    if (dev_ptr) *dev_ptr = h->compact_only ? const_cast<void*>(h->compact_ptr()) : (void*)h->slots;
+    if (meta) {
+      *meta = h->meta;
+      if (h->compact_only) {  // the buffer is the compact form
+        meta->compact_kind = h->ckind;
+        meta->bytes = h->cbytes;
+      } else {
+        meta->compact_kind = 0;
+      }
+    }
   });
 }
 
@@ -476,6 +484,29 @@ hq_status hq_hash_import(hq_ctx* ctx, const hq_hash_meta* meta, void* dev_ptr, h
         (meta->slot_words == 1 && meta->npayload != 0))
       HQ_THROW(HQ_ERR_ARG, "import: npayload");
     if (((uintptr_t)dev_ptr & 15) != 0) HQ_THROW(HQ_ERR_ARG, "import: pointer must be 16-byte aligned");
+    if (meta->compact_kind != 0) {  // a compact-only direct table: the buffer is its compact form
+      if (meta->layout != HQ_HT_DIRECT ||
+          meta->compact_kind != hq_compact_kind(meta->npayload, meta->pay_min, meta->pay_max))
+        HQ_THROW(HQ_ERR_ARG, "import: compact_kind does not match the table");
+      if (meta->bytes < hq_compact_words(meta->compact_kind, cap) * 4) HQ_THROW(HQ_ERR_ARG, "import: compact form too small");
+      hq_hash* h = new hq_hash();
+      h->ctx = ctx;
+      h->meta = *meta;
+      h->meta.compact_kind = 0;
+      h->meta.bytes = cap * meta->slot_words * 4;
+      h->compact_borrow = dev_ptr;
+      h->ckind = meta->compact_kind;
+      unsigned char lut[256];
+      h->crank = h->ckind == 2 ? hq_rank_lut(*meta, lut) : 0;
+      h->cbytes = hq_compact_words(h->ckind, cap) * 4;
+      h->compact_only = true;
+      int l = 0;
+      while ((1LL << l) < cap) ++l;
+      h->log2cap = l;
+      h->checked = true;
+      *out = h;
+      return;
+    }
     hq_hash* h = new hq_hash();
     h->ctx = ctx;
     h->meta = *meta;

@@ -218,6 +218,101 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __gri
   }
 }
 
+// A direct table whose only consumers read its compact form (generated kernels) is
+// built straight into that form: one pass over the dimension rows, one atomic per
+// qualifying row on the (memset) bitmap / byte map / nibble map, which also detects a
+// duplicate key (the atomic returns the previous bits) -- no slot array, no fill, no
+// separate compaction.  kind: 1 bitmap, 2 byte (payload - pay_min, or its rank through
+// lut), 3 nibble.  The slot array is derived later only if a consumer needs it.
+struct CLut {
+  unsigned char r[256];
+};
+__global__ void __launch_bounds__(BUILD_BLOCK) hq_build_direct_compact_kernel(const __grid_constant__ KBuild b, int kind,
+                                                                             uint32_t* out, long long range, int pay_min,
+                                                                             int use_lut, const __grid_constant__ CLut lut) {
+  int fault = 0;
+  unsigned long long qual = 0;
+  const long long base = (long long)blockIdx.x * BUILD_BLOCK * BUILD_U + threadIdx.x;
+  bool pass[BUILD_U];
+  long long kv[BUILD_U], pv[BUILD_U] = {};
+  load_rows(b, base, pass, kv, pv);
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u) {
+    if (!pass[u]) continue;
+    int pc = 0;
+    if (b.npay > 0) {
+      pc = pv[u] < (long long)INT_MIN ? INT_MIN : (pv[u] > (long long)INT_MAX ? INT_MAX : (int)pv[u]);
+      if (pv[u] < (long long)INT_MIN || pv[u] > (long long)INT_MAX) fault |= HQF_BAD_PAYLOAD;
+    }
+    if (b.verify) {
+      ++qual;
+      if (kv[u] > (long long)INT_MIN && kv[u] <= (long long)INT_MAX && (kv[u] < b.vs.kmin || kv[u] > b.vs.kmax))
+        fault |= HQF_STALE;
+      if (b.npay > 0 && (pc < b.vs.pmin || pc > b.vs.pmax || !((b.vs.set[(pc & 255) >> 5] >> (pc & 31)) & 1u)))
+        fault |= HQF_STALE;
+    }
+    if (kv[u] <= (long long)INT_MIN || kv[u] > (long long)INT_MAX) {
+      fault |= HQF_BAD_KEY;
+      continue;
+    }
+    const long long d = kv[u] - (long long)b.dmin;
+    if (d < 0 || d >= range) {  // cannot happen with exact or verified statistics
+      fault |= HQF_HT_FULL;
+      continue;
+    }
+    if (kind == 1) {
+      const uint32_t bit = 1u << (d & 31);
+      if (atomicOr(out + (d >> 5), bit) & bit) fault |= HQF_DUP_KEY;
+    } else if (kind == 2) {
+      uint32_t v = (uint32_t)(pc - pay_min) & 0xFFu;
+      if (use_lut) v = lut.r[v];
+      const uint32_t sh = (uint32_t)(d & 3) * 8u;
+      if (((atomicAnd(out + (d >> 2), ~((0xFFu ^ v) << sh)) >> sh) & 0xFFu) != 0xFFu) fault |= HQF_DUP_KEY;
+    } else {
+      const uint32_t v = (uint32_t)(pc - pay_min) & 0xFu;
+      const uint32_t sh = (uint32_t)(d & 7) * 4u;
+      if (((atomicAnd(out + (d >> 3), ~((0xFu ^ v) << sh)) >> sh) & 0xFu) != 0xFu) fault |= HQF_DUP_KEY;
+    }
+  }
+  if (fault) atomicOr(b.err, fault);
+  if (b.verify) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) qual += __shfl_xor_sync(0xffffffffu, qual, o);
+    __shared__ unsigned long long vred[BUILD_BLOCK / 32];
+    if ((threadIdx.x & 31) == 0) vred[threadIdx.x >> 5] = qual;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long t = 0;
+      for (int k = 0; k < BUILD_BLOCK / 32; ++k) t += vred[k];
+      if (t) atomicAdd(b.vqual, t);
+      __threadfence();
+      if (atomicAdd(b.ticket, 1u) == gridDim.x - 1) {
+        __threadfence();
+        if (*(volatile unsigned long long*)b.vqual != b.vs.cnt) atomicOr(b.err, HQF_STALE);
+      }
+    }
+  }
+}
+
+// the slot array of a compact-only direct table, derived from its compact form (for the
+// consumers that read slots: interpreter, operator-at-a-time, hq_hash_device_view)
+__global__ void hq_slots_from_compact_kernel(const uint32_t* c, int kind, long long range, int key_min, int pay_min,
+                                             int use_rv, const __grid_constant__ CLut rv_lo, const __grid_constant__ CLut rv_hi,
+                                             uint32_t* slots) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < range; i += (long long)gridDim.x * blockDim.x) {
+    if (kind == 1) {
+      slots[i] = ((c[i >> 5] >> (i & 31)) & 1u) ? (uint32_t)(key_min + (int)i) : 0x80000000u;
+      continue;
+    }
+    const uint32_t v = kind == 2 ? (c[i >> 2] >> ((i & 3) * 8)) & 0xFFu : (c[i >> 3] >> ((i & 7) * 4)) & 0xFu;
+    const bool present = kind == 2 ? v != 0xFFu : v != 0xFu;
+    // rank -> offset from pay_min (two byte tables: offsets up to 65535 are not needed, < 256)
+    const int off = use_rv ? (int)rv_lo.r[v] | ((int)rv_hi.r[v] << 8) : (int)v;
+    slots[2 * i] = present ? (uint32_t)(key_min + (int)i) : 0x80000000u;
+    slots[2 * i + 1] = present ? (uint32_t)(pay_min + off) : 0u;
+  }
+}
+
 __global__ void hq_fill_kernel(uint32_t* p, long long n, uint32_t v) {
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
     p[i] = v;
@@ -248,8 +343,18 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid
       pay[u][k] = (int)v[u];
     }
   }
+  // The thread's rows claim their slots in rounds: every pending row issues its CAS at
+  // its current slot before any result is inspected, so the U atomics of a thread are in
+  // flight together (a row-after-row loop waited one memory round trip per row: TPC-H
+  // Q3's orders table, 4.4 M keys into 16-B slots, took 0.45 ms); a row that lost its
+  // slot to another key moves on to the next slot in the following round.
+  const uint32_t lmask = b.direct ? 0xFFFFFFFFu : b.mask;
+  uint32_t pos[BUILD_U];
+  bool pend[BUILD_U];
 #pragma unroll
   for (int u = 0; u < BUILD_U; ++u) {
+    pend[u] = false;
+    pos[u] = 0;
     if (!pass[u]) continue;
     if (b.verify) {  // the rows the count pass would have summarised
       ++qual;
@@ -265,29 +370,43 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid
       continue;
     }
     const int key = (int)kv[u];
-    uint32_t pos = b.direct ? (uint32_t)(key - b.dmin) : ((uint32_t)key * 0x9E3779B1u) >> shift;
-    if (b.direct && pos >= b.mask) {  // cannot happen: the range comes from the count pass
+    pos[u] = b.direct ? (uint32_t)(key - b.dmin) : ((uint32_t)key * 0x9E3779B1u) >> shift;
+    if (b.direct && pos[u] >= b.mask) {  // cannot happen: the range comes from the count pass
       fault |= HQF_HT_FULL;
       continue;
     }
-    uint32_t i = 0;
-    for (; i <= b.mask; ++i) {
-      uint32_t* slot = b.slots + (size_t)pos * b.words;
-      const int old = atomicCAS((int*)slot, INT_MIN, key);
-      if (old == INT_MIN) {
+    pend[u] = true;
+  }
+  for (uint32_t round = 0;; ++round) {
+    bool any = false;
+#pragma unroll
+    for (int u = 0; u < BUILD_U; ++u) any = any || pend[u];
+    if (!any) break;
+    if (round > b.mask || (b.direct && round > 0)) {  // every slot visited: full
+      fault |= HQF_HT_FULL;
+      break;
+    }
+    int old[BUILD_U];
+#pragma unroll
+    for (int u = 0; u < BUILD_U; ++u)
+      old[u] = pend[u] ? atomicCAS((int*)(b.slots + (size_t)pos[u] * b.words), INT_MIN, (int)kv[u]) : 0;
+#pragma unroll
+    for (int u = 0; u < BUILD_U; ++u) {
+      if (!pend[u]) continue;
+      if (old[u] == INT_MIN) {
+        uint32_t* slot = b.slots + (size_t)pos[u] * b.words;
 #pragma unroll
         for (int k = 0; k < HQ_MAX_PAYLOAD; ++k)
           if (k < b.npay) slot[1 + k] = (uint32_t)pay[u][k];
         ++inserted;
-        break;
-      }
-      if (!b.composite && (old == key || b.direct)) {
+        pend[u] = false;
+      } else if (!b.composite && (old[u] == (int)kv[u] || b.direct)) {
         fault |= HQF_DUP_KEY;  // join keys must be unique (R6)
-        break;
+        pend[u] = false;
+      } else {
+        pos[u] = (pos[u] + 1) & lmask;
       }
-      pos = (pos + 1) & b.mask;
     }
-    if (i > b.mask) fault |= HQF_HT_FULL;
   }
   if (fault) atomicOr(b.err, fault);
   if (b.verify) {  // the number of qualifying rows must equal the cached count
@@ -331,6 +450,37 @@ bool stats_cache_on() {
   return !(e && e[0] == '0');
 }
 
+}  // namespace
+
+// compact form of a direct table: 1 = bitmap (no payload), 2 = byte per key (payload 0
+// spans < 255 values), 3 = nibble per key (< 15 values), 0 = none
+int hq_compact_kind(int npayload, int pay_min, int pay_max) {
+  if (npayload == 0) return 1;
+  if (npayload != 1 || pay_min > pay_max) return 0;
+  const long long pr = (long long)pay_max - pay_min;
+  return pr < 15 ? 3 : (pr < 255 ? 2 : 0);
+}
+long long hq_compact_words(int kind, long long range) {
+  return kind == 1 ? (range + 31) / 32 : (kind == 3 ? (range + 7) / 8 : (range + 3) / 4);
+}
+// rank LUT of a byte map over a sparse payload set (value - pay_min -> rank, 0xFF
+// absent); returns 1 when the map is rank-coded (the set is known and sparse)
+int hq_rank_lut(const hq_hash_meta& m, unsigned char* lut) {
+  for (int i = 0; i < 256; ++i) lut[i] = 0xFF;
+  int n = 0;
+  const int span = m.pay_max - m.pay_min + 1;
+  if (span < 1 || span > 255) return 0;
+  for (int d = 0; d < span; ++d) {
+    const uint32_t v = (uint32_t)(m.pay_min + d) & 255u;
+    if ((m.pay_set[v >> 6] >> (v & 63)) & 1ull) lut[d] = (unsigned char)n++;
+  }
+  const int crank = (n > 0 && n < span && !getenv("HQ_NO_RANKMAP")) ? 1 : 0;
+  if (!crank)
+    for (int d = 0; d < span; ++d) lut[d] = (unsigned char)d;
+  return crank;
+}
+
+namespace {
 void to_kpred(const hq_pred& in, KBuildPred& out, int ncols) {
   if (in.reg < 0 || in.reg >= ncols) HQ_THROW(HQ_ERR_ARG, "build predicate column out of range");
   out.col = (int16_t)in.reg;
@@ -470,8 +620,14 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   if (cap > (1LL << 31)) HQ_THROW(HQ_ERR_UNSUPPORTED, "build: hash table too large");
   int log2 = 0;
   while ((1LL << log2) < cap) ++log2;
-  h->owned = DevBuf(ctx, (size_t)cap * words * 4);
-  h->slots = h->owned.as<uint32_t>();
+  // compact-only direct table (hq_build_direct_compact_kernel): the compact form is
+  // derived from the statistics alone, so no slot array is written at all
+  const int ckind = direct && bs.counted ? hq_compact_kind(d->npayload, bs.st.pmin, bs.st.pmax) : 0;
+  const bool conly = ckind != 0 && !b.composite && !getenv("HQ_BUILD_SLOTS");
+  if (!conly) {
+    h->owned = DevBuf(ctx, (size_t)cap * words * 4);
+    h->slots = h->owned.as<uint32_t>();
+  }
   h->log2cap = log2;
   h->meta.capacity = cap;
   h->meta.slot_words = words;
@@ -482,6 +638,26 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   h->meta.layout = direct ? HQ_HT_DIRECT : HQ_HT_LINEAR;
   h->meta.key_min = kmin;
   h->meta.key_max = range > 0 ? (int32_t)(kmin + range - 1) : (int32_t)kmin - 1;  // empty range when unknown
+  h->stats_key = bs.stats_key;
+  if (conly) {
+    const long long cwords = hq_compact_words(ckind, range);
+    h->compact = DevBuf(ctx, (size_t)cwords * 4 + 16);
+    HQ_CUDA(cudaMemsetAsync(h->compact.p, ckind == 1 ? 0x00 : 0xFF, (size_t)cwords * 4 + 16, ctx->stream));
+    CLut lut{};
+    const int crank = ckind == 2 ? hq_rank_lut(h->meta, lut.r) : 0;
+    b.dmin = (int32_t)kmin;
+    if (b.n > 0) {
+      ctx->launches++;
+      hq_build_direct_compact_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b, ckind, h->compact.as<uint32_t>(), range,
+                                                                               h->meta.pay_min, crank, lut);
+    }
+    HQ_CUDA(cudaGetLastError());
+    h->ckind = ckind;
+    h->crank = crank;
+    h->cbytes = cwords * 4;
+    h->compact_only = true;
+    return;
+  }
   const int64_t nw = cap * words;
   const int fgrid = (int)std::max<int64_t>(1, std::min<int64_t>((nw + 255) / 256, (int64_t)ctx->num_sms * 8));
   ctx->launches++;
@@ -494,7 +670,6 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   b.direct = direct;
   b.dmin = (int32_t)kmin;
   b.count_inserts = bs.counted ? 0 : 1;
-  h->stats_key = bs.stats_key;
   if (b.n > 0) { ctx->launches++; hq_build_hash_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b); }
   HQ_CUDA(cudaGetLastError());
   hq_build_compact(ctx, h);
@@ -671,14 +846,9 @@ void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
   }
   if (h->meta.layout != HQ_HT_DIRECT) return;
   const long long range = h->meta.capacity;
-  int kind = 0;
-  if (h->meta.npayload == 0) kind = 1;
-  else if (h->meta.npayload == 1 && h->meta.pay_min <= h->meta.pay_max) {
-    const long long pr = (long long)h->meta.pay_max - h->meta.pay_min;
-    kind = pr < 15 ? 3 : (pr < 255 ? 2 : 0);
-  }
+  const int kind = h->meta.composite ? 0 : hq_compact_kind(h->meta.npayload, h->meta.pay_min, h->meta.pay_max);
   if (!kind) return;
-  const long long words = kind == 1 ? (range + 31) / 32 : (kind == 3 ? (range + 7) / 8 : (range + 3) / 4);
+  const long long words = hq_compact_words(kind, range);
   h->compact = DevBuf(ctx, (size_t)words * 4 + 16);
   const int grid = (int)std::max<long long>(1, std::min<long long>((range + 255) / 256, (long long)ctx->num_sms * 8));
   ctx->launches++;
@@ -686,13 +856,7 @@ void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
   else if (kind == 2) {
     // a sparse payload-value set (SSB Q3.1's five ASIA nations among codes 8..24): rank-code
     RankLut lut{};
-    int n = 0, span = h->meta.pay_max - h->meta.pay_min + 1;
-    for (int d = 0; d < span; ++d) {
-      const uint32_t v = (uint32_t)(h->meta.pay_min + d) & 255u;
-      lut.r[d] = (unsigned char)0xFF;
-      if ((h->meta.pay_set[v >> 6] >> (v & 63)) & 1ull) lut.r[d] = (unsigned char)n++;
-    }
-    h->crank = (n > 0 && n < span && span <= 255 && !getenv("HQ_NO_RANKMAP")) ? 1 : 0;
+    h->crank = hq_rank_lut(h->meta, lut.r);
     hq_compact_u8_kernel<<<grid, 256, 0, ctx->stream>>>(h->slots, range, h->meta.pay_min, h->compact.as<uint32_t>(),
                                                         h->crank, lut);
   }
@@ -700,6 +864,33 @@ void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
   HQ_CUDA(cudaGetLastError());
   h->ckind = kind;
   h->cbytes = words * 4;
+}
+
+const uint32_t* hq_hash_slots(hq_ctx* ctx, hq_hash* h) {
+  if (h->slots || !h->compact_only) return h->slots;
+  const long long range = h->meta.capacity;
+  const int words = h->meta.slot_words;
+  h->owned = DevBuf(ctx, (size_t)range * words * 4 + 16);
+  CLut lo{}, hi{};
+  int use_rv = 0;
+  if (h->ckind == 2 && h->crank) {  // rank -> offset from pay_min
+    unsigned char lut[256];
+    hq_rank_lut(h->meta, lut);
+    for (int d = 0; d < 255; ++d)
+      if (lut[d] != 0xFF) {
+        lo.r[lut[d]] = (unsigned char)(d & 255);
+        hi.r[lut[d]] = (unsigned char)(d >> 8);
+      }
+    use_rv = 1;
+  }
+  const int grid = (int)std::max<long long>(1, std::min<long long>((range + 255) / 256, (long long)ctx->num_sms * 8));
+  ctx->launches++;
+  hq_slots_from_compact_kernel<<<grid, 256, 0, ctx->stream>>>((const uint32_t*)h->compact_ptr(), h->ckind, range,
+                                                                (int)h->meta.key_min, h->meta.pay_min, use_rv, lo, hi,
+                                                                h->owned.as<uint32_t>());
+  HQ_CUDA(cudaGetLastError());
+  h->slots = h->owned.as<uint32_t>();
+  return h->slots;
 }
 
 // Sync and report build faults (HQ_ERR_DUP_KEY etc.).

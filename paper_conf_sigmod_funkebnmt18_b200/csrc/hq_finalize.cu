@@ -334,43 +334,129 @@ __device__ void tk_sort(const KCompact& k, const KSort& s, long long* idx, unsig
     }
   }
 }
-__global__ void __launch_bounds__(1024) hq_topk1_kernel(const __grid_constant__ KTopK q) {
-  __shared__ long long idx[SORT_CHUNK];
-  __shared__ unsigned long long pk[SORT_CHUNK];
-  __shared__ unsigned long long qual_s, live_s;
+// primary sort key of a live entry: order-preserving image of the first ORDER BY column
+// (or the first group key), ascending = the result order
+__device__ __forceinline__ unsigned long long tk_pk(const KCompact& k, const KSort& s, long long g) {
+  if (s.norder == 0 && s.nkeys == 0) return 0;
+  const int c0 = s.norder > 0 ? s.ocol[0] : 0;
+  const long long v = tk_col(k, g, c0);
+  unsigned long long t = s.isf[c0] ? (v < 0 ? ~(unsigned long long)v : (unsigned long long)v ^ 0x8000000000000000ull)
+                                   : (unsigned long long)v ^ 0x8000000000000000ull;
+  return (s.norder > 0 && s.odesc[0]) ? ~t : t;
+}
+// radix-select state: [0] min pk, [1] max pk, [2] shift, [3] selected bin, [4] candidates, [5] overflow
+constexpr int TK_BINS = 4096;
+constexpr int TK_CAND = 16384;
+// pass 1: min / max primary key, qualifying rows, live groups
+__global__ void __launch_bounds__(256) hq_topk_minmax_kernel(const __grid_constant__ KTopK q, unsigned long long* sel) {
   const KCompact& k = q.k;
-  if (threadIdx.x == 0) { qual_s = 0; live_s = 0; }
-  // chunk of SORT_CHUNK - keep entries; the block's running top-k occupies idx[0..keep)
-  const long long chunk = SORT_CHUNK - q.keep;
-  const long long per = (k.ngroups + gridDim.x - 1) / gridDim.x;
-  const long long g0 = (long long)blockIdx.x * per, g1 = g0 + per < k.ngroups ? g0 + per : k.ngroups;
-  for (int i = threadIdx.x; i < q.keep; i += blockDim.x) idx[i] = -1;
-  unsigned long long qsum = 0, lsum = 0;
-  for (long long c0 = g0; c0 < g1; c0 += chunk) {
-    __syncthreads();
-    for (int i = threadIdx.x; i < (int)chunk; i += blockDim.x) {
-      const long long g = c0 + i;
-      const bool live = g < g1 && tk_live(k, g);
-      if (live) {
-        qsum += (unsigned long long)tk_entry(k, g)[0];
-        ++lsum;
-      }
-      idx[q.keep + i] = live ? g : -1;
-    }
-    __syncthreads();
-    tk_sort(k, q.s, idx, pk, SORT_CHUNK);
+  unsigned long long mn = ~0ull, mx = 0, qs = 0, ls = 0;
+  for (long long g = blockIdx.x * (long long)blockDim.x + threadIdx.x; g < k.ngroups; g += (long long)gridDim.x * blockDim.x) {
+    if (!tk_live(k, g)) continue;
+    const unsigned long long pk = tk_pk(k, q.s, g);
+    mn = pk < mn ? pk : mn;
+    mx = pk > mx ? pk : mx;
+    qs += (unsigned long long)tk_entry(k, g)[0];
+    ++ls;
   }
-  __syncthreads();
-  for (int i = threadIdx.x; i < q.keep; i += blockDim.x) q.cand[(long long)blockIdx.x * q.keep + i] = (int)idx[i];
-  if (qsum) atomicAdd(&qual_s, qsum);
-  if (lsum) atomicAdd(&live_s, lsum);
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    if (qual_s) atomicAdd(q.stats + 1, qual_s);
-    if (live_s) atomicAdd(q.stats + 3, live_s);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long a = __shfl_xor_sync(0xffffffffu, mn, o), b = __shfl_xor_sync(0xffffffffu, mx, o);
+    mn = a < mn ? a : mn;
+    mx = b > mx ? b : mx;
+    qs += __shfl_xor_sync(0xffffffffu, qs, o);
+    ls += __shfl_xor_sync(0xffffffffu, ls, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (ls) {
+      atomicMin(sel + 0, mn);
+      atomicMax(sel + 1, mx);
+      atomicAdd(q.stats + 1, qs);
+      atomicAdd(q.stats + 3, ls);
+    }
   }
 }
-__global__ void __launch_bounds__(1024) hq_topk2_kernel(const __grid_constant__ KTopK q, int ncand) {
+__device__ __forceinline__ int tk_bin(unsigned long long pk, const unsigned long long* sel) {
+  return (int)((pk - sel[0]) >> sel[2]);
+}
+// pass 2: histogram of the primary keys over TK_BINS bins spanning [min, max]
+__global__ void __launch_bounds__(256) hq_topk_hist_kernel(const __grid_constant__ KTopK q, const unsigned long long* sel,
+                                                           unsigned* hist) {
+  __shared__ unsigned h[TK_BINS];
+  for (int i = threadIdx.x; i < TK_BINS; i += blockDim.x) h[i] = 0;
+  __syncthreads();
+  const KCompact& k = q.k;
+  if (sel[0] <= sel[1])
+    for (long long g = blockIdx.x * (long long)blockDim.x + threadIdx.x; g < k.ngroups; g += (long long)gridDim.x * blockDim.x)
+      if (tk_live(k, g)) atomicAdd(&h[tk_bin(tk_pk(k, q.s, g), sel)], 1u);
+  __syncthreads();
+  for (int i = threadIdx.x; i < TK_BINS; i += blockDim.x)
+    if (h[i]) atomicAdd(hist + i, h[i]);
+}
+// bins of 2^shift keys: TK_BINS bins cover [min, max]
+__global__ void hq_topk_shift_kernel(unsigned long long* sel) {
+  const unsigned long long span = sel[0] <= sel[1] ? sel[1] - sel[0] : 0;
+  int sh = 0;
+  while (sh < 63 && (span >> sh) >= (unsigned long long)TK_BINS) ++sh;
+  sel[2] = (unsigned long long)sh;
+}
+// pass 3 (one block): the bin holding the k-th smallest key; every entry of a lower bin
+// is in the top k, the k-th one's bin supplies the rest
+__global__ void hq_topk_select_kernel(const unsigned* hist, int keep, unsigned long long* sel) {
+  __shared__ unsigned part[32];
+  const int tid = threadIdx.x;  // 1024 threads x 4 bins
+  unsigned c[4], t = 0;
+  for (int i = 0; i < 4; ++i) { c[i] = hist[tid * 4 + i]; t += c[i]; }
+  unsigned incl = t;
+  const int lane = tid & 31, w = tid >> 5;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned x = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += x;
+  }
+  if (lane == 31) part[w] = incl;
+  __syncthreads();
+  if (w == 0) {
+    unsigned v = part[lane], iv = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned x = __shfl_up_sync(0xffffffffu, iv, o);
+      if (lane >= o) iv += x;
+    }
+    part[lane] = iv - v;
+  }
+  __syncthreads();
+  unsigned before = part[w] + incl - t;
+  for (int i = 0; i < 4; ++i) {
+    if (before < (unsigned)keep && before + c[i] >= (unsigned)keep) sel[3] = (unsigned long long)(tid * 4 + i);
+    before += c[i];
+  }
+  if (tid == blockDim.x - 1 && before < (unsigned)keep) sel[3] = TK_BINS - 1;  // fewer live groups than k: all
+}
+// pass 4: the candidates -- every live entry in the selected bin or below
+__global__ void __launch_bounds__(256) hq_topk_collect_kernel(const __grid_constant__ KTopK q, unsigned long long* sel) {
+  const KCompact& k = q.k;
+  if (sel[0] > sel[1]) return;
+  const int bstar = (int)sel[3];
+  const int lane = threadIdx.x & 31;
+  // warp-uniform trip count: one atomic per warp and round claims the warp's candidates
+  for (long long b0 = (blockIdx.x * (long long)blockDim.x + threadIdx.x) & ~31ll; b0 < k.ngroups;
+       b0 += (long long)gridDim.x * blockDim.x) {
+    const long long g = b0 + lane;
+    const bool take = g < k.ngroups && tk_live(k, g) && tk_bin(tk_pk(k, q.s, g), sel) <= bstar;
+    const unsigned bal = __ballot_sync(0xffffffffu, take);
+    if (!bal) continue;
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(sel + 4, (unsigned long long)__popc(bal));
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (!take) continue;
+    const unsigned long long i = base + __popc(bal & ((1u << lane) - 1u));
+    if (i < (unsigned long long)TK_CAND) q.cand[i] = (int)g;
+    else sel[5] = 1;  // overflow: the host finalizes the long way
+  }
+}
+__global__ void __launch_bounds__(1024) hq_topk2_kernel(const __grid_constant__ KTopK q, const unsigned long long* sel) {
+  const int ncand = sel[5] ? 0 : (int)(sel[4] < (unsigned long long)TK_CAND ? sel[4] : (unsigned long long)TK_CAND);
   __shared__ long long idx[SORT_CHUNK];
   __shared__ unsigned long long pk[SORT_CHUNK];
   __shared__ int err_s;
@@ -380,10 +466,14 @@ __global__ void __launch_bounds__(1024) hq_topk2_kernel(const __grid_constant__ 
   const int chunk = SORT_CHUNK - q.keep;
   for (int i = threadIdx.x; i < q.keep; i += blockDim.x) idx[i] = -1;
   for (int c0 = 0; c0 < ncand; c0 += chunk) {
+    // the smallest network that holds the running top-k and this round's candidates
+    const int m = q.keep + (ncand - c0 < chunk ? ncand - c0 : chunk);
+    int net = 32;
+    while (net < m) net <<= 1;
     __syncthreads();
-    for (int i = threadIdx.x; i < chunk; i += blockDim.x) idx[q.keep + i] = c0 + i < ncand ? q.cand[c0 + i] : -1;
+    for (int i = threadIdx.x; i < net - q.keep; i += blockDim.x) idx[q.keep + i] = c0 + i < ncand ? q.cand[c0 + i] : -1;
     __syncthreads();
-    tk_sort(k, q.s, idx, pk, SORT_CHUNK);
+    tk_sort(k, q.s, idx, pk, net);
   }
   __syncthreads();
   const int nc = k.nkeys + k.naggs;
@@ -402,6 +492,7 @@ __global__ void __launch_bounds__(1024) hq_topk2_kernel(const __grid_constant__ 
     const unsigned long long live = q.stats[3];
     q.stats[0] = live < (unsigned long long)q.keep ? live : (unsigned long long)q.keep;
     q.stats[2] = (unsigned long long)err_s;
+    q.stats[5] = sel[5];  // candidate overflow
     int e_ = *q.pipe_err;
     for (int i = 0; i < q.nhash; ++i) e_ |= *(volatile const int*)q.hash_err[i];
     q.stats[4] = (unsigned long long)(unsigned)e_;
@@ -716,19 +807,29 @@ static bool finalize_topk(hq_ctx* ctx, hq_result* r) {
   HQ_CUDA(cudaMemsetAsync(pack.p, 0, 64, ctx->stream));
   q.stats = pack.as<unsigned long long>();
   for (int c = 0; c < nc; ++c) q.res[c] = (long long*)(pack.as<char>() + 64 + (size_t)c * rcap * 8);
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)ctx->num_sms * 2, (r->ngroups + 4095) / 4096));
-  DevBuf cand(ctx, (size_t)grid * q.keep * 4 + 16);
+  DevBuf cand(ctx, (size_t)TK_CAND * 4 + 16);
   q.cand = cand.as<int>();
+  // selection state + histogram: [0] min (all ones) [1] max [2] shift [3] bin [4] count [5] overflow, then the bins
+  DevBuf selb(ctx, 64 + (size_t)TK_BINS * 4);
+  unsigned long long* sel = selb.as<unsigned long long>();
+  HQ_CUDA(cudaMemsetAsync(selb.p, 0, 64 + (size_t)TK_BINS * 4, ctx->stream));
+  HQ_CUDA(cudaMemsetAsync(selb.p, 0xFF, 8, ctx->stream));
   q.pipe_err = (const int*)(r->dstate.as<char>() + 8);
   for (hq_hash* hh : r->hashes)
     if (hh->dstate.p && !hh->checked && q.nhash < 8) q.hash_err[q.nhash++] = hh->dstate.as<int>();
-  ctx->launches += 2;
-  hq_topk1_kernel<<<grid, 1024, 0, ctx->stream>>>(q);
-  hq_topk2_kernel<<<1, 1024, 0, ctx->stream>>>(q, grid * q.keep);
+  const int grid = grid_for(ctx, r->ngroups);
+  ctx->launches += 6;
+  hq_topk_minmax_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel);
+  hq_topk_shift_kernel<<<1, 1, 0, ctx->stream>>>(sel);
+  hq_topk_hist_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel, (unsigned*)(selb.as<char>() + 64));
+  hq_topk_select_kernel<<<1, 1024, 0, ctx->stream>>>((const unsigned*)(selb.as<char>() + 64), q.keep, sel);
+  hq_topk_collect_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel);
+  hq_topk2_kernel<<<1, 1024, 0, ctx->stream>>>(q, sel);
   HQ_CUDA(cudaGetLastError());
   char* h = (char*)pinned_staging(ctx, 64 + body);
   HQ_CUDA(cudaMemcpyAsync(h, pack.p, 64 + body, cudaMemcpyDeviceToHost, ctx->stream));
   hq_sync(ctx, "a top-k finalize");
+  if (((const unsigned long long*)h)[5]) return false;  // the k-th key's bin held too many ties
   if (!decode_small(r, h, rcap, nc)) return false;
   r->rescol.assign((size_t)nc, nullptr);
   for (int c = 0; c < nc; ++c) r->rescol[c] = pack.as<char>() + 64 + (size_t)c * rcap * 8;
@@ -792,7 +893,7 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered) {
       !getenv("HQ_NO_TOPK")) {
     if (finalize_topk(ctx, r)) return;
     hq_check_result_faults(ctx, r);  // throws, or re-runs the pipeline with a larger group table
-    if (finalize_topk(ctx, r)) return;
+    if (finalize_topk(ctx, r)) return;  // (else: too many ties at the k-th key -- the full sort below)
   }
   hq_check_result_faults(ctx, r);
   const hq_plan& P = r->plan;

@@ -224,12 +224,22 @@ struct hq_hash : RefObj {
   DevBuf compact;
   int ckind = 0;
   int crank = 0;  // ckind 2 holds the rank of payload 0 in meta.pay_set instead of payload - pay_min
+  // built straight into the compact form (no slot array until a consumer asks for it:
+  // hq_hash_slots); compact_borrow = an imported compact form (not owned)
+  bool compact_only = false;
+  void* compact_borrow = nullptr;
+  const void* compact_ptr() const { return compact.p ? compact.p : compact_borrow; }
   int64_t cbytes = 0;
   // linear tables: exact bitmap over [key_min, key_max] (prefilter before the slots)
   DevBuf prefilter;
   int64_t pf_words = 0;
 };
 void hq_build_compact(hq_ctx* ctx, hq_hash* h);  // derive hq_hash::compact from the slots
+int hq_compact_kind(int npayload, int pay_min, int pay_max);
+long long hq_compact_words(int kind, long long range);
+int hq_rank_lut(const hq_hash_meta& m, unsigned char* lut);
+// the slot array of a compact-only table, derived on first use (hq_build.cu)
+const uint32_t* hq_hash_slots(hq_ctx* ctx, hq_hash* h);
 
 // ------------------------------------------------- device plan (kernel param)
 namespace hqk {
@@ -365,6 +375,12 @@ struct KPlan {
   // generated kernels: copy the tile's columns into registers and release the
   // stage before the operators run (long-latency probes do not hold the ring)
   uint8_t early_release;
+  // generated A3 with deferred write-out: a tile's rows are staged in shared memory
+  // (two buffers of a3_buf bytes at off_agg, column j at a3_col[j]) and written to
+  // global memory during the next tile, when its atomicAdd has returned
+  uint8_t a3stage;
+  uint32_t a3_buf;
+  uint32_t a3_col[HQ_MAX_OUT];
   // multi-pass execution (HQ_EXEC_MULTIPASS, hq_multipass.cu): 1 = count kernel
   // (relational primitives -> one flag per row), 2 = write kernel (rows whose
   // flag is set; projections / aggregation inputs written at the prefix-sum

@@ -134,7 +134,7 @@ struct Gen {
     // when they span 8 or 16 bytes (stage columns are 16-B aligned)
     const int vb = compacted_R ? 0 : (int)c.width * kp.R;
     const char* vt = vb == 16 ? (c.width == 4 ? "int4" : "longlong2") : (vb == 8 ? (c.width == 4 ? "int2" : "long long") : nullptr);
-    o << "      " << ctype(c.width) << " " << var(reg) << "[R];\n";
+    dvar(ctype(c.width), var(reg));
     if (vt && c.width >= 4) {
       vec_loaded.insert(reg);
       o << "      { const " << vt << " q_ = *(const " << vt << "*)((const " << ctype(c.width) << "*)(st + " << c.soff << "u) + row0);";
@@ -153,6 +153,20 @@ struct Gen {
   // block stays structured (nested ifs, closed in generate()) so that the
   // compiler reconverges the warp at its end -- with break-style exits a warp
   // could stay split for the rest of the kernel and run at half speed
+  // software pipelining (generate(): two tiles per warp in flight): the arrays the
+  // first phase of a tile defines are declared once at function scope (`decl`) and
+  // renamed per tile parity; otherwise declarations stay inline
+  std::ostringstream* decl = nullptr;
+  std::vector<std::string> hoisted;
+  void dvar(const std::string& ty, const std::string& name, bool zero = false) {
+    if (decl) {
+      *decl << "  " << ty << " " << name << "[R];\n";
+      hoisted.push_back(name);
+      if (zero) o << "#pragma unroll\n      for (int r = 0; r < R; ++r) " << name << "[r] = 0;\n";
+    } else {
+      o << "      " << ty << " " << name << (zero ? "[R] = {};\n" : "[R];\n");
+    }
+  }
   int open = 0;
   void early_exit() {
     sync_mask();  // mask must be right on the path that skips the block
@@ -167,7 +181,7 @@ struct Gen {
   bool al_declared = false;
   void begin_al() {
     if (!al_declared) {
-      o << "      bool al_[R];\n";
+      dvar("bool", "al_");
       al_declared = true;
       live = LIVE_MASK;
     }
@@ -249,7 +263,7 @@ struct Gen {
       bitmaps << "};\n";
     }
     for (int k = 0; k < npay; ++k) {
-      o << "      int " << var(pr.dst[k]) << (outer ? "[R] = {};\n" : "[R];\n");
+      dvar("int", var(pr.dst[k]), outer);
       if (k == 0 && pr.pay_min <= pr.pay_max)
         known[pr.dst[0]] = {outer ? std::min(pr.pay_min, 0) : pr.pay_min, outer ? std::max(pr.pay_max, 0) : pr.pay_max};
       loaded.insert(pr.dst[k]);
@@ -265,7 +279,9 @@ struct Gen {
     const std::string key = val(pr.key_reg);
     const std::string D = pv(i, "d_"), M = pv(i, "m_");
     sync_al();
-    o << "      u32 " << D << "[R]; bool " << M << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) {";
+    dvar("u32", D);
+    dvar("bool", M);
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) {";
     if (width(pr.key_reg) <= 4)  // int32 keys: (k - min) mod 2^32 < range  <=>  min <= k < min + range
       o << " const u32 d_ = (u32)(int)" << key << " - " << (uint32_t)pr.dmin << "u; const bool in_ = d_ < " << pr.mask << "u;";
     else
@@ -278,7 +294,8 @@ struct Gen {
     const int ak = access(pr);
     if (ak == AK_DIRECT) {
       const int W = pr.words;
-      o << "      int4 " << V << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) if (" << M << "[r]) ";
+      dvar("int4", V);
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (" << M << "[r]) ";
       if (W == 1) o << V << "[r].x = __ldg((const int*)p.ht[" << i << "] + " << D << "[r]);\n";
       else if (W == 2)
         o << "{ const int2 q_ = __ldg((const int2*)p.ht[" << i << "] + " << D << "[r]); " << V << "[r].x = q_.x; " << V
@@ -298,8 +315,8 @@ struct Gen {
     else
       ld = pr.ckind == 1 ? "__ldg((const u32*)p.ctab[" + std::to_string(i) + "] + " + idx + ")"
                          : "(u32)__ldg((const unsigned char*)p.ctab[" + std::to_string(i) + "] + " + idx + ")";
-    o << "      u32 " << V << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) if (" << M << "[r]) " << V
-      << "[r] = " << ld << ";\n";
+    dvar("u32", V);
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (" << M << "[r]) " << V << "[r] = " << ld << ";\n";
   }
   void probe_resolve(const KProbe& pr, int i) {
     const std::string D = pv(i, "d_"), M = pv(i, "m_"), V = pv(i, "v_");
@@ -383,7 +400,14 @@ struct Gen {
   }
 
   // ops [i, end): one probe batch starting at op i (see probe_addr)
-  int probe_batch(int i) {
+  // part 0: the whole batch; 1: definitions, addresses and loads (the batch is kept);
+  // 2: the kept batch's resolution (software pipelining splits a tile there)
+  std::vector<int> kept_batch;
+  int probe_batch(int i, int part = 0) {
+    if (part == 2) {
+      for (int j : kept_batch) probe_resolve(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
+      return kept_batch.back() + 1;
+    }
     const KProbe& first = kp.probes[kp.ops[i].idx];
     const int ak = access(first);
     if (ak == AK_LINEAR) {
@@ -406,6 +430,10 @@ struct Gen {
     for (int j : b) probe_defs(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
     for (int j : b) probe_addr(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
     for (int j : b) probe_load(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
+    if (part == 1) {
+      kept_batch = b;
+      return b.back() + 1;
+    }
     for (int j : b) probe_resolve(kp.probes[kp.ops[j].idx], kp.ops[j].idx);
     return b.back() + 1;
   }
@@ -420,7 +448,8 @@ struct Gen {
     std::vector<std::string> ops;
     for (int k = 0; k < c.n; ++k) ops.push_back(operand(kp.insns[c.first + k]));
     const std::string dst = var(c.dst);
-    o << "      long long " << dst << "[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) { long long a_ = 0;\n";
+    dvar("long long", dst);
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { long long a_ = 0;\n";
     for (int k = 0; k < c.n; ++k) {
       const KInsn& in = kp.insns[c.first + k];
       const std::string& x = ops[k];
@@ -523,6 +552,24 @@ std::string lcol_tables(const KPlan& kp) {
     if (kp.lcol[a]) fn[kp.lcol[a]] = kp.agg_fn[a];
   for (size_t c = 0; c < fn.size(); ++c) s << (c ? ", " : "") << fn[c];
   s << "};\n";
+  return s.str();
+}
+
+// staged A3: copy a tile's rows [0, n) from its staging buffer to base + i (all
+// consumer threads, coalesced per column); positions past the capacity set F_CAPACITY
+std::string a3_flush_fn(const KPlan& kp) {
+  if (!kp.a3stage) return "";
+  std::ostringstream s;
+  s << "#define A3BUF " << kp.a3_buf << "u\n"
+    << "__device__ __forceinline__ void a3_flush(const JParams& p, long long base, int n, const char* sb) {\n"
+    << "  for (int i = threadIdx.x; i < n; i += NW * 32) {\n"
+    << "    const long long pos = base + i;\n"
+    << "    if (pos >= p.capacity) { atomicOr(p.err, 1); continue; }\n";
+  for (int j = 0; j < kp.nout; ++j) {
+    const char* ty = kp.out_width[j] == 1 ? "signed char" : (kp.out_width[j] == 4 ? "int" : "long long");
+    s << "    ((" << ty << "*)p.out[" << j << "])[pos] = ((const " << ty << "*)(sb + " << kp.a3_col[j] << "u))[i];\n";
+  }
+  s << "  }\n}\n";
   return s.str();
 }
 
@@ -648,186 +695,9 @@ std::string generate(const KPlan& kp) {
   const bool we = kp.resolution == HQ_RES_WE;
   const int sk = kp.sink == HQ_SINK_MATERIALISE ? 2 : (kp.nkeys == 0 ? 0 : 1);
   const int mp = kp.mp_pass;  // multi-pass: 1 = count kernel, 2 = write kernel (hq_multipass.cu)
-  // ---------------------------------------------------------------- kernel
-  o << "extern \"C\" __global__ void __launch_bounds__((NW + 1) * 32, 1) hq_jit_kernel(const __grid_constant__ JParams p) {\n"
-    << "  extern __shared__ __align__(128) char smem[];\n"
-    << "  u64* full = (u64*)smem; u64* empty = full + 10;\n"
-    << "  u64* s_base = (u64*)(empty + 10); int* s_wtot = (int*)(s_base + 32); i64* s_red = (i64*)(s_wtot + 32);\n"
-    << "  char* sagg = smem + OFF_AGG; char* stages = smem + OFF_STAGE;\n"
-    << "  const u32 sm0_ = smem_u32(smem); (void)sm0_;\n"
-    << "  (void)s_base; (void)s_wtot; (void)s_red; (void)sagg;\n"
-    << "  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n"
-    << "  const long long first_tile = p.row_begin / T;\n"
-    << "  const long long ntiles = p.row_end > p.row_begin ? (p.row_end + T - 1) / T - first_tile : 0;\n"
-    << "  const long long nj = ntiles > blockIdx.x ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;\n"
-    << "  const long long tstep = (long long)gridDim.x * T;\n"
-    << "  if (threadIdx.x == 0) { for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], NW); } fence_mbar_init(); }\n";
-  if (prof) o << "  long long pt0_ = 0; if (threadIdx.x == 0) asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(pt0_));\n"
-              << "  long long pw_ = 0, pl0_ = clock64(); int pdv_ = 0;\n";
-  // smem table init
-  if (sk == 1 && kp.smode == SM_LANE) {
-    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * NACC * NW * 32; i += NW * 32) {"
-      << " const int a_ = (int)((i / (NW * 32)) % NACC); t_[i] = a_ == 0 ? 0 : agg_identity(ACC_FN[a_]); } }\n";
-  } else if (sk == 1 && kp.smode == SM_DENSE) {
-    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * LVWORDS * SCOPIES; i += NW * 32) {"
-      << " const int c_ = (int)(i % LVWORDS); t_[i] = c_ == 0 ? 0 : agg_identity(LFN[c_]); } }\n";
-  } else if (sk == 1 && kp.smode == SM_HASH) {
-    o << "  if (warp < NW) { u64* k_ = (u64*)sagg; i64* e_ = (i64*)sagg + SMEM_CAP;\n"
-      << "    for (u32 i = threadIdx.x; i < SMEM_CAP; i += NW * 32) k_[i] = HQ_EMPTY_KEY;\n"
-      << "    for (u32 i = threadIdx.x; i < SMEM_CAP * LVWORDS; i += NW * 32) { const int c_ = (int)(i % LVWORDS); e_[i] = c_ == 0 ? 0 : agg_identity(LFN[c_]); } }\n";
-  }
-  // staged compact probe tables: one cooperative 16-B copy per CTA
-  for (int i = 0; i < MAX_PROBES; ++i) {
-    const KProbe& pr = kp.probes[i];
-    if (!pr.smem_off) continue;
-    o << "  { const uint4* src_ = (const uint4*)p.ctab[" << i << "]; uint4* dst_ = (uint4*)(smem + " << pr.smem_off << "u);\n"
-      << "    for (u32 x = threadIdx.x; x < " << (pr.cbytes + 15) / 16 << "u; x += blockDim.x) dst_[x] = __ldg(src_ + x); }\n";
-  }
-  o << "  __syncthreads();\n";
-  // producer
-  o << "  if (warp == NW) {\n    if (lane == 0) {\n      const u64 pol = policy_evict_first();\n"
-    << "      int s = 0; u32 ph = 0; long long t0 = (first_tile + blockIdx.x) * (long long)T;\n"
-    << "      for (long long j = 0; j < nj; ++j, t0 += tstep) {\n"
-    << "        " << (prof ? "{ const long long c_ = clock64(); if (j >= S) mbar_wait(&empty[s], ph ^ 1u); pw_ += clock64() - c_; }" : "if (j >= S) mbar_wait(&empty[s], ph ^ 1u);") << "\n"
-    << "        char* st = stages + (size_t)s * STAGE_STRIDE;\n"
-    << "        if (t0 >= p.row_begin && t0 + T <= p.row_end) {\n          mbar_expect_tx(&full[s], STAGE_BYTES);\n";
-  for (int k = 0; k < kp.ncols; ++k)
-    o << "          tma_load_1d(st + " << kp.cols[k].soff << "u, p.col[" << k << "] + t0 * " << kp.cols[k].width << ", "
-      << kp.tile_rows * kp.cols[k].width << "u, &full[s], pol);\n";
-  o << "        } else mbar_arrive(&full[s]);\n        if (++s == S) { s = 0; ph ^= 1u; }\n      }\n";
-  if (prof) o << "      p.prof[blockIdx.x * 128 + 3] = pw_; p.prof[blockIdx.x * 128 + 4] = clock64() - pl0_;\n";
-  o << "    }\n    return;\n  }\n";
-  // consumer state
-  o << "  const int row0 = warp * 32 * R + lane * R;  // the lane's rows: row0 .. row0 + R - 1\n";
-  if (sk == 0 && !c2 && !we) {
-    o << "  u64 scount_ = 0;\n";
-    for (int a = 0; a < kp.naggs; ++a) o << "  i64 sacc" << a << " = agg_identity(AGG_FN[" << a << "]);\n";
-  }
-  // HQ_JIT_WAIT=sleep: the older poll + nanosleep loop (A/B)
-  const char* wm = getenv("HQ_JIT_WAIT");
-  const std::string cwait = (wm && std::string(wm) == "sleep") ? "mbar_wait_sleep(&full[s], ph);" : "mbar_wait_suspend_a(sm0_ + 8u * (u32)s, ph);";
-  o << "  int s = 0; u32 ph = 0; long long t0 = (first_tile + blockIdx.x) * (long long)T;\n"
-    << "  const int njc = (int)nj;\n"
-    // only a CTA's first and last tile can be ragged (partition boundaries): decided once
-    << "  const long long tl_ = t0 + (nj - 1) * tstep;\n"
-    << "  const int rj0_ = (nj > 0 && (t0 < p.row_begin || t0 + T > p.row_end)) ? 0 : -1;\n"
-    << "  const int rj1_ = (nj > 0 && (tl_ < p.row_begin || tl_ + T > p.row_end)) ? njc - 1 : -1;\n"
-    << "  for (int j = 0; j < njc; ++j, t0 += tstep) {\n"
-    << (prof ? "    { const long long c_ = clock64(); " + cwait + " pw_ += clock64() - c_; if (__activemask() != 0xffffffffu) ++pdv_; }\n" : "    " + cwait + "\n")
-    << "    const char* st = stages + (size_t)s * STAGE_STRIDE;\n"
-    << "    const long long tb_ = t0;  // tile start (temporaries t0, t1, ... shadow it below)\n"
-    << "    u32 mask = (1u << R) - 1u;\n"
-    << "    if (j == rj0_ || j == rj1_) {  // ragged head / tail tile: lanes copy their rows\n"
-    << "      const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
-    << "      const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
-    << "      mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r; if (row >= lo && row < hi) mask |= 1u << r; }\n";
-  for (int k = 0; k < kp.ncols; ++k) {
-    const char* ty = ctype(kp.cols[k].width);
-    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r; ((" << ty
-      << "*)(st + " << kp.cols[k].soff << "u))[row] = ((const " << ty << "*)p.col[" << k << "])[t0 + row]; }\n";
-  }
-  o << "      fence_proxy_async(); __syncwarp();\n    }\n";
-  if (sk == 2)  // output values leave the operator block in registers; the block scan runs after it
-    for (int j = 0; j < kp.nout; ++j) o << "    long long ov" << j << "[R];\n";
-  if (we && sk == 0 && !mp) {  // the tile's per-thread partials leave the operator block for the WE tree
-    o << "    u32 wc_ = 0u; i64 wa_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n    for (int a = 0; a < NAGGS; ++a) wa_[a] = agg_identity(AGG_FN[a]);\n";
-  } else if (we && sk == 1 && !mp) {  // the tile's live (key, values) leave it for the WE sort + segmented scan
-    o << "    u32 wm_ = 0u; u64 wk_[R]; i64 wv_[NAGGS > 0 ? NAGGS : 1][R];\n";
-  }
-  o << "    {\n";
-  if (kp.early_release) {
-    // every referenced column of the lane's rows into registers, then the stage
-    // goes back to the producer (mbarrier.arrive releases the warp's prior
-    // shared loads); the operators below run on registers only
-    for (const auto& sk2 : g.stage_k) g.use(sk2.first);
-    // The arrive must not overtake the lanes' shared loads of the stage (the
-    // producer's next TMA overwrites it): measured on B200, a bare __syncwarp +
-    // arrive let ~1 % of SSB Q4.1 runs read a refilled value.  Every lane folds
-    // its loaded registers, a ballot over the fold completes only after all
-    // loads did, and lane 0 stores the ballot before its (release) arrive.
-    const char* rf = getenv("HQ_JIT_RELFIX");  // A/B: dep (default), fence, none
-    const std::string fix = rf ? rf : "dep";
-    if (fix == "dep") {
-      // one destination register per shared load instruction: a vector load
-      // completes all its registers together, so element 0 stands for it
-      o << "    { u32 f_ = 0u";
-      for (const auto& sk2 : g.stage_k)
-        if (g.vec_loaded.count(sk2.first)) o << " ^ (u32)" << g.var(sk2.first) << "[0]";
-      o << ";\n";
-      bool scalar = false;
-      for (const auto& sk2 : g.stage_k) scalar = scalar || !g.vec_loaded.count(sk2.first);
-      if (scalar) {
-        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) f_ ^= 0u";
-        for (const auto& sk2 : g.stage_k)
-          if (!g.vec_loaded.count(sk2.first)) o << " ^ (u32)" << g.var(sk2.first) << "[r]";
-        o << ";\n";
-      }
-      o << "      const u32 b_ = __ballot_sync(HQ_FULL, f_ == 0x9E3779B9u);\n"
-        << "      if (lane == 0) { *(volatile u32*)(smem + " << (MISC_DEP) << "u + 4u * warp) = b_; mbar_arrive_a(sm0_ + 80u + 8u * (u32)s); } }\n";
-    } else if (fix == "fence") {
-      o << "    fence_proxy_async(); __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
-    } else {
-      o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
-    }
-  }
-  if (mp == 2) {  // the count kernel's flags select the rows
-    const std::string f = g.val(kp.mp_flag_reg);
-    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (!" << f << ") mask &= ~(1u << r);\n";
-  }
-  // compaction point (Gen::compact): after the first probe that passes at most
-  // half of the rows (build-side key density), aggregation sinks only, R >= 2
-  int cpt = -1;
-  if (sk != 2 && !c2 && kp.R >= 4 && kp.smode != SM_LANE)  // at R = 2 the shuffles cost more than they save (B200)
-    for (int i = 0; i < kp.nops && cpt < 0; ++i)
-      if (kp.ops[i].kind == OP_PROBE && kp.probes[kp.ops[i].idx].pass_est <= 0.5f) cpt = i;
-  if (const char* e = getenv("HQ_JIT_CPT")) cpt = (e[0] == 'o') ? -1 : (sk != 2 ? atoi(e) : -1);
-  if (mp) cpt = -1;
-  g.begin_al();
-  for (int i = 0; i < kp.nops;) {
-    if (cpt >= 0 && !g.compacted_R && i > cpt) g.compact(i);
-    if (kp.op_skip[i]) { ++i; continue; }  // not executed in this pass
-    const KOp op = kp.ops[i];
-    if (op.kind == OP_PROBE) { i = g.probe_batch(i); continue; }
-    if (op.kind == OP_FILTER) g.filter(kp.preds[op.idx], op.idx);
-    else g.compute(kp.comps[op.idx]);
-    ++i;
-  }
-  if (cpt >= 0 && !g.compacted_R) g.compact(kp.nops);
-  g.sync_mask();  // the sinks, the block scan and the count kernel's flags read mask
-  if (mp == 1) {
-    // count kernel: the flags are written below, after the early-exit blocks
-    // close -- every row of the range gets its flag, also in a warp whose rows
-    // all died before a linear probe (the buffer is not cleared)
-  } else if (mp == 2) {
-    // write kernel (Fig 8): flagged rows write at their prefix-sum position --
-    // the projections (A1) or the aggregation inputs: packed group key, values (B1/C1)
-    const std::string pv = g.val(kp.mp_pos_reg);
-    if (sk == 2) {
-      std::vector<std::string> ov;
-      for (int j = 0; j < kp.nout; ++j) ov.push_back(g.val(kp.out_reg[j]));
-      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = (u64)(u32)" << pv << ";";
-      for (int j = 0; j < kp.nout; ++j)
-        o << " ((" << ctype(kp.out_width[j]) << "*)p.out[" << j << "])[pos_] = (" << ctype(kp.out_width[j]) << ")" << ov[j] << ";";
-      o << " }\n";
-    } else {
-      o << "      u64 gk_[R]; bool bad_ = false;\n#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = 0;\n";
-      for (int i = 0; i < kp.nkeys; ++i) {
-        const std::string v = g.val(kp.key_reg[i]);
-        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kp.key_min[i])
-          << "; if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }"
-          << " gk_[r] += (u64)d_ * " << kp.key_stride[i] << "ull; }\n";
-      }
-      o << "      if (bad_) atomicOr(p.err, F_KEY_DOMAIN);\n";
-      std::vector<std::string> vv;
-      for (int a = 0; a < kp.naggs; ++a) vv.push_back(kp.agg_fn[a] == HQ_AGG_COUNT ? std::string() : g.val(kp.agg_reg[a]));
-      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = (u64)(u32)" << pv << ";";
-      int oc = 0;
-      if (kp.nkeys > 0) o << " ((u64*)p.out[" << oc++ << "])[pos_] = gk_[r];";
-      for (int a = 0; a < kp.naggs; ++a)
-        if (kp.agg_fn[a] != HQ_AGG_COUNT) o << " ((i64*)p.out[" << oc++ << "])[pos_] = (i64)" << vv[a] << ";";
-      o << " }\n";
-    }
-  } else {
+  // the sink's per-tile code (aggregation into registers / shared tables, or the
+  // materialised values handed to the block scan), emitted where the ops end
+  auto sink_tile = [&]() {
   if (sk != 2) g.early_exit();  // the sinks below only touch live rows
   // ------------------------------------------------------------ sink (tile)
   auto aggval = [&](int a) -> std::string {
@@ -1033,6 +903,293 @@ std::string generate(const KPlan& kp) {
     for (int j = 0; j < kp.nout; ++j) o << " ov" << j << "[r] = (long long)" << ov[j] << ";";
     o << " }\n";
   }
+  };
+  // ---------------------------------------------------------------- kernel
+  o << "extern \"C\" __global__ void __launch_bounds__((NW + 1) * 32, 1) hq_jit_kernel(const __grid_constant__ JParams p) {\n"
+    << "  extern __shared__ __align__(128) char smem[];\n"
+    << "  u64* full = (u64*)smem; u64* empty = full + 10;\n"
+    << "  u64* s_base = (u64*)(empty + 10); int* s_wtot = (int*)(s_base + 32); i64* s_red = (i64*)(s_wtot + 32);\n"
+    << "  char* sagg = smem + OFF_AGG; char* stages = smem + OFF_STAGE;\n"
+    << "  const u32 sm0_ = smem_u32(smem); (void)sm0_;\n"
+    << "  (void)s_base; (void)s_wtot; (void)s_red; (void)sagg;\n"
+    << "  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n"
+    << "  const long long first_tile = p.row_begin / T;\n"
+    << "  const long long ntiles = p.row_end > p.row_begin ? (p.row_end + T - 1) / T - first_tile : 0;\n"
+    << "  const long long nj = ntiles > blockIdx.x ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;\n"
+    << "  const long long tstep = (long long)gridDim.x * T;\n"
+    << "  if (threadIdx.x == 0) { for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], NW); } fence_mbar_init(); }\n";
+  if (prof) o << "  long long pt0_ = 0; if (threadIdx.x == 0) asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(pt0_));\n"
+              << "  long long pw_ = 0, pl0_ = clock64(); int pdv_ = 0;\n";
+  // smem table init
+  if (sk == 1 && kp.smode == SM_LANE) {
+    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * NACC * NW * 32; i += NW * 32) {"
+      << " const int a_ = (int)((i / (NW * 32)) % NACC); t_[i] = a_ == 0 ? 0 : agg_identity(ACC_FN[a_]); } }\n";
+  } else if (sk == 1 && kp.smode == SM_DENSE) {
+    o << "  if (warp < NW) { i64* t_ = (i64*)sagg; for (u32 i = threadIdx.x; i < SMEM_CAP * LVWORDS * SCOPIES; i += NW * 32) {"
+      << " const int c_ = (int)(i % LVWORDS); t_[i] = c_ == 0 ? 0 : agg_identity(LFN[c_]); } }\n";
+  } else if (sk == 1 && kp.smode == SM_HASH) {
+    o << "  if (warp < NW) { u64* k_ = (u64*)sagg; i64* e_ = (i64*)sagg + SMEM_CAP;\n"
+      << "    for (u32 i = threadIdx.x; i < SMEM_CAP; i += NW * 32) k_[i] = HQ_EMPTY_KEY;\n"
+      << "    for (u32 i = threadIdx.x; i < SMEM_CAP * LVWORDS; i += NW * 32) { const int c_ = (int)(i % LVWORDS); e_[i] = c_ == 0 ? 0 : agg_identity(LFN[c_]); } }\n";
+  }
+  // staged compact probe tables: one cooperative 16-B copy per CTA
+  for (int i = 0; i < MAX_PROBES; ++i) {
+    const KProbe& pr = kp.probes[i];
+    if (!pr.smem_off) continue;
+    o << "  { const uint4* src_ = (const uint4*)p.ctab[" << i << "]; uint4* dst_ = (uint4*)(smem + " << pr.smem_off << "u);\n"
+      << "    for (u32 x = threadIdx.x; x < " << (pr.cbytes + 15) / 16 << "u; x += blockDim.x) dst_[x] = __ldg(src_ + x); }\n";
+  }
+  o << "  __syncthreads();\n";
+  // producer
+  o << "  if (warp == NW) {\n    if (lane == 0) {\n      const u64 pol = policy_evict_first();\n"
+    << "      int s = 0; u32 ph = 0; long long t0 = (first_tile + blockIdx.x) * (long long)T;\n"
+    << "      for (long long j = 0; j < nj; ++j, t0 += tstep) {\n"
+    << "        " << (prof ? "{ const long long c_ = clock64(); if (j >= S) mbar_wait(&empty[s], ph ^ 1u); pw_ += clock64() - c_; }" : "if (j >= S) mbar_wait(&empty[s], ph ^ 1u);") << "\n"
+    << "        char* st = stages + (size_t)s * STAGE_STRIDE;\n"
+    << "        if (t0 >= p.row_begin && t0 + T <= p.row_end) {\n          mbar_expect_tx(&full[s], STAGE_BYTES);\n";
+  for (int k = 0; k < kp.ncols; ++k)
+    o << "          tma_load_1d(st + " << kp.cols[k].soff << "u, p.col[" << k << "] + t0 * " << kp.cols[k].width << ", "
+      << kp.tile_rows * kp.cols[k].width << "u, &full[s], pol);\n";
+  o << "        } else mbar_arrive(&full[s]);\n        if (++s == S) { s = 0; ph ^= 1u; }\n      }\n";
+  if (prof) o << "      p.prof[blockIdx.x * 128 + 3] = pw_; p.prof[blockIdx.x * 128 + 4] = clock64() - pl0_;\n";
+  o << "    }\n    return;\n  }\n";
+  // consumer state
+  o << "  const int row0 = warp * 32 * R + lane * R;  // the lane's rows: row0 .. row0 + R - 1\n";
+  if (kp.a3stage) o << "  u64 a3pend_ = 0;  // thread 0: the pending atomicAdd of the last tile (staged A3)\n";
+  if (sk == 0 && !c2 && !we) {
+    o << "  u64 scount_ = 0;\n";
+    for (int a = 0; a < kp.naggs; ++a) o << "  i64 sacc" << a << " = agg_identity(AGG_FN[" << a << "]);\n";
+  }
+  // HQ_JIT_WAIT=sleep: the older poll + nanosleep loop (A/B)
+  const char* wm = getenv("HQ_JIT_WAIT");
+  const std::string cwait = (wm && std::string(wm) == "sleep") ? "mbar_wait_sleep(&full[s], ph);" : "mbar_wait_suspend_a(sm0_ + 8u * (u32)s, ph);";
+  // ---- software pipelining (two tiles per warp in flight).  A star join whose first
+  // global-memory probe batch (byte maps / bitmaps in L2) every row waits on is split
+  // there: phase A of a tile = stage wait, ragged copy, columns, filters and shared-memory
+  // probes, and the batch's address + LOAD; phase B = the batch's resolution, the rest
+  // of the operators and the sink.  The loop runs A(j+1) before B(j), so each warp has
+  // two tiles' probe loads in flight instead of stalling on every tile's round trip.
+  // The stage of tile j is held until B(j) ends (no early release), A's arrays are
+  // declared once per tile parity (a / b, renamed with #define).
+  int swp_split = -1;
+  if (!mp && !c2 && !we && (sk == 0 || sk == 1) && kp.R == 2 && kp.smode != SM_LANE && !prof &&
+      !(wm && std::string(wm) == "sleep") && getenv("HQ_JIT_SWP") && getenv("HQ_JIT_SWP")[0] == '1') {
+    // opt-in: measured on B200 it LOSES (SSB Q3.1 SF30 0.56 -> 0.73 ms, Q4.1 SF100
+    // 2.50 -> 3.29 ms): holding two stages per warp starves the 3-stage TMA ring and
+    // the second tile's arrays spill at 64 registers; kept for experiments
+    for (int i = 0; i < kp.nops && swp_split < 0; ++i) {
+      if (kp.op_skip[i] || kp.ops[i].kind != OP_PROBE) continue;
+      const int ak = Gen::access(kp.probes[kp.ops[i].idx]);
+      if (ak == Gen::AK_LINEAR) break;
+      if (ak == Gen::AK_GCOMPACT || ak == Gen::AK_DIRECT) swp_split = i;
+    }
+  }
+  if (swp_split >= 0) {
+    const std::string pre = o.str();
+    o.str(std::string());
+    o.clear();
+    std::ostringstream decls;
+    // ---- phase A (as text with base names)
+    g.decl = &decls;
+    decls << "  int si_; const char* st; long long tt_; u32 mask;\n";
+    g.hoisted = {"si_", "st", "tt_", "mask"};
+    o << "      mbar_wait_suspend_a(sm0_ + 8u * (u32)s, ph);\n"
+      << "      si_ = s; st = stages + (size_t)s * STAGE_STRIDE; tt_ = t00_ + (long long)jt_ * tstep;\n"
+      << "      mask = (1u << R) - 1u;\n"
+      << "      if (jt_ == rj0_ || jt_ == rj1_) {  // ragged head / tail tile: lanes copy their rows\n"
+      << "        const int lo = (int)(p.row_begin > tt_ ? p.row_begin - tt_ : 0);\n"
+      << "        const int hi = (int)(p.row_end - tt_ < T ? p.row_end - tt_ : T);\n"
+      << "        mask = 0;\n#pragma unroll\n        for (int r = 0; r < R; ++r) { const int row = row0 + r; if (row >= lo && row < hi) mask |= 1u << r; }\n";
+    for (int k = 0; k < kp.ncols; ++k) {
+      const char* ty = ctype(kp.cols[k].width);
+      o << "#pragma unroll\n        for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r; ((" << ty
+        << "*)(st + " << kp.cols[k].soff << "u))[row] = ((const " << ty << "*)p.col[" << k << "])[tt_ + row]; }\n";
+    }
+    o << "        fence_proxy_async(); __syncwarp();\n      }\n";
+    g.begin_al();
+    int i = 0;
+    while (i < swp_split) {
+      if (kp.op_skip[i]) { ++i; continue; }
+      const KOp op = kp.ops[i];
+      if (op.kind == OP_PROBE) { i = g.probe_batch(i); continue; }
+      if (op.kind == OP_FILTER) g.filter(kp.preds[op.idx], op.idx);
+      else g.compute(kp.comps[op.idx]);
+      ++i;
+    }
+    i = g.probe_batch(swp_split, 1);
+    o << "      if (++s == S) { s = 0; ph ^= 1u; }\n";
+    const std::string acode = o.str();
+    o.str(std::string());
+    o.clear();
+    // ---- phase B
+    g.decl = nullptr;
+    g.probe_batch(swp_split, 2);
+    while (i < kp.nops) {
+      if (kp.op_skip[i]) { ++i; continue; }
+      const KOp op = kp.ops[i];
+      if (op.kind == OP_PROBE) { i = g.probe_batch(i); continue; }
+      if (op.kind == OP_FILTER) g.filter(kp.preds[op.idx], op.idx);
+      else g.compute(kp.comps[op.idx]);
+      ++i;
+    }
+    g.sync_mask();
+    sink_tile();
+    for (int k = 0; k < g.open; ++k) o << "      }\n";
+    g.open = 0;
+    o << "      __syncwarp();\n      if (lane == 0) mbar_arrive_a(sm0_ + 80u + 8u * (u32)si_);\n";
+    const std::string bcode = o.str();
+    // ---- assembly
+    auto def = [&](const char* x) {
+      std::string d;
+      for (const auto& n : g.hoisted) d += "#define " + n + " " + n + "_" + x + "\n";
+      return d;
+    };
+    auto undef = [&]() {
+      std::string d;
+      for (const auto& n : g.hoisted) d += "#undef " + n + "\n";
+      return d;
+    };
+    o.str(pre);
+    o.seekp(0, std::ios_base::end);
+    o << "  // software-pipelined tile loop: A(j+1) before B(j)\n" << def("a") << decls.str() << undef() << def("b")
+      << decls.str() << undef()
+      << "  int s = 0; u32 ph = 0; const long long t00_ = (first_tile + blockIdx.x) * (long long)T;\n"
+      << "  const int njc = (int)nj;\n"
+      << "  const long long tl_ = t00_ + (nj - 1) * tstep;\n"
+      << "  const int rj0_ = (nj > 0 && (t00_ < p.row_begin || t00_ + T > p.row_end)) ? 0 : -1;\n"
+      << "  const int rj1_ = (nj > 0 && (tl_ < p.row_begin || tl_ + T > p.row_end)) ? njc - 1 : -1;\n"
+      << "  if (njc > 0) {\n    const int jt_ = 0;\n" << def("a") << acode << undef() << "  }\n"
+      << "  for (int j = 0; j < njc; j += 2) {\n"
+      << "    if (j + 1 < njc) {\n      const int jt_ = j + 1;\n" << def("b") << acode << undef() << "    }\n"
+      << "    {\n" << def("a") << bcode << undef() << "    }\n"
+      << "    if (j + 1 >= njc) break;\n"
+      << "    if (j + 2 < njc) {\n      const int jt_ = j + 2;\n" << def("a") << acode << undef() << "    }\n"
+      << "    {\n" << def("b") << bcode << undef() << "    }\n"
+      << "  }\n";
+  } else {
+  o << "  int s = 0; u32 ph = 0; long long t0 = (first_tile + blockIdx.x) * (long long)T;\n"
+    << "  const int njc = (int)nj;\n"
+    // only a CTA's first and last tile can be ragged (partition boundaries): decided once
+    << "  const long long tl_ = t0 + (nj - 1) * tstep;\n"
+    << "  const int rj0_ = (nj > 0 && (t0 < p.row_begin || t0 + T > p.row_end)) ? 0 : -1;\n"
+    << "  const int rj1_ = (nj > 0 && (tl_ < p.row_begin || tl_ + T > p.row_end)) ? njc - 1 : -1;\n"
+    << "  for (int j = 0; j < njc; ++j, t0 += tstep) {\n"
+    << (prof ? "    { const long long c_ = clock64(); " + cwait + " pw_ += clock64() - c_; if (__activemask() != 0xffffffffu) ++pdv_; }\n" : "    " + cwait + "\n")
+    << "    const char* st = stages + (size_t)s * STAGE_STRIDE;\n"
+    << "    const long long tb_ = t0;  // tile start (temporaries t0, t1, ... shadow it below)\n"
+    << "    u32 mask = (1u << R) - 1u;\n"
+    << "    if (j == rj0_ || j == rj1_) {  // ragged head / tail tile: lanes copy their rows\n"
+    << "      const int lo = (int)(p.row_begin > t0 ? p.row_begin - t0 : 0);\n"
+    << "      const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
+    << "      mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r; if (row >= lo && row < hi) mask |= 1u << r; }\n";
+  for (int k = 0; k < kp.ncols; ++k) {
+    const char* ty = ctype(kp.cols[k].width);
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r; ((" << ty
+      << "*)(st + " << kp.cols[k].soff << "u))[row] = ((const " << ty << "*)p.col[" << k << "])[t0 + row]; }\n";
+  }
+  o << "      fence_proxy_async(); __syncwarp();\n    }\n";
+  if (sk == 2)  // output values leave the operator block in registers; the block scan runs after it
+    for (int j = 0; j < kp.nout; ++j) o << "    long long ov" << j << "[R];\n";
+  if (we && sk == 0 && !mp) {  // the tile's per-thread partials leave the operator block for the WE tree
+    o << "    u32 wc_ = 0u; i64 wa_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n    for (int a = 0; a < NAGGS; ++a) wa_[a] = agg_identity(AGG_FN[a]);\n";
+  } else if (we && sk == 1 && !mp) {  // the tile's live (key, values) leave it for the WE sort + segmented scan
+    o << "    u32 wm_ = 0u; u64 wk_[R]; i64 wv_[NAGGS > 0 ? NAGGS : 1][R];\n";
+  }
+  o << "    {\n";
+  if (kp.early_release) {
+    // every referenced column of the lane's rows into registers, then the stage
+    // goes back to the producer (mbarrier.arrive releases the warp's prior
+    // shared loads); the operators below run on registers only
+    for (const auto& sk2 : g.stage_k) g.use(sk2.first);
+    // The arrive must not overtake the lanes' shared loads of the stage (the
+    // producer's next TMA overwrites it): measured on B200, a bare __syncwarp +
+    // arrive let ~1 % of SSB Q4.1 runs read a refilled value.  Every lane folds
+    // its loaded registers, a ballot over the fold completes only after all
+    // loads did, and lane 0 stores the ballot before its (release) arrive.
+    const char* rf = getenv("HQ_JIT_RELFIX");  // A/B: dep (default), fence, none
+    const std::string fix = rf ? rf : "dep";
+    if (fix == "dep") {
+      // one destination register per shared load instruction: a vector load
+      // completes all its registers together, so element 0 stands for it
+      o << "    { u32 f_ = 0u";
+      for (const auto& sk2 : g.stage_k)
+        if (g.vec_loaded.count(sk2.first)) o << " ^ (u32)" << g.var(sk2.first) << "[0]";
+      o << ";\n";
+      bool scalar = false;
+      for (const auto& sk2 : g.stage_k) scalar = scalar || !g.vec_loaded.count(sk2.first);
+      if (scalar) {
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) f_ ^= 0u";
+        for (const auto& sk2 : g.stage_k)
+          if (!g.vec_loaded.count(sk2.first)) o << " ^ (u32)" << g.var(sk2.first) << "[r]";
+        o << ";\n";
+      }
+      o << "      const u32 b_ = __ballot_sync(HQ_FULL, f_ == 0x9E3779B9u);\n"
+        << "      if (lane == 0) { *(volatile u32*)(smem + " << (MISC_DEP) << "u + 4u * warp) = b_; mbar_arrive_a(sm0_ + 80u + 8u * (u32)s); } }\n";
+    } else if (fix == "fence") {
+      o << "    fence_proxy_async(); __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
+    } else {
+      o << "    __syncwarp();\n    if (lane == 0) mbar_arrive(&empty[s]);\n";
+    }
+  }
+  if (mp == 2) {  // the count kernel's flags select the rows
+    const std::string f = g.val(kp.mp_flag_reg);
+    o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (!" << f << ") mask &= ~(1u << r);\n";
+  }
+  // compaction point (Gen::compact): after the first probe that passes at most
+  // half of the rows (build-side key density), aggregation sinks only, R >= 2
+  int cpt = -1;
+  if (sk != 2 && !c2 && kp.R >= 4 && kp.smode != SM_LANE)  // at R = 2 the shuffles cost more than they save (B200)
+    for (int i = 0; i < kp.nops && cpt < 0; ++i)
+      if (kp.ops[i].kind == OP_PROBE && kp.probes[kp.ops[i].idx].pass_est <= 0.5f) cpt = i;
+  if (const char* e = getenv("HQ_JIT_CPT")) cpt = (e[0] == 'o') ? -1 : (sk != 2 ? atoi(e) : -1);
+  if (mp) cpt = -1;
+  g.begin_al();
+  for (int i = 0; i < kp.nops;) {
+    if (cpt >= 0 && !g.compacted_R && i > cpt) g.compact(i);
+    if (kp.op_skip[i]) { ++i; continue; }  // not executed in this pass
+    const KOp op = kp.ops[i];
+    if (op.kind == OP_PROBE) { i = g.probe_batch(i); continue; }
+    if (op.kind == OP_FILTER) g.filter(kp.preds[op.idx], op.idx);
+    else g.compute(kp.comps[op.idx]);
+    ++i;
+  }
+  if (cpt >= 0 && !g.compacted_R) g.compact(kp.nops);
+  g.sync_mask();  // the sinks, the block scan and the count kernel's flags read mask
+  if (mp == 1) {
+    // count kernel: the flags are written below, after the early-exit blocks
+    // close -- every row of the range gets its flag, also in a warp whose rows
+    // all died before a linear probe (the buffer is not cleared)
+  } else if (mp == 2) {
+    // write kernel (Fig 8): flagged rows write at their prefix-sum position --
+    // the projections (A1) or the aggregation inputs: packed group key, values (B1/C1)
+    const std::string pv = g.val(kp.mp_pos_reg);
+    if (sk == 2) {
+      std::vector<std::string> ov;
+      for (int j = 0; j < kp.nout; ++j) ov.push_back(g.val(kp.out_reg[j]));
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = (u64)(u32)" << pv << ";";
+      for (int j = 0; j < kp.nout; ++j)
+        o << " ((" << ctype(kp.out_width[j]) << "*)p.out[" << j << "])[pos_] = (" << ctype(kp.out_width[j]) << ")" << ov[j] << ";";
+      o << " }\n";
+    } else {
+      o << "      u64 gk_[R]; bool bad_ = false;\n#pragma unroll\n      for (int r = 0; r < R; ++r) gk_[r] = 0;\n";
+      for (int i = 0; i < kp.nkeys; ++i) {
+        const std::string v = g.val(kp.key_reg[i]);
+        o << "#pragma unroll\n      for (int r = 0; r < R; ++r) { const long long d_ = (long long)" << v << " - " << lit(kp.key_min[i])
+          << "; if (d_ < 0 || d_ >= " << lit(kp.key_card[i]) << ") { if ((mask >> r) & 1u) bad_ = true; mask &= ~(1u << r); }"
+          << " gk_[r] += (u64)d_ * " << kp.key_stride[i] << "ull; }\n";
+      }
+      o << "      if (bad_) atomicOr(p.err, F_KEY_DOMAIN);\n";
+      std::vector<std::string> vv;
+      for (int a = 0; a < kp.naggs; ++a) vv.push_back(kp.agg_fn[a] == HQ_AGG_COUNT ? std::string() : g.val(kp.agg_reg[a]));
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const u64 pos_ = (u64)(u32)" << pv << ";";
+      int oc = 0;
+      if (kp.nkeys > 0) o << " ((u64*)p.out[" << oc++ << "])[pos_] = gk_[r];";
+      for (int a = 0; a < kp.naggs; ++a)
+        if (kp.agg_fn[a] != HQ_AGG_COUNT) o << " ((i64*)p.out[" << oc++ << "])[pos_] = (i64)" << vv[a] << ";";
+      o << " }\n";
+    }
+  } else {
+  sink_tile();
   }  // !mp
   for (int k = 0; k < g.open; ++k) o << "    }\n";
   if (mp == 1)  // count kernel (Fig 8): one int32 flag per row, indexed by absolute row (base offset by the host)
@@ -1041,7 +1198,33 @@ std::string generate(const KPlan& kp) {
   if (g.compacted_R) o << "#undef R\n#define R " << g.compacted_R << "\n";
   o << "    }\n";
   if (we && !mp) gen_we_tile(o, kp, sk);
-  if (sk == 2 && !mp && !we) {
+  if (sk == 2 && !mp && !we && !c2 && kp.a3stage) {
+    // A3 (Fig 25 / P:1069-1072) with a deferred write-out: warp ballots -> block scan
+    // over the warps -> ONE atomicAdd per block and tile, issued by thread 0 and not
+    // waited for: the tile's rows go to a shared staging buffer at their tile-local
+    // positions, and during the NEXT tile (after its first barrier) the whole CTA
+    // copies them, coalesced, to base + position -- the atomic's round trip is off the
+    // tile's critical path.  Output order: each tile's rows contiguous, in row order.
+    o << "    {\n      const int buf_ = j & 1;\n"
+      << "      if (threadIdx.x == 0 && j > 0) s_red[buf_ ^ 1] = (i64)a3pend_;  // the previous tile's base\n"
+      << "      const int mine_ = __popc(mask); int lin_ = mine_;\n"
+      << "#pragma unroll\n      for (int o_ = 1; o_ < 32; o_ <<= 1) { const int t_ = __shfl_up_sync(HQ_FULL, lin_, o_); if (lane >= o_) lin_ += t_; }\n"
+      << "      const int wtot_ = __shfl_sync(HQ_FULL, lin_, 31);\n"
+      << "      if (lane == 0) s_wtot[warp] = wtot_;\n      consumer_bar();\n"
+      << "      if (j > 0) a3_flush(p, s_red[buf_ ^ 1], (int)s_red[2 + (buf_ ^ 1)], smem + OFF_AGG + (buf_ ^ 1) * A3BUF);\n"
+      << "      if (warp == 0) { const int v_ = lane < NW ? s_wtot[lane] : 0; int incl_ = v_;\n"
+      << "#pragma unroll\n        for (int o_ = 1; o_ < 32; o_ <<= 1) { const int t_ = __shfl_up_sync(HQ_FULL, incl_, o_); if (lane >= o_) incl_ += t_; }\n"
+      << "        const int total_ = __shfl_sync(HQ_FULL, incl_, 31);\n"
+      << "        if (lane < NW) s_base[lane] = (u64)(incl_ - v_);\n"
+      << "        if (lane == 0) { s_red[2 + buf_] = total_; a3pend_ = total_ > 0 ? atomicAdd(p.counter, (u64)total_) : 0ull; } }\n"
+      << "      consumer_bar();\n"
+      << "      char* sb_ = smem + OFF_AGG + buf_ * A3BUF;\n"
+      << "      const int wo_ = (int)s_base[warp] + (lin_ - mine_);\n"
+      << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const int pos_ = wo_ + __popc(mask & ((1u << r) - 1u));\n";
+    for (int j = 0; j < kp.nout; ++j)
+      o << "        ((" << ctype(kp.out_width[j]) << "*)(sb_ + " << kp.a3_col[j] << "u))[pos_] = (" << ctype(kp.out_width[j]) << ")ov" << j << "[r];\n";
+    o << "      }\n    }\n";
+  } else if (sk == 2 && !mp && !we) {
     // A3 (Fig 25 / P:1069-1072): warp ballots -> block scan over the warps ->
     // one atomicAdd per block and tile -> writes at local + global offset.
     // Every consumer warp takes part in every tile (its mask may be empty).
@@ -1072,7 +1255,11 @@ std::string generate(const KPlan& kp) {
   }
   if (kp.early_release) o << "    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
   else o << "    __syncwarp();\n    if (lane == 0) mbar_arrive_a(sm0_ + 80u + 8u * (u32)s);\n    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
+  }  // software pipelining
   if (prof) o << "  if (lane == 0) { p.prof[blockIdx.x * 128 + 8 + warp] = pw_; p.prof[blockIdx.x * 128 + 40 + warp] = clock64() - pl0_; } if (pdv_) atomicAdd((unsigned long long*)&p.prof[blockIdx.x * 128 + 72 + warp], (unsigned long long)pdv_);\n";
+  if (kp.a3stage && sk == 2 && !mp && !we && !c2)  // the last tile's staged rows
+    o << "  if (njc > 0) { const int lb_ = (njc - 1) & 1; if (threadIdx.x == 0) s_red[lb_] = (i64)a3pend_; consumer_bar();\n"
+      << "    a3_flush(p, s_red[lb_], (int)s_red[2 + lb_], smem + OFF_AGG + lb_ * A3BUF); }\n";
   // ------------------------------------------------------------- sink (end)
   if (mp) {
   } else if (sk == 0 && !c2 && !we) {
@@ -1149,7 +1336,7 @@ std::string generate(const KPlan& kp) {
     << "static constexpr __device__ int ACC_FN[" << (kp.nacc > 0 ? kp.nacc : 1) << "] = " << fn_list(kp.acc_fn, kp.nacc) << ";\n"
     << "#define LVWORDS " << kp.lvwords << "\n" << lcol_tables(kp)
     << HQ_STR(HQ_JPARAMS_DEF) << "\n"
-    << kPrelude << "\n"
+    << kPrelude << "\n" << a3_flush_fn(kp)
     << g.bitmaps.str() << "\n";
   return h.str() + o.str();
 }

@@ -122,14 +122,15 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       if (op.mode < HQ_PROBE_INNER || op.mode > HQ_PROBE_OUTER) HQ_THROW(HQ_ERR_ARG, "plan: bad probe mode");
       KProbe& pr = kp.probes[nprobe];
       pr.key_reg = (int16_t)use(op.key_reg, "probe key");
-      pr.slots = op.ht->slots;
+      // generated kernels read a direct table's compact form; the other executions its slots
+      pr.slots = jit ? op.ht->slots : hq_hash_slots(ctx, const_cast<hq_hash*>(op.ht));
       pr.direct = op.ht->meta.layout == HQ_HT_DIRECT;
       pr.mask = pr.direct ? (uint32_t)op.ht->meta.capacity : (uint32_t)(op.ht->meta.capacity - 1);
       pr.dmin = (int32_t)op.ht->meta.key_min;
       pr.log2cap = (uint8_t)op.ht->log2cap;
       pr.ckind = (uint8_t)op.ht->ckind;
       pr.crank = (uint8_t)op.ht->crank;
-      pr.compact = op.ht->compact.p;
+      pr.compact = op.ht->compact_ptr();
       pr.pay_min = op.ht->meta.pay_min;
       pr.pay_max = op.ht->meta.pay_max;
       for (int k = 0; k < 4; ++k) pr.pay_set[k] = op.ht->meta.pay_set[k];
@@ -545,6 +546,16 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     }
   }
   int chosen_R = 0;
+  // generated materialisation (A3): stage the tile's output rows in shared memory when
+  // two tile buffers fit beside the ring (the global write-out moves to the next tile)
+  uint32_t outbytes = 0;
+  for (int j = 0; j < kp.nout; ++j) outbytes += kp.out_width[j];
+  // opt-in (HQ_JIT_A3STAGE=1): measured on B200 it does not pay -- TPC-H Q3 SF30 orders side
+  // 0.367 -> 0.377 ms, SSB Q3.1 materialised 1.165 -> 1.166 ms, Exp 1 Query 1 0.26 -> 0.32 ms:
+  // the per-tile barriers, not the atomic's round trip, bound A3 behind a global probe
+  const char* a3e = getenv("HQ_JIT_A3STAGE");
+  bool a3try = jit && !mp_pass && P.sink == HQ_SINK_MATERIALISE && P.resolution == HQ_RES_LRGP && a3e && a3e[0] == '1';
+  kp.a3stage = 0;
   for (;;) {
     uint32_t tab_total = 0;
     for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
@@ -553,7 +564,8 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       const uint32_t T = (uint32_t)(kp.nw * 32 * R);
       const uint32_t off_tmp = MISC_BYTES;
       const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
-      const uint32_t off_tab = align_up(off_agg + agg_smem, 128);
+      const uint32_t a3buf = a3try ? align_up(T * outbytes, 128) : 0;
+      const uint32_t off_tab = align_up(off_agg + agg_smem + 2 * a3buf, 128);
       const uint32_t off_stage = align_up(off_tab + tab_total, 128);
       const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
       if (off_stage >= ctx->max_smem) continue;
@@ -570,11 +582,25 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         kp.off_tab = off_tab;
         kp.tab_bytes = tab_total;
         kp.off_stage = off_stage;
+        kp.a3stage = a3try ? 1 : 0;
+        kp.a3_buf = a3buf;
         break;
       }
     }
-    if (chosen_R || nstaged == 0) break;
+    if (chosen_R) break;
+    if (a3try) {  // no room for the staging buffers: write rows straight to global memory
+      a3try = false;
+      continue;
+    }
+    if (nstaged == 0) break;
     --nstaged;  // give the last staged table back to the ring
+  }
+  if (kp.a3stage) {
+    uint32_t off = 0;
+    for (int j = 0; j < kp.nout; ++j) {
+      kp.a3_col[j] = off;
+      off += (uint32_t)kp.tile_rows * kp.out_width[j];
+    }
   }
   if (!chosen_R) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: rows too wide for the shared-memory stage ring");
   kp.early_release = 0;

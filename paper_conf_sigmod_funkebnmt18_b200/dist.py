@@ -38,13 +38,13 @@ def _i64(u: int) -> int:
     return u - (1 << 64) if u >= (1 << 63) else u
 
 
-# hq_hash_meta <-> one int64 row of the metadata broadcast (column 15 is spare)
+# hq_hash_meta <-> one int64 row of the metadata broadcast
 META_COLS = 16
 
 
 def meta_row(m: hq.HashMeta) -> List[int]:
     return ([m.capacity, m.slot_words, m.npayload, m.nkeys, m.bytes, m.key_min, m.layout, m.pay_min, m.pay_max,
-             m.key_max] + [_i64(w) for w in m.pay_set] + [m.composite, 0])
+             m.key_max] + [_i64(w) for w in m.pay_set] + [m.composite, m.compact_kind])
 
 
 def meta_from_row(r: Sequence[int]) -> hq.HashMeta:
@@ -54,6 +54,7 @@ def meta_from_row(r: Sequence[int]) -> hq.HashMeta:
     for k in range(4):
         hm.pay_set[k] = int(r[10 + k]) & 0xFFFFFFFFFFFFFFFF
     hm.composite = int(r[14])
+    hm.compact_kind = int(r[15])
     return hm
 
 

@@ -67,7 +67,8 @@ class HashMeta(ctypes.Structure):
     _fields_ = [("capacity", ctypes.c_int64), ("slot_words", ctypes.c_int32), ("npayload", ctypes.c_int32),
                 ("nkeys", ctypes.c_int64), ("bytes", ctypes.c_int64), ("key_min", ctypes.c_int64),
                 ("layout", ctypes.c_int32), ("pay_min", ctypes.c_int32), ("pay_max", ctypes.c_int32),
-                ("key_max", ctypes.c_int32), ("pay_set", ctypes.c_uint64 * 4), ("composite", ctypes.c_int32)]
+                ("key_max", ctypes.c_int32), ("pay_set", ctypes.c_uint64 * 4), ("composite", ctypes.c_int32),
+                ("compact_kind", ctypes.c_int32)]
 
 
 class Insn(ctypes.Structure):

@@ -2,10 +2,12 @@
 """Reduction micro-benchmarks of the paper on B200:
 
 * Exp 1 (Fig 16-17): Query 1 selection + projection, materialised,
-  selectivity swept 0..1 -- A1 (multi-pass), A2 (per-row atomics), A3 (LRGP);
-* App G.1 (P:2171-2185): the same query as a single-tuple aggregation -- B1, B2, B3;
+  selectivity swept 0..1 -- A1 (multi-pass), A2 (per-row atomics), A3 with SIMD-style
+  local resolution (warp ballots/shuffles, the default) and A3-WE (work-efficient
+  Blelloch scan over the workgroup, App C Fig 24, P:1989-2029);
+* App G.1 (P:2171-2185): the same query as a single-tuple aggregation -- B1, B2, B3, B3-WE;
 * Exp 2 (Fig 26): SUM(lo_extendedprice) GROUP BY lo_orderkey % x,
-  x = 2 .. 16384 groups -- C1, C2, C3;
+  x = 2 .. 16384 groups -- C1, C2, C3, C3-WE (sort + segmented scan, P:2040-2057);
 
 each also as the operator-at-a-time plan.  Times are the pipeline's device time
 (CUDA events around the fused kernel, or around the whole multi-pass sequence),
@@ -34,6 +36,7 @@ MODES = {  # technique letter -> (exec mode, resolution)
     "1": (hq.EXEC_MULTIPASS, hq.RES_LRGP),
     "2": (hq.EXEC_FUSED, hq.RES_ATOMIC),
     "3": (hq.EXEC_FUSED, hq.RES_LRGP),
+    "3WE": (hq.EXEC_FUSED, hq.RES_WE),
 }
 
 
@@ -96,18 +99,20 @@ def main():
     L = [f"Reduction micro-benchmarks on one B200, SSB lineorder SF {a.sf:g} ({n} rows, resident in HBM); "
          "pipeline device time in ms (median of "
          f"{a.reps}); 1 = multi-pass (count kernel, prefix sum, write kernel, library reduce/sort), 2 = per-row global "
-         "atomics, 3 = local resolution + global propagation (LRGP, the default); op-at-a-time = wall clock around the "
-         "plan (its kernels plus host synchronisations).", "",
+         "atomics, 3 = local resolution + global propagation (LRGP with SIMD-style warp resolution, the default), 3WE = "
+         "the same with work-efficient (Blelloch) resolution over the workgroup (App C, Fig 24); op-at-a-time = wall "
+         "clock around the plan (its kernels plus host synchronisations).", "",
          "Exp 1 / App G.1: `lo_quantity BETWEEN 25-x AND 25+x`, revenue = extendedprice*discount+tax; A = materialised, "
          "B = single-tuple SUM", "",
-         "| x | selectivity | A1 | A2 | A3 | A op-at-a-time | B1 | B2 | B3 |", "|---|---|---|---|---|---|---|---|---|"]
+         "| x | selectivity | A1 | A2 | A3 (SIMD) | A3-WE | A op-at-a-time | B1 | B2 | B3 (SIMD) | B3-WE |",
+         "|---|---|---|---|---|---|---|---|---|---|---|"]
     for r in res["exp1"]:
-        L.append(f"| {r['x']} | {r['selectivity']:.2f} | {r['A1']:.3f} | {r['A2']:.3f} | {r['A3']:.3f} | {r['A_oaat']:.3f} | "
-                 f"{r['B1']:.3f} | {r['B2']:.3f} | {r['B3']:.3f} |")
+        L.append(f"| {r['x']} | {r['selectivity']:.2f} | {r['A1']:.3f} | {r['A2']:.3f} | {r['A3']:.3f} | {r['A3WE']:.3f} | "
+                 f"{r['A_oaat']:.3f} | {r['B1']:.3f} | {r['B2']:.3f} | {r['B3']:.3f} | {r['B3WE']:.3f} |")
     L += ["", "Exp 2: `SUM(lo_extendedprice) GROUP BY lo_orderkey % x`", "",
-          "| groups | C1 | C2 | C3 | C op-at-a-time |", "|---|---|---|---|---|"]
+          "| groups | C1 | C2 | C3 (SIMD) | C3-WE | C op-at-a-time |", "|---|---|---|---|---|---|"]
     for r in res["exp2"]:
-        L.append(f"| {r['groups']} | {r['C1']:.3f} | {r['C2']:.3f} | {r['C3']:.3f} | {r['C_oaat']:.3f} |")
+        L.append(f"| {r['groups']} | {r['C1']:.3f} | {r['C2']:.3f} | {r['C3']:.3f} | {r['C3WE']:.3f} | {r['C_oaat']:.3f} |")
     with open(os.path.join(d, "micro_sweeps.md"), "w") as f:
         f.write("\n".join(L) + "\n")
     print("\n".join(L))

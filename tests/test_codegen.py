@@ -45,6 +45,7 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "p.pf[" in srcs["materialise_lrgp"]                     # linear prefilter
     assert "match_any" in srcs["global_hash_groups"] and "pre_[R]" in srcs["global_hash_groups_r4"]
     # group keys narrowed to the build-side payload ranges: dense shared table + key remap at the merge
+    assert "software-pipelined" not in star  # opt-in only (HQ_JIT_SWP=1)
     assert "#define SMODE 0" in srcs["star_smem_hash"]  # dense domain larger than any shared table: global (C2 + warp merging)
     narrowed = srcs["star_narrowed_dense"]
     assert "#define SMODE 1" in narrowed and "#define SMEM_CAP 1183u" in narrowed and "gkey_ +=" in narrowed

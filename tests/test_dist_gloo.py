@@ -55,6 +55,7 @@ def _stub_meta(k, nbytes):
     for i in range(4):
         m.pay_set[i] = (1 << 63) | (0x0123456789ABCDEF >> i) | k
     m.composite = k % 2
+    m.compact_kind = k % 4
     return m
 
 
