@@ -103,14 +103,15 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
-def gen_host(q, sf, seed, fact_range, with_dims, pinned=True):
-    """Referenced columns as numpy arrays (pinned host memory for the fact table)."""
+def gen_host(q, sf, seed, fact_range, with_dims, pinned=True, copart_range=None):
+    """Referenced columns as numpy arrays (pinned host memory for the fact table).
+    copart_range: this rank's rows of the co-partitioned order table (q.copart)."""
     import torch
     host = {}
     for t, cols in q.columns.items():
         if t != q.fact and not with_dims:
             continue
-        rr = fact_range if t == q.fact else None
+        rr = fact_range if t == q.fact else (copart_range if t == q.copart else None)
         n = (rr[1] - rr[0]) if rr else hqgen.table_rows(t, sf, seed)
         out = None
         if pinned and t == q.fact:
@@ -201,7 +202,7 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
     import torch
     import torch.distributed as dist
     from paper_conf_sigmod_funkebnmt18_b200 import hq
-    from paper_conf_sigmod_funkebnmt18_b200.dist import DistributedEngine, partition
+    from paper_conf_sigmod_funkebnmt18_b200.dist import DistributedEngine, partition, run_query
     from paper_conf_sigmod_funkebnmt18_b200.engine import Engine
     from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
 
@@ -210,8 +211,15 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
     n = hqgen.table_rows(q.fact, sf, seed)
     a, b = partition(n, rank, world)
     root = rank == 0
+    dist_mode = world > 1 or os.environ.get("HQ_FORCE_DIST") == "1"
+    # co-partitioned queries (TPC-H Q3): orders and lineitem partitioned together by order,
+    # every rank builds locally (dist.DistributedEngine copartitioned)
+    copart = dist_mode and q.copart is not None and os.environ.get("HQ_DIST_COPART", "1") == "1"
+    crange = None
+    if copart:
+        crange, (a, b) = hqgen.copartition(q.fact, q.copart, sf, rank, world, seed)
     if host is None:
-        host = gen_host(q, sf, seed, (a, b), with_dims=root or world == 1)
+        host = gen_host(q, sf, seed, (a, b), with_dims=root or world == 1 or copart, copart_range=crange)
     ctx = hq.Context(local)
     # HBM-resident copies (torch memory, borrowed by libhq)
     dtab = {t: {c: torch.from_numpy(np.asarray(arr)).to(dev) for c, arr in cols.items()} for t, cols in host.items()}
@@ -220,15 +228,14 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
 
     def make_engine(tbls):
         # HQ_FORCE_DIST=1 runs the distributed engine (broadcast + reduce) even at N=1
-        if world > 1 or os.environ.get("HQ_FORCE_DIST") == "1":
-            return DistributedEngine(ctx, tbls)
+        if dist_mode:
+            return DistributedEngine(ctx, tbls, copartitioned=copart)
         return Engine(ctx, tbls)
 
     E = make_engine(tables)
 
     def step(Eng):
-        res, pb = q.run(Eng)
-        return Eng.finish(res, pb)
+        return run_query(Eng, q)
 
     def barrier():
         if world > 1:
@@ -297,7 +304,7 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
            "local_rows": b - a, "result": out, "mode": mode, "step_ms_median": statistics.median(per),
            "step_ms_min": min(per), "eager": {"ms_per_step": ms_eager, "median": statistics.median(per_eager),
                                                "min": min(per_eager), "launches": launches_eager},
-           "prepared": prep}
+           "prepared": prep, "copart": copart}
     # ---- e2e: host (pinned) buffers through the public API, H2D inside the timed region.
     # Dimension tables are copied (HQ_HOST_COPY); the fact table streams from its pinned
     # host buffers through the fused kernel in blocks (HQ_HOST_STREAM, batch processing:
@@ -309,10 +316,9 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
         def e2e_step():
             tb = {t: ctx.load_columns(cols, stream=(t == q.fact)) for t, cols in host.items()}
             Eng = make_engine(tb)
-            r, pb = q.run(Eng)
-            o = Eng.finish(r, pb)
+            o = run_query(Eng, q)
             d2h = sum(c.nbytes for c in o.columns.values()) if o is not None else 0
-            del r, Eng, tb
+            del Eng, tb
             return d2h
 
         e2e_step()
@@ -438,7 +444,9 @@ def run_hq(args):
                 "config": {"workload": f"{args.query}_sf{args.sf:g}", "query": args.query, "sf": args.sf,
                            "fact_rows": r["rows"], "fact_bytes": r["rows"] * q.fact_bytes_per_row(),
                            "l2": "inputs larger than L2 (no flush needed)",
-                           "parallelism": f"fact range partition dp{world}, dimension HTs broadcast, 1 reduce",
+                           "parallelism": (f"orders/lineitem co-partitioned by order dp{world}, local builds, "
+                                           "top-k rows gathered" if r["copart"] else
+                                           f"fact range partition dp{world}, dimension HTs broadcast, 1 reduce"),
                            "step": "hash builds + fused pipeline + reduce + finalize/fetch",
                            "step_mode": r["mode"] + (" (CUDA graph of the whole step; every kernel re-executed per step)"
                                                      if r["mode"] == "prepared" else "")},

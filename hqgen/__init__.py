@@ -151,6 +151,9 @@ def lib():
                                    ctypes.POINTER(ctypes.c_void_p), ctypes.c_int]
         L.hqg_date_from_day.restype = ctypes.c_int32
         L.hqg_date_from_day.argtypes = [ctypes.c_int32]
+        L.hqg_line_row_of_order.restype = ctypes.c_int64
+        L.hqg_line_row_of_order.argtypes = [ctypes.c_int, ctypes.c_double, ctypes.c_uint64, ctypes.c_int64,
+                                            ctypes.c_int]
         _lib = L
     return _lib
 
@@ -164,6 +167,23 @@ def table_rows(table, sf: float, seed: int = DEFAULT_SEED, nthreads: int = 0) ->
     if n < 0:
         raise ValueError(f"bad table/sf {table} {sf}")
     return int(n)
+
+
+def line_row_of_order(table, sf: float, order: int, seed: int = DEFAULT_SEED, nthreads: int = 0) -> int:
+    """First row of order `order`'s lines in a line table (lineorder / lineitem)."""
+    r = lib().hqg_line_row_of_order(table_id(table), float(sf), int(seed), int(order), int(nthreads))
+    if r < 0:
+        raise ValueError(f"bad line table / sf / order {table} {sf} {order}")
+    return int(r)
+
+
+def copartition(line_table, order_table, sf: float, rank: int, world: int, seed: int = DEFAULT_SEED):
+    """Rank `rank`'s share of a line table and its order table partitioned together by
+    order (orderkey): ((order rows a, b), (line rows la, lb)) with the lines of orders
+    [a, b) exactly the line rows [la, lb)."""
+    no = table_rows(order_table, sf, seed)
+    a, b = no * rank // world, no * (rank + 1) // world
+    return (a, b), (line_row_of_order(line_table, sf, a, seed), line_row_of_order(line_table, sf, b, seed))
 
 
 def column_names(table) -> list:

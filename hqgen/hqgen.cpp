@@ -463,4 +463,17 @@ int hqg_generate(int table, double sf, uint64_t seed, int64_t a, int64_t b, int 
 
 int32_t hqg_date_from_day(int32_t d) { return yyyymmdd(d); }
 
+int64_t hqg_line_row_of_order(int table, double sf, uint64_t seed, int64_t order, int nthreads) {
+  // first line row of order `order` (== nrows for order == norders): the line tables are
+  // generated order by order, so [row_of(a), row_of(b)) holds exactly the lines of orders
+  // [a, b) -- a range partition of the line table aligned to one of the order table
+  if (!(sf > 0) || (table != HQG_SSB_LINEORDER && table != HQG_TPCH_LINEITEM)) return -1;
+  auto li = line_index(table, sf, seed, nthreads);
+  if (order < 0 || order > li->norders) return -1;
+  if (order == li->norders) return li->nrows;
+  int64_t c = order / kChunk, off = li->chunk_off[c];
+  for (int64_t i = c * kChunk; i < order; ++i) off += nlines(table, seed, i);
+  return off;
+}
+
 }  // extern "C"

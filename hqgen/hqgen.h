@@ -106,6 +106,13 @@ int hqg_generate(int table, double sf, uint64_t seed, int64_t row_begin, int64_t
 /* yyyymmdd of day d counted from 1992-01-01 (d=0). */
 int32_t hqg_date_from_day(int32_t d);
 
+/* First row of the lines of order `order` in a line table (SSB lineorder / TPC-H
+ * lineitem; order == number of orders gives the row count).  The line tables are
+ * generated order by order, so rows [row_of(a), row_of(b)) hold exactly the lines of
+ * orders [a, b): a partition of the line table co-aligned with one of the order
+ * table (multi-GPU co-partitioning by orderkey).  -1 on a bad table / sf / order. */
+int64_t hqg_line_row_of_order(int table, double sf, uint64_t seed, int64_t order, int nthreads);
+
 #ifdef __cplusplus
 }
 #endif

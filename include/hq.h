@@ -220,7 +220,8 @@ typedef struct {
   int32_t compact_kind; /* hq_hash_device_view / hq_hash_import: 0 = the buffer is the slot array; 1 / 2 / 3 =
                          * the buffer is the compact form of a direct table (1 bitmap of present keys, 2 one
                          * byte per key, 3 one nibble per key; see below) -- tables whose only consumers
-                         * read that form are built straight into it */
+                         * read that form are built straight into it; 4 = the ranked form of a linear
+                         * table (below; needs key_min / key_max / nkeys) */
 } hq_hash_meta;
 /* Derived forms (rebuilt on import): direct tables get a compact form -- a
  * bitmap of present keys for semi-join tables, or one byte per key (payload -
@@ -231,9 +232,17 @@ typedef struct {
  * keys detected by it); its slot array is derived only if a consumer that reads slots
  * (precompiled interpreter, operator-at-a-time) probes it.  hq_hash_device_view then
  * returns the compact form (meta.compact_kind != 0), which hq_hash_import accepts.
- * Linear tables whose key range fits in 64 MiB of bits get an exact key-range
- * bitmap that generated kernels test before touching the slot array (most probe
- * misses then never leave L2). */
+ * Sparse unique keys with a counted range that fits in 64 MiB of bits (layout
+ * HQ_HT_LINEAR) are built into the *ranked form* instead of a slot array: one buffer
+ * [bitmap of present keys over [key_min, key_max] | int32 rank directory, the number
+ * of keys before each 32-bit bitmap word | payload rows by rank, 1 / 2 / 4 int32
+ * words each (npayload 1 / 2 / 3; none without payload)], each part padded to whole
+ * 8,192-word blocks and 256-B aligned -- a probe tests the key's bit (misses stop
+ * there) and reads row dir[w] + popcount(bits below it).  The linear slot array the
+ * meta describes (capacity, slot_words, bytes) is derived only for consumers that
+ * read slots.  Other linear tables (expected_rows builds, composite keys, wider
+ * ranges) keep the slot array, with an exact key-range bitmap in front of it when
+ * the range fits in 64 MiB of bits. */
 hq_status hq_hash_info(hq_ctx* ctx, const hq_hash* h, hq_hash_meta* meta);  /* syncs, reports build faults */
 /* Multi-GPU glue: raw device view of the slot array (to broadcast it with NCCL)
  * and import of such a buffer on another device (borrowed, caller keeps it). */
@@ -405,6 +414,16 @@ hq_status hq_result_partials_view(hq_result* r, void** dev_ptr, size_t* bytes);
  * finalized yet; bytes must equal the view's size (HQ_ERR_ARG).  (The reduce itself
  * may also run in place on the view, which needs no call.) */
 hq_status hq_result_from_partials(hq_ctx* ctx, hq_result* r, const void* dev_ptr, size_t bytes);
+/* The reverse copy: the result's dense partials into the caller's device buffer
+ * dev_dst (bytes = the view's size, HQ_ERR_ARG otherwise), async on the ctx stream --
+ * e.g. into the [partials | fault words] buffer a multi-rank caller all-reduces, so no
+ * collective writes library memory. */
+hq_status hq_result_to_partials(hq_ctx* ctx, const hq_result* r, void* dev_dst, size_t bytes);
+/* Multi-GPU glue: copy the device views of n hash tables (hq_hash_device_view's
+ * buffers, meta.bytes each) into ONE caller buffer dev_dst at byte offsets offs[i]
+ * (host array; each 16-B aligned, the caller sized the buffer), async on the ctx
+ * stream -- the packed payload of a single table broadcast. */
+hq_status hq_hash_pack(hq_ctx* ctx, const hq_hash* const* hashes, int32_t n, const int64_t* offs, void* dev_dst);
 
 /* Fault words gathered on the device, without a host synchronisation, so that a
  * multi-rank caller can combine every rank's faults with the collective it runs

@@ -281,6 +281,7 @@ hq_status hq_graph_launch(hq_ctx* ctx, hq_graph* g) {
       r->host_ready = false;
       r->finalized = false;
       r->checked = false;
+      r->checked_counter = -1;
     }
     ctx->launches += g->nkernels;
     HQ_CUDA(cudaGraphLaunch(g->exec, ctx->stream));
@@ -484,6 +485,33 @@ hq_status hq_hash_import(hq_ctx* ctx, const hq_hash_meta* meta, void* dev_ptr, h
         (meta->slot_words == 1 && meta->npayload != 0))
       HQ_THROW(HQ_ERR_ARG, "import: npayload");
     if (((uintptr_t)dev_ptr & 15) != 0) HQ_THROW(HQ_ERR_ARG, "import: pointer must be 16-byte aligned");
+    if (meta->compact_kind == 4) {  // the ranked form of a sparse-key table (hq_build.cu)
+      const int64_t range = (int64_t)meta->key_max - meta->key_min + 1;
+      if (meta->layout != HQ_HT_LINEAR || meta->composite || meta->nkeys < 1 || range < 1 || range > (1LL << 31))
+        HQ_THROW(HQ_ERR_ARG, "import: a ranked form needs a linear, non-composite table with its key range and count");
+      int64_t od = 0, op = 0, tot = 0;
+      int stride = 0;
+      hq_ranked_layout(range, meta->nkeys, meta->npayload, &od, &op, &tot, &stride);
+      if (meta->bytes < tot) HQ_THROW(HQ_ERR_ARG, "import: ranked form too small");
+      hq_hash* h = new hq_hash();
+      h->ctx = ctx;
+      h->meta = *meta;
+      h->meta.compact_kind = 0;
+      h->meta.bytes = cap * meta->slot_words * 4;
+      h->compact_borrow = dev_ptr;
+      h->ckind = 4;
+      h->cbytes = tot;
+      h->roff_dir = od;
+      h->roff_pay = op;
+      h->rstride = stride;
+      h->compact_only = true;
+      int l = 0;
+      while ((1LL << l) < cap) ++l;
+      h->log2cap = l;
+      h->checked = true;
+      *out = h;
+      return;
+    }
     if (meta->compact_kind != 0) {  // a compact-only direct table: the buffer is its compact form
       if (meta->layout != HQ_HT_DIRECT ||
           meta->compact_kind != hq_compact_kind(meta->npayload, meta->pay_min, meta->pay_max))
@@ -663,6 +691,32 @@ hq_status hq_result_from_partials(hq_ctx* ctx, hq_result* r, const void* dev_ptr
     if (st != HQ_OK) HQ_THROW(st, g_last_error);
     if (bytes != n) HQ_THROW(HQ_ERR_ARG, "hq_result_from_partials: size differs from the partials view");
     if (p != dev_ptr && n > 0) HQ_CUDA(cudaMemcpyAsync(p, dev_ptr, n, cudaMemcpyDeviceToDevice, ctx->stream));
+  });
+}
+
+hq_status hq_result_to_partials(hq_ctx* ctx, const hq_result* r, void* dev_dst, size_t bytes) {
+  return guarded([&] {
+    if (!ctx || !r || !dev_dst) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    void* p = nullptr;
+    size_t n = 0;
+    const hq_status st = hq_result_partials_view(const_cast<hq_result*>(r), &p, &n);
+    if (st != HQ_OK) HQ_THROW(st, g_last_error);
+    if (bytes != n) HQ_THROW(HQ_ERR_ARG, "hq_result_to_partials: size differs from the partials view");
+    if (p != dev_dst && n > 0) HQ_CUDA(cudaMemcpyAsync(dev_dst, p, n, cudaMemcpyDeviceToDevice, ctx->stream));
+  });
+}
+
+hq_status hq_hash_pack(hq_ctx* ctx, const hq_hash* const* hashes, int32_t n, const int64_t* offs, void* dev_dst) {
+  return guarded([&] {
+    if (!ctx || n < 0 || (n > 0 && (!hashes || !offs || !dev_dst))) HQ_THROW(HQ_ERR_ARG, "NULL argument");
+    for (int i = 0; i < n; ++i) {
+      const hq_hash* h = hashes[i];
+      if (!h) HQ_THROW(HQ_ERR_ARG, "hq_hash_pack: NULL hash");
+      if (offs[i] < 0 || (offs[i] & 15)) HQ_THROW(HQ_ERR_ARG, "hq_hash_pack: offsets must be 16-B aligned");
+      const void* src = h->compact_only ? h->compact_ptr() : (const void*)h->slots;
+      const size_t bytes = (size_t)(h->compact_only ? h->cbytes : h->meta.bytes);
+      if (bytes) HQ_CUDA(cudaMemcpyAsync((char*)dev_dst + offs[i], src, bytes, cudaMemcpyDeviceToDevice, ctx->stream));
+    }
   });
 }
 

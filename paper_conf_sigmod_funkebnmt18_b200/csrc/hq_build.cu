@@ -9,6 +9,9 @@
 // by the claiming thread (readers only run in later kernels, stream-ordered).
 // Capacity: next_pow2(ceil(keys / 0.6)) >= 16, keys counted exactly by a
 // predicate-only count pass unless the caller supplies expected_rows.
+#include <cub/block/block_reduce.cuh>
+#include <cub/block/block_scan.cuh>
+
 #include <climits>
 
 #include "hq_internal.h"
@@ -318,6 +321,141 @@ __global__ void hq_fill_kernel(uint32_t* p, long long n, uint32_t v) {
     p[i] = v;
 }
 
+// ---- ranked form of a sparse-key table (hq_hash::ranked): the bitmap of
+// present keys over the key range (built by hq_build_direct_compact_kernel, kind 1), a
+// rank directory (keys before each bitmap word: an exclusive scan of the words' popcounts)
+// and the payload rows stored densely by rank.  It replaces a linear table's slot array,
+// its fill and its key-range prefilter: no CAS, no probe sequence, a probe that misses
+// reads one bitmap word and a hit one directory word and one payload row.
+constexpr int RSCAN_T = 1024, RSCAN_W = 8;  // directory scan: 8 words (two 16-B loads) per thread
+__device__ __forceinline__ void rank_words(const uint32_t* bm, long long base, uint32_t (&c)[RSCAN_W]) {
+  const uint4 a = __ldg((const uint4*)(bm + base)), b = __ldg((const uint4*)(bm + base) + 1);
+  c[0] = a.x; c[1] = a.y; c[2] = a.z; c[3] = a.w; c[4] = b.x; c[5] = b.y; c[6] = b.z; c[7] = b.w;
+}
+// per block (8,192 words): number of present keys
+__global__ void __launch_bounds__(RSCAN_T) hq_rank_blocksum_kernel(const uint32_t* bm, unsigned* bsum) {
+  uint32_t c[RSCAN_W];
+  rank_words(bm, ((long long)blockIdx.x * RSCAN_T + threadIdx.x) * RSCAN_W, c);
+  unsigned n = 0;
+#pragma unroll
+  for (int j = 0; j < RSCAN_W; ++j) n += __popc(c[j]);
+  typedef cub::BlockReduce<unsigned, RSCAN_T> BR;
+  __shared__ typename BR::TempStorage tmp;
+  const unsigned t = BR(tmp).Sum(n);
+  if (threadIdx.x == 0) bsum[blockIdx.x] = t;
+}
+// exclusive scan of the block sums (one block, chunks of 1,024 with a carry)
+__global__ void __launch_bounds__(RSCAN_T) hq_rank_topscan_kernel(unsigned* bsum, int n) {
+  typedef cub::BlockScan<unsigned, RSCAN_T> BS;
+  __shared__ typename BS::TempStorage tmp;
+  unsigned carry = 0;
+  for (int b = 0; b < n; b += RSCAN_T) {
+    const int i = b + (int)threadIdx.x;
+    unsigned v = i < n ? bsum[i] : 0u, ex, tot;
+    BS(tmp).ExclusiveSum(v, ex, tot);
+    if (i < n) bsum[i] = carry + ex;
+    carry += tot;
+    __syncthreads();  // tmp reuse
+  }
+}
+// directory: keys before each word = block offset + block-exclusive scan + running sum
+__global__ void __launch_bounds__(RSCAN_T) hq_rank_dir_kernel(const uint32_t* bm, const unsigned* bsum, unsigned* dir) {
+  const long long base = ((long long)blockIdx.x * RSCAN_T + threadIdx.x) * RSCAN_W;
+  uint32_t c[RSCAN_W];
+  rank_words(bm, base, c);
+  unsigned n = 0;
+#pragma unroll
+  for (int j = 0; j < RSCAN_W; ++j) n += __popc(c[j]);
+  typedef cub::BlockScan<unsigned, RSCAN_T> BS;
+  __shared__ typename BS::TempStorage tmp;
+  unsigned ex;
+  BS(tmp).ExclusiveSum(n, ex);
+  unsigned run = bsum[blockIdx.x] + ex, d[RSCAN_W];
+#pragma unroll
+  for (int j = 0; j < RSCAN_W; ++j) {
+    d[j] = run;
+    run += __popc(c[j]);
+  }
+  ((uint4*)(dir + base))[0] = make_uint4(d[0], d[1], d[2], d[3]);
+  ((uint4*)(dir + base))[1] = make_uint4(d[4], d[5], d[6], d[7]);
+}
+// payload rows by rank: each qualifying row finds its key's rank and writes its payloads
+__global__ void __launch_bounds__(BUILD_BLOCK) hq_build_ranked_scatter_kernel(const __grid_constant__ KBuild b,
+                                                                             const uint32_t* bm, const unsigned* dir,
+                                                                             int* rpay, int stride, long long range,
+                                                                             unsigned long long nkeys) {
+  int fault = 0;
+  const long long base = (long long)blockIdx.x * BUILD_BLOCK * BUILD_U + threadIdx.x;
+  bool pass[BUILD_U];
+  long long kv[BUILD_U], pv0[BUILD_U] = {};
+  int pay[BUILD_U][HQ_MAX_PAYLOAD] = {};
+  load_rows(b, base, pass, kv, pv0);
+#pragma unroll
+  for (int k = 0; k < HQ_MAX_PAYLOAD; ++k) {
+    if (k >= b.npay) break;
+    long long v[BUILD_U];
+    if (k == 0) {
+#pragma unroll
+      for (int u = 0; u < BUILD_U; ++u) v[u] = pv0[u];
+    } else {
+      ld_rows(b, b.pay_col[k], base, v);
+    }
+#pragma unroll
+    for (int u = 0; u < BUILD_U; ++u) pay[u][k] = (int)v[u];
+  }
+  unsigned rk[BUILD_U];
+  bool ok[BUILD_U];
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u) {  // the directory and bitmap loads of all U rows in flight together
+    const long long d = kv[u] - (long long)b.dmin;
+    ok[u] = pass[u] && kv[u] > (long long)INT_MIN && kv[u] <= (long long)INT_MAX && d >= 0 && d < range;
+    rk[u] = 0;
+    if (ok[u]) {
+      const uint32_t w = __ldg(bm + (d >> 5)), bit = 1u << (d & 31);
+      ok[u] = (w & bit) != 0;
+      rk[u] = __ldg(dir + (d >> 5)) + __popc(w & (bit - 1u));
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u) {
+    if (!ok[u]) continue;  // (bad keys and out-of-range keys were flagged by the bitmap pass)
+    if (rk[u] >= nkeys) {  // more keys than the (cached) statistics said: flagged stale by the bitmap pass
+      fault |= HQF_STALE;
+      continue;
+    }
+    int* dst = rpay + (size_t)rk[u] * stride;
+#pragma unroll
+    for (int k = 0; k < HQ_MAX_PAYLOAD; ++k)
+      if (k < b.npay) dst[k] = pay[u][k];
+  }
+  if (fault) atomicOr(b.err, fault);
+}
+// the linear slot array of a ranked table, for consumers that read slots (interpreter,
+// operator-at-a-time): every present key claims a slot as in hq_build_hash_kernel
+__global__ void hq_slots_from_ranked_kernel(const uint32_t* bm, const unsigned* dir, const int* rpay, int stride,
+                                            int npay, long long range, int kmin, uint32_t* slots, uint32_t mask,
+                                            int log2cap, int words, int* err) {
+  for (long long d = blockIdx.x * (long long)blockDim.x + threadIdx.x; d < range; d += (long long)gridDim.x * blockDim.x) {
+    const uint32_t w = bm[d >> 5], bit = 1u << (d & 31);
+    if (!(w & bit)) continue;
+    const int key = kmin + (int)d;
+    const int* src = stride ? rpay + (size_t)(dir[d >> 5] + __popc(w & (bit - 1u))) * stride : nullptr;
+    uint32_t pos = ((uint32_t)key * 0x9E3779B1u) >> (32 - log2cap);
+    for (uint32_t n = 0;; ++n) {
+      if (n > mask) {
+        atomicOr(err, HQF_HT_FULL);
+        break;
+      }
+      uint32_t* slot = slots + (size_t)pos * words;
+      if (atomicCAS((int*)slot, INT_MIN, key) == INT_MIN) {
+        for (int k = 0; k < npay; ++k) slot[1 + k] = (uint32_t)src[k];
+        break;
+      }
+      pos = (pos + 1) & mask;
+    }
+  }
+}
+
 __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid_constant__ KBuild b) {
   unsigned long long inserted = 0, qual = 0;
   int fault = 0;
@@ -462,6 +600,20 @@ int hq_compact_kind(int npayload, int pay_min, int pay_max) {
 }
 long long hq_compact_words(int kind, long long range) {
   return kind == 1 ? (range + 31) / 32 : (kind == 3 ? (range + 7) / 8 : (range + 3) / 4);
+}
+// ranked form: [bitmap | directory | payload rows], the bitmap and directory padded to
+// whole 8,192-word scan blocks (the scan kernels read and write them without bounds
+// checks; the bitmap's padding is zero), every part 256-B aligned; no directory or
+// payload rows for a table without payload (a semi / anti join reads the bitmap only)
+void hq_ranked_layout(int64_t range, int64_t nkeys, int npay, int64_t* off_dir, int64_t* off_pay, int64_t* total,
+                      int* stride) {
+  const int64_t blk = 1024 * 8;
+  const int64_t words = ((range + 31) / 32 + blk - 1) / blk * blk;
+  const int st = npay == 0 ? 0 : (npay == 1 ? 1 : (npay == 2 ? 2 : 4));
+  *stride = st;
+  *off_dir = words * 4;
+  *off_pay = *off_dir + (st ? words * 4 : 0);
+  *total = *off_pay + (int64_t)st * 4 * (nkeys > 0 ? nkeys : 0);
 }
 // rank LUT of a byte map over a sparse payload set (value - pay_min -> rank, 0xFF
 // absent); returns 1 when the map is rank-coded (the set is known and sparse)
@@ -624,7 +776,10 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   // derived from the statistics alone, so no slot array is written at all
   const int ckind = direct && bs.counted ? hq_compact_kind(d->npayload, bs.st.pmin, bs.st.pmax) : 0;
   const bool conly = ckind != 0 && !b.composite && !getenv("HQ_BUILD_SLOTS");
-  if (!conly) {
+  // sparse unique keys with a known range (counted): the ranked form instead of a slot array
+  const bool rform = !direct && !b.composite && bs.counted && keys > 0 && range > 0 &&
+                     (range + 31) / 32 * 4 <= (64LL << 20) && !getenv("HQ_BUILD_SLOTS");
+  if (!conly && !rform) {
     h->owned = DevBuf(ctx, (size_t)cap * words * 4);
     h->slots = h->owned.as<uint32_t>();
   }
@@ -634,11 +789,45 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   h->meta.npayload = d->npayload;
   h->meta.composite = b.composite;
   h->meta.nkeys = bs.counted ? keys : -1;  // exact after the count pass (confirmed at hq_hash_info)
+  h->src_rows = b.n;
   h->meta.bytes = cap * words * 4;
   h->meta.layout = direct ? HQ_HT_DIRECT : HQ_HT_LINEAR;
   h->meta.key_min = kmin;
   h->meta.key_max = range > 0 ? (int32_t)(kmin + range - 1) : (int32_t)kmin - 1;  // empty range when unknown
   h->stats_key = bs.stats_key;
+  if (rform) {
+    int64_t od = 0, op = 0, tot = 0;
+    int stride = 0;
+    hq_ranked_layout(range, keys, d->npayload, &od, &op, &tot, &stride);
+    h->compact = DevBuf(ctx, (size_t)tot + 16);
+    HQ_CUDA(cudaMemsetAsync(h->compact.p, 0, (size_t)od, ctx->stream));  // the bitmap and its padding
+    uint32_t* bm = h->compact.as<uint32_t>();
+    b.dmin = (int32_t)kmin;
+    if (b.n > 0) {  // bitmap + duplicate / bad-key / statistics checks
+      ctx->launches++;
+      hq_build_direct_compact_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b, 1, bm, range, 0, 0, CLut{});
+    }
+    HQ_CUDA(cudaGetLastError());
+    if (stride && b.n > 0) {
+      const int nblk = (int)(od / 4 / (RSCAN_T * RSCAN_W));
+      DevBuf bsum(ctx, (size_t)nblk * 4 + 16);
+      unsigned* dir = (unsigned*)(h->compact.as<char>() + od);
+      ctx->launches += 4;
+      hq_rank_blocksum_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, bsum.as<unsigned>());
+      hq_rank_topscan_kernel<<<1, RSCAN_T, 0, ctx->stream>>>(bsum.as<unsigned>(), nblk);
+      hq_rank_dir_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, bsum.as<unsigned>(), dir);
+      hq_build_ranked_scatter_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(
+          b, bm, dir, (int*)(h->compact.as<char>() + op), stride, range, (unsigned long long)keys);
+      HQ_CUDA(cudaGetLastError());
+    }
+    h->ckind = 4;
+    h->cbytes = tot;
+    h->roff_dir = od;
+    h->roff_pay = op;
+    h->rstride = stride;
+    h->compact_only = true;
+    return;
+  }
   if (conly) {
     const long long cwords = hq_compact_words(ckind, range);
     h->compact = DevBuf(ctx, (size_t)cwords * 4 + 16);
@@ -868,6 +1057,28 @@ void hq_build_compact(hq_ctx* ctx, hq_hash* h) {
 
 const uint32_t* hq_hash_slots(hq_ctx* ctx, hq_hash* h) {
   if (h->slots || !h->compact_only) return h->slots;
+  if (h->ranked()) {  // a linear slot array with the same capacity the meta describes
+    const long long cap = h->meta.capacity;
+    const int words = h->meta.slot_words;
+    h->owned = DevBuf(ctx, (size_t)cap * words * 4 + 16);
+    const int fgrid = (int)std::max<long long>(1, std::min<long long>((cap * words + 255) / 256, (long long)ctx->num_sms * 8));
+    const long long range = (long long)h->meta.key_max - h->meta.key_min + 1;
+    const int grid = (int)std::max<long long>(1, std::min<long long>((range + 255) / 256, (long long)ctx->num_sms * 8));
+    const char* base = (const char*)h->compact_ptr();
+    if (!h->dstate.p) {  // an imported table: a fault word for the derivation
+      h->dstate = DevBuf(ctx, 128);
+      HQ_CUDA(cudaMemsetAsync(h->dstate.p, 0, 128, ctx->stream));
+    }
+    ctx->launches += 2;
+    hq_fill_kernel<<<fgrid, 256, 0, ctx->stream>>>(h->owned.as<uint32_t>(), cap * words, 0x80000000u);
+    hq_slots_from_ranked_kernel<<<grid, 256, 0, ctx->stream>>>(
+        (const uint32_t*)base, (const unsigned*)(base + h->roff_dir), (const int*)(base + h->roff_pay), h->rstride,
+        h->meta.npayload, range, (int)h->meta.key_min, h->owned.as<uint32_t>(), (uint32_t)(cap - 1), h->log2cap, words,
+        h->dstate.as<int>());
+    HQ_CUDA(cudaGetLastError());
+    h->slots = h->owned.as<uint32_t>();
+    return h->slots;
+  }
   const long long range = h->meta.capacity;
   const int words = h->meta.slot_words;
   h->owned = DevBuf(ctx, (size_t)range * words * 4 + 16);

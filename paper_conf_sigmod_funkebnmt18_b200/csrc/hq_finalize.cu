@@ -898,9 +898,11 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered) {
   hq_check_result_faults(ctx, r);
   const hq_plan& P = r->plan;
   if (r->sink == HQ_SINK_MATERIALISE) {
-    unsigned long long cnt = 0;
-    HQ_CUDA(cudaMemcpyAsync(&cnt, r->dstate.p, 8, cudaMemcpyDeviceToHost, ctx->stream));
-    HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    unsigned long long cnt = (unsigned long long)r->checked_counter;  // read by the fault check
+    if (r->checked_counter < 0) {
+      HQ_CUDA(cudaMemcpyAsync(&cnt, r->dstate.p, 8, cudaMemcpyDeviceToHost, ctx->stream));
+      HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+    }
     r->qualifying = (int64_t)cnt;
     r->nrows = std::min<int64_t>((int64_t)cnt, r->capacity);
     r->ncols = P.nout;

@@ -233,7 +233,18 @@ struct hq_hash : RefObj {
   // linear tables: exact bitmap over [key_min, key_max] (prefilter before the slots)
   DevBuf prefilter;
   int64_t pf_words = 0;
+  // ckind 4 (compact_only): the *ranked* form of a sparse-key (linear) table, one buffer
+  // [bitmap of present keys over key_max - key_min + 1 | rank directory: int32 number of
+  // keys before each bitmap word | payload rows by rank, rstride int32 words each]
+  // (hq_ranked_layout); a key's payload row = dir[w] + popc(bitmap[w] below its bit)
+  int64_t src_rows = -1;  // rows of the build's source table (-1: imported / unknown)
+  int64_t roff_dir = 0, roff_pay = 0;
+  int rstride = 0;
+  bool ranked() const { return ckind == 4; }
 };
+// byte offsets of the ranked form's parts (and its size) for a key range / key count
+void hq_ranked_layout(int64_t range, int64_t nkeys, int npay, int64_t* off_dir, int64_t* off_pay, int64_t* total,
+                      int* stride);
 void hq_build_compact(hq_ctx* ctx, hq_hash* h);  // derive hq_hash::compact from the slots
 int hq_compact_kind(int npayload, int pay_min, int pay_max);
 long long hq_compact_words(int kind, long long range);
@@ -272,13 +283,14 @@ constexpr int SMEM_LANE_BYTES = 96 * 1024; // lane-private table budget
 struct KReg {
   uint32_t off;      // byte offset of row 0 in the stage (column) or tmp region (temporary)
   uint8_t width;     // 1, 4, 8
-  uint8_t in_stage;  // 1 = fact column staged by TMA, 0 = temporary
+  uint8_t in_stage;  // 1 = fact column staged by TMA, 2 = lazy fact column (global loads), 0 = temporary
   uint8_t pad[2];
 };
 struct KCol {
   const char* ptr;
   uint32_t width;
   uint32_t soff;     // byte offset inside a stage
+  uint32_t lazy;     // 1 = not streamed: the rows still live at its first use read it from global memory
 };
 struct KPred {
   int16_t reg;
@@ -307,12 +319,18 @@ struct KProbe {
   uint32_t smem_off; // generated kernels: byte offset of the staged compact table (0 = not staged)
   uint64_t pay_set[4];  // payload-0 values present, bit (v & 255) (hq_hash_meta::pay_set)
   float pass_est;      // expected fraction of probing rows that pass (key density of the build side)
+  float pass_src;      // the same over the build side's source rows (lazy-load decision)
   const uint32_t* pf;  // linear tables: key-range bitmap (NULL = none)
   int32_t pf_min;
   uint32_t pf_range;
   uint8_t composite;   // two-column key: slot word 1 must equal key2_reg; payloads from word 2
   int16_t key2_reg;
   uint8_t crank;       // ckind 2: the byte is the payload's RANK in pay_set (sparse value sets)
+  // ranked form of a linear table (hq_hash::ranked): pf = its bitmap, rdir = rank
+  // directory, rpay = payload rows (rstride words) by rank; slots unused
+  uint8_t ranked, rstride;
+  const uint32_t* rdir;
+  const int32_t* rpay;
 };
 struct KCompute {
   int16_t dst;
@@ -430,6 +448,7 @@ struct hq_result : RefObj {
   // finalized AGG rows
   bool finalized = false;
   bool checked = false;
+  int64_t checked_counter = -1;  // the output counter read by the fault check (materialise: row count)
   int64_t nrows = 0;
   int64_t qualifying = 0;
   int ncols = 0;

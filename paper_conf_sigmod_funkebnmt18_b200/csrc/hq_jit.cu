@@ -32,6 +32,8 @@ using namespace hqk;
     const unsigned* ht[8];                                                                                     \
     const void* ctab[8];                                                                                       \
     const unsigned* pf[8];                                                                                     \
+    const unsigned* rdir[8];                                                                                   \
+    const int* rpay[8];                                                                                        \
     long long* gtab;                                                                                           \
     unsigned long long gmask;                                                                                  \
     int glog2, pad;                                                                                            \
@@ -104,11 +106,15 @@ struct Gen {
   std::map<int, std::pair<long long, long long>> known;  // value range of probe payloads (count pass)
   std::map<int, int> stage_k;  // table column -> stage column index
   std::set<int> vec_loaded;    // stage columns read with ONE vector load per lane (all R rows)
+  std::map<int, int> lazy_k;   // lazy fact column register -> kernel column index
   explicit Gen(const KPlan& k) : kp(k) {
-    for (int c = 0; c < HQ_MAX_COLS; ++c) {
-      if (!kp.regs[c].in_stage || !kp.regs[c].width) continue;
-      for (int k2 = 0; k2 < kp.ncols; ++k2)
-        if (kp.cols[k2].soff == kp.regs[c].off) stage_k[c] = k2;
+    // kernel columns follow the fact columns in order (hq_build_kplan)
+    int k2 = 0;
+    for (int c = 0; c < HQ_MAX_COLS && k2 < kp.ncols; ++c) {
+      if (!kp.regs[c].width || !kp.regs[c].in_stage) continue;
+      if (kp.regs[c].in_stage == 2) lazy_k[c] = k2;
+      else stage_k[c] = k2;
+      ++k2;
     }
   }
   std::string var(int reg) const { return reg < HQ_MAX_COLS ? "c" + std::to_string(reg) : "t" + std::to_string(reg - HQ_MAX_COLS); }
@@ -129,6 +135,17 @@ struct Gen {
     if (dead.count(reg)) HQ_THROW(HQ_ERR_STATE, "jit: register used after compaction but not carried over");
     if (loaded.count(reg)) return;
     if (reg >= HQ_MAX_COLS) HQ_THROW(HQ_ERR_ARG, "jit: temporary read before definition");
+    auto lz = lazy_k.find(reg);
+    if (lz != lazy_k.end()) {  // lazy column: only the rows still live read it, from global memory
+      const KCol& c = kp.cols[lz->second];
+      sync_mask();
+      dvar(ctype(c.width), var(reg));
+      o << "#pragma unroll\n      for (int r = 0; r < R; ++r) " << var(reg) << "[r] = ((mask >> r) & 1u) ? __ldg((const "
+        << ctype(c.width) << "*)p.col[" << lz->second << "] + (tb_ + row0 + r)) : (" << ctype(c.width) << ")0;\n";
+      loaded.insert(reg);
+      vtype[reg] = ctype(c.width);
+      return;
+    }
     const KCol& c = kp.cols[stage_k.at(reg)];
     // a lane's R rows are consecutive (row0 .. row0 + R - 1): one vector load
     // when they span 8 or 16 bytes (stage columns are 16-B aligned)
@@ -346,10 +363,48 @@ struct Gen {
     live = LIVE_AL;
   }
 
+  // ranked sparse-key table (hq_hash::ranked): the key's bit in the range bitmap
+  // (misses stop here, L2-resident), then for a hit that needs payloads its rank =
+  // directory word + popcount of the bits below it, and the payload row at that rank;
+  // each step's loads for the lane's R rows are issued together
+  void probe_ranked(const KProbe& pr, int idx) {
+    const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
+    probe_defs(pr);
+    const std::string key = val(pr.key_reg), I = std::to_string(idx);
+    o << "      { u32 found_ = 0u; u32 w_[R]; u32 e_[R]; bool h_[R];\n"
+      << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n"
+      << "          const long long d_ = (long long)" << key << " - (" << pr.pf_min << "LL); e_[r] = (u32)d_;\n"
+      << "          h_[r] = ((mask >> r) & 1u) && d_ >= 0 && d_ < " << pr.pf_range << "LL;\n"
+      << "          w_[r] = h_[r] ? __ldg(p.pf[" << I << "] + (e_[r] >> 5)) : 0u; }\n"
+      << "#pragma unroll\n        for (int r = 0; r < R; ++r) { h_[r] = (w_[r] >> (e_[r] & 31u)) & 1u;"
+      << " if (h_[r]) found_ |= 1u << r; }\n";
+    if (npay > 0) {
+      static const char* comp[4] = {"x", "y", "z", "w"};
+      o << "        u32 k_[R];\n"
+        << "#pragma unroll\n        for (int r = 0; r < R; ++r) if (h_[r]) k_[r] = __ldg(p.rdir[" << I
+        << "] + (e_[r] >> 5)) + __popc(w_[r] & ((1u << (e_[r] & 31u)) - 1u));\n"
+        << "#pragma unroll\n        for (int r = 0; r < R; ++r) if (h_[r]) {";
+      if (pr.rstride == 1) {
+        o << " " << var(pr.dst[0]) << "[r] = __ldg(p.rpay[" << I << "] + k_[r]);";
+      } else {
+        o << " const " << (pr.rstride == 2 ? "int2" : "int4") << " q_ = __ldg((const " << (pr.rstride == 2 ? "int2" : "int4")
+          << "*)p.rpay[" << I << "] + k_[r]);";
+        for (int k = 0; k < npay; ++k) o << " " << var(pr.dst[k]) << "[r] = q_." << comp[k] << ";";
+      }
+      o << " }\n";
+    }
+    o << "        mask = " << mask_after(pr) << "; }\n";
+    mask_written();
+  }
+
   // linear-probing table (sparse keys): optional exact key-range bitmap, then
   // 16-B group scans until the key or an empty slot
   void probe_linear(const KProbe& pr, int idx) {
     sync_mask();
+    if (pr.ranked) {
+      probe_ranked(pr, idx);
+      return;
+    }
     const int W = pr.words;
     const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
     probe_defs(pr);
@@ -833,7 +888,10 @@ std::string generate(const KPlan& kp) {
         // split and run the rest of the kernel at half speed.  Otherwise rows
         // of equal keys are combined in registers first (match_any + reduce).
         o << "      u32 act_[R]; int nact_ = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { act_[r] = __ballot_sync(HQ_FULL, (mask >> r) & 1u); nact_ += __popc(act_[r]); }\n"
-          << "      if (SCOPIES > 1 || nact_ <= 4 * R) {  // replicated tables: every live lane updates directly\n"
+          // replicated tables, few live rows, or a dense shared domain of >= 1,024 groups
+          // (keys rarely repeat inside a warp: match_any would find 32 singletons)
+          << "      if (SCOPIES > 1 || nact_ <= 4 * R" << (kp.smode == SM_DENSE && kp.smem_cap >= 1024 ? " || true" : "")
+          << ") {  // every live lane updates directly\n"
           // a lane's consecutive rows of one group (clustered keys: the lines of
           // an order) are folded first: one table update instead of a chain of
           // dependent global round trips (TPC-H Q3)
@@ -948,6 +1006,7 @@ std::string generate(const KPlan& kp) {
     << "        char* st = stages + (size_t)s * STAGE_STRIDE;\n"
     << "        if (t0 >= p.row_begin && t0 + T <= p.row_end) {\n          mbar_expect_tx(&full[s], STAGE_BYTES);\n";
   for (int k = 0; k < kp.ncols; ++k)
+    if (!kp.cols[k].lazy)
     o << "          tma_load_1d(st + " << kp.cols[k].soff << "u, p.col[" << k << "] + t0 * " << kp.cols[k].width << ", "
       << kp.tile_rows * kp.cols[k].width << "u, &full[s], pol);\n";
   o << "        } else mbar_arrive(&full[s]);\n        if (++s == S) { s = 0; ph ^= 1u; }\n      }\n";
@@ -973,7 +1032,7 @@ std::string generate(const KPlan& kp) {
   // declared once per tile parity (a / b, renamed with #define).
   int swp_split = -1;
   if (!mp && !c2 && !we && (sk == 0 || sk == 1) && kp.R == 2 && kp.smode != SM_LANE && !prof &&
-      !(wm && std::string(wm) == "sleep") && getenv("HQ_JIT_SWP") && getenv("HQ_JIT_SWP")[0] == '1') {
+      !(wm && std::string(wm) == "sleep") && g.lazy_k.empty() && getenv("HQ_JIT_SWP") && getenv("HQ_JIT_SWP")[0] == '1') {
     // opt-in: measured on B200 it LOSES (SSB Q3.1 SF30 0.56 -> 0.73 ms, Q4.1 SF100
     // 2.50 -> 3.29 ms): holding two stages per warp starves the 3-stage TMA ring and
     // the second tile's arrays spill at 64 registers; kept for experiments
@@ -1001,6 +1060,7 @@ std::string generate(const KPlan& kp) {
       << "        const int hi = (int)(p.row_end - tt_ < T ? p.row_end - tt_ : T);\n"
       << "        mask = 0;\n#pragma unroll\n        for (int r = 0; r < R; ++r) { const int row = row0 + r; if (row >= lo && row < hi) mask |= 1u << r; }\n";
     for (int k = 0; k < kp.ncols; ++k) {
+      if (kp.cols[k].lazy) continue;
       const char* ty = ctype(kp.cols[k].width);
       o << "#pragma unroll\n        for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r; ((" << ty
         << "*)(st + " << kp.cols[k].soff << "u))[row] = ((const " << ty << "*)p.col[" << k << "])[tt_ + row]; }\n";
@@ -1083,6 +1143,7 @@ std::string generate(const KPlan& kp) {
     << "      const int hi = (int)(p.row_end - t0 < T ? p.row_end - t0 : T);\n"
     << "      mask = 0;\n#pragma unroll\n      for (int r = 0; r < R; ++r) { const int row = row0 + r; if (row >= lo && row < hi) mask |= 1u << r; }\n";
   for (int k = 0; k < kp.ncols; ++k) {
+    if (kp.cols[k].lazy) continue;
     const char* ty = ctype(kp.cols[k].width);
     o << "#pragma unroll\n      for (int r = 0; r < R; ++r) if (mask & (1u << r)) { const int row = row0 + r; ((" << ty
       << "*)(st + " << kp.cols[k].soff << "u))[row] = ((const " << ty << "*)p.col[" << k << "])[t0 + row]; }\n";
@@ -1415,6 +1476,8 @@ std::string plan_key(const KPlan& kp) {
     pr.slots = (const uint32_t*)nz(pr.slots);
     pr.compact = nz(pr.compact);
     pr.pf = (const uint32_t*)nz(pr.pf);
+    pr.rdir = (const uint32_t*)nz(pr.rdir);
+    pr.rpay = (const int32_t*)nz(pr.rpay);
   }
   k.gtab = (long long*)nz(k.gtab);
   for (auto& o : k.out_ptr) o = (void*)nz(o);
@@ -1455,6 +1518,8 @@ void hq_jit_launch(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
     jp.ht[i] = kp.probes[i].slots;
     jp.ctab[i] = kp.probes[i].compact;
     jp.pf[i] = kp.probes[i].pf;
+    jp.rdir[i] = kp.probes[i].rdir;
+    jp.rpay[i] = kp.probes[i].rpay;
   }
   jp.gtab = kp.gtab;
   jp.gmask = kp.gmask;

@@ -128,21 +128,42 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.mask = pr.direct ? (uint32_t)op.ht->meta.capacity : (uint32_t)(op.ht->meta.capacity - 1);
       pr.dmin = (int32_t)op.ht->meta.key_min;
       pr.log2cap = (uint8_t)op.ht->log2cap;
-      pr.ckind = (uint8_t)op.ht->ckind;
+      // a ranked sparse-key table (hq_hash::ranked): generated kernels probe its bitmap,
+      // directory and payload rows; the other executions its derived slot array
+      const bool rk = op.ht->ranked();
+      pr.ranked = (uint8_t)(jit && rk);
+      pr.ckind = rk ? 0 : (uint8_t)op.ht->ckind;
       pr.crank = (uint8_t)op.ht->crank;
-      pr.compact = op.ht->compact_ptr();
+      pr.compact = rk ? nullptr : op.ht->compact_ptr();
+      pr.rstride = (uint8_t)op.ht->rstride;
+      pr.rdir = nullptr;
+      pr.rpay = nullptr;
       pr.pay_min = op.ht->meta.pay_min;
       pr.pay_max = op.ht->meta.pay_max;
       for (int k = 0; k < 4; ++k) pr.pay_set[k] = op.ht->meta.pay_set[k];
-      {  // uniform foreign keys over the key range: pass fraction = key density (anti: the rest)
+      {  // uniform foreign keys over the key range: pass fraction = key density (anti: the rest);
+         // pass_src: over the build side's source rows (star joins: qualifying / all dimension
+         // rows -- SSB Q1.2's date table, 31 of 2,557 days, is dense over its own key range)
         const double range = (double)op.ht->meta.key_max - (double)op.ht->meta.key_min + 1.0;
         double est = (op.ht->meta.nkeys >= 0 && range >= 1.0) ? (double)op.ht->meta.nkeys / range : 1.0;
         est = est > 1.0 ? 1.0 : est;
+        double src = est;
+        if (op.ht->meta.nkeys >= 0 && op.ht->src_rows > 0)
+          src = std::min(est, (double)op.ht->meta.nkeys / (double)op.ht->src_rows);
         pr.pass_est = (float)(op.mode == HQ_PROBE_ANTI ? 1.0 - est : (op.mode == HQ_PROBE_OUTER ? 1.0 : est));
+        pr.pass_src = (float)(op.mode == HQ_PROBE_ANTI ? 1.0 - src : (op.mode == HQ_PROBE_OUTER ? 1.0 : src));
       }
-      pr.cbytes = (uint32_t)op.ht->cbytes;
+      pr.cbytes = rk ? 0u : (uint32_t)op.ht->cbytes;
       pr.smem_off = 0;
       pr.pf = op.ht->pf_words ? op.ht->prefilter.as<uint32_t>() : nullptr;
+      if (pr.ranked) {
+        const char* base = (const char*)op.ht->compact_ptr();
+        pr.pf = (const uint32_t*)base;
+        if (pr.rstride) {
+          pr.rdir = (const uint32_t*)(base + op.ht->roff_dir);
+          pr.rpay = (const int32_t*)(base + op.ht->roff_pay);
+        }
+      }
       pr.pf_min = (int32_t)op.ht->meta.key_min;
       pr.pf_range = (uint32_t)((int64_t)op.ht->meta.key_max - op.ht->meta.key_min + 1);
       pr.words = (uint8_t)op.ht->meta.slot_words;
@@ -484,11 +505,58 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     agg_smem = 0;
   }
 
+  // ---- lazy columns (generated kernels): a fact column first read where only a few rows
+  // are still expected to be live (the paper's lazy loading, Table 3) is not
+  // streamed; the live rows read it from global memory at its first use.  Expected
+  // survival before op i = product of the earlier ops' estimates (probe: build-side key
+  // density; filter: 1/2; compute: 1); lazy when <= 15 %.
+  bool lazy[HQ_MAX_COLS] = {false};
+  if (jit && !mp_pass && !getenv("HQ_JIT_NOLAZY")) {
+    int first[HQ_MAX_COLS];
+    for (int c = 0; c < HQ_MAX_COLS; ++c) first[c] = -1;
+    auto mark = [&](int reg, int at) {
+      if (reg >= 0 && reg < F->ncols && first[reg] < 0) first[reg] = at;
+    };
+    for (int o = 0; o < kp.nops; ++o) {
+      const KOp& op = kp.ops[o];
+      if (op.kind == OP_FILTER) mark(kp.preds[op.idx].reg, o);
+      else if (op.kind == OP_PROBE) {
+        mark(kp.probes[op.idx].key_reg, o);
+        if (kp.probes[op.idx].composite) mark(kp.probes[op.idx].key2_reg, o);
+      } else {
+        const KCompute& c = kp.comps[op.idx];
+        for (int k = 0; k < c.n; ++k) mark(kp.insns[c.first + k].reg, o);
+      }
+    }
+    for (int c = 0; c < F->ncols; ++c)
+      if (col_used[c] && first[c] < 0) first[c] = kp.nops;  // read by the sink only
+    double est[HQ_MAX_OPS + 1];
+    est[0] = 1.0;
+    for (int o = 0; o < kp.nops; ++o) {
+      const KOp& op = kp.ops[o];
+      const double e = op.kind == OP_FILTER ? 0.5 : (op.kind == OP_PROBE ? (double)kp.probes[op.idx].pass_src : 1.0);
+      est[o + 1] = est[o] * e;
+    }
+    // only where the rows wait on no global-memory probe: a lazy load is one more
+    // dependent DRAM round trip per tile, which HBM-bound pipelines hide (TPC-H Q6 SF10
+    // 0.248 -> 0.196 ms) but latency-bound star joins do not (SSB Q3.1 SF30 0.56 -> 0.97,
+    // Q4.1 SF100 2.48 -> 3.45 ms, measured)
+    uint64_t ctab = 0;
+    bool stageable = true;
+    for (int q = 0; q < nprobe; ++q) {
+      const KProbe& pr = kp.probes[q];
+      stageable = stageable && pr.direct && pr.ckind;
+      ctab += (pr.cbytes + 127) / 128 * 128;
+    }
+    stageable = stageable && ctab <= 64 * 1024;
+    for (int c = 0; c < F->ncols; ++c)
+      lazy[c] = stageable && col_used[c] && first[c] > 0 && est[first[c]] <= 0.15;
+  }
   // ---- stage layout: only referenced columns are streamed
   kp.ncols = 0;
   uint32_t rowbytes = 0;
   for (int c = 0; c < ncols_all; ++c) {
-    if (!col_used[c]) continue;
+    if (!col_used[c] || lazy[c]) continue;
     // (host-streamed columns are copied into 256-B aligned ring slots)
     if (!F->host_stream && ((uintptr_t)colptr[c] & 15) != 0) HQ_THROW(HQ_ERR_ARG, "column pointer not 16-byte aligned");
     rowbytes += (uint32_t)colw[c];
@@ -536,7 +604,15 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   // lane, and R = 4 applies only when the ring still holds 3 stages with every
   // table staged (SSB Q3.1 at R = 4 lost its staged tables: 0.61 -> 1.85 ms).
   bool prefer4 = false;
-  if (jit && force_R == 2 && !getenv("HQ_JIT_R") && !we) {
+  if (jit && force_R == 2 && !getenv("HQ_JIT_R") && !we && P.sink == HQ_SINK_MATERIALISE) {
+    // A3 behind a global probe: its per-tile barriers wait for the slowest warp's probe,
+    // so fewer, larger tiles pay (TPC-H Q3 SF30 orders side 0.367 -> 0.336 ms, SSB Q3.1
+    // materialised 1.165 -> 0.98 ms at 4 rows per lane, measured)
+    prefer4 = true;
+  } else if (jit && force_R == 2 && !getenv("HQ_JIT_R") && !we && !(P.sink == HQ_SINK_AGG && P.nkeys > 0)) {
+    // (not for group-by sinks: their R >= 4 path compacts the live rows of a warp
+    // before the table updates, pure overhead when every row is live -- Exp 2 with
+    // 32-512 groups 0.115 ms at R = 2 vs 1.1-1.25 ms at R = 4, measured)
     prefer4 = true;
     for (int o = 0; o < kp.nops; ++o) {
       if (kp.ops[o].kind != OP_PROBE) continue;
@@ -633,6 +709,13 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     KCol& kc = kp.cols[kp.ncols++];
     kc.ptr = colptr[c];
     kc.width = (uint32_t)colw[c];
+    if (lazy[c]) {  // read from global memory, not staged
+      if (((uintptr_t)colptr[c] & 15) != 0 && !F->host_stream) HQ_THROW(HQ_ERR_ARG, "column pointer not 16-byte aligned");
+      kc.soff = 0;
+      kc.lazy = 1;
+      kp.regs[c] = {0, (uint8_t)kc.width, 2, {0, 0}};
+      continue;
+    }
     kc.soff = soff;
     kp.regs[c] = {soff, (uint8_t)kc.width, 1, {0, 0}};
     soff += T * kc.width;
@@ -745,42 +828,53 @@ void hq_prepare_result(hq_ctx* ctx, const hq_plan* plan, hq_result* r) {
 
 // Sync, read the device fault bits; re-run once with the exact size when an
 // output capacity or group table overflowed (SURVEY.md §5 failure handling).
-// Build faults of the hash tables a result probed (duplicate keys, stale cached
-// statistics, ...): one gather of their fault words and one read; raised through
-// hq_hash_check (which names the fault) when any is set.
-static void check_result_hashes(hq_ctx* ctx, hq_result* r) {
-  std::vector<const int*> hw;
-  for (hq_hash* h : r->hashes)
-    if (h->dstate.p && !h->checked) hw.push_back(h->dstate.as<int>());
-  if (hw.empty()) return;
-  DevBuf out(ctx, 32 * 8);
-  hq_launch_gather_faults(ctx, hw, {}, out.as<long long>());
-  long long w[32];
-  HQ_CUDA(cudaMemcpyAsync(w, out.p, sizeof(w), cudaMemcpyDeviceToHost, ctx->stream));
-  HQ_CUDA(cudaStreamSynchronize(ctx->stream));
-  bool any = false;
-  for (int k = 0; k < 16; ++k) any = any || w[k] != 0;
-  if (!any) return;
-  for (hq_hash* h : r->hashes)
-    if (h->dstate.p) hq_hash_check(ctx, h);
-}
-
+// Faults of a result: the build faults of the hash tables it probed (duplicate keys,
+// stale cached statistics, ...; gathered on the device) and its own pipeline's fault
+// word and output counter, read back together with ONE host synchronisation; a build
+// fault is raised through hq_hash_check (which names it).  Capacity faults re-run the
+// pipeline with larger outputs and read again.
 void hq_check_result_faults(hq_ctx* ctx, hq_result* r) {
   if (r->checked) return;
   hq_require_eager(ctx, "a result's fault check");
-  check_result_hashes(ctx, r);
+  std::vector<const int*> hw;
+  for (hq_hash* h : r->hashes)
+    if (h->dstate.p && !h->checked) hw.push_back(h->dstate.as<int>());
   for (int attempt = 0;; ++attempt) {
-    struct { unsigned long long counter; int err; int pad; } st{};
-    HQ_CUDA(cudaMemcpyAsync(&st, r->dstate.p, sizeof(st), cudaMemcpyDeviceToHost, ctx->stream));
+    struct St {
+      unsigned long long counter;
+      int err;
+      int pad;
+      long long hw[32];
+    };
+    St* st = (St*)pinned_staging(ctx, sizeof(St));
+    DevBuf out;
+    const bool gather = attempt == 0 && !hw.empty();
+    if (gather) {
+      out = DevBuf(ctx, 32 * 8);
+      hq_launch_gather_faults(ctx, hw, {}, out.as<long long>());
+      HQ_CUDA(cudaMemcpyAsync(st->hw, out.p, 32 * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    }
+    HQ_CUDA(cudaMemcpyAsync(st, r->dstate.p, 16, cudaMemcpyDeviceToHost, ctx->stream));
     HQ_CUDA(cudaStreamSynchronize(ctx->stream));
-    const int err = st.err;
+    if (gather) {
+      bool any = false;
+      for (int k = 0; k < 16; ++k) any = any || st->hw[k] != 0;
+      if (any)
+        for (hq_hash* h : r->hashes)
+          if (h->dstate.p) hq_hash_check(ctx, h);
+    }
+    const int err = st->err;
+    const unsigned long long counter = st->counter;
     if (err & HQF_DIV_ZERO) HQ_THROW(HQ_ERR_ARG, "pipeline: division by zero");
     if (err & HQF_KEY_DOMAIN) HQ_THROW(HQ_ERR_ARG, "pipeline: group key outside its declared [min, min+card)");
     const bool fixable = (err & (HQF_CAPACITY | HQF_GROUP_FULL)) != 0;
-    if (!fixable) break;
+    if (!fixable) {
+      r->checked_counter = (int64_t)counter;
+      break;
+    }
     if (attempt >= 3 || r->plan.exec == HQ_EXEC_OAAT) HQ_THROW(HQ_ERR_OVERFLOW, "pipeline: capacity exceeded");
     if (r->plan.exec == HQ_EXEC_MULTIPASS) hq_run_multipass(ctx, &r->plan, r, r->ngroups * 4);
-    else if (err & HQF_CAPACITY) launch_pipeline(ctx, r, 0, (int64_t)st.counter);
+    else if (err & HQF_CAPACITY) launch_pipeline(ctx, r, 0, (int64_t)counter);
     else launch_pipeline(ctx, r, r->ngroups * 4, 0);
   }
   r->checked = true;

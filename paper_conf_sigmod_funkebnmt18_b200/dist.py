@@ -8,7 +8,13 @@
   on the root only;
 * each rank runs the fused pipeline over its range; dense partial aggregates
   ([count, agg...] per group, int64) are combined with ONE ``dist.reduce``
-  (SUM) to the root, which finalizes (ORDER BY / LIMIT on GPU 0).
+  (SUM) to the root, which finalizes (ORDER BY / LIMIT on GPU 0);
+* co-partitioned queries (``Query.copart``, TPC-H Q3): the order table and the line
+  table are partitioned together by order (``hqgen.copartition``: rank r's lines are
+  exactly the lines of its orders), every rank builds all of its tables locally (no
+  broadcast: the orders table a rank probes holds only its own orders), its groups --
+  keyed by the orderkey -- are disjoint from the other ranks', so ORDER BY / LIMIT run
+  per rank and only the ranks' top-k rows are gathered and merged on the root.
 
 The collectives here are backend-agnostic torch.distributed calls (NCCL on the
 GPUs; the CPU tests drive the same functions with gloo and a test-only
@@ -21,6 +27,7 @@ import os
 import sys
 from typing import List, Optional, Sequence, Tuple
 
+import numpy as np
 import torch
 import torch.distributed as dist
 
@@ -31,6 +38,18 @@ from .engine import Engine, PlanBuilder, QueryResult, fetch
 def partition(n: int, rank: int, world: int) -> Tuple[int, int]:
     """Row range of `rank` in a range partition of n rows over `world` ranks."""
     return n * rank // world, n * (rank + 1) // world
+
+
+def run_query(E: Engine, q) -> Optional[QueryResult]:
+    """One query through an Engine or DistributedEngine: q.run + finish, with the
+    co-partitioned abort protocol (a rank that raises joins the status collective)."""
+    try:
+        res, pb = q.run(E)
+    except hq.HQError as e:
+        if isinstance(E, DistributedEngine) and E.copartitioned:
+            E.abort(e)
+        raise
+    return E.finish(res, pb)
 
 
 def _i64(u: int) -> int:
@@ -72,49 +91,107 @@ def _offsets(rows: Sequence[Sequence[int]]) -> Tuple[List[int], int]:
     return offs, tot
 
 
-def broadcast_tables(rows: Optional[List[List[int]]], bufs: Optional[List[torch.Tensor]], n: int, root: int,
-                     device, err: Optional[BaseException] = None) -> Tuple[List[List[int]], List[torch.Tensor]]:
-    """Broadcast n root-built tables with TWO collectives: an (n+1) x 16 int64 metadata
-    block (row n = the root's status: error code or 0), then ONE byte buffer holding every
-    slot array at 256-B aligned offsets (the root packs them with device copies; the
-    other ranks get views into it).  Root: rows / bufs given; other ranks: None.  A
+# The step's collectives go straight to the default process group (its broadcast /
+# allreduce methods): the torch.distributed wrappers (argument checks, the c10d logger)
+# cost ~50-100 us of host time per call, which a step's critical path pays (the table
+# broadcast sits between the builds and the pipeline launch).  Same semantics as the
+# synchronous dist.* calls: work.wait() makes the current stream wait for the collective.
+def _pg():
+    return dist.distributed_c10d._get_default_group()
+
+
+def _broadcast(t: torch.Tensor, src: int) -> None:
+    opts = dist.BroadcastOptions()
+    opts.rootRank = src
+    opts.rootTensor = 0
+    _pg().broadcast([t], opts).wait()
+
+
+def _all_reduce(t: torch.Tensor, op=dist.ReduceOp.SUM) -> None:
+    opts = dist.AllreduceOptions()
+    opts.reduceOp = op
+    _pg().allreduce([t], opts).wait()
+
+
+def _align(x: int, a: int = 256) -> int:
+    return (x + a - 1) // a * a
+
+
+def broadcast_tables(rows: Optional[List[List[int]]], pack, n: int, root: int, device,
+                     err: Optional[BaseException] = None, state: Optional[dict] = None
+                     ) -> Tuple[List[List[int]], List[torch.Tensor]]:
+    """Broadcast n root-built tables, normally with ONE collective: a byte buffer
+    [(n+1) x 16 int64 metadata (row n = the root's status) | every table's buffer at a
+    256-B aligned offset].  The other ranks size their receive buffer from ``state``
+    (the largest message so far, the same on every rank); when the root's message is
+    larger, the first broadcast carries only the metadata with the new size in row n,
+    and a second one the whole message.  Root: rows and ``pack`` given -- a list of
+    tensors, or a callable(dev_ptr, offsets) that copies the tables into the buffer
+    (hq_hash_pack); other ranks: None (they get views into the received buffer).  A
     root-side error is broadcast before the root re-raises it, so the other ranks raise
     RootError instead of blocking in the next collective."""
     rank = dist.get_rank()
-    meta = torch.zeros((n + 1, META_COLS), dtype=torch.int64, device=device)
+    st = state if state is not None else {}
+    hdr = _align((n + 1) * META_COLS * 8)
+    first = max(int(st.get("cap", 0)), hdr)
     if rank == root:
+        offs, tot = _offsets(rows) if (err is None and n) else ([], 0)
+        need = hdr + tot
+        grow = need > first
+        meta = np.zeros((n + 1, META_COLS), dtype=np.int64)
         if err is not None:
             meta[n, 0] = getattr(err, "code", hq.HQ_ERR_STATE) or hq.HQ_ERR_STATE
         elif n:
-            meta[:n] = torch.tensor(rows, dtype=torch.int64)
-    dist.broadcast(meta, src=root)
-    if rank == root:
+            meta[:n] = np.asarray(rows, dtype=np.int64)
+            meta[n, 1] = need if grow else 0
+        buf = torch.empty(max(first, need), dtype=torch.uint8, device=device)
+        host = torch.from_numpy(meta.view(np.uint8).ravel())
+        if buf.is_cuda:  # pinned staging, reused (steps synchronise before the next call)
+            ph = st.get("pinned")
+            if ph is None or ph.numel() < host.numel():
+                ph = st["pinned"] = torch.empty(max(host.numel(), 4096), dtype=torch.uint8, pin_memory=True)
+            ph[:host.numel()].copy_(host)
+            host = ph[:host.numel()]
+        buf[:host.numel()].copy_(host, non_blocking=True)
+
+        def fill():
+            base = hdr
+            if callable(pack):
+                pack(buf.data_ptr() + base, offs)
+            else:
+                for o, b in zip(offs, pack):
+                    buf[base + o:base + o + b.numel()].copy_(b.reshape(-1).view(torch.uint8))
+        if err is None and n and not grow:
+            fill()
+        _broadcast(buf[:first], root)
         if err is not None:
             raise err
-        if n == 0:
-            return rows, bufs
-        offs, tot = _offsets(rows)
-        packed = torch.empty(tot, dtype=torch.uint8, device=device)
-        for o, b in zip(offs, bufs):
-            packed[o:o + b.numel()].copy_(b)
-        dist.broadcast(packed, src=root)
-        return rows, bufs
-    m = meta.cpu().tolist()
+        if grow:
+            fill()
+            _broadcast(buf[:need], root)
+            st["cap"] = need
+        return rows, ([] if not n else list(pack) if not callable(pack) else [])
+    buf = torch.empty(first, dtype=torch.uint8, device=device)
+    _broadcast(buf, root)
+    m = buf[:(n + 1) * META_COLS * 8].view(torch.int64).reshape(n + 1, META_COLS).cpu().tolist()
     if m[n][0] != 0:
         raise RootError(int(m[n][0]), "hash build failed on the root rank")
     rows = m[:n]
     if n == 0:
         return rows, []
-    offs, tot = _offsets(rows)
-    packed = torch.empty(tot, dtype=torch.uint8, device=device)
-    dist.broadcast(packed, src=root)
-    return rows, [packed[o:o + int(r[4])] for o, r in zip(offs, rows)]
+    need = int(m[n][1])
+    if need:
+        buf = torch.empty(need, dtype=torch.uint8, device=device)
+        _broadcast(buf, root)
+        st["cap"] = need
+    offs, _ = _offsets(rows)
+    return rows, [buf[hdr + o:hdr + o + int(r[4])] for o, r in zip(offs, rows)]
 
 
 def reduce_partials(t: torch.Tensor, root: int) -> None:
     """Exact integer SUM of the ranks' partial aggregates (one all-reduce: NCCL
     over NVLink on the GPUs; gloo in the CPU tests).  Only the root finalizes."""
-    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    _all_reduce(t)
 
 
 class _CudaView:
@@ -134,41 +211,51 @@ class DistributedEngine(Engine):
     """Engine whose builds happen on the root and are broadcast, and whose
     partitioned pipelines end with one reduce of the dense partials."""
 
-    def __init__(self, ctx: hq.Context, tables, root: int = 0, **kw):
+    def __init__(self, ctx: hq.Context, tables, root: int = 0, copartitioned: bool = False, **kw):
         super().__init__(ctx, tables, **kw)
         self.rank = dist.get_rank()
         self.world = dist.get_world_size()
         self.root = root
         self.device = torch.device("cuda", ctx.device)
         self._built: List[hq.Hash] = []
-        self.builds_here = self.rank == root
+        self._bcast: dict = {}  # broadcast_tables state (receive size), identical on every rank
+        # copartitioned: the tables are this rank's co-partition (hqgen.copartition) plus
+        # full copies of the small dimensions; every rank builds and runs locally
+        self.copartitioned = copartitioned
+        self.builds_here = copartitioned or self.rank == root
         # HQ_DIST_FAULT_TRACE=1 (debug): re-read every root build's fault word after the
         # final fetch and report the ones that changed since the build
         self._trace: Optional[List[Tuple[str, hq.Hash, List[int]]]] = (
             [] if os.environ.get("HQ_DIST_FAULT_TRACE") == "1" else None)
 
     def _share_many(self, hs: Optional[Sequence[hq.Hash]], n: int, err: Optional[BaseException] = None) -> List[hq.Hash]:
-        """Broadcast n root-built tables (broadcast_tables: one metadata broadcast, one
-        asynchronous broadcast per slot array, no host read on the root) and import them
-        on the other ranks.  Build faults are not read here (that would sync per table):
-        the root's fault words travel with the pipeline's reduce (_reduce_checked)."""
+        """Broadcast n root-built tables (broadcast_tables: metadata and every table in one
+        buffer, normally one collective; the root packs them with hq_hash_pack, no host
+        read on the root) and import them on the other ranks.  Build faults are not read
+        here (that would sync per table): the root's fault words travel with the
+        pipeline's reduce (_reduce_checked)."""
         if self.rank == self.root:
-            rows, views = [], []
+            rows = []
             if err is None:
                 for h in hs:
-                    ptr, m = h.device_view()
+                    _, m = h.device_view()
                     self._built.append(h)
                     if self._trace is not None:
                         self._trace.append((f"build#{len(self._trace)} rows={m.nkeys} cap={m.capacity}", h,
                                             self._faults_of(h)))
-                    views.append(device_view(ptr, int(m.bytes)))
                     rows.append(meta_row(m))
-            broadcast_tables(rows, views, n, self.root, self.device, err)
-            return list(hs)
-        rows, bufs = broadcast_tables(None, None, n, self.root, self.device)
+            hl = list(hs) if hs is not None else []
+            broadcast_tables(rows, lambda ptr, offs: self.ctx.pack_hashes(hl, offs, ptr), n, self.root, self.device,
+                             err, self._bcast)
+            return hl
+        rows, bufs = broadcast_tables(None, None, n, self.root, self.device, state=self._bcast)
         return [self.ctx.import_hash(meta_from_row(r), b.data_ptr(), keep=b) for r, b in zip(rows, bufs)]  # views keep the buffer
 
     def _root_build(self, fn, n: int):
+        if self.copartitioned:  # local build over this rank's co-partition: nothing to share
+            hs = fn()
+            self._built.extend(hs)
+            return hs
         hs, err = None, None
         if self.rank == self.root:
             try:
@@ -200,6 +287,18 @@ class DistributedEngine(Engine):
         return prod > 65536  # libhq's dense/hash switch (hqk::DENSE_LIMIT)
 
     def run(self, pb: PlanBuilder, partitioned: bool = True) -> Optional[hq.Result]:
+        if self.copartitioned:
+            if not partitioned:  # a build-side pipeline over this rank's co-partition
+                return super().run(pb, partitioned)
+            P = pb.plan
+            if not self._hash_grouped(P):
+                raise NotImplementedError("co-partitioned execution: the final pipeline must group by the "
+                                          "co-partitioning key (hash group-by)")
+            # groups are disjoint across ranks: ORDER BY / LIMIT stay in the local plan,
+            # the root merges the ranks' top rows
+            pb.dist_order = ([(P.order_col[i], P.order_desc[i]) for i in range(P.norder)], P.limit)
+            pb.copart_local_order = True
+            return super().run(pb, partitioned)
         if not partitioned:
             pb.root_only = True  # a build-side or post-merge pipeline: the root's result is complete
             if self.rank != self.root:
@@ -232,21 +331,35 @@ class DistributedEngine(Engine):
                       flush=True)
         self._trace.clear()
 
-    def _reduce_checked(self, res: hq.Result) -> None:
+    def _reduce_checked(self, res: hq.Result, defer: bool = False) -> Optional[torch.Tensor]:
         """ONE all-reduce of [dense partials | fault words]: the partials are summed
         (exact int64), and the fault words -- the root's build faults and every rank's
         pipeline faults, gathered on the device (hq_gather_faults) -- are summed too, so
         every rank sees every rank's faults and raises, or none does.  One host read of
-        the 32 fault words at the end; no per-table synchronisation."""
+        the 32 fault words at the end; no per-table synchronisation.  defer: the words are
+        copied to pinned host memory asynchronously and returned; the caller raises them
+        after its next synchronisation (the root's fetch), saving a host round trip."""
         ptr, nbytes = res.partials_view()
         n = nbytes // 8
         red = torch.empty(n + hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
-        red[:n].copy_(device_view(ptr, nbytes, torch.int64))
+        res.to_partials(red.data_ptr(), nbytes)
         built, self._built = self._built, []
         self.ctx.gather_faults(built, [res], red.data_ptr() + n * 8)
         reduce_partials(red, self.root)
         res.from_partials(red.data_ptr(), nbytes)
-        hq.raise_faults(red[n:].tolist())
+        if not defer:
+            hq.raise_faults(red[n:].tolist())
+            return None
+        if getattr(self, "_fault_host", None) is None:
+            self._fault_host = torch.empty(hq.FAULT_WORDS, dtype=torch.int64, pin_memory=True)
+        self._fault_host.copy_(red[n:], non_blocking=True)
+        self._fault_event = torch.cuda.Event()
+        self._fault_event.record(torch.cuda.current_stream(self.device))
+        return self._fault_host
+
+    def _raise_deferred(self, words: torch.Tensor) -> None:
+        self._fault_event.synchronize()  # (already complete after the root's fetch)
+        hq.raise_faults(words.tolist())
 
     def _root_only_checked(self, res: Optional[hq.Result]) -> None:
         """A root-only final pipeline: the root's build and pipeline faults are shared
@@ -255,7 +368,7 @@ class DistributedEngine(Engine):
         built, self._built = self._built, []
         if self.rank == self.root:
             self.ctx.gather_faults(built, [res] if res is not None else [], st.data_ptr())
-        dist.all_reduce(st)
+        _all_reduce(st)
         hq.raise_faults(st.tolist())
 
     def finish(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
@@ -267,8 +380,11 @@ class DistributedEngine(Engine):
             self._root_only_checked(res)
             out = fetch(res, pb.result_names) if self.rank == self.root else None
         elif not hasattr(pb, "dist_order"):
-            self._reduce_checked(res)
-            out = fetch(res, pb.result_names) if self.rank == self.root else None
+            words = self._reduce_checked(res, defer=True)
+            try:
+                out = fetch(res, pb.result_names) if self.rank == self.root else None
+            finally:
+                self._raise_deferred(words)  # every rank raises the summed faults (before a fetch error)
         else:
             out = self._merge_groups(res, pb)
         if self._trace is not None:
@@ -280,9 +396,19 @@ class DistributedEngine(Engine):
         declares the same group table."""
         lo, hi = self.tables[table].column_range(col)
         t = torch.tensor([-lo, hi], dtype=torch.int64, device=self.device)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        _all_reduce(t, dist.ReduceOp.MAX)
         lo, hi = -int(t[0].item()), int(t[1].item())
         return (0, 1) if lo > hi else (lo, hi - lo + 1)
+
+    def abort(self, err: BaseException) -> None:
+        """A co-partitioned rank whose local builds or pipeline raised on the host: join
+        the first collective of finish() (the status all-reduce) with the failure flag
+        set, so the other ranks raise RootError instead of waiting; then re-raise."""
+        st = torch.zeros(2 + hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
+        st[1] = 1
+        self._built = []
+        _all_reduce(st)
+        raise err
 
     def gather(self, res: Optional[hq.Result], pb: PlanBuilder) -> Optional[hq.Result]:
         """Complete result of a partitioned pipeline whose aggregation feeds a later build
@@ -292,6 +418,8 @@ class DistributedEngine(Engine):
         summed with one all-reduce.  Returns the device result on the root, None elsewhere."""
         if getattr(pb, "root_only", False):
             return res
+        if self.copartitioned:
+            raise NotImplementedError("co-partitioned execution: intermediate gathers are not supported")
         if hasattr(pb, "dist_order"):
             merged = self._merge_device(res, pb)
             return merged[0] if merged is not None else None
@@ -318,15 +446,25 @@ class DistributedEngine(Engine):
         st = torch.zeros(2 + hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
         built, self._built = self._built, []
         self.ctx.gather_faults(built, [], st.data_ptr() + 16)  # the root's build faults
-        err, tab, nrows = None, None, 0
+        err, tab, nrows, cols = None, None, 0, None
+        local_top = getattr(pb, "copart_local_order", False)
         try:
-            tab = res.as_table(names)  # finalized local groups (re-runs a full group table)
-            nrows = tab.nrows
-            st[0] = res.qualifying()
+            if local_top:  # disjoint groups: this rank's ORDER BY / LIMIT rows are final candidates
+                top = fetch(res, names)
+                if any(top.columns[nm].dtype.kind == "f" for nm in names):
+                    raise hq.HQError(hq.HQ_ERR_UNSUPPORTED, "co-partitioned merge: fp64 (AVG) result column")
+                nrows = top.nrows
+                cols = torch.from_numpy(np.stack([np.asarray(top.columns[nm], dtype=np.int64) for nm in names])
+                                        if nrows else np.zeros((len(names), 0), np.int64))
+                st[0] = top.qualifying
+            else:
+                tab = res.as_table(names)  # finalized local groups (re-runs a full group table)
+                nrows = tab.nrows
+                st[0] = res.qualifying()
         except hq.HQError as e:
             err = e
             st[1] = 1
-        dist.all_reduce(st)
+        _all_reduce(st)
         stl = st.tolist()
         if err is not None:
             raise err
@@ -342,10 +480,13 @@ class DistributedEngine(Engine):
         m = max(max(sizes), 1)
         # ONE all-gather of the packed [ncol, m] group rows
         pad = torch.zeros((ncol, m), dtype=torch.int64, device=self.device)
-        for c in range(ncol):
-            ptr, _ = tab.column_ptr(c)
-            if nrows:
-                pad[c, :nrows] = device_view(ptr, nrows * 8, torch.int64)
+        if cols is not None:
+            pad[:, :nrows] = cols.to(self.device)
+        else:
+            for c in range(ncol):
+                ptr, _ = tab.column_ptr(c)
+                if nrows:
+                    pad[c, :nrows] = device_view(ptr, nrows * 8, torch.int64)
         bufs = [torch.empty_like(pad) for _ in range(self.world)]
         dist.all_gather(bufs, pad)
         if self.rank != self.root:

@@ -122,7 +122,7 @@ EXPORTS = ["hq_ctx_create", "hq_ctx_destroy", "hq_ctx_set_stream", "hq_ctx_sync"
            "hq_hash_device_view", "hq_hash_import", "hq_free_hash", "hq_run_pipeline", "hq_run_pipeline_streamed",
            "hq_finalize",
            "hq_result_info_get", "hq_fetch_result", "hq_result_as_table", "hq_result_partials_view",
-           "hq_result_from_partials", "hq_gather_faults", "hq_raise_faults", "hq_free_result",
+           "hq_result_from_partials", "hq_result_to_partials", "hq_hash_pack", "hq_gather_faults", "hq_raise_faults", "hq_free_result",
            "hq_ctx_capture_begin", "hq_ctx_capture_end", "hq_ctx_capture_abort", "hq_graph_launch", "hq_graph_destroy"]
 FAULT_WORDS = 32
 
@@ -164,6 +164,8 @@ def lib():
             "hq_result_as_table": [vp, vp, P(vp)],
             "hq_result_partials_view": [vp, P(vp), P(ctypes.c_size_t)], "hq_free_result": [vp],
             "hq_result_from_partials": [vp, vp, vp, ctypes.c_size_t],
+            "hq_result_to_partials": [vp, vp, vp, ctypes.c_size_t],
+            "hq_hash_pack": [vp, P(vp), i32, P(i64), vp],
             "hq_gather_faults": [vp, P(vp), i32, P(vp), i32, vp],
             "hq_raise_faults": [P(i64)],
             "hq_ctx_capture_begin": [vp], "hq_ctx_capture_end": [vp, P(vp)], "hq_ctx_capture_abort": [vp],
@@ -327,6 +329,12 @@ class Context:
         hs = (ctypes.c_void_p * max(len(hashes), 1))(*[h.h for h in hashes])
         rs = (ctypes.c_void_p * max(len(results), 1))(*[r.h for r in results])
         check(lib().hq_gather_faults(self.h, hs, len(hashes), rs, len(results), ctypes.c_void_p(dev_out)))
+
+    def pack_hashes(self, hashes: Sequence["Hash"], offs: Sequence[int], dev_dst: int) -> None:
+        """Copy the hashes' device views into one device buffer at byte offsets (hq_hash_pack)."""
+        hs = (ctypes.c_void_p * max(len(hashes), 1))(*[h.h for h in hashes])
+        os_ = (ctypes.c_int64 * max(len(offs), 1))(*[int(o) for o in offs])
+        check(lib().hq_hash_pack(self.h, hs, len(hashes), os_, ctypes.c_void_p(dev_dst)))
 
     def run(self, plan: Plan, keep=(), block_rows: Optional[int] = None) -> "Result":
         """Enqueue a pipeline.  block_rows: batch processing of an HQ_HOST_STREAM fact
@@ -509,6 +517,10 @@ class Result:
         n = ctypes.c_size_t()
         check(lib().hq_result_partials_view(self.h, ctypes.byref(p), ctypes.byref(n)))
         return p.value, n.value
+
+    def to_partials(self, dev_ptr: int, nbytes: int) -> None:
+        """Copy the dense partials into a caller device buffer (hq_result_to_partials)."""
+        check(lib().hq_result_to_partials(self.ctx.h, self.h, ctypes.c_void_p(dev_ptr), nbytes))
 
     def from_partials(self, dev_ptr: int, nbytes: int) -> None:
         """Copy reduced partials back into the result's group table (hq_result_from_partials)."""

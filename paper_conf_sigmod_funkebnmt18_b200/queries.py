@@ -34,8 +34,12 @@ class Query:
     """A query: fact table, referenced columns per table, and run(E) which
     builds the hash tables and returns (final Result, final PlanBuilder)."""
 
-    def __init__(self, name: str, bench: str, fact: str, columns: Dict[str, List[str]], run: Callable):
+    def __init__(self, name: str, bench: str, fact: str, columns: Dict[str, List[str]], run: Callable,
+                 copart: Optional[str] = None):
         self.name, self.bench, self.fact, self.columns, self._run = name, bench, fact, columns, run
+        # copart: the order table partitioned together with the fact (line) table by order
+        # for multi-GPU runs (hqgen.copartition; the final GROUP BY contains the orderkey)
+        self.copart = copart
 
     def run(self, E: Engine, **kw):
         return self._run(E, **kw)
@@ -725,7 +729,7 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
     Query("tpch_q3", "tpch", "lineitem",
           {"lineitem": ["l_orderkey", "l_shipdate", "l_extendedprice", "l_discount"],
            "orders": ["o_orderkey", "o_custkey", "o_orderdate", "o_shippriority"],
-           "tpch_customer": ["c_custkey", "c_mktsegment"]}, _tpch_q3),
+           "tpch_customer": ["c_custkey", "c_mktsegment"]}, _tpch_q3, copart="orders"),
     Query("tpch_q5", "tpch", "lineitem",
           {"lineitem": ["l_orderkey", "l_suppkey", "l_extendedprice", "l_discount"],
            "orders": ["o_orderkey", "o_custkey", "o_orderdate"], "tpch_customer": ["c_custkey", "c_nationkey"],
@@ -774,19 +778,22 @@ QUERIES: Dict[str, Query] = {q.name: q for q in [
 
 def load_tables(ctx: hq.Context, query: Query, sf: float, seed: int = hqgen.DEFAULT_SEED,
                 fact_range: Optional[tuple] = None, host: Optional[Dict[str, Dict]] = None,
-                skip_dims: bool = False, stream_fact: bool = False) -> Dict[str, hq.Table]:
+                skip_dims: bool = False, stream_fact: bool = False,
+                copart_range: Optional[tuple] = None) -> Dict[str, hq.Table]:
     """Generate (or take from ``host``) the referenced columns and load them onto
     the context's device.  fact_range: rows of the fact table to load (a range
     partition).  skip_dims: load only the fact table (non-root ranks).  stream_fact:
-    leave the fact table in host memory (HQ_HOST_STREAM, batch processing)."""
+    leave the fact table in host memory (HQ_HOST_STREAM, batch processing).
+    copart_range: rows of ``query.copart`` (the order table co-partitioned with the
+    fact table, hqgen.copartition)."""
     tables = {}
     for t, cols in query.columns.items():
-        if skip_dims and t != query.fact:
+        if skip_dims and t != query.fact and t != query.copart:
             continue
         if host is not None and t in host:
             data = {c: host[t][c] for c in cols}
         else:
-            rr = fact_range if t == query.fact else None
+            rr = fact_range if t == query.fact else (copart_range if t == query.copart else None)
             data = hqgen.generate(t, sf, seed, columns=cols, row_range=rr)
         tables[t] = ctx.load_columns(data, stream=stream_fact and t == query.fact)
     return tables

@@ -1,5 +1,6 @@
 """cProfile of the host side of repeated query steps (where the Python / C++ host time
-between kernel launches goes).  python scripts/hostprof.py --query ssb_q11 --sf 1 --steps 200"""
+between kernel launches goes).  python scripts/hostprof.py --query ssb_q11 --sf 1 --steps 200
+[--dist: the distributed engine over NCCL at world size 1]"""
 import argparse
 import cProfile
 import os
@@ -19,17 +20,34 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--query", default="ssb_q11")
 ap.add_argument("--sf", type=float, default=1)
 ap.add_argument("--steps", type=int, default=200)
+ap.add_argument("--dist", action="store_true")
 a = ap.parse_args()
 torch.cuda.set_device(0)
 q = QUERIES[a.query]
 ctx = hq.Context(0)
-E = Engine(ctx, load_tables(ctx, q, a.sf))
+tables = load_tables(ctx, q, a.sf)
+if a.dist:
+    import torch.distributed as dist
+    from paper_conf_sigmod_funkebnmt18_b200.dist import DistributedEngine, run_query
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29572")
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    E = DistributedEngine(ctx, tables)
+
+    def step():
+        return run_query(E, q)
+else:
+    E = Engine(ctx, tables)
+
+    def step():
+        return q.execute(E)
 for _ in range(5):
-    q.execute(E)
+    step()
 pr = cProfile.Profile()
 pr.enable()
 for _ in range(a.steps):
-    q.execute(E)
+    step()
 pr.disable()
 st = pstats.Stats(pr)
-st.sort_stats("tottime").print_stats(25)
+st.sort_stats("tottime").print_stats(30)
+st.sort_stats("cumtime").print_stats(40)

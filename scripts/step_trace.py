@@ -4,7 +4,10 @@ memcpy of the step with its start offset and duration, the idle gaps between the
 and the CUDA runtime calls that block the host (stream syncs) -- where the time
 outside the fused kernel goes.
 
-    python scripts/step_trace.py --query ssb_q41 --sf 100 [--steps 3] [--json out.json]
+    python scripts/step_trace.py --query ssb_q41 --sf 100 [--steps 3] [--json out.json] [--dist]
+
+--dist: the distributed engine (dist.DistributedEngine over NCCL) at world size 1 -- the
+fixed cost of its collectives and fault exchange over the single-device step.
 """
 import argparse
 import json
@@ -27,15 +30,30 @@ def main():
     ap.add_argument("--sf", type=float, default=10)
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--json", default="")
+    ap.add_argument("--dist", action="store_true")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     q = QUERIES[a.query]
     ctx = hq.Context(0)
     tables = load_tables(ctx, q, a.sf)
     ctx.sync()
-    E = Engine(ctx, tables)
+    if a.dist:
+        import torch.distributed as dist
+        from paper_conf_sigmod_funkebnmt18_b200.dist import DistributedEngine, run_query
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29571")
+        dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+        E = DistributedEngine(ctx, tables)
+
+        def execute():
+            return run_query(E, q)
+    else:
+        E = Engine(ctx, tables)
+
+        def execute():
+            return q.execute(E)
     for _ in range(3):
-        q.execute(E)
+        execute()
     torch.cuda.synchronize()
     from torch.profiler import ProfilerActivity, profile
     marker = torch.zeros(1024, device="cuda")
@@ -44,7 +62,7 @@ def main():
             torch.cuda.synchronize()
             with torch.profiler.record_function("hq_step"):
                 marker.mul_(1.5)  # a step-start marker kernel on the GPU timeline
-                q.execute(E)
+                execute()
             torch.cuda.synchronize()
     evs = prof.events()
     hsteps = sorted([e for e in evs if e.name == "hq_step" and e.device_type == torch.autograd.DeviceType.CPU],
@@ -53,7 +71,7 @@ def main():
                  key=lambda e: e.time_range.start)
     syncs = [e for e in evs if e.device_type == torch.autograd.DeviceType.CPU and "Synchronize" in e.name]
     # GPU ops of step k: from its marker kernel to the next marker (CPU and GPU clocks may differ)
-    mk = [i for i, e in enumerate(gpu) if "elementwise" in e.name.lower()]
+    mk = [i for i, e in enumerate(gpu) if "MulFunctor" in e.name]
     out = []
     for si, st in enumerate(hsteps):
         if si >= len(mk):

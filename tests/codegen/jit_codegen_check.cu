@@ -77,7 +77,25 @@ hq_hash* make_hash(hq_ctx* c, int layout, int npay, int ckind, int64_t range, bo
   return h;
 }
 
-hq_op probe(const hq_hash* h, int key, int mode, int dst = -1) {
+// ranked form of a sparse-key linear table (hq_hash::ranked): bitmap | directory | rows
+hq_hash* make_ranked(hq_ctx* c, int npay, int64_t range, int64_t nkeys) {
+  hq_hash* h = make_hash(c, HQ_HT_LINEAR, npay, 0, range);
+  h->slots = nullptr;
+  h->meta.nkeys = nkeys;
+  int64_t od, op, tot;
+  int st;
+  hq_ranked_layout(range, nkeys, npay, &od, &op, &tot, &st);
+  h->ckind = 4;
+  h->cbytes = tot;
+  h->roff_dir = od;
+  h->roff_pay = op;
+  h->rstride = st;
+  h->compact = DevBuf(c, 64);
+  h->compact_only = true;
+  return h;
+}
+
+hq_op probe(const hq_hash* h, int key, int mode, int dst = -1, int dst2 = -1) {
   hq_op o{};
   o.kind = HQ_OP_PROBE;
   o.ht = h;
@@ -86,6 +104,10 @@ hq_op probe(const hq_hash* h, int key, int mode, int dst = -1) {
   if (dst >= 0) {
     o.npayload = 1;
     o.payload_dst[0] = dst;
+  }
+  if (dst2 >= 0) {
+    o.npayload = 2;
+    o.payload_dst[1] = dst2;
   }
   return o;
 }
@@ -290,6 +312,30 @@ int main(int argc, char** argv) {
     shapes.push_back({"global_hash_groups_r4", P, "4"});
   }
 
+  {  // ranked sparse-key tables: an inner probe with two payloads (TPC-H Q3's orders:
+     // orderdate, shippriority), a semi-join (bitmap only) and an outer probe with one payload
+    hq_hash* rk2 = make_ranked(c, 2, 180000000, 4400000);
+    hq_hash* rk0 = make_ranked(c, 0, 6000000, 1000000);
+    hq_hash* rk1 = make_ranked(c, 1, 3000000, 200000);
+    hq_plan P{};
+    P.fact = F;
+    P.row_end = -1;
+    P.ops[P.nops++] = filter(3, HQ_GT, 19950315);
+    P.ops[P.nops++] = probe(rk2, 1, HQ_PROBE_INNER, HQ_TMP(0), HQ_TMP(1));
+    P.ops[P.nops++] = probe(rk0, 2, HQ_PROBE_SEMI);
+    P.ops[P.nops++] = probe(rk1, 0, HQ_PROBE_OUTER, HQ_TMP(2));
+    P.sink = HQ_SINK_AGG;
+    P.nkeys = 3;
+    P.key_reg[0] = 1; P.key_card[0] = 1ll << 31;
+    P.key_reg[1] = HQ_TMP(0); P.key_min[1] = 19920101; P.key_card[1] = 70000;
+    P.key_reg[2] = HQ_TMP(1); P.key_card[2] = 8;
+    P.naggs = 2;
+    P.agg_fn[0] = HQ_AGG_SUM; P.agg_reg[0] = HQ_TMP(2);
+    P.agg_fn[1] = HQ_AGG_COUNT;
+    P.group_capacity = 600000;
+    shapes.push_back({"ranked_probes", P, nullptr});
+  }
+
   {  // LEFT OUTER probes (byte map, linear, direct) and predicate expressions (TPC-H Q13 / Q19 shapes)
     // the byte map rank-coded over a sparse payload set (Q13's orders-per-customer counts)
     byte_big = make_hash(c, HQ_HT_DIRECT, 1, 2, 3000000);
@@ -342,7 +388,7 @@ int main(int argc, char** argv) {
     std::vector<Shape> wes;
     for (const Shape& s : shapes) {
       if (s.name != "star_ranked_dense" && s.name != "materialise_lrgp" && s.name != "scalar_filters" &&
-          s.name != "global_hash_groups")
+          s.name != "global_hash_groups" && s.name != "ranked_probes")
         continue;
       Shape w = s;
       w.name = s.name + "_we";
@@ -358,7 +404,7 @@ int main(int argc, char** argv) {
     std::vector<Shape> mps;
     for (const Shape& s : shapes) {
       if (s.name != "star_ranked_dense" && s.name != "materialise_lrgp" && s.name != "scalar_filters" &&
-          s.name != "outer_predicates" && s.name != "composite_probe")
+          s.name != "outer_predicates" && s.name != "composite_probe" && s.name != "ranked_probes")
         continue;
       for (int pass : {1, 2}) {
         Shape m = s;

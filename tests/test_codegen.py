@@ -32,9 +32,13 @@ def test_generated_kernels_compile(checker, tmp_path):
     env = {k: v for k, v in os.environ.items() if not k.startswith("HQ_")}
     p = subprocess.run([checker, str(tmp_path)], capture_output=True, text=True, env=env, timeout=600)
     assert p.returncode == 0, p.stdout + p.stderr
-    assert p.stdout.startswith("OK 28 of 28"), p.stdout
+    assert p.stdout.startswith("OK 32 of 32"), p.stdout
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
+    rk = srcs["ranked_probes"]  # ranked sparse-key tables: bitmap, directory + popcount, payload rows
+    assert "__ldg(p.pf[0] + (e_[r] >> 5))" in rk and "__ldg(p.rdir[0] + (e_[r] >> 5)) + __popc(w_[r]" in rk
+    assert "(const int2*)p.rpay[0]" in rk and "__ldg(p.rpay[2] + k_[r])" in rk and "p.rdir[1]" not in rk
+    assert "p.ht[0]" not in rk and "0x9E3779B1u" not in rk.split("gk_")[0]
     star = srcs["star_dense_lrgp"]
     assert "lds_u32(sm0_ + " in star                 # staged bitmap
     assert "__ldg((const unsigned char*)p.ctab[" in star  # global byte map

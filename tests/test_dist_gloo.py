@@ -70,14 +70,19 @@ def _worker(rank, world, port, q):
         dims = {t: hqgen.generate(t, SF) for t in ("customer", "supplier", "part", "date")}
         # root "builds" and broadcasts tables (the hash-table slot arrays on GPUs): n = 0, 1, 3
         blob = np.ascontiguousarray(dims["customer"]["c_custkey"][dims["customer"]["c_region"] == 1]).view(np.uint8)
-        for nt in (0, 1, 3):
-            blobs = [np.roll(blob, k).copy() for k in range(nt)]
+        # with a shared receive-size state (the engine's): the first message grows it (two
+        # collectives), repeated and smaller ones fit in one
+        state = {}
+        for nt, stateful in ((0, False), (1, False), (3, False), (1, True), (3, True), (3, True), (1, True),
+                             (0, True)):
+            blobs = [np.roll(blob, k + nt).copy() for k in range(nt)]
             metas = [_stub_meta(k, x.nbytes) for k, x in enumerate(blobs)]
+            st = state if stateful else None
             if rank == 0:
                 rows, bufs = broadcast_tables([meta_row(m) for m in metas], [torch.from_numpy(x) for x in blobs], nt, 0,
-                                              "cpu")
+                                              "cpu", state=st)
             else:
-                rows, bufs = broadcast_tables(None, None, nt, 0, "cpu")
+                rows, bufs = broadcast_tables(None, None, nt, 0, "cpu", state=st)
             assert len(rows) == len(bufs) == nt
             for m, r, buf, ref in zip(metas, rows, bufs, blobs):
                 got = meta_from_row(r)
@@ -86,13 +91,13 @@ def _worker(rank, world, port, q):
         # a root-side build error: the root re-raises it, the other rank raises RootError
         if rank == 0:
             try:
-                broadcast_tables(None, None, 2, 0, "cpu", err=hq.HQError(hq.HQ_ERR_DUP_KEY, "dup"))
+                broadcast_tables(None, None, 2, 0, "cpu", err=hq.HQError(hq.HQ_ERR_DUP_KEY, "dup"), state=state)
                 raise AssertionError("root did not re-raise")
             except hq.HQError as e:
                 assert e.code == hq.HQ_ERR_DUP_KEY and not isinstance(e, RootError)
         else:
             try:
-                broadcast_tables(None, None, 2, 0, "cpu")
+                broadcast_tables(None, None, 2, 0, "cpu", state=state)
                 raise AssertionError("rank 1 did not raise")
             except RootError as e:
                 assert e.code == hq.HQ_ERR_DUP_KEY

@@ -175,3 +175,32 @@ def test_tpch_derived_columns():
     assert len(m) == len(li)
     assert hqgen.BRANDS[hqgen.code(hqgen.BRANDS, "Brand#23")] == "Brand#23" and hqgen.BRANDS == sorted(hqgen.BRANDS)
     assert len(hqgen.CONTAINERS) == 40 and hqgen.CONTAINERS == sorted(hqgen.CONTAINERS)
+
+
+@pytest.mark.parametrize("line,order", [("lineitem", "orders"), ("lineorder", None)])
+def test_copartition_by_order(line, order):
+    """hqgen.copartition: rank r's line rows are exactly the lines of its orders (the
+    ranks' line ranges tile the table; every line's orderkey is one of its rank's
+    orders), and line_row_of_order is the first row carrying the order's key."""
+    sf = 0.01
+    key = "l_orderkey" if line == "lineitem" else "lo_orderkey"
+    lk = hqgen.generate(line, sf, columns=[key])[key]
+    first = {}
+    for i, k in enumerate(lk.tolist()):
+        first.setdefault(k, i)
+    ks = sorted(first)
+    for j in (0, 1, 7, 8, 9, len(ks) // 2, len(ks) - 1):
+        assert hqgen.line_row_of_order(line, sf, j) == first[ks[j]]
+    assert hqgen.line_row_of_order(line, sf, len(ks)) == len(lk)
+    if order is None:
+        return
+    ok = hqgen.generate(order, sf, columns=["o_orderkey"])["o_orderkey"]
+    for world in (1, 2, 3, 8):
+        end = 0
+        for r in range(world):
+            (a, b), (la, lb) = hqgen.copartition(line, order, sf, r, world)
+            assert la == end
+            end = lb
+            assert np.isin(lk[la:lb], ok[a:b]).all()
+            assert set(ok[a:b].tolist()) >= set(lk[la:lb].tolist())
+        assert end == len(lk)

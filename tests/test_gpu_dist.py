@@ -24,7 +24,7 @@ def _port():
     return p
 
 
-def _worker(rank, world, port, q, qs=None, sf=None):
+def _worker(rank, world, port, q, qs=None, sf=None, copart=False):
     qs = QS if qs is None else qs
     sf = SF if sf is None else sf
     try:
@@ -33,7 +33,7 @@ def _worker(rank, world, port, q, qs=None, sf=None):
 
         import hqgen
         from paper_conf_sigmod_funkebnmt18_b200 import hq
-        from paper_conf_sigmod_funkebnmt18_b200.dist import DistributedEngine, partition
+        from paper_conf_sigmod_funkebnmt18_b200.dist import DistributedEngine, partition, run_query
         from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES, load_tables
 
         os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -45,12 +45,15 @@ def _worker(rank, world, port, q, qs=None, sf=None):
         for qn in qs:
             qq = QUERIES[qn]
             n = hqgen.table_rows(qq.fact, sf)
-            rng = partition(n, rank, world)
-            tables = load_tables(ctx, qq, sf, fact_range=rng, skip_dims=rank != 0)
-            E = DistributedEngine(ctx, tables)
-            res, pb = qq.run(E)
-            r = E.finish(res, pb)
-            out[qn] = r.rows() if r is not None else None
+            if copart:  # orders + lineitem co-partitioned by order, every rank builds locally
+                crng, rng = hqgen.copartition(qq.fact, qq.copart, sf, rank, world)
+                tables = load_tables(ctx, qq, sf, fact_range=rng, copart_range=crng)
+            else:
+                rng = partition(n, rank, world)
+                tables = load_tables(ctx, qq, sf, fact_range=rng, skip_dims=rank != 0)
+            E = DistributedEngine(ctx, tables, copartitioned=copart)
+            r = run_query(E, qq)
+            out[qn] = (r.rows(), r.qualifying) if r is not None else None
         q.put(("ok", rank, out))
         dist.barrier()
         dist.destroy_process_group()
@@ -74,7 +77,7 @@ def test_two_ranks_on_one_device_match_oracle():
     errs = [o for o in outs if o[0] != "ok"]
     if errs:
         pytest.fail("\n\n".join(f"rank {o[1]}:\n{o[2]}" for o in errs))
-    root = next(o[2] for o in outs if o[1] == 0)
+    root = {k: v[0] for k, v in next(o[2] for o in outs if o[1] == 0).items()}
     ssb = {t: hqgen.generate(t, SF) for t in hqgen.SSB_TABLES}
     tpch = {t: hqgen.generate(t, SF) for t in hqgen.TPCH_TABLES}
     exp = {
@@ -132,7 +135,7 @@ def test_two_ranks_tpch_multi_pipeline_sf1():
     errs = [o for o in outs if o[0] != "ok"]
     if errs:
         pytest.fail("\n\n".join(f"rank {o[1]}:\n{o[2]}" for o in errs))
-    root = next(o[2] for o in outs if o[1] == 0)
+    root = {k: v[0] for k, v in next(o[2] for o in outs if o[1] == 0).items()}
     assert all(o[2][qn] is None for o in outs if o[1] != 0 for qn in F3)
     t = {x: hqgen.generate(x, 1.0) for x in hqgen.TPCH_TABLES}
     exp = {
@@ -147,3 +150,31 @@ def test_two_ranks_tpch_multi_pipeline_sf1():
     for qn, rows in exp.items():
         assert root[qn] == rows, qn
         assert len(rows) > 0, qn
+
+
+@pytest.mark.parametrize("world,sf", [(2, 0.01), (3, 1.0)])
+def test_copartitioned_tpch_q3(world, sf):
+    """TPC-H Q3 with orders and lineitem co-partitioned by order (hqgen.copartition):
+    every rank builds its customer / orders tables locally (no broadcast), runs its
+    ORDER BY / LIMIT over its own (disjoint) orderkey groups, and the root merges the
+    ranks' top rows; rows and the qualifying count equal the oracle's."""
+    import hqgen
+    import oracle
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, ["tpch_q3"], sf, True)) for r in range(world)]
+    for p in procs:
+        p.start()
+    outs = [q.get(timeout=900) for _ in procs]
+    for p in procs:
+        p.join(timeout=120)
+    errs = [o for o in outs if o[0] != "ok"]
+    if errs:
+        pytest.fail("\n\n".join(f"rank {o[1]}:\n{o[2]}" for o in errs))
+    rows, qual = next(o[2] for o in outs if o[1] == 0)["tpch_q3"]
+    assert all(o[2]["tpch_q3"] is None for o in outs if o[1] != 0)
+    t = {x: hqgen.generate(x, sf) for x in ("tpch_customer", "orders", "lineitem")}
+    o3 = oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    assert rows == o3.rows(["l_orderkey", "o_orderdate", "o_shippriority", "revenue", "count"])[:10]
+    assert qual == int(o3.columns["count"].sum())  # lineitem rows that reached the GROUP BY, all ranks
