@@ -645,6 +645,31 @@ hq_status hq_fetch_result(hq_ctx* ctx, hq_result* r, void* const* host_cols, int
   });
 }
 
+// Identity of a result viewed as a table: its plan with every input replaced by the
+// input's own identity (the fact table's uid, each probed table's build-statistics key),
+// so that the same pipeline over the same tables yields the same uid step after step and
+// a build over it (TPC-H Q3's orders side) finds its cached statistics -- verified on the
+// device like any other (hq_build.cu).  0 (a fresh uid) when an input has no identity
+// (an imported or expected_rows-sized table).
+static uint64_t derived_uid(const hq_result* r) {
+  if (!r->fact) return 0;
+  hq_plan P = r->plan;
+  std::string k;
+  k.append((const char*)&r->fact->uid, sizeof(r->fact->uid));
+  P.fact = nullptr;
+  for (int i = 0; i < P.nops; ++i) {
+    if (P.ops[i].kind != HQ_OP_PROBE) continue;
+    if (!P.ops[i].ht || P.ops[i].ht->stats_key.empty()) return 0;
+    const std::string& sk = P.ops[i].ht->stats_key;
+    const uint64_t n = sk.size();
+    k.append((const char*)&n, sizeof n);
+    k.append(sk);
+    P.ops[i].ht = nullptr;
+  }
+  k.append((const char*)&P, sizeof P);
+  return std::hash<std::string>{}(k) | (1ull << 63);  // (counter uids stay below 2^63)
+}
+
 hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out) {
   return guarded([&] {
     if (ctx) hq_require_eager(ctx, "hq_result_as_table");
@@ -655,6 +680,7 @@ hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out) {
       if (r->types[c] == HQ_F64) HQ_THROW(HQ_ERR_UNSUPPORTED, "result has fp64 (AVG) columns: not a table");
     hq_table* t = new hq_table();
     t->ctx = ctx;
+    if (const uint64_t d = derived_uid(r)) t->uid = d;
     t->nrows = r->nrows;
     t->ncols = r->ncols;
     for (int c = 0; c < r->ncols; ++c) {

@@ -635,8 +635,8 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   for (;;) {
     uint32_t tab_total = 0;
     for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
-    for (int R : {8, 4, 2, 1}) {
-      if (prefer4 ? (R != 4 && R != 2) : (force_R ? R != force_R : (R == 8 || R == 1))) continue;
+    for (int R : {8, 4, 3, 2, 1}) {  // (3: only when forced, HQ_JIT_R=3 experiments)
+      if (prefer4 ? (R != 4 && R != 2) : (force_R ? R != force_R : (R == 8 || R == 1 || R == 3))) continue;
       const uint32_t T = (uint32_t)(kp.nw * 32 * R);
       const uint32_t off_tmp = MISC_BYTES;
       const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
