@@ -564,6 +564,17 @@ hq_status hq_free_hash(hq_hash* h) {
 static void run_pipeline(hq_ctx* ctx, const hq_plan* plan, int64_t block_rows, hq_result** out) {
     if (!ctx || !plan || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
     if (!plan->fact) HQ_THROW(HQ_ERR_ARG, "plan: fact table is NULL");
+    if (plan->fact->dev_rows) {  // a view sized by a cached row count: check it once (host read)
+      hq_require_eager(ctx, "a pipeline over a result view sized by its cached row count");
+      unsigned long long* hc = (unsigned long long*)pinned_staging(ctx, 8);
+      HQ_CUDA(cudaMemcpyAsync(hc, plan->fact->dev_rows, 8, cudaMemcpyDeviceToHost, ctx->stream));
+      HQ_CUDA(cudaStreamSynchronize(ctx->stream));
+      if ((int64_t)*hc != plan->fact->nrows) {
+        ctx->derived_rows.erase(plan->fact->uid);
+        HQ_THROW(HQ_ERR_STATE, "result view: the result's row count differs from the cached one (re-run the query)");
+      }
+      const_cast<hq_table*>(plan->fact)->dev_rows = nullptr;
+    }
     hq_result* r = new hq_result();
     if (plan->fact->host_stream) r->stream_block = block_rows > 0 ? block_rows : HQ_STREAM_BLOCK_ROWS;
     r->fact = const_cast<hq_table*>(plan->fact);
@@ -672,15 +683,37 @@ static uint64_t derived_uid(const hq_result* r) {
 
 hq_status hq_result_as_table(hq_ctx* ctx, hq_result* r, hq_table** out) {
   return guarded([&] {
-    if (ctx) hq_require_eager(ctx, "hq_result_as_table");
     if (!ctx || !r || !out) HQ_THROW(HQ_ERR_ARG, "NULL argument");
-    hq_finalize_impl(ctx, r, /*unordered=*/true);
     const bool mat = r->sink == HQ_SINK_MATERIALISE;
+    const uint64_t duid = derived_uid(r);
+    // a materialised result seen before under the same identity: its row count is known,
+    // the view needs no finalize (no host sync; also inside a graph capture) -- the row
+    // counter on the device is checked by the table's consumers instead (dev_rows)
+    // (only where the count is the result's one possible fault: no division / modulo in
+    // its expressions, whose faults only the finalize would read)
+    bool faultless = true;
+    for (int i = 0; i < r->plan.nops; ++i)
+      if (r->plan.ops[i].kind == HQ_OP_COMPUTE)
+        for (int k = 0; k < r->plan.ops[i].ninsn && k < HQ_MAX_INSN; ++k)
+          faultless = faultless && r->plan.ops[i].code[k].opc != HQ_I_DIV && r->plan.ops[i].code[k].opc != HQ_I_MOD;
+    auto known = duid && mat && faultless && !r->finalized ? ctx->derived_rows.find(duid) : ctx->derived_rows.end();
+    const bool lazy = known != ctx->derived_rows.end() && !getenv("HQ_NO_DERIVED_ROWS");
+    if (lazy) {
+      r->nrows = known->second;
+      r->ncols = r->plan.nout;
+      for (int j = 0; j < r->plan.nout; ++j) r->types[j] = r->plan.out_type[j];
+      if (r->capacity < r->nrows) HQ_THROW(HQ_ERR_STATE, "result view: cached row count exceeds the capacity");
+    } else {
+      hq_require_eager(ctx, "hq_result_as_table");
+      hq_finalize_impl(ctx, r, /*unordered=*/true);
+      if (duid && mat) ctx->derived_rows[duid] = r->nrows;
+    }
     for (int c = 0; c < r->ncols; ++c)
       if (r->types[c] == HQ_F64) HQ_THROW(HQ_ERR_UNSUPPORTED, "result has fp64 (AVG) columns: not a table");
     hq_table* t = new hq_table();
     t->ctx = ctx;
-    if (const uint64_t d = derived_uid(r)) t->uid = d;
+    if (duid) t->uid = duid;
+    if (lazy) t->dev_rows = (const unsigned long long*)r->dstate.p;  // the materialise counter
     t->nrows = r->nrows;
     t->ncols = r->ncols;
     for (int c = 0; c < r->ncols; ++c) {
@@ -770,11 +803,12 @@ hq_status hq_raise_faults(const int64_t* w) {
     auto b = [&](int bit) { return w[bit] != 0; };
     auto pb = [&](int flag) { int k = 0; while ((1 << k) != flag) ++k; return w[16 + k] != 0; };
     auto hb = [&](int flag) { int k = 0; while ((1 << k) != flag) ++k; return b(k); };
+    // (stale statistics first: a table sized from them can also report keys out of range)
+    if (hb(HQF_STALE)) HQ_THROW(HQ_ERR_STATE, "hash build: source rows differ from the cached build statistics");
     if (hb(HQF_DUP_KEY)) HQ_THROW(HQ_ERR_DUP_KEY, "hash build: duplicate key (join keys must be unique)");
     if (hb(HQF_BAD_KEY)) HQ_THROW(HQ_ERR_ARG, "hash build: key INT32_MIN or outside int32");
     if (hb(HQF_BAD_PAYLOAD)) HQ_THROW(HQ_ERR_ARG, "hash build: payload outside int32");
     if (hb(HQF_HT_FULL)) HQ_THROW(HQ_ERR_OVERFLOW, "hash build: table full (expected_rows too small)");
-    if (hb(HQF_STALE)) HQ_THROW(HQ_ERR_STATE, "hash build: source rows differ from the cached build statistics");
     if (pb(HQF_DIV_ZERO)) HQ_THROW(HQ_ERR_ARG, "pipeline: division by zero");
     if (pb(HQF_KEY_DOMAIN)) HQ_THROW(HQ_ERR_ARG, "pipeline: group key outside its declared [min, min+card)");
     if (pb(HQF_OVERFLOW)) HQ_THROW(HQ_ERR_OVERFLOW, "aggregate exceeds the int64 guard (|v| >= 2^62)");

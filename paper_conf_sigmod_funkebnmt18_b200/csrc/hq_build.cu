@@ -50,7 +50,17 @@ struct KBuild {
   int verify;
   BuildStats vs;
   unsigned long long* vqual;  // qualifying rows seen by the insert pass
+  // a source table sized by a cached row count (hq_table::dev_rows): the real count
+  // on the device; rows at or past it do not qualify, and a difference is HQF_STALE
+  const unsigned long long* ndev;
 };
+
+__device__ __forceinline__ long long live_rows(const KBuild& b) {
+  if (!b.ndev) return b.n;
+  const long long d = (long long)*(const volatile unsigned long long*)b.ndev;
+  if (d != b.n && blockIdx.x == 0 && threadIdx.x == 0) atomicOr(b.err, HQF_STALE);
+  return d < b.n ? d : b.n;
+}
 
 __device__ __forceinline__ long long ld_col(const KBuild& b, int c, long long row) {
   const int w = b.colw[c];
@@ -107,8 +117,9 @@ __device__ __forceinline__ void load_rows(const KBuild& b, long long base, bool 
                                           long long (&kv)[BUILD_U], long long (&pv)[BUILD_U]) {
   ld_rows(b, b.key_col, base, kv);
   if (b.npay > 0) ld_rows(b, b.pay_col[0], base, pv);
+  const long long nl = live_rows(b);
 #pragma unroll
-  for (int u = 0; u < BUILD_U; ++u) pass[u] = base + (long long)u * BUILD_BLOCK < b.n;
+  for (int u = 0; u < BUILD_U; ++u) pass[u] = base + (long long)u * BUILD_BLOCK < nl;
   for (int i = 0; i < b.npreds; ++i) {
     const KBuildPred& f = b.preds[i];
     long long v[BUILD_U];
@@ -684,6 +695,7 @@ void build_prepare(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& 
   if (d->key_col < 0 || d->key_col >= t->ncols) HQ_THROW(HQ_ERR_ARG, "build: key column out of range");
   KBuild& b = bs.b;
   b.n = t->nrows;
+  b.ndev = t->dev_rows;
   for (int c = 0; c < t->ncols; ++c) {
     b.col[c] = (const char*)t->cols[c].ptr;
     b.colw[c] = t->cols[c].width;
@@ -790,6 +802,7 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
   h->meta.composite = b.composite;
   h->meta.nkeys = bs.counted ? keys : -1;  // exact after the count pass (confirmed at hq_hash_info)
   h->src_rows = b.n;
+  h->src_uid = d->src->uid;
   h->meta.bytes = cap * words * 4;
   h->meta.layout = direct ? HQ_HT_DIRECT : HQ_HT_LINEAR;
   h->meta.key_min = kmin;
@@ -1113,15 +1126,17 @@ void hq_hash_check(hq_ctx* ctx, hq_hash* h) {
   HQ_CUDA(cudaStreamSynchronize(ctx->stream));
   if (h->meta.nkeys < 0) h->meta.nkeys = (int64_t)(*(unsigned long long*)(st + 2));  // expected_rows builds
   h->checked = true;
+  // stale statistics first: a table sized from them can also report keys out of range
+  if (st[0] & HQF_STALE) {
+    ctx->build_stats.erase(h->stats_key);  // the next build of this descriptor counts again
+    ctx->derived_rows.erase(h->src_uid);   // (and a result view re-reads its row count)
+    HQ_THROW(HQ_ERR_STATE, "hash build: the source table's rows differ from the statistics cached when it was "
+                           "last built (tables are immutable; the statistics were dropped, re-run the query)");
+  }
   if (st[0] & HQF_DUP_KEY) HQ_THROW(HQ_ERR_DUP_KEY, "hash build: duplicate key (join keys must be unique)");
   if (st[0] & HQF_BAD_KEY) HQ_THROW(HQ_ERR_ARG, "hash build: key INT32_MIN or outside int32");
   if (st[0] & HQF_BAD_PAYLOAD) HQ_THROW(HQ_ERR_ARG, "hash build: payload outside int32");
   if (st[0] & HQF_HT_FULL) HQ_THROW(HQ_ERR_OVERFLOW, "hash build: table full (expected_rows too small)");
-  if (st[0] & HQF_STALE) {
-    ctx->build_stats.erase(h->stats_key);  // the next build of this descriptor counts again
-    HQ_THROW(HQ_ERR_STATE, "hash build: the source table's rows differ from the statistics cached when it was "
-                           "last built (tables are immutable; the statistics were dropped, re-run the query)");
-  }
 }
 
 // ------------------------------------------------------------ column statistics

@@ -752,6 +752,9 @@ static bool decode_small(hq_result* r, const char* h, int64_t rcap, int nc) {
 
 void hq_decode_captured(hq_ctx* ctx, hq_result* r) {
   if (!r->stage_host) HQ_THROW(HQ_ERR_STATE, "result has no capture staging");
+  if (r->stage_topk && ((const unsigned long long*)r->stage_host)[5])
+    HQ_THROW(HQ_ERR_STATE, "captured query: more ties at the LIMIT boundary than the top-k selection holds "
+                           "(run the query eagerly)");
   if (decode_small(r, (const char*)r->stage_host, r->stage_rcap, r->ncols)) return;
   // a fault (pipeline, or a probed table's build): raised by the syncing check; the
   // re-runnable ones cannot occur in a dense small result
@@ -826,6 +829,21 @@ static bool finalize_topk(hq_ctx* ctx, hq_result* r) {
   hq_topk_collect_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel);
   hq_topk2_kernel<<<1, 1024, 0, ctx->stream>>>(q, sel);
   HQ_CUDA(cudaGetLastError());
+  if (ctx->capturing) {  // as finalize_small: the rows land in the result's pinned staging per launch
+    if (r->stage_host) HQ_THROW(HQ_ERR_STATE, "result finalized twice in one capture");
+    HQ_CUDA(cudaHostAlloc(&r->stage_host, 64 + body, cudaHostAllocDefault));
+    HQ_CUDA(cudaMemcpyAsync(r->stage_host, pack.p, 64 + body, cudaMemcpyDeviceToHost, ctx->stream));
+    r->stage_rcap = rcap;
+    r->stage_topk = true;
+    r->ncols = nc;
+    r->rescol.assign((size_t)nc, nullptr);
+    for (int c = 0; c < nc; ++c) r->rescol[c] = pack.as<char>() + 64 + (size_t)c * rcap * 8;
+    r->respack = std::move(pack);
+    r->capture_retain(ctx);
+    ctx->cap_results.push_back(r);
+    r->finalized = true;  // for this capture; hq_graph_launch re-opens it
+    return true;
+  }
   char* h = (char*)pinned_staging(ctx, 64 + body);
   HQ_CUDA(cudaMemcpyAsync(h, pack.p, 64 + body, cudaMemcpyDeviceToHost, ctx->stream));
   hq_sync(ctx, "a top-k finalize");
@@ -888,13 +906,13 @@ void hq_finalize_impl(hq_ctx* ctx, hq_result* r, bool unordered) {
     hq_check_result_faults(ctx, r);  // throws, or re-runs the pipeline with more room
     if (finalize_small(ctx, r)) return;
   }
-  hq_require_eager(ctx, "the finalize of a large, hash-grouped or materialised result");
   if (r->sink == HQ_SINK_AGG && r->plan.limit > 0 && r->plan.limit <= TOPK_MAX && r->plan.nkeys > 0 &&
       !getenv("HQ_NO_TOPK")) {
-    if (finalize_topk(ctx, r)) return;
+    if (finalize_topk(ctx, r)) return;  // (capturable: rows staged per launch)
     hq_check_result_faults(ctx, r);  // throws, or re-runs the pipeline with a larger group table
     if (finalize_topk(ctx, r)) return;  // (else: too many ties at the k-th key -- the full sort below)
   }
+  hq_require_eager(ctx, "the finalize of a large, hash-grouped or materialised result");
   hq_check_result_faults(ctx, r);
   const hq_plan& P = r->plan;
   if (r->sink == HQ_SINK_MATERIALISE) {

@@ -104,6 +104,9 @@ struct hq_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join[NSIDE] = {};
   // build statistics by (source table uid, descriptor bytes); HQ_BUILD_STATS=0 disables
   std::map<std::string, BuildStats> build_stats;
+  // row counts of materialised results viewed as tables, by derived table identity
+  // (hq_result_as_table): a repeated view skips the finalize's host synchronisation
+  std::map<uint64_t, int64_t> derived_rows;
   // CUDA-graph capture of a prepared query (hq_ctx_capture_begin/_end): the work is
   // captured on cap_stream; allocations come from the pool through alloc_stream (not
   // captured), frees are deferred to the graph's destruction, objects created or
@@ -205,6 +208,10 @@ struct hq_table : RefObj {
   TableCol cols[HQ_MAX_COLS];
   std::vector<DevBuf> owned;
   hq_result* backing = nullptr;  // retained when the table views a result
+  // a view of a materialised result sized by its cached row count (no host sync): the
+  // result's device row counter; consumers check it (builds on the device, pipelines by
+  // a host read) and raise HQ_ERR_STATE when it differs from nrows
+  const unsigned long long* dev_rows = nullptr;
   bool host_stream = false;      // HQ_HOST_STREAM: cols[].ptr are caller-owned host pointers
   ~hq_table() override;
 };
@@ -238,6 +245,7 @@ struct hq_hash : RefObj {
   // keys before each bitmap word | payload rows by rank, rstride int32 words each]
   // (hq_ranked_layout); a key's payload row = dir[w] + popc(bitmap[w] below its bit)
   int64_t src_rows = -1;  // rows of the build's source table (-1: imported / unknown)
+  uint64_t src_uid = 0;    // the build's source table (its cached derived row count is dropped on HQF_STALE)
   int64_t roff_dir = 0, roff_pay = 0;
   int rstride = 0;
   bool ranked() const { return ckind == 4; }
@@ -468,6 +476,7 @@ struct hq_result : RefObj {
   // finalized inside a graph capture: rows + stats land in stage_host at every launch
   void* stage_host = nullptr;        // pinned (cudaHostAlloc), owned
   int64_t stage_rcap = 0;
+  bool stage_topk = false;           // staged by the top-k finalize (stats word 5: too many ties)
   ~hq_result() override;
 };
 

@@ -733,7 +733,7 @@ void gen_we_tile(std::ostringstream& o, const KPlan& kp, int sk) {
     << "        const bool last_ = e_ + 1 == " << n << "; i64 v_[NAGGS > 0 ? NAGGS : 1];\n"
     << "        const u64 cnt_ = (u64)(last_ ? s_red[0] : wn_[e_ + 1]);\n";
   for (int a = 0; a < na; ++a) o << "        v_[" << a << "] = last_ ? s_red[" << 1 + a << "] : wv_s[" << a * N << " + e_ + 1];\n";
-  o << "        group_update(p, sagg, key_, false, cnt_, v_); }\n      consumer_bar();  // the next tile rewrites the sort buffers\n    }\n";
+  o << "        group_update(p, sagg, sl0_, key_, false, cnt_, v_); }\n      consumer_bar();  // the next tile rewrites the sort buffers\n    }\n";
 }
 
 std::string generate(const KPlan& kp) {
@@ -903,7 +903,7 @@ std::string generate(const KPlan& kp) {
         o
           << "#pragma unroll\n        for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) {\n"
           << "          i64 v_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n"
-          << "          group_update(p, sagg, gk_[r], true, cn_[r], v_); }\n"
+          << "          group_update(p, sagg, sl0_, gk_[r], true, cn_[r], v_); }\n"
           << "        nact_ = __popc(__ballot_sync(HQ_FULL, nact_ > 0));\n";
         o << "      } else {\n"
           << "#pragma unroll\n      for (int r = 0; r < R; ++r) {\n"
@@ -917,7 +917,7 @@ std::string generate(const KPlan& kp) {
       }
       if (wcompact || c2) o << "        const u32 am_ = __ballot_sync(HQ_FULL, live_);\n";
       if (c2) {
-        o << "        if (live_) group_update(p, sagg, key_, false, 1ull, v_);\n      }\n";
+        o << "        if (live_) group_update(p, sagg, sl0_, key_, false, 1ull, v_);\n      }\n";
       } else {
         o << "        const bool sparse_ = __popc(am_) <= 4;\n"
           << "        const u64 mk_ = live_ ? key_ : HQ_EMPTY_KEY;\n"
@@ -935,11 +935,11 @@ std::string generate(const KPlan& kp) {
         const char* op1 = getenv("HQ_JIT_ONEPASS");
         const bool onepass = op1 ? op1[0] == '1' : kp.smode == SM_NONE;
         if (!onepass) {
-          o << "        if (single_) group_update(p, sagg, key_, true, 1ull, v_);\n"
+          o << "        if (single_) group_update(p, sagg, sl0_, key_, true, 1ull, v_);\n"
             << "        while (multi_) {\n          const int leader_ = __ffs(multi_) - 1;\n"
             << "          const u32 grp_ = __shfl_sync(HQ_FULL, peers_, leader_); const bool mine_ = (grp_ >> lane) & 1u;\n"
             << "          i64 w_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n          for (int a = 0; a < NAGGS; ++a) w_[a] = warp_reduce(AGG_FN[a], mine_ ? v_[a] : agg_identity(AGG_FN[a]));\n"
-            << "          if (lane == leader_) group_update(p, sagg, key_, true, (u64)__popc(grp_), w_);\n"
+            << "          if (lane == leader_) group_update(p, sagg, sl0_, key_, true, (u64)__popc(grp_), w_);\n"
             << "          multi_ &= ~grp_;\n        }\n      }\n";
         } else {
           o << "        bool upd_ = single_; u64 uc_ = 1ull;\n"
@@ -949,7 +949,7 @@ std::string generate(const KPlan& kp) {
             << "          if (lane == leader_) {\n#pragma unroll\n            for (int a = 0; a < NAGGS; ++a) v_[a] = w_[a];\n"
             << "            uc_ = (u64)__popc(grp_); upd_ = true; }\n"
             << "          multi_ &= ~grp_;\n        }\n"
-            << "        if (upd_) group_update(p, sagg, key_, true, uc_, v_);\n      }\n";
+            << "        if (upd_) group_update(p, sagg, sl0_, key_, true, uc_, v_);\n      }\n";
         }
         if (!wcompact) o << "      }\n";  // else of the sparse path
       }
@@ -968,6 +968,7 @@ std::string generate(const KPlan& kp) {
     << "  u64* full = (u64*)smem; u64* empty = full + 10;\n"
     << "  u64* s_base = (u64*)(empty + 10); int* s_wtot = (int*)(s_base + 32); i64* s_red = (i64*)(s_wtot + 32);\n"
     << "  char* sagg = smem + OFF_AGG; char* stages = smem + OFF_STAGE;\n"
+    << "  const u32 sl0_ = smem_u32(sagg) + (u32)(((threadIdx.x >> 5) % SCOPIES) * SMEM_CAP * LVWORDS * 8u); (void)sl0_;\n"
     << "  const u32 sm0_ = smem_u32(smem); (void)sm0_;\n"
     << "  (void)s_base; (void)s_wtot; (void)s_red; (void)sagg;\n"
     << "  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;\n"
@@ -1345,7 +1346,7 @@ std::string generate(const KPlan& kp) {
       << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n";
     for (int a = 0; a < kp.naggs; ++a)
       o << "      vals_[" << a << "] = " << (kp.acc_of[a] ? "acc_[" + std::to_string(kp.acc_of[a]) + "]" : std::string("(i64)cnt_")) << ";\n";
-    o << "      group_update(p, sagg, g, false, cnt_, vals_);\n    } }\n";
+    o << "      group_update(p, sagg, sl0_, g, false, cnt_, vals_);\n    } }\n";
   } else if (sk == 1 && kp.smode == SM_DENSE) {
     // the group's entries in every replica are combined first
     o << "  consumer_bar();\n  { const i64* t_ = (const i64*)sagg;\n"
@@ -1372,12 +1373,12 @@ std::string generate(const KPlan& kp) {
       }
       o << " }\n";
     }
-    o << "        group_update(p, sagg, gkey_, false, (u64)cnt_, vals_); } } }\n";
+    o << "        group_update(p, sagg, sl0_, gkey_, false, (u64)cnt_, vals_); } } }\n";
   } else if (sk == 1 && kp.smode == SM_HASH) {
     o << "  consumer_bar();\n  { const u64* k_ = (const u64*)sagg; const i64* t_ = (const i64*)sagg + SMEM_CAP;\n"
       << "    for (u32 h = threadIdx.x; h < SMEM_CAP; h += NW * 32) if (k_[h] != HQ_EMPTY_KEY) { const i64* e_ = t_ + (u64)h * LVWORDS;\n"
       << "      i64 vals_[NAGGS > 0 ? NAGGS : 1];\n#pragma unroll\n      for (int a = 0; a < NAGGS; ++a) vals_[a] = AGG_FN[a] == F_COUNT ? e_[0] : e_[LCOL[a]];\n"
-      << "      group_update(p, sagg, k_[h], false, (u64)e_[0], vals_); } }\n";
+      << "      group_update(p, sagg, sl0_, k_[h], false, (u64)e_[0], vals_); } }\n";
   }
   if (prof) o << "  if (threadIdx.x == 0) { long long t_; asm volatile(\"mov.u64 %0, %%globaltimer;\" : \"=l\"(t_)); p.prof[blockIdx.x * 128] = pt0_; p.prof[blockIdx.x * 128 + 5] = t_;"
               << " unsigned sm_; asm(\"mov.u32 %0, %%smid;\" : \"=r\"(sm_)); p.prof[blockIdx.x * 128 + 6] = sm_; }\n";

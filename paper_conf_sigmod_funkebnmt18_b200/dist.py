@@ -347,8 +347,9 @@ class DistributedEngine(Engine):
         self.ctx.gather_faults(built, [res], red.data_ptr() + n * 8)
         reduce_partials(red, self.root)
         res.from_partials(red.data_ptr(), nbytes)
+        self._checked_built = built
         if not defer:
-            hq.raise_faults(red[n:].tolist())
+            self._raise(red[n:].tolist(), built)
             return None
         if getattr(self, "_fault_host", None) is None:
             self._fault_host = torch.empty(hq.FAULT_WORDS, dtype=torch.int64, pin_memory=True)
@@ -357,9 +358,25 @@ class DistributedEngine(Engine):
         self._fault_event.record(torch.cuda.current_stream(self.device))
         return self._fault_host
 
-    def _raise_deferred(self, words: torch.Tensor) -> None:
+    def _raise_deferred(self, words: torch.Tensor, built: Sequence[hq.Hash] = ()) -> None:
         self._fault_event.synchronize()  # (already complete after the root's fetch)
-        hq.raise_faults(words.tolist())
+        self._raise(words.tolist(), built)
+
+    @staticmethod
+    def _raise(words: Sequence[int], built: Sequence[hq.Hash]) -> None:
+        """hq.raise_faults; on stale build statistics, the tables this rank built are
+        checked first (hq_hash_info), which drops their cached statistics so that the
+        next run counts afresh instead of failing again."""
+        try:
+            hq.raise_faults(words)
+        except hq.HQError as e:
+            if e.code == hq.HQ_ERR_STATE:
+                for h in built:
+                    try:
+                        h.info()
+                    except hq.HQError:
+                        pass
+            raise
 
     def _root_only_checked(self, res: Optional[hq.Result]) -> None:
         """A root-only final pipeline: the root's build and pipeline faults are shared
@@ -369,7 +386,7 @@ class DistributedEngine(Engine):
         if self.rank == self.root:
             self.ctx.gather_faults(built, [res] if res is not None else [], st.data_ptr())
         _all_reduce(st)
-        hq.raise_faults(st.tolist())
+        self._raise(st.tolist(), built)
 
     def finish(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
         """Dense aggregates: one all-reduce of the partials (with every rank's fault
@@ -383,8 +400,8 @@ class DistributedEngine(Engine):
             words = self._reduce_checked(res, defer=True)
             try:
                 out = fetch(res, pb.result_names) if self.rank == self.root else None
-            finally:
-                self._raise_deferred(words)  # every rank raises the summed faults (before a fetch error)
+            finally:  # every rank raises the summed faults (before a fetch error)
+                self._raise_deferred(words, self._checked_built)
         else:
             out = self._merge_groups(res, pb)
         if self._trace is not None:
@@ -470,7 +487,7 @@ class DistributedEngine(Engine):
             raise err
         if stl[1]:
             raise RootError(hq.HQ_ERR_STATE, "pipeline failed on another rank")
-        hq.raise_faults(stl[2:])
+        self._raise(stl[2:], built)
         qual = int(stl[0])
         ncol = len(names)
         n = torch.tensor([nrows], dtype=torch.int64, device=self.device)

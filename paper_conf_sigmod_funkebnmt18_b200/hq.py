@@ -508,9 +508,13 @@ class Result:
         return int(self.info().qualifying_rows)
 
     def as_table(self, names: List[str]) -> Table:
+        """The result as a table (no host sync when a materialised result of the same
+        identity was viewed before: its row count is cached and checked on the device)."""
         h = ctypes.c_void_p()
         check(lib().hq_result_as_table(self.ctx.h, self.h, ctypes.byref(h)))
-        return Table(self.ctx, h, int(self.info().nrows), names, keep=[self])
+        n, nc = ctypes.c_int64(), ctypes.c_int32()
+        check(lib().hq_table_info(h, ctypes.byref(n), ctypes.byref(nc)))
+        return Table(self.ctx, h, int(n.value), names, keep=[self])
 
     def partials_view(self):
         p = ctypes.c_void_p()
