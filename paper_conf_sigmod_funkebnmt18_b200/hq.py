@@ -34,6 +34,7 @@ AGG_SUM, AGG_COUNT, AGG_MIN, AGG_MAX, AGG_AVG = 1, 2, 3, 4, 5
 SINK_AGG, SINK_MATERIALISE = 1, 2
 RES_LRGP, RES_ATOMIC, RES_WE = 0, 1, 2
 EXEC_FUSED, EXEC_OAAT, EXEC_FUSED_INTERP, EXEC_MULTIPASS = 0, 1, 2, 3
+HT_LINEAR, HT_DIRECT = 0, 1  # hq_hash_meta.layout
 
 
 def TMP(k: int) -> int:
