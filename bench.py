@@ -215,11 +215,15 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
     # co-partitioned queries (TPC-H Q3): orders and lineitem partitioned together by order,
     # every rank builds locally (dist.DistributedEngine copartitioned)
     copart = dist_mode and q.copart is not None and os.environ.get("HQ_DIST_COPART", "1") == "1"
+    # dimension tables replicated on every rank and built there (no table broadcast);
+    # HQ_DIST_BROADCAST=1: the root builds and broadcasts them
+    replicated = dist_mode and not copart and os.environ.get("HQ_DIST_BROADCAST") != "1"
     crange = None
     if copart:
         crange, (a, b) = hqgen.copartition(q.fact, q.copart, sf, rank, world, seed)
     if host is None:
-        host = gen_host(q, sf, seed, (a, b), with_dims=root or world == 1 or copart, copart_range=crange)
+        host = gen_host(q, sf, seed, (a, b), with_dims=root or world == 1 or copart or replicated,
+                        copart_range=crange)
     ctx = hq.Context(local)
     # HBM-resident copies (torch memory, borrowed by libhq)
     dtab = {t: {c: torch.from_numpy(np.asarray(arr)).to(dev) for c, arr in cols.items()} for t, cols in host.items()}
@@ -229,7 +233,7 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
     def make_engine(tbls):
         # HQ_FORCE_DIST=1 runs the distributed engine (broadcast + reduce) even at N=1
         if dist_mode:
-            return DistributedEngine(ctx, tbls, copartitioned=copart)
+            return DistributedEngine(ctx, tbls, copartitioned=copart, replicated=replicated)
         return Engine(ctx, tbls)
 
     E = make_engine(tables)
@@ -304,7 +308,7 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
            "local_rows": b - a, "result": out, "mode": mode, "step_ms_median": statistics.median(per),
            "step_ms_min": min(per), "eager": {"ms_per_step": ms_eager, "median": statistics.median(per_eager),
                                                "min": min(per_eager), "launches": launches_eager},
-           "prepared": prep, "copart": copart}
+           "prepared": prep, "copart": copart, "replicated": replicated}
     # ---- e2e: host (pinned) buffers through the public API, H2D inside the timed region.
     # Dimension tables are copied (HQ_HOST_COPY); the fact table streams from its pinned
     # host buffers through the fused kernel in blocks (HQ_HOST_STREAM, batch processing:
@@ -446,6 +450,8 @@ def run_hq(args):
                            "l2": "inputs larger than L2 (no flush needed)",
                            "parallelism": (f"orders/lineitem co-partitioned by order dp{world}, local builds, "
                                            "top-k rows gathered" if r["copart"] else
+                                           f"fact range partition dp{world}, dimensions replicated and built on every "
+                                           "rank, 1 reduce" if r["replicated"] else
                                            f"fact range partition dp{world}, dimension HTs broadcast, 1 reduce"),
                            "step": "hash builds + fused pipeline + reduce + finalize/fetch",
                            "step_mode": r["mode"] + (" (CUDA graph of the whole step; every kernel re-executed per step)"

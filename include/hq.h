@@ -234,11 +234,11 @@ typedef struct {
  * returns the compact form (meta.compact_kind != 0), which hq_hash_import accepts.
  * Sparse unique keys with a counted range that fits in 64 MiB of bits (layout
  * HQ_HT_LINEAR) are built into the *ranked form* instead of a slot array: one buffer
- * [bitmap of present keys over [key_min, key_max] | int32 rank directory, the number
- * of keys before each 32-bit bitmap word | payload rows by rank, 1 / 2 / 4 int32
- * words each (npayload 1 / 2 / 3; none without payload)], each part padded to whole
- * 8,192-word blocks and 256-B aligned -- a probe tests the key's bit (misses stop
- * there) and reads row dir[w] + popcount(bits below it).  The linear slot array the
+ * [the bitmap of present keys over [key_min, key_max] in 32-bit words -- with payloads
+ * as {bits, dir} word pairs, dir = the number of keys before the word | payload rows
+ * by rank, 1 / 2 / 4 int32 words each (npayload 1 / 2 / 3)], the bitmap padded to
+ * whole 8,192-word blocks -- a probe tests the key's bit (misses stop there) and reads
+ * row dir + popcount(bits below it).  The linear slot array the
  * meta describes (capacity, slot_words, bytes) is derived only for consumers that
  * read slots.  Other linear tables (expected_rows builds, composite keys, wider
  * ranges) keep the slot array, with an exact key-range bitmap in front of it when

@@ -57,7 +57,9 @@ struct KBuild {
 
 __device__ __forceinline__ long long live_rows(const KBuild& b) {
   if (!b.ndev) return b.n;
-  const long long d = (long long)*(const volatile unsigned long long*)b.ndev;
+  // (written by an earlier kernel: the read-only path, so that an SM's warps share one
+  // L2 request -- a volatile load from every warp made one hot L2 line)
+  const long long d = (long long)__ldg(b.ndev);
   if (d != b.n && blockIdx.x == 0 && threadIdx.x == 0) atomicOr(b.err, HQF_STALE);
   return d < b.n ? d : b.n;
 }
@@ -335,18 +337,29 @@ __global__ void hq_fill_kernel(uint32_t* p, long long n, uint32_t v) {
 // ---- ranked form of a sparse-key table (hq_hash::ranked): the bitmap of
 // present keys over the key range (built by hq_build_direct_compact_kernel, kind 1), a
 // rank directory (keys before each bitmap word: an exclusive scan of the words' popcounts)
-// and the payload rows stored densely by rank.  It replaces a linear table's slot array,
-// its fill and its key-range prefilter: no CAS, no probe sequence, a probe that misses
-// reads one bitmap word and a hit one directory word and one payload row.
-constexpr int RSCAN_T = 1024, RSCAN_W = 8;  // directory scan: 8 words (two 16-B loads) per thread
-__device__ __forceinline__ void rank_words(const uint32_t* bm, long long base, uint32_t (&c)[RSCAN_W]) {
-  const uint4 a = __ldg((const uint4*)(bm + base)), b = __ldg((const uint4*)(bm + base) + 1);
-  c[0] = a.x; c[1] = a.y; c[2] = a.z; c[3] = a.w; c[4] = b.x; c[5] = b.y; c[6] = b.z; c[7] = b.w;
+// and the payload rows stored densely by rank.  A table with payloads interleaves bitmap
+// and directory as {bits, dir} word pairs (ws = 2): a probe's one 8-B load gives both, so a
+// hit costs two dependent L2 loads (pair, payload row), not three.  It replaces a linear
+// table's slot array, its fill and its key-range prefilter: no CAS, no probe sequence.
+constexpr int RSCAN_T = 1024, RSCAN_W = 8;  // directory scan: 8 bitmap words per thread
+// the thread's 8 bitmap words (16-B loads; ws = 2: the .x of 8 {bits, dir} pairs)
+__device__ __forceinline__ void rank_words(const uint32_t* bm, int ws, long long base, uint32_t (&c)[RSCAN_W]) {
+  if (ws == 1) {
+    const uint4 a = __ldg((const uint4*)(bm + base)), b = __ldg((const uint4*)(bm + base) + 1);
+    c[0] = a.x; c[1] = a.y; c[2] = a.z; c[3] = a.w; c[4] = b.x; c[5] = b.y; c[6] = b.z; c[7] = b.w;
+    return;
+  }
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint4 a = __ldg((const uint4*)(bm + 2 * base) + q);
+    c[2 * q] = a.x;
+    c[2 * q + 1] = a.z;
+  }
 }
 // per block (8,192 words): number of present keys
-__global__ void __launch_bounds__(RSCAN_T) hq_rank_blocksum_kernel(const uint32_t* bm, unsigned* bsum) {
+__global__ void __launch_bounds__(RSCAN_T) hq_rank_blocksum_kernel(const uint32_t* bm, int ws, unsigned* bsum) {
   uint32_t c[RSCAN_W];
-  rank_words(bm, ((long long)blockIdx.x * RSCAN_T + threadIdx.x) * RSCAN_W, c);
+  rank_words(bm, ws, ((long long)blockIdx.x * RSCAN_T + threadIdx.x) * RSCAN_W, c);
   unsigned n = 0;
 #pragma unroll
   for (int j = 0; j < RSCAN_W; ++j) n += __popc(c[j]);
@@ -369,11 +382,12 @@ __global__ void __launch_bounds__(RSCAN_T) hq_rank_topscan_kernel(unsigned* bsum
     __syncthreads();  // tmp reuse
   }
 }
-// directory: keys before each word = block offset + block-exclusive scan + running sum
-__global__ void __launch_bounds__(RSCAN_T) hq_rank_dir_kernel(const uint32_t* bm, const unsigned* bsum, unsigned* dir) {
+// directory: keys before each word = block offset + block-exclusive scan + running sum,
+// written with the bitmap words as the {bits, dir} pairs
+__global__ void __launch_bounds__(RSCAN_T) hq_rank_dir_kernel(const uint32_t* bm, const unsigned* bsum, uint32_t* bd) {
   const long long base = ((long long)blockIdx.x * RSCAN_T + threadIdx.x) * RSCAN_W;
   uint32_t c[RSCAN_W];
-  rank_words(bm, base, c);
+  rank_words(bm, 1, base, c);
   unsigned n = 0;
 #pragma unroll
   for (int j = 0; j < RSCAN_W; ++j) n += __popc(c[j]);
@@ -381,20 +395,20 @@ __global__ void __launch_bounds__(RSCAN_T) hq_rank_dir_kernel(const uint32_t* bm
   __shared__ typename BS::TempStorage tmp;
   unsigned ex;
   BS(tmp).ExclusiveSum(n, ex);
-  unsigned run = bsum[blockIdx.x] + ex, d[RSCAN_W];
+  unsigned run = bsum[blockIdx.x] + ex;
 #pragma unroll
-  for (int j = 0; j < RSCAN_W; ++j) {
-    d[j] = run;
-    run += __popc(c[j]);
+  for (int q = 0; q < 4; ++q) {
+    const unsigned d0 = run;
+    run += __popc(c[2 * q]);
+    const unsigned d1 = run;
+    run += __popc(c[2 * q + 1]);
+    ((uint4*)(bd + 2 * base))[q] = make_uint4(c[2 * q], d0, c[2 * q + 1], d1);
   }
-  ((uint4*)(dir + base))[0] = make_uint4(d[0], d[1], d[2], d[3]);
-  ((uint4*)(dir + base))[1] = make_uint4(d[4], d[5], d[6], d[7]);
 }
 // payload rows by rank: each qualifying row finds its key's rank and writes its payloads
 __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_ranked_scatter_kernel(const __grid_constant__ KBuild b,
-                                                                             const uint32_t* bm, const unsigned* dir,
-                                                                             int* rpay, int stride, long long range,
-                                                                             unsigned long long nkeys) {
+                                                                             const uint2* bd, int* rpay, int stride,
+                                                                             long long range, unsigned long long nkeys) {
   int fault = 0;
   const long long base = (long long)blockIdx.x * BUILD_BLOCK * BUILD_U + threadIdx.x;
   bool pass[BUILD_U];
@@ -417,14 +431,15 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_ranked_scatter_kernel(co
   unsigned rk[BUILD_U];
   bool ok[BUILD_U];
 #pragma unroll
-  for (int u = 0; u < BUILD_U; ++u) {  // the directory and bitmap loads of all U rows in flight together
+  for (int u = 0; u < BUILD_U; ++u) {  // the pair loads of all U rows in flight together
     const long long d = kv[u] - (long long)b.dmin;
     ok[u] = pass[u] && kv[u] > (long long)INT_MIN && kv[u] <= (long long)INT_MAX && d >= 0 && d < range;
     rk[u] = 0;
     if (ok[u]) {
-      const uint32_t w = __ldg(bm + (d >> 5)), bit = 1u << (d & 31);
-      ok[u] = (w & bit) != 0;
-      rk[u] = __ldg(dir + (d >> 5)) + __popc(w & (bit - 1u));
+      const uint2 q = __ldg(bd + (d >> 5));
+      const uint32_t bit = 1u << (d & 31);
+      ok[u] = (q.x & bit) != 0;
+      rk[u] = q.y + __popc(q.x & (bit - 1u));
     }
   }
 #pragma unroll
@@ -443,14 +458,14 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_ranked_scatter_kernel(co
 }
 // the linear slot array of a ranked table, for consumers that read slots (interpreter,
 // operator-at-a-time): every present key claims a slot as in hq_build_hash_kernel
-__global__ void hq_slots_from_ranked_kernel(const uint32_t* bm, const unsigned* dir, const int* rpay, int stride,
-                                            int npay, long long range, int kmin, uint32_t* slots, uint32_t mask,
-                                            int log2cap, int words, int* err) {
+__global__ void hq_slots_from_ranked_kernel(const uint32_t* bm, const int* rpay, int stride, int npay, long long range,
+                                            int kmin, uint32_t* slots, uint32_t mask, int log2cap, int words, int* err) {
+  const int ws = stride ? 2 : 1;
   for (long long d = blockIdx.x * (long long)blockDim.x + threadIdx.x; d < range; d += (long long)gridDim.x * blockDim.x) {
-    const uint32_t w = bm[d >> 5], bit = 1u << (d & 31);
+    const uint32_t w = bm[(d >> 5) * ws], bit = 1u << (d & 31);
     if (!(w & bit)) continue;
     const int key = kmin + (int)d;
-    const int* src = stride ? rpay + (size_t)(dir[d >> 5] + __popc(w & (bit - 1u))) * stride : nullptr;
+    const int* src = stride ? rpay + (size_t)(bm[(d >> 5) * 2 + 1] + __popc(w & (bit - 1u))) * stride : nullptr;
     uint32_t pos = ((uint32_t)key * 0x9E3779B1u) >> (32 - log2cap);
     for (uint32_t n = 0;; ++n) {
       if (n > mask) {
@@ -612,18 +627,18 @@ int hq_compact_kind(int npayload, int pay_min, int pay_max) {
 long long hq_compact_words(int kind, long long range) {
   return kind == 1 ? (range + 31) / 32 : (kind == 3 ? (range + 7) / 8 : (range + 3) / 4);
 }
-// ranked form: [bitmap | directory | payload rows], the bitmap and directory padded to
-// whole 8,192-word scan blocks (the scan kernels read and write them without bounds
-// checks; the bitmap's padding is zero), every part 256-B aligned; no directory or
-// payload rows for a table without payload (a semi / anti join reads the bitmap only)
+// ranked form: [bitmap words | payload rows], or with payloads [{bits, dir} word pairs |
+// payload rows]; the bitmap padded to whole 8,192-word scan blocks (the scan kernels read
+// and write them without bounds checks; the padding is zero), the rows 256-B aligned.
+// off_dir: byte offset of directory word 0 (word w's at off_dir + 8 w), 0 without payload.
 void hq_ranked_layout(int64_t range, int64_t nkeys, int npay, int64_t* off_dir, int64_t* off_pay, int64_t* total,
                       int* stride) {
   const int64_t blk = 1024 * 8;
   const int64_t words = ((range + 31) / 32 + blk - 1) / blk * blk;
   const int st = npay == 0 ? 0 : (npay == 1 ? 1 : (npay == 2 ? 2 : 4));
   *stride = st;
-  *off_dir = words * 4;
-  *off_pay = *off_dir + (st ? words * 4 : 0);
+  *off_dir = st ? 4 : 0;
+  *off_pay = words * 4 * (st ? 2 : 1);
   *total = *off_pay + (int64_t)st * 4 * (nkeys > 0 ? nkeys : 0);
 }
 // rank LUT of a byte map over a sparse payload set (value - pay_min -> rank, 0xFF
@@ -813,24 +828,34 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
     int stride = 0;
     hq_ranked_layout(range, keys, d->npayload, &od, &op, &tot, &stride);
     h->compact = DevBuf(ctx, (size_t)tot + 16);
-    HQ_CUDA(cudaMemsetAsync(h->compact.p, 0, (size_t)od, ctx->stream));  // the bitmap and its padding
+    // the bitmap is built apart (dense words: contiguous atomics, a half-size scan) and the
+    // directory kernel writes it out with the directory as the {bits, dir} pairs
+    const int64_t bwords = stride ? op / 8 : op / 4;
+    DevBuf scratch;
     uint32_t* bm = h->compact.as<uint32_t>();
+    if (stride) {
+      scratch = DevBuf(ctx, (size_t)bwords * 4 + 16);
+      bm = scratch.as<uint32_t>();
+    }
+    HQ_CUDA(cudaMemsetAsync(bm, 0, (size_t)bwords * 4, ctx->stream));  // the bitmap and its padding
     b.dmin = (int32_t)kmin;
     if (b.n > 0) {  // bitmap + duplicate / bad-key / statistics checks
       ctx->launches++;
       hq_build_direct_compact_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(b, 1, bm, range, 0, 0, CLut{});
     }
     HQ_CUDA(cudaGetLastError());
-    if (stride && b.n > 0) {
-      const int nblk = (int)(od / 4 / (RSCAN_T * RSCAN_W));
+    if (stride) {
+      const int nblk = (int)(bwords / (RSCAN_T * RSCAN_W));
       DevBuf bsum(ctx, (size_t)nblk * 4 + 16);
-      unsigned* dir = (unsigned*)(h->compact.as<char>() + od);
-      ctx->launches += 4;
-      hq_rank_blocksum_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, bsum.as<unsigned>());
+      ctx->launches += 3;
+      hq_rank_blocksum_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, 1, bsum.as<unsigned>());
       hq_rank_topscan_kernel<<<1, RSCAN_T, 0, ctx->stream>>>(bsum.as<unsigned>(), nblk);
-      hq_rank_dir_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, bsum.as<unsigned>(), dir);
-      hq_build_ranked_scatter_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(
-          b, bm, dir, (int*)(h->compact.as<char>() + op), stride, range, (unsigned long long)keys);
+      hq_rank_dir_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, bsum.as<unsigned>(), h->compact.as<uint32_t>());
+      if (b.n > 0) {
+        ctx->launches++;
+        hq_build_ranked_scatter_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(
+            b, h->compact.as<uint2>(), (int*)(h->compact.as<char>() + op), stride, range, (unsigned long long)keys);
+      }
       HQ_CUDA(cudaGetLastError());
     }
     h->ckind = 4;
@@ -1085,9 +1110,8 @@ const uint32_t* hq_hash_slots(hq_ctx* ctx, hq_hash* h) {
     ctx->launches += 2;
     hq_fill_kernel<<<fgrid, 256, 0, ctx->stream>>>(h->owned.as<uint32_t>(), cap * words, 0x80000000u);
     hq_slots_from_ranked_kernel<<<grid, 256, 0, ctx->stream>>>(
-        (const uint32_t*)base, (const unsigned*)(base + h->roff_dir), (const int*)(base + h->roff_pay), h->rstride,
-        h->meta.npayload, range, (int)h->meta.key_min, h->owned.as<uint32_t>(), (uint32_t)(cap - 1), h->log2cap, words,
-        h->dstate.as<int>());
+        (const uint32_t*)base, (const int*)(base + h->roff_pay), h->rstride, h->meta.npayload, range,
+        (int)h->meta.key_min, h->owned.as<uint32_t>(), (uint32_t)(cap - 1), h->log2cap, words, h->dstate.as<int>());
     HQ_CUDA(cudaGetLastError());
     h->slots = h->owned.as<uint32_t>();
     return h->slots;

@@ -367,7 +367,24 @@ __global__ void __launch_bounds__(256) hq_topk_minmax_kernel(const __grid_consta
     qs += __shfl_xor_sync(0xffffffffu, qs, o);
     ls += __shfl_xor_sync(0xffffffffu, ls, o);
   }
+  // one set of atomics per block, not per warp (same-address atomics serialise: ~9 K
+  // warps on four words took most of the kernel's 24 us at TPC-H Q3 SF30)
+  __shared__ unsigned long long red[4][8];
+  const int w = threadIdx.x >> 5;
   if ((threadIdx.x & 31) == 0) {
+    red[0][w] = mn;
+    red[1][w] = mx;
+    red[2][w] = qs;
+    red[3][w] = ls;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int i = 1; i < (int)(blockDim.x >> 5); ++i) {
+      mn = red[0][i] < mn ? red[0][i] : mn;
+      mx = red[1][i] > mx ? red[1][i] : mx;
+      qs += red[2][i];
+      ls += red[3][i];
+    }
     if (ls) {
       atomicMin(sel + 0, mn);
       atomicMax(sel + 1, mx);

@@ -241,9 +241,9 @@ struct hq_hash : RefObj {
   DevBuf prefilter;
   int64_t pf_words = 0;
   // ckind 4 (compact_only): the *ranked* form of a sparse-key (linear) table, one buffer
-  // [bitmap of present keys over key_max - key_min + 1 | rank directory: int32 number of
-  // keys before each bitmap word | payload rows by rank, rstride int32 words each]
-  // (hq_ranked_layout); a key's payload row = dir[w] + popc(bitmap[w] below its bit)
+  // [bitmap of present keys over key_max - key_min + 1 -- with payloads as {bits, dir}
+  // word pairs, dir = the number of keys before the word | payload rows by rank, rstride
+  // int32 words each] (hq_ranked_layout); a key's payload row = dir + popc(bits below it)
   int64_t src_rows = -1;  // rows of the build's source table (-1: imported / unknown)
   uint64_t src_uid = 0;    // the build's source table (its cached derived row count is dropped on HQF_STALE)
   int64_t roff_dir = 0, roff_pay = 0;
@@ -334,10 +334,9 @@ struct KProbe {
   uint8_t composite;   // two-column key: slot word 1 must equal key2_reg; payloads from word 2
   int16_t key2_reg;
   uint8_t crank;       // ckind 2: the byte is the payload's RANK in pay_set (sparse value sets)
-  // ranked form of a linear table (hq_hash::ranked): pf = its bitmap, rdir = rank
-  // directory, rpay = payload rows (rstride words) by rank; slots unused
+  // ranked form of a linear table (hq_hash::ranked): pf = its bitmap (rstride > 0: the
+  // {bits, rank directory} word pairs), rpay = payload rows (rstride words) by rank
   uint8_t ranked, rstride;
-  const uint32_t* rdir;
   const int32_t* rpay;
 };
 struct KCompute {

@@ -32,7 +32,6 @@ using namespace hqk;
     const unsigned* ht[8];                                                                                     \
     const void* ctab[8];                                                                                       \
     const unsigned* pf[8];                                                                                     \
-    const unsigned* rdir[8];                                                                                   \
     const int* rpay[8];                                                                                        \
     long long* gtab;                                                                                           \
     unsigned long long gmask;                                                                                  \
@@ -364,32 +363,35 @@ struct Gen {
   }
 
   // ranked sparse-key table (hq_hash::ranked): the key's bit in the range bitmap
-  // (misses stop here, L2-resident), then for a hit that needs payloads its rank =
-  // directory word + popcount of the bits below it, and the payload row at that rank;
-  // each step's loads for the lane's R rows are issued together
+  // (misses stop here, L2-resident); with payloads the bitmap word comes with the rank
+  // directory word in one 8-B load, and a hit's payload row is at dir + popcount(bits
+  // below it) -- two dependent loads; each step's loads for the lane's R rows together
   void probe_ranked(const KProbe& pr, int idx) {
     const int npay = hq_probe_has_payload(pr.mode) ? pr.npay : 0;
     probe_defs(pr);
     const std::string key = val(pr.key_reg), I = std::to_string(idx);
-    o << "      { u32 found_ = 0u; u32 w_[R]; u32 e_[R]; bool h_[R];\n"
+    const bool pairs = pr.rstride > 0;  // the table's layout (a semi-join may probe a table with payloads)
+    o << "      { u32 found_ = 0u; u32 w_[R]; u32 e_[R]; bool h_[R];" << (npay > 0 ? " u32 k_[R];" : "") << "\n"
       << "#pragma unroll\n        for (int r = 0; r < R; ++r) {\n"
       << "          const long long d_ = (long long)" << key << " - (" << pr.pf_min << "LL); e_[r] = (u32)d_;\n"
-      << "          h_[r] = ((mask >> r) & 1u) && d_ >= 0 && d_ < " << pr.pf_range << "LL;\n"
-      << "          w_[r] = h_[r] ? __ldg(p.pf[" << I << "] + (e_[r] >> 5)) : 0u; }\n"
-      << "#pragma unroll\n        for (int r = 0; r < R; ++r) { h_[r] = (w_[r] >> (e_[r] & 31u)) & 1u;"
+      << "          h_[r] = ((mask >> r) & 1u) && d_ >= 0 && d_ < " << pr.pf_range << "LL;\n";
+    if (pairs && npay > 0)
+      o << "          uint2 q_ = make_uint2(0u, 0u); if (h_[r]) q_ = __ldg((const uint2*)p.pf[" << I
+        << "] + (e_[r] >> 5)); w_[r] = q_.x; k_[r] = q_.y; }\n";
+    else
+      o << "          w_[r] = h_[r] ? __ldg(p.pf[" << I << "] + (e_[r] >> 5)" << (pairs ? " * 2u" : "") << ") : 0u; }\n";
+    o << "#pragma unroll\n        for (int r = 0; r < R; ++r) { h_[r] = (w_[r] >> (e_[r] & 31u)) & 1u;"
       << " if (h_[r]) found_ |= 1u << r; }\n";
     if (npay > 0) {
       static const char* comp[4] = {"x", "y", "z", "w"};
-      o << "        u32 k_[R];\n"
-        << "#pragma unroll\n        for (int r = 0; r < R; ++r) if (h_[r]) k_[r] = __ldg(p.rdir[" << I
-        << "] + (e_[r] >> 5)) + __popc(w_[r] & ((1u << (e_[r] & 31u)) - 1u));\n"
-        << "#pragma unroll\n        for (int r = 0; r < R; ++r) if (h_[r]) {";
+      o << "#pragma unroll\n        for (int r = 0; r < R; ++r) if (h_[r]) {"
+        << " const u32 rk_ = k_[r] + __popc(w_[r] & ((1u << (e_[r] & 31u)) - 1u));";
       if (pr.rstride == 1) {
-        o << " " << var(pr.dst[0]) << "[r] = __ldg(p.rpay[" << I << "] + k_[r]);";
+        o << " " << var(pr.dst[0]) << "[r] = __ldg(p.rpay[" << I << "] + rk_);";
       } else {
-        o << " const " << (pr.rstride == 2 ? "int2" : "int4") << " q_ = __ldg((const " << (pr.rstride == 2 ? "int2" : "int4")
-          << "*)p.rpay[" << I << "] + k_[r]);";
-        for (int k = 0; k < npay; ++k) o << " " << var(pr.dst[k]) << "[r] = q_." << comp[k] << ";";
+        o << " const " << (pr.rstride == 2 ? "int2" : "int4") << " v_ = __ldg((const " << (pr.rstride == 2 ? "int2" : "int4")
+          << "*)p.rpay[" << I << "] + rk_);";
+        for (int k = 0; k < npay; ++k) o << " " << var(pr.dst[k]) << "[r] = v_." << comp[k] << ";";
       }
       o << " }\n";
     }
@@ -473,11 +475,14 @@ struct Gen {
     std::vector<int> b = {i};
     if (ak != AK_SMEM) {  // a global probe: the following independent global probes join its batch
       // (no early exit in front: the warp rarely has no live row here, and the
-      // extra branch measured slower)
+      // extra branch measured slower); so do following shared-memory probes, whose
+      // loads then issue under the global round trip instead of after it (they cost a
+      // few shared loads for rows the batch drops; HQ_JIT_NOSMEMJOIN=1: not joined)
+      const bool smem_join = !getenv("HQ_JIT_NOSMEMJOIN");
       std::set<int> defs(first.dst, first.dst + (hq_probe_has_payload(first.mode) ? first.npay : 0));
       for (int j = i + 1; j < kp.nops && kp.ops[j].kind == OP_PROBE && !kp.op_skip[j]; ++j) {
         const KProbe& pr = kp.probes[kp.ops[j].idx];
-        if (access(pr) == AK_LINEAR || access(pr) == AK_SMEM || defs.count(pr.key_reg)) break;
+        if (access(pr) == AK_LINEAR || (access(pr) == AK_SMEM && !smem_join) || defs.count(pr.key_reg)) break;
         b.push_back(j);
         for (int k = 0; k < (hq_probe_has_payload(pr.mode) ? pr.npay : 0); ++k) defs.insert(pr.dst[k]);
       }
@@ -1477,7 +1482,6 @@ std::string plan_key(const KPlan& kp) {
     pr.slots = (const uint32_t*)nz(pr.slots);
     pr.compact = nz(pr.compact);
     pr.pf = (const uint32_t*)nz(pr.pf);
-    pr.rdir = (const uint32_t*)nz(pr.rdir);
     pr.rpay = (const int32_t*)nz(pr.rpay);
   }
   k.gtab = (long long*)nz(k.gtab);
@@ -1519,7 +1523,6 @@ void hq_jit_launch(hq_ctx* ctx, const KPlan& kp, int grid, size_t smem) {
     jp.ht[i] = kp.probes[i].slots;
     jp.ctab[i] = kp.probes[i].compact;
     jp.pf[i] = kp.probes[i].pf;
-    jp.rdir[i] = kp.probes[i].rdir;
     jp.rpay[i] = kp.probes[i].rpay;
   }
   jp.gtab = kp.gtab;

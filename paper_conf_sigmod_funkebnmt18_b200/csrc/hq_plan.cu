@@ -136,7 +136,6 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.crank = (uint8_t)op.ht->crank;
       pr.compact = rk ? nullptr : op.ht->compact_ptr();
       pr.rstride = (uint8_t)op.ht->rstride;
-      pr.rdir = nullptr;
       pr.rpay = nullptr;
       pr.pay_min = op.ht->meta.pay_min;
       pr.pay_max = op.ht->meta.pay_max;
@@ -158,11 +157,8 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       pr.pf = op.ht->pf_words ? op.ht->prefilter.as<uint32_t>() : nullptr;
       if (pr.ranked) {
         const char* base = (const char*)op.ht->compact_ptr();
-        pr.pf = (const uint32_t*)base;
-        if (pr.rstride) {
-          pr.rdir = (const uint32_t*)(base + op.ht->roff_dir);
-          pr.rpay = (const int32_t*)(base + op.ht->roff_pay);
-        }
+        pr.pf = (const uint32_t*)base;  // bitmap words, or {bits, dir} pairs when the table has payloads
+        if (pr.rstride) pr.rpay = (const int32_t*)(base + op.ht->roff_pay);
       }
       pr.pf_min = (int32_t)op.ht->meta.key_min;
       pr.pf_range = (uint32_t)((int64_t)op.ht->meta.key_max - op.ht->meta.key_min + 1);

@@ -9,6 +9,9 @@
 * each rank runs the fused pipeline over its range; dense partial aggregates
   ([count, agg...] per group, int64) are combined with ONE ``dist.reduce``
   (SUM) to the root, which finalizes (ORDER BY / LIMIT on GPU 0);
+* replicated dimensions (``DistributedEngine(replicated=True)``, the bench's default):
+  every rank holds the dimension tables and builds them itself -- no broadcast; only
+  tables built over a result that exists on the root alone (after a gather) are sent;
 * co-partitioned queries (``Query.copart``, TPC-H Q3): the order table and the line
   table are partitioned together by order (``hqgen.copartition``: rank r's lines are
   exactly the lines of its orders), every rank builds all of its tables locally (no
@@ -211,7 +214,8 @@ class DistributedEngine(Engine):
     """Engine whose builds happen on the root and are broadcast, and whose
     partitioned pipelines end with one reduce of the dense partials."""
 
-    def __init__(self, ctx: hq.Context, tables, root: int = 0, copartitioned: bool = False, **kw):
+    def __init__(self, ctx: hq.Context, tables, root: int = 0, copartitioned: bool = False, replicated: bool = False,
+                 **kw):
         super().__init__(ctx, tables, **kw)
         self.rank = dist.get_rank()
         self.world = dist.get_world_size()
@@ -222,7 +226,13 @@ class DistributedEngine(Engine):
         # copartitioned: the tables are this rank's co-partition (hqgen.copartition) plus
         # full copies of the small dimensions; every rank builds and runs locally
         self.copartitioned = copartitioned
-        self.builds_here = copartitioned or self.rank == root
+        # replicated: every rank holds the full dimension tables (the fact table stays range-
+        # partitioned) and runs the build side itself -- builds over base tables and the
+        # unpartitioned pipelines over them -- so no table is broadcast; only builds over a
+        # result that exists on the root alone (after a gather) still are
+        self.replicated = replicated
+        self._local_results: set = set()  # ids of results every rank computed itself
+        self.builds_here = copartitioned or replicated or self.rank == root
         # HQ_DIST_FAULT_TRACE=1 (debug): re-read every root build's fault word after the
         # final fetch and report the ones that changed since the build
         self._trace: Optional[List[Tuple[str, hq.Hash, List[int]]]] = (
@@ -251,8 +261,8 @@ class DistributedEngine(Engine):
         rows, bufs = broadcast_tables(None, None, n, self.root, self.device, state=self._bcast)
         return [self.ctx.import_hash(meta_from_row(r), b.data_ptr(), keep=b) for r, b in zip(rows, bufs)]  # views keep the buffer
 
-    def _root_build(self, fn, n: int):
-        if self.copartitioned:  # local build over this rank's co-partition: nothing to share
+    def _root_build(self, fn, n: int, local: bool = False):
+        if self.copartitioned or local:  # built on every rank from data it holds: nothing to share
             hs = fn()
             self._built.extend(hs)
             return hs
@@ -266,14 +276,16 @@ class DistributedEngine(Engine):
 
     def hash(self, table, key, payload=(), preds=(), expected_rows=0, key2=None) -> hq.Hash:
         return self._root_build(lambda: [super(DistributedEngine, self).hash(table, key, payload, preds,
-                                                                             expected_rows, key2)], 1)[0]
+                                                                             expected_rows, key2)], 1,
+                                self.replicated)[0]
 
     def hashes(self, specs) -> List[hq.Hash]:
-        return self._root_build(lambda: super(DistributedEngine, self).hashes(specs), len(specs))
+        return self._root_build(lambda: super(DistributedEngine, self).hashes(specs), len(specs), self.replicated)
 
     def hash_from(self, res, names, key, payload=(), preds=()) -> hq.Hash:
+        local = self.replicated and res is not None and id(res) in self._local_results
         return self._root_build(lambda: [super(DistributedEngine, self).hash_from(res, names, key, payload,
-                                                                                  preds)], 1)[0]
+                                                                                  preds)], 1, local)[0]
 
     @staticmethod
     def _hash_grouped(P: hq.Plan) -> bool:
@@ -299,6 +311,13 @@ class DistributedEngine(Engine):
             pb.dist_order = ([(P.order_col[i], P.order_desc[i]) for i in range(P.norder)], P.limit)
             pb.copart_local_order = True
             return super().run(pb, partitioned)
+        if not partitioned and self.replicated and any(pb.fact is t for t in self.tables.values()):
+            # a build-side pipeline over (replicated) base tables: every rank runs it
+            res = super().run(pb, partitioned)
+            pb.replicated_local = True
+            self._local_results.add(id(res))
+            pb.keep.append(res)  # (keeps the id valid while the plan lives)
+            return res
         if not partitioned:
             pb.root_only = True  # a build-side or post-merge pipeline: the root's result is complete
             if self.rank != self.root:
@@ -393,7 +412,12 @@ class DistributedEngine(Engine):
         words), root finalizes.  Hash group-bys (e.g. TPC-H Q3 by l_orderkey): every rank
         finalizes its groups, the rows are all-gathered to the root, which merges them
         with one more fused GROUP BY pipeline on its GPU (and applies ORDER BY / LIMIT)."""
-        if getattr(pb, "root_only", False):  # no data collective: the root ran the whole pipeline
+        if getattr(pb, "replicated_local", False):  # every rank computed the whole result
+            if self.rank != self.root:
+                res.finalize()  # (the same faults as the root's: every rank raises, or none)
+            self._built = []
+            out = fetch(res, pb.result_names) if self.rank == self.root else None
+        elif getattr(pb, "root_only", False):  # no data collective: the root ran the whole pipeline
             self._root_only_checked(res)
             out = fetch(res, pb.result_names) if self.rank == self.root else None
         elif not hasattr(pb, "dist_order"):
@@ -433,7 +457,7 @@ class DistributedEngine(Engine):
         group-bys are merged on the root (all-gather of the ranks' groups + one fused merge
         pipeline; an order split by the range partition is combined there), dense ones are
         summed with one all-reduce.  Returns the device result on the root, None elsewhere."""
-        if getattr(pb, "root_only", False):
+        if getattr(pb, "root_only", False) or getattr(pb, "replicated_local", False):
             return res
         if self.copartitioned:
             raise NotImplementedError("co-partitioned execution: intermediate gathers are not supported")

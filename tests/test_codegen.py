@@ -35,9 +35,10 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert p.stdout.startswith("OK 32 of 32"), p.stdout
     srcs = {f[:-3]: open(tmp_path / f).read() for f in os.listdir(tmp_path)}
     # the probe kinds the shapes were built to exercise are present
-    rk = srcs["ranked_probes"]  # ranked sparse-key tables: bitmap, directory + popcount, payload rows
-    assert "__ldg(p.pf[0] + (e_[r] >> 5))" in rk and "__ldg(p.rdir[0] + (e_[r] >> 5)) + __popc(w_[r]" in rk
-    assert "(const int2*)p.rpay[0]" in rk and "__ldg(p.rpay[2] + k_[r])" in rk and "p.rdir[1]" not in rk
+    rk = srcs["ranked_probes"]  # ranked sparse-key tables: {bits, dir} pair, popcount, payload row
+    assert "__ldg((const uint2*)p.pf[0] + (e_[r] >> 5))" in rk and "k_[r] + __popc(w_[r]" in rk
+    assert "(const int2*)p.rpay[0] + rk_" in rk and "__ldg(p.rpay[2] + rk_)" in rk
+    assert "__ldg(p.pf[1] + (e_[r] >> 5)) : 0u" in rk and "p.rpay[1]" not in rk  # semi-join: bits only
     assert "p.ht[0]" not in rk and "0x9E3779B1u" not in rk.split("gk_")[0]
     star = srcs["star_dense_lrgp"]
     assert "lds_u32(sm0_ + " in star                 # staged bitmap

@@ -24,7 +24,7 @@ def _port():
     return p
 
 
-def _worker(rank, world, port, q, qs=None, sf=None, copart=False):
+def _worker(rank, world, port, q, qs=None, sf=None, copart=False, replicated=False):
     qs = QS if qs is None else qs
     sf = SF if sf is None else sf
     try:
@@ -50,8 +50,8 @@ def _worker(rank, world, port, q, qs=None, sf=None, copart=False):
                 tables = load_tables(ctx, qq, sf, fact_range=rng, copart_range=crng)
             else:
                 rng = partition(n, rank, world)
-                tables = load_tables(ctx, qq, sf, fact_range=rng, skip_dims=rank != 0)
-            E = DistributedEngine(ctx, tables, copartitioned=copart)
+                tables = load_tables(ctx, qq, sf, fact_range=rng, skip_dims=rank != 0 and not replicated)
+            E = DistributedEngine(ctx, tables, copartitioned=copart, replicated=replicated)
             r = run_query(E, qq)
             out[qn] = (r.rows(), r.qualifying) if r is not None else None
         q.put(("ok", rank, out))
@@ -178,3 +178,48 @@ def test_copartitioned_tpch_q3(world, sf):
     o3 = oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
     assert rows == o3.rows(["l_orderkey", "o_orderdate", "o_shippriority", "revenue", "count"])[:10]
     assert qual == int(o3.columns["count"].sum())  # lineitem rows that reached the GROUP BY, all ranks
+
+
+REPL = ["ssb_q41", "ssb_q31", "tpch_q1", "tpch_q3", "tpch_q5", "tpch_q4", "tpch_q13", "tpch_q18", "tpch_q21"]
+
+
+def test_replicated_dimensions_match_oracle():
+    """Replicated dimensions (the bench's default multi-GPU mode): every rank builds the
+    dimension tables and runs the build-side pipelines itself (no broadcast), only
+    tables over a gathered result are sent; two ranks at SF 0.01, rows equal the oracle."""
+    import hqgen
+    import oracle
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, REPL, 0.01, False, True)) for r in range(2)]
+    for p in procs:
+        p.start()
+    outs = [q.get(timeout=900) for _ in procs]
+    for p in procs:
+        p.join(timeout=120)
+    errs = [o for o in outs if o[0] != "ok"]
+    if errs:
+        pytest.fail("\n\n".join(f"rank {o[1]}:\n{o[2]}" for o in errs))
+    root = {k: v[0] for k, v in next(o[2] for o in outs if o[1] == 0).items()}
+    assert all(o[2][qn] is None for o in outs if o[1] != 0 for qn in REPL)
+    ssb = {t: hqgen.generate(t, 0.01) for t in hqgen.SSB_TABLES}
+    t = {x: hqgen.generate(x, 0.01) for x in hqgen.TPCH_TABLES}
+    exp = {
+        "ssb_q41": oracle.ssb_q41(ssb["lineorder"], ssb["date"], ssb["customer"], ssb["supplier"], ssb["part"]).rows(),
+        "ssb_q31": oracle.ssb_q31(ssb["lineorder"], ssb["customer"], ssb["supplier"], ssb["date"]).rows(),
+        "tpch_q5": oracle.tpch_q5(t["tpch_customer"], t["orders"], t["lineitem"], t["tpch_supplier"], t["nation"],
+                                  t["region"]).rows(),
+        "tpch_q4": oracle.tpch_q4(t["orders"], t["lineitem"]).rows(),
+        "tpch_q13": oracle.tpch_q13(t["tpch_customer"], t["orders"]).rows(),
+        "tpch_q18": oracle.tpch_q18(t["tpch_customer"], t["orders"], t["lineitem"]).rows(
+            ["o_orderkey", "c_custkey", "o_orderdate", "o_totalprice", "sum_qty", "count"])[:100],
+        "tpch_q21": oracle.tpch_q21(t["tpch_supplier"], t["orders"], t["lineitem"], t["nation"]).rows()[:100],
+    }
+    for qn, rows in exp.items():
+        assert root[qn] == rows, qn
+    o3 = oracle.tpch_q3(t["tpch_customer"], t["orders"], t["lineitem"])
+    assert root["tpch_q3"] == o3.rows(["l_orderkey", "o_orderdate", "o_shippriority", "revenue", "count"])[:10]
+    o1 = oracle.tpch_q1(t["lineitem"])
+    assert [r[:6] + (r[9],) for r in root["tpch_q1"]] == o1.rows(
+        ["l_returnflag", "l_linestatus", "sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "count_order"])
