@@ -392,7 +392,9 @@ typedef struct {
   int32_t ncols;
   int32_t types[HQ_MAX_KEYS + HQ_MAX_AGGS]; /* hq_type of each result column */
   int32_t segment_rows;     /* MATERIALISE: fact rows per LRGP segment (the kernel's tile);
-                               output is ordered within a segment's rows, segments permuted */
+                               output is ordered within a segment's rows, segments permuted.
+                               0: warp workgroups (generated kernels behind a global probe) --
+                               each warp's buffered rows are one segment, in row order */
 } hq_result_info;
 hq_status hq_result_info_get(hq_ctx* ctx, hq_result* r, hq_result_info* out); /* syncs */
 /* Copy the result into caller host buffers host_cols[c] (capacity_rows rows

@@ -347,17 +347,28 @@ __device__ __forceinline__ unsigned long long tk_pk(const KCompact& k, const KSo
 // radix-select state: [0] min pk, [1] max pk, [2] shift, [3] selected bin, [4] candidates, [5] overflow
 constexpr int TK_BINS = 4096;
 constexpr int TK_CAND = 16384;
+constexpr int TK_U = 4;  // table entries per thread and round in the full-table passes
 // pass 1: min / max primary key, qualifying rows, live groups
 __global__ void __launch_bounds__(256) hq_topk_minmax_kernel(const __grid_constant__ KTopK q, unsigned long long* sel) {
   const KCompact& k = q.k;
   unsigned long long mn = ~0ull, mx = 0, qs = 0, ls = 0;
-  for (long long g = blockIdx.x * (long long)blockDim.x + threadIdx.x; g < k.ngroups; g += (long long)gridDim.x * blockDim.x) {
-    if (!tk_live(k, g)) continue;
-    const unsigned long long pk = tk_pk(k, q.s, g);
-    mn = pk < mn ? pk : mn;
-    mx = pk > mx ? pk : mx;
-    qs += (unsigned long long)tk_entry(k, g)[0];
-    ++ls;
+  // TK_U entries per thread and round, their loads issued together (one entry at a time
+  // left each thread waiting on two dependent loads per entry: ~1 TB/s over the table)
+  const long long st = (long long)gridDim.x * blockDim.x;
+  for (long long g0 = blockIdx.x * (long long)blockDim.x + threadIdx.x; g0 < k.ngroups; g0 += TK_U * st) {
+    bool live[TK_U];
+#pragma unroll
+    for (int u = 0; u < TK_U; ++u) live[u] = g0 + u * st < k.ngroups && tk_live(k, g0 + u * st);
+#pragma unroll
+    for (int u = 0; u < TK_U; ++u) {
+      if (!live[u]) continue;
+      const long long g = g0 + u * st;
+      const unsigned long long pk = tk_pk(k, q.s, g);
+      mn = pk < mn ? pk : mn;
+      mx = pk > mx ? pk : mx;
+      qs += (unsigned long long)tk_entry(k, g)[0];
+      ++ls;
+    }
   }
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
@@ -403,9 +414,16 @@ __global__ void __launch_bounds__(256) hq_topk_hist_kernel(const __grid_constant
   for (int i = threadIdx.x; i < TK_BINS; i += blockDim.x) h[i] = 0;
   __syncthreads();
   const KCompact& k = q.k;
+  const long long st = (long long)gridDim.x * blockDim.x;
   if (sel[0] <= sel[1])
-    for (long long g = blockIdx.x * (long long)blockDim.x + threadIdx.x; g < k.ngroups; g += (long long)gridDim.x * blockDim.x)
-      if (tk_live(k, g)) atomicAdd(&h[tk_bin(tk_pk(k, q.s, g), sel)], 1u);
+    for (long long g0 = blockIdx.x * (long long)blockDim.x + threadIdx.x; g0 < k.ngroups; g0 += TK_U * st) {
+      bool live[TK_U];
+#pragma unroll
+      for (int u = 0; u < TK_U; ++u) live[u] = g0 + u * st < k.ngroups && tk_live(k, g0 + u * st);
+#pragma unroll
+      for (int u = 0; u < TK_U; ++u)
+        if (live[u]) atomicAdd(&h[tk_bin(tk_pk(k, q.s, g0 + u * st), sel)], 1u);
+    }
   __syncthreads();
   for (int i = threadIdx.x; i < TK_BINS; i += blockDim.x)
     if (h[i]) atomicAdd(hist + i, h[i]);

@@ -400,11 +400,16 @@ struct KPlan {
   // generated kernels: copy the tile's columns into registers and release the
   // stage before the operators run (long-latency probes do not hold the ring)
   uint8_t early_release;
-  // generated A3 with deferred write-out: a tile's rows are staged in shared memory
-  // (two buffers of a3_buf bytes at off_agg, column j at a3_col[j]) and written to
-  // global memory during the next tile, when its atomicAdd has returned
+  // generated A3 variants: 1 = deferred write-out, a tile's rows are staged in shared
+  // memory (two buffers of a3_buf bytes at off_agg, column j at a3_col[j]) and written to
+  // global memory during the next tile, when its atomicAdd has returned (opt-in);
+  // 2 = warp workgroups: each consumer warp collects its rows in its own shared buffer
+  // (a3_rows rows, a3_buf bytes per warp at off_agg + warp * a3_buf, column j at a3_col[j])
+  // and claims global positions for a full buffer with one atomicAdd -- no block barrier
+  // per tile (behind a global probe)
   uint8_t a3stage;
   uint32_t a3_buf;
+  uint32_t a3_rows;
   uint32_t a3_col[HQ_MAX_OUT];
   // multi-pass execution (HQ_EXEC_MULTIPASS, hq_multipass.cu): 1 = count kernel
   // (relational primitives -> one flag per row), 2 = write kernel (rows whose

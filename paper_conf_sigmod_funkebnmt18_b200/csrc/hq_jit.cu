@@ -620,6 +620,25 @@ std::string lcol_tables(const KPlan& kp) {
 std::string a3_flush_fn(const KPlan& kp) {
   if (!kp.a3stage) return "";
   std::ostringstream s;
+  if (kp.a3stage == 2) {
+    // warp-workgroup A3: the warp's n buffered rows get n global positions with one
+    // atomicAdd and are copied out, coalesced per column (positions past the capacity
+    // set F_CAPACITY; the counter still counts them, for the re-run)
+    s << "#define A3WBYTES " << kp.a3_buf << "u\n#define A3WROWS " << kp.a3_rows << "\n"
+      << "__device__ __forceinline__ void a3w_flush(const JParams& p, const char* wb, int n) {\n"
+      << "  unsigned long long g = 0;\n"
+      << "  if ((threadIdx.x & 31) == 0) g = atomicAdd(p.counter, (unsigned long long)n);\n"
+      << "  g = __shfl_sync(0xffffffffu, g, 0);\n"
+      << "  for (int i = threadIdx.x & 31; i < n; i += 32) {\n"
+      << "    const long long pos = (long long)(g + i);\n"
+      << "    if (pos >= p.capacity) { atomicOr(p.err, 1); continue; }\n";
+    for (int j = 0; j < kp.nout; ++j) {
+      const char* ty = kp.out_width[j] == 1 ? "signed char" : (kp.out_width[j] == 4 ? "int" : "long long");
+      s << "    ((" << ty << "*)p.out[" << j << "])[pos] = ((const " << ty << "*)(wb + " << kp.a3_col[j] << "u))[i];\n";
+    }
+    s << "  }\n  __syncwarp();\n}\n";
+    return s.str();
+  }
   s << "#define A3BUF " << kp.a3_buf << "u\n"
     << "__device__ __forceinline__ void a3_flush(const JParams& p, long long base, int n, const char* sb) {\n"
     << "  for (int i = threadIdx.x; i < n; i += NW * 32) {\n"
@@ -1020,7 +1039,9 @@ std::string generate(const KPlan& kp) {
   o << "    }\n    return;\n  }\n";
   // consumer state
   o << "  const int row0 = warp * 32 * R + lane * R;  // the lane's rows: row0 .. row0 + R - 1\n";
-  if (kp.a3stage) o << "  u64 a3pend_ = 0;  // thread 0: the pending atomicAdd of the last tile (staged A3)\n";
+  if (kp.a3stage == 1) o << "  u64 a3pend_ = 0;  // thread 0: the pending atomicAdd of the last tile (staged A3)\n";
+  if (kp.a3stage == 2)
+    o << "  char* wb_ = smem + OFF_AGG + (u32)warp * A3WBYTES; int wcnt_ = 0;  // the warp's row buffer (A3, warp workgroups)\n";
   if (sk == 0 && !c2 && !we) {
     o << "  u64 scount_ = 0;\n";
     for (int a = 0; a < kp.naggs; ++a) o << "  i64 sacc" << a << " = agg_identity(AGG_FN[" << a << "]);\n";
@@ -1265,7 +1286,22 @@ std::string generate(const KPlan& kp) {
   if (g.compacted_R) o << "#undef R\n#define R " << g.compacted_R << "\n";
   o << "    }\n";
   if (we && !mp) gen_we_tile(o, kp, sk);
-  if (sk == 2 && !mp && !we && !c2 && kp.a3stage) {
+  if (sk == 2 && !mp && !we && !c2 && kp.a3stage == 2) {
+    // A3 with warp workgroups (LRGP: local resolution = the warp's ballot
+    // prefix over its buffer, global propagation = one atomicAdd per full buffer): the
+    // warp appends its live rows to its shared buffer and flushes it when the next tile's
+    // rows might not fit -- no block barrier, no atomic round trip per tile.  Output:
+    // each flush's rows contiguous, in row order; flushes permuted.
+    o << "    {\n      const int mine_ = __popc(mask); int lin_ = mine_;\n"
+      << "#pragma unroll\n      for (int o_ = 1; o_ < 32; o_ <<= 1) { const int t_ = __shfl_up_sync(HQ_FULL, lin_, o_); if (lane >= o_) lin_ += t_; }\n"
+      << "      const int wtot_ = __shfl_sync(HQ_FULL, lin_, 31);\n"
+      << "      if (wcnt_ + wtot_ > A3WROWS) { a3w_flush(p, wb_, wcnt_); wcnt_ = 0; }\n"
+      << "      const int wo_ = wcnt_ + lin_ - mine_;\n"
+      << "#pragma unroll\n      for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { const int pos_ = wo_ + __popc(mask & ((1u << r) - 1u));\n";
+    for (int j = 0; j < kp.nout; ++j)
+      o << "        ((" << ctype(kp.out_width[j]) << "*)(wb_ + " << kp.a3_col[j] << "u))[pos_] = (" << ctype(kp.out_width[j]) << ")ov" << j << "[r];\n";
+    o << "      }\n      wcnt_ += wtot_;\n      __syncwarp();\n    }\n";
+  } else if (sk == 2 && !mp && !we && !c2 && kp.a3stage == 1) {
     // A3 (Fig 25 / P:1069-1072) with a deferred write-out: warp ballots -> block scan
     // over the warps -> ONE atomicAdd per block and tile, issued by thread 0 and not
     // waited for: the tile's rows go to a shared staging buffer at their tile-local
@@ -1324,7 +1360,9 @@ std::string generate(const KPlan& kp) {
   else o << "    __syncwarp();\n    if (lane == 0) mbar_arrive_a(sm0_ + 80u + 8u * (u32)s);\n    if (++s == S) { s = 0; ph ^= 1u; }\n  }\n";
   }  // software pipelining
   if (prof) o << "  if (lane == 0) { p.prof[blockIdx.x * 128 + 8 + warp] = pw_; p.prof[blockIdx.x * 128 + 40 + warp] = clock64() - pl0_; } if (pdv_) atomicAdd((unsigned long long*)&p.prof[blockIdx.x * 128 + 72 + warp], (unsigned long long)pdv_);\n";
-  if (kp.a3stage && sk == 2 && !mp && !we && !c2)  // the last tile's staged rows
+  if (kp.a3stage == 2 && sk == 2 && !mp && !we && !c2)  // the rows still in the warp's buffer
+    o << "  if (wcnt_ > 0) a3w_flush(p, wb_, wcnt_);\n";
+  if (kp.a3stage == 1 && sk == 2 && !mp && !we && !c2)  // the last tile's staged rows
     o << "  if (njc > 0) { const int lb_ = (njc - 1) & 1; if (threadIdx.x == 0) s_red[lb_] = (i64)a3pend_; consumer_bar();\n"
       << "    a3_flush(p, s_red[lb_], (int)s_red[2 + lb_], smem + OFF_AGG + lb_ * A3BUF); }\n";
   // ------------------------------------------------------------- sink (end)

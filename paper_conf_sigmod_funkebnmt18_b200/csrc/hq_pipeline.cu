@@ -773,9 +773,11 @@ __global__ void __launch_bounds__(NTHREADS, 1) hq_fused_pipeline_kernel(const __
 // group table initialisation (identities; hash keys EMPTY)
 __global__ void hq_init_groups_kernel(long long* tab, long long n, uint32_t vwords, int hash, uint64_t fns_lo) {
   const uint32_t stride = vwords + (hash ? 1 : 0);
-  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n * stride;
+  const long long total = n * stride;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
        i += (long long)gridDim.x * blockDim.x) {
-    const uint32_t c = (uint32_t)(i % stride);
+    // (a 32-bit remainder where the table allows: the 64-bit one is a long software sequence)
+    const uint32_t c = total <= 0xFFFFFFFFll ? (uint32_t)i % stride : (uint32_t)(i % stride);
     long long v;
     if (hash && c == 0) v = (long long)EMPTY_KEY;
     else {

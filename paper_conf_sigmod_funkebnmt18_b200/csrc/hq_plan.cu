@@ -627,7 +627,21 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   // the per-tile barriers, not the atomic's round trip, bound A3 behind a global probe
   const char* a3e = getenv("HQ_JIT_A3STAGE");
   bool a3try = jit && !mp_pass && P.sink == HQ_SINK_MATERIALISE && P.resolution == HQ_RES_LRGP && a3e && a3e[0] == '1';
+  // warp-workgroup A3 (a3stage 2) behind a global probe: the per-tile block scan would make
+  // every warp wait for the slowest warp's probe and for the tile's atomicAdd round trip
+  bool a3w = false;
+  if (jit && !mp_pass && !we && !a3try && P.sink == HQ_SINK_MATERIALISE && P.resolution == HQ_RES_LRGP &&
+      !getenv("HQ_JIT_NOA3W")) {
+    for (int o = 0; o < kp.nops; ++o) {
+      if (kp.ops[o].kind != OP_PROBE) continue;
+      const KProbe& pr = kp.probes[kp.ops[o].idx];
+      bool st = false;
+      for (int i = 0; i < nstaged; ++i) st = st || staged[i] == kp.ops[o].idx;
+      a3w = a3w || !pr.direct || !st;
+    }
+  }
   kp.a3stage = 0;
+  uint32_t a3w_tiles = 2;
   for (;;) {
     uint32_t tab_total = 0;
     for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
@@ -636,7 +650,11 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       const uint32_t T = (uint32_t)(kp.nw * 32 * R);
       const uint32_t off_tmp = MISC_BYTES;
       const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
-      const uint32_t a3buf = a3try ? align_up(T * outbytes, 128) : 0;
+      // (a3w: one buffer per warp at off_agg of a3w_tiles x 32 R rows, i.e. that many of the
+      // warp's tiles at full selectivity: 2, or 1 when two do not fit beside the ring)
+      uint32_t a3wb = 0;
+      for (int j = 0; a3w && j < kp.nout; ++j) a3wb += align_up(32u * a3w_tiles * (uint32_t)R * kp.out_width[j], 16);
+      const uint32_t a3buf = a3try ? align_up(T * outbytes, 128) : (a3w ? (uint32_t)kp.nw * a3wb / 2 : 0);
       const uint32_t off_tab = align_up(off_agg + agg_smem + 2 * a3buf, 128);
       const uint32_t off_stage = align_up(off_tab + tab_total, 128);
       const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
@@ -654,24 +672,35 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         kp.off_tab = off_tab;
         kp.tab_bytes = tab_total;
         kp.off_stage = off_stage;
-        kp.a3stage = a3try ? 1 : 0;
-        kp.a3_buf = a3buf;
+        kp.a3stage = a3try ? 1 : (a3w ? 2 : 0);
+        kp.a3_buf = a3w ? a3wb : a3buf;
+        kp.a3_rows = a3w ? 32u * a3w_tiles * (uint32_t)R : 0;
         break;
       }
     }
     if (chosen_R) break;
-    if (a3try) {  // no room for the staging buffers: write rows straight to global memory
-      a3try = false;
+    if (a3w && a3w_tiles > 1) {  // a smaller warp buffer
+      --a3w_tiles;
+      continue;
+    }
+    if (a3try || a3w) {  // no room for the buffers: write rows straight to global memory
+      a3try = a3w = false;
       continue;
     }
     if (nstaged == 0) break;
     --nstaged;  // give the last staged table back to the ring
   }
-  if (kp.a3stage) {
+  if (kp.a3stage == 1) {
     uint32_t off = 0;
     for (int j = 0; j < kp.nout; ++j) {
       kp.a3_col[j] = off;
       off += (uint32_t)kp.tile_rows * kp.out_width[j];
+    }
+  } else if (kp.a3stage == 2) {
+    uint32_t off = 0;
+    for (int j = 0; j < kp.nout; ++j) {
+      kp.a3_col[j] = off;
+      off += align_up(kp.a3_rows * kp.out_width[j], 16);
     }
   }
   if (!chosen_R) HQ_THROW(HQ_ERR_UNSUPPORTED, "plan: rows too wide for the shared-memory stage ring");
@@ -690,7 +719,7 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     kp.early_release = slow ? 1 : 0;
     if (const char* e = getenv("HQ_JIT_EARLY")) kp.early_release = e[0] == '1' ? 1 : 0;
   }
-  r->segment_rows = kp.tile_rows;
+  r->segment_rows = kp.a3stage == 2 ? 0 : kp.tile_rows;  // (warp workgroups: no tile segments)
   {
     uint32_t off = kp.off_tab;
     for (int i = 0; i < nstaged; ++i) {
