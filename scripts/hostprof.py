@@ -21,6 +21,7 @@ ap.add_argument("--query", default="ssb_q11")
 ap.add_argument("--sf", type=float, default=1)
 ap.add_argument("--steps", type=int, default=200)
 ap.add_argument("--dist", action="store_true")
+ap.add_argument("--broadcast", action="store_true", help="--dist with the root-broadcast design")
 a = ap.parse_args()
 torch.cuda.set_device(0)
 q = QUERIES[a.query]
@@ -32,7 +33,7 @@ if a.dist:
     os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
     os.environ.setdefault("MASTER_PORT", "29572")
     dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
-    E = DistributedEngine(ctx, tables)
+    E = DistributedEngine(ctx, tables, replicated=not a.broadcast)
 
     def step():
         return run_query(E, q)

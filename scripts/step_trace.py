@@ -31,6 +31,7 @@ def main():
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--json", default="")
     ap.add_argument("--dist", action="store_true")
+    ap.add_argument("--broadcast", action="store_true", help="--dist with the root-broadcast design")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     q = QUERIES[a.query]
@@ -43,7 +44,7 @@ def main():
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         os.environ.setdefault("MASTER_PORT", "29571")
         dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
-        E = DistributedEngine(ctx, tables)
+        E = DistributedEngine(ctx, tables, replicated=not a.broadcast)
 
         def execute():
             return run_query(E, q)

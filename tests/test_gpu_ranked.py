@@ -135,3 +135,32 @@ def test_ranked_edges(ctx):
         want = [int(found.sum()), int(pv[found].astype(np.int64).sum())]
         for ex in EXECS:
             assert _run(ctx, fact, h, "inner", 1, ex) == want, (keys, ex)
+
+
+@pytest.mark.parametrize("hit_rate", [1.0, 0.37, 0.0])
+def test_materialise_behind_a_global_probe(ctx, hit_rate):
+    """A3 with warp workgroups: a materialising pipeline behind a global
+    probe buffers each warp's rows and flushes them with one atomic; every selected row
+    lands exactly once (dense positions), including full selectivity (a flush per tile),
+    none, and the capacity re-run; segment_rows is 0 (no tile segments)."""
+    rng = np.random.default_rng(21)
+    nd, nf = 30_000, 700_001  # a ragged last tile
+    keys = (10 + rng.choice(5_000_000, nd, replace=False)).astype(np.int32)
+    pay = rng.integers(0, 1 << 30, nd).astype(np.int32)
+    hit = rng.random(nf) < hit_rate
+    fk = np.where(hit, keys[rng.integers(0, nd, nf)], -5).astype(np.int32)
+    rowid = np.arange(nf, dtype=np.int32)
+    dim = ctx.load_columns({"k": keys, "p": pay})
+    fact = ctx.load_columns({"fk": fk, "rowid": rowid})
+    h = ctx.build_hash(dim, 0, [1])
+    found, (pv,) = _lookup(keys, [pay], fk)
+    want = sorted(zip(rowid[found].tolist(), pv[found].tolist()))
+    for cap in (0, 1000):  # 1000: undersized -> F_CAPACITY -> one exact re-run
+        pb = PlanBuilder(fact)
+        pb.probe(h, "fk", "inner", ["p"])
+        pb.materialise([("rowid", "i32"), ("p", "i32")], capacity=cap)
+        r = ctx.run(pb.plan, keep=pb.keep + [h])
+        a, b = r.fetch()
+        assert r.qualifying() == len(a) == len(want)
+        assert sorted(zip(a.tolist(), b.tolist())) == want
+        assert r.info().segment_rows == 0
