@@ -88,6 +88,11 @@ __device__ __forceinline__ bool row_passes(const KBuild& b, long long row) {
 // through 2-3 dependent DRAM round trips each).
 constexpr int BUILD_U = 8;
 constexpr int BUILD_BLOCK = 256;
+// the count and compact-build kernels are latency-bound: at 72 registers only 3 blocks
+// fit an SM; capped at 64 (4 blocks, a few spilled bytes) the SSB Q4.1 SF100 customer
+// build takes 31.8 instead of 38 us, TPC-H Q3's customer / orders builds 37 / 41 instead
+// of 45 / 46 us (measured)
+constexpr int BUILD_MINB = 4;
 
 // column c for the thread's U rows: the width dispatch is uniform, the U loads
 // are independent (all in flight)
@@ -145,7 +150,7 @@ struct CountPart {
   int kmin, kmax, pmin, pmax;
   unsigned set[8];  // payload-0 values present, bit (v & 255)
 };
-__global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __grid_constant__ KBuild b) {
+__global__ void __launch_bounds__(BUILD_BLOCK, BUILD_MINB) hq_build_count_kernel(const __grid_constant__ KBuild b) {
   unsigned long long c = 0;
   int kmin = INT_MAX, kmax = INT_MIN, pmin = INT_MAX, pmax = INT_MIN;
   unsigned pset[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};  // registers: constant indices only
@@ -243,7 +248,7 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_count_kernel(const __gri
 struct CLut {
   unsigned char r[256];
 };
-__global__ void __launch_bounds__(BUILD_BLOCK) hq_build_direct_compact_kernel(const __grid_constant__ KBuild b, int kind,
+__global__ void __launch_bounds__(BUILD_BLOCK, BUILD_MINB) hq_build_direct_compact_kernel(const __grid_constant__ KBuild b, int kind,
                                                                              uint32_t* out, long long range, int pay_min,
                                                                              int use_lut, const __grid_constant__ CLut lut) {
   int fault = 0;
