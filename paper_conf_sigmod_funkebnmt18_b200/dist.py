@@ -324,6 +324,8 @@ class DistributedEngine(Engine):
                 return None
             return super().run(pb, partitioned)
         P = pb.plan
+        if partitioned and P.sink == hq.SINK_MATERIALISE:
+            pb.dist_rows = True  # each rank materialises its rows; finish() gathers them to the root
         if partitioned and self._hash_grouped(P):
             # ranks keep all their groups; ORDER BY / LIMIT run after the root's merge
             pb.dist_order = ([(P.order_col[i], P.order_desc[i]) for i in range(P.norder)], P.limit)
@@ -420,6 +422,8 @@ class DistributedEngine(Engine):
         elif getattr(pb, "root_only", False):  # no data collective: the root ran the whole pipeline
             self._root_only_checked(res)
             out = fetch(res, pb.result_names) if self.rank == self.root else None
+        elif getattr(pb, "dist_rows", False):
+            out = self._gather_rows(res, pb)
         elif not hasattr(pb, "dist_order"):
             words = self._reduce_checked(res, defer=True)
             try:
@@ -466,6 +470,54 @@ class DistributedEngine(Engine):
             return merged[0] if merged is not None else None
         self._reduce_checked(res)
         return res if self.rank == self.root else None
+
+    def _gather_rows(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
+        """A partitioned materialising pipeline (SURVEY §8(e) "materialise sinks"): one
+        status all-reduce (row counts, failures, fault words), one all-gather of each
+        rank's rows packed as int64 [ncols, m], the root concatenates them (each rank's
+        rows one segment; the segments in rank order) and casts back to the column types."""
+        names = list(pb.result_names)
+        st = torch.zeros(2 + hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
+        built, self._built = self._built, []
+        self.ctx.gather_faults(built, [], st.data_ptr() + 16)
+        err, tab, nrows = None, None, 0
+        try:
+            tab = res.as_table(names)
+            nrows = tab.nrows
+            st[0] = res.qualifying()
+        except hq.HQError as e:
+            err = e
+            st[1] = 1
+        _all_reduce(st)
+        stl = st.tolist()
+        if err is not None:
+            raise err
+        if stl[1]:
+            raise RootError(hq.HQ_ERR_STATE, "pipeline failed on another rank")
+        self._raise(stl[2:], built)
+        ncol = len(names)
+        n = torch.tensor([nrows], dtype=torch.int64, device=self.device)
+        sizes = [torch.zeros_like(n) for _ in range(self.world)]
+        dist.all_gather(sizes, n)
+        sizes = [int(x.item()) for x in sizes]
+        m = max(max(sizes), 1)
+        pad = torch.zeros((ncol, m), dtype=torch.int64, device=self.device)
+        types = []
+        for c in range(ncol):
+            ptr, t = tab.column_ptr(c)
+            dt = {hq.HQ_I8: torch.int8, hq.HQ_I32: torch.int32, hq.HQ_I64: torch.int64}[t]
+            types.append(dt)
+            if nrows:
+                w = torch.empty((), dtype=dt).element_size()
+                v = device_view(ptr, nrows * w, torch.uint8).view(dt)
+                pad[c, :nrows] = v.to(torch.int64)
+        bufs = [torch.empty_like(pad) for _ in range(self.world)]
+        dist.all_gather(bufs, pad)
+        if self.rank != self.root:
+            return None
+        cols = {nm: torch.cat([b[c, :sz] for b, sz in zip(bufs, sizes)]).to(types[c]).cpu().numpy()
+                for c, nm in enumerate(names)}
+        return QueryResult(cols, int(stl[0]))
 
     def _merge_groups(self, res: hq.Result, pb: PlanBuilder) -> Optional[QueryResult]:
         merged = self._merge_device(res, pb)

@@ -223,3 +223,30 @@ def test_replicated_dimensions_match_oracle():
     o1 = oracle.tpch_q1(t["lineitem"])
     assert [r[:6] + (r[9],) for r in root["tpch_q1"]] == o1.rows(
         ["l_returnflag", "l_linestatus", "sum_qty", "sum_base_price", "sum_disc_price", "sum_charge", "count_order"])
+
+
+@pytest.mark.parametrize("replicated", [False, True])
+def test_two_ranks_materialise_gathers_rows(replicated):
+    """A partitioned materialising pipeline (SSB Q3.1 materialised, SURVEY §8(e)
+    "materialise sinks"): each rank's rows are all-gathered to the root; the root's rows
+    (sorted) and qualifying count equal the oracle's on the whole table."""
+    import hqgen
+    import oracle
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, ["ssb_q31_mat"], 0.01, False, replicated))
+             for r in range(2)]
+    for p in procs:
+        p.start()
+    outs = [q.get(timeout=600) for _ in procs]
+    for p in procs:
+        p.join(timeout=120)
+    errs = [o for o in outs if o[0] != "ok"]
+    if errs:
+        pytest.fail("\n\n".join(f"rank {o[1]}:\n{o[2]}" for o in errs))
+    rows, qual = next(o[2] for o in outs if o[1] == 0)["ssb_q31_mat"]
+    ssb = {t: hqgen.generate(t, 0.01) for t in hqgen.SSB_TABLES}
+    o = oracle.ssb_q31_mat(ssb["lineorder"], ssb["customer"], ssb["supplier"], ssb["date"])
+    assert sorted(rows) == o.rows()
+    assert qual == o.nrows
