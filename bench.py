@@ -281,7 +281,8 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
     # prepared query (CUDA graph of the whole step: builds + fused pipeline + finalize
     # re-executed every launch; include/hq.h "prepared queries") where the plan is static
     prep = None
-    if world == 1 and os.environ.get("HQ_BENCH_EAGER") != "1" and os.environ.get("HQ_FORCE_DIST") != "1":
+    # (distributed: the two-graph prepared step of dist.PreparedDistQuery, replicated dimensions)
+    if os.environ.get("HQ_BENCH_EAGER") != "1" and ((not dist_mode) or replicated):
         try:
             pq = E.prepare(q)
             for _ in range(warmup):
@@ -289,7 +290,7 @@ def measure(qname, sf, steps, warmup, seed, rank, world, local, with_e2e=True, h
             l1 = ctx.launches()
             with ClockSampler(local) as clk2:
                 ms_prep, per_prep, out_p = timed(pq.execute, steps)
-            if out_p.rows() != out.rows():
+            if (out_p is None) != (out is None) or (out_p is not None and out_p.rows() != out.rows()):
                 raise RuntimeError("prepared result differs from the eager one")
             prep = {"ms": ms_prep, "per": per_prep, "launches": ctx.launches() - l1, "clocks": clk2.summary()}
             pq.close()
@@ -454,7 +455,9 @@ def run_hq(args):
                                            "rank, 1 reduce" if r["replicated"] else
                                            f"fact range partition dp{world}, dimension HTs broadcast, 1 reduce"),
                            "step": "hash builds + fused pipeline + reduce + finalize/fetch",
-                           "step_mode": r["mode"] + (" (CUDA graph of the whole step; every kernel re-executed per step)"
+                           "step_mode": r["mode"] + ((" (two CUDA graphs around the partials all-reduce; every kernel "
+                                                      "re-executed per step)" if (world > 1 or os.environ.get("HQ_FORCE_DIST") == "1")
+                                                      else " (CUDA graph of the whole step; every kernel re-executed per step)")
                                                      if r["mode"] == "prepared" else "")},
                 "step_ms_median": r["step_ms_median"], "step_ms_min": r["step_ms_min"], "eager": r["eager"],
                 "roofline": roofline(q, r["local_rows"], r["kernel_ms"], peak, peak_src),

@@ -465,7 +465,9 @@ hq_status hq_free_result(hq_result* r);
  * multi-pass / operator-at-a-time execution, batch processing, hq_load_columns.
  * The graph keeps the objects its nodes use (results, hashes, build source tables)
  * until hq_graph_destroy.  The capture runs on a private stream; launches run on the
- * context stream and synchronise it (the rows are decoded on the host).  Needs the
+ * context stream and synchronise it (the rows are decoded on the host) -- a graph that
+ * finalizes no result (e.g. the part of a distributed step before its collective) is
+ * launched asynchronously.  Needs the
  * default stream-ordered allocator (no hq_allocator hooks: HQ_ERR_UNSUPPORTED). */
 hq_status hq_ctx_capture_begin(hq_ctx* ctx);
 hq_status hq_ctx_capture_end(hq_ctx* ctx, hq_graph** out);

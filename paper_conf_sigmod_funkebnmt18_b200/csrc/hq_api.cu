@@ -285,6 +285,7 @@ hq_status hq_graph_launch(hq_ctx* ctx, hq_graph* g) {
     }
     ctx->launches += g->nkernels;
     HQ_CUDA(cudaGraphLaunch(g->exec, ctx->stream));
+    if (g->results.empty()) return;  // nothing to decode: the launch stays asynchronous
     HQ_CUDA(cudaStreamSynchronize(ctx->stream));
     for (hq_result* r : g->results) hq_decode_captured(ctx, r);
   });

@@ -332,6 +332,14 @@ class DistributedEngine(Engine):
             P.norder, P.limit = 0, 0
         return super().run(pb, partitioned)
 
+    def prepare(self, query, **kw) -> "PreparedDistQuery":
+        """A prepared distributed step (replicated dimensions, a dense final aggregation):
+        two CUDA graphs around the collective -- the builds, the pipeline and the packing
+        of [partials | fault words] into a persistent buffer; the all-reduce on the device
+        between them; the partials' copy-back and the finalize.  Raises HQError(HQ_ERR_STATE)
+        or NotImplementedError for steps it cannot hold (the caller runs them eagerly)."""
+        return PreparedDistQuery(self, query, **kw)
+
     def _faults_of(self, h: hq.Hash) -> List[int]:
         st = torch.zeros(hq.FAULT_WORDS, dtype=torch.int64, device=self.device)
         self.ctx.gather_faults([h], [], st.data_ptr())
@@ -599,3 +607,62 @@ class DistributedEngine(Engine):
                      group_capacity=max(1024, sum(sizes)), agg_names=names[P.nkeys:])
         mb.root_only = True
         return self.ctx.run(mb.plan, keep=mb.keep + [merged]), mb, qual
+
+
+class PreparedDistQuery:
+    """DistributedEngine.prepare: graph A (builds + fused pipeline + partials and fault
+    words packed into a persistent device buffer), the all-reduce of that buffer over the
+    process group, graph B (partials copied back, finalize).  Graph A launches
+    asynchronously, so the collective's host call overlaps the pipeline.  Every launch
+    re-executes all device work; the fault words are read after B's synchronisation and
+    raised on every rank together."""
+
+    def __init__(self, E: DistributedEngine, query, **kw):
+        if not E.replicated or E.copartitioned:
+            raise NotImplementedError("prepared distributed steps need replicated dimensions")
+        self.E, self.query = E, query
+        run_query(E, query)  # eager: kernels compiled, build statistics and result views cached
+        ctx = E.ctx
+        E._built = []
+        ctx.capture_begin()
+        try:
+            res, pb = query.run(E, **kw)
+            if res is None or getattr(pb, "dist_rows", False) or hasattr(pb, "dist_order") or \
+                    getattr(pb, "root_only", False) or getattr(pb, "replicated_local", False):
+                raise NotImplementedError("prepared distributed steps: a dense final aggregation only")
+            ptr, nbytes = res.partials_view()
+            self.n = nbytes // 8
+            self.red = torch.zeros(self.n + hq.FAULT_WORDS, dtype=torch.int64, device=E.device)
+            res.to_partials(self.red.data_ptr(), nbytes)
+            built, E._built = E._built, []
+            ctx.gather_faults(built, [res], self.red.data_ptr() + self.n * 8)
+        except BaseException:
+            ctx.capture_abort()
+            E._built = []
+            raise
+        self.graph_a = ctx.capture_end()
+        self.built = built
+        ctx.capture_begin()
+        try:
+            res.from_partials(self.red.data_ptr(), nbytes)
+            res.finalize()
+        except BaseException:
+            ctx.capture_abort()
+            self.graph_a.free()
+            raise
+        self.graph_b = ctx.capture_end()
+        self.res, self.pb = res, pb
+        self.words = torch.empty(hq.FAULT_WORDS, dtype=torch.int64, pin_memory=True)
+
+    def execute(self) -> Optional[QueryResult]:
+        E = self.E
+        self.graph_a.launch()  # asynchronous
+        _all_reduce(self.red)  # the device-side collective, ordered after graph A
+        self.words.copy_(self.red[self.n:], non_blocking=True)
+        self.graph_b.launch()  # synchronises (the finalized rows are decoded on the host)
+        E._raise(self.words.tolist(), self.built)
+        return fetch(self.res, self.pb.result_names) if E.rank == E.root else None
+
+    def close(self) -> None:
+        self.graph_a.free()
+        self.graph_b.free()

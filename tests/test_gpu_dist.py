@@ -250,3 +250,66 @@ def test_two_ranks_materialise_gathers_rows(replicated):
     o = oracle.ssb_q31_mat(ssb["lineorder"], ssb["customer"], ssb["supplier"], ssb["date"])
     assert sorted(rows) == o.rows()
     assert qual == o.nrows
+
+
+def _prepared_worker(rank, world, port, q, qs, sf):
+    try:
+        import torch
+        import torch.distributed as dist
+
+        import hqgen
+        from paper_conf_sigmod_funkebnmt18_b200 import hq
+        from paper_conf_sigmod_funkebnmt18_b200.dist import DistributedEngine, partition
+        from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES, load_tables
+
+        os.environ["MASTER_ADDR"] = "127.0.0.1"
+        os.environ["MASTER_PORT"] = str(port)
+        torch.cuda.set_device(0)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        ctx = hq.Context(0)
+        out = {}
+        for qn in qs:
+            qq = QUERIES[qn]
+            rng = partition(hqgen.table_rows(qq.fact, sf), rank, world)
+            E = DistributedEngine(ctx, load_tables(ctx, qq, sf, fact_range=rng), replicated=True)
+            pq = E.prepare(qq)
+            runs = [pq.execute() for _ in range(3)]
+            pq.close()
+            out[qn] = [r.rows() if r is not None else None for r in runs]
+        q.put(("ok", rank, out))
+        dist.barrier()
+        dist.destroy_process_group()
+    except Exception:  # pragma: no cover
+        import traceback
+        q.put(("err", rank, traceback.format_exc()))
+
+
+def test_prepared_distributed_step_matches_oracle():
+    """dist.PreparedDistQuery: graph A (builds, pipeline, [partials | faults] packed),
+    the all-reduce between the graphs, graph B (copy-back, finalize) -- three launches per
+    query over two ranks, every launch's root rows equal the oracle."""
+    import hqgen
+    import oracle
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    qs = ["ssb_q41", "ssb_q31", "tpch_q6"]
+    procs = [ctx.Process(target=_prepared_worker, args=(r, 2, port, q, qs, 0.01)) for r in range(2)]
+    for p in procs:
+        p.start()
+    outs = [q.get(timeout=600) for _ in procs]
+    for p in procs:
+        p.join(timeout=120)
+    errs = [o for o in outs if o[0] != "ok"]
+    if errs:
+        pytest.fail("\n\n".join(f"rank {o[1]}:\n{o[2]}" for o in errs))
+    root = next(o[2] for o in outs if o[1] == 0)
+    assert all(r is None for o in outs if o[1] != 0 for qn in qs for r in o[2][qn])
+    ssb = {t: hqgen.generate(t, 0.01) for t in hqgen.SSB_TABLES}
+    li = hqgen.generate("lineitem", 0.01)
+    exp = {"ssb_q41": oracle.ssb_q41(ssb["lineorder"], ssb["date"], ssb["customer"], ssb["supplier"], ssb["part"]).rows(),
+           "ssb_q31": oracle.ssb_q31(ssb["lineorder"], ssb["customer"], ssb["supplier"], ssb["date"]).rows(),
+           "tpch_q6": oracle.tpch_q6(li).rows()}
+    for qn in qs:
+        for rows in root[qn]:
+            assert rows == exp[qn], qn
