@@ -642,6 +642,31 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   }
   kp.a3stage = 0;
   uint32_t a3w_tiles = 2;
+  // The unified L1 / shared-memory array is 256 KB per SM and the driver carves the
+  // shared part out of it in steps (.., 164, 196, 228 KB) by the kernel's request: a
+  // ring that fills 228 KB leaves 28 KB of L1 for the probes that read global memory
+  // (byte maps / bitmaps in L2), one that stays within 196 KB leaves 60 KB.  Generated
+  // kernels with such probes therefore trade consumer warps for L1 (measured on B200,
+  // SSB Q4.1 SF100: 31 warps / 228 KB 2.465 ms, 29 warps / 196 KB 2.19 ms -- the 175-KB
+  // part bitmap's hits; SF30 already fit 196 KB).  HQ_JIT_CARVE=<KB> overrides (A/B).
+  bool l1_probe = false;
+  for (int o = 0; jit && o < kp.nops; ++o) {
+    if (kp.ops[o].kind != OP_PROBE) continue;
+    bool st = false;
+    for (int i = 0; i < nstaged; ++i) st = st || staged[i] == kp.ops[o].idx;
+    l1_probe = l1_probe || !st;
+  }
+  uint64_t carve_kb = l1_probe && !getenv("HQ_JIT_NW") ? 196 : 0;
+  if (const char* e = getenv("HQ_JIT_CARVE")) carve_kb = jit ? (uint64_t)atoi(e) : 0;
+  const int nstaged0 = nstaged, nw0 = kp.nw;
+  const bool a3try0 = a3try, a3w0 = a3w;
+  const uint64_t carve_cap = carve_kb ? std::min<uint64_t>(ctx->max_smem, carve_kb * 1024 - 1024) : ctx->max_smem;
+  // search: the most consumer warps (>= 16) whose ring keeps >= 3 stages and every staged
+  // table within the carve-out; else the full shared memory with the default warps
+  bool carve_ok = false;
+  for (int nw = nw0; carve_cap < ctx->max_smem && !carve_ok && nw >= 16; --nw) {
+    nstaged = nstaged0; a3try = a3try0; a3w = a3w0; a3w_tiles = 2; kp.nw = nw;
+    const uint64_t smem_cap = carve_cap;
   for (;;) {
     uint32_t tab_total = 0;
     for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
@@ -658,8 +683,9 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
       const uint32_t off_tab = align_up(off_agg + agg_smem + 2 * a3buf, 128);
       const uint32_t off_stage = align_up(off_tab + tab_total, 128);
       const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
-      if (off_stage >= ctx->max_smem) continue;
-      const int S = (int)std::min<int64_t>(MAX_STAGES, (ctx->max_smem - off_stage) / stride);
+      if (off_stage >= smem_cap) continue;
+      int S = (int)std::min<int64_t>(MAX_STAGES, (smem_cap - off_stage) / stride);
+      if (const char* e = jit ? getenv("HQ_JIT_MAXS") : nullptr) S = std::min(S, std::max(2, atoi(e)));  // A/B
       if (S >= 3 || (R <= 2 && S >= 2 && nstaged == 0)) {
         chosen_R = R;
         kp.R = R;
@@ -689,6 +715,62 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     }
     if (nstaged == 0) break;
     --nstaged;  // give the last staged table back to the ring
+  }
+    carve_ok = chosen_R != 0 && nstaged == nstaged0 && kp.nstages >= 3 && a3w == a3w0 && a3try == a3try0;
+    if (!carve_ok) chosen_R = 0;
+  }
+  if (!carve_ok) {
+    nstaged = nstaged0; a3try = a3try0; a3w = a3w0; a3w_tiles = 2; kp.nw = nw0;
+    const uint64_t smem_cap = ctx->max_smem;
+  for (;;) {
+    uint32_t tab_total = 0;
+    for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
+    for (int R : {8, 4, 3, 2, 1}) {  // (3: only when forced, HQ_JIT_R=3 experiments)
+      if (prefer4 ? (R != 4 && R != 2) : (force_R ? R != force_R : (R == 8 || R == 1 || R == 3))) continue;
+      const uint32_t T = (uint32_t)(kp.nw * 32 * R);
+      const uint32_t off_tmp = MISC_BYTES;
+      const uint32_t off_agg = align_up(off_tmp + T * tmp_row, 128);
+      // (a3w: one buffer per warp at off_agg of a3w_tiles x 32 R rows, i.e. that many of the
+      // warp's tiles at full selectivity: 2, or 1 when two do not fit beside the ring)
+      uint32_t a3wb = 0;
+      for (int j = 0; a3w && j < kp.nout; ++j) a3wb += align_up(32u * a3w_tiles * (uint32_t)R * kp.out_width[j], 16);
+      const uint32_t a3buf = a3try ? align_up(T * outbytes, 128) : (a3w ? (uint32_t)kp.nw * a3wb / 2 : 0);
+      const uint32_t off_tab = align_up(off_agg + agg_smem + 2 * a3buf, 128);
+      const uint32_t off_stage = align_up(off_tab + tab_total, 128);
+      const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
+      if (off_stage >= smem_cap) continue;
+      int S = (int)std::min<int64_t>(MAX_STAGES, (smem_cap - off_stage) / stride);
+      if (const char* e = jit ? getenv("HQ_JIT_MAXS") : nullptr) S = std::min(S, std::max(2, atoi(e)));  // A/B
+      if (S >= 3 || (R <= 2 && S >= 2 && nstaged == 0)) {
+        chosen_R = R;
+        kp.R = R;
+        kp.tile_rows = (int32_t)T;
+        kp.nstages = S;
+        kp.stage_bytes = T * rowbytes;
+        kp.stage_stride = stride;
+        kp.off_tmp = off_tmp;
+        kp.off_agg = off_agg;
+        kp.off_tab = off_tab;
+        kp.tab_bytes = tab_total;
+        kp.off_stage = off_stage;
+        kp.a3stage = a3try ? 1 : (a3w ? 2 : 0);
+        kp.a3_buf = a3w ? a3wb : a3buf;
+        kp.a3_rows = a3w ? 32u * a3w_tiles * (uint32_t)R : 0;
+        break;
+      }
+    }
+    if (chosen_R) break;
+    if (a3w && a3w_tiles > 1) {  // a smaller warp buffer
+      --a3w_tiles;
+      continue;
+    }
+    if (a3try || a3w) {  // no room for the buffers: write rows straight to global memory
+      a3try = a3w = false;
+      continue;
+    }
+    if (nstaged == 0) break;
+    --nstaged;  // give the last staged table back to the ring
+  }
   }
   if (kp.a3stage == 1) {
     uint32_t off = 0;
