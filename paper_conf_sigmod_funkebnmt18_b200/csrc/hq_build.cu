@@ -257,6 +257,10 @@ __global__ void __launch_bounds__(BUILD_BLOCK, BUILD_MINB) hq_build_direct_compa
   bool pass[BUILD_U];
   long long kv[BUILD_U], pv[BUILD_U] = {};
   load_rows(b, base, pass, kv, pv);
+  int aw[BUILD_U];  // target word of the row's atomic (< 2^30: range <= 2^32 keys), -1: none
+  uint32_t am[BUILD_U], ash = 0;  // ash: the slot's shift / 4, 3 bits per row
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u) { aw[u] = -1; am[u] = 0; }
 #pragma unroll
   for (int u = 0; u < BUILD_U; ++u) {
     if (!pass[u]) continue;
@@ -281,19 +285,37 @@ __global__ void __launch_bounds__(BUILD_BLOCK, BUILD_MINB) hq_build_direct_compa
       fault |= HQF_HT_FULL;
       continue;
     }
+    // word index and bits of the row; the atomics are issued in a separate loop
     if (kind == 1) {
-      const uint32_t bit = 1u << (d & 31);
-      if (atomicOr(out + (d >> 5), bit) & bit) fault |= HQF_DUP_KEY;
+      aw[u] = (int)(d >> 5);
+      am[u] = 1u << (d & 31);
     } else if (kind == 2) {
       uint32_t v = (uint32_t)(pc - pay_min) & 0xFFu;
       if (use_lut) v = lut.r[v];
       const uint32_t sh = (uint32_t)(d & 3) * 8u;
-      if (((atomicAnd(out + (d >> 2), ~((0xFFu ^ v) << sh)) >> sh) & 0xFFu) != 0xFFu) fault |= HQF_DUP_KEY;
+      aw[u] = (int)(d >> 2);
+      am[u] = ~((0xFFu ^ v) << sh);
+      ash |= (sh >> 2) << (3 * u);
     } else {
       const uint32_t v = (uint32_t)(pc - pay_min) & 0xFu;
       const uint32_t sh = (uint32_t)(d & 7) * 4u;
-      if (((atomicAnd(out + (d >> 3), ~((0xFu ^ v) << sh)) >> sh) & 0xFu) != 0xFu) fault |= HQF_DUP_KEY;
+      aw[u] = (int)(d >> 3);
+      am[u] = ~((0xFu ^ v) << sh);
+      ash |= (sh >> 2) << (3 * u);
     }
+  }
+  // all of the thread's atomics in flight at once: a duplicate-key test right after each
+  // one made every atomic a dependent L2 round trip (the test branches on its result)
+  uint32_t old[BUILD_U];
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u)
+    if (aw[u] >= 0) old[u] = kind == 1 ? atomicOr(out + aw[u], am[u]) : atomicAnd(out + aw[u], am[u]);
+#pragma unroll
+  for (int u = 0; u < BUILD_U; ++u) {
+    if (aw[u] < 0) continue;
+    const uint32_t sh = ((ash >> (3 * u)) & 7u) * 4u, full = kind == 2 ? 0xFFu : 0xFu;
+    const uint32_t f = kind == 1 ? (old[u] & am[u]) : ((old[u] >> sh) & full) ^ full;
+    if (f) fault |= HQF_DUP_KEY;
   }
   if (fault) atomicOr(b.err, fault);
   if (b.verify) {

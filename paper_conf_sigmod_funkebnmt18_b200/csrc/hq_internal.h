@@ -439,6 +439,12 @@ struct KPlan {
   // status
   unsigned long long* counter;  // qualifying rows / write counter
   int* err;
+  // generated kernels, global hash group table without a shared table: each consumer warp
+  // queues its live rows' group updates in shared memory (gq_cap entries at
+  // off_agg + warp * gq_cap * (2 + naggs) * 8, column-major: keys, counts, values) and
+  // applies a full queue with one update per lane -- the hash round trips of up to
+  // gq_cap rows overlap instead of stalling every tile that has a live row (0 = off)
+  uint16_t gq_cap;
 };
 }  // namespace hqk
 

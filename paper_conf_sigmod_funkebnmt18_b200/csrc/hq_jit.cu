@@ -772,6 +772,9 @@ std::string generate(const KPlan& kp) {
   // (Blelloch) tree in shared memory with one consumer barrier per level produces one
   // pre-aggregate / write offset per workgroup (the CTA) for global propagation
   const bool we = kp.resolution == HQ_RES_WE;
+  // warp update queues (kp.gq_cap) in front of a global hash group table
+  const bool gq = kp.gq_cap > 0 && !c2 && !we && !kp.mp_pass && kp.sink == HQ_SINK_AGG && kp.nkeys > 0 &&
+                  kp.smode == SM_NONE && kp.gmode == GM_HASH && kp.R <= 2 && !getenv("HQ_JIT_COMPACT");
   const int sk = kp.sink == HQ_SINK_MATERIALISE ? 2 : (kp.nkeys == 0 ? 0 : 1);
   const int mp = kp.mp_pass;  // multi-pass: 1 = count kernel, 2 = write kernel (hq_multipass.cu)
   // the sink's per-tile code (aggregation into registers / shared tables, or the
@@ -888,6 +891,30 @@ std::string generate(const KPlan& kp) {
       o << "      i64 va_[NAGGS > 0 ? NAGGS : 1][R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) {";
       for (int a = 0; a < kp.naggs; ++a) o << " va_[" << a << "][r] = " << vv[a] << ";";
       o << " }\n";
+      if (gq) {
+        // warp update queue (kp.gq_cap): a lane's consecutive rows of one group are folded
+        // (the lines of an order), the live rows are appended at the warp's ballot prefix;
+        // a queue that cannot take them is applied first, one update per lane (gq_flush),
+        // and a tile with more live rows than the queue holds updates directly
+        o << "      u64 cn_[R];\n#pragma unroll\n      for (int r = 0; r < R; ++r) cn_[r] = 1ull;\n"
+          << "#pragma unroll\n      for (int r = 1; r < R; ++r) if (((mask >> r) & 1u) && ((mask >> (r - 1)) & 1u) && gk_[r] == gk_[r - 1]) {\n"
+          << "#pragma unroll\n        for (int a = 0; a < NAGGS; ++a) va_[a][r] = agg_combine(AGG_FN[a], va_[a][r], va_[a][r - 1]);\n"
+          << "        cn_[r] += cn_[r - 1]; mask &= ~(1u << (r - 1)); }\n"
+          << "      { const int mine_ = __popc(mask); int lin_ = mine_;\n"
+          << "#pragma unroll\n        for (int o_ = 1; o_ < 32; o_ <<= 1) { const int t_ = __shfl_up_sync(HQ_FULL, lin_, o_); if (lane >= o_) lin_ += t_; }\n"
+          << "        const int wtot_ = __shfl_sync(HQ_FULL, lin_, 31);\n"
+          << "        if (gqn_ + wtot_ > GQ_CAP) { gq_flush(p, sagg, sl0_, gq_, gqn_); gqn_ = 0; }\n"
+          << "        if (wtot_ > GQ_CAP) {\n"
+          << "#pragma unroll\n          for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { i64 v_[NAGGS > 0 ? NAGGS : 1];\n"
+          << "#pragma unroll\n            for (int a = 0; a < NAGGS; ++a) v_[a] = va_[a][r];\n"
+          << "            group_update(p, sagg, sl0_, gk_[r], false, cn_[r], v_); }\n"
+          << "        } else {\n"
+          << "          int pos_ = gqn_ + lin_ - mine_;\n"
+          << "#pragma unroll\n          for (int r = 0; r < R; ++r) if ((mask >> r) & 1u) { gq_[pos_] = gk_[r]; gq_[GQ_CAP + pos_] = cn_[r];\n"
+          << "#pragma unroll\n            for (int a = 0; a < NAGGS; ++a) gq_[(2 + a) * GQ_CAP + pos_] = (u64)va_[a][r];\n"
+          << "            ++pos_; }\n"
+          << "          gqn_ += wtot_;\n        }\n      }\n";
+      } else {
       const char* ce = getenv("HQ_JIT_COMPACT");  // A/B: compaction of R >= 4 row slots
       const bool wcompact = ce ? ce[0] == '1' : kp.R >= 4;
       if (wcompact) {
@@ -977,6 +1004,7 @@ std::string generate(const KPlan& kp) {
         }
         if (!wcompact) o << "      }\n";  // else of the sparse path
       }
+      }  // !gq
     }
   } else {  // materialise: hand the output values to the block scan below
     std::vector<std::string> ov;
@@ -1042,6 +1070,8 @@ std::string generate(const KPlan& kp) {
   if (kp.a3stage == 1) o << "  u64 a3pend_ = 0;  // thread 0: the pending atomicAdd of the last tile (staged A3)\n";
   if (kp.a3stage == 2)
     o << "  char* wb_ = smem + OFF_AGG + (u32)warp * A3WBYTES; int wcnt_ = 0;  // the warp's row buffer (A3, warp workgroups)\n";
+  if (gq)
+    o << "  u64* gq_ = (u64*)(smem + OFF_AGG + (u32)warp * (GQ_CAP * (2u + NAGGS) * 8u)); int gqn_ = 0;  // the warp's update queue\n";
   if (sk == 0 && !c2 && !we) {
     o << "  u64 scount_ = 0;\n";
     for (int a = 0; a < kp.naggs; ++a) o << "  i64 sacc" << a << " = agg_identity(AGG_FN[" << a << "]);\n";
@@ -1362,6 +1392,7 @@ std::string generate(const KPlan& kp) {
   if (prof) o << "  if (lane == 0) { p.prof[blockIdx.x * 128 + 8 + warp] = pw_; p.prof[blockIdx.x * 128 + 40 + warp] = clock64() - pl0_; } if (pdv_) atomicAdd((unsigned long long*)&p.prof[blockIdx.x * 128 + 72 + warp], (unsigned long long)pdv_);\n";
   if (kp.a3stage == 2 && sk == 2 && !mp && !we && !c2)  // the rows still in the warp's buffer
     o << "  if (wcnt_ > 0) a3w_flush(p, wb_, wcnt_);\n";
+  if (gq) o << "  if (gqn_ > 0) gq_flush(p, sagg, sl0_, gq_, gqn_);  // the updates still queued\n";
   if (kp.a3stage == 1 && sk == 2 && !mp && !we && !c2)  // the last tile's staged rows
     o << "  if (njc > 0) { const int lb_ = (njc - 1) & 1; if (threadIdx.x == 0) s_red[lb_] = (i64)a3pend_; consumer_bar();\n"
       << "    a3_flush(p, s_red[lb_], (int)s_red[2 + lb_], smem + OFF_AGG + lb_ * A3BUF); }\n";
@@ -1441,7 +1472,15 @@ std::string generate(const KPlan& kp) {
     << "static constexpr __device__ int ACC_FN[" << (kp.nacc > 0 ? kp.nacc : 1) << "] = " << fn_list(kp.acc_fn, kp.nacc) << ";\n"
     << "#define LVWORDS " << kp.lvwords << "\n" << lcol_tables(kp)
     << HQ_STR(HQ_JPARAMS_DEF) << "\n"
+    << "#define GQ_CAP " << (gq ? (int)kp.gq_cap : 0) << "u\n"
     << kPrelude << "\n" << a3_flush_fn(kp)
+    << (gq ? "// a warp's queued group updates, one per lane (all lanes of the warp call it)\n"
+             "__device__ __noinline__ void gq_flush(const JParams& p, char* sagg, u32 sl0, u64* q, int n) {\n"
+             "  __syncwarp();\n"
+             "  for (int i = (int)(threadIdx.x & 31); i < n; i += 32) { i64 v_[NAGGS > 0 ? NAGGS : 1];\n"
+             "#pragma unroll\n    for (int a = 0; a < NAGGS; ++a) v_[a] = (i64)q[(2 + a) * GQ_CAP + i];\n"
+             "    group_update(p, sagg, sl0, q[i], false, q[GQ_CAP + i], v_); }\n"
+             "  __syncwarp();\n}\n" : "")
     << g.bitmaps.str() << "\n";
   return h.str() + o.str();
 }

@@ -382,6 +382,13 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
         const char* nl = getenv("HQ_JIT_NOLOCAL");
         if (jit && expect > (kp.gmode == GM_DENSE ? 1 : 4) * (int64_t)cap && !(nl && nl[0] == '0')) {
           kp.smode = SM_NONE;
+          // per-warp update queues in front of the global hash table (hq_jit.cu): 16 rows
+          // per warp, for the 31 warps of the widest layout
+          if (kp.gmode == GM_HASH && !mp_pass && P.resolution == HQ_RES_LRGP && !getenv("HQ_JIT_NOGQ")) {
+            kp.gq_cap = 16;
+            if (const char* e = getenv("HQ_JIT_GQ")) kp.gq_cap = (uint16_t)std::max(1, std::min(64, atoi(e)));  // A/B
+            agg_smem = 31u * kp.gq_cap * (2u + (uint32_t)P.naggs) * 8u;
+          }
         } else {
         kp.smode = SM_HASH;
         kp.smem_cap = cap;
@@ -661,6 +668,27 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
   const int nstaged0 = nstaged, nw0 = kp.nw;
   const bool a3try0 = a3try, a3w0 = a3w;
   const uint64_t carve_cap = carve_kb ? std::min<uint64_t>(ctx->max_smem, carve_kb * 1024 - 1024) : ctx->max_smem;
+  // warp update queues: the longest (16 .. 4 rows per warp) that keeps the ring's depth
+  // (up to 4 stages) -- a stage less cost more than the queue saved (TPC-H Q3 SF30 lineitem:
+  // no queue 0.752 ms, 6 rows at 4 stages 0.721 ms, 16 rows at 3 stages 0.777 ms; TPC-H Q10
+  // SF10 0.397 / 0.281 / 0.255 ms, measured)
+  if (kp.gq_cap && !getenv("HQ_JIT_GQ")) {
+    uint32_t tab_total = 0;
+    for (int i = 0; i < nstaged; ++i) tab_total += align_up(kp.probes[staged[i]].cbytes, 128);
+    const uint32_t T = (uint32_t)kp.nw * 32u * 2u;
+    const uint32_t stride = std::max<uint32_t>(128, align_up(T * rowbytes, 128));
+    const uint32_t off_agg = align_up(MISC_BYTES + T * tmp_row, 128);
+    const uint32_t per = 31u * (2u + (uint32_t)kp.naggs) * 8u;
+    auto stages = [&](uint32_t q) -> int64_t {
+      const uint32_t off_stage = align_up(align_up(off_agg + q * per, 128) + tab_total, 128);
+      return off_stage >= carve_cap ? 0 : std::min<int64_t>(MAX_STAGES, (int64_t)(carve_cap - off_stage) / stride);
+    };
+    const int64_t want = std::min<int64_t>(stages(0), 4);
+    uint32_t q = 16;
+    while (q >= 4 && stages(q) < want) --q;
+    kp.gq_cap = (uint16_t)(q >= 4 ? q : 0);
+    agg_smem = kp.gq_cap * per;
+  }
   // search: the most consumer warps (>= 16) whose ring keeps >= 3 stages and every staged
   // table within the carve-out; else the full shared memory with the default warps
   bool carve_ok = false;

@@ -667,3 +667,22 @@ def test_bench_configs_full_size(ctx, qname, sf):
     assert_same(qname, g, o)
     assert g.qualifying == o.qualifying
     del E
+
+
+@pytest.mark.parametrize("gq", ["1", "2", "4", "16", "off"])
+@pytest.mark.parametrize("qname", ["tpch_q3", "tpch_q10", "tpch_q4"])
+def test_warp_update_queue_lengths(ctx, tpch1, qname, gq, monkeypatch):
+    """Warp update queues in front of the global hash group table (hq_jit.cu gq_flush): every
+    queue length -- 1 and 2 rows per warp send most tiles' live rows past the queue (direct
+    updates), 16 fills it over many tiles -- and none (HQ_JIT_NOGQ) give the oracle's rows
+    at SF 1 (multi-tile, ragged tail)."""
+    if gq == "off":
+        monkeypatch.setenv("HQ_JIT_NOGQ", "1")
+    else:
+        monkeypatch.setenv("HQ_JIT_GQ", gq)
+    o = oracle_run(qname, tpch1)
+    assert o.nrows > 0
+    kw = {"limit": 0} if qname in ("tpch_q3", "tpch_q10") else {}
+    g = gpu_run(ctx, qname, tpch1, **kw)  # the full pre-LIMIT set under the total order
+    assert_same(qname, g, o)
+    assert g.qualifying == o.qualifying
