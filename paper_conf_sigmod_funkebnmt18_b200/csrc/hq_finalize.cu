@@ -349,7 +349,8 @@ constexpr int TK_BINS = 4096;
 constexpr int TK_CAND = 16384;
 constexpr int TK_U = 4;  // table entries per thread and round in the full-table passes
 // pass 1: min / max primary key, qualifying rows, live groups
-__global__ void __launch_bounds__(256) hq_topk_minmax_kernel(const __grid_constant__ KTopK q, unsigned long long* sel) {
+__global__ void __launch_bounds__(256) hq_topk_minmax_kernel(const __grid_constant__ KTopK q, unsigned long long* sel,
+                                                             unsigned long long* bmin) {
   const KCompact& k = q.k;
   unsigned long long mn = ~0ull, mx = 0, qs = 0, ls = 0;
   // TK_U entries per thread and round, their loads issued together (one entry at a time
@@ -396,12 +397,93 @@ __global__ void __launch_bounds__(256) hq_topk_minmax_kernel(const __grid_consta
       qs += red[2][i];
       ls += red[3][i];
     }
+    if (bmin) bmin[blockIdx.x] = ls ? mn : ~0ull;  // the block's smallest key (threshold select)
     if (ls) {
       atomicMin(sel + 0, mn);
       atomicMax(sel + 1, mx);
       atomicAdd(q.stats + 1, qs);
       atomicAdd(q.stats + 3, ls);
     }
+  }
+}
+// threshold select (one block, replaces the histogram pass when every block's share of
+// the table times k fits the candidate buffer): a 2,048-bin histogram of the blocks'
+// smallest keys over their own [min, max] and a scan give the bin b of the k-th smallest
+// minimum; tau = b's upper edge.  At least k entries have a key <= tau (k blocks' minima),
+// so the top k all do; entries <= tau come only from blocks whose minimum is <= tau -- the
+// k - 1 below b's and those in b (the candidate buffer's overflow flag sends a crowded bin
+// the long way).
+constexpr int TK_TAU_MAX = TK_BINS * 4 / 8;  // block minima held in the histogram's space
+__global__ void __launch_bounds__(1024) hq_topk_tau_kernel(const unsigned long long* bmin, int n, int keep,
+                                                          unsigned long long* sel) {
+  __shared__ unsigned h[TK_TAU_MAX];
+  __shared__ unsigned long long rmn[32], rmx[32];
+  __shared__ unsigned part[32];
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  unsigned long long v[2], mn = ~0ull, mx = 0;
+  for (int i = 0; i < 2; ++i) {
+    const int x = tid * 2 + i;
+    v[i] = x < n ? bmin[x] : ~0ull;
+    h[x] = 0;
+    if (v[i] != ~0ull) { mn = v[i] < mn ? v[i] : mn; mx = v[i] > mx ? v[i] : mx; }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long a = __shfl_xor_sync(0xffffffffu, mn, o), b = __shfl_xor_sync(0xffffffffu, mx, o);
+    mn = a < mn ? a : mn;
+    mx = b > mx ? b : mx;
+  }
+  if (lane == 0) { rmn[w] = mn; rmx[w] = mx; }
+  __syncthreads();
+  mn = rmn[lane];
+  mx = rmx[lane];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const unsigned long long a = __shfl_xor_sync(0xffffffffu, mn, o), b = __shfl_xor_sync(0xffffffffu, mx, o);
+    mn = a < mn ? a : mn;
+    mx = b > mx ? b : mx;
+  }
+  if (mn > mx) {  // no live entry
+    if (tid == 0) { sel[6] = 0; sel[7] = 1; }
+    return;
+  }
+  int sh = 0;
+  while (sh < 63 && ((mx - mn) >> sh) >= (unsigned long long)TK_TAU_MAX) ++sh;
+  for (int i = 0; i < 2; ++i)
+    if (v[i] != ~0ull) atomicAdd(&h[(v[i] - mn) >> sh], 1u);
+  __syncthreads();
+  const unsigned c0 = h[tid * 2], c1 = h[tid * 2 + 1], t = c0 + c1;
+  unsigned incl = t;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned x = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += x;
+  }
+  if (lane == 31) part[w] = incl;
+  __syncthreads();
+  if (w == 0) {
+    const unsigned pv = part[lane];
+    unsigned iv = pv;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned x = __shfl_up_sync(0xffffffffu, iv, o);
+      if (lane >= o) iv += x;
+    }
+    part[lane] = iv - pv;
+  }
+  __syncthreads();
+  const unsigned before = part[w] + incl - t;  // minima in the bins below this thread's two
+  int b = -1;
+  if (before < (unsigned)keep && before + c0 >= (unsigned)keep) b = tid * 2;
+  else if (before + c0 < (unsigned)keep && before + t >= (unsigned)keep) b = tid * 2 + 1;
+  if (tid == blockDim.x - 1 && before + t < (unsigned)keep) {  // fewer than k blocks hold entries: all of them
+    sel[6] = ~0ull;
+    sel[7] = 1;
+  }
+  if (b >= 0) {  // the bin of the k-th smallest minimum
+    const unsigned long long top = mn + ((((unsigned long long)b + 1) << sh) - 1);
+    sel[6] = top < mx && top >= mn ? top : mx;
+    sel[7] = 1;  // collect takes key <= sel[6]
   }
 }
 __device__ __forceinline__ int tk_bin(unsigned long long pk, const unsigned long long* sel) {
@@ -473,12 +555,18 @@ __global__ void __launch_bounds__(256) hq_topk_collect_kernel(const __grid_const
   const KCompact& k = q.k;
   if (sel[0] > sel[1]) return;
   const int bstar = (int)sel[3];
+  const bool tau = sel[7] != 0;
+  const unsigned long long tv = sel[6];
   const int lane = threadIdx.x & 31;
   // warp-uniform trip count: one atomic per warp and round claims the warp's candidates
   for (long long b0 = (blockIdx.x * (long long)blockDim.x + threadIdx.x) & ~31ll; b0 < k.ngroups;
        b0 += (long long)gridDim.x * blockDim.x) {
     const long long g = b0 + lane;
-    const bool take = g < k.ngroups && tk_live(k, g) && tk_bin(tk_pk(k, q.s, g), sel) <= bstar;
+    bool take = g < k.ngroups && tk_live(k, g);
+    if (take) {
+      const unsigned long long pk = tk_pk(k, q.s, g);
+      take = tau ? pk <= tv : tk_bin(pk, sel) <= bstar;
+    }
     const unsigned bal = __ballot_sync(0xffffffffu, take);
     if (!bal) continue;
     unsigned long long base = 0;
@@ -856,11 +944,21 @@ static bool finalize_topk(hq_ctx* ctx, hq_result* r) {
   for (hq_hash* hh : r->hashes)
     if (hh->dstate.p && !hh->checked && q.nhash < 8) q.hash_err[q.nhash++] = hh->dstate.as<int>();
   const int grid = grid_for(ctx, r->ngroups);
-  ctx->launches += 6;
-  hq_topk_minmax_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel);
-  hq_topk_shift_kernel<<<1, 1, 0, ctx->stream>>>(sel);
-  hq_topk_hist_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel, (unsigned*)(selb.as<char>() + 64));
-  hq_topk_select_kernel<<<1, 1024, 0, ctx->stream>>>((const unsigned*)(selb.as<char>() + 64), q.keep, sel);
+  // threshold select (one table pass less) when k x a block's share of the table fits the
+  // candidate buffer: TPC-H Q3 SF30, k = 10 over 2^20 entries; HQ_TOPK_RADIX=1 forces the
+  // histogram select (A/B)
+  const int64_t per_block = (r->ngroups + (int64_t)grid * 256 - 1) / ((int64_t)grid * 256) * 256;  // minmax's share
+  const bool tau = grid <= TK_TAU_MAX && q.keep <= grid && (int64_t)q.keep * per_block <= TK_CAND && !getenv("HQ_TOPK_RADIX");
+  unsigned long long* bmin = tau ? (unsigned long long*)(selb.as<char>() + 64) : nullptr;
+  ctx->launches += tau ? 4 : 6;
+  hq_topk_minmax_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel, bmin);
+  if (tau) {
+    hq_topk_tau_kernel<<<1, 1024, 0, ctx->stream>>>(bmin, grid, q.keep, sel);
+  } else {
+    hq_topk_shift_kernel<<<1, 1, 0, ctx->stream>>>(sel);
+    hq_topk_hist_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel, (unsigned*)(selb.as<char>() + 64));
+    hq_topk_select_kernel<<<1, 1024, 0, ctx->stream>>>((const unsigned*)(selb.as<char>() + 64), q.keep, sel);
+  }
   hq_topk_collect_kernel<<<grid, 256, 0, ctx->stream>>>(q, sel);
   hq_topk2_kernel<<<1, 1024, 0, ctx->stream>>>(q, sel);
   HQ_CUDA(cudaGetLastError());
