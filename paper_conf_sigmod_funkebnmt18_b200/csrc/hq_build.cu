@@ -327,12 +327,11 @@ __global__ void __launch_bounds__(BUILD_BLOCK, BUILD_MINB) hq_build_direct_compa
     if (threadIdx.x == 0) {
       unsigned long long t = 0;
       for (int k = 0; k < BUILD_BLOCK / 32; ++k) t += vred[k];
-      if (t) atomicAdd(b.vqual, t);
-      __threadfence();
-      if (atomicAdd(b.ticket, 1u) == gridDim.x - 1) {
-        __threadfence();
-        if (*(volatile unsigned long long*)b.vqual != b.vs.cnt) atomicOr(b.err, HQF_STALE);
-      }
+      // the block's count and its ticket in ONE 64-bit atomic (count: low 40 bits, blocks
+      // done: high 24): the last block reads the total from the returned word -- no fences
+      // (two atomics ordered by __threadfence held every block's exit for microseconds)
+      const unsigned long long old = atomicAdd(b.vqual, (1ull << 40) | t);
+      if ((old >> 40) == gridDim.x - 1 && (old & ((1ull << 40) - 1)) + t != b.vs.cnt) atomicOr(b.err, HQF_STALE);
     }
   }
 }
@@ -423,6 +422,64 @@ __global__ void __launch_bounds__(RSCAN_T) hq_rank_dir_kernel(const uint32_t* bm
   unsigned ex;
   BS(tmp).ExclusiveSum(n, ex);
   unsigned run = bsum[blockIdx.x] + ex;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const unsigned d0 = run;
+    run += __popc(c[2 * q]);
+    const unsigned d1 = run;
+    run += __popc(c[2 * q + 1]);
+    ((uint4*)(bd + 2 * base))[q] = make_uint4(c[2 * q], d0, c[2 * q + 1], d1);
+  }
+}
+// the directory in ONE pass (replaces blocksum + topscan + dir: one bitmap read, two
+// launches less): blocks take their tile in launch order from a ticket, publish the tile's
+// key count, and warp 0 looks back over the 32 preceding status words at a time (decoupled
+// look-back) until it meets an inclusive prefix.  status: 0 = not ready, flag 1 = the tile's
+// count only, flag 2 = the inclusive prefix through the tile (value in the low 62 bits).
+constexpr unsigned long long RS_AGG = 1ull << 62, RS_INC = 2ull << 62, RS_VAL = RS_AGG - 1;
+__global__ void __launch_bounds__(RSCAN_T) hq_rank_dir1_kernel(const uint32_t* bm, unsigned long long* status,
+                                                             unsigned* ticket, uint32_t* bd) {
+  __shared__ unsigned s_blk;
+  __shared__ unsigned long long s_excl;
+  if (threadIdx.x == 0) s_blk = atomicAdd(ticket, 1u);
+  __syncthreads();
+  const unsigned blk = s_blk;
+  const long long base = ((long long)blk * RSCAN_T + threadIdx.x) * RSCAN_W;
+  uint32_t c[RSCAN_W];
+  rank_words(bm, 1, base, c);
+  unsigned n = 0;
+#pragma unroll
+  for (int j = 0; j < RSCAN_W; ++j) n += __popc(c[j]);
+  typedef cub::BlockScan<unsigned, RSCAN_T> BS;
+  __shared__ typename BS::TempStorage tmp;
+  unsigned ex, tot;
+  BS(tmp).ExclusiveSum(n, ex, tot);
+  if (threadIdx.x < 32) {
+    const int lane = threadIdx.x;
+    unsigned long long excl = 0;
+    if (blk == 0) {
+      if (lane == 0) atomicExch(status, RS_INC | tot);
+    } else {
+      if (lane == 0) atomicExch(status + blk, RS_AGG | tot);
+      long long j = (long long)blk - 1 - lane;  // this lane's predecessor in the window
+      for (;;) {
+        const unsigned long long v = j >= 0 ? *(volatile const unsigned long long*)(status + j) : RS_INC;
+        if (__any_sync(0xffffffffu, v == 0)) continue;  // a predecessor not ready yet: re-read the window
+        const unsigned inc = __ballot_sync(0xffffffffu, (v & ~RS_VAL) == RS_INC);
+        const int stop = inc ? __ffs(inc) - 1 : 32;  // nearest inclusive prefix in the window
+        unsigned long long part = lane <= stop ? (v & RS_VAL) : 0ull;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+        excl += part;
+        if (inc) break;
+        j -= 32;
+      }
+      if (lane == 0) atomicExch(status + blk, RS_INC | (excl + tot));
+    }
+    if (lane == 0) s_excl = excl;
+  }
+  __syncthreads();
+  unsigned run = (unsigned)s_excl + ex;
 #pragma unroll
   for (int q = 0; q < 4; ++q) {
     const unsigned d0 = run;
@@ -609,12 +666,11 @@ __global__ void __launch_bounds__(BUILD_BLOCK) hq_build_hash_kernel(const __grid
     if (threadIdx.x == 0) {
       unsigned long long t = 0;
       for (int k = 0; k < BUILD_BLOCK / 32; ++k) t += vred[k];
-      if (t) atomicAdd(b.vqual, t);
-      __threadfence();
-      if (atomicAdd(b.ticket, 1u) == gridDim.x - 1) {  // last block: every block's rows are in
-        __threadfence();
-        if (*(volatile unsigned long long*)b.vqual != b.vs.cnt) atomicOr(b.err, HQF_STALE);
-      }
+      // the block's count and its ticket in ONE 64-bit atomic (count: low 40 bits, blocks
+      // done: high 24): the last block reads the total from the returned word -- no fences
+      // (two atomics ordered by __threadfence held every block's exit for microseconds)
+      const unsigned long long old = atomicAdd(b.vqual, (1ull << 40) | t);
+      if ((old >> 40) == gridDim.x - 1 && (old & ((1ull << 40) - 1)) + t != b.vs.cnt) atomicOr(b.err, HQF_STALE);
     }
   }
   if (!b.count_inserts) return;  // counted builds know their key count already
@@ -873,11 +929,19 @@ void build_finish(hq_ctx* ctx, const hq_build_desc* d, hq_hash* h, BuildState& b
     HQ_CUDA(cudaGetLastError());
     if (stride) {
       const int nblk = (int)(bwords / (RSCAN_T * RSCAN_W));
+      if (!getenv("HQ_RANK_3PASS")) {  // single-pass directory (decoupled look-back)
+        DevBuf st(ctx, (size_t)nblk * 8 + 16);
+        HQ_CUDA(cudaMemsetAsync(st.p, 0, (size_t)nblk * 8 + 16, ctx->stream));
+        ctx->launches += 1;
+        hq_rank_dir1_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, st.as<unsigned long long>(),
+                                                               (unsigned*)(st.as<char>() + (size_t)nblk * 8), h->compact.as<uint32_t>());
+      } else {
       DevBuf bsum(ctx, (size_t)nblk * 4 + 16);
       ctx->launches += 3;
       hq_rank_blocksum_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, 1, bsum.as<unsigned>());
       hq_rank_topscan_kernel<<<1, RSCAN_T, 0, ctx->stream>>>(bsum.as<unsigned>(), nblk);
       hq_rank_dir_kernel<<<nblk, RSCAN_T, 0, ctx->stream>>>(bm, bsum.as<unsigned>(), h->compact.as<uint32_t>());
+      }
       if (b.n > 0) {
         ctx->launches++;
         hq_build_ranked_scatter_kernel<<<bs.grid, BUILD_BLOCK, 0, ctx->stream>>>(
