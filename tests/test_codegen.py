@@ -48,7 +48,10 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "mbar_wait_sleep" in star
     assert "__ldg((const int4*)p.ht[" in srcs["materialise_lrgp"]  # 4-word direct slots
     assert "p.pf[" in srcs["materialise_lrgp"]                     # linear prefilter
-    assert "match_any" in srcs["global_hash_groups"] and "pre_[R]" in srcs["global_hash_groups_r4"]
+    # global hash groups behind no shared table: warp update queues (gq_flush) at R = 2,
+    # warp compaction at R = 4
+    assert "gq_flush(p, sagg, sl0_, gq_, gqn_)" in srcs["global_hash_groups"] and "pre_[R]" in srcs["global_hash_groups_r4"]
+    assert "#define GQ_CAP 0u" in srcs["global_hash_groups_r4"]
     # group keys narrowed to the build-side payload ranges: dense shared table + key remap at the merge
     assert "software-pipelined" not in star  # opt-in only (HQ_JIT_SWP=1)
     assert "#define SMODE 0" in srcs["star_smem_hash"]  # dense domain larger than any shared table: global (C2 + warp merging)
