@@ -86,13 +86,24 @@ __device__ __forceinline__ bool row_passes(const KBuild& b, long long row) {
 // issued before any is used, and no grid-stride loop: a dimension table's rows
 // are all in flight at once (a grid-stride loop made each thread walk ~10 rows
 // through 2-3 dependent DRAM round trips each).
-constexpr int BUILD_U = 8;
+#ifndef HQ_BUILD_U
+#define HQ_BUILD_U 4
+#endif
+constexpr int BUILD_U = HQ_BUILD_U;  // (-DHQ_BUILD_U=..: A/B builds of the library)
 constexpr int BUILD_BLOCK = 256;
 // the count and compact-build kernels are latency-bound: at 72 registers only 3 blocks
 // fit an SM; capped at 64 (4 blocks, a few spilled bytes) the SSB Q4.1 SF100 customer
 // build takes 31.8 instead of 38 us, TPC-H Q3's customer / orders builds 37 / 41 instead
 // of 45 / 46 us (measured)
-constexpr int BUILD_MINB = 4;
+#ifndef HQ_BUILD_MINB
+#define HQ_BUILD_MINB 8
+#endif
+constexpr int BUILD_MINB = HQ_BUILD_MINB;
+// (round 2: 4 rows per thread at 8 blocks per SM beat 8 rows at 4 -- more warps, fewer waves'
+// worth of latency per thread: SSB Q4.1 SF100 customer / part builds 26.3 / 17.0 -> 23.2 /
+// 14.6 us, TPC-H Q3 SF30 customer / orders bitmap / ranked scatter 30.3 / 32.1 / 33.0 ->
+// 27.0 / 26.0 / 29.9 us; 16 rows at 4 blocks spilled 820 bytes, measured)
+static_assert(BUILD_U <= 10, "the compact build packs a 3-bit slot shift per row into 32 bits");
 
 // column c for the thread's U rows: the width dispatch is uniform, the U loads
 // are independent (all in flight)
