@@ -8,7 +8,7 @@ import pytest
 import hqgen
 import oracle
 from paper_conf_sigmod_funkebnmt18_b200 import hq
-from paper_conf_sigmod_funkebnmt18_b200.engine import Engine
+from paper_conf_sigmod_funkebnmt18_b200.engine import Engine, fetch
 from paper_conf_sigmod_funkebnmt18_b200.queries import QUERIES
 
 pytestmark = pytest.mark.gpu
@@ -686,3 +686,36 @@ def test_warp_update_queue_lengths(ctx, tpch1, qname, gq, monkeypatch):
     g = gpu_run(ctx, qname, tpch1, **kw)  # the full pre-LIMIT set under the total order
     assert_same(qname, g, o)
     assert g.qualifying == o.qualifying
+
+
+@pytest.mark.parametrize("sf", [0.01, 1.0])
+@pytest.mark.parametrize("mode", ["threshold", "radix"])
+@pytest.mark.parametrize("order", ["count", "revenue"])
+def test_topk_ties_and_threshold(ctx, ssb, ssb_sf1, sf, mode, order, monkeypatch):
+    """ORDER BY ... LIMIT k over a hash group table (hq_finalize.cu finalize_topk): the
+    threshold select from the blocks' smallest keys and the histogram select (HQ_TOPK_RADIX),
+    with few ties (SUM(revenue) per order) and with massive ties at the boundary (COUNT per
+    order: 1..7 lines, thousands of groups per value; at SF 1 ~200 K tie at 7 -- the candidate
+    buffer overflows and the long way finishes), against numpy under the total order
+    (aggregate, then the key)."""
+    if mode == "radix":
+        monkeypatch.setenv("HQ_TOPK_RADIX", "1")
+    lo = (ssb if sf == 0.01 else ssb_sf1)["lineorder"]
+    E = Engine(ctx, {"lineorder": ctx.load_columns({c: lo[c] for c in ("lo_orderkey", "lo_revenue")})})
+    k = 25
+    pb = E.plan("lineorder")
+    pb.compute("rev", [("load", "lo_revenue")])
+    pb.aggregate(keys=[("lo_orderkey", 0, 1 << 31)], aggs=[("sum", "rev"), ("count", None)],
+                 order=[(order, True)], limit=k, group_capacity=1 << (16 if sf == 0.01 else 21),
+                 agg_names=["revenue", "count"])
+    g = fetch(E.run(pb), pb.result_names)
+    keys, inv = np.unique(lo["lo_orderkey"].astype(np.int64), return_inverse=True)
+    rev = np.zeros(len(keys), np.int64)
+    np.add.at(rev, inv, lo["lo_revenue"].astype(np.int64))
+    cnt = np.bincount(inv, minlength=len(keys)).astype(np.int64)
+    val = cnt if order == "count" else rev
+    top = np.lexsort((keys, -val))[:k]  # aggregate descending, then the key ascending
+    assert g.nrows == k
+    np.testing.assert_array_equal(np.asarray(g.columns["lo_orderkey"], np.int64), keys[top])
+    np.testing.assert_array_equal(np.asarray(g.columns["revenue"], np.int64), rev[top])
+    np.testing.assert_array_equal(np.asarray(g.columns["count"], np.int64), cnt[top])
