@@ -40,6 +40,21 @@ def test_generated_kernels_compile(checker, tmp_path):
     assert "(const int2*)p.rpay[0] + rk_" in rk and "__ldg(p.rpay[2] + rk_)" in rk
     assert "__ldg(p.pf[1] + (e_[r] >> 5)) : 0u" in rk and "p.rpay[1]" not in rk  # semi-join: bits only
     assert "p.ht[0]" not in rk and "0x9E3779B1u" not in rk.split("gk_")[0]
+    # the shared-memory request of a kernel whose probes read global memory stays inside the
+    # 196-KB carve-out (60 KB of L1 for those probes; hq_plan.cu layout search)
+    def defs(src):
+        out = {}
+        for line in src.splitlines():
+            if line.startswith("#define ") and len(line.split()) == 3:
+                _, k, v = line.split()
+                out[k] = v.rstrip("u")
+        return out
+    for name in ("star_dense_lrgp", "ranked_probes", "global_hash_groups"):
+        d = defs(srcs[name])
+        request = int(d["OFF_STAGE"]) + int(d["S"]) * int(d["STAGE_STRIDE"])
+        assert request <= 196 * 1024 - 1024 and int(d["S"]) >= 3, (name, request, d["S"], d["NW"])
+    # the warp update queue of a global hash group table keeps the ring's stages
+    assert int(defs(srcs["global_hash_groups"])["GQ_CAP"]) >= 4
     star = srcs["star_dense_lrgp"]
     assert "lds_u32(sm0_ + " in star                 # staged bitmap
     assert "__ldg((const unsigned char*)p.ctab[" in star  # global byte map
