@@ -82,7 +82,7 @@ class ClockSampler:
                         self.reasons.add(name)
             except Exception:  # noqa: BLE001
                 pass
-            time.sleep(0.02)
+            time.sleep(0.005)  # ~5 samples over a 10-step timed region of the headline query
 
     def __enter__(self):
         self.stop = False
