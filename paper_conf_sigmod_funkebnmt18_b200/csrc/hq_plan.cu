@@ -428,9 +428,11 @@ void hq_build_kplan(hq_ctx* ctx, hq_result* r, KPlan& kp, int64_t group_cap, int
     // (star joins: 1-4 % of the rows) contention is low and the shared memory
     // is worth more to the staged probe tables and the TMA ring
     const uint64_t one = (uint64_t)kp.smem_cap * kp.lvwords * 8;
-    const uint64_t budget = nprobe == 0 ? (uint64_t)SMEM_AGG_BYTES : 4096;
+    const uint64_t budget = nprobe == 0 ? (uint64_t)SMEM_AGG_BYTES : 16384;
     uint32_t c = 1;
-    while (c < 31 && one * (c + 1) <= budget) ++c;
+    // behind probes: up to 4 replicas within 16 KB (SSB Q4.1 SF100 7 replicas 2.197 ms, 4:
+    // 2.167 ms; Q3.1 SF30 1 replica 0.485 ms, 4: 0.473 ms, 16: 0.529 ms, measured)
+    while (c < (nprobe == 0 ? 31u : 4u) && one * (c + 1) <= budget) ++c;
     if (const char* e = getenv("HQ_JIT_SCOPIES")) c = std::max(1, std::min(31, atoi(e)));
     kp.scopies = c;
     agg_smem = (uint32_t)(one * c);
